@@ -1,0 +1,166 @@
+/*
+ * mgj.h — C ABI of libmgj.so, the B200-native hot path of MG-Join
+ * (Paul, Lu, He, Lau, "MG-Join: A Scalable Join for Massively Parallel
+ * Multi-GPU Architectures", SIGMOD '21; text in PAPER.md, cited P:line).
+ *
+ * The operation: an equi-join of two relations R and S of fixed-width
+ * (key, payload) tuples, "distributed over multiple GPUs in the same
+ * machine", inputs "evenly distributed" and resident on the
+ * GPUs, 4-byte key + 4-byte id tuples;
+ * the result must not depend on data placement.  The join runs
+ * the paper's four phases: histogram generation,
+ * global partitioning = partition + assignment + data distribution
+ * (§4), local partitioning and probe.
+ *
+ * Result (readings C1-C3): match count, a 64-bit checksum
+ *   checksum = sum over matches (k,a,b) of (a*C + b) mod 2^64,
+ *   C = 2^32 for 4-byte payloads, 0x9E3779B97F4A7C15 for 8-byte payloads,
+ * and optionally the materialised (key, payloadR, payloadS) triples (bag
+ * semantics: every equal-key (R,S) pair once).
+ *
+ * Conventions
+ *  - Every call returns mgj_status (0 = MGJ_OK, < 0 = error); nothing throws
+ *    or aborts.  Argument/state errors (EINVAL, EALIGN, ESTATE) are returned
+ *    synchronously.  Device-side errors (ECUDA, EPEER on a peer-signal
+ *    timeout, ECAPACITY when a receive/output buffer would overflow) are
+ *    sticky per run and returned by mgj_result.
+ *  - Collective calls (mgj_plan, mgj_partition, mgj_shuffle, mgj_join) must
+ *    be made by every rank in the same order, like NCCL.  They only enqueue
+ *    work on the given CUDA stream (passed as void*, a cudaStream_t) and
+ *    return.  Several ranks may live in ONE process on ONE GPU ("virtual
+ *    ranks", each with its own handle): then call each phase for all ranks
+ *    before the next phase, on one stream.
+ *  - Ownership: input columns are borrowed (valid until mgj_join's work has
+ *    completed).  The handle owns its workspace and the materialised output
+ *    (valid until the next mgj_partition or mgj_destroy).  A caller-provided
+ *    symmetric arena (mgj_peers) is owned by the caller and must outlive the
+ *    handle.
+ */
+#ifndef MGJ_H
+#define MGJ_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+    MGJ_OK = 0,
+    MGJ_EINVAL = -1,     /* bad argument / config */
+    MGJ_EALIGN = -2,     /* a device pointer is not 16-byte aligned */
+    MGJ_ENOMEM = -3,     /* device allocation failed */
+    MGJ_ECUDA = -4,      /* a CUDA runtime call or kernel failed */
+    MGJ_ESTATE = -5,     /* call out of order (plan -> partition -> shuffle -> join -> result) */
+    MGJ_ECAPACITY = -6,  /* receive / chunk / work-item / output capacity exceeded */
+    MGJ_EPEER = -7       /* a peer did not signal within the timeout */
+} mgj_status;
+
+enum { MGJ_MAX_RANKS = 8 };
+
+typedef struct {
+    int32_t  rank, world_size;         /* 0 <= rank < world_size <= 8; one handle per rank */
+    int32_t  key_bytes, payload_bytes; /* {4,4} (paper's tuples) or {8,8} */
+    uint64_t r_capacity, s_capacity;   /* max local tuples this rank passes to mgj_partition */
+    uint64_t recv_capacity_r;          /* tuples of R this rank can receive (0 = auto) */
+    uint64_t recv_capacity_s;          /* tuples of S this rank can receive (0 = auto); identical on all ranks */
+    int32_t  radix_bits_global;        /* B1: 2^B1 global partitions, Eq. 1 analogue (0 = auto = 10) */
+    int32_t  radix_bits_local;         /* B2: local fan-out per pass (0 = auto from sizes, chosen on device) */
+    int32_t  materialize;              /* 0/1: emit (key, payR, payS) triples */
+    int32_t  num_sms;                  /* 0 = device attribute */
+    uint64_t out_capacity;             /* max materialised triples on this rank (0 = auto) */
+    int32_t  reserved[8];              /* must be zero */
+} mgj_config;
+
+typedef struct mgj_plan_s *mgj_handle;
+
+/*
+ * Peer-mapped symmetric memory (e.g. torch.distributed._symmetric_memory
+ * buffer_ptrs).  arena_ptrs[g] is rank g's arena as mapped in THIS process;
+ * every arena has the same size >= mgj_arena_bytes(cfg) and must be
+ * zero-filled on every rank before any rank calls mgj_partition (caller
+ * barrier).  Pass NULL peers when world_size == 1: the handle then
+ * allocates its own arena.
+ */
+typedef struct {
+    void *const *arena_ptrs;   /* [world_size] */
+    uint64_t     arena_bytes;
+} mgj_peers;
+
+typedef struct {
+    uint64_t match_count;          /* global (summed over ranks, a6) */
+    uint64_t checksum;             /* global, wrapping sum mod 2^64 */
+    uint64_t local_count;          /* this rank's co-partitions */
+    uint64_t local_checksum;
+    uint64_t n_materialized;       /* triples in this rank's output shard */
+    const void *out_key;           /* device SoA of n_materialized entries, */
+    const void *out_payload_r;     /*   key_bytes wide each; owned by the handle */
+    const void *out_payload_s;
+    uint64_t recv_r, recv_s;       /* tuples this rank received in the shuffle */
+    float    phase_ms[6];          /* device time of: hist, plan, shuffle, local_part, probe, reduce */
+    int32_t  status;               /* sticky device status of the run (mgj_status) */
+    int32_t  radix_bits_global;    /* B1 used */
+    int32_t  radix_bits_local;     /* B2 chosen on device for this rank */
+    int32_t  n_items;              /* probe work items (co-partition slices) on this rank */
+} mgj_result_t;
+
+/* Bytes each rank's symmetric arena needs for cfg (0 if cfg is invalid). */
+uint64_t mgj_arena_bytes(const mgj_config *cfg);
+
+/* Validate cfg, allocate the workspace on the current CUDA device, bind peers.
+ * Collective (every rank, same cfg except rank).  *out = NULL on error. */
+mgj_status mgj_plan(const mgj_config *cfg, const mgj_peers *peers, mgj_handle *out);
+
+/*
+ * Phase a1: radix histogram of both key columns (2^B1 bins, key
+ * low bits), fused with its all-gather: the rank histogram is stored into
+ * every peer's arena and a release flag is raised.  Columns are SoA
+ * (keys[n], payloads[n]), key_bytes/payload_bytes wide; device pointers must
+ * be 16-byte aligned.  Host pointers are accepted too: they are copied into
+ * handle-owned device staging on `stream` (the end-to-end path).
+ */
+mgj_status mgj_partition(mgj_handle h,
+                         const void *r_keys, const void *r_payloads, uint64_t n_r,
+                         const void *s_keys, const void *s_payloads, uint64_t n_s,
+                         void *stream);
+
+/*
+ * Phases a2 + a3 (§4): waits for every rank's histogram, computes
+ * the partition->GPU assignment (contiguous balanced owner ranges) and the
+ * exact receive offsets, then scatters every tuple straight into its owner's
+ * receive buffer (peer stores over NVLink/NVSwitch through shared-memory
+ * write-combining lines) and raises a data-done flag at every peer.
+ */
+mgj_status mgj_shuffle(mgj_handle h, void *stream);
+
+/*
+ * Phases a4 + a5 + a6: waits for every rank's data, radix
+ * partitions the received segments by the next B2 key bits into
+ * shared-memory-sized co-partitions, builds a shared-memory hash table per
+ * R co-partition and probes it with S, then sums (count, checksum) over
+ * ranks.  Materialised triples stay on the owning rank.
+ */
+mgj_status mgj_join(mgj_handle h, void *stream);
+
+/* Synchronise the last stream and fill *out.  Returns the run's sticky status. */
+mgj_status mgj_result(mgj_handle h, mgj_result_t *out);
+
+void        mgj_destroy(mgj_handle h);
+const char *mgj_strerror(mgj_status s);
+
+/*
+ * Host reference of the partition assignment of phase a2, used by the
+ * multi-process CPU tests: from the all-gathered histograms
+ * hist[world][2][2^bits] (u32) compute owner[2^bits], this rank's send
+ * offsets send_off[2][2^bits] (tuples, into the owner's receive buffer) and
+ * recv_size[2][world].  Same formulas as the device plan kernel
+ * (csrc/plan.cuh).  Pure host code, no CUDA call.
+ */
+mgj_status mgj_plan_host(int32_t world_size, int32_t rank, int32_t bits,
+                         const uint32_t *hist, int32_t *owner,
+                         uint64_t *send_off, uint64_t *recv_size);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* MGJ_H */

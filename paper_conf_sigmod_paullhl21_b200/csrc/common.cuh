@@ -1,0 +1,256 @@
+// common.cuh — shared device helpers, the per-run kernel context and the
+// symmetric-arena layout of libmgj (B200 / sm_100a).
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "mgj.h"
+
+namespace mgj {
+
+constexpr int MAX_RANKS = MGJ_MAX_RANKS;
+constexpr int MAX_B1 = 12;              // scatter WC lines need >= 32 B per partition in 128 KB SMEM
+constexpr int MAX_B2 = 11;              // local fan-out per pass
+constexpr int PROBE_CAP = 4096;         // R tuples per shared-memory hash table (a5)
+constexpr int PROBE_TARGET = 2048;      // expected R tuples per co-partition when B2 is auto
+constexpr int PROBE_S_TARGET = 32768;   // S tuples per probe work item (heavy S co-partitions split)
+constexpr int SCATTER_THREADS = 1024;
+constexpr int SCATTER_V = 4;            // tuples per thread per batch
+constexpr int SCATTER_BATCH = SCATTER_THREADS * SCATTER_V;
+constexpr int LOCAL_THREADS = 512;
+constexpr int LOCAL_V = 16;             // tuples per thread per chunk (8-byte tuples)
+constexpr int PROBE_THREADS = 512;
+constexpr int PROBE_WIN = 1024;         // chunk runs staged per window in the probe
+constexpr uint64_t WAIT_TIMEOUT_NS = 20ull * 1000 * 1000 * 1000;
+
+enum Sig { SIG_HIST = 0, SIG_DATA = 1, SIG_RES = 2, SIG_COUNT = 3 };
+enum Ticket { TK_HIST = 0, TK_SCAT_R = 1, TK_SCAT_S = 2, TK_SCAT_DONE = 3, TK_ITEMS = 4,
+              TK_PROBE = 5, TK_LOCAL = 6, TK_COUNT = 8 };
+enum Meta { MT_PLO = 0, MT_PHI = 1, MT_B2 = 2, MT_OK = 3, MT_NCH_R = 4, MT_NCH_S = 5,
+            MT_NITEMS = 6, MT_COUNT = 16 };
+
+// Arena layout (bytes from each rank's arena base; identical on all ranks).
+struct Arena {
+    uint64_t sig;      // u64 flags[SIG_COUNT][MAX_RANKS], written by peers
+    uint64_t mail;     // u32 hist[MAX_RANKS][2][P]
+    uint64_t resmail;  // u64 res[MAX_RANKS][4] (count, checksum, n_out, status)
+    uint64_t recv[2];  // received tuples of R, S
+    uint64_t total;
+};
+
+struct Item {           // one probe work item: co-partition (p, q) slice
+    uint32_t pi;        // owned partition index (p - p_lo)
+    uint32_t q;         // local sub-partition
+    uint32_t r_lo, r_hi;// logical range in the concatenation of R runs of (p,q)
+    uint32_t s_lo, s_hi;
+};
+
+// Everything a kernel needs, passed by value (param space).
+struct Ctx {
+    int32_t rank, world, B1, P, b2_cfg, b2_max;
+    int32_t line_tuples;          // scatter WC line length (tuples)
+    int32_t chunk_tuples;         // local-partition chunk size C (tuples)
+    int32_t materialize;
+    uint32_t max_items;
+    uint64_t epoch;
+    uint64_t recv_cap[2];
+    uint64_t max_chunks;
+    uint64_t out_cap;
+    Arena lay;
+    char *arena[MAX_RANKS];       // arena bases as mapped in this process
+    const void *in_key[2];
+    const void *in_pay[2];
+    uint64_t n_in[2];
+    // workspace (this rank's device memory)
+    uint32_t *rank_hist;          // [2][P]
+    uint32_t *ticket;             // [TK_COUNT]
+    int32_t *meta;                // [MT_COUNT]
+    int32_t *owner;               // [P]
+    uint64_t *send_off;           // [2][P]
+    uint32_t *gcur;               // [2][P]  reservation cursor inside this rank's block
+    uint64_t *seg_start;          // [2][P]
+    uint64_t *seg_len;            // [2][P]
+    uint64_t *recv_size;          // [2][MAX_RANKS]
+    uint32_t *chunk_base;         // [2][P+1]
+    uint16_t *chunk_off[2];       // [max_chunks][2^b2_max + 1]
+    uint32_t *cop_count;          // [2][P][2^b2_max]
+    Item *items;                  // [max_items]
+    void *local[2];               // locally partitioned tuples (a4 output)
+    unsigned long long *acc;      // [4] local count, checksum, n_out
+    int32_t *err;                 // sticky device status
+    unsigned long long *result;   // [4] global count, checksum; local n_out; status
+    void *out_key, *out_a, *out_b;
+};
+
+template <typename K> struct TupT;
+template <> struct TupT<uint32_t> { using T = uint2; };       // {key, payload}
+template <> struct TupT<uint64_t> { using T = ulonglong2; };  // {key, payload}
+
+__device__ __forceinline__ uint64_t *sig_ptr(char *arena, const Arena &lay, int kind, int g) {
+    return reinterpret_cast<uint64_t *>(arena + lay.sig) + kind * MAX_RANKS + g;
+}
+
+__device__ __forceinline__ void st_release_sys(uint64_t *p, uint64_t v) {
+    asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+
+__device__ __forceinline__ uint64_t ld_acquire_sys(const uint64_t *p) {
+    uint64_t v;
+    asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+
+__device__ __forceinline__ uint64_t globaltimer() {
+    uint64_t t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
+
+__device__ __forceinline__ void set_err(const Ctx &c, int code) {
+    atomicCAS(c.err, 0, code);
+}
+
+// Thread-0 helper: wait until every rank g raised flag `kind` for this epoch.
+__device__ inline bool wait_all_flags(const Ctx &c, int kind) {
+    const uint64_t t0 = globaltimer();
+    for (int g = 0; g < c.world; ++g) {
+        const uint64_t *f = sig_ptr(c.arena[c.rank], c.lay, kind, g);
+        while (ld_acquire_sys(f) < c.epoch) {
+            if (globaltimer() - t0 > WAIT_TIMEOUT_NS) {
+                set_err(c, MGJ_EPEER);
+                return false;
+            }
+            __nanosleep(100);
+        }
+    }
+    return true;
+}
+
+// Raise flag `kind` of this rank at every peer (call after a system fence).
+__device__ inline void signal_all(const Ctx &c, int kind) {
+    for (int d = 0; d < c.world; ++d) st_release_sys(sig_ptr(c.arena[d], c.lay, kind, c.rank), c.epoch);
+}
+
+// Radix digits: digit1 = low B1 key bits (global partition), digit2 = the
+// next B2 bits (local sub-partition); SURVEY.md §8 notation, reading C5.
+template <typename T>
+__device__ __forceinline__ uint32_t digit1(T k, int P) {
+    return (uint32_t)k & (uint32_t)(P - 1);
+}
+template <typename T>
+__device__ __forceinline__ uint32_t digit2(T k, int B1, int Q) {
+    return (uint32_t)((unsigned long long)k >> B1) & (uint32_t)(Q - 1);
+}
+
+// Shared-memory hash of the key bits above the radix digits (a5).  A
+// multiplicative (Weyl) hash; deliberately unrelated to the oracle's.
+template <typename T>
+__device__ __forceinline__ uint32_t tab_hash(T k, int shift, int logT) {
+    if constexpr (sizeof(T) == 4) {
+        return (((uint32_t)k >> shift) * 0x2545F491u) >> (32 - logT);
+    } else {
+        const unsigned long long v = (unsigned long long)k;
+        const uint32_t x = (uint32_t)(v >> shift) ^ (uint32_t)(v >> 32) * 0x9E3779B1u;
+        return (x * 0x2545F491u) >> (32 - logT);
+    }
+}
+
+// Checksum term a*C + b (reading C3): C = 2^32 for 4-byte
+// payloads, 0x9E3779B97F4A7C15 for 8-byte payloads.
+template <typename T>
+__device__ __forceinline__ unsigned long long chk_term(T a, T b) {
+    if constexpr (sizeof(T) == 4) {
+        return ((unsigned long long)(uint32_t)a << 32) + (uint32_t)b;
+    } else {
+        return (unsigned long long)a * 0x9E3779B97F4A7C15ull + (unsigned long long)b;
+    }
+}
+
+__device__ __forceinline__ unsigned long long warp_sum(unsigned long long v) {
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+    return v;
+}
+
+// Block-wide exclusive scan of u32 values in shared memory `a[0..n)`, n <= 32*blockDim.
+// Uses `tmp` (>= 33 u32).  Returns the total.  All threads must call.
+__device__ inline uint32_t block_excl_scan_u32(uint32_t *a, int n, uint32_t *tmp) {
+    const int tid = threadIdx.x, nt = blockDim.x;
+    const int per = (n + nt - 1) / nt;
+    const int lo = min(n, tid * per), hi = min(n, lo + per);
+    uint32_t s = 0;
+    for (int i = lo; i < hi; ++i) s += a[i];
+    // warp inclusive scan of s
+    const int lane = tid & 31, w = tid >> 5;
+    uint32_t x = s;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+        if (lane >= o) x += y;
+    }
+    if (lane == 31) tmp[w] = x;
+    __syncthreads();
+    if (w == 0) {
+        const int nw = (nt + 31) >> 5;
+        uint32_t v = lane < nw ? tmp[lane] : 0;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            uint32_t y = __shfl_up_sync(0xffffffffu, v, o);
+            if (lane >= o) v += y;
+        }
+        if (lane < nw) tmp[lane] = v;  // inclusive per-warp totals
+        if (lane == 31) tmp[32] = v;
+    }
+    __syncthreads();
+    uint32_t run = x - s + (w > 0 ? tmp[w - 1] : 0);
+    for (int i = lo; i < hi; ++i) {
+        uint32_t v = a[i];
+        a[i] = run;
+        run += v;
+    }
+    uint32_t total = tmp[32];
+    __syncthreads();
+    return total;
+}
+
+// Same for u64 (plan kernel).
+__device__ inline uint64_t block_excl_scan_u64(uint64_t *a, int n, uint64_t *tmp) {
+    const int tid = threadIdx.x, nt = blockDim.x;
+    const int per = (n + nt - 1) / nt;
+    const int lo = min(n, tid * per), hi = min(n, lo + per);
+    uint64_t s = 0;
+    for (int i = lo; i < hi; ++i) s += a[i];
+    const int lane = tid & 31, w = tid >> 5;
+    uint64_t x = s;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        uint64_t y = __shfl_up_sync(0xffffffffu, x, o);
+        if (lane >= o) x += y;
+    }
+    if (lane == 31) tmp[w] = x;
+    __syncthreads();
+    if (w == 0) {
+        const int nw = (nt + 31) >> 5;
+        uint64_t v = lane < nw ? tmp[lane] : 0;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            uint64_t y = __shfl_up_sync(0xffffffffu, v, o);
+            if (lane >= o) v += y;
+        }
+        if (lane < nw) tmp[lane] = v;
+        if (lane == 31) tmp[32] = v;
+    }
+    __syncthreads();
+    uint64_t run = x - s + (w > 0 ? tmp[w - 1] : 0);
+    for (int i = lo; i < hi; ++i) {
+        uint64_t v = a[i];
+        a[i] = run;
+        run += v;
+    }
+    uint64_t total = tmp[32];
+    __syncthreads();
+    return total;
+}
+
+}  // namespace mgj

@@ -1,0 +1,215 @@
+// hist_plan.cuh — phase a1 (radix histogram fused with its all-gather) and
+// phase a2 (partition -> GPU assignment and exact receive offsets).
+#pragma once
+
+#include "common.cuh"
+
+namespace mgj {
+
+// ---------------------------------------------------------------------------
+// a1: per-GPU radix histogram (§3.2 "Histogram generation",
+// P:356-370, built in shared memory after Rui et al. [38]; bin count from the
+// Eq. 1 analogue).  H[rel][p] = #{t in rel_g : digit1(t.key) = p}.
+// Reads only the key column with 16-byte vector loads.  The last CTA to
+// finish stores this rank's histogram into every peer's arena mailbox and
+// raises SIG_HIST there (the histogram exchange X4, fused into K1).
+// grid = (G, 2): blockIdx.y selects the relation.
+// ---------------------------------------------------------------------------
+template <typename K>
+__global__ void __launch_bounds__(512) k_hist(Ctx c) {
+    extern __shared__ uint32_t sh[];  // [P]
+    const int P = c.P;
+    const int rel = blockIdx.y;
+    const K *keys = static_cast<const K *>(c.in_key[rel]);
+    const uint64_t n = c.n_in[rel];
+    for (int i = threadIdx.x; i < P; i += blockDim.x) sh[i] = 0;
+    __syncthreads();
+
+    constexpr int VEC = 16 / sizeof(K);
+    const uint64_t nvec = n / VEC;
+    const uint4 *kv = reinterpret_cast<const uint4 *>(keys);
+    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+    uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    auto count = [&](const uint4 &v) {
+        if (sizeof(K) == 4) {
+            atomicAdd(&sh[v.x & (P - 1)], 1u);
+            atomicAdd(&sh[v.y & (P - 1)], 1u);
+            atomicAdd(&sh[v.z & (P - 1)], 1u);
+            atomicAdd(&sh[v.w & (P - 1)], 1u);
+        } else {  // two 8-byte keys: low words are .x and .z
+            atomicAdd(&sh[v.x & (P - 1)], 1u);
+            atomicAdd(&sh[v.z & (P - 1)], 1u);
+        }
+    };
+    for (; i + 3 * stride < nvec; i += 4 * stride) {
+        uint4 v0 = __ldcs(kv + i), v1 = __ldcs(kv + i + stride);
+        uint4 v2 = __ldcs(kv + i + 2 * stride), v3 = __ldcs(kv + i + 3 * stride);
+        count(v0); count(v1); count(v2); count(v3);
+    }
+    for (; i < nvec; i += stride) count(__ldcs(kv + i));
+    if (blockIdx.x == 0)
+        for (uint64_t t = nvec * VEC + threadIdx.x; t < n; t += blockDim.x) atomicAdd(&sh[digit1(keys[t], P)], 1u);
+    __syncthreads();
+    for (int p = threadIdx.x; p < P; p += blockDim.x)
+        if (sh[p]) atomicAdd(&c.rank_hist[rel * P + p], sh[p]);
+
+    // ---- fused exchange: the last CTA publishes the rank histogram ----
+    __threadfence();
+    __syncthreads();
+    __shared__ int last;
+    if (threadIdx.x == 0) last = (atomicAdd(&c.ticket[TK_HIST], 1u) == gridDim.x * gridDim.y - 1);
+    __syncthreads();
+    if (!last) return;
+    __threadfence();
+    for (int d = 0; d < c.world; ++d) {
+        uint32_t *mb = reinterpret_cast<uint32_t *>(c.arena[d] + c.lay.mail) + (size_t)c.rank * 2 * P;
+        for (int j = threadIdx.x; j < 2 * P; j += blockDim.x) mb[j] = __ldcg(&c.rank_hist[j]);
+    }
+    __threadfence_system();
+    __syncthreads();
+    if (threadIdx.x == 0) signal_all(c, SIG_HIST);
+}
+
+// ---------------------------------------------------------------------------
+// a2 formulas, shared by the device plan kernel and mgj_plan_host.
+// Owner of global partition p (reduced form, DESIGN.md
+// §4): contiguous ranges of p cut where the cumulative tuple count (both
+// relations, all ranks) crosses multiples of total/N, using the partition's
+// midpoint; identity ranges p*N/P for uniform data.
+// ---------------------------------------------------------------------------
+__host__ __device__ inline int owner_of(uint64_t cum_before, uint64_t T, uint64_t total, int N, int p, int P) {
+    if (total == 0) return (int)(((uint64_t)p * (uint64_t)N) / (uint64_t)P);
+    const uint64_t o = ((2 * cum_before + T) * (uint64_t)N) / (2 * total);
+    return o >= (uint64_t)N ? N - 1 : (int)o;
+}
+
+__host__ __device__ inline int ceil_log2_u64(uint64_t x) {
+    int l = 0;
+    while (l < 63 && (1ull << l) < x) ++l;
+    return l;
+}
+
+// B2 from the largest owned R partition: co-partitions of ~PROBE_TARGET tuples.
+__host__ __device__ inline int choose_b2(uint64_t max_r, int b2_cfg, int b2_max) {
+    if (b2_cfg > 0) return b2_cfg < b2_max ? b2_cfg : b2_max;
+    const uint64_t need = (max_r + PROBE_TARGET - 1) / PROBE_TARGET;
+    int b = ceil_log2_u64(need);
+    if (b > b2_max) b = b2_max;
+    return b;
+}
+
+// ---------------------------------------------------------------------------
+// a2 device plan: one CTA of 1024 threads.  Every rank computes the same
+// owner[] and receive sizes from the same all-gathered histograms, plus its
+// own send offsets (u64 tuples into the owner's receive buffer, layout:
+// owned p ascending, then source rank ascending), its owned segments, the
+// local radix bits B2 and the chunk table of the local pass.
+// ---------------------------------------------------------------------------
+__global__ void __launch_bounds__(1024) k_plan(Ctx c) {
+    extern __shared__ uint64_t sp[];
+    const int P = c.P, N = c.world, tid = threadIdx.x;
+    uint64_t *tot0 = sp, *tot1 = sp + P, *pre0 = sp + 2 * P, *pre1 = sp + 3 * P, *cum = sp + 4 * P;
+    int32_t *own = reinterpret_cast<int32_t *>(sp + 5 * P);
+    uint32_t *chn = reinterpret_cast<uint32_t *>(own + P);  // [P+1] chunk counts -> base (one rel at a time)
+    __shared__ uint64_t tmp[33];
+    __shared__ uint32_t tmp32[33];
+    __shared__ int first[MAX_RANKS], endp[MAX_RANKS];
+    __shared__ int ok, cap_bad;
+    __shared__ unsigned long long maxr;
+    if (tid == 0) {
+        ok = wait_all_flags(c, SIG_HIST);
+        cap_bad = 0;
+        maxr = 0;
+    }
+    if (tid < MAX_RANKS) first[tid] = endp[tid] = P;
+    __syncthreads();
+    if (!ok) {
+        if (tid == 0) c.meta[MT_OK] = 0;
+        return;
+    }
+    const uint32_t *mail = reinterpret_cast<const uint32_t *>(c.arena[c.rank] + c.lay.mail);
+    for (int p = tid; p < P; p += blockDim.x) {
+        uint64_t t0 = 0, t1 = 0;
+        for (int g = 0; g < N; ++g) {
+            t0 += __ldcg(mail + (size_t)(g * 2 + 0) * P + p);
+            t1 += __ldcg(mail + (size_t)(g * 2 + 1) * P + p);
+        }
+        tot0[p] = pre0[p] = t0;
+        tot1[p] = pre1[p] = t1;
+        cum[p] = t0 + t1;
+    }
+    __syncthreads();
+    block_excl_scan_u64(pre0, P, tmp);
+    block_excl_scan_u64(pre1, P, tmp);
+    const uint64_t total = block_excl_scan_u64(cum, P, tmp);
+    for (int p = tid; p < P; p += blockDim.x) {
+        const int o = owner_of(cum[p], tot0[p] + tot1[p], total, N, p, P);
+        own[p] = o;
+        c.owner[p] = o;
+    }
+    __syncthreads();
+    for (int p = tid; p < P; p += blockDim.x) {
+        if (p == 0 || own[p - 1] != own[p]) first[own[p]] = p;
+        if (p == P - 1 || own[p + 1] != own[p]) endp[own[p]] = p + 1;
+    }
+    __syncthreads();
+    for (int p = tid; p < P; p += blockDim.x) {
+        const int f = first[own[p]];
+        uint64_t m0 = 0, m1 = 0;
+        for (int g = 0; g < c.rank; ++g) {
+            m0 += __ldcg(mail + (size_t)(g * 2 + 0) * P + p);
+            m1 += __ldcg(mail + (size_t)(g * 2 + 1) * P + p);
+        }
+        const uint64_t b0 = pre0[p] - pre0[f], b1 = pre1[p] - pre1[f];
+        c.send_off[p] = b0 + m0;
+        c.send_off[P + p] = b1 + m1;
+        c.seg_start[p] = b0;
+        c.seg_start[P + p] = b1;
+        c.seg_len[p] = tot0[p];
+        c.seg_len[P + p] = tot1[p];
+    }
+    if (tid < 2 * MAX_RANKS) {
+        const int d = tid >> 1, rel = tid & 1;
+        uint64_t size = 0;
+        if (d < N && first[d] < P) {
+            const uint64_t *pre = rel ? pre1 : pre0;
+            const uint64_t *tot = rel ? tot1 : tot0;
+            size = pre[endp[d] - 1] + tot[endp[d] - 1] - pre[first[d]];
+        }
+        c.recv_size[rel * MAX_RANKS + d] = size;
+        if (size > c.recv_cap[rel]) atomicOr(&cap_bad, 1);
+    }
+    const int plo = first[c.rank] < P ? first[c.rank] : 0;
+    const int phi = first[c.rank] < P ? endp[c.rank] : 0;
+    for (int p = plo + tid; p < phi; p += blockDim.x) atomicMax(&maxr, (unsigned long long)tot0[p]);
+    __syncthreads();
+    const int B2 = choose_b2(maxr, c.b2_cfg, c.b2_max);
+    // chunk table of the local pass: chunk_base[rel][pi] = first chunk of owned partition plo+pi
+    const int np = phi - plo;
+    const uint64_t C = (uint64_t)c.chunk_tuples;
+    uint32_t nch[2];
+    for (int rel = 0; rel < 2; ++rel) {
+        const uint64_t *tot = rel ? tot1 : tot0;
+        for (int i = tid; i <= np; i += blockDim.x) chn[i] = i < np ? (uint32_t)((tot[plo + i] + C - 1) / C) : 0;
+        __syncthreads();
+        nch[rel] = block_excl_scan_u32(chn, np + 1, tmp32);
+        for (int i = tid; i <= np; i += blockDim.x) c.chunk_base[rel * (P + 1) + i] = chn[i];
+        __syncthreads();
+    }
+    if (tid == 0) {
+        const bool fits = nch[0] <= c.max_chunks && nch[1] <= c.max_chunks;
+        if (cap_bad || !fits) set_err(c, MGJ_ECAPACITY);
+        c.meta[MT_PLO] = plo;
+        c.meta[MT_PHI] = phi;
+        c.meta[MT_B2] = B2;
+        c.meta[MT_NCH_R] = (int)nch[0];
+        c.meta[MT_NCH_S] = (int)nch[1];
+        c.meta[MT_OK] = (cap_bad || !fits) ? 0 : 1;
+    }
+}
+
+__global__ void k_wait(Ctx c, int kind) {
+    if (threadIdx.x == 0 && blockIdx.x == 0) wait_all_flags(c, kind);
+}
+
+}  // namespace mgj

@@ -1,0 +1,603 @@
+// mgj.cu — C ABI of libmgj.so (include/mgj.h, include/mgj_aux.h): handle,
+// workspace and arena management, phase launches, result read-back.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <new>
+
+#include "common.cuh"
+#include "gen.cuh"
+#include "hist_plan.cuh"
+#include "local_probe.cuh"
+#include "mgj.h"
+#include "mgj_aux.h"
+#include "scatter.cuh"
+
+using namespace mgj;
+
+namespace {
+
+enum State { ST_PLANNED = 1, ST_PARTITIONED = 2, ST_SHUFFLED = 3, ST_JOINED = 4, ST_DONE = 5 };
+
+uint64_t align_up(uint64_t x, uint64_t a) { return (x + a - 1) / a * a; }
+
+struct Norm {  // validated config with the automatic fields filled in
+    mgj_config c;
+    int B1, P, b2_max, tuple_bytes, line_tuples, chunk_tuples;
+    uint64_t recv_cap[2], max_chunks, max_items, out_cap;
+    Arena lay;
+};
+
+int ceil_log2(uint64_t x) {
+    int l = 0;
+    while (l < 63 && (1ull << l) < x) ++l;
+    return l;
+}
+
+mgj_status normalize(const mgj_config *in, Norm *o) {
+    if (!in) return MGJ_EINVAL;
+    mgj_config c = *in;
+    for (int i = 0; i < 8; ++i)
+        if (c.reserved[i]) return MGJ_EINVAL;
+    if (c.world_size < 1 || c.world_size > MAX_RANKS || c.rank < 0 || c.rank >= c.world_size) return MGJ_EINVAL;
+    if (!((c.key_bytes == 4 && c.payload_bytes == 4) || (c.key_bytes == 8 && c.payload_bytes == 8)))
+        return MGJ_EINVAL;
+    if (c.radix_bits_global == 0) c.radix_bits_global = 10;
+    if (c.radix_bits_global < 1 || c.radix_bits_global > MAX_B1) return MGJ_EINVAL;
+    if (c.radix_bits_local < 0 || c.radix_bits_local > MAX_B2) return MGJ_EINVAL;
+    if (c.materialize != 0 && c.materialize != 1) return MGJ_EINVAL;
+    if (c.num_sms < 0) return MGJ_EINVAL;
+    if (c.r_capacity > (1ull << 32) - 1 || c.s_capacity > (1ull << 32) - 1) return MGJ_EINVAL;
+    const uint64_t slack = c.world_size > 1 ? 4 : 0;  // N>1: +25% for imbalance
+    if (c.recv_capacity_r == 0) c.recv_capacity_r = c.r_capacity + (slack ? c.r_capacity / slack + 65536 : 0);
+    if (c.recv_capacity_s == 0) c.recv_capacity_s = c.s_capacity + (slack ? c.s_capacity / slack + 65536 : 0);
+    if (c.recv_capacity_r > (1ull << 32) - 1 || c.recv_capacity_s > (1ull << 32) - 1) return MGJ_EINVAL;
+    o->B1 = c.radix_bits_global;
+    o->P = 1 << o->B1;
+    o->tuple_bytes = 2 * c.key_bytes;
+    const int line_bytes = std::min(128, (128 * 1024) / o->P);
+    o->line_tuples = line_bytes / o->tuple_bytes;
+    if (o->line_tuples < 1) return MGJ_EINVAL;
+    o->chunk_tuples = LOCAL_THREADS * LOCAL_V * 8 / o->tuple_bytes;
+    o->recv_cap[0] = c.recv_capacity_r;
+    o->recv_cap[1] = c.recv_capacity_s;
+    // B2 upper bound: the largest R segment this rank could own is recv_cap_r.
+    if (c.radix_bits_local > 0) {
+        o->b2_max = c.radix_bits_local;
+    } else {
+        o->b2_max = std::min(MAX_B2, std::max(1, ceil_log2((c.recv_capacity_r + PROBE_TARGET - 1) / PROBE_TARGET)));
+    }
+    const uint64_t rmax = std::max(o->recv_cap[0], o->recv_cap[1]);
+    o->max_chunks = rmax / o->chunk_tuples + o->P + 2;
+    const uint64_t Qm = 1ull << o->b2_max;
+    o->max_items = (uint64_t)o->P * Qm + o->recv_cap[1] / PROBE_S_TARGET * 4 + o->recv_cap[0] / PROBE_CAP * 4 + 4096;
+    if (o->max_items > 0xffffffffull) o->max_items = 0xffffffffull;
+    o->out_cap = c.out_capacity ? c.out_capacity : (c.materialize ? std::max(o->recv_cap[0], o->recv_cap[1]) : 0);
+    Arena &L = o->lay;
+    uint64_t off = 0;
+    L.sig = off;
+    off = align_up(off + SIG_COUNT * MAX_RANKS * 8, 4096);
+    L.mail = off;
+    off = align_up(off + (uint64_t)MAX_RANKS * 2 * o->P * 4, 4096);
+    L.resmail = off;
+    off = align_up(off + MAX_RANKS * 4 * 8, 4096);
+    L.recv[0] = off;
+    off = align_up(off + o->recv_cap[0] * o->tuple_bytes, 4096);
+    L.recv[1] = off;
+    off = align_up(off + o->recv_cap[1] * o->tuple_bytes, 4096);
+    L.total = off;
+    o->c = c;
+    return MGJ_OK;
+}
+
+}  // namespace
+
+struct mgj_plan_s {
+    Norm n;
+    int dev = 0, nsm = 0;
+    char *own_arena = nullptr;
+    char *arena[MAX_RANKS] = {};
+    void *zero_block = nullptr;
+    size_t zero_bytes = 0;
+    void *allocs[24] = {};
+    int nalloc = 0;
+    Ctx ctx{};
+    uint64_t epoch = 0;
+    int state = 0;
+    cudaStream_t stream = nullptr;
+    cudaEvent_t ev[7] = {};
+    void *stage = nullptr;
+    size_t stage_bytes = 0;
+    unsigned long long *h_res = nullptr;  // pinned [4] + meta [16 ints]
+    int32_t *h_meta = nullptr;
+    uint64_t recv_r = 0, recv_s = 0;
+    int32_t host_err = 0;
+};
+
+namespace {
+
+mgj_status cuda_ok(cudaError_t e) {
+    if (e == cudaSuccess) return MGJ_OK;
+    return e == cudaErrorMemoryAllocation ? MGJ_ENOMEM : MGJ_ECUDA;
+}
+
+void *dalloc(mgj_plan_s *h, size_t bytes, mgj_status *st) {
+    void *p = nullptr;
+    if (*st != MGJ_OK) return nullptr;
+    cudaError_t e = cudaMalloc(&p, std::max<size_t>(bytes, 256));
+    if (e != cudaSuccess) {
+        (void)cudaGetLastError();
+        *st = MGJ_ENOMEM;
+        return nullptr;
+    }
+    h->allocs[h->nalloc++] = p;
+    return p;
+}
+
+size_t hist_smem(const Norm &n) { return (size_t)n.P * 4; }
+size_t plan_smem(const Norm &n) { return (size_t)n.P * 5 * 8 + (size_t)n.P * 4 + (size_t)(n.P + 1) * 4; }
+size_t scatter_smem(const Norm &n) {
+    return (size_t)n.P * n.line_tuples * n.tuple_bytes + (size_t)n.P * 4 + SCATTER_BATCH * 2;
+}
+size_t local_smem(const Norm &n) { return (size_t)n.chunk_tuples * n.tuple_bytes + ((size_t)1 << n.b2_max) * 4; }
+size_t probe_smem(const Norm &n) {
+    return (size_t)PROBE_CAP * n.tuple_bytes + (size_t)PROBE_CAP * 4 * 2 + (size_t)PROBE_WIN * 4 * 2;
+}
+
+template <typename K>
+cudaError_t set_attrs(const Norm &n) {
+    cudaError_t e;
+    if ((e = cudaFuncSetAttribute(k_hist<K>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)hist_smem(n)))) return e;
+    if ((e = cudaFuncSetAttribute(k_plan, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)plan_smem(n)))) return e;
+    if ((e = cudaFuncSetAttribute(k_scatter<K>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)scatter_smem(n))))
+        return e;
+    if ((e = cudaFuncSetAttribute(k_local<K>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)local_smem(n))))
+        return e;
+    if ((e = cudaFuncSetAttribute(k_probe<K, false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                  (int)probe_smem(n))))
+        return e;
+    return cudaFuncSetAttribute(k_probe<K, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)probe_smem(n));
+}
+
+bool is_device_ptr(const void *p) {
+    cudaPointerAttributes a;
+    if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+        (void)cudaGetLastError();
+        return false;
+    }
+    return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
+}
+
+template <typename K>
+void launch_partition(mgj_plan_s *h, cudaStream_t s) {
+    const Norm &n = h->n;
+    dim3 g(h->nsm * 4, 2);
+    k_hist<K><<<g, 512, hist_smem(n), s>>>(h->ctx);
+}
+
+template <typename K>
+void launch_shuffle(mgj_plan_s *h, cudaStream_t s) {
+    const Norm &n = h->n;
+    k_plan<<<1, 1024, plan_smem(n), s>>>(h->ctx);
+    cudaEventRecord(h->ev[2], s);
+    k_scatter<K><<<h->nsm, SCATTER_THREADS, scatter_smem(n), s>>>(h->ctx);
+}
+
+template <typename K>
+void launch_join(mgj_plan_s *h, cudaStream_t s) {
+    const Norm &n = h->n;
+    k_wait<<<1, 32, 0, s>>>(h->ctx, SIG_DATA);
+    k_local<K><<<h->nsm * 3, LOCAL_THREADS, local_smem(n), s>>>(h->ctx);
+    cudaEventRecord(h->ev[4], s);
+    k_itemize<<<h->nsm * 4, 256, 0, s>>>(h->ctx);
+    if (n.c.materialize)
+        k_probe<K, true><<<h->nsm * 3, PROBE_THREADS, probe_smem(n), s>>>(h->ctx);
+    else
+        k_probe<K, false><<<h->nsm * 3, PROBE_THREADS, probe_smem(n), s>>>(h->ctx);
+    cudaEventRecord(h->ev[5], s);
+    k_publish<<<1, 32, 0, s>>>(h->ctx);
+}
+
+}  // namespace
+
+extern "C" {
+
+const char *mgj_strerror(mgj_status s) {
+    switch (s) {
+        case MGJ_OK: return "ok";
+        case MGJ_EINVAL: return "invalid argument or configuration";
+        case MGJ_EALIGN: return "device pointer not 16-byte aligned";
+        case MGJ_ENOMEM: return "device allocation failed";
+        case MGJ_ECUDA: return "CUDA error";
+        case MGJ_ESTATE: return "call out of order";
+        case MGJ_ECAPACITY: return "capacity exceeded";
+        case MGJ_EPEER: return "peer signal timeout";
+    }
+    return "unknown status";
+}
+
+uint64_t mgj_arena_bytes(const mgj_config *cfg) {
+    Norm n;
+    if (normalize(cfg, &n) != MGJ_OK) return 0;
+    return n.lay.total;
+}
+
+mgj_status mgj_plan(const mgj_config *cfg, const mgj_peers *peers, mgj_handle *out) {
+    if (!out) return MGJ_EINVAL;
+    *out = nullptr;
+    Norm n;
+    mgj_status st = normalize(cfg, &n);
+    if (st != MGJ_OK) return st;
+    const int W = n.c.world_size;
+    if (W > 1) {
+        if (!peers || !peers->arena_ptrs || peers->arena_bytes < n.lay.total) return MGJ_EINVAL;
+        for (int g = 0; g < W; ++g)
+            if (!peers->arena_ptrs[g] || ((uintptr_t)peers->arena_ptrs[g] & 15)) return MGJ_EALIGN;
+    } else if (peers && peers->arena_ptrs) {
+        if (peers->arena_bytes < n.lay.total || !peers->arena_ptrs[0]) return MGJ_EINVAL;
+    }
+    mgj_plan_s *h = new (std::nothrow) mgj_plan_s();
+    if (!h) return MGJ_ENOMEM;
+    h->n = n;
+    if ((st = cuda_ok(cudaGetDevice(&h->dev))) != MGJ_OK) { delete h; return st; }
+    int nsm = 0;
+    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, h->dev);
+    h->nsm = n.c.num_sms ? std::min(n.c.num_sms, nsm) : nsm;
+    if (h->nsm <= 0) { delete h; return MGJ_ECUDA; }
+
+    if (peers && peers->arena_ptrs) {
+        for (int g = 0; g < W; ++g) h->arena[g] = static_cast<char *>(peers->arena_ptrs[g]);
+    } else {
+        h->own_arena = static_cast<char *>(dalloc(h, n.lay.total, &st));
+        if (st == MGJ_OK) st = cuda_ok(cudaMemset(h->own_arena, 0, n.lay.total));
+        h->arena[0] = h->own_arena;
+    }
+    const int P = n.P;
+    const uint64_t Qm = 1ull << n.b2_max;
+    // per-run zero block: rank_hist, ticket, gcur, meta, acc, err, cop_count
+    size_t zo = 0;
+    const size_t z_hist = zo; zo += align_up(2ull * P * 4, 256);
+    const size_t z_tick = zo; zo += 256;
+    const size_t z_gcur = zo; zo += align_up(2ull * P * 4, 256);
+    const size_t z_meta = zo; zo += 256;
+    const size_t z_acc = zo; zo += 256;
+    const size_t z_err = zo; zo += 256;
+    const size_t z_cop = zo; zo += align_up(2ull * P * Qm * 4, 256);
+    h->zero_bytes = zo;
+    char *zb = static_cast<char *>(dalloc(h, zo, &st));
+    h->zero_block = zb;
+    Ctx &c = h->ctx;
+    c.rank = n.c.rank;
+    c.world = W;
+    c.B1 = n.B1;
+    c.P = P;
+    c.b2_cfg = n.c.radix_bits_local;
+    c.b2_max = n.b2_max;
+    c.line_tuples = n.line_tuples;
+    c.chunk_tuples = n.chunk_tuples;
+    c.materialize = n.c.materialize;
+    c.max_items = (uint32_t)n.max_items;
+    c.recv_cap[0] = n.recv_cap[0];
+    c.recv_cap[1] = n.recv_cap[1];
+    c.max_chunks = n.max_chunks;
+    c.out_cap = n.out_cap;
+    c.lay = n.lay;
+    for (int g = 0; g < MAX_RANKS; ++g) c.arena[g] = h->arena[g];
+    if (zb) {
+        c.rank_hist = reinterpret_cast<uint32_t *>(zb + z_hist);
+        c.ticket = reinterpret_cast<uint32_t *>(zb + z_tick);
+        c.gcur = reinterpret_cast<uint32_t *>(zb + z_gcur);
+        c.meta = reinterpret_cast<int32_t *>(zb + z_meta);
+        c.acc = reinterpret_cast<unsigned long long *>(zb + z_acc);
+        c.err = reinterpret_cast<int32_t *>(zb + z_err);
+        c.cop_count = reinterpret_cast<uint32_t *>(zb + z_cop);
+    }
+    c.owner = static_cast<int32_t *>(dalloc(h, P * 4, &st));
+    c.send_off = static_cast<uint64_t *>(dalloc(h, 2ull * P * 8, &st));
+    c.seg_start = static_cast<uint64_t *>(dalloc(h, 2ull * P * 8, &st));
+    c.seg_len = static_cast<uint64_t *>(dalloc(h, 2ull * P * 8, &st));
+    c.recv_size = static_cast<uint64_t *>(dalloc(h, 2ull * MAX_RANKS * 8, &st));
+    c.chunk_base = static_cast<uint32_t *>(dalloc(h, 2ull * (P + 1) * 4, &st));
+    for (int r = 0; r < 2; ++r)
+        c.chunk_off[r] = static_cast<uint16_t *>(dalloc(h, n.max_chunks * (Qm + 1) * 2, &st));
+    c.items = static_cast<Item *>(dalloc(h, n.max_items * sizeof(Item), &st));
+    c.local[0] = dalloc(h, n.recv_cap[0] * n.tuple_bytes, &st);
+    c.local[1] = dalloc(h, n.recv_cap[1] * n.tuple_bytes, &st);
+    c.result = static_cast<unsigned long long *>(dalloc(h, 64, &st));
+    if (n.c.materialize) {
+        c.out_key = dalloc(h, n.out_cap * n.c.key_bytes, &st);
+        c.out_a = dalloc(h, n.out_cap * n.c.key_bytes, &st);
+        c.out_b = dalloc(h, n.out_cap * n.c.key_bytes, &st);
+    }
+    if (st == MGJ_OK) st = cuda_ok(cudaMallocHost(&h->h_res, 4 * 8 + MT_COUNT * 4));
+    if (st == MGJ_OK) h->h_meta = reinterpret_cast<int32_t *>(h->h_res + 4);
+    for (int i = 0; i < 7 && st == MGJ_OK; ++i) st = cuda_ok(cudaEventCreate(&h->ev[i]));
+    if (st == MGJ_OK) st = cuda_ok(n.c.key_bytes == 4 ? set_attrs<uint32_t>(n) : set_attrs<uint64_t>(n));
+    if (st != MGJ_OK) {
+        mgj_destroy(h);
+        return st;
+    }
+    h->state = ST_PLANNED;
+    *out = h;
+    return MGJ_OK;
+}
+
+mgj_status mgj_partition(mgj_handle h, const void *r_keys, const void *r_payloads, uint64_t n_r,
+                         const void *s_keys, const void *s_payloads, uint64_t n_s, void *stream) {
+    if (!h) return MGJ_EINVAL;
+    if (h->state != ST_PLANNED && h->state != ST_JOINED && h->state != ST_DONE) return MGJ_ESTATE;
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    if (h->state == ST_JOINED && h->stream != s) {  // previous run on another stream: let it finish
+        if (cudaStreamSynchronize(h->stream) != cudaSuccess) return MGJ_ECUDA;
+    }
+    const Norm &n = h->n;
+    if (n_r > n.c.r_capacity || n_s > n.c.s_capacity) return MGJ_EINVAL;
+    if ((n_r && (!r_keys || !r_payloads)) || (n_s && (!s_keys || !s_payloads))) return MGJ_EINVAL;
+    const void *ptr[4] = {r_keys, r_payloads, s_keys, s_payloads};
+    const uint64_t cnt[4] = {n_r, n_r, n_s, n_s};
+    const size_t w = n.c.key_bytes;
+    bool host[4];
+    size_t need = 0;
+    for (int i = 0; i < 4; ++i) {
+        host[i] = cnt[i] && !is_device_ptr(ptr[i]);
+        if (host[i]) need += align_up(cnt[i] * w, 256);
+        else if (cnt[i] && ((uintptr_t)ptr[i] & 15)) return MGJ_EALIGN;
+    }
+    if (need > h->stage_bytes) {
+        if (h->stage) cudaFree(h->stage);
+        h->stage = nullptr;
+        h->stage_bytes = 0;
+        const size_t cap = align_up(n.c.r_capacity * w, 256) * 2 + align_up(n.c.s_capacity * w, 256) * 2;
+        if (cudaMalloc(&h->stage, cap) != cudaSuccess) {
+            (void)cudaGetLastError();
+            return MGJ_ENOMEM;
+        }
+        h->stage_bytes = cap;
+    }
+    const void *dptr[4];
+    size_t so = 0;
+    for (int i = 0; i < 4; ++i) {
+        dptr[i] = ptr[i];
+        if (host[i]) {
+            char *d = static_cast<char *>(h->stage) + so;
+            if (cudaMemcpyAsync(d, ptr[i], cnt[i] * w, cudaMemcpyHostToDevice, s) != cudaSuccess) return MGJ_ECUDA;
+            dptr[i] = d;
+            so += align_up(cnt[i] * w, 256);
+        }
+    }
+    h->epoch += 1;
+    Ctx &c = h->ctx;
+    c.epoch = h->epoch;
+    c.in_key[0] = dptr[0];
+    c.in_pay[0] = dptr[1];
+    c.in_key[1] = dptr[2];
+    c.in_pay[1] = dptr[3];
+    c.n_in[0] = n_r;
+    c.n_in[1] = n_s;
+    h->stream = s;
+    if (cudaMemsetAsync(h->zero_block, 0, h->zero_bytes, s) != cudaSuccess) return MGJ_ECUDA;
+    cudaEventRecord(h->ev[0], s);
+    if (n.c.key_bytes == 4) launch_partition<uint32_t>(h, s);
+    else launch_partition<uint64_t>(h, s);
+    cudaEventRecord(h->ev[1], s);
+    if (cudaGetLastError() != cudaSuccess) return MGJ_ECUDA;
+    h->state = ST_PARTITIONED;
+    return MGJ_OK;
+}
+
+mgj_status mgj_shuffle(mgj_handle h, void *stream) {
+    if (!h) return MGJ_EINVAL;
+    if (h->state != ST_PARTITIONED) return MGJ_ESTATE;
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    h->stream = s;
+    if (h->n.c.key_bytes == 4) launch_shuffle<uint32_t>(h, s);
+    else launch_shuffle<uint64_t>(h, s);
+    cudaEventRecord(h->ev[3], s);
+    if (cudaGetLastError() != cudaSuccess) return MGJ_ECUDA;
+    h->state = ST_SHUFFLED;
+    return MGJ_OK;
+}
+
+mgj_status mgj_join(mgj_handle h, void *stream) {
+    if (!h) return MGJ_EINVAL;
+    if (h->state != ST_SHUFFLED) return MGJ_ESTATE;
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    h->stream = s;
+    if (h->n.c.key_bytes == 4) launch_join<uint32_t>(h, s);
+    else launch_join<uint64_t>(h, s);
+    cudaEventRecord(h->ev[6], s);
+    if (cudaGetLastError() != cudaSuccess) return MGJ_ECUDA;
+    h->state = ST_JOINED;
+    return MGJ_OK;
+}
+
+mgj_status mgj_result(mgj_handle h, mgj_result_t *out) {
+    if (!h || !out) return MGJ_EINVAL;
+    if (h->state != ST_JOINED && h->state != ST_DONE) return MGJ_ESTATE;
+    if (h->state == ST_JOINED) {  // a6: wait for every rank's partial result and sum
+        k_gather<<<1, 32, 0, h->stream>>>(h->ctx);
+        cudaMemcpyAsync(h->h_res, h->ctx.result, 4 * 8, cudaMemcpyDeviceToHost, h->stream);
+        cudaMemcpyAsync(h->h_meta, h->ctx.meta, MT_COUNT * 4, cudaMemcpyDeviceToHost, h->stream);
+    }
+    if (cudaStreamSynchronize(h->stream) != cudaSuccess) return MGJ_ECUDA;
+    memset(out, 0, sizeof(*out));
+    const Ctx &c = h->ctx;
+    uint64_t rs[2 * MAX_RANKS] = {};
+    if (cudaMemcpy(rs, c.recv_size, sizeof(rs), cudaMemcpyDeviceToHost) != cudaSuccess) return MGJ_ECUDA;
+    unsigned long long acc[3] = {};
+    if (cudaMemcpy(acc, c.acc, sizeof(acc), cudaMemcpyDeviceToHost) != cudaSuccess) return MGJ_ECUDA;
+    out->match_count = h->h_res[0];
+    out->checksum = h->h_res[1];
+    out->local_count = acc[0];
+    out->local_checksum = acc[1];
+    out->n_materialized = std::min<uint64_t>(h->h_res[2], h->n.out_cap);
+    out->out_key = c.out_key;
+    out->out_payload_r = c.out_a;
+    out->out_payload_s = c.out_b;
+    out->recv_r = rs[c.rank];
+    out->recv_s = rs[MAX_RANKS + c.rank];
+    for (int i = 0; i < 6; ++i) {
+        float ms = 0.f;
+        cudaEventElapsedTime(&ms, h->ev[i], h->ev[i + 1]);
+        out->phase_ms[i] = ms;
+    }
+    out->status = (int32_t)(uint32_t)h->h_res[3];
+    out->radix_bits_global = h->n.B1;
+    out->radix_bits_local = h->h_meta[MT_B2];
+    out->n_items = (int32_t)std::min<uint64_t>(h->h_meta[MT_NITEMS] ? h->h_meta[MT_NITEMS] : 0, h->n.max_items);
+    unsigned int ni = 0;
+    cudaMemcpy(&ni, c.ticket + TK_ITEMS, 4, cudaMemcpyDeviceToHost);
+    out->n_items = (int32_t)std::min<uint64_t>(ni, h->n.max_items);
+    h->state = ST_DONE;
+    return (mgj_status)out->status;
+}
+
+void mgj_destroy(mgj_handle h) {
+    if (!h) return;
+    if (h->stream) cudaStreamSynchronize(h->stream);
+    for (int i = 0; i < h->nalloc; ++i) cudaFree(h->allocs[i]);
+    if (h->stage) cudaFree(h->stage);
+    if (h->h_res) cudaFreeHost(h->h_res);
+    for (int i = 0; i < 7; ++i)
+        if (h->ev[i]) cudaEventDestroy(h->ev[i]);
+    delete h;
+}
+
+mgj_status mgj_plan_host(int32_t world_size, int32_t rank, int32_t bits, const uint32_t *hist, int32_t *owner,
+                         uint64_t *send_off, uint64_t *recv_size) {
+    if (world_size < 1 || world_size > MAX_RANKS || rank < 0 || rank >= world_size || bits < 1 || bits > MAX_B1 ||
+        !hist || !owner || !send_off || !recv_size)
+        return MGJ_EINVAL;
+    const int P = 1 << bits, N = world_size;
+    auto H = [&](int g, int rel, int p) -> uint64_t { return hist[((size_t)g * 2 + rel) * P + p]; };
+    uint64_t *tot = new (std::nothrow) uint64_t[2 * (size_t)P];
+    uint64_t *pre = new (std::nothrow) uint64_t[2 * (size_t)P];
+    if (!tot || !pre) {
+        delete[] tot;
+        delete[] pre;
+        return MGJ_ENOMEM;
+    }
+    uint64_t total = 0, run[2] = {0, 0};
+    for (int p = 0; p < P; ++p)
+        for (int rel = 0; rel < 2; ++rel) {
+            uint64_t t = 0;
+            for (int g = 0; g < N; ++g) t += H(g, rel, p);
+            tot[rel * P + p] = t;
+            pre[rel * P + p] = run[rel];
+            run[rel] += t;
+            total += t;
+        }
+    uint64_t cum = 0;
+    int first[MAX_RANKS], endp[MAX_RANKS];
+    for (int d = 0; d < MAX_RANKS; ++d) first[d] = endp[d] = P;
+    for (int p = 0; p < P; ++p) {
+        const uint64_t T = tot[p] + tot[P + p];
+        owner[p] = owner_of(cum, T, total, N, p, P);
+        cum += T;
+    }
+    for (int p = 0; p < P; ++p) {
+        if (p == 0 || owner[p - 1] != owner[p]) first[owner[p]] = p;
+        if (p == P - 1 || owner[p + 1] != owner[p]) endp[owner[p]] = p + 1;
+    }
+    for (int rel = 0; rel < 2; ++rel) {
+        for (int p = 0; p < P; ++p) {
+            uint64_t mine = 0;
+            for (int g = 0; g < rank; ++g) mine += H(g, rel, p);
+            send_off[rel * P + p] = pre[rel * P + p] - pre[rel * P + first[owner[p]]] + mine;
+        }
+        for (int d = 0; d < N; ++d) {
+            uint64_t sz = 0;
+            if (first[d] < P) sz = pre[rel * P + endp[d] - 1] + tot[rel * P + endp[d] - 1] - pre[rel * P + first[d]];
+            recv_size[rel * N + d] = sz;
+        }
+    }
+    delete[] tot;
+    delete[] pre;
+    return MGJ_OK;
+}
+
+mgj_status mgj_gen_relation(int32_t kind, int32_t rel, uint64_t n_r, uint64_t n_s, double z, uint64_t row0,
+                            uint64_t count, void *keys, void *payloads, void *stream) {
+    if (kind < 0 || kind > 2 || rel < 0 || rel > 1) return MGJ_EINVAL;
+    if (count && (!keys || !payloads)) return MGJ_EINVAL;
+    const uint64_t n = rel == 0 ? n_r : n_s;
+    if (n == 0 || n > (1ull << 32) || row0 + count > n) return MGJ_EINVAL;
+    int zmode = 0;
+    if (kind == 1) {
+        if (n_r & (n_r - 1)) return MGJ_EINVAL;
+        if (z == 0.0) zmode = 0;
+        else if (z == 0.5) zmode = 1;
+        else if (z == 1.0) zmode = 2;
+        else return MGJ_EINVAL;
+    }
+    if (!count) return MGJ_OK;
+    int dev = 0, nsm = 148;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+    const uint64_t blocks = std::min<uint64_t>((count + 255) / 256, (uint64_t)nsm * 16);
+    mgj_gen::k_gen<<<(unsigned)blocks, 256, 0, static_cast<cudaStream_t>(stream)>>>(kind, rel, n_r, n_s, zmode, row0,
+                                                                                    count, keys, payloads);
+    return cudaGetLastError() == cudaSuccess ? MGJ_OK : MGJ_ECUDA;
+}
+
+mgj_status mgj_debug_copy(mgj_handle h, int32_t what, void *dst, uint64_t bytes, uint64_t *size_out) {
+    if (!h) return MGJ_EINVAL;
+    if (cudaDeviceSynchronize() != cudaSuccess) return MGJ_ECUDA;
+    const Ctx &c = h->ctx;
+    const Norm &n = h->n;
+    const int P = n.P;
+    int32_t meta[MT_COUNT];
+    if (cudaMemcpy(meta, c.meta, sizeof(meta), cudaMemcpyDeviceToHost) != cudaSuccess) return MGJ_ECUDA;
+    uint64_t rs[2 * MAX_RANKS];
+    if (cudaMemcpy(rs, c.recv_size, sizeof(rs), cudaMemcpyDeviceToHost) != cudaSuccess) return MGJ_ECUDA;
+    const int Q = 1 << meta[MT_B2];
+    const void *src = nullptr;
+    uint64_t size = 0;
+    switch (what) {
+        case MGJ_DBG_RANK_HIST: src = c.rank_hist; size = 2ull * P * 4; break;
+        case MGJ_DBG_MAIL_HIST: src = h->arena[c.rank] + n.lay.mail; size = (uint64_t)c.world * 2 * P * 4; break;
+        case MGJ_DBG_OWNER: src = c.owner; size = (uint64_t)P * 4; break;
+        case MGJ_DBG_SEND_OFF: src = c.send_off; size = 2ull * P * 8; break;
+        case MGJ_DBG_RECV_SIZE: src = c.recv_size; size = sizeof(rs); break;
+        case MGJ_DBG_RECV_R: src = h->arena[c.rank] + n.lay.recv[0]; size = rs[c.rank] * n.tuple_bytes; break;
+        case MGJ_DBG_RECV_S:
+            src = h->arena[c.rank] + n.lay.recv[1];
+            size = rs[MAX_RANKS + c.rank] * n.tuple_bytes;
+            break;
+        case MGJ_DBG_LOCAL_R: src = c.local[0]; size = rs[c.rank] * n.tuple_bytes; break;
+        case MGJ_DBG_LOCAL_S: src = c.local[1]; size = rs[MAX_RANKS + c.rank] * n.tuple_bytes; break;
+        case MGJ_DBG_META: src = c.meta; size = sizeof(meta); break;
+        case MGJ_DBG_CHUNK_OFF_R: src = c.chunk_off[0]; size = (uint64_t)(uint32_t)meta[MT_NCH_R] * (Q + 1) * 2; break;
+        case MGJ_DBG_CHUNK_OFF_S: src = c.chunk_off[1]; size = (uint64_t)(uint32_t)meta[MT_NCH_S] * (Q + 1) * 2; break;
+        case MGJ_DBG_CHUNK_BASE: src = c.chunk_base; size = 2ull * (P + 1) * 4; break;
+        case MGJ_DBG_OUT_KEY:
+        case MGJ_DBG_OUT_PAY_R:
+        case MGJ_DBG_OUT_PAY_S: {
+            if (!n.c.materialize) return MGJ_EINVAL;
+            unsigned long long no = 0;
+            if (cudaMemcpy(&no, c.acc + 2, 8, cudaMemcpyDeviceToHost) != cudaSuccess) return MGJ_ECUDA;
+            src = what == MGJ_DBG_OUT_KEY ? c.out_key : (what == MGJ_DBG_OUT_PAY_R ? c.out_a : c.out_b);
+            size = std::min<uint64_t>(no, n.out_cap) * n.c.key_bytes;
+            break;
+        }
+        case MGJ_DBG_SEGMENTS: {
+            if (size_out) *size_out = 4ull * P * 8;
+            if (!dst) return MGJ_OK;
+            uint64_t tmp[4 * 4096];
+            if (cudaMemcpy(tmp, c.seg_start, 2ull * P * 8, cudaMemcpyDeviceToHost) != cudaSuccess) return MGJ_ECUDA;
+            if (cudaMemcpy(tmp + 2 * P, c.seg_len, 2ull * P * 8, cudaMemcpyDeviceToHost) != cudaSuccess)
+                return MGJ_ECUDA;
+            memcpy(dst, tmp, std::min<uint64_t>(bytes, 4ull * P * 8));
+            return MGJ_OK;
+        }
+        default: return MGJ_EINVAL;
+    }
+    if (size_out) *size_out = size;
+    if (!dst || !bytes) return MGJ_OK;
+    return cudaMemcpy(dst, src, std::min(bytes, size), cudaMemcpyDeviceToHost) == cudaSuccess ? MGJ_OK : MGJ_ECUDA;
+}
+
+}  // extern "C"

@@ -1,0 +1,348 @@
+"""GPU parity tests: the CUDA path through the C ABI vs the CPU oracle.
+
+Bit-exact bar (integer work): match count, 64-bit checksum and the sorted
+materialised triples equal the oracle's; per-phase intermediate state is
+checked against library routines (np.bincount, sorting) and invariants.
+"""
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+import oracle  # noqa: E402
+from paper_conf_sigmod_paullhl21_b200 import datagen  # noqa: E402
+
+M64 = (1 << 64) - 1
+
+
+@pytest.fixture(scope="module")
+def mgj():
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    import __graft_entry__
+    __graft_entry__.build()
+    from paper_conf_sigmod_paullhl21_b200 import mgj as m
+    return m
+
+
+def dev(a: np.ndarray):
+    v = a.view(np.int32) if a.dtype == np.uint32 else a.view(np.int64)
+    return torch.from_numpy(np.ascontiguousarray(v)).cuda()
+
+
+def sort_trip(k, a, b):
+    o = np.lexsort((b, a, k))
+    return k[o], a[o], b[o]
+
+
+def run_one(mgj, d, materialize=False, **kw):
+    kb = 8 if d["r_keys"].dtype == np.uint64 else 4
+    cfg = mgj.make_config(key_bytes=kb, r_capacity=max(d["r_keys"].size, 1), s_capacity=max(d["s_keys"].size, 1),
+                          materialize=materialize, **kw)
+    j = mgj.Join(cfg)
+    res = j.run(dev(d["r_keys"]), dev(d["r_pays"]), dev(d["s_keys"]), dev(d["s_pays"]))
+    return j, res
+
+
+def check_vs_oracle(mgj, d, materialize=True, **kw):
+    ref = oracle.join(d["r_keys"], d["r_pays"], d["s_keys"], d["s_pays"], materialize=materialize)
+    if materialize:
+        kw.setdefault("out_capacity", max(ref["count"], 1))
+    j, res = run_one(mgj, d, materialize=materialize, **kw)
+    assert res["match_count"] == ref["count"]
+    assert res["checksum"] == ref["checksum"]
+    if materialize:
+        assert res["n_materialized"] == ref["count"]
+        k, a, b = sort_trip(*j.materialized(res))
+        np.testing.assert_array_equal(k, ref["key"])
+        np.testing.assert_array_equal(a, ref["pay_r"])
+        np.testing.assert_array_equal(b, ref["pay_s"])
+    j.close()
+    return res
+
+
+# ----------------------------------------------------------------- generator
+@pytest.mark.parametrize("kind,n_r,n_s,z,row0,count", [
+    ("unique", 1000003, 1000003, 0.0, 0, 1000003),
+    ("unique", 1 << 20, 1 << 20, 0.0, 12345, 99999),
+    ("zipf", 1 << 16, 1 << 18, 0.5, 0, 1 << 18),
+    ("zipf", 1 << 16, 1 << 18, 1.0, 777, 100000),
+    ("zipf", 1 << 16, 1 << 18, 0.0, 0, 1 << 18),
+    ("wide", 1 << 16, 1 << 16, 0.0, 5, 60000),
+])
+def test_gen_matches_numpy(mgj, kind, n_r, n_s, z, row0, count):
+    w = datagen.Workload(kind, n_r, n_s, z)
+    for rel, name in ((0, "R"), (1, "S")):
+        n = n_r if rel == 0 else n_s
+        c = min(count, n - row0)
+        dt = torch.int64 if kind == "wide" else torch.int32
+        k = torch.empty(c, dtype=dt, device="cuda")
+        p = torch.empty(c, dtype=dt, device="cuda")
+        mgj.gen_relation(kind, rel, n_r, n_s, z, row0, c, k, p)
+        torch.cuda.synchronize()
+        ek, ep = w.relation(name, row0, row0 + c)
+        np.testing.assert_array_equal(k.cpu().numpy().view(ek.dtype), ek)
+        np.testing.assert_array_equal(p.cpu().numpy().view(ep.dtype), ep)
+
+
+# ------------------------------------------------------------ per-phase state
+def test_phases_m1(mgj):
+    """a1 histogram == np.bincount, a2 plan invariants, a3 received multiset,
+    a4 sub-partition property, at M1 (2^20 x 2^20, one GPU)."""
+    d = datagen.M1().rank_inputs()
+    n = d["r_keys"].size
+    j, res = run_one(mgj, d)
+    P = 1 << res["radix_bits_global"]
+    B1 = res["radix_bits_global"]
+    hist = j.debug("RANK_HIST", np.uint32).reshape(2, P)
+    np.testing.assert_array_equal(hist[0], np.bincount(d["r_keys"] & (P - 1), minlength=P))
+    np.testing.assert_array_equal(hist[1], np.bincount(d["s_keys"] & (P - 1), minlength=P))
+    owner = j.debug("OWNER", np.int32)
+    assert (owner == 0).all()
+    send_off = j.debug("SEND_OFF", np.uint64).reshape(2, P)
+    for rel in range(2):
+        exp = np.concatenate([[0], np.cumsum(hist[rel].astype(np.uint64))[:-1]])
+        np.testing.assert_array_equal(send_off[rel], exp)
+    assert res["recv_r"] == n and res["recv_s"] == n
+    for rel, (kk, pp) in enumerate(((d["r_keys"], d["r_pays"]), (d["s_keys"], d["s_pays"]))):
+        recv = j.debug("RECV_R" if rel == 0 else "RECV_S", np.uint32).reshape(-1, 2)
+        # received layout: partition p occupies [send_off[p], send_off[p] + hist[p])
+        digit = recv[:, 0] & (P - 1)
+        assert np.all(np.diff(digit.astype(np.int64)) >= 0)
+        packed = recv[:, 0].astype(np.uint64) | (recv[:, 1].astype(np.uint64) << np.uint64(32))
+        exp = kk.astype(np.uint64) | (pp.astype(np.uint64) << np.uint64(32))
+        np.testing.assert_array_equal(np.sort(packed), np.sort(exp))
+        # a4: every chunk of every segment is ordered by digit2 and keeps its multiset
+        loc = j.debug("LOCAL_R" if rel == 0 else "LOCAL_S", np.uint32).reshape(-1, 2)
+        B2 = res["radix_bits_local"]
+        Q = 1 << B2
+        C = 8192
+        seg = j.debug("SEGMENTS", np.uint64).reshape(4, P)
+        start, ln = seg[rel], seg[2 + rel]
+        coff = j.debug("CHUNK_OFF_R" if rel == 0 else "CHUNK_OFF_S", np.uint16).reshape(-1, Q + 1)
+        ci = 0
+        for p in range(P):
+            for k0 in range(0, int(ln[p]), C):
+                a, b = int(start[p]) + k0, int(start[p]) + min(int(ln[p]), k0 + C)
+                d2 = (loc[a:b, 0] >> B1) & (Q - 1)
+                assert np.all(np.diff(d2.astype(np.int64)) >= 0)
+                np.testing.assert_array_equal(coff[ci], np.searchsorted(d2, np.arange(Q + 1)))
+                src = recv[a:b, 0].astype(np.uint64) | (recv[a:b, 1].astype(np.uint64) << np.uint64(32))
+                dst = loc[a:b, 0].astype(np.uint64) | (loc[a:b, 1].astype(np.uint64) << np.uint64(32))
+                np.testing.assert_array_equal(np.sort(src), np.sort(dst))
+                ci += 1
+    j.close()
+
+
+# ------------------------------------------------------------ end-to-end parity
+def test_m1_parity_materialized(mgj):
+    res = check_vs_oracle(mgj, datagen.M1().rank_inputs(), materialize=True)
+    assert res["match_count"] == 1 << 20
+    assert res["checksum"] == 0xfff8007ffff80000
+
+
+@pytest.mark.parametrize("b1,b2", [(1, 0), (4, 3), (8, 0), (11, 2), (12, 5)])
+def test_radix_bit_variants(mgj, b1, b2):
+    d = datagen.Workload("unique", 300007, 300007).rank_inputs()
+    check_vs_oracle(mgj, d, materialize=True, radix_bits_global=b1, radix_bits_local=b2)
+
+
+@pytest.mark.parametrize("nr,ns,dom", [(0, 1000, 100), (1000, 0, 100), (0, 0, 1), (1, 1, 1), (3, 5, 2),
+                                       (100003, 70001, 1 << 32), (50000, 60000, 4096), (20000, 30000, 37)])
+def test_random_duplicates(mgj, nr, ns, dom):
+    rng = np.random.default_rng(nr * 7 + ns)
+    d = {"r_keys": rng.integers(0, dom, nr, dtype=np.uint64).astype(np.uint32),
+         "s_keys": rng.integers(0, dom, ns, dtype=np.uint64).astype(np.uint32),
+         "r_pays": rng.integers(0, 1 << 32, nr, dtype=np.uint64).astype(np.uint32),
+         "s_pays": rng.integers(0, 1 << 32, ns, dtype=np.uint64).astype(np.uint32)}
+    check_vs_oracle(mgj, d, materialize=(nr * ns < 10**8 and dom > 50) or nr * ns < 100)
+
+
+def test_edge_key_values(mgj):
+    edge = np.array([0, 1, 2**31 - 1, 2**31, 2**32 - 2, 2**32 - 1], dtype=np.uint32)
+    rng = np.random.default_rng(3)
+    d = {"r_keys": rng.choice(edge, 3000), "s_keys": rng.choice(edge, 2000),
+         "r_pays": np.arange(3000, dtype=np.uint32) - np.uint32(10), "s_pays": np.arange(2000, dtype=np.uint32)}
+    check_vs_oracle(mgj, d, materialize=True)
+
+
+def test_heavy_single_key(mgj):
+    """All R and S tuples share one key: R co-partition 10000 > table capacity
+    (chunked builds), S split over several probe items."""
+    nr, ns = 10000, 70000
+    d = {"r_keys": np.full(nr, 0xDEADBEEF, np.uint32), "s_keys": np.full(ns, 0xDEADBEEF, np.uint32),
+         "r_pays": np.arange(nr, dtype=np.uint32), "s_pays": np.arange(ns, dtype=np.uint32) * np.uint32(3)}
+    res = check_vs_oracle(mgj, d, materialize=False)
+    assert res["match_count"] == nr * ns
+
+
+@pytest.mark.parametrize("z", [0.5, 1.0])
+def test_zipf_small(mgj, z):
+    w = datagen.Workload("zipf", 1 << 16, 1 << 18, z)
+    d = w.rank_inputs()
+    res = check_vs_oracle(mgj, d, materialize=True)
+    assert res["match_count"] == 1 << 17
+
+
+def test_wide_small_materialized(mgj):
+    n = 1 << 16
+    d = datagen.Workload("wide", n, n).rank_inputs()
+    res = check_vs_oracle(mgj, d, materialize=True)
+    h = n * (n - 1) // 2
+    assert res["checksum"] == (oracle.C_WIDE * (n * (1 << 40) + h) + n * (1 << 41) + h) & M64
+
+
+def test_wide_high_bits_only(mgj):
+    rng = np.random.default_rng(11)
+    low = rng.integers(0, 64, 40000, dtype=np.uint64)
+    rk = (rng.integers(0, 8, 40000, dtype=np.uint64) << np.uint64(32)) | low
+    low2 = rng.integers(0, 64, 30000, dtype=np.uint64)
+    sk = (rng.integers(0, 8, 30000, dtype=np.uint64) << np.uint64(32)) | low2
+    d = {"r_keys": rk, "s_keys": sk, "r_pays": np.arange(40000, dtype=np.uint64) << np.uint64(33),
+         "s_pays": np.arange(30000, dtype=np.uint64) + np.uint64(2**63)}
+    check_vs_oracle(mgj, d, materialize=False)
+
+
+def test_host_pointer_path(mgj):
+    """Host (numpy) inputs are staged by the library: same result (end-to-end path)."""
+    d = datagen.Workload("unique", 1 << 18, 1 << 18).rank_inputs()
+    cfg = mgj.make_config(r_capacity=1 << 18, s_capacity=1 << 18)
+    j = mgj.Join(cfg)
+    res = j.run(d["r_keys"], d["r_pays"], d["s_keys"], d["s_pays"])
+    ref = oracle.join(d["r_keys"], d["r_pays"], d["s_keys"], d["s_pays"])
+    assert (res["match_count"], res["checksum"]) == (ref["count"], ref["checksum"])
+    j.close()
+
+
+def test_repeated_runs_same_handle(mgj):
+    d = datagen.Workload("unique", 100000, 100000).rank_inputs()
+    cfg = mgj.make_config(r_capacity=200000, s_capacity=200000)
+    j = mgj.Join(cfg)
+    ref = oracle.join(d["r_keys"], d["r_pays"], d["s_keys"], d["s_pays"])
+    t = [dev(d[k]) for k in ("r_keys", "r_pays", "s_keys", "s_pays")]
+    for _ in range(3):
+        res = j.run(*t)
+        assert (res["match_count"], res["checksum"]) == (ref["count"], ref["checksum"])
+    j.close()
+
+
+# ------------------------------------------------------------ virtual ranks
+def run_virtual(mgj, w: datagen.Workload, N: int, materialize: bool, **kw):
+    """N ranks in one process on GPU 0: arenas are plain device buffers, every
+    phase is issued for all ranks before the next (mgj.h conventions)."""
+    parts = [w.rank_inputs(g, N) for g in range(N)]
+    kb = w.key_bytes
+    cap_r = max(p["r_keys"].size for p in parts)
+    cap_s = max(p["s_keys"].size for p in parts)
+    cfgs = [mgj.make_config(rank=g, world_size=N, key_bytes=kb, r_capacity=cap_r, s_capacity=cap_s,
+                            materialize=materialize, recv_capacity_r=w.n_r, recv_capacity_s=w.n_s, **kw)
+            for g in range(N)]
+    nb = mgj.arena_bytes(cfgs[0])
+    arenas = [torch.zeros(nb, dtype=torch.uint8, device="cuda") for _ in range(N)]
+    ptrs = [a.data_ptr() for a in arenas]
+    joins = [mgj.Join(cfgs[g], ptrs, nb) for g in range(N)]
+    tens = [[dev(p[k]) for k in ("r_keys", "r_pays", "s_keys", "s_pays")] for p in parts]
+    for g in range(N):
+        joins[g].partition(*tens[g])
+    for g in range(N):
+        joins[g].shuffle()
+    for g in range(N):
+        joins[g].join()
+    res = [joins[g].result() for g in range(N)]
+    return joins, res, arenas
+
+
+@pytest.mark.parametrize("N", [2, 3, 4, 8])
+def test_virtual_ranks_m1(mgj, N):
+    w = datagen.M1()
+    joins, res, _ = run_virtual(mgj, w, N, materialize=True)
+    d = w.rank_inputs()
+    ref = oracle.join(d["r_keys"], d["r_pays"], d["s_keys"], d["s_pays"], materialize=True)
+    for r in res:
+        assert (r["match_count"], r["checksum"]) == (ref["count"], ref["checksum"])
+    assert sum(r["local_count"] for r in res) == ref["count"]
+    trip = [j.materialized(r) for j, r in zip(joins, res)]
+    k, a, b = sort_trip(*(np.concatenate([t[i] for t in trip]) for i in range(3)))
+    np.testing.assert_array_equal(k, ref["key"])
+    np.testing.assert_array_equal(a, ref["pay_r"])
+    np.testing.assert_array_equal(b, ref["pay_s"])
+    # device plan == host reference plan, and every received tuple belongs to its owner
+    P = 1 << res[0]["radix_bits_global"]
+    mail = joins[0].debug("MAIL_HIST", np.uint32).reshape(N, 2, P)
+    for g, j in enumerate(joins):
+        owner, send_off, recv_size = mgj.plan_host(N, g, res[0]["radix_bits_global"], mail)
+        np.testing.assert_array_equal(j.debug("OWNER", np.int32), owner)
+        np.testing.assert_array_equal(j.debug("SEND_OFF", np.uint64).reshape(2, P), send_off)
+        assert res[g]["recv_r"] == recv_size[0, g] and res[g]["recv_s"] == recv_size[1, g]
+        recv = j.debug("RECV_R", np.uint32).reshape(-1, 2)
+        assert np.all(owner[recv[:, 0] & (P - 1)] == g)
+    for j in joins:
+        j.close()
+
+
+def test_virtual_ranks_zipf_skew(mgj):
+    w = datagen.Workload("zipf", 1 << 16, 1 << 18, 1.0)
+    joins, res, _ = run_virtual(mgj, w, 4, materialize=False)
+    d = w.rank_inputs()
+    ref = oracle.join(d["r_keys"], d["r_pays"], d["s_keys"], d["s_pays"])
+    assert (res[0]["match_count"], res[0]["checksum"]) == (ref["count"], ref["checksum"])
+    for j in joins:
+        j.close()
+
+
+def test_virtual_ranks_wide(mgj):
+    w = datagen.Workload("wide", 1 << 17, 1 << 17)
+    joins, res, _ = run_virtual(mgj, w, 2, materialize=True)
+    d = w.rank_inputs()
+    ref = oracle.join(d["r_keys"], d["r_pays"], d["s_keys"], d["s_pays"])
+    assert (res[1]["match_count"], res[1]["checksum"]) == (ref["count"], ref["checksum"])
+    for j in joins:
+        j.close()
+
+
+# ------------------------------------------------------------ error paths
+def test_error_paths(mgj):
+    n = 4096
+    cfg = mgj.make_config(r_capacity=n, s_capacity=n)
+    j = mgj.Join(cfg)
+    t = torch.zeros(n + 4, dtype=torch.int32, device="cuda")
+    with pytest.raises(mgj.MGJError) as e:
+        j.shuffle()
+    assert e.value.status == -5  # ESTATE
+    with pytest.raises(mgj.MGJError) as e:
+        j.partition(t[1:n + 1], t[:n], t[:n], t[:n])
+    assert e.value.status == -2  # EALIGN
+    with pytest.raises(mgj.MGJError) as e:
+        j.partition(t, t, t, t)  # n + 4 > capacity
+    assert e.value.status == -1
+    j.close()
+    # receive capacity smaller than the data: sticky ECAPACITY from mgj_result
+    d = datagen.Workload("unique", n, n).rank_inputs()
+    j = mgj.Join(mgj.make_config(r_capacity=n, s_capacity=n, recv_capacity_r=n // 2, recv_capacity_s=n))
+    j.partition(dev(d["r_keys"]), dev(d["r_pays"]), dev(d["s_keys"]), dev(d["s_pays"]))
+    j.shuffle()
+    j.join()
+    with pytest.raises(mgj.MGJError) as e:
+        j.result()
+    assert e.value.status == -6
+    j.close()
+
+
+# ------------------------------------------------------------ full size (bench config)
+@pytest.mark.slow
+def test_m2_full_size_closed_form(mgj):
+    """M2 at N=1 (2^29 R x 2^29 S, the bench workload): closed-form count and
+    checksum (tests/golden/appendix_a_closed_forms.json)."""
+    n = 1 << 29
+    cols = [torch.empty(n, dtype=torch.int32, device="cuda") for _ in range(4)]
+    mgj.gen_relation("unique", 0, n, n, 0.0, 0, n, cols[0], cols[1])
+    mgj.gen_relation("unique", 1, n, n, 0.0, 0, n, cols[2], cols[3])
+    j = mgj.Join(mgj.make_config(r_capacity=n, s_capacity=n))
+    res = j.run(*cols)
+    assert res["match_count"] == n
+    assert res["checksum"] == 0xf1fffffff0000000
+    # sampled structural check at full size: received R is a permutation of the input
+    hist = j.debug("RANK_HIST", np.uint32).reshape(2, -1)
+    assert int(hist[0].sum()) == n and int(hist[1].sum()) == n
+    j.close()

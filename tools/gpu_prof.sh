@@ -1,0 +1,11 @@
+# GPU session: tests + ncu launch list + full capture of the hot kernels.
+cd $GRAFT_REPO_ROOT
+python -c "import __graft_entry__ as g; g.build()" 2>&1 | tail -3
+timeout 1200 python -m pytest tests -m gpu -q --timeout 300 -rf 2>&1 | tail -15
+timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/launches.csv \
+    python bench.py --steps 2 --warmup 1 --profile > gpurun_out/launch_bench.log 2>&1
+echo "launch list rc=$?"
+timeout 1500 ncu --set full --clock-control none --import-source on -k regex:'k_(hist|scatter|local|probe)' -s 4 -c 4 \
+    -o gpurun_out/prof -f python bench.py --steps 1 --warmup 1 --profile > gpurun_out/prof.log 2>&1
+echo "full capture rc=$?"
+tail -3 gpurun_out/prof.log

@@ -10,18 +10,17 @@
 namespace mgj {
 
 constexpr int MAX_RANKS = MGJ_MAX_RANKS;
-constexpr int MAX_B1 = 12;              // scatter WC lines need >= 32 B per partition in 128 KB SMEM
+constexpr int MAX_B1 = 12;              // 2^12 global partitions at most
 constexpr int MAX_B2 = 11;              // local fan-out per pass
-constexpr int PROBE_CAP = 4096;         // R tuples per shared-memory hash table (a5)
-constexpr int PROBE_TARGET = 2048;      // expected R tuples per co-partition when B2 is auto
-constexpr int PROBE_S_TARGET = 32768;   // S tuples per probe work item (heavy S co-partitions split)
+constexpr int HIST_THREADS = 1024;
 constexpr int SCATTER_THREADS = 1024;
-constexpr int SCATTER_V = 4;            // tuples per thread per batch
-constexpr int SCATTER_BATCH = SCATTER_THREADS * SCATTER_V;
-constexpr int LOCAL_THREADS = 512;
-constexpr int LOCAL_V = 16;             // tuples per thread per chunk (8-byte tuples)
-constexpr int PROBE_THREADS = 512;
-constexpr int PROBE_WIN = 1024;         // chunk runs staged per window in the probe
+constexpr int SCAT_T8 = 8192;           // scatter sub-tile (tuples) for 8-byte tuples; 4096 for 16-byte
+constexpr int LOCAL_THREADS = 1024;
+constexpr int LOCAL_C8 = 8192;          // local-pass chunk (tuples) for 8-byte tuples; 4096 for 16-byte
+constexpr int PROBE_THREADS = 1024;     // warp 0 = TMA producer, warps 1..31 = build/probe consumers
+constexpr int PROBE_NST = 3;            // pipeline stages (items in flight per CTA)
+constexpr int PROBE_SLOTS8 = 3072;      // stage capacity per relation (slots) for 8-byte tuples; half for 16-byte
+constexpr int PROBE_MAXP = 1024;        // chunk pieces per relation per item
 constexpr uint64_t WAIT_TIMEOUT_NS = 20ull * 1000 * 1000 * 1000;
 
 enum Sig { SIG_HIST = 0, SIG_DATA = 1, SIG_RES = 2, SIG_COUNT = 3 };
@@ -39,18 +38,25 @@ struct Arena {
     uint64_t total;
 };
 
-struct Item {           // one probe work item: co-partition (p, q) slice
-    uint32_t pi;        // owned partition index (p - p_lo)
-    uint32_t q;         // local sub-partition
-    uint32_t r_lo, r_hi;// logical range in the concatenation of R runs of (p,q)
-    uint32_t s_lo, s_hi;
+// One probe work item: a slice of co-partition (p, q).  Each side is the
+// half-open range of (chunk k, slot offset a) positions [(k0, a0), (k1, a1))
+// over the q-runs of p's chunks (a counts padded 8/16-byte slots, even).
+struct Side {
+    uint32_t k0, a0, k1, a1;
+};
+struct Item {
+    uint32_t pi;  // owned partition index (p - p_lo)
+    uint32_t q;   // local sub-partition
+    Side r, s;
 };
 
 // Everything a kernel needs, passed by value (param space).
 struct Ctx {
     int32_t rank, world, B1, P, b2_cfg, b2_max;
-    int32_t line_tuples;          // scatter WC line length (tuples)
-    int32_t chunk_tuples;         // local-partition chunk size C (tuples)
+    int32_t G;                    // tiles per relation (= scatter CTAs)
+    int32_t chunk_tuples;         // local-pass chunk C (tuples)
+    int32_t chunk_region;         // slots per chunk in the local buffer (C + 2^b2_max, even)
+    int32_t probe_slots;          // probe stage capacity per relation (slots)
     int32_t materialize;
     uint32_t max_items;
     uint64_t epoch;
@@ -64,24 +70,32 @@ struct Ctx {
     uint64_t n_in[2];
     // workspace (this rank's device memory)
     uint32_t *rank_hist;          // [2][P]
+    uint32_t *tile_hist;          // [2][G][P] per-tile histograms (a1)
+    uint32_t *tile_base;          // [2][G][P] exclusive prefix over tiles
     uint32_t *ticket;             // [TK_COUNT]
     int32_t *meta;                // [MT_COUNT]
     int32_t *owner;               // [P]
     uint64_t *send_off;           // [2][P]
-    uint32_t *gcur;               // [2][P]  reservation cursor inside this rank's block
     uint64_t *seg_start;          // [2][P]
     uint64_t *seg_len;            // [2][P]
     uint64_t *recv_size;          // [2][MAX_RANKS]
     uint32_t *chunk_base;         // [2][P+1]
-    uint16_t *chunk_off[2];       // [max_chunks][2^b2_max + 1]
-    uint32_t *cop_count;          // [2][P][2^b2_max]
+    uint16_t *eoff[2];            // run offsets, [(Q+1)*chunk_base[p] + q*nch_p + k]
+    uint32_t *cop_slots;          // [2][P][2^b2_max] padded slots per co-partition
     Item *items;                  // [max_items]
-    void *local[2];               // locally partitioned tuples (a4 output)
+    void *local[2];               // locally partitioned tuples (a4 output), chunk regions
     unsigned long long *acc;      // [4] local count, checksum, n_out
     int32_t *err;                 // sticky device status
     unsigned long long *result;   // [4] global count, checksum; local n_out; status
     void *out_key, *out_a, *out_b;
 };
+
+// Tile c of G over n tuples: boundaries are multiples of 4 tuples (16-byte
+// aligned for the TMA loads); the last tile ends at n.
+__host__ __device__ __forceinline__ void tile_range(uint64_t n, int G, int c, uint64_t &lo, uint64_t &hi) {
+    lo = (n * (uint64_t)c / (uint64_t)G) & ~3ull;
+    hi = (c == G - 1) ? n : ((n * (uint64_t)(c + 1) / (uint64_t)G) & ~3ull);
+}
 
 template <typename K> struct TupT;
 template <> struct TupT<uint32_t> { using T = uint2; };       // {key, payload}

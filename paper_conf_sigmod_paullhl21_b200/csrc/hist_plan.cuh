@@ -10,48 +10,58 @@ namespace mgj {
 // a1: per-GPU radix histogram (§3.2 "Histogram generation",
 // P:356-370, built in shared memory after Rui et al. [38]; bin count from the
 // Eq. 1 analogue).  H[rel][p] = #{t in rel_g : digit1(t.key) = p}.
-// Reads only the key column with 16-byte vector loads.  The last CTA to
-// finish stores this rank's histogram into every peer's arena mailbox and
-// raises SIG_HIST there (the histogram exchange X4, fused into K1).
-// grid = (G, 2): blockIdx.y selects the relation.
+// grid = (G, 2): CTA (c, rel) counts tile c of relation rel (the same tiles
+// the scatter kernel processes) reading only the key column with 16-byte
+// streaming loads, and stores its per-tile histogram (so the scatter knows
+// its exact output offsets without atomics) and adds it into the rank
+// histogram.  The last CTA stores the rank histogram into every peer's
+// arena mailbox and raises SIG_HIST there (histogram exchange X4 fused).
 // ---------------------------------------------------------------------------
 template <typename K>
-__global__ void __launch_bounds__(512) k_hist(Ctx c) {
+__global__ void __launch_bounds__(HIST_THREADS) k_hist(Ctx c) {
     extern __shared__ uint32_t sh[];  // [P]
     const int P = c.P;
-    const int rel = blockIdx.y;
+    const int rel = blockIdx.y, tile = blockIdx.x;
     const K *keys = static_cast<const K *>(c.in_key[rel]);
-    const uint64_t n = c.n_in[rel];
+    uint64_t lo, hi;
+    tile_range(c.n_in[rel], c.G, tile, lo, hi);
     for (int i = threadIdx.x; i < P; i += blockDim.x) sh[i] = 0;
     __syncthreads();
 
     constexpr int VEC = 16 / sizeof(K);
-    const uint64_t nvec = n / VEC;
-    const uint4 *kv = reinterpret_cast<const uint4 *>(keys);
-    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
-    uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const uint64_t nvec = (hi - lo) / VEC;
+    const uint4 *kv = reinterpret_cast<const uint4 *>(keys + lo);
+    const uint32_t m = (uint32_t)(P - 1);
     auto count = [&](const uint4 &v) {
         if (sizeof(K) == 4) {
-            atomicAdd(&sh[v.x & (P - 1)], 1u);
-            atomicAdd(&sh[v.y & (P - 1)], 1u);
-            atomicAdd(&sh[v.z & (P - 1)], 1u);
-            atomicAdd(&sh[v.w & (P - 1)], 1u);
+            atomicAdd(&sh[v.x & m], 1u);
+            atomicAdd(&sh[v.y & m], 1u);
+            atomicAdd(&sh[v.z & m], 1u);
+            atomicAdd(&sh[v.w & m], 1u);
         } else {  // two 8-byte keys: low words are .x and .z
-            atomicAdd(&sh[v.x & (P - 1)], 1u);
-            atomicAdd(&sh[v.z & (P - 1)], 1u);
+            atomicAdd(&sh[v.x & m], 1u);
+            atomicAdd(&sh[v.z & m], 1u);
         }
     };
+    const uint64_t stride = blockDim.x;
+    uint64_t i = threadIdx.x;
     for (; i + 3 * stride < nvec; i += 4 * stride) {
-        uint4 v0 = __ldcs(kv + i), v1 = __ldcs(kv + i + stride);
-        uint4 v2 = __ldcs(kv + i + 2 * stride), v3 = __ldcs(kv + i + 3 * stride);
-        count(v0); count(v1); count(v2); count(v3);
+        const uint4 v0 = __ldcs(kv + i), v1 = __ldcs(kv + i + stride);
+        const uint4 v2 = __ldcs(kv + i + 2 * stride), v3 = __ldcs(kv + i + 3 * stride);
+        count(v0);
+        count(v1);
+        count(v2);
+        count(v3);
     }
     for (; i < nvec; i += stride) count(__ldcs(kv + i));
-    if (blockIdx.x == 0)
-        for (uint64_t t = nvec * VEC + threadIdx.x; t < n; t += blockDim.x) atomicAdd(&sh[digit1(keys[t], P)], 1u);
+    for (uint64_t t = lo + nvec * VEC + threadIdx.x; t < hi; t += blockDim.x) atomicAdd(&sh[digit1(keys[t], P)], 1u);
     __syncthreads();
-    for (int p = threadIdx.x; p < P; p += blockDim.x)
-        if (sh[p]) atomicAdd(&c.rank_hist[rel * P + p], sh[p]);
+    uint32_t *th = c.tile_hist + ((size_t)rel * c.G + tile) * P;
+    for (int p = threadIdx.x; p < P; p += blockDim.x) {
+        const uint32_t v = sh[p];
+        th[p] = v;
+        if (v) atomicAdd(&c.rank_hist[rel * P + p], v);
+    }
 
     // ---- fused exchange: the last CTA publishes the rank histogram ----
     __threadfence();
@@ -68,6 +78,37 @@ __global__ void __launch_bounds__(512) k_hist(Ctx c) {
     __threadfence_system();
     __syncthreads();
     if (threadIdx.x == 0) signal_all(c, SIG_HIST);
+}
+
+// Exclusive prefix of the per-tile histograms over tiles: tile c's tuples of
+// partition p start at send_off[p] + tile_base[rel][c][p] in the owner's
+// receive range (deterministic placement; one thread per (rel, p)).
+__global__ void k_tilescan(Ctx c) {
+    const int idx = blockIdx.x * blockDim.x + threadIdx.x;
+    if (idx >= 2 * c.P) return;
+    const int rel = idx / c.P, p = idx % c.P;
+    const size_t stride = c.P;
+    const uint32_t *src = c.tile_hist + (size_t)rel * c.G * c.P + p;
+    uint32_t *dst = c.tile_base + (size_t)rel * c.G * c.P + p;
+    uint32_t run = 0;
+    int t = 0;
+    for (; t + 4 <= c.G; t += 4) {
+        const uint32_t v0 = src[(t + 0) * stride], v1 = src[(t + 1) * stride];
+        const uint32_t v2 = src[(t + 2) * stride], v3 = src[(t + 3) * stride];
+        dst[(t + 0) * stride] = run;
+        run += v0;
+        dst[(t + 1) * stride] = run;
+        run += v1;
+        dst[(t + 2) * stride] = run;
+        run += v2;
+        dst[(t + 3) * stride] = run;
+        run += v3;
+    }
+    for (; t < c.G; ++t) {
+        const uint32_t v = src[t * stride];
+        dst[t * stride] = run;
+        run += v;
+    }
 }
 
 // ---------------------------------------------------------------------------
@@ -89,10 +130,11 @@ __host__ __device__ inline int ceil_log2_u64(uint64_t x) {
     return l;
 }
 
-// B2 from the largest owned R partition: co-partitions of ~PROBE_TARGET tuples.
-__host__ __device__ inline int choose_b2(uint64_t max_r, int b2_cfg, int b2_max) {
+// B2 from the largest owned R partition: co-partitions of ~target tuples
+// (2/3 of the probe stage capacity, so they fit one shared-memory table).
+__host__ __device__ inline int choose_b2(uint64_t max_r, int b2_cfg, int b2_max, uint64_t target) {
     if (b2_cfg > 0) return b2_cfg < b2_max ? b2_cfg : b2_max;
-    const uint64_t need = (max_r + PROBE_TARGET - 1) / PROBE_TARGET;
+    const uint64_t need = (max_r + target - 1) / target;
     int b = ceil_log2_u64(need);
     if (b > b2_max) b = b2_max;
     return b;
@@ -183,7 +225,7 @@ __global__ void __launch_bounds__(1024) k_plan(Ctx c) {
     const int phi = first[c.rank] < P ? endp[c.rank] : 0;
     for (int p = plo + tid; p < phi; p += blockDim.x) atomicMax(&maxr, (unsigned long long)tot0[p]);
     __syncthreads();
-    const int B2 = choose_b2(maxr, c.b2_cfg, c.b2_max);
+    const int B2 = choose_b2(maxr, c.b2_cfg, c.b2_max, (uint64_t)c.probe_slots * 2 / 3);
     // chunk table of the local pass: chunk_base[rel][pi] = first chunk of owned partition plo+pi
     const int np = phi - plo;
     const uint64_t C = (uint64_t)c.chunk_tuples;

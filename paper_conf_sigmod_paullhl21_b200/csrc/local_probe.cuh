@@ -3,312 +3,524 @@
 #pragma once
 
 #include "common.cuh"
+#include "tma.cuh"
 
 namespace mgj {
 
-template <typename K> struct LocalCfg {
+template <typename K> struct Layout {
     using Tup = typename TupT<K>::T;
-    static constexpr int V = LOCAL_V * 8 / (int)sizeof(Tup);  // 16 (8-byte) / 8 (16-byte) tuples per thread
-    static constexpr int C = V * LOCAL_THREADS;                // chunk size: 8192 / 4096 tuples
+    static constexpr int TB = (int)sizeof(Tup);
+    static constexpr int ALIGN = 16 / TB;  // tuples per 16 bytes: runs are padded to this (2 / 1)
 };
+
+// Run q of a chunk, decoded from the chunk's offset row E (reading of the
+// padded layout written by k_local): first slot, slots (padded length) and
+// valid tuples.  For 8-byte tuples E[q] = start | (count odd), E[Q] = end.
+template <int ALIGN>
+__device__ __forceinline__ void decode_run(uint32_t e0, uint32_t e1, uint32_t &start, uint32_t &slots,
+                                           uint32_t &valid) {
+    if (ALIGN == 2) {
+        start = e0 & ~1u;
+        slots = (e1 & ~1u) - start;
+        valid = slots - (e0 & 1u);
+    } else {
+        start = e0;
+        slots = e1 - e0;
+        valid = slots;
+    }
+}
+
+__host__ __device__ inline size_t local_smem_bytes(int C, int Qmax, int TB) {
+    return 2 * (size_t)(C + 2) * TB + (size_t)(C + Qmax) * TB + 2 * (size_t)Qmax * 4;
+}
+
+// Chunk descriptors for the local pass: chunk ci of owned partition pi covers
+// received tuples [start, start + len).
+struct ChunkDesc {
+    uint64_t start;
+    uint32_t len;
+    uint32_t pi;
+};
+
+__global__ void k_chunkmap(Ctx c, ChunkDesc *desc) {
+    if (!c.meta[MT_OK]) return;
+    const int P = c.P, plo = c.meta[MT_PLO], np = c.meta[MT_PHI] - plo;
+    const uint32_t nch_r = (uint32_t)c.meta[MT_NCH_R], total = nch_r + (uint32_t)c.meta[MT_NCH_S];
+    const uint64_t C = (uint64_t)c.chunk_tuples;
+    for (uint32_t ci = blockIdx.x * blockDim.x + threadIdx.x; ci < total; ci += gridDim.x * blockDim.x) {
+        const int rel = ci < nch_r ? 0 : 1;
+        const uint32_t li = rel ? ci - nch_r : ci;
+        const uint32_t *cb = c.chunk_base + rel * (P + 1);
+        int lo = 0, hi = np - 1;
+        while (lo < hi) {
+            const int mid = (lo + hi + 1) >> 1;
+            if (__ldg(cb + mid) <= li) lo = mid; else hi = mid - 1;
+        }
+        const uint64_t k = li - cb[lo];
+        const int p = plo + lo;
+        ChunkDesc d;
+        d.start = c.seg_start[rel * P + p] + k * C;
+        d.len = (uint32_t)min(C, c.seg_len[rel * P + p] - k * C);
+        d.pi = (uint32_t)lo;
+        desc[ci] = d;
+    }
+}
 
 // ---------------------------------------------------------------------------
 // a4 (§3.2 "Local partitioning"): the received data of
 // each owned global partition p is partitioned again by the next B2 key bits
-// so that every R co-partition fits the shared-memory hash table of a5.
-// B200 form: each CTA takes one chunk of C consecutive received tuples of a
-// segment, counting-sorts it by digit2 in shared memory (one SMEM atomic per
-// tuple gives both the bin count and the tuple's rank in its bin) and writes
-// the chunk back contiguously, plus its 2^B2+1 sub-partition offsets.  The
-// pass needs no global histogram and a chunk can be processed as soon as it
-// has arrived (the property P:455-468 asks of [44]); co-partition q of p is
-// the concatenation of the q-runs of p's chunks.  One pass suffices for every
-// configured size; R runs larger than the table are handled
-// by chunked builds in a5 (the skew case of P:450-452).
-// Grid: persistent over all chunks of both relations.
+// so that every R co-partition fits a shared-memory hash table.
+// B200 form: a persistent CTA per SM streams chunks of C received tuples in
+// by TMA (double-buffered, two chunks ahead), counting-sorts each chunk by
+// digit2 in shared memory (one SMEM atomic per tuple gives bin count and
+// rank), and streams the sorted chunk out with one TMA bulk store.  Runs are
+// padded to 16 bytes so the probe can fetch them with bulk copies; the run
+// offsets go to E[(Q+1)*chunk_base[p] + q*nch_p + k], i.e. contiguous per
+// (p, q).  No global histogram is needed and a chunk can be processed as soon
+// as it has arrived — the property the paper takes [44] for.
+// One pass suffices for every configured size; R co-partitions
+// larger than the table are built in pieces by a5 (P:450-452's skew case).
 // ---------------------------------------------------------------------------
 template <typename K>
-__global__ void __launch_bounds__(LOCAL_THREADS, 2) k_local(Ctx c) {
-    using Tup = typename TupT<K>::T;
-    constexpr int V = LocalCfg<K>::V;
-    constexpr int C = LocalCfg<K>::C;
-    extern __shared__ __align__(16) unsigned char smem[];
-    Tup *sbuf = reinterpret_cast<Tup *>(smem);
-    uint32_t *bins = reinterpret_cast<uint32_t *>(sbuf + C);  // [Q]
+__global__ void __launch_bounds__(LOCAL_THREADS, 1) k_local(Ctx c, const ChunkDesc *cdesc) {
+    using Tup = typename Layout<K>::Tup;
+    constexpr int TB = Layout<K>::TB, ALIGN = Layout<K>::ALIGN;
+    constexpr int VMAX = LOCAL_C8 * 8 / TB / LOCAL_THREADS;
+    extern __shared__ __align__(128) unsigned char smem[];
+    __shared__ __align__(8) uint64_t bar[2];
+    __shared__ ChunkDesc sdesc[2];
     __shared__ uint32_t tmp[33];
-    __shared__ int s_pi;
-    const int tid = threadIdx.x;
     if (!c.meta[MT_OK]) return;
-    const int P = c.P, plo = c.meta[MT_PLO], phi = c.meta[MT_PHI], B2 = c.meta[MT_B2];
-    const int Q = 1 << B2, np = phi - plo;
-    const uint32_t nch_r = (uint32_t)c.meta[MT_NCH_R], nch_s = (uint32_t)c.meta[MT_NCH_S];
-    const uint32_t total = nch_r + nch_s;
-    for (uint32_t ci = blockIdx.x; ci < total; ci += gridDim.x) {
+    const int tid = threadIdx.x;
+    const int C = c.chunk_tuples, CR = c.chunk_region, V = C / LOCAL_THREADS;
+    const int P = c.P, B2 = c.meta[MT_B2], Q = 1 << B2;
+    const int Qmax = 1 << c.b2_max;
+    Tup *const stage0 = reinterpret_cast<Tup *>(smem);
+    auto stage = [&](int s) { return stage0 + (size_t)s * (C + 2); };
+    Tup *sorted = stage0 + (size_t)2 * (C + 2);
+    uint32_t *bins = reinterpret_cast<uint32_t *>(sorted + C + Qmax);
+    uint32_t *abin = bins + Qmax;
+    const uint32_t nch_r = (uint32_t)c.meta[MT_NCH_R];
+    const uint32_t total = nch_r + (uint32_t)c.meta[MT_NCH_S];
+    const uint32_t mine = total > blockIdx.x ? (total - blockIdx.x + gridDim.x - 1) / gridDim.x : 0;
+    const char *recv0 = c.arena[c.rank];
+    if (tid == 0) {
+        mbar_init(&bar[0], 1);
+        mbar_init(&bar[1], 1);
+        fence_mbar_init();
+    }
+    __syncthreads();
+    const uint64_t pol = policy_evict_first();
+    // thread 0 keeps the descriptor of the next chunk to issue in registers (prefetched)
+    auto issue = [&](uint32_t j, const ChunkDesc &d) {
+        const uint32_t ci = blockIdx.x + j * gridDim.x;
+        const int rel = ci < nch_r ? 0 : 1;
+        const uint64_t g0 = d.start & ~(uint64_t)(ALIGN - 1);
+        const uint64_t g1 = (d.start + d.len + ALIGN - 1) & ~(uint64_t)(ALIGN - 1);
+        const uint32_t bytes = (uint32_t)((g1 - g0) * TB);
+        sdesc[j & 1] = d;
+        uint64_t *b = &bar[j & 1];
+        mbar_arrive_expect_tx(b, bytes);
+        if (bytes)
+            tma_load_1d(stage(j & 1), reinterpret_cast<const Tup *>(recv0 + c.lay.recv[rel]) + g0, bytes, b, pol);
+    };
+    ChunkDesc nxt{};
+    if (tid == 0) {
+        if (mine > 0) issue(0, cdesc[blockIdx.x]);
+        if (mine > 1) issue(1, cdesc[blockIdx.x + gridDim.x]);
+        if (mine > 2) nxt = cdesc[blockIdx.x + 2 * gridDim.x];
+    }
+    for (uint32_t j = 0; j < mine; ++j) {
+        const uint32_t ci = blockIdx.x + j * gridDim.x;
         const int rel = ci < nch_r ? 0 : 1;
         const uint32_t li = rel ? ci - nch_r : ci;
-        const uint32_t *cb = c.chunk_base + rel * (P + 1);
-        if (tid == 0) {  // owned partition of this chunk: last pi with cb[pi] <= li
-            int lo = 0, hi = np - 1;
-            while (lo < hi) {
-                const int mid = (lo + hi + 1) >> 1;
-                if (cb[mid] <= li) lo = mid; else hi = mid - 1;
-            }
-            s_pi = lo;
-        }
-        for (int i = tid; i < Q; i += LOCAL_THREADS) bins[i] = 0;
-        __syncthreads();
-        const int pi = s_pi, p = plo + pi;
-        const uint64_t k = li - cb[pi];
-        const uint64_t start = c.seg_start[rel * P + p] + k * C;
-        const uint32_t len = (uint32_t)min((uint64_t)C, c.seg_len[rel * P + p] - k * C);
-        const Tup *src = reinterpret_cast<const Tup *>(c.arena[c.rank] + c.lay.recv[rel]) + start;
-        Tup *dst = static_cast<Tup *>(c.local[rel]) + start;
-        Tup t[V];
-        uint32_t qr[V];  // (rank in bin) << 16 | digit2
+        const int s = j & 1;
+        mbar_wait(&bar[s], (j >> 1) & 1);
+        const ChunkDesc d = sdesc[s];
+        const uint32_t len = d.len, skip = (uint32_t)(d.start & (ALIGN - 1));
+        Tup t[VMAX];
 #pragma unroll
-        for (int j = 0; j < V; ++j) {
-            const uint32_t i = tid + j * LOCAL_THREADS;
-            if (i < len) t[j] = __ldcs(src + i);
+        for (int v = 0; v < VMAX; ++v) {
+            const uint32_t i = tid + v * LOCAL_THREADS;
+            if (v < V && i < len) t[v] = stage(s)[skip + i];
         }
+        for (int q = tid; q < Q; q += LOCAL_THREADS) bins[q] = 0;
+        __syncthreads();  // S1: stage s consumed
+        if (tid == 0 && j + 2 < mine) {
+            issue(j + 2, nxt);
+            if (j + 3 < mine) nxt = cdesc[blockIdx.x + (j + 3) * gridDim.x];
+        }
+        uint32_t rq[VMAX];  // rank << 16 | digit2
 #pragma unroll
-        for (int j = 0; j < V; ++j) {
-            const uint32_t i = tid + j * LOCAL_THREADS;
-            if (i < len) {
-                const uint32_t q = digit2(t[j].x, c.B1, Q);
-                qr[j] = (atomicAdd(&bins[q], 1u) << 16) | q;
+        for (int v = 0; v < VMAX; ++v) {
+            const uint32_t i = tid + v * LOCAL_THREADS;
+            if (v < V && i < len) {
+                const uint32_t q = digit2(t[v].x, c.B1, Q);
+                rq[v] = (atomicAdd(&bins[q], 1u) << 16) | q;
             }
         }
+        if (tid == 0) bulk_wait_read0();  // previous chunk's bulk store has read `sorted`
+        __syncthreads();  // S2
+        for (int q = tid; q < Q; q += LOCAL_THREADS) abin[q] = (bins[q] + ALIGN - 1) & ~(uint32_t)(ALIGN - 1);
         __syncthreads();
-        block_excl_scan_u32(bins, Q, tmp);
-        uint16_t *coff = c.chunk_off[rel] + (size_t)li * (Q + 1);
-        uint32_t *cop = c.cop_count + ((size_t)rel * P + pi) * Q;
-        for (int i = tid; i <= Q; i += LOCAL_THREADS) {
-            const uint32_t b = i < Q ? bins[i] : len;
-            coff[i] = (uint16_t)b;
-            if (i < Q) {
-                const uint32_t e = (i + 1 < Q) ? bins[i + 1] : len;
-                if (e > b) atomicAdd(&cop[i], e - b);
+        const uint32_t tot = block_excl_scan_u32(abin, Q, tmp);
+        {
+            const uint32_t *cb = c.chunk_base + rel * (P + 1);
+            const uint32_t cbp = cb[d.pi], nchp = cb[d.pi + 1] - cbp;
+            uint16_t *E = c.eoff[rel] + (size_t)(Q + 1) * cbp + (li - cbp);
+            uint32_t *cop = c.cop_slots + ((size_t)rel * P + d.pi) * Q;
+            for (int q = tid; q <= Q; q += LOCAL_THREADS) {
+                if (q < Q) {
+                    const uint32_t n = bins[q];
+                    E[(size_t)q * nchp] = (uint16_t)(abin[q] | (ALIGN == 2 ? (n & 1u) : 0u));
+                    if (n) atomicAdd(&cop[q], (n + ALIGN - 1) & ~(uint32_t)(ALIGN - 1));
+                } else {
+                    E[(size_t)q * nchp] = (uint16_t)tot;
+                }
             }
         }
 #pragma unroll
-        for (int j = 0; j < V; ++j) {
-            const uint32_t i = tid + j * LOCAL_THREADS;
-            if (i < len) sbuf[bins[qr[j] & 0xffffu] + (qr[j] >> 16)] = t[j];
+        for (int v = 0; v < VMAX; ++v) {
+            const uint32_t i = tid + v * LOCAL_THREADS;
+            if (v < V && i < len) sorted[abin[rq[v] & 0xffffu] + (rq[v] >> 16)] = t[v];
         }
-        __syncthreads();
-        for (uint32_t i = tid; i < len; i += LOCAL_THREADS) __stcs(dst + i, sbuf[i]);
-        __syncthreads();
+        fence_proxy_async_smem();
+        __syncthreads();  // S3
+        if (tid == 0 && tot) {
+            Tup *dst = static_cast<Tup *>(c.local[rel]) + (size_t)li * CR;
+            tma_store_1d(dst, sorted, tot * TB);
+            bulk_commit();
+        }
     }
+    if (tid == 0) bulk_wait0();
 }
 
 // ---------------------------------------------------------------------------
-// Probe work items: co-partition (p, q) becomes ceil(|R_pq|/PROBE_CAP) x
-// ceil(|S_pq|/PROBE_S_TARGET) items, so an oversized R co-partition is built
-// in table-sized chunks (block nested loop over R chunks, the "both
-// relations heavily skewed" case of P:450-452) and a heavy S co-partition is
-// probed by many CTAs.
+// Probe work items.  Co-partition (p, q) is one item when both of its sides
+// fit a pipeline stage (the common case); otherwise each side is cut into
+// stage-sized slices (at even slot offsets) and every R slice is paired with
+// every S slice: an oversized R co-partition is built in table-sized pieces
+// (block nested loop over R slices — the "both relations heavily skewed"
+// case of P:450-452) and a heavy S co-partition is spread over many CTAs.
 // ---------------------------------------------------------------------------
+struct ItemX {
+    Item it;
+    uint32_t cb[2], nch[2];  // first chunk / chunk count of p per relation
+};
+
+// Walk the q-runs of one side in chunk order and cut it into slices of at
+// most `cap` slots and `maxp` chunk pieces; call emit(slice) for each.
+template <int ALIGN, typename F>
+__device__ inline void walk_side(const uint16_t *E0, const uint16_t *E1, uint32_t nch, uint32_t cap,
+                                 uint32_t maxp, F &&emit) {
+    uint32_t acc = 0, npc = 0;
+    Side cur{0, 0, 0, 0};
+    for (uint32_t k = 0; k < nch; ++k) {
+        uint32_t st, slots, valid;
+        decode_run<ALIGN>(E0[k], E1[k], st, slots, valid);
+        uint32_t a = 0;
+        do {
+            if (npc == maxp || (acc == cap && a < slots)) {
+                cur.k1 = k;
+                cur.a1 = a;
+                emit(cur);
+                cur = Side{k, a, 0, 0};
+                acc = 0;
+                npc = 0;
+            }
+            const uint32_t take = min(slots - a, cap - acc);
+            acc += take;
+            a += take;
+            ++npc;
+        } while (a < slots);
+    }
+    if (acc > 0) {
+        cur.k1 = nch;
+        cur.a1 = 0;
+        emit(cur);
+    }
+}
+
+template <typename K>
 __global__ void k_itemize(Ctx c) {
+    constexpr int ALIGN = Layout<K>::ALIGN;
     if (!c.meta[MT_OK]) return;
     const int P = c.P, plo = c.meta[MT_PLO], phi = c.meta[MT_PHI];
     const int Q = 1 << c.meta[MT_B2];
+    const uint32_t cap = (uint32_t)c.probe_slots;
+    ItemX *items = reinterpret_cast<ItemX *>(c.items);
     const uint64_t total = (uint64_t)(phi - plo) * Q;
     for (uint64_t idx = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; idx < total;
          idx += (uint64_t)gridDim.x * blockDim.x) {
         const uint32_t pi = (uint32_t)(idx / Q), q = (uint32_t)(idx % Q);
-        const uint32_t r = c.cop_count[(size_t)pi * Q + q];
-        const uint32_t s = c.cop_count[((size_t)P + pi) * Q + q];
+        const uint32_t r = c.cop_slots[(size_t)pi * Q + q];
+        const uint32_t s = c.cop_slots[((size_t)P + pi) * Q + q];
         if (r == 0 || s == 0) continue;
-        const uint32_t nr = (r + PROBE_CAP - 1) / PROBE_CAP;
-        const uint32_t ns = (s + PROBE_S_TARGET - 1) / PROBE_S_TARGET;
+        ItemX x;
+        x.it.pi = pi;
+        x.it.q = q;
+        for (int rel = 0; rel < 2; ++rel) {
+            const uint32_t *cb = c.chunk_base + rel * (P + 1);
+            x.cb[rel] = cb[pi];
+            x.nch[rel] = cb[pi + 1] - cb[pi];
+        }
+        if (r <= cap && s <= cap && x.nch[0] <= PROBE_MAXP && x.nch[1] <= PROBE_MAXP) {
+            x.it.r = Side{0, 0, x.nch[0], 0};
+            x.it.s = Side{0, 0, x.nch[1], 0};
+            const uint32_t b = atomicAdd(&c.ticket[TK_ITEMS], 1u);
+            if (b < c.max_items) items[b] = x;
+            else set_err(c, MGJ_ECAPACITY);
+            continue;
+        }
+        // slow path: slice both sides, pair every R slice with every S slice
+        const uint16_t *E[2][2];
+        for (int rel = 0; rel < 2; ++rel) {
+            E[rel][0] = c.eoff[rel] + (size_t)(Q + 1) * x.cb[rel] + (size_t)q * x.nch[rel];
+            E[rel][1] = E[rel][0] + x.nch[rel];
+        }
+        uint32_t nr = 0, ns = 0;
+        walk_side<ALIGN>(E[0][0], E[0][1], x.nch[0], cap, PROBE_MAXP, [&](const Side &) { ++nr; });
+        walk_side<ALIGN>(E[1][0], E[1][1], x.nch[1], cap, PROBE_MAXP, [&](const Side &) { ++ns; });
         const uint64_t n = (uint64_t)nr * ns;
-        const uint32_t base = atomicAdd(&c.ticket[TK_ITEMS], (uint32_t)n);
-        if ((uint64_t)base + n > c.max_items) {
+        const uint32_t b = atomicAdd(&c.ticket[TK_ITEMS], (uint32_t)min(n, (uint64_t)0x7fffffffu));
+        if ((uint64_t)b + n > c.max_items) {
             set_err(c, MGJ_ECAPACITY);
             continue;
         }
-        for (uint32_t a = 0; a < nr; ++a)
-            for (uint32_t b = 0; b < ns; ++b) {
-                Item it;
-                it.pi = pi;
-                it.q = q;
-                it.r_lo = (uint32_t)((uint64_t)r * a / nr);
-                it.r_hi = (uint32_t)((uint64_t)r * (a + 1) / nr);
-                it.s_lo = (uint32_t)((uint64_t)s * b / ns);
-                it.s_hi = (uint32_t)((uint64_t)s * (b + 1) / ns);
-                c.items[base + a * ns + b] = it;
-            }
+        uint32_t ir = 0;
+        walk_side<ALIGN>(E[0][0], E[0][1], x.nch[0], cap, PROBE_MAXP, [&](const Side &rs) {
+            uint32_t is = 0;
+            walk_side<ALIGN>(E[1][0], E[1][1], x.nch[1], cap, PROBE_MAXP, [&](const Side &ss) {
+                ItemX y = x;
+                y.it.r = rs;
+                y.it.s = ss;
+                items[b + (uint64_t)ir * ns + is] = y;
+                ++is;
+            });
+            ++ir;
+        });
     }
 }
 
-// Walk the q-runs of owned partition pi (= p - p_lo) of relation rel in
-// logical order (chunk order) and hand every part of a run that falls in the
-// logical range [lo, hi) to a warp: f(src, n, first) is called by all 32
-// lanes of one warp for n consecutive tuples at src whose first tuple has
-// logical index lo + first.  Chunk runs are staged PROBE_WIN at a time.
-template <typename Tup, typename F>
-__device__ inline void for_runs(const Ctx &c, int rel, int pi, int p, uint32_t q, int Q, uint32_t lo, uint32_t hi,
-                                int C, uint32_t *rlen, uint32_t *rpos, uint32_t *tmp, F &&f) {
-    const int tid = threadIdx.x, warp = tid >> 5, nw = blockDim.x >> 5;
-    const uint32_t *cbp = c.chunk_base + rel * (c.P + 1);
-    const uint32_t cb = cbp[pi], nch = cbp[pi + 1] - cb;
-    const uint16_t *coff = c.chunk_off[rel] + (size_t)cb * (Q + 1);
-    const Tup *base = static_cast<const Tup *>(c.local[rel]) + c.seg_start[rel * c.P + p];
-    uint32_t logical = 0;
-    for (uint32_t w0 = 0; w0 < nch && logical < hi; w0 += PROBE_WIN) {
-        const uint32_t wn = min((uint32_t)PROBE_WIN, nch - w0);
-        for (uint32_t k = tid; k < wn; k += blockDim.x) {
-            const uint16_t *row = coff + (size_t)(w0 + k) * (Q + 1);
-            const uint32_t s = row[q], e = row[q + 1];
-            rlen[k] = e - s;
-            rpos[k] = (w0 + k) * (uint32_t)C + s;
-        }
-        __syncthreads();
-        const uint32_t tot = block_excl_scan_u32(rlen, (int)wn, tmp);
-        for (uint32_t k = warp; k < wn; k += nw) {
-            const uint32_t a = logical + rlen[k];
-            const uint32_t b = logical + (k + 1 < wn ? rlen[k + 1] : tot);
-            const uint32_t x0 = max(a, lo), x1 = min(b, hi);
-            if (x0 < x1) f(base + rpos[k] + (x0 - a), x1 - x0, x0 - lo);
-        }
-        logical += tot;
-        __syncthreads();
-    }
+__host__ __device__ inline size_t probe_smem_bytes(int slots, int TB) {
+    return (size_t)PROBE_NST * 2 * slots * TB        // stages (R, S)
+           + (size_t)PROBE_NST * 2 * PROBE_MAXP * 4  // piece descriptors
+           + 4096 * 4                                // head
+           + (size_t)slots * 2;                      // next
 }
 
 // ---------------------------------------------------------------------------
-// a5 (§3.2 "Probe"): per work item, the R slice of
-// co-partition (p, q) is gathered into shared memory and a chained hash
-// table is built over it (the SMEM hash-table variant of P:471-472, which the
-// north star asks for; the paper's nested loop is its degenerate form), then
-// the S slice streams through: one warp per run, lanes walk chains and
-// compare full keys.  count += 1 and checksum += a*C + b (mod 2^64) for every
-// equal-key pair; with MAT the item's matches are first counted, one
-// reservation is taken in the output, and a second pass over the (L2-
-// resident) S slice writes the (key, payR, payS) triples at exact positions.
+// a5 (§3.2 "Probe"): the co-partitions of R and S with
+// the same partition id are joined; the paper notes the nested-loop and the
+// shared-memory hash-table variants perform alike and the north
+// star asks for the hash table.  Warp-specialised, PROBE_NST-stage pipeline:
+//  - warp 0 (producer) walks the run offsets of the next items and issues
+//    one TMA bulk copy per (chunk, relation) run into a free stage;
+//  - warps 1..31 (consumers) build a chained hash table over the stage's R
+//    runs (head entries tagged with the item, so the table is never
+//    cleared), then stream the S runs through it: count += 1 and
+//    checksum += a*C + b (mod 2^64) for every equal-key pair.  With MAT the
+//    item's matches are counted, one output reservation is taken, and a
+//    second pass over the S runs in shared memory writes (key, payR, payS).
 // ---------------------------------------------------------------------------
 template <typename K, bool MAT>
-__global__ void __launch_bounds__(PROBE_THREADS) k_probe(Ctx c) {
-    using Tup = typename TupT<K>::T;
-    constexpr int C = LocalCfg<K>::C;
-    constexpr int T = PROBE_CAP;
-    constexpr int LOGT = 12;
-    constexpr uint32_t EMPTY = 0xffffffffu;
-    static_assert((1 << LOGT) == T, "table size");
-    extern __shared__ __align__(16) unsigned char smem[];
-    Tup *rt = reinterpret_cast<Tup *>(smem);
-    uint32_t *head = reinterpret_cast<uint32_t *>(rt + PROBE_CAP);
-    uint32_t *nxt = head + T;
-    uint32_t *rlen = nxt + PROBE_CAP;
-    uint32_t *rpos = rlen + PROBE_WIN;
-    __shared__ uint32_t tmp[33];
+__global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
+    using Tup = typename Layout<K>::Tup;
+    constexpr int TB = Layout<K>::TB, ALIGN = Layout<K>::ALIGN;
+    constexpr int LOGT = 12, T = 1 << LOGT;
+    constexpr uint16_t END = 0xffff;
+    constexpr int NCONS = PROBE_THREADS - 32;
+    extern __shared__ __align__(128) unsigned char smem[];
+    __shared__ __align__(8) uint64_t full[PROBE_NST], empty[PROBE_NST];
+    __shared__ uint32_t npieces[PROBE_NST][2];
+    __shared__ uint32_t s_m;
     __shared__ unsigned long long s_base;
-    __shared__ uint32_t s_cur, s_m;
     __shared__ int s_write;
     if (!c.meta[MT_OK]) return;
-    const int tid = threadIdx.x, lane = tid & 31;
-    const int plo = c.meta[MT_PLO], B2 = c.meta[MT_B2];
+    const int SL = c.probe_slots;
+    Tup *stages = reinterpret_cast<Tup *>(smem);  // [NST][2][SL]
+    uint32_t *desc = reinterpret_cast<uint32_t *>(stages + (size_t)PROBE_NST * 2 * SL);  // [NST][2][MAXP]
+    uint32_t *head = desc + PROBE_NST * 2 * PROBE_MAXP;
+    uint16_t *nxt = reinterpret_cast<uint16_t *>(head + T);
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const int B2 = c.meta[MT_B2];
     const int Q = 1 << B2, shift = c.B1 + B2;
     const uint32_t nitems = min(__ldcg(&c.ticket[TK_ITEMS]), c.max_items);
+    const uint32_t mine = nitems > blockIdx.x ? (nitems - blockIdx.x + gridDim.x - 1) / gridDim.x : 0;
+    const ItemX *items = reinterpret_cast<const ItemX *>(c.items);
+    if (tid == 0) {
+        for (int s = 0; s < PROBE_NST; ++s) {
+            mbar_init(&full[s], 1);
+            mbar_init(&empty[s], 1);
+        }
+        fence_mbar_init();
+    }
+    for (int i = tid; i < T; i += PROBE_THREADS) head[i] = 0;
+    __syncthreads();
+
+    if (warp == 0) {
+        // ------------------------------------------------------- producer
+        const uint64_t pol = policy_evict_first();
+        for (uint32_t j = 0; j < mine; ++j) {
+            const int s = j % PROBE_NST;
+            if (j >= PROBE_NST) mbar_wait(&empty[s], ((j / PROBE_NST) - 1) & 1);
+            const ItemX x = items[blockIdx.x + j * gridDim.x];
+            for (int rel = 0; rel < 2; ++rel) {
+                const Side sd = rel ? x.it.s : x.it.r;
+                const uint16_t *E0 = c.eoff[rel] + (size_t)(Q + 1) * x.cb[rel] + (size_t)x.it.q * x.nch[rel];
+                const uint16_t *E1 = E0 + x.nch[rel];
+                const uint32_t kend = min(sd.k1, x.nch[rel] - 1);
+                const uint32_t np = sd.k0 <= kend ? kend - sd.k0 + 1 : 0;
+                Tup *dstbase = stages + ((size_t)s * 2 + rel) * SL;
+                uint32_t *dsc = desc + ((size_t)s * 2 + rel) * PROBE_MAXP;
+                const Tup *lbase = static_cast<const Tup *>(c.local[rel]);
+                uint32_t run = 0;
+                for (uint32_t m0 = 0; m0 < np; m0 += 32) {
+                    const uint32_t m = m0 + lane;
+                    uint32_t sz = 0, valid = 0;
+                    uint64_t src = 0;
+                    if (m < np) {
+                        const uint32_t k = sd.k0 + m;
+                        uint32_t st, slots, v;
+                        decode_run<ALIGN>(E0[k], E1[k], st, slots, v);
+                        const uint32_t alo = (k == sd.k0) ? sd.a0 : 0;
+                        const uint32_t ahi = (k == sd.k1) ? sd.a1 : slots;
+                        if (ahi > alo) {
+                            sz = ahi - alo;
+                            valid = min(ahi, v) > alo ? min(ahi, v) - alo : 0;
+                            src = (uint64_t)(x.cb[rel] + k) * c.chunk_region + st + alo;
+                        }
+                    }
+                    uint32_t incl = sz;
+#pragma unroll
+                    for (int o = 1; o < 32; o <<= 1) {
+                        const uint32_t y = __shfl_up_sync(0xffffffffu, incl, o);
+                        if (lane >= o) incl += y;
+                    }
+                    const uint32_t dst = run + incl - sz;
+                    const uint32_t gsum = __shfl_sync(0xffffffffu, incl, 31);
+                    if (m < np) dsc[m] = dst | (valid << 16);
+                    if (lane == 0 && gsum)
+                        asm volatile("mbarrier.expect_tx.relaxed.cta.shared::cta.b64 [%0], %1;" ::"r"(
+                                         smem_u32(&full[s])),
+                                     "r"(gsum * TB)
+                                     : "memory");
+                    __syncwarp();
+                    if (sz) tma_load_1d(dstbase + dst, lbase + src, sz * TB, &full[s], pol);
+                    run += gsum;
+                }
+                if (lane == 0) npieces[s][rel] = np;
+            }
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&full[s]);
+        }
+        return;
+    }
+
+    // ------------------------------------------------------------ consumers
+    const int cw = warp - 1, ncw = PROBE_THREADS / 32 - 1;
     unsigned long long my_cnt = 0, my_chk = 0;
-
-    for (uint32_t it = blockIdx.x; it < nitems; it += gridDim.x) {
-        const Item I = c.items[it];
-        const int pi = (int)I.pi, p = plo + pi;
-        const uint32_t nr = I.r_hi - I.r_lo;
-        for (int i = tid; i < T; i += PROBE_THREADS) head[i] = EMPTY;
-        for_runs<Tup>(c, 0, pi, p, I.q, Q, I.r_lo, I.r_hi, C, rlen, rpos, tmp,
-                      [&](const Tup *src, uint32_t n, uint32_t first) {
-                          for (uint32_t x = lane; x < n; x += 32) rt[first + x] = src[x];
-                      });
-        for (uint32_t i = tid; i < nr; i += PROBE_THREADS) nxt[i] = atomicExch(&head[tab_hash(rt[i].x, shift, LOGT)], i);
-        __syncthreads();
-
-        if (!MAT) {
-            for_runs<Tup>(c, 1, pi, p, I.q, Q, I.s_lo, I.s_hi, C, rlen, rpos, tmp,
-                          [&](const Tup *src, uint32_t n, uint32_t) {
-                              for (uint32_t x = lane; x < n; x += 32) {
-                                  const Tup s = src[x];
-                                  for (uint32_t i = head[tab_hash(s.x, shift, LOGT)]; i != EMPTY; i = nxt[i]) {
-                                      const Tup r = rt[i];
-                                      if (r.x == s.x) {
-                                          ++my_cnt;
-                                          my_chk += chk_term(r.y, s.y);
-                                      }
-                                  }
-                              }
-                          });
-        } else {
-            uint32_t m = 0;
-            for_runs<Tup>(c, 1, pi, p, I.q, Q, I.s_lo, I.s_hi, C, rlen, rpos, tmp,
-                          [&](const Tup *src, uint32_t n, uint32_t) {
-                              for (uint32_t x = lane; x < n; x += 32) {
-                                  const Tup s = src[x];
-                                  for (uint32_t i = head[tab_hash(s.x, shift, LOGT)]; i != EMPTY; i = nxt[i]) {
-                                      const Tup r = rt[i];
-                                      if (r.x == s.x) {
-                                          ++m;
-                                          my_chk += chk_term(r.y, s.y);
-                                      }
-                                  }
-                              }
-                          });
-            my_cnt += m;
-            if (tid == 0) s_m = 0;
-            __syncthreads();
-            const uint32_t wm = (uint32_t)warp_sum(m);
+    uint32_t tag = 0;
+    for (uint32_t j = 0; j < mine; ++j) {
+        const int s = j % PROBE_NST;
+        if (++tag == 0x10000u) {  // tag wrap: clear the table once every 65535 items
+            for (int i = tid - 32; i < T; i += NCONS) head[i] = 0;
+            named_bar_sync(1, NCONS);
+            tag = 1;
+        }
+        mbar_wait(&full[s], (j / PROBE_NST) & 1);
+        const Tup *rt = stages + ((size_t)s * 2 + 0) * SL;
+        const Tup *st = stages + ((size_t)s * 2 + 1) * SL;
+        const uint32_t *dR = desc + ((size_t)s * 2 + 0) * PROBE_MAXP;
+        const uint32_t *dS = desc + ((size_t)s * 2 + 1) * PROBE_MAXP;
+        const uint32_t npR = npieces[s][0], npS = npieces[s][1];
+        // build
+        for (uint32_t m = cw; m < npR; m += ncw) {
+            const uint32_t d = dR[m], base = d & 0xffffu, v = d >> 16;
+            for (uint32_t x = lane; x < v; x += 32) {
+                const uint32_t slot = base + x;
+                const uint32_t h = tab_hash(rt[slot].x, shift, LOGT);
+                const uint32_t old = atomicExch(&head[h], (tag << 16) | slot);
+                nxt[slot] = (old >> 16) == tag ? (uint16_t)(old & 0xffffu) : END;
+            }
+        }
+        named_bar_sync(1, NCONS);
+        // probe
+        uint32_t m_item = 0;
+        for (uint32_t m = cw; m < npS; m += ncw) {
+            const uint32_t d = dS[m], base = d & 0xffffu, v = d >> 16;
+            for (uint32_t x = lane; x < v; x += 32) {
+                const Tup sv = st[base + x];
+                const uint32_t hv = head[tab_hash(sv.x, shift, LOGT)];
+                uint32_t i = (hv >> 16) == tag ? (hv & 0xffffu) : END;
+                while (i != END) {
+                    const Tup rv = rt[i];
+                    if (rv.x == sv.x) {
+                        ++m_item;
+                        my_chk += chk_term(rv.y, sv.y);
+                    }
+                    i = nxt[i];
+                }
+            }
+        }
+        my_cnt += m_item;
+        if (MAT) {
+            if (tid == 32) s_m = 0;
+            named_bar_sync(1, NCONS);
+            const uint32_t wm = (uint32_t)warp_sum(m_item);
             if (lane == 0 && wm) atomicAdd(&s_m, wm);
-            __syncthreads();
-            if (tid == 0) {
+            named_bar_sync(1, NCONS);
+            if (tid == 32) {
                 const uint32_t M = s_m;
-                s_cur = 0;
                 s_base = M ? atomicAdd(&c.acc[2], (unsigned long long)M) : 0;
                 s_write = M && (s_base + M <= c.out_cap);
                 if (M && !s_write) set_err(c, MGJ_ECAPACITY);
+                s_m = 0;  // reused as the write cursor
             }
-            __syncthreads();
+            named_bar_sync(1, NCONS);
             if (s_write) {
                 K *ok = static_cast<K *>(c.out_key);
                 K *oa = static_cast<K *>(c.out_a);
                 K *ob = static_cast<K *>(c.out_b);
-                const unsigned long long base = s_base;
-                for_runs<Tup>(c, 1, pi, p, I.q, Q, I.s_lo, I.s_hi, C, rlen, rpos, tmp,
-                              [&](const Tup *src, uint32_t n, uint32_t) {
-                                  for (uint32_t x0 = 0; x0 < n; x0 += 32) {
-                                      const uint32_t x = x0 + lane;
-                                      Tup s;
-                                      uint32_t i = EMPTY;
-                                      if (x < n) {
-                                          s = src[x];
-                                          i = head[tab_hash(s.x, shift, LOGT)];
-                                      }
-                                      while (__any_sync(0xffffffffu, i != EMPTY)) {
-                                          bool hit = false;
-                                          Tup r;
-                                          if (i != EMPTY) {
-                                              r = rt[i];
-                                              hit = r.x == s.x;
-                                              i = nxt[i];
-                                          }
-                                          const uint32_t bal = __ballot_sync(0xffffffffu, hit);
-                                          if (bal) {
-                                              uint32_t wb = 0;
-                                              if (lane == 0) wb = atomicAdd(&s_cur, (uint32_t)__popc(bal));
-                                              wb = __shfl_sync(0xffffffffu, wb, 0);
-                                              if (hit) {
-                                                  const unsigned long long pos =
-                                                      base + wb + __popc(bal & ((1u << lane) - 1u));
-                                                  ok[pos] = (K)s.x;
-                                                  oa[pos] = (K)r.y;
-                                                  ob[pos] = (K)s.y;
-                                              }
-                                          }
-                                      }
-                                  }
-                              });
+                const unsigned long long obase = s_base;
+                for (uint32_t m = cw; m < npS; m += ncw) {
+                    const uint32_t d = dS[m], base = d & 0xffffu, v = d >> 16;
+                    for (uint32_t x0 = 0; x0 < v; x0 += 32) {
+                        const uint32_t x = x0 + lane;
+                        Tup sv;
+                        uint32_t i = END;
+                        if (x < v) {
+                            sv = st[base + x];
+                            const uint32_t hv = head[tab_hash(sv.x, shift, LOGT)];
+                            i = (hv >> 16) == tag ? (hv & 0xffffu) : END;
+                        }
+                        while (__any_sync(0xffffffffu, i != END)) {
+                            bool hit = false;
+                            Tup rv;
+                            if (i != END) {
+                                rv = rt[i];
+                                hit = rv.x == sv.x;
+                                i = nxt[i];
+                            }
+                            const uint32_t bal = __ballot_sync(0xffffffffu, hit);
+                            if (bal) {
+                                uint32_t wb = 0;
+                                if (lane == 0) wb = atomicAdd(&s_m, (uint32_t)__popc(bal));
+                                wb = __shfl_sync(0xffffffffu, wb, 0);
+                                if (hit) {
+                                    const unsigned long long pos = obase + wb + __popc(bal & ((1u << lane) - 1u));
+                                    ok[pos] = (K)sv.x;
+                                    oa[pos] = (K)rv.y;
+                                    ob[pos] = (K)sv.y;
+                                }
+                            }
+                        }
+                    }
+                }
             }
         }
-        __syncthreads();
+        named_bar_sync(1, NCONS);  // stage s and the table are free
+        if (tid == 32) mbar_arrive(&empty[s]);
     }
     my_cnt = warp_sum(my_cnt);
     my_chk = warp_sum(my_chk);

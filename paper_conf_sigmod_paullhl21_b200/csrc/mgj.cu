@@ -26,7 +26,7 @@ uint64_t align_up(uint64_t x, uint64_t a) { return (x + a - 1) / a * a; }
 
 struct Norm {  // validated config with the automatic fields filled in
     mgj_config c;
-    int B1, P, b2_max, tuple_bytes, line_tuples, chunk_tuples;
+    int B1, P, b2_max, tuple_bytes, chunk_tuples, chunk_region, probe_slots;
     uint64_t recv_cap[2], max_chunks, max_items, out_cap;
     Arena lay;
 };
@@ -58,23 +58,26 @@ mgj_status normalize(const mgj_config *in, Norm *o) {
     o->B1 = c.radix_bits_global;
     o->P = 1 << o->B1;
     o->tuple_bytes = 2 * c.key_bytes;
-    const int line_bytes = std::min(128, (128 * 1024) / o->P);
-    o->line_tuples = line_bytes / o->tuple_bytes;
-    if (o->line_tuples < 1) return MGJ_EINVAL;
-    o->chunk_tuples = LOCAL_THREADS * LOCAL_V * 8 / o->tuple_bytes;
     o->recv_cap[0] = c.recv_capacity_r;
     o->recv_cap[1] = c.recv_capacity_s;
+    o->probe_slots = PROBE_SLOTS8 * 8 / o->tuple_bytes;
+    const uint64_t target = (uint64_t)o->probe_slots * 2 / 3;
     // B2 upper bound: the largest R segment this rank could own is recv_cap_r.
     if (c.radix_bits_local > 0) {
         o->b2_max = c.radix_bits_local;
     } else {
-        o->b2_max = std::min(MAX_B2, std::max(1, ceil_log2((c.recv_capacity_r + PROBE_TARGET - 1) / PROBE_TARGET)));
+        o->b2_max = std::min(MAX_B2, std::max(1, ceil_log2((c.recv_capacity_r + target - 1) / target)));
     }
+    const int Qm = 1 << o->b2_max;
+    int C = LOCAL_C8 * 8 / o->tuple_bytes;
+    while (C > LOCAL_THREADS && local_smem_bytes(C, Qm, o->tuple_bytes) > 225 * 1024) C /= 2;
+    o->chunk_tuples = C;
+    o->chunk_region = C + Qm;  // worst-case padding: one slot per run
     const uint64_t rmax = std::max(o->recv_cap[0], o->recv_cap[1]);
-    o->max_chunks = rmax / o->chunk_tuples + o->P + 2;
-    const uint64_t Qm = 1ull << o->b2_max;
-    o->max_items = (uint64_t)o->P * Qm + o->recv_cap[1] / PROBE_S_TARGET * 4 + o->recv_cap[0] / PROBE_CAP * 4 + 4096;
-    if (o->max_items > 0xffffffffull) o->max_items = 0xffffffffull;
+    o->max_chunks = rmax / C + o->P + 2;
+    o->max_items = (uint64_t)o->P * Qm + o->recv_cap[1] / (o->probe_slots / 2) * 2 +
+                   o->recv_cap[0] / (o->probe_slots / 2) * 2 + 4096;
+    if (o->max_items > 0x7fffffffull) o->max_items = 0x7fffffffull;
     o->out_cap = c.out_capacity ? c.out_capacity : (c.materialize ? std::max(o->recv_cap[0], o->recv_cap[1]) : 0);
     Arena &L = o->lay;
     uint64_t off = 0;
@@ -102,9 +105,10 @@ struct mgj_plan_s {
     char *arena[MAX_RANKS] = {};
     void *zero_block = nullptr;
     size_t zero_bytes = 0;
-    void *allocs[24] = {};
+    void *allocs[32] = {};
     int nalloc = 0;
     Ctx ctx{};
+    ChunkDesc *cdesc = nullptr;
     uint64_t epoch = 0;
     int state = 0;
     cudaStream_t stream = nullptr;
@@ -139,27 +143,20 @@ void *dalloc(mgj_plan_s *h, size_t bytes, mgj_status *st) {
 
 size_t hist_smem(const Norm &n) { return (size_t)n.P * 4; }
 size_t plan_smem(const Norm &n) { return (size_t)n.P * 5 * 8 + (size_t)n.P * 4 + (size_t)(n.P + 1) * 4; }
-size_t scatter_smem(const Norm &n) {
-    return (size_t)n.P * n.line_tuples * n.tuple_bytes + (size_t)n.P * 4 + SCATTER_BATCH * 2;
-}
-size_t local_smem(const Norm &n) { return (size_t)n.chunk_tuples * n.tuple_bytes + ((size_t)1 << n.b2_max) * 4; }
-size_t probe_smem(const Norm &n) {
-    return (size_t)PROBE_CAP * n.tuple_bytes + (size_t)PROBE_CAP * 4 * 2 + (size_t)PROBE_WIN * 4 * 2;
-}
+size_t scatter_smem(const Norm &n) { return scat_smem_bytes(n.P, n.c.key_bytes); }
+size_t local_smem(const Norm &n) { return local_smem_bytes(n.chunk_tuples, 1 << n.b2_max, n.tuple_bytes); }
+size_t probe_smem(const Norm &n) { return probe_smem_bytes(n.probe_slots, n.tuple_bytes); }
 
 template <typename K>
 cudaError_t set_attrs(const Norm &n) {
     cudaError_t e;
-    if ((e = cudaFuncSetAttribute(k_hist<K>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)hist_smem(n)))) return e;
-    if ((e = cudaFuncSetAttribute(k_plan, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)plan_smem(n)))) return e;
-    if ((e = cudaFuncSetAttribute(k_scatter<K>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)scatter_smem(n))))
-        return e;
-    if ((e = cudaFuncSetAttribute(k_local<K>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)local_smem(n))))
-        return e;
-    if ((e = cudaFuncSetAttribute(k_probe<K, false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                  (int)probe_smem(n))))
-        return e;
-    return cudaFuncSetAttribute(k_probe<K, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)probe_smem(n));
+    const auto A = cudaFuncAttributeMaxDynamicSharedMemorySize;
+    if ((e = cudaFuncSetAttribute(k_hist<K>, A, (int)hist_smem(n)))) return e;
+    if ((e = cudaFuncSetAttribute(k_plan, A, (int)plan_smem(n)))) return e;
+    if ((e = cudaFuncSetAttribute(k_scatter<K>, A, (int)scatter_smem(n)))) return e;
+    if ((e = cudaFuncSetAttribute(k_local<K>, A, (int)local_smem(n)))) return e;
+    if ((e = cudaFuncSetAttribute(k_probe<K, false>, A, (int)probe_smem(n)))) return e;
+    return cudaFuncSetAttribute(k_probe<K, true>, A, (int)probe_smem(n));
 }
 
 bool is_device_ptr(const void *p) {
@@ -174,29 +171,31 @@ bool is_device_ptr(const void *p) {
 template <typename K>
 void launch_partition(mgj_plan_s *h, cudaStream_t s) {
     const Norm &n = h->n;
-    dim3 g(h->nsm * 4, 2);
-    k_hist<K><<<g, 512, hist_smem(n), s>>>(h->ctx);
+    dim3 g(h->ctx.G, 2);
+    k_hist<K><<<g, HIST_THREADS, hist_smem(n), s>>>(h->ctx);
 }
 
 template <typename K>
 void launch_shuffle(mgj_plan_s *h, cudaStream_t s) {
     const Norm &n = h->n;
+    k_tilescan<<<(2 * n.P + 127) / 128, 128, 0, s>>>(h->ctx);
     k_plan<<<1, 1024, plan_smem(n), s>>>(h->ctx);
+    k_chunkmap<<<h->nsm * 2, 256, 0, s>>>(h->ctx, h->cdesc);
     cudaEventRecord(h->ev[2], s);
-    k_scatter<K><<<h->nsm, SCATTER_THREADS, scatter_smem(n), s>>>(h->ctx);
+    k_scatter<K><<<h->ctx.G, SCATTER_THREADS, scatter_smem(n), s>>>(h->ctx);
 }
 
 template <typename K>
 void launch_join(mgj_plan_s *h, cudaStream_t s) {
     const Norm &n = h->n;
     k_wait<<<1, 32, 0, s>>>(h->ctx, SIG_DATA);
-    k_local<K><<<h->nsm * 3, LOCAL_THREADS, local_smem(n), s>>>(h->ctx);
+    k_local<K><<<h->nsm, LOCAL_THREADS, local_smem(n), s>>>(h->ctx, h->cdesc);
     cudaEventRecord(h->ev[4], s);
-    k_itemize<<<h->nsm * 4, 256, 0, s>>>(h->ctx);
+    k_itemize<K><<<h->nsm * 4, 256, 0, s>>>(h->ctx);
     if (n.c.materialize)
-        k_probe<K, true><<<h->nsm * 3, PROBE_THREADS, probe_smem(n), s>>>(h->ctx);
+        k_probe<K, true><<<h->nsm, PROBE_THREADS, probe_smem(n), s>>>(h->ctx);
     else
-        k_probe<K, false><<<h->nsm * 3, PROBE_THREADS, probe_smem(n), s>>>(h->ctx);
+        k_probe<K, false><<<h->nsm, PROBE_THREADS, probe_smem(n), s>>>(h->ctx);
     cudaEventRecord(h->ev[5], s);
     k_publish<<<1, 32, 0, s>>>(h->ctx);
 }
@@ -257,11 +256,10 @@ mgj_status mgj_plan(const mgj_config *cfg, const mgj_peers *peers, mgj_handle *o
     }
     const int P = n.P;
     const uint64_t Qm = 1ull << n.b2_max;
-    // per-run zero block: rank_hist, ticket, gcur, meta, acc, err, cop_count
+    // per-run zero block: rank_hist, ticket, meta, acc, err, cop_slots
     size_t zo = 0;
     const size_t z_hist = zo; zo += align_up(2ull * P * 4, 256);
     const size_t z_tick = zo; zo += 256;
-    const size_t z_gcur = zo; zo += align_up(2ull * P * 4, 256);
     const size_t z_meta = zo; zo += 256;
     const size_t z_acc = zo; zo += 256;
     const size_t z_err = zo; zo += 256;
@@ -276,8 +274,10 @@ mgj_status mgj_plan(const mgj_config *cfg, const mgj_peers *peers, mgj_handle *o
     c.P = P;
     c.b2_cfg = n.c.radix_bits_local;
     c.b2_max = n.b2_max;
-    c.line_tuples = n.line_tuples;
+    c.G = h->nsm;
     c.chunk_tuples = n.chunk_tuples;
+    c.chunk_region = n.chunk_region;
+    c.probe_slots = n.probe_slots;
     c.materialize = n.c.materialize;
     c.max_items = (uint32_t)n.max_items;
     c.recv_cap[0] = n.recv_cap[0];
@@ -289,12 +289,14 @@ mgj_status mgj_plan(const mgj_config *cfg, const mgj_peers *peers, mgj_handle *o
     if (zb) {
         c.rank_hist = reinterpret_cast<uint32_t *>(zb + z_hist);
         c.ticket = reinterpret_cast<uint32_t *>(zb + z_tick);
-        c.gcur = reinterpret_cast<uint32_t *>(zb + z_gcur);
         c.meta = reinterpret_cast<int32_t *>(zb + z_meta);
         c.acc = reinterpret_cast<unsigned long long *>(zb + z_acc);
         c.err = reinterpret_cast<int32_t *>(zb + z_err);
-        c.cop_count = reinterpret_cast<uint32_t *>(zb + z_cop);
+        c.cop_slots = reinterpret_cast<uint32_t *>(zb + z_cop);
     }
+    c.tile_hist = static_cast<uint32_t *>(dalloc(h, 2ull * c.G * P * 4, &st));
+    c.tile_base = static_cast<uint32_t *>(dalloc(h, 2ull * c.G * P * 4, &st));
+    h->cdesc = static_cast<ChunkDesc *>(dalloc(h, 2 * n.max_chunks * sizeof(ChunkDesc), &st));
     c.owner = static_cast<int32_t *>(dalloc(h, P * 4, &st));
     c.send_off = static_cast<uint64_t *>(dalloc(h, 2ull * P * 8, &st));
     c.seg_start = static_cast<uint64_t *>(dalloc(h, 2ull * P * 8, &st));
@@ -302,10 +304,9 @@ mgj_status mgj_plan(const mgj_config *cfg, const mgj_peers *peers, mgj_handle *o
     c.recv_size = static_cast<uint64_t *>(dalloc(h, 2ull * MAX_RANKS * 8, &st));
     c.chunk_base = static_cast<uint32_t *>(dalloc(h, 2ull * (P + 1) * 4, &st));
     for (int r = 0; r < 2; ++r)
-        c.chunk_off[r] = static_cast<uint16_t *>(dalloc(h, n.max_chunks * (Qm + 1) * 2, &st));
-    c.items = static_cast<Item *>(dalloc(h, n.max_items * sizeof(Item), &st));
-    c.local[0] = dalloc(h, n.recv_cap[0] * n.tuple_bytes, &st);
-    c.local[1] = dalloc(h, n.recv_cap[1] * n.tuple_bytes, &st);
+        c.eoff[r] = static_cast<uint16_t *>(dalloc(h, n.max_chunks * (Qm + 1) * 2, &st));
+    c.items = static_cast<Item *>(dalloc(h, n.max_items * sizeof(ItemX), &st));
+    for (int r = 0; r < 2; ++r) c.local[r] = dalloc(h, n.max_chunks * n.chunk_region * n.tuple_bytes, &st);
     c.result = static_cast<unsigned long long *>(dalloc(h, 64, &st));
     if (n.c.materialize) {
         c.out_key = dalloc(h, n.out_cap * n.c.key_bytes, &st);
@@ -567,11 +568,17 @@ mgj_status mgj_debug_copy(mgj_handle h, int32_t what, void *dst, uint64_t bytes,
             src = h->arena[c.rank] + n.lay.recv[1];
             size = rs[MAX_RANKS + c.rank] * n.tuple_bytes;
             break;
-        case MGJ_DBG_LOCAL_R: src = c.local[0]; size = rs[c.rank] * n.tuple_bytes; break;
-        case MGJ_DBG_LOCAL_S: src = c.local[1]; size = rs[MAX_RANKS + c.rank] * n.tuple_bytes; break;
+        case MGJ_DBG_LOCAL_R:
+            src = c.local[0];
+            size = (uint64_t)(uint32_t)meta[MT_NCH_R] * n.chunk_region * n.tuple_bytes;
+            break;
+        case MGJ_DBG_LOCAL_S:
+            src = c.local[1];
+            size = (uint64_t)(uint32_t)meta[MT_NCH_S] * n.chunk_region * n.tuple_bytes;
+            break;
         case MGJ_DBG_META: src = c.meta; size = sizeof(meta); break;
-        case MGJ_DBG_CHUNK_OFF_R: src = c.chunk_off[0]; size = (uint64_t)(uint32_t)meta[MT_NCH_R] * (Q + 1) * 2; break;
-        case MGJ_DBG_CHUNK_OFF_S: src = c.chunk_off[1]; size = (uint64_t)(uint32_t)meta[MT_NCH_S] * (Q + 1) * 2; break;
+        case MGJ_DBG_CHUNK_OFF_R: src = c.eoff[0]; size = (uint64_t)(uint32_t)meta[MT_NCH_R] * (Q + 1) * 2; break;
+        case MGJ_DBG_CHUNK_OFF_S: src = c.eoff[1]; size = (uint64_t)(uint32_t)meta[MT_NCH_S] * (Q + 1) * 2; break;
         case MGJ_DBG_CHUNK_BASE: src = c.chunk_base; size = 2ull * (P + 1) * 4; break;
         case MGJ_DBG_OUT_KEY:
         case MGJ_DBG_OUT_PAY_R:

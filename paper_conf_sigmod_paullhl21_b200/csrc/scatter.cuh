@@ -3,196 +3,188 @@
 #pragma once
 
 #include "common.cuh"
+#include "tma.cuh"
 
 namespace mgj {
 
+template <typename K> struct ScatCfg {
+    using Tup = typename TupT<K>::T;
+    static constexpr int TMAX = SCAT_T8 * 4 / (int)sizeof(K);     // 8192 (4-byte) / 4096 (8-byte) tuples
+    static constexpr int VMAX = TMAX / SCATTER_THREADS;           // tuples per thread per sub-tile
+};
+
+// Sub-tile size for P partitions: keeps stages + sorted buffer + per-partition
+// arrays inside 227 KB of shared memory.
+__host__ __device__ inline int scat_subtile(int P, int key_bytes) {
+    const int tmax = SCAT_T8 * 4 / key_bytes;
+    return P <= 1024 ? tmax : tmax / 2;
+}
+
+__host__ __device__ inline size_t scat_smem_bytes(int P, int key_bytes) {
+    const size_t T = (size_t)scat_subtile(P, key_bytes);
+    return 2 * 2 * T * key_bytes     // two input stages, keys + payloads
+           + T * 2 * key_bytes       // partition-sorted sub-tile
+           + (size_t)P * 4           // bins
+           + (size_t)P * 8 * 2;      // wbase, base
+}
+
 // ---------------------------------------------------------------------------
-// a3 (§3.2 "Global partitioning phase" step 1, after Rui
-// et al. [38]; step 3 data distribution, P:405-407 and §4).  On NVSwitch every
-// pair of GPUs is one hop, so the paper's packets, routing buffers and
-// adaptive multi-hop routing (§4) reduce to this: each CTA stages tuples in
-// a shared-memory write-combining line per global partition and, when a line
-// is full, reserves L slots in the owner's receive range with one atomic and
-// writes the line there (a peer store over NVLink when the owner is another
-// GPU).  The receive layout per relation is: owned p ascending, then source
-// rank ascending, exactly tiled by the plan's offsets.  Order inside a
-// (source rank, p) range is unspecified (reading C17).
+// a3 (§3.2 "Global partitioning phase" step 1, P:408-416 — "each
+// thread ... reads a unique input tuple, determines the index for the tuple
+// after partitioning based on the histogram and then writes the tuple" —
+// after Rui et al. [38]; step 3 data distribution, P:405-407 and §4).
 //
-// Persistent grid (1 CTA/SM, 1024 threads); input batches are claimed
-// dynamically; each thread holds SCATTER_V tuples loaded with 16-byte
-// streaming loads, prefetching the next batch while the current one is
-// placed.  The last CTA raises SIG_DATA at every peer after a system fence.
+// B200 form: one persistent CTA per SM processes tile c = blockIdx.x of R and
+// then of S, in sub-tiles of T tuples brought into shared memory by TMA bulk
+// copies (double-buffered, two sub-tiles ahead).  Each sub-tile is counting-
+// sorted by digit1 in shared memory (one SMEM atomic per tuple gives the rank
+// in its bin), then written out in sorted order so that each warp store
+// covers a few contiguous runs.  The destination of every tuple is exact:
+// owner(p)'s receive buffer at send_off[p] (a2) + tile_base[c][p] (a1 tile
+// prefix) + the running count of p in this tile, so no global atomics and no
+// buffer flushes are needed.  On NVSwitch the owner may be another GPU: the
+// same store goes over NVLink (a peer-mapped address); the paper's packets,
+// routing buffers and multi-hop routing (§4) have no role on a one-hop
+// fabric.  The last CTA raises SIG_DATA at every peer after a system fence.
 // ---------------------------------------------------------------------------
 template <typename K>
 __global__ void __launch_bounds__(SCATTER_THREADS, 1) k_scatter(Ctx c) {
     using Tup = typename TupT<K>::T;
-    constexpr int V = SCATTER_V;
-    constexpr int NW = SCATTER_THREADS / 32;
-    extern __shared__ __align__(16) unsigned char smem[];
-    const int P = c.P, L = c.line_tuples;
-    Tup *buf = reinterpret_cast<Tup *>(smem);
-    uint32_t *cnt = reinterpret_cast<uint32_t *>(buf + (size_t)P * L);
-    uint16_t *flist = reinterpret_cast<uint16_t *>(cnt + P);
-    __shared__ uint32_t s_nf[2], s_batch[2];
-    __shared__ int s_ok;
-    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    constexpr int VMAX = ScatCfg<K>::VMAX;
+    constexpr int TB = (int)sizeof(Tup);
+    extern __shared__ __align__(128) unsigned char smem[];
+    const int P = c.P;
+    const int T = scat_subtile(P, (int)sizeof(K));
+    const int V = T / SCATTER_THREADS;
+    K *const stage0 = reinterpret_cast<K *>(smem);  // [2][keys T | payloads T]
+    auto skey = [&](int s) { return stage0 + (size_t)s * 2 * T; };
+    auto spay = [&](int s) { return stage0 + (size_t)s * 2 * T + T; };
+    Tup *sorted = reinterpret_cast<Tup *>(stage0 + (size_t)4 * T);
+    uint32_t *bins = reinterpret_cast<uint32_t *>(sorted + T);
+    unsigned long long *wbase = reinterpret_cast<unsigned long long *>(bins + P);
+    unsigned long long *base = wbase + P;
+    __shared__ __align__(8) uint64_t bar[2];
+    __shared__ uint32_t tmp[33];
+    const int tid = threadIdx.x;
+    const int tile = blockIdx.x;
+    const int ok = *(volatile int32_t *)&c.meta[MT_OK];
+
+    uint64_t lo[2], hi[2];
+    uint32_t nsub[2];
+    for (int r = 0; r < 2; ++r) {
+        tile_range(c.n_in[r], c.G, tile, lo[r], hi[r]);
+        nsub[r] = ok ? (uint32_t)((hi[r] - lo[r] + T - 1) / T) : 0;
+    }
+    const uint32_t ntot = nsub[0] + nsub[1];
     if (tid == 0) {
-        s_ok = *(volatile int32_t *)&c.meta[MT_OK];
-        s_nf[0] = s_nf[1] = 0;
+        mbar_init(&bar[0], 1);
+        mbar_init(&bar[1], 1);
+        fence_mbar_init();
     }
     __syncthreads();
-    uint32_t gr = 0;  // global round counter (parity of the flush-list counter)
+    const uint64_t pol = policy_evict_first();
 
-    for (int rel = 0; rel < 2 && s_ok; ++rel) {
-        const uint64_t n = c.n_in[rel];
-        const K *keys = static_cast<const K *>(c.in_key[rel]);
-        const K *pays = static_cast<const K *>(c.in_pay[rel]);
-        const uint32_t nb = (uint32_t)((n + SCATTER_BATCH - 1) / SCATTER_BATCH);
-        const uint64_t *soff = c.send_off + (size_t)rel * P;
-        uint32_t *gcur = c.gcur + (size_t)rel * P;
-        const uint64_t recv_off = c.lay.recv[rel];
-        for (int i = tid; i < P; i += SCATTER_THREADS) cnt[i] = 0;
+    // sub-tile g of the R-then-S sequence -> (rel, first tuple, length)
+    auto subtile = [&](uint32_t g, int &rel, uint64_t &first, uint32_t &len) {
+        rel = g < nsub[0] ? 0 : 1;
+        const uint32_t j = rel ? g - nsub[0] : g;
+        first = lo[rel] + (uint64_t)j * T;
+        len = (uint32_t)min((uint64_t)T, hi[rel] - first);
+    };
+    auto issue = [&](uint32_t g) {  // thread 0: TMA the 16-byte-aligned body of sub-tile g
+        int rel;
+        uint64_t first;
+        uint32_t len;
+        subtile(g, rel, first, len);
+        const uint32_t body = len & ~(uint32_t)(16 / sizeof(K) - 1);
+        const uint32_t bytes = body * (uint32_t)sizeof(K);
+        uint64_t *b = &bar[g & 1];
+        mbar_arrive_expect_tx(b, 2 * bytes);
+        if (bytes) {
+            tma_load_1d(skey(g & 1), static_cast<const K *>(c.in_key[rel]) + first, bytes, b, pol);
+            tma_load_1d(spay(g & 1), static_cast<const K *>(c.in_pay[rel]) + first, bytes, b, pol);
+        }
+    };
+    auto set_base = [&](int rel) {  // destination of this tile's first tuple of each partition
+        const uint32_t *tb = c.tile_base + ((size_t)rel * c.G + tile) * P;
+        const uint64_t *so = c.send_off + (size_t)rel * P;
+        for (int p = tid; p < P; p += SCATTER_THREADS) {
+            const int own = c.owner[p];
+            base[p] = (unsigned long long)(c.arena[own] + c.lay.recv[rel]) + (so[p] + tb[p]) * (uint64_t)TB;
+        }
+    };
 
-        auto load = [&](uint32_t b, K (&kk)[V], K (&pp)[V]) {
-            const uint64_t base = (uint64_t)b * SCATTER_BATCH + (uint64_t)tid * V;
-            if (b < nb && base + V <= n) {
-                if (sizeof(K) == 4) {
-                    uint4 a = __ldcs(reinterpret_cast<const uint4 *>(keys + base));
-                    uint4 d = __ldcs(reinterpret_cast<const uint4 *>(pays + base));
-                    kk[0] = (K)a.x; kk[1] = (K)a.y; kk[2] = (K)a.z; kk[3] = (K)a.w;
-                    pp[0] = (K)d.x; pp[1] = (K)d.y; pp[2] = (K)d.z; pp[3] = (K)d.w;
-                } else {
-#pragma unroll
-                    for (int h = 0; h < V / 2; ++h) {
-                        ulonglong2 a = __ldcs(reinterpret_cast<const ulonglong2 *>(keys + base) + h);
-                        ulonglong2 d = __ldcs(reinterpret_cast<const ulonglong2 *>(pays + base) + h);
-                        kk[2 * h] = (K)a.x; kk[2 * h + 1] = (K)a.y;
-                        pp[2 * h] = (K)d.x; pp[2 * h + 1] = (K)d.y;
-                    }
-                }
-            } else {
-#pragma unroll
-                for (int v = 0; v < V; ++v) {
-                    const bool ok = b < nb && base + v < n;
-                    kk[v] = ok ? keys[base + v] : (K)0;
-                    pp[v] = ok ? pays[base + v] : (K)0;
-                }
-            }
-        };
-
-        // Write the nf full lines listed in flist: one reservation atomic per line.
-        auto flush_lines = [&](uint32_t nf, uint32_t round) {
-            const int epw = 32 / L, sub = lane / L, li = lane % L;
-            for (uint32_t e0 = (uint32_t)warp * 32; e0 < nf; e0 += NW * 32) {
-                const uint32_t e = e0 + lane;
-                uint32_t p = 0, own = 0;
-                uint64_t off = 0;
-                if (e < nf) {
-                    p = flist[e];
-                    off = soff[p] + atomicAdd(&gcur[p], (uint32_t)L);
-                    own = (uint32_t)c.owner[p];
-                }
-                const uint32_t ne = min(32u, nf - e0);
-                for (uint32_t j = 0; j < ne; j += epw) {
-                    const uint32_t sl = j + sub;
-                    const uint32_t pj = __shfl_sync(0xffffffffu, p, sl & 31);
-                    const uint64_t oj = __shfl_sync(0xffffffffu, off, sl & 31);
-                    const uint32_t ow = __shfl_sync(0xffffffffu, own, sl & 31);
-                    if (sl < ne) {
-                        Tup *dst = reinterpret_cast<Tup *>(c.arena[ow] + recv_off) + oj + li;
-                        *dst = buf[(size_t)pj * L + li];
-                    }
-                }
-            }
-        };
-
-        uint32_t it = 0;
-        if (tid == 0) s_batch[0] = atomicAdd(&c.ticket[TK_SCAT_R + rel], 1u);
-        __syncthreads();
-        uint32_t b = s_batch[0];
-        K kk[V], pp[V];
-        load(b, kk, pp);
-        while (b < nb) {
-            ++it;
-            if (tid == 0) s_batch[it & 1] = atomicAdd(&c.ticket[TK_SCAT_R + rel], 1u);
+    if (tid == 0) {
+        if (ntot > 0) issue(0);
+        if (ntot > 1) issue(1);
+    }
+    int cur_rel = -1;
+    for (uint32_t g = 0; g < ntot; ++g) {
+        int rel;
+        uint64_t first;
+        uint32_t len;
+        subtile(g, rel, first, len);
+        if (rel != cur_rel) {  // (previous sub-tile's write-out is ordered by the barriers below)
             __syncthreads();
-            const uint32_t bn = s_batch[it & 1];
-            K kn[V], pn[V];
-            load(bn, kn, pn);  // prefetch the next batch while this one is placed
-
-            const uint64_t base = (uint64_t)b * SCATTER_BATCH + (uint64_t)tid * V;
-            uint32_t pd[V], pos[V];
-#pragma unroll
-            for (int v = 0; v < V; ++v) {
-                if (base + v < n) {
-                    pd[v] = digit1(kk[v], P);
-                    pos[v] = atomicAdd(&cnt[pd[v]], 1u);
-                } else {
-                    pd[v] = 0;
-                    pos[v] = 0xffffffffu;
-                }
-            }
-            for (uint32_t r = 0;; ++r, ++gr) {
-                const uint32_t lo = r * (uint32_t)L, hi = lo + (uint32_t)L;
-                int more = 0;
-#pragma unroll
-                for (int v = 0; v < V; ++v) {
-                    if (pos[v] >= lo && pos[v] < hi) {
-                        Tup t;
-                        t.x = kk[v];
-                        t.y = pp[v];
-                        buf[(size_t)pd[v] * L + (pos[v] - lo)] = t;
-                        if (pos[v] == hi - 1) flist[atomicAdd(&s_nf[gr & 1], 1u)] = (uint16_t)pd[v];
-                    } else if (pos[v] != 0xffffffffu && pos[v] >= hi) {
-                        more = 1;
-                    }
-                }
-                __syncthreads();
-                const uint32_t nf = s_nf[gr & 1];
-                if (tid == 0) s_nf[(gr + 1) & 1] = 0;
-                flush_lines(nf, r);
-                more = __syncthreads_or(more);
-                if (!more) break;
-            }
-            ++gr;
-            for (int i = tid; i < P; i += SCATTER_THREADS) cnt[i] &= (uint32_t)(L - 1);
-#pragma unroll
-            for (int v = 0; v < V; ++v) {
-                kk[v] = kn[v];
-                pp[v] = pn[v];
-            }
-            b = bn;
+            set_base(rel);
+            cur_rel = rel;
         }
-        __syncthreads();
-        // drain partially filled lines
-        for (int p0 = warp * 32; p0 < P; p0 += NW * 32) {
-            const int p = p0 + lane;
-            const uint32_t m = p < P ? cnt[p] : 0;
-            uint64_t off = 0;
-            uint32_t own = 0;
-            if (m) {
-                off = soff[p] + atomicAdd(&gcur[p], m);
-                own = (uint32_t)c.owner[p];
+        const int s = g & 1;
+        mbar_wait(&bar[s], (g >> 1) & 1);
+        const uint32_t body = len & ~(uint32_t)(16 / sizeof(K) - 1);
+        const K *gk = static_cast<const K *>(c.in_key[rel]) + first;
+        const K *gp = static_cast<const K *>(c.in_pay[rel]) + first;
+        K kk[VMAX], pp[VMAX];
+#pragma unroll
+        for (int v = 0; v < VMAX; ++v) {
+            const uint32_t i = tid + v * SCATTER_THREADS;
+            if (v < V && i < body) {
+                kk[v] = skey(s)[i];
+                pp[v] = spay(s)[i];
+            } else if (v < V && i < len) {  // < 4 trailing tuples of the relation
+                kk[v] = gk[i];
+                pp[v] = gp[i];
             }
-            uint32_t msk = __ballot_sync(0xffffffffu, m > 0);
-            while (msk) {
-                const int src = __ffs(msk) - 1;
-                msk &= msk - 1;
-                const uint32_t mm = __shfl_sync(0xffffffffu, m, src);
-                const uint64_t oo = __shfl_sync(0xffffffffu, off, src);
-                const uint32_t ow = __shfl_sync(0xffffffffu, own, src);
-                if ((uint32_t)lane < mm) {
-                    Tup *dst = reinterpret_cast<Tup *>(c.arena[ow] + recv_off) + oo + lane;
-                    *dst = buf[(size_t)(p0 + src) * L + lane];
-                }
+        }
+        for (int p = tid; p < P; p += SCATTER_THREADS) bins[p] = 0;
+        __syncthreads();  // stage s consumed, bins cleared
+        if (tid == 0 && g + 2 < ntot) issue(g + 2);
+        uint32_t rp[VMAX];  // rank in bin << 16 | partition
+#pragma unroll
+        for (int v = 0; v < VMAX; ++v) {
+            const uint32_t i = tid + v * SCATTER_THREADS;
+            if (v < V && i < len) {
+                const uint32_t p = digit1(kk[v], P);
+                rp[v] = (atomicAdd(&bins[p], 1u) << 16) | p;
             }
         }
         __syncthreads();
-        if (tid == 0) s_nf[gr & 1] = 0;
+        block_excl_scan_u32(bins, P, tmp);
+        for (int p = tid; p < P; p += SCATTER_THREADS) {
+            const uint32_t o = bins[p], e = (p + 1 < P) ? bins[p + 1] : len;
+            const unsigned long long b = base[p];
+            wbase[p] = b - (unsigned long long)o * TB;
+            base[p] = b + (unsigned long long)(e - o) * TB;
+        }
+#pragma unroll
+        for (int v = 0; v < VMAX; ++v) {
+            const uint32_t i = tid + v * SCATTER_THREADS;
+            if (v < V && i < len) {
+                Tup t;
+                t.x = kk[v];
+                t.y = pp[v];
+                sorted[bins[rp[v] & 0xffffu] + (rp[v] >> 16)] = t;
+            }
+        }
         __syncthreads();
+        for (uint32_t i = tid; i < len; i += SCATTER_THREADS) {
+            const Tup t = sorted[i];
+            Tup *dst = reinterpret_cast<Tup *>(wbase[digit1(t.x, P)] + (unsigned long long)i * TB);
+            *dst = t;
+        }
     }
 
-    // ---- every CTA: make its peer stores visible, the last one signals ----
+    // ---- every CTA: make its (peer) stores visible, the last one signals ----
     __threadfence_system();
     __syncthreads();
     if (tid == 0) {

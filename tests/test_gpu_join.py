@@ -87,12 +87,13 @@ def test_gen_matches_numpy(mgj, kind, n_r, n_s, z, row0, count):
 
 
 # ------------------------------------------------------------ per-phase state
-def test_phases_m1(mgj):
+@pytest.mark.parametrize("b1", [10, 4])
+def test_phases_m1(mgj, b1):
     """a1 histogram == np.bincount, a2 plan invariants, a3 received multiset,
     a4 sub-partition property, at M1 (2^20 x 2^20, one GPU)."""
     d = datagen.M1().rank_inputs()
     n = d["r_keys"].size
-    j, res = run_one(mgj, d)
+    j, res = run_one(mgj, d, radix_bits_global=b1)
     P = 1 << res["radix_bits_global"]
     B1 = res["radix_bits_global"]
     hist = j.debug("RANK_HIST", np.uint32).reshape(2, P)
@@ -113,25 +114,36 @@ def test_phases_m1(mgj):
         packed = recv[:, 0].astype(np.uint64) | (recv[:, 1].astype(np.uint64) << np.uint64(32))
         exp = kk.astype(np.uint64) | (pp.astype(np.uint64) << np.uint64(32))
         np.testing.assert_array_equal(np.sort(packed), np.sort(exp))
-        # a4: every chunk of every segment is ordered by digit2 and keeps its multiset
-        loc = j.debug("LOCAL_R" if rel == 0 else "LOCAL_S", np.uint32).reshape(-1, 2)
+        # a4: every chunk of every segment is split into q-runs (16-byte padded)
+        # whose tuples all have digit2 == q, and the chunk's multiset is kept
         B2 = res["radix_bits_local"]
         Q = 1 << B2
         C = 8192
         seg = j.debug("SEGMENTS", np.uint64).reshape(4, P)
         start, ln = seg[rel], seg[2 + rel]
-        coff = j.debug("CHUNK_OFF_R" if rel == 0 else "CHUNK_OFF_S", np.uint16).reshape(-1, Q + 1)
-        ci = 0
+        E = j.debug("CHUNK_OFF_R" if rel == 0 else "CHUNK_OFF_S", np.uint16).astype(np.int64)
+        nch_p = (ln.astype(np.int64) + C - 1) // C
+        loc = j.debug("LOCAL_R" if rel == 0 else "LOCAL_S", np.uint32).reshape(-1, 2)
+        CR = loc.shape[0] // int(nch_p.sum())
+        cb = np.concatenate([[0], np.cumsum(nch_p)])
         for p in range(P):
-            for k0 in range(0, int(ln[p]), C):
-                a, b = int(start[p]) + k0, int(start[p]) + min(int(ln[p]), k0 + C)
-                d2 = (loc[a:b, 0] >> B1) & (Q - 1)
-                assert np.all(np.diff(d2.astype(np.int64)) >= 0)
-                np.testing.assert_array_equal(coff[ci], np.searchsorted(d2, np.arange(Q + 1)))
+            for k in range(int(nch_p[p])):
+                a = int(start[p]) + k * C
+                b = min(int(start[p]) + int(ln[p]), a + C)
+                li = cb[p] + k
+                row = lambda q: E[(Q + 1) * cb[p] + q * nch_p[p] + k]
+                got = []
+                for q in range(Q):
+                    e0, e1 = row(q), row(q + 1)
+                    st, slots = e0 & ~1, (e1 & ~1) - (e0 & ~1)
+                    valid = slots - (e0 & 1)
+                    run = loc[li * CR + st: li * CR + st + valid]
+                    assert np.all(((run[:, 0] >> B1) & (Q - 1)) == q)
+                    got.append(run)
+                got = np.concatenate(got)
                 src = recv[a:b, 0].astype(np.uint64) | (recv[a:b, 1].astype(np.uint64) << np.uint64(32))
-                dst = loc[a:b, 0].astype(np.uint64) | (loc[a:b, 1].astype(np.uint64) << np.uint64(32))
+                dst = got[:, 0].astype(np.uint64) | (got[:, 1].astype(np.uint64) << np.uint64(32))
                 np.testing.assert_array_equal(np.sort(src), np.sort(dst))
-                ci += 1
     j.close()
 
 

@@ -182,7 +182,19 @@ __global__ void __launch_bounds__(LOCAL_THREADS, 1) k_local(Ctx c, const ChunkDe
 #pragma unroll
         for (int v = 0; v < VMAX; ++v) {
             const uint32_t i = tid + v * LOCAL_THREADS;
-            if (v < V && i < len) sorted[abin[rq[v] & 0xffffu] + (rq[v] >> 16)] = t[v];
+            if (v < V && i < len) {
+                const uint32_t q = rq[v] & 0xffffu, r = rq[v] >> 16;
+                sorted[abin[q] + r] = t[v];
+                // 16-byte padding slot of an odd run: a tuple whose key has its
+                // lowest bit flipped, i.e. lies in another global partition, so
+                // it never equals a real key of this co-partition; the probe
+                // skips S padding slots (bitmap), R padding is inert
+                if (ALIGN == 2 && r == 0 && (bins[q] & 1u)) {
+                    Tup pad = t[v];
+                    pad.x ^= 1;
+                    sorted[abin[q] + bins[q]] = pad;
+                }
+            }
         }
         fence_proxy_async_smem();
         __syncthreads();  // S3
@@ -303,10 +315,10 @@ __global__ void k_itemize(Ctx c) {
 }
 
 __host__ __device__ inline size_t probe_smem_bytes(int slots, int TB) {
-    return (size_t)PROBE_NST * 2 * slots * TB        // stages (R, S)
-           + (size_t)PROBE_NST * 2 * PROBE_MAXP * 4  // piece descriptors
-           + 4096 * 4                                // head
-           + (size_t)slots * 2;                      // next
+    return (size_t)PROBE_NST * 2 * slots * TB  // stages (R, S)
+           + (size_t)PROBE_NST * (slots / 32 + 1) * 4  // S padding-slot bitmaps
+           + 4096 * 4                          // head
+           + (size_t)slots * 2;                // next
 }
 
 // ---------------------------------------------------------------------------
@@ -314,33 +326,36 @@ __host__ __device__ inline size_t probe_smem_bytes(int slots, int TB) {
 // the same partition id are joined; the paper notes the nested-loop and the
 // shared-memory hash-table variants perform alike and the north
 // star asks for the hash table.  Warp-specialised, PROBE_NST-stage pipeline:
-//  - warp 0 (producer) walks the run offsets of the next items and issues
-//    one TMA bulk copy per (chunk, relation) run into a free stage;
-//  - warps 1..31 (consumers) build a chained hash table over the stage's R
-//    runs (head entries tagged with the item, so the table is never
-//    cleared), then stream the S runs through it: count += 1 and
-//    checksum += a*C + b (mod 2^64) for every equal-key pair.  With MAT the
-//    item's matches are counted, one output reservation is taken, and a
-//    second pass over the S runs in shared memory writes (key, payR, payS).
+//  - warps 0..PROBE_NP-1 (producers, items round-robin) read the run offsets
+//    of their next item and issue one TMA bulk copy per (chunk, relation)
+//    run into a free stage, packing the runs back to back;
+//  - the other warps (consumers) build a chained hash table over the stage's
+//    R slots (head entries tagged with the item, so the table is never
+//    cleared), then stream the S slots through it: count += 1 and
+//    checksum += a*C + b (mod 2^64) for every equal-key pair.  Padding slots
+//    hold keys of another partition and never match.  With MAT the item's
+//    matches are counted, one output reservation is taken, and a second pass
+//    over the S slots in shared memory writes (key, payR, payS).
 // ---------------------------------------------------------------------------
 template <typename K, bool MAT>
 __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
     using Tup = typename Layout<K>::Tup;
-    constexpr int TB = Layout<K>::TB, ALIGN = Layout<K>::ALIGN;
+    constexpr int TB = Layout<K>::TB;
     constexpr int LOGT = 12, T = 1 << LOGT;
     constexpr uint16_t END = 0xffff;
-    constexpr int NCONS = PROBE_THREADS - 32;
+    constexpr int NCONS = PROBE_THREADS - 32 * PROBE_NP;
     extern __shared__ __align__(128) unsigned char smem[];
     __shared__ __align__(8) uint64_t full[PROBE_NST], empty[PROBE_NST];
-    __shared__ uint32_t npieces[PROBE_NST][2];
+    __shared__ uint32_t totals[PROBE_NST][2];
     __shared__ uint32_t s_m;
     __shared__ unsigned long long s_base;
     __shared__ int s_write;
     if (!c.meta[MT_OK]) return;
     const int SL = c.probe_slots;
     Tup *stages = reinterpret_cast<Tup *>(smem);  // [NST][2][SL]
-    uint32_t *desc = reinterpret_cast<uint32_t *>(stages + (size_t)PROBE_NST * 2 * SL);  // [NST][2][MAXP]
-    uint32_t *head = desc + PROBE_NST * 2 * PROBE_MAXP;
+    const int PW = SL / 32 + 1;  // words per S padding bitmap
+    uint32_t *padbits = reinterpret_cast<uint32_t *>(stages + (size_t)PROBE_NST * 2 * SL);  // [NST][PW]
+    uint32_t *head = padbits + PROBE_NST * PW;
     uint16_t *nxt = reinterpret_cast<uint16_t *>(head + T);
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const int B2 = c.meta[MT_B2];
@@ -358,13 +373,22 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
     for (int i = tid; i < T; i += PROBE_THREADS) head[i] = 0;
     __syncthreads();
 
-    if (warp == 0) {
-        // ------------------------------------------------------- producer
+    if (warp < PROBE_NP) {
+        // ------------------------------------------------------- producers
+        constexpr int ALIGN = Layout<K>::ALIGN;
         const uint64_t pol = policy_evict_first();
-        for (uint32_t j = 0; j < mine; ++j) {
+        ItemX x;
+        if (warp < (int)mine) x = items[blockIdx.x + warp * gridDim.x];
+        for (uint32_t j = warp; j < mine; j += PROBE_NP) {
+            ItemX xn;
+            if (j + PROBE_NP < mine) xn = items[blockIdx.x + (j + PROBE_NP) * gridDim.x];  // prefetch
             const int s = j % PROBE_NST;
             if (j >= PROBE_NST) mbar_wait(&empty[s], ((j / PROBE_NST) - 1) & 1);
-            const ItemX x = items[blockIdx.x + j * gridDim.x];
+            uint32_t *pb = padbits + s * PW;
+            if (ALIGN == 2) {
+                for (int w = lane; w < PW; w += 32) pb[w] = 0;
+                __syncwarp();
+            }
             for (int rel = 0; rel < 2; ++rel) {
                 const Side sd = rel ? x.it.s : x.it.r;
                 const uint16_t *E0 = c.eoff[rel] + (size_t)(Q + 1) * x.cb[rel] + (size_t)x.it.q * x.nch[rel];
@@ -372,12 +396,11 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
                 const uint32_t kend = min(sd.k1, x.nch[rel] - 1);
                 const uint32_t np = sd.k0 <= kend ? kend - sd.k0 + 1 : 0;
                 Tup *dstbase = stages + ((size_t)s * 2 + rel) * SL;
-                uint32_t *dsc = desc + ((size_t)s * 2 + rel) * PROBE_MAXP;
                 const Tup *lbase = static_cast<const Tup *>(c.local[rel]);
                 uint32_t run = 0;
                 for (uint32_t m0 = 0; m0 < np; m0 += 32) {
                     const uint32_t m = m0 + lane;
-                    uint32_t sz = 0, valid = 0;
+                    uint32_t sz = 0, pad = 0xffffffffu;
                     uint64_t src = 0;
                     if (m < np) {
                         const uint32_t k = sd.k0 + m;
@@ -387,9 +410,9 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
                         const uint32_t ahi = (k == sd.k1) ? sd.a1 : slots;
                         if (ahi > alo) {
                             sz = ahi - alo;
-                            valid = min(ahi, v) > alo ? min(ahi, v) - alo : 0;
                             src = (uint64_t)(x.cb[rel] + k) * c.chunk_region + st + alo;
                         }
+                        pad = (ALIGN == 2 && rel == 1 && v < slots && v >= alo && v < ahi) ? v - alo : 0xffffffffu;
                     }
                     uint32_t incl = sz;
 #pragma unroll
@@ -399,7 +422,6 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
                     }
                     const uint32_t dst = run + incl - sz;
                     const uint32_t gsum = __shfl_sync(0xffffffffu, incl, 31);
-                    if (m < np) dsc[m] = dst | (valid << 16);
                     if (lane == 0 && gsum)
                         asm volatile("mbarrier.expect_tx.relaxed.cta.shared::cta.b64 [%0], %1;" ::"r"(
                                          smem_u32(&full[s])),
@@ -407,70 +429,65 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
                                      : "memory");
                     __syncwarp();
                     if (sz) tma_load_1d(dstbase + dst, lbase + src, sz * TB, &full[s], pol);
+                    if (pad != 0xffffffffu) atomicOr(&pb[(dst + pad) >> 5], 1u << ((dst + pad) & 31));
                     run += gsum;
                 }
-                if (lane == 0) npieces[s][rel] = np;
+                if (lane == 0) totals[s][rel] = run;
             }
             __syncwarp();
             if (lane == 0) mbar_arrive(&full[s]);
+            x = xn;
         }
         return;
     }
 
     // ------------------------------------------------------------ consumers
-    const int cw = warp - 1, ncw = PROBE_THREADS / 32 - 1;
+    const int ct = tid - 32 * PROBE_NP;
     unsigned long long my_cnt = 0, my_chk = 0;
     uint32_t tag = 0;
     for (uint32_t j = 0; j < mine; ++j) {
         const int s = j % PROBE_NST;
         if (++tag == 0x10000u) {  // tag wrap: clear the table once every 65535 items
-            for (int i = tid - 32; i < T; i += NCONS) head[i] = 0;
+            for (int i = ct; i < T; i += NCONS) head[i] = 0;
             named_bar_sync(1, NCONS);
             tag = 1;
         }
         mbar_wait(&full[s], (j / PROBE_NST) & 1);
         const Tup *rt = stages + ((size_t)s * 2 + 0) * SL;
         const Tup *st = stages + ((size_t)s * 2 + 1) * SL;
-        const uint32_t *dR = desc + ((size_t)s * 2 + 0) * PROBE_MAXP;
-        const uint32_t *dS = desc + ((size_t)s * 2 + 1) * PROBE_MAXP;
-        const uint32_t npR = npieces[s][0], npS = npieces[s][1];
+        const uint32_t rtot = totals[s][0], stot = totals[s][1];
         // build
-        for (uint32_t m = cw; m < npR; m += ncw) {
-            const uint32_t d = dR[m], base = d & 0xffffu, v = d >> 16;
-            for (uint32_t x = lane; x < v; x += 32) {
-                const uint32_t slot = base + x;
-                const uint32_t h = tab_hash(rt[slot].x, shift, LOGT);
-                const uint32_t old = atomicExch(&head[h], (tag << 16) | slot);
-                nxt[slot] = (old >> 16) == tag ? (uint16_t)(old & 0xffffu) : END;
-            }
+        for (uint32_t slot = ct; slot < rtot; slot += NCONS) {
+            const uint32_t h = tab_hash(rt[slot].x, shift, LOGT);
+            const uint32_t old = atomicExch(&head[h], (tag << 16) | slot);
+            nxt[slot] = (old >> 16) == tag ? (uint16_t)(old & 0xffffu) : END;
         }
         named_bar_sync(1, NCONS);
         // probe
+        const uint32_t *pb = padbits + s * PW;
         uint32_t m_item = 0;
-        for (uint32_t m = cw; m < npS; m += ncw) {
-            const uint32_t d = dS[m], base = d & 0xffffu, v = d >> 16;
-            for (uint32_t x = lane; x < v; x += 32) {
-                const Tup sv = st[base + x];
-                const uint32_t hv = head[tab_hash(sv.x, shift, LOGT)];
-                uint32_t i = (hv >> 16) == tag ? (hv & 0xffffu) : END;
-                while (i != END) {
-                    const Tup rv = rt[i];
-                    if (rv.x == sv.x) {
-                        ++m_item;
-                        my_chk += chk_term(rv.y, sv.y);
-                    }
-                    i = nxt[i];
+        for (uint32_t x = ct; x < stot; x += NCONS) {
+            if (Layout<K>::ALIGN == 2 && ((pb[x >> 5] >> (x & 31)) & 1u)) continue;  // padding slot
+            const Tup sv = st[x];
+            const uint32_t hv = head[tab_hash(sv.x, shift, LOGT)];
+            uint32_t i = (hv >> 16) == tag ? (hv & 0xffffu) : END;
+            while (i != END) {
+                const Tup rv = rt[i];
+                if (rv.x == sv.x) {
+                    ++m_item;
+                    my_chk += chk_term(rv.y, sv.y);
                 }
+                i = nxt[i];
             }
         }
         my_cnt += m_item;
         if (MAT) {
-            if (tid == 32) s_m = 0;
+            if (ct == 0) s_m = 0;
             named_bar_sync(1, NCONS);
             const uint32_t wm = (uint32_t)warp_sum(m_item);
             if (lane == 0 && wm) atomicAdd(&s_m, wm);
             named_bar_sync(1, NCONS);
-            if (tid == 32) {
+            if (ct == 0) {
                 const uint32_t M = s_m;
                 s_base = M ? atomicAdd(&c.acc[2], (unsigned long long)M) : 0;
                 s_write = M && (s_base + M <= c.out_cap);
@@ -483,36 +500,33 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
                 K *oa = static_cast<K *>(c.out_a);
                 K *ob = static_cast<K *>(c.out_b);
                 const unsigned long long obase = s_base;
-                for (uint32_t m = cw; m < npS; m += ncw) {
-                    const uint32_t d = dS[m], base = d & 0xffffu, v = d >> 16;
-                    for (uint32_t x0 = 0; x0 < v; x0 += 32) {
-                        const uint32_t x = x0 + lane;
-                        Tup sv;
-                        uint32_t i = END;
-                        if (x < v) {
-                            sv = st[base + x];
-                            const uint32_t hv = head[tab_hash(sv.x, shift, LOGT)];
-                            i = (hv >> 16) == tag ? (hv & 0xffffu) : END;
+                const uint32_t sround = (stot + 31) & ~31u;
+                for (uint32_t x = ct; x < sround; x += NCONS) {  // warp-uniform trip count
+                    Tup sv;
+                    uint32_t i = END;
+                    if (x < stot && !(Layout<K>::ALIGN == 2 && ((pb[x >> 5] >> (x & 31)) & 1u))) {
+                        sv = st[x];
+                        const uint32_t hv = head[tab_hash(sv.x, shift, LOGT)];
+                        i = (hv >> 16) == tag ? (hv & 0xffffu) : END;
+                    }
+                    while (__any_sync(0xffffffffu, i != END)) {
+                        bool hit = false;
+                        Tup rv;
+                        if (i != END) {
+                            rv = rt[i];
+                            hit = rv.x == sv.x;
+                            i = nxt[i];
                         }
-                        while (__any_sync(0xffffffffu, i != END)) {
-                            bool hit = false;
-                            Tup rv;
-                            if (i != END) {
-                                rv = rt[i];
-                                hit = rv.x == sv.x;
-                                i = nxt[i];
-                            }
-                            const uint32_t bal = __ballot_sync(0xffffffffu, hit);
-                            if (bal) {
-                                uint32_t wb = 0;
-                                if (lane == 0) wb = atomicAdd(&s_m, (uint32_t)__popc(bal));
-                                wb = __shfl_sync(0xffffffffu, wb, 0);
-                                if (hit) {
-                                    const unsigned long long pos = obase + wb + __popc(bal & ((1u << lane) - 1u));
-                                    ok[pos] = (K)sv.x;
-                                    oa[pos] = (K)rv.y;
-                                    ob[pos] = (K)sv.y;
-                                }
+                        const uint32_t bal = __ballot_sync(0xffffffffu, hit);
+                        if (bal) {
+                            uint32_t wb = 0;
+                            if (lane == 0) wb = atomicAdd(&s_m, (uint32_t)__popc(bal));
+                            wb = __shfl_sync(0xffffffffu, wb, 0);
+                            if (hit) {
+                                const unsigned long long pos = obase + wb + __popc(bal & ((1u << lane) - 1u));
+                                ok[pos] = (K)sv.x;
+                                oa[pos] = (K)rv.y;
+                                ob[pos] = (K)sv.y;
                             }
                         }
                     }
@@ -520,7 +534,7 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
             }
         }
         named_bar_sync(1, NCONS);  // stage s and the table are free
-        if (tid == 32) mbar_arrive(&empty[s]);
+        if (ct == 0) mbar_arrive(&empty[s]);
     }
     my_cnt = warp_sum(my_cnt);
     my_chk = warp_sum(my_chk);

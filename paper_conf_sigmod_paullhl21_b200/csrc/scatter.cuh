@@ -9,23 +9,28 @@ namespace mgj {
 
 template <typename K> struct ScatCfg {
     using Tup = typename TupT<K>::T;
-    static constexpr int TMAX = SCAT_T8 * 4 / (int)sizeof(K);     // 8192 (4-byte) / 4096 (8-byte) tuples
-    static constexpr int VMAX = TMAX / SCATTER_THREADS;           // tuples per thread per sub-tile
+    static constexpr int TMAX = SCAT_T8 * 4 / (int)sizeof(K);  // 8192 (4-byte) / 4096 (8-byte) tuples
+    static constexpr int VMAX = TMAX / SCATTER_THREADS;        // tuples per thread per sub-tile
 };
 
-// Sub-tile size for P partitions: keeps stages + sorted buffer + per-partition
-// arrays inside 227 KB of shared memory.
+// Sub-tile size and per-partition carry capacity for P partitions (shared
+// memory stays within 227 KB).  The carry holds the < 32-byte tail of each
+// partition's output so that global stores cover whole 32-byte sectors.
 __host__ __device__ inline int scat_subtile(int P, int key_bytes) {
     const int tmax = SCAT_T8 * 4 / key_bytes;
     return P <= 1024 ? tmax : tmax / 2;
 }
+__host__ __device__ inline int scat_carry(int P, int tuple_bytes) { return P <= 2048 ? 32 / tuple_bytes - 1 : 0; }
 
 __host__ __device__ inline size_t scat_smem_bytes(int P, int key_bytes) {
     const size_t T = (size_t)scat_subtile(P, key_bytes);
-    return 2 * 2 * T * key_bytes     // two input stages, keys + payloads
-           + T * 2 * key_bytes       // partition-sorted sub-tile
-           + (size_t)P * 4           // bins
-           + (size_t)P * 8 * 2;      // wbase, base
+    const size_t TB = 2 * (size_t)key_bytes;
+    const size_t CC = (size_t)scat_carry(P, (int)TB);
+    return 2 * T * key_bytes      // input stage: keys + payloads
+           + (T + CC * P) * TB    // partition-sorted sub-tile (+ carried tails)
+           + (size_t)P * 4 * 4    // bins, pos, lim, ccount
+           + (size_t)P * 8 * 2    // wb, base
+           + (size_t)P * CC * TB; // carry
 }
 
 // ---------------------------------------------------------------------------
@@ -35,35 +40,43 @@ __host__ __device__ inline size_t scat_smem_bytes(int P, int key_bytes) {
 // after Rui et al. [38]; step 3 data distribution, P:405-407 and §4).
 //
 // B200 form: one persistent CTA per SM processes tile c = blockIdx.x of R and
-// then of S, in sub-tiles of T tuples brought into shared memory by TMA bulk
-// copies (double-buffered, two sub-tiles ahead).  Each sub-tile is counting-
-// sorted by digit1 in shared memory (one SMEM atomic per tuple gives the rank
-// in its bin), then written out in sorted order so that each warp store
-// covers a few contiguous runs.  The destination of every tuple is exact:
-// owner(p)'s receive buffer at send_off[p] (a2) + tile_base[c][p] (a1 tile
-// prefix) + the running count of p in this tile, so no global atomics and no
-// buffer flushes are needed.  On NVSwitch the owner may be another GPU: the
-// same store goes over NVLink (a peer-mapped address); the paper's packets,
-// routing buffers and multi-hop routing (§4) have no role on a one-hop
-// fabric.  The last CTA raises SIG_DATA at every peer after a system fence.
+// then of S, in sub-tiles of T tuples brought into shared memory by a TMA
+// bulk copy issued one sub-tile ahead.  Each sub-tile is counting-sorted by
+// digit1 in shared memory (one SMEM atomic per tuple gives the rank in its
+// bin) and written out in sorted order, so each warp store covers a few
+// contiguous runs.  Destinations are exact: owner(p)'s receive buffer at
+// send_off[p] (a2) + tile_base[c][p] (a1 tile prefix) + the running count of
+// p in this tile — no global atomics.  Every partition keeps its < 32-byte
+// tail in shared memory until the next sub-tile completes the sector, so
+// (except at tile boundaries) every store covers whole 32-byte sectors and
+// DRAM never sees a partial-sector read-modify-write.  On NVSwitch the owner
+// may be another GPU: the same store goes over NVLink to a peer-mapped
+// address; the paper's packets, routing buffers and multi-hop routing (§4)
+// have no role on a one-hop fabric.  The last CTA raises SIG_DATA at every
+// peer after a system fence.
 // ---------------------------------------------------------------------------
 template <typename K>
 __global__ void __launch_bounds__(SCATTER_THREADS, 1) k_scatter(Ctx c) {
     using Tup = typename TupT<K>::T;
     constexpr int VMAX = ScatCfg<K>::VMAX;
     constexpr int TB = (int)sizeof(Tup);
+    typedef unsigned long long ull;
     extern __shared__ __align__(128) unsigned char smem[];
     const int P = c.P;
     const int T = scat_subtile(P, (int)sizeof(K));
     const int V = T / SCATTER_THREADS;
-    K *const stage0 = reinterpret_cast<K *>(smem);  // [2][keys T | payloads T]
-    auto skey = [&](int s) { return stage0 + (size_t)s * 2 * T; };
-    auto spay = [&](int s) { return stage0 + (size_t)s * 2 * T + T; };
-    Tup *sorted = reinterpret_cast<Tup *>(stage0 + (size_t)4 * T);
-    uint32_t *bins = reinterpret_cast<uint32_t *>(sorted + T);
-    unsigned long long *wbase = reinterpret_cast<unsigned long long *>(bins + P);
-    unsigned long long *base = wbase + P;
-    __shared__ __align__(8) uint64_t bar[2];
+    const int CC = scat_carry(P, TB);
+    K *const skey = reinterpret_cast<K *>(smem);
+    K *const spay = skey + T;
+    Tup *const sorted = reinterpret_cast<Tup *>(spay + T);
+    uint32_t *const bins = reinterpret_cast<uint32_t *>(sorted + T + (size_t)CC * P);
+    uint32_t *const pos = bins + P;
+    uint32_t *const lim = pos + P;
+    uint32_t *const ccount = lim + P;
+    ull *const wb = reinterpret_cast<ull *>(ccount + P);
+    ull *const base = wb + P;
+    Tup *const carry = reinterpret_cast<Tup *>(base + P);
+    __shared__ __align__(8) uint64_t bar;
     __shared__ uint32_t tmp[33];
     const int tid = threadIdx.x;
     const int tile = blockIdx.x;
@@ -77,8 +90,7 @@ __global__ void __launch_bounds__(SCATTER_THREADS, 1) k_scatter(Ctx c) {
     }
     const uint32_t ntot = nsub[0] + nsub[1];
     if (tid == 0) {
-        mbar_init(&bar[0], 1);
-        mbar_init(&bar[1], 1);
+        mbar_init(&bar, 1);
         fence_mbar_init();
     }
     __syncthreads();
@@ -98,11 +110,10 @@ __global__ void __launch_bounds__(SCATTER_THREADS, 1) k_scatter(Ctx c) {
         subtile(g, rel, first, len);
         const uint32_t body = len & ~(uint32_t)(16 / sizeof(K) - 1);
         const uint32_t bytes = body * (uint32_t)sizeof(K);
-        uint64_t *b = &bar[g & 1];
-        mbar_arrive_expect_tx(b, 2 * bytes);
+        mbar_arrive_expect_tx(&bar, 2 * bytes);
         if (bytes) {
-            tma_load_1d(skey(g & 1), static_cast<const K *>(c.in_key[rel]) + first, bytes, b, pol);
-            tma_load_1d(spay(g & 1), static_cast<const K *>(c.in_pay[rel]) + first, bytes, b, pol);
+            tma_load_1d(skey, static_cast<const K *>(c.in_key[rel]) + first, bytes, &bar, pol);
+            tma_load_1d(spay, static_cast<const K *>(c.in_pay[rel]) + first, bytes, &bar, pol);
         }
     };
     auto set_base = [&](int rel) {  // destination of this tile's first tuple of each partition
@@ -110,27 +121,31 @@ __global__ void __launch_bounds__(SCATTER_THREADS, 1) k_scatter(Ctx c) {
         const uint64_t *so = c.send_off + (size_t)rel * P;
         for (int p = tid; p < P; p += SCATTER_THREADS) {
             const int own = c.owner[p];
-            base[p] = (unsigned long long)(c.arena[own] + c.lay.recv[rel]) + (so[p] + tb[p]) * (uint64_t)TB;
+            base[p] = (ull)(c.arena[own] + c.lay.recv[rel]) + (so[p] + tb[p]) * (uint64_t)TB;
+            ccount[p] = 0;
         }
     };
+    auto flush_carry = [&]() {  // end of a relation: write the remaining tails
+        for (int p = tid; p < P; p += SCATTER_THREADS)
+            for (uint32_t k = 0; k < ccount[p]; ++k)
+                reinterpret_cast<Tup *>(base[p])[k] = carry[(size_t)p * CC + k];
+    };
 
-    if (tid == 0) {
-        if (ntot > 0) issue(0);
-        if (ntot > 1) issue(1);
-    }
+    if (tid == 0 && ntot > 0) issue(0);
     int cur_rel = -1;
     for (uint32_t g = 0; g < ntot; ++g) {
         int rel;
         uint64_t first;
         uint32_t len;
         subtile(g, rel, first, len);
-        if (rel != cur_rel) {  // (previous sub-tile's write-out is ordered by the barriers below)
+        if (rel != cur_rel) {
+            __syncthreads();
+            if (cur_rel >= 0) flush_carry();
             __syncthreads();
             set_base(rel);
             cur_rel = rel;
         }
-        const int s = g & 1;
-        mbar_wait(&bar[s], (g >> 1) & 1);
+        mbar_wait(&bar, g & 1);
         const uint32_t body = len & ~(uint32_t)(16 / sizeof(K) - 1);
         const K *gk = static_cast<const K *>(c.in_key[rel]) + first;
         const K *gp = static_cast<const K *>(c.in_pay[rel]) + first;
@@ -139,16 +154,16 @@ __global__ void __launch_bounds__(SCATTER_THREADS, 1) k_scatter(Ctx c) {
         for (int v = 0; v < VMAX; ++v) {
             const uint32_t i = tid + v * SCATTER_THREADS;
             if (v < V && i < body) {
-                kk[v] = skey(s)[i];
-                pp[v] = spay(s)[i];
+                kk[v] = skey[i];
+                pp[v] = spay[i];
             } else if (v < V && i < len) {  // < 4 trailing tuples of the relation
                 kk[v] = gk[i];
                 pp[v] = gp[i];
             }
         }
         for (int p = tid; p < P; p += SCATTER_THREADS) bins[p] = 0;
-        __syncthreads();  // stage s consumed, bins cleared
-        if (tid == 0 && g + 2 < ntot) issue(g + 2);
+        __syncthreads();  // S1: stage consumed, bins cleared
+        if (tid == 0 && g + 1 < ntot) issue(g + 1);
         uint32_t rp[VMAX];  // rank in bin << 16 | partition
 #pragma unroll
         for (int v = 0; v < VMAX; ++v) {
@@ -158,14 +173,26 @@ __global__ void __launch_bounds__(SCATTER_THREADS, 1) k_scatter(Ctx c) {
                 rp[v] = (atomicAdd(&bins[p], 1u) << 16) | p;
             }
         }
+        __syncthreads();  // S2
+        for (int p = tid; p < P; p += SCATTER_THREADS) bins[p] += ccount[p];
         __syncthreads();
-        block_excl_scan_u32(bins, P, tmp);
+        const uint32_t ttot = block_excl_scan_u32(bins, P, tmp);
         for (int p = tid; p < P; p += SCATTER_THREADS) {
-            const uint32_t o = bins[p], e = (p + 1 < P) ? bins[p + 1] : len;
-            const unsigned long long b = base[p];
-            wbase[p] = b - (unsigned long long)o * TB;
-            base[p] = b + (unsigned long long)(e - o) * TB;
+            const uint32_t o = bins[p];
+            const uint32_t tp = ((p + 1 < P) ? bins[p + 1] : ttot) - o;
+            const uint32_t cc = ccount[p];
+            const ull G = base[p];
+            const ull end = G + (ull)tp * TB;
+            const ull aend = CC ? (end & ~31ull) : end;
+            const uint32_t L = aend > G ? (uint32_t)((aend - G) / TB) : 0;
+            lim[p] = o + L;
+            wb[p] = G - (ull)o * TB;
+            base[p] = G + (ull)L * TB;
+            for (uint32_t k = 0; k < cc; ++k) sorted[o + k] = carry[(size_t)p * CC + k];
+            pos[p] = o + cc;
+            ccount[p] = tp - L;
         }
+        __syncthreads();  // S3
 #pragma unroll
         for (int v = 0; v < VMAX; ++v) {
             const uint32_t i = tid + v * SCATTER_THREADS;
@@ -173,16 +200,20 @@ __global__ void __launch_bounds__(SCATTER_THREADS, 1) k_scatter(Ctx c) {
                 Tup t;
                 t.x = kk[v];
                 t.y = pp[v];
-                sorted[bins[rp[v] & 0xffffu] + (rp[v] >> 16)] = t;
+                sorted[pos[rp[v] & 0xffffu] + (rp[v] >> 16)] = t;
             }
         }
-        __syncthreads();
-        for (uint32_t i = tid; i < len; i += SCATTER_THREADS) {
+        __syncthreads();  // S4
+        for (uint32_t i = tid; i < ttot; i += SCATTER_THREADS) {
             const Tup t = sorted[i];
-            Tup *dst = reinterpret_cast<Tup *>(wbase[digit1(t.x, P)] + (unsigned long long)i * TB);
-            *dst = t;
+            const uint32_t p = digit1(t.x, P);
+            const uint32_t l = lim[p];
+            if (i < l) reinterpret_cast<Tup *>(wb[p] + (ull)i * TB)[0] = t;
+            else carry[(size_t)p * CC + (i - l)] = t;
         }
     }
+    __syncthreads();
+    if (cur_rel >= 0) flush_carry();
 
     // ---- every CTA: make its (peer) stores visible, the last one signals ----
     __threadfence_system();

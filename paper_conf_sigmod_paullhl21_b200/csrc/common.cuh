@@ -18,7 +18,7 @@ constexpr int SCAT_T8 = 8192;           // scatter sub-tile (tuples) for 8-byte 
 constexpr int LOCAL_THREADS = 1024;
 constexpr int LOCAL_C8 = 8192;          // local-pass chunk (tuples) for 8-byte tuples; 4096 for 16-byte
 constexpr int PROBE_THREADS = 1024;     // warps 0..PROBE_NP-1 = TMA producers, the rest build/probe
-constexpr int PROBE_NP = 2;             // producer warps
+constexpr int PROBE_NP = 4;             // producer warps (<= PROBE_NST: parity waits are one phase ahead)
 constexpr int PROBE_NST = 4;            // pipeline stages (items in flight per CTA)
 constexpr int PROBE_SLOTS8 = 3072;      // stage capacity per relation (slots) for 8-byte tuples; half for 16-byte
 constexpr int PROBE_MAXP = 1024;        // chunk pieces per relation per item

@@ -12,7 +12,8 @@ namespace mgj {
 constexpr int MAX_RANKS = MGJ_MAX_RANKS;
 constexpr int MAX_B1 = 12;              // 2^12 global partitions at most
 constexpr int MAX_B2 = 11;              // local fan-out per pass
-constexpr int HIST_THREADS = 1024;
+constexpr int HIST_THREADS = 512;
+constexpr int HIST_SPLIT = 4;           // CTAs per histogram tile
 constexpr int SCATTER_THREADS = 1024;
 constexpr int SCAT_T8 = 8192;           // scatter sub-tile (tuples) for 8-byte tuples; 4096 for 16-byte
 constexpr int LOCAL_THREADS = 1024;

@@ -21,10 +21,15 @@ template <typename K>
 __global__ void __launch_bounds__(HIST_THREADS) k_hist(Ctx c) {
     extern __shared__ uint32_t sh[];  // [P]
     const int P = c.P;
-    const int rel = blockIdx.y, tile = blockIdx.x;
+    const int rel = blockIdx.y, tile = blockIdx.x / HIST_SPLIT, part = blockIdx.x % HIST_SPLIT;
     const K *keys = static_cast<const K *>(c.in_key[rel]);
-    uint64_t lo, hi;
-    tile_range(c.n_in[rel], c.G, tile, lo, hi);
+    uint64_t tlo, thi, lo, hi;
+    tile_range(c.n_in[rel], c.G, tile, tlo, thi);
+    {  // HIST_SPLIT CTAs share a tile (16-byte aligned parts)
+        const uint64_t n = thi - tlo;
+        lo = tlo + ((n * part / HIST_SPLIT) & ~3ull);
+        hi = part == HIST_SPLIT - 1 ? thi : tlo + ((n * (part + 1) / HIST_SPLIT) & ~3ull);
+    }
     for (int i = threadIdx.x; i < P; i += blockDim.x) sh[i] = 0;
     __syncthreads();
 
@@ -59,8 +64,10 @@ __global__ void __launch_bounds__(HIST_THREADS) k_hist(Ctx c) {
     uint32_t *th = c.tile_hist + ((size_t)rel * c.G + tile) * P;
     for (int p = threadIdx.x; p < P; p += blockDim.x) {
         const uint32_t v = sh[p];
-        th[p] = v;
-        if (v) atomicAdd(&c.rank_hist[rel * P + p], v);
+        if (v) {
+            atomicAdd(&th[p], v);
+            atomicAdd(&c.rank_hist[rel * P + p], v);
+        }
     }
 
     // ---- fused exchange: the last CTA publishes the rank histogram ----

@@ -171,7 +171,7 @@ bool is_device_ptr(const void *p) {
 template <typename K>
 void launch_partition(mgj_plan_s *h, cudaStream_t s) {
     const Norm &n = h->n;
-    dim3 g(h->ctx.G, 2);
+    dim3 g(h->ctx.G * HIST_SPLIT, 2);
     k_hist<K><<<g, HIST_THREADS, hist_smem(n), s>>>(h->ctx);
 }
 
@@ -264,6 +264,7 @@ mgj_status mgj_plan(const mgj_config *cfg, const mgj_peers *peers, mgj_handle *o
     const size_t z_acc = zo; zo += 256;
     const size_t z_err = zo; zo += 256;
     const size_t z_cop = zo; zo += align_up(2ull * P * Qm * 4, 256);
+    const size_t z_th = zo; zo += align_up(2ull * h->nsm * P * 4, 256);
     h->zero_bytes = zo;
     char *zb = static_cast<char *>(dalloc(h, zo, &st));
     h->zero_block = zb;
@@ -293,8 +294,8 @@ mgj_status mgj_plan(const mgj_config *cfg, const mgj_peers *peers, mgj_handle *o
         c.acc = reinterpret_cast<unsigned long long *>(zb + z_acc);
         c.err = reinterpret_cast<int32_t *>(zb + z_err);
         c.cop_slots = reinterpret_cast<uint32_t *>(zb + z_cop);
+        c.tile_hist = reinterpret_cast<uint32_t *>(zb + z_th);
     }
-    c.tile_hist = static_cast<uint32_t *>(dalloc(h, 2ull * c.G * P * 4, &st));
     c.tile_base = static_cast<uint32_t *>(dalloc(h, 2ull * c.G * P * 4, &st));
     h->cdesc = static_cast<ChunkDesc *>(dalloc(h, 2 * n.max_chunks * sizeof(ChunkDesc), &st));
     c.owner = static_cast<int32_t *>(dalloc(h, P * 4, &st));

@@ -44,7 +44,7 @@ def parse():
     ap.add_argument("--materialize", action="store_true")
     ap.add_argument("--radix-bits-global", type=int, default=0)
     ap.add_argument("--radix-bits-local", type=int, default=0)
-    ap.add_argument("--cpu-sample-log2", type=int, default=26,
+    ap.add_argument("--cpu-sample-log2", type=int, default=28,
                     help="oracle sample: 2^k R + 2^k S unique tuples (cpu_baseline / --impl reference)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")

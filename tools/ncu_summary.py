@@ -43,3 +43,20 @@ if __name__ == "__main__":
     if len(sys.argv) > 2 and sys.argv[2] != "-":
         print("\n## ncu --set full (one launch per kernel, M2 N=1)\n")
         print(full(sys.argv[2]))
+
+
+def traffic_json(path):
+    """{kernel: dram_read+dram_write bytes per launch} from a --set full capture."""
+    out = subprocess.run(["ncu", "-i", path, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
+    rows = list(csv.reader(io.StringIO(out)))
+    h, u = rows[0], rows[1]
+    scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "Tbyte": 1e12}
+    res = {}
+    for r in rows[2:]:
+        name = r[h.index("Kernel Name")].split("(")[0].replace("void ", "").split("<")[0].split("::")[-1]
+        tot = 0.0
+        for m in ("dram__bytes_read.sum", "dram__bytes_write.sum"):
+            i = h.index(m)
+            tot += float(r[i].replace(",", "")) * scale.get(u[i], 1)
+        res[name] = tot
+    return res

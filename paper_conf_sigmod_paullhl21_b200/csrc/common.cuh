@@ -17,7 +17,8 @@ constexpr int HIST_SPLIT = 4;           // CTAs per histogram tile
 constexpr int SCATTER_THREADS = 1024;
 constexpr int SCAT_T8 = 8192;           // scatter sub-tile (tuples) for 8-byte tuples; 4096 for 16-byte
 constexpr int LOCAL_THREADS = 1024;
-constexpr int LOCAL_C8 = 8192;          // local-pass chunk (tuples) for 8-byte tuples; 4096 for 16-byte
+constexpr int LOCAL_VMAX = 12;          // local-pass tuples per thread (chunk C <= 12 * LOCAL_THREADS), 8-byte tuples
+__host__ __device__ constexpr int local_vmax(int tuple_bytes) { return LOCAL_VMAX * 8 / tuple_bytes; }
 constexpr int PROBE_THREADS = 1024;     // warps 0..PROBE_NP-1 = TMA producers, the rest build/probe
 constexpr int PROBE_NP = 4;             // producer warps (<= PROBE_NST: parity waits are one phase ahead)
 constexpr int PROBE_NST = 4;            // pipeline stages (items in flight per CTA)
@@ -29,7 +30,7 @@ enum Sig { SIG_HIST = 0, SIG_DATA = 1, SIG_RES = 2, SIG_COUNT = 3 };
 enum Ticket { TK_HIST = 0, TK_SCAT_R = 1, TK_SCAT_S = 2, TK_SCAT_DONE = 3, TK_ITEMS = 4,
               TK_PROBE = 5, TK_LOCAL = 6, TK_COUNT = 8 };
 enum Meta { MT_PLO = 0, MT_PHI = 1, MT_B2 = 2, MT_OK = 3, MT_NCH_R = 4, MT_NCH_S = 5,
-            MT_NITEMS = 6, MT_COUNT = 16 };
+            MT_NITEMS = 6, MT_CHUNK = 7, MT_COUNT = 16 };
 
 // Arena layout (bytes from each rank's arena base; identical on all ranks).
 struct Arena {

@@ -253,6 +253,7 @@ __global__ void __launch_bounds__(1024) k_plan(Ctx c) {
         c.meta[MT_B2] = B2;
         c.meta[MT_NCH_R] = (int)nch[0];
         c.meta[MT_NCH_S] = (int)nch[1];
+        c.meta[MT_CHUNK] = c.chunk_tuples;
         c.meta[MT_OK] = (cap_bad || !fits) ? 0 : 1;
     }
 }

@@ -30,8 +30,10 @@ __device__ __forceinline__ void decode_run(uint32_t e0, uint32_t e1, uint32_t &s
     }
 }
 
+// Two chunk buffers that alternate roles (TMA load target of chunk j+1 /
+// sorted output of chunk j), plus the bin counters.
 __host__ __device__ inline size_t local_smem_bytes(int C, int Qmax, int TB) {
-    return 2 * (size_t)(C + 2) * TB + (size_t)(C + Qmax) * TB + 2 * (size_t)Qmax * 4;
+    return 2 * (size_t)(C + Qmax + 2) * TB + 2 * (size_t)Qmax * 4;
 }
 
 // Chunk descriptors for the local pass: chunk ci of owned partition pi covers
@@ -85,7 +87,7 @@ template <typename K>
 __global__ void __launch_bounds__(LOCAL_THREADS, 1) k_local(Ctx c, const ChunkDesc *cdesc) {
     using Tup = typename Layout<K>::Tup;
     constexpr int TB = Layout<K>::TB, ALIGN = Layout<K>::ALIGN;
-    constexpr int VMAX = LOCAL_C8 * 8 / TB / LOCAL_THREADS;
+    constexpr int VMAX = local_vmax(TB);
     extern __shared__ __align__(128) unsigned char smem[];
     __shared__ __align__(8) uint64_t bar[2];
     __shared__ ChunkDesc sdesc[2];
@@ -95,10 +97,10 @@ __global__ void __launch_bounds__(LOCAL_THREADS, 1) k_local(Ctx c, const ChunkDe
     const int C = c.chunk_tuples, CR = c.chunk_region, V = C / LOCAL_THREADS;
     const int P = c.P, B2 = c.meta[MT_B2], Q = 1 << B2;
     const int Qmax = 1 << c.b2_max;
-    Tup *const stage0 = reinterpret_cast<Tup *>(smem);
-    auto stage = [&](int s) { return stage0 + (size_t)s * (C + 2); };
-    Tup *sorted = stage0 + (size_t)2 * (C + 2);
-    uint32_t *bins = reinterpret_cast<uint32_t *>(sorted + C + Qmax);
+    const int BUF = C + Qmax + 2;  // slots per buffer
+    Tup *const buf0 = reinterpret_cast<Tup *>(smem);
+    auto buf = [&](int x) { return buf0 + (size_t)x * BUF; };
+    uint32_t *bins = reinterpret_cast<uint32_t *>(buf0 + (size_t)2 * BUF);
     uint32_t *abin = bins + Qmax;
     const uint32_t nch_r = (uint32_t)c.meta[MT_NCH_R];
     const uint32_t total = nch_r + (uint32_t)c.meta[MT_NCH_S];
@@ -111,7 +113,7 @@ __global__ void __launch_bounds__(LOCAL_THREADS, 1) k_local(Ctx c, const ChunkDe
     }
     __syncthreads();
     const uint64_t pol = policy_evict_first();
-    // thread 0 keeps the descriptor of the next chunk to issue in registers (prefetched)
+    // thread 0: TMA chunk j (16-byte-aligned superset) into buffer j & 1
     auto issue = [&](uint32_t j, const ChunkDesc &d) {
         const uint32_t ci = blockIdx.x + j * gridDim.x;
         const int rel = ci < nch_r ? 0 : 1;
@@ -122,33 +124,33 @@ __global__ void __launch_bounds__(LOCAL_THREADS, 1) k_local(Ctx c, const ChunkDe
         uint64_t *b = &bar[j & 1];
         mbar_arrive_expect_tx(b, bytes);
         if (bytes)
-            tma_load_1d(stage(j & 1), reinterpret_cast<const Tup *>(recv0 + c.lay.recv[rel]) + g0, bytes, b, pol);
+            tma_load_1d(buf(j & 1), reinterpret_cast<const Tup *>(recv0 + c.lay.recv[rel]) + g0, bytes, b, pol);
     };
     ChunkDesc nxt{};
     if (tid == 0) {
         if (mine > 0) issue(0, cdesc[blockIdx.x]);
-        if (mine > 1) issue(1, cdesc[blockIdx.x + gridDim.x]);
-        if (mine > 2) nxt = cdesc[blockIdx.x + 2 * gridDim.x];
+        if (mine > 1) nxt = cdesc[blockIdx.x + gridDim.x];
     }
     for (uint32_t j = 0; j < mine; ++j) {
         const uint32_t ci = blockIdx.x + j * gridDim.x;
         const int rel = ci < nch_r ? 0 : 1;
         const uint32_t li = rel ? ci - nch_r : ci;
-        const int s = j & 1;
-        mbar_wait(&bar[s], (j >> 1) & 1);
-        const ChunkDesc d = sdesc[s];
+        const int X = j & 1;
+        mbar_wait(&bar[X], (j >> 1) & 1);
+        const ChunkDesc d = sdesc[X];
         const uint32_t len = d.len, skip = (uint32_t)(d.start & (ALIGN - 1));
         Tup t[VMAX];
 #pragma unroll
         for (int v = 0; v < VMAX; ++v) {
             const uint32_t i = tid + v * LOCAL_THREADS;
-            if (v < V && i < len) t[v] = stage(s)[skip + i];
+            if (v < V && i < len) t[v] = buf(X)[skip + i];
         }
         for (int q = tid; q < Q; q += LOCAL_THREADS) bins[q] = 0;
-        __syncthreads();  // S1: stage s consumed
-        if (tid == 0 && j + 2 < mine) {
-            issue(j + 2, nxt);
-            if (j + 3 < mine) nxt = cdesc[blockIdx.x + (j + 3) * gridDim.x];
+        __syncthreads();  // S1: buffer X consumed (it becomes this chunk's sorted output)
+        if (tid == 0 && j + 1 < mine) {
+            bulk_wait_read0();  // chunk j-1's bulk store has finished reading buffer X^1
+            issue(j + 1, nxt);
+            if (j + 2 < mine) nxt = cdesc[blockIdx.x + (j + 2) * gridDim.x];
         }
         uint32_t rq[VMAX];  // rank << 16 | digit2
 #pragma unroll
@@ -159,7 +161,6 @@ __global__ void __launch_bounds__(LOCAL_THREADS, 1) k_local(Ctx c, const ChunkDe
                 rq[v] = (atomicAdd(&bins[q], 1u) << 16) | q;
             }
         }
-        if (tid == 0) bulk_wait_read0();  // previous chunk's bulk store has read `sorted`
         __syncthreads();  // S2
         for (int q = tid; q < Q; q += LOCAL_THREADS) abin[q] = (bins[q] + ALIGN - 1) & ~(uint32_t)(ALIGN - 1);
         __syncthreads();
@@ -179,6 +180,7 @@ __global__ void __launch_bounds__(LOCAL_THREADS, 1) k_local(Ctx c, const ChunkDe
                 }
             }
         }
+        Tup *const sorted = buf(X);
 #pragma unroll
         for (int v = 0; v < VMAX; ++v) {
             const uint32_t i = tid + v * LOCAL_THREADS;
@@ -188,7 +190,7 @@ __global__ void __launch_bounds__(LOCAL_THREADS, 1) k_local(Ctx c, const ChunkDe
                 // 16-byte padding slot of an odd run: a tuple whose key has its
                 // lowest bit flipped, i.e. lies in another global partition, so
                 // it never equals a real key of this co-partition; the probe
-                // skips S padding slots (bitmap), R padding is inert
+                // skips S padding slots (bitmap), R padding is inert (DESIGN.md §2 R2)
                 if (ALIGN == 2 && r == 0 && (bins[q] & 1u)) {
                     Tup pad = t[v];
                     pad.x ^= 1;

@@ -66,11 +66,15 @@ mgj_status normalize(const mgj_config *in, Norm *o) {
     if (c.radix_bits_local > 0) {
         o->b2_max = c.radix_bits_local;
     } else {
-        o->b2_max = std::min(MAX_B2, std::max(1, ceil_log2((c.recv_capacity_r + target - 1) / target)));
+        // expected largest owned R partition ~ recv_cap / P; +2 bits of headroom for skew
+        const uint64_t per_p = (c.recv_capacity_r + o->P - 1) / o->P;
+        o->b2_max = std::min(MAX_B2, std::max(1, ceil_log2((per_p + target - 1) / target) + 2));
     }
     const int Qm = 1 << o->b2_max;
-    int C = LOCAL_C8 * 8 / o->tuple_bytes;
-    while (C > LOCAL_THREADS && local_smem_bytes(C, Qm, o->tuple_bytes) > 225 * 1024) C /= 2;
+    int C = 0;  // largest chunk (multiple of LOCAL_THREADS) whose buffers fit shared memory
+    for (int v = local_vmax(o->tuple_bytes); v >= 1 && !C; --v)
+        if (local_smem_bytes(v * LOCAL_THREADS, Qm, o->tuple_bytes) <= 225 * 1024) C = v * LOCAL_THREADS;
+    if (!C) return MGJ_EINVAL;
     o->chunk_tuples = C;
     o->chunk_region = C + Qm;  // worst-case padding: one slot per run
     const uint64_t rmax = std::max(o->recv_cap[0], o->recv_cap[1]);

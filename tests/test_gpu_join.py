@@ -118,7 +118,7 @@ def test_phases_m1(mgj, b1):
         # whose tuples all have digit2 == q, and the chunk's multiset is kept
         B2 = res["radix_bits_local"]
         Q = 1 << B2
-        C = 8192
+        C = int(j.debug("META", np.int32)[7])  # local-pass chunk size
         seg = j.debug("SEGMENTS", np.uint64).reshape(4, P)
         start, ln = seg[rel], seg[2 + rel]
         E = j.debug("CHUNK_OFF_R" if rel == 0 else "CHUNK_OFF_S", np.uint16).astype(np.int64)

@@ -240,10 +240,17 @@ def main():
     for _ in range(max(a.warmup, 1)):
         step()
         res = join.result()
-    expect_ok = True
+    # closed forms (tests/golden/appendix_a_closed_forms.json)
+    M64 = (1 << 64) - 1
     if a.workload == "unique":
         n = n_r
-        expect_ok = res["match_count"] == n and res["checksum"] == ((1 << 32) + 1) * n * (n - 1) // 2 % (1 << 64)
+        expect_ok = res["match_count"] == n and res["checksum"] == ((1 << 32) + 1) * n * (n - 1) // 2 & M64
+    elif a.workload == "wide":
+        n, h = n_r, n_r * (n_r - 1) // 2
+        chk = (0x9E3779B97F4A7C15 * (n * (1 << 40) + h) + n * (1 << 41) + h) & M64
+        expect_ok = res["match_count"] == n and res["checksum"] == chk
+    else:  # zipf: every even S row matches exactly one R tuple, odd rows never match
+        expect_ok = res["match_count"] == n_s // 2
 
     sampler = ClockSampler(local) if (rank == 0 and not a.profile) else None
     if sampler:

@@ -1,0 +1,47 @@
+"""Small joins for compute-sanitizer (memcheck / racecheck / synccheck): unique,
+duplicate-heavy, wide, and 2 virtual ranks."""
+import sys, os
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np
+import torch
+import oracle
+from paper_conf_sigmod_paullhl21_b200 import datagen, mgj
+
+
+def dev(a):
+    return torch.from_numpy(np.ascontiguousarray(a.view(np.int32 if a.dtype == np.uint32 else np.int64))).cuda()
+
+
+def one(d, **kw):
+    kb = 8 if d["r_keys"].dtype == np.uint64 else 4
+    ref = oracle.join(d["r_keys"], d["r_pays"], d["s_keys"], d["s_pays"])
+    j = mgj.Join(mgj.make_config(key_bytes=kb, r_capacity=d["r_keys"].size, s_capacity=d["s_keys"].size,
+                                 out_capacity=max(ref["count"], 1), **kw))
+    r = j.run(*[dev(d[k]) for k in ("r_keys", "r_pays", "s_keys", "s_pays")])
+    assert (r["match_count"], r["checksum"]) == (ref["count"], ref["checksum"]), (r, ref)
+    j.close()
+
+
+one(datagen.Workload("unique", 1 << 16, 1 << 16).rank_inputs(), materialize=True)
+rng = np.random.default_rng(0)
+one({"r_keys": rng.integers(0, 300, 20000, dtype=np.uint64).astype(np.uint32), "r_pays": np.arange(20000, dtype=np.uint32),
+     "s_keys": rng.integers(0, 300, 30000, dtype=np.uint64).astype(np.uint32), "s_pays": np.arange(30000, dtype=np.uint32)},
+    materialize=False, radix_bits_global=4)
+one(datagen.Workload("wide", 1 << 14, 1 << 14).rank_inputs(), materialize=True)
+# two virtual ranks
+w = datagen.Workload("unique", 1 << 15, 1 << 15)
+parts = [w.rank_inputs(g, 2) for g in range(2)]
+cfgs = [mgj.make_config(rank=g, world_size=2, r_capacity=1 << 14, s_capacity=1 << 14, recv_capacity_r=1 << 15,
+                        recv_capacity_s=1 << 15) for g in range(2)]
+nb = mgj.arena_bytes(cfgs[0])
+arenas = [torch.zeros(nb, dtype=torch.uint8, device="cuda") for _ in range(2)]
+js = [mgj.Join(cfgs[g], [a.data_ptr() for a in arenas], nb) for g in range(2)]
+ts = [[dev(p[k]) for k in ("r_keys", "r_pays", "s_keys", "s_pays")] for p in parts]
+for g in range(2): js[g].partition(*ts[g])
+for g in range(2): js[g].shuffle()
+for g in range(2): js[g].join()
+res = [js[g].result() for g in range(2)]
+full = w.rank_inputs()
+ref = oracle.join(full["r_keys"], full["r_pays"], full["s_keys"], full["s_pays"])
+assert (res[0]["match_count"], res[0]["checksum"]) == (ref["count"], ref["checksum"])
+print("sanitize workload ok")

@@ -20,9 +20,10 @@ constexpr int LOCAL_THREADS = 1024;
 constexpr int LOCAL_VMAX = 12;          // local-pass tuples per thread (chunk C <= 12 * LOCAL_THREADS), 8-byte tuples
 __host__ __device__ constexpr int local_vmax(int tuple_bytes) { return LOCAL_VMAX * 8 / tuple_bytes; }
 constexpr int PROBE_THREADS = 1024;     // warps 0..PROBE_NP-1 = TMA producers, the rest build/probe
-constexpr int PROBE_NP = 4;             // producer warps (<= PROBE_NST: parity waits are one phase ahead)
-constexpr int PROBE_NST = 4;            // pipeline stages (items in flight per CTA)
-constexpr int PROBE_SLOTS8 = 3072;      // stage capacity per relation (slots) for 8-byte tuples; half for 16-byte
+constexpr int PROBE_NP = 3;             // producer warps (<= PROBE_NST: parity waits are one phase ahead)
+constexpr int PROBE_NST = 3;            // pipeline stages (items in flight per CTA)
+constexpr int PROBE_SLOTS8 = 4224;      // stage capacity per relation (slots) for 8-byte tuples; half for 16-byte
+constexpr int PROBE_HEAD8 = 128;        // headroom: co-partition target = capacity - headroom (padding, spread)
 constexpr int PROBE_MAXP = 1024;        // chunk pieces per relation per item
 constexpr uint64_t WAIT_TIMEOUT_NS = 20ull * 1000 * 1000 * 1000;
 
@@ -60,6 +61,7 @@ struct Ctx {
     int32_t chunk_tuples;         // local-pass chunk C (tuples)
     int32_t chunk_region;         // slots per chunk in the local buffer (C + 2^b2_max, even)
     int32_t probe_slots;          // probe stage capacity per relation (slots)
+    int32_t probe_target;         // co-partition size B2 aims at (tuples)
     int32_t materialize;
     uint32_t max_items;
     uint64_t epoch;

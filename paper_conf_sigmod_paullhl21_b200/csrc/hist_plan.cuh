@@ -232,7 +232,7 @@ __global__ void __launch_bounds__(1024) k_plan(Ctx c) {
     const int phi = first[c.rank] < P ? endp[c.rank] : 0;
     for (int p = plo + tid; p < phi; p += blockDim.x) atomicMax(&maxr, (unsigned long long)tot0[p]);
     __syncthreads();
-    const int B2 = choose_b2(maxr, c.b2_cfg, c.b2_max, (uint64_t)c.probe_slots * 2 / 3);
+    const int B2 = choose_b2(maxr, c.b2_cfg, c.b2_max, (uint64_t)c.probe_target);
     // chunk table of the local pass: chunk_base[rel][pi] = first chunk of owned partition plo+pi
     const int np = phi - plo;
     const uint64_t C = (uint64_t)c.chunk_tuples;

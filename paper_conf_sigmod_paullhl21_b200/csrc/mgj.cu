@@ -26,7 +26,7 @@ uint64_t align_up(uint64_t x, uint64_t a) { return (x + a - 1) / a * a; }
 
 struct Norm {  // validated config with the automatic fields filled in
     mgj_config c;
-    int B1, P, b2_max, tuple_bytes, chunk_tuples, chunk_region, probe_slots;
+    int B1, P, b2_max, tuple_bytes, chunk_tuples, chunk_region, probe_slots, probe_target;
     uint64_t recv_cap[2], max_chunks, max_items, out_cap;
     Arena lay;
 };
@@ -61,7 +61,8 @@ mgj_status normalize(const mgj_config *in, Norm *o) {
     o->recv_cap[0] = c.recv_capacity_r;
     o->recv_cap[1] = c.recv_capacity_s;
     o->probe_slots = PROBE_SLOTS8 * 8 / o->tuple_bytes;
-    const uint64_t target = (uint64_t)o->probe_slots * 2 / 3;
+    o->probe_target = (PROBE_SLOTS8 - PROBE_HEAD8) * 8 / o->tuple_bytes;
+    const uint64_t target = (uint64_t)o->probe_target;
     // B2 upper bound: the largest R segment this rank could own is recv_cap_r.
     if (c.radix_bits_local > 0) {
         o->b2_max = c.radix_bits_local;
@@ -283,6 +284,7 @@ mgj_status mgj_plan(const mgj_config *cfg, const mgj_peers *peers, mgj_handle *o
     c.chunk_tuples = n.chunk_tuples;
     c.chunk_region = n.chunk_region;
     c.probe_slots = n.probe_slots;
+    c.probe_target = n.probe_target;
     c.materialize = n.c.materialize;
     c.max_items = (uint32_t)n.max_items;
     c.recv_cap[0] = n.recv_cap[0];

@@ -141,7 +141,7 @@ def _cpu_model() -> str:
     return "unknown"
 
 
-def run_reference(a) -> None:
+def run_reference(a, out) -> None:
     rank, world, _ = dist_env()
     if rank != 0:
         return
@@ -160,7 +160,7 @@ def run_reference(a) -> None:
     v = 2 * n / (ms / 1000)
     sample = (f"each step joins a bounded sample: 2^{int(np.log2(n))} R + 2^{int(np.log2(n))} S unique tuples "
               f"of the M2 workload shape, single-threaded, 1 of {os.cpu_count()} cores ({_cpu_model()})")
-    print(json.dumps({
+    emit(out, {
         "impl": "reference", "metric": METRIC, "value": v, "unit": UNIT, "n_gpus": world, "steps": a.steps,
         "warmup": a.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
         "vs_baseline": None, "dtype": "u32", "data": "synthetic",
@@ -168,14 +168,29 @@ def run_reference(a) -> None:
                    "tuple_bytes": 8},
         "cpu_baseline": {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
         "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
-    }))
+    })
 
 
 # ------------------------------------------------------------------ main bench
+def _claim_stdout():
+    """Keep the process's stdout for the single JSON line: everything else
+    (NCCL banners, library chatter) is redirected to stderr."""
+    sys.stdout.flush()
+    out = os.fdopen(os.dup(1), "w")
+    os.dup2(2, 1)
+    return out
+
+
+def emit(out, obj) -> None:
+    out.write(json.dumps(obj) + "\n")
+    out.flush()
+
+
 def main():
     a = parse()
+    out = _claim_stdout()
     if a.impl == "reference":
-        run_reference(a)
+        run_reference(a, out)
         return
     import torch
     import torch.distributed as dist
@@ -185,7 +200,10 @@ def main():
     rank, world, local = dist_env()
     assert world == a.gpus or (world == 1 and a.gpus == 1), "launch N>1 with torchrun --nproc-per-node N"
     torch.cuda.set_device(local)
-    if world > 1:
+    # N>1: one rank per GPU over NCCL with symmetric-memory arenas.  MGJ_SYMM_ARENA=1 forces the
+    # same symmetric-memory path at N=1 (under torchrun) to exercise it on a single GPU.
+    distributed = world > 1 or os.environ.get("MGJ_SYMM_ARENA") == "1"
+    if distributed:
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     dev = torch.device("cuda", local)
     stream = torch.cuda.Stream(device=dev)
@@ -213,7 +231,7 @@ def main():
                           recv_capacity_r=(n_r if world > 1 and a.workload == "zipf" else 0),
                           recv_capacity_s=(n_s // 2 if world > 1 and a.workload == "zipf" else 0))
     arena = None
-    if world > 1:
+    if distributed:
         import torch.distributed._symmetric_memory as symm_mem
         nbytes = mgj.arena_bytes(cfg)
         arena = symm_mem.empty(nbytes, dtype=torch.uint8, device=dev)
@@ -383,9 +401,9 @@ def main():
             "gpu_launches": 8 * a.steps,
             "clocks": clocks,
         }
-        print(json.dumps(line))
+        emit(out, line)
     join.close()
-    if world > 1:
+    if distributed:
         dist.destroy_process_group()
 
 

@@ -69,8 +69,20 @@ typedef struct {
     int32_t  materialize;              /* 0/1: emit (key, payR, payS) triples */
     int32_t  num_sms;                  /* 0 = device attribute */
     uint64_t out_capacity;             /* max materialised triples on this rank (0 = auto) */
-    int32_t  reserved[8];              /* must be zero */
+    int32_t  shuffle_mode;             /* MGJ_SHUFFLE_P2P (0, default) | MGJ_SHUFFLE_EXTERNAL (1) */
+    int32_t  reserved[7];              /* must be zero */
 } mgj_config;
+
+/*
+ * Shuffle modes.  P2P (the product path): k_scatter stores every tuple
+ * straight into its owner's receive buffer through peer-mapped symmetric
+ * memory (NVLink/NVSwitch).  EXTERNAL (the measured NCCL baseline): k_scatter
+ * packs the tuples into a per-relation send buffer laid out by destination
+ * rank, the caller exchanges it with its own collective (e.g. NCCL
+ * all_to_all_single) into each rank's receive area between mgj_shuffle and
+ * mgj_join, using the sizes from mgj_exchange_layout.
+ */
+enum { MGJ_SHUFFLE_P2P = 0, MGJ_SHUFFLE_EXTERNAL = 1 };
 
 typedef struct mgj_plan_s *mgj_handle;
 
@@ -141,6 +153,22 @@ mgj_status mgj_shuffle(mgj_handle h, void *stream);
  * ranks.  Materialised triples stay on the owning rank.
  */
 mgj_status mgj_join(mgj_handle h, void *stream);
+
+/* EXTERNAL shuffle: buffers and per-rank sizes (tuples) of the exchange the
+ * caller performs between mgj_shuffle and mgj_join.  send[rel] holds the
+ * tuples for rank 0, then rank 1, ...; recv[rel] (this rank's arena) must
+ * receive the tuples from rank 0, then rank 1, ...  Synchronises the stream
+ * of the last call (the sizes are computed on the device). */
+typedef struct {
+    void    *send[2];
+    void    *recv[2];
+    uint64_t send_count[2][MGJ_MAX_RANKS];
+    uint64_t recv_count[2][MGJ_MAX_RANKS];
+    int32_t  tuple_bytes;
+    int32_t  world_size;
+} mgj_exchange_t;
+
+mgj_status mgj_exchange_layout(mgj_handle h, mgj_exchange_t *out);
 
 /* Synchronise the last stream and fill *out.  Returns the run's sticky status. */
 mgj_status mgj_result(mgj_handle h, mgj_result_t *out);

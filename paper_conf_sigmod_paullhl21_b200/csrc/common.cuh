@@ -63,6 +63,7 @@ struct Ctx {
     int32_t probe_slots;          // probe stage capacity per relation (slots)
     int32_t probe_target;         // co-partition size B2 aims at (tuples)
     int32_t materialize;
+    int32_t ext;                  // shuffle mode EXTERNAL: scatter into send_buf, caller exchanges
     uint32_t max_items;
     uint64_t epoch;
     uint64_t recv_cap[2];
@@ -84,6 +85,10 @@ struct Ctx {
     uint64_t *seg_start;          // [2][P]
     uint64_t *seg_len;            // [2][P]
     uint64_t *recv_size;          // [2][MAX_RANKS]
+    uint64_t *piece_start;        // [2][P][MAX_RANKS] received piece of owned partition pi from source g
+    uint32_t *piece_len;          // [2][P][MAX_RANKS]
+    uint32_t *piece_chunk;        // [2][P][MAX_RANKS+1] chunk prefix over the pieces of pi
+    uint64_t *ext_counts;         // [2 (send, recv)][2 rel][MAX_RANKS] (EXTERNAL shuffle)
     uint32_t *chunk_base;         // [2][P+1]
     uint16_t *eoff[2];            // run offsets, [(Q+1)*chunk_base[p] + q*nch_p + k]
     uint32_t *cop_slots;          // [2][P][2^b2_max] padded slots per co-partition

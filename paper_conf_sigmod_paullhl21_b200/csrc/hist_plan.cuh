@@ -210,8 +210,10 @@ __global__ void __launch_bounds__(1024) k_plan(Ctx c) {
             m1 += __ldcg(mail + (size_t)(g * 2 + 1) * P + p);
         }
         const uint64_t b0 = pre0[p] - pre0[f], b1 = pre1[p] - pre1[f];
-        c.send_off[p] = b0 + m0;
-        c.send_off[P + p] = b1 + m1;
+        if (!c.ext) {
+            c.send_off[p] = b0 + m0;
+            c.send_off[P + p] = b1 + m1;
+        }
         c.seg_start[p] = b0;
         c.seg_start[P + p] = b1;
         c.seg_len[p] = tot0[p];
@@ -233,13 +235,69 @@ __global__ void __launch_bounds__(1024) k_plan(Ctx c) {
     for (int p = plo + tid; p < phi; p += blockDim.x) atomicMax(&maxr, (unsigned long long)tot0[p]);
     __syncthreads();
     const int B2 = choose_b2(maxr, c.b2_cfg, c.b2_max, (uint64_t)c.probe_target);
-    // chunk table of the local pass: chunk_base[rel][pi] = first chunk of owned partition plo+pi
+    // received pieces of every owned partition pi: P2P — one piece (the whole
+    // segment, sources ascending inside it); EXTERNAL — one piece per source
+    // rank g, the receive area being [g0 | g1 | ...], each [owned p ascending]
     const int np = phi - plo;
     const uint64_t C = (uint64_t)c.chunk_tuples;
+    const uint32_t *mine = mail + (size_t)c.rank * 2 * P;
+    for (int rel = 0; rel < 2; ++rel) {
+        uint64_t *ps = c.piece_start + (size_t)rel * P * MAX_RANKS;
+        uint32_t *pl = c.piece_len + (size_t)rel * P * MAX_RANKS;
+        if (!c.ext) {
+            for (int i = tid; i < np; i += blockDim.x)
+                for (int g = 0; g < MAX_RANKS; ++g) {
+                    ps[(size_t)i * MAX_RANKS + g] = g == 0 ? c.seg_start[rel * P + plo + i] : 0;
+                    pl[(size_t)i * MAX_RANKS + g] = g == 0 ? (uint32_t)(rel ? tot1 : tot0)[plo + i] : 0;
+                }
+            continue;
+        }
+        uint64_t displ = 0;  // start of source g's block in this rank's receive area
+        for (int g = 0; g < N; ++g) {
+            for (int i = tid; i <= np; i += blockDim.x)
+                chn[i] = i < np ? __ldcg(mail + (size_t)(g * 2 + rel) * P + plo + i) : 0;
+            __syncthreads();
+            const uint32_t from_g = block_excl_scan_u32(chn, np + 1, tmp32);
+            for (int i = tid; i < np; i += blockDim.x) {
+                ps[(size_t)i * MAX_RANKS + g] = displ + chn[i];
+                pl[(size_t)i * MAX_RANKS + g] = __ldcg(mail + (size_t)(g * 2 + rel) * P + plo + i);
+            }
+            if (tid == 0) c.ext_counts[(1 * 2 + rel) * MAX_RANKS + g] = from_g;
+            displ += from_g;
+            __syncthreads();
+        }
+        // send side: owners are contiguous ascending ranges, so the send buffer
+        // ordered by destination is ordered by partition: offsets = prefix of H_me
+        for (int p = tid; p <= P; p += blockDim.x) {
+            if (p < P) cum[p] = __ldcg(mine + rel * P + p);
+        }
+        __syncthreads();
+        block_excl_scan_u64(cum, P, tmp);
+        for (int p = tid; p < P; p += blockDim.x) c.send_off[rel * P + p] = cum[p];
+        if (tid < N) {
+            uint64_t cnt = 0;
+            for (int p = first[tid]; p < endp[tid] && first[tid] < P; ++p) cnt += __ldcg(mine + rel * P + p);
+            c.ext_counts[(0 * 2 + rel) * MAX_RANKS + tid] = cnt;
+        }
+        __syncthreads();
+    }
+    __syncthreads();
+    // chunk table of the local pass: chunk_base[rel][pi] = first chunk of owned partition plo+pi,
+    // piece_chunk[rel][pi][g] = first chunk of piece g inside pi
     uint32_t nch[2];
     for (int rel = 0; rel < 2; ++rel) {
-        const uint64_t *tot = rel ? tot1 : tot0;
-        for (int i = tid; i <= np; i += blockDim.x) chn[i] = i < np ? (uint32_t)((tot[plo + i] + C - 1) / C) : 0;
+        const uint32_t *pl = c.piece_len + (size_t)rel * P * MAX_RANKS;
+        uint32_t *pc = c.piece_chunk + (size_t)rel * P * (MAX_RANKS + 1);
+        for (int i = tid; i <= np; i += blockDim.x) {
+            uint32_t t = 0;
+            if (i < np)
+                for (int g = 0; g < MAX_RANKS; ++g) {
+                    pc[(size_t)i * (MAX_RANKS + 1) + g] = t;
+                    t += (uint32_t)((pl[(size_t)i * MAX_RANKS + g] + C - 1) / C);
+                }
+            if (i < np) pc[(size_t)i * (MAX_RANKS + 1) + MAX_RANKS] = t;
+            chn[i] = t;
+        }
         __syncthreads();
         nch[rel] = block_excl_scan_u32(chn, np + 1, tmp32);
         for (int i = tid; i <= np; i += blockDim.x) c.chunk_base[rel * (P + 1) + i] = chn[i];

@@ -58,11 +58,15 @@ __global__ void k_chunkmap(Ctx c, ChunkDesc *desc) {
             const int mid = (lo + hi + 1) >> 1;
             if (__ldg(cb + mid) <= li) lo = mid; else hi = mid - 1;
         }
-        const uint64_t k = li - cb[lo];
-        const int p = plo + lo;
+        const uint32_t j = li - cb[lo];
+        const uint32_t *pc = c.piece_chunk + ((size_t)rel * P + lo) * (MAX_RANKS + 1);
+        int g = 0;
+        while (g + 1 < MAX_RANKS && pc[g + 1] <= j) ++g;  // piece holding chunk j of partition lo
+        const uint64_t k = j - pc[g];
+        const size_t pidx = ((size_t)rel * P + lo) * MAX_RANKS + g;
         ChunkDesc d;
-        d.start = c.seg_start[rel * P + p] + k * C;
-        d.len = (uint32_t)min(C, c.seg_len[rel * P + p] - k * C);
+        d.start = c.piece_start[pidx] + k * C;
+        d.len = (uint32_t)min(C, (uint64_t)c.piece_len[pidx] - k * C);
         d.pi = (uint32_t)lo;
         desc[ci] = d;
     }

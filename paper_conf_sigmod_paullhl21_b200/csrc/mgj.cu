@@ -40,8 +40,9 @@ int ceil_log2(uint64_t x) {
 mgj_status normalize(const mgj_config *in, Norm *o) {
     if (!in) return MGJ_EINVAL;
     mgj_config c = *in;
-    for (int i = 0; i < 8; ++i)
+    for (int i = 0; i < 7; ++i)
         if (c.reserved[i]) return MGJ_EINVAL;
+    if (c.shuffle_mode != MGJ_SHUFFLE_P2P && c.shuffle_mode != MGJ_SHUFFLE_EXTERNAL) return MGJ_EINVAL;
     if (c.world_size < 1 || c.world_size > MAX_RANKS || c.rank < 0 || c.rank >= c.world_size) return MGJ_EINVAL;
     if (!((c.key_bytes == 4 && c.payload_bytes == 4) || (c.key_bytes == 8 && c.payload_bytes == 8)))
         return MGJ_EINVAL;
@@ -114,6 +115,7 @@ struct mgj_plan_s {
     int nalloc = 0;
     Ctx ctx{};
     ChunkDesc *cdesc = nullptr;
+    char *send_arena = nullptr;  // EXTERNAL shuffle
     uint64_t epoch = 0;
     int state = 0;
     cudaStream_t stream = nullptr;
@@ -187,13 +189,16 @@ void launch_shuffle(mgj_plan_s *h, cudaStream_t s) {
     k_plan<<<1, 1024, plan_smem(n), s>>>(h->ctx);
     k_chunkmap<<<h->nsm * 2, 256, 0, s>>>(h->ctx, h->cdesc);
     cudaEventRecord(h->ev[2], s);
-    k_scatter<K><<<h->ctx.G, SCATTER_THREADS, scatter_smem(n), s>>>(h->ctx);
+    Ctx cs = h->ctx;
+    if (cs.ext)
+        for (int g = 0; g < MAX_RANKS; ++g) cs.arena[g] = h->send_arena;
+    k_scatter<K><<<h->ctx.G, SCATTER_THREADS, scatter_smem(n), s>>>(cs);
 }
 
 template <typename K>
 void launch_join(mgj_plan_s *h, cudaStream_t s) {
     const Norm &n = h->n;
-    k_wait<<<1, 32, 0, s>>>(h->ctx, SIG_DATA);
+    if (!h->ctx.ext) k_wait<<<1, 32, 0, s>>>(h->ctx, SIG_DATA);  // EXTERNAL: the caller's exchange is stream-ordered
     k_local<K><<<h->nsm, LOCAL_THREADS, local_smem(n), s>>>(h->ctx, h->cdesc);
     cudaEventRecord(h->ev[4], s);
     k_itemize<K><<<h->nsm * 4, 256, 0, s>>>(h->ctx);
@@ -286,6 +291,7 @@ mgj_status mgj_plan(const mgj_config *cfg, const mgj_peers *peers, mgj_handle *o
     c.probe_slots = n.probe_slots;
     c.probe_target = n.probe_target;
     c.materialize = n.c.materialize;
+    c.ext = n.c.shuffle_mode == MGJ_SHUFFLE_EXTERNAL;
     c.max_items = (uint32_t)n.max_items;
     c.recv_cap[0] = n.recv_cap[0];
     c.recv_cap[1] = n.recv_cap[1];
@@ -309,6 +315,14 @@ mgj_status mgj_plan(const mgj_config *cfg, const mgj_peers *peers, mgj_handle *o
     c.seg_start = static_cast<uint64_t *>(dalloc(h, 2ull * P * 8, &st));
     c.seg_len = static_cast<uint64_t *>(dalloc(h, 2ull * P * 8, &st));
     c.recv_size = static_cast<uint64_t *>(dalloc(h, 2ull * MAX_RANKS * 8, &st));
+    c.piece_start = static_cast<uint64_t *>(dalloc(h, 2ull * P * MAX_RANKS * 8, &st));
+    c.piece_len = static_cast<uint32_t *>(dalloc(h, 2ull * P * MAX_RANKS * 4, &st));
+    c.piece_chunk = static_cast<uint32_t *>(dalloc(h, 2ull * P * (MAX_RANKS + 1) * 4, &st));
+    c.ext_counts = static_cast<uint64_t *>(dalloc(h, 2ull * 2 * MAX_RANKS * 8, &st));
+    // EXTERNAL shuffle: a send arena with the receive layout; the scatter is
+    // launched with every peer pointer aimed at it (tuples land ordered by
+    // destination rank, see k_plan)
+    if (c.ext) h->send_arena = static_cast<char *>(dalloc(h, n.lay.total, &st));
     c.chunk_base = static_cast<uint32_t *>(dalloc(h, 2ull * (P + 1) * 4, &st));
     for (int r = 0; r < 2; ++r)
         c.eoff[r] = static_cast<uint16_t *>(dalloc(h, n.max_chunks * (Qm + 1) * 2, &st));
@@ -461,6 +475,27 @@ mgj_status mgj_result(mgj_handle h, mgj_result_t *out) {
     out->n_items = (int32_t)std::min<uint64_t>(ni, h->n.max_items);
     h->state = ST_DONE;
     return (mgj_status)out->status;
+}
+
+mgj_status mgj_exchange_layout(mgj_handle h, mgj_exchange_t *out) {
+    if (!h || !out) return MGJ_EINVAL;
+    if (!h->ctx.ext) return MGJ_EINVAL;
+    if (h->state != ST_SHUFFLED) return MGJ_ESTATE;
+    if (cudaStreamSynchronize(h->stream) != cudaSuccess) return MGJ_ECUDA;
+    memset(out, 0, sizeof(*out));
+    uint64_t cnt[2 * 2 * MAX_RANKS];
+    if (cudaMemcpy(cnt, h->ctx.ext_counts, sizeof(cnt), cudaMemcpyDeviceToHost) != cudaSuccess) return MGJ_ECUDA;
+    for (int rel = 0; rel < 2; ++rel) {
+        out->send[rel] = h->send_arena + h->n.lay.recv[rel];
+        out->recv[rel] = h->arena[h->ctx.rank] + h->n.lay.recv[rel];
+        for (int g = 0; g < MAX_RANKS; ++g) {
+            out->send_count[rel][g] = g < h->ctx.world ? cnt[(0 * 2 + rel) * MAX_RANKS + g] : 0;
+            out->recv_count[rel][g] = g < h->ctx.world ? cnt[(1 * 2 + rel) * MAX_RANKS + g] : 0;
+        }
+    }
+    out->tuple_bytes = h->n.tuple_bytes;
+    out->world_size = h->ctx.world;
+    return MGJ_OK;
 }
 
 void mgj_destroy(mgj_handle h) {

@@ -46,7 +46,14 @@ class Config(ctypes.Structure):
                 ("recv_capacity_r", ctypes.c_uint64), ("recv_capacity_s", ctypes.c_uint64),
                 ("radix_bits_global", ctypes.c_int32), ("radix_bits_local", ctypes.c_int32),
                 ("materialize", ctypes.c_int32), ("num_sms", ctypes.c_int32),
-                ("out_capacity", ctypes.c_uint64), ("reserved", ctypes.c_int32 * 8)]
+                ("out_capacity", ctypes.c_uint64), ("shuffle_mode", ctypes.c_int32),
+                ("reserved", ctypes.c_int32 * 7)]
+
+
+class Exchange(ctypes.Structure):
+    _fields_ = [("send", ctypes.c_void_p * 2), ("recv", ctypes.c_void_p * 2),
+                ("send_count", (ctypes.c_uint64 * MAX_RANKS) * 2), ("recv_count", (ctypes.c_uint64 * MAX_RANKS) * 2),
+                ("tuple_bytes", ctypes.c_int32), ("world_size", ctypes.c_int32)]
 
 
 class Peers(ctypes.Structure):
@@ -89,11 +96,15 @@ _lib.mgj_plan_host.argtypes = [ctypes.c_int32, ctypes.c_int32, ctypes.c_int32, _
 _lib.mgj_gen_relation.restype = ctypes.c_int
 _lib.mgj_gen_relation.argtypes = [ctypes.c_int32, ctypes.c_int32, _U64, _U64, ctypes.c_double,
                                   _U64, _U64, _P, _P, _P]
+_lib.mgj_exchange_layout.restype = ctypes.c_int
+_lib.mgj_exchange_layout.argtypes = [_H, ctypes.POINTER(Exchange)]
 _lib.mgj_debug_copy.restype = ctypes.c_int
 _lib.mgj_debug_copy.argtypes = [_H, ctypes.c_int32, _P, _U64, ctypes.POINTER(_U64)]
 
 EXPORTED = ["mgj_arena_bytes", "mgj_plan", "mgj_partition", "mgj_shuffle", "mgj_join", "mgj_result",
-            "mgj_destroy", "mgj_strerror", "mgj_plan_host", "mgj_gen_relation", "mgj_debug_copy"]
+            "mgj_destroy", "mgj_strerror", "mgj_plan_host", "mgj_exchange_layout", "mgj_gen_relation",
+            "mgj_debug_copy"]
+SHUFFLE_P2P, SHUFFLE_EXTERNAL = 0, 1
 
 
 def _check(st: int, where: str):
@@ -119,7 +130,7 @@ def _stream(stream):
 
 def make_config(rank=0, world_size=1, key_bytes=4, r_capacity=0, s_capacity=0, recv_capacity_r=0,
                 recv_capacity_s=0, radix_bits_global=0, radix_bits_local=0, materialize=False,
-                num_sms=0, out_capacity=0) -> Config:
+                num_sms=0, out_capacity=0, shuffle_mode=0) -> Config:
     c = Config()
     c.rank, c.world_size = rank, world_size
     c.key_bytes = c.payload_bytes = key_bytes
@@ -129,6 +140,7 @@ def make_config(rank=0, world_size=1, key_bytes=4, r_capacity=0, s_capacity=0, r
     c.materialize = int(bool(materialize))
     c.num_sms = num_sms
     c.out_capacity = out_capacity
+    c.shuffle_mode = shuffle_mode
     return c
 
 
@@ -159,6 +171,16 @@ class Join:
 
     def shuffle(self, stream=None):
         _check(_lib.mgj_shuffle(self._h, _stream(stream)), "mgj_shuffle")
+
+    def exchange_layout(self) -> dict:
+        """EXTERNAL shuffle: buffers and per-rank tuple counts of the exchange (mgj_exchange_layout)."""
+        e = Exchange()
+        _check(_lib.mgj_exchange_layout(self._h, ctypes.byref(e)), "mgj_exchange_layout")
+        W = e.world_size
+        return {"send": [e.send[0], e.send[1]], "recv": [e.recv[0], e.recv[1]],
+                "send_count": [[int(e.send_count[r][g]) for g in range(W)] for r in range(2)],
+                "recv_count": [[int(e.recv_count[r][g]) for g in range(W)] for r in range(2)],
+                "tuple_bytes": int(e.tuple_bytes)}
 
     def join(self, stream=None):
         _check(_lib.mgj_join(self._h, _stream(stream)), "mgj_join")
@@ -207,6 +229,22 @@ class Join:
             self.close()
         except Exception:
             pass
+
+
+class _DevBuf:
+    """Byte view of a raw device pointer for torch.as_tensor (__cuda_array_interface__)."""
+
+    def __init__(self, ptr: int, nbytes: int):
+        self.__cuda_array_interface__ = {"shape": (nbytes,), "typestr": "|u1", "data": (ptr, False),
+                                         "version": 3}
+
+
+def device_bytes(ptr: int, nbytes: int):
+    """torch uint8 tensor aliasing device memory [ptr, ptr + nbytes)."""
+    import torch
+    if nbytes == 0:
+        return torch.empty(0, dtype=torch.uint8, device="cuda")
+    return torch.as_tensor(_DevBuf(ptr, nbytes), device="cuda")
 
 
 def plan_host(world: int, rank: int, bits: int, hist: np.ndarray):

@@ -358,3 +358,51 @@ def test_m2_full_size_closed_form(mgj):
     hist = j.debug("RANK_HIST", np.uint32).reshape(2, -1)
     assert int(hist[0].sum()) == n and int(hist[1].sum()) == n
     j.close()
+
+
+# ------------------------------------------------------------ EXTERNAL (NCCL-baseline) shuffle
+@pytest.mark.parametrize("N,kind", [(1, "unique"), (2, "unique"), (4, "unique"), (3, "zipf"), (2, "wide")])
+def test_external_shuffle_virtual_ranks(mgj, N, kind):
+    """shuffle_mode EXTERNAL: the library packs per-destination send buffers, the
+    caller's all-to-all (emulated here with device copies, as NCCL
+    all_to_all_single would do) fills the receive areas, mgj_join finishes."""
+    w = {"unique": datagen.M1(), "zipf": datagen.Workload("zipf", 1 << 16, 1 << 18, 1.0),
+         "wide": datagen.Workload("wide", 1 << 17, 1 << 17)}[kind]
+    parts = [w.rank_inputs(g, N) for g in range(N)]
+    cap_r = max(p["r_keys"].size for p in parts)
+    cap_s = max(p["s_keys"].size for p in parts)
+    cfgs = [mgj.make_config(rank=g, world_size=N, key_bytes=w.key_bytes, r_capacity=cap_r, s_capacity=cap_s,
+                            recv_capacity_r=w.n_r, recv_capacity_s=w.n_s, shuffle_mode=mgj.SHUFFLE_EXTERNAL)
+            for g in range(N)]
+    nb = mgj.arena_bytes(cfgs[0])
+    arenas = [torch.zeros(nb, dtype=torch.uint8, device="cuda") for _ in range(N)]
+    ptrs = [a.data_ptr() for a in arenas]
+    joins = [mgj.Join(cfgs[g], ptrs, nb) for g in range(N)]
+    tens = [[dev(p[k]) for k in ("r_keys", "r_pays", "s_keys", "s_pays")] for p in parts]
+    for g in range(N):
+        joins[g].partition(*tens[g])
+    for g in range(N):
+        joins[g].shuffle()
+    lays = [j.exchange_layout() for j in joins]
+    tb = lays[0]["tuple_bytes"]
+    for rel in range(2):
+        assert sum(sum(l["send_count"][rel]) for l in lays) == (w.n_r if rel == 0 else w.n_s)
+        for g in range(N):
+            so = 0
+            for d in range(N):
+                cnt = lays[g]["send_count"][rel][d]
+                assert lays[d]["recv_count"][rel][g] == cnt
+                ro = sum(lays[d]["recv_count"][rel][:g])
+                mgj.device_bytes(lays[d]["recv"][rel] + ro * tb, cnt * tb).copy_(
+                    mgj.device_bytes(lays[g]["send"][rel] + so * tb, cnt * tb))
+                so += cnt
+    torch.cuda.synchronize()
+    for g in range(N):
+        joins[g].join()
+    res = [joins[g].result() for g in range(N)]
+    d = w.rank_inputs()
+    ref = oracle.join(d["r_keys"], d["r_pays"], d["s_keys"], d["s_pays"])
+    for r in res:
+        assert (r["match_count"], r["checksum"]) == (ref["count"], ref["checksum"])
+    for j in joins:
+        j.close()

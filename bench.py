@@ -50,6 +50,8 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--profile", action="store_true", help="short run for ncu (no clocks/cpu/e2e)")
+    ap.add_argument("--shuffle", default="p2p", choices=["p2p", "nccl"],
+                    help="p2p: in-kernel peer stores (product); nccl: NCCL all_to_all_single baseline")
     return ap.parse_args()
 
 
@@ -203,6 +205,7 @@ def main():
     # N>1: one rank per GPU over NCCL with symmetric-memory arenas.  MGJ_SYMM_ARENA=1 forces the
     # same symmetric-memory path at N=1 (under torchrun) to exercise it on a single GPU.
     distributed = world > 1 or os.environ.get("MGJ_SYMM_ARENA") == "1"
+    assert a.shuffle == "p2p" or distributed, "--shuffle nccl needs torchrun (or MGJ_SYMM_ARENA=1)"
     if distributed:
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     dev = torch.device("cuda", local)
@@ -229,7 +232,8 @@ def main():
                           materialize=a.materialize, radix_bits_global=a.radix_bits_global,
                           radix_bits_local=a.radix_bits_local,
                           recv_capacity_r=(n_r if world > 1 and a.workload == "zipf" else 0),
-                          recv_capacity_s=(n_s // 2 if world > 1 and a.workload == "zipf" else 0))
+                          recv_capacity_s=(n_s // 2 if world > 1 and a.workload == "zipf" else 0),
+                          shuffle_mode=(mgj.SHUFFLE_EXTERNAL if a.shuffle == "nccl" else mgj.SHUFFLE_P2P))
     arena = None
     if distributed:
         import torch.distributed._symmetric_memory as symm_mem
@@ -244,9 +248,22 @@ def main():
     else:
         join = mgj.Join(cfg)
 
-    def step():
-        join.partition(*cols, stream=stream)
+    def nccl_exchange():
+        """Baseline shuffle: NCCL all_to_all_single of the per-destination send buffers."""
+        lay = join.exchange_layout()  # synchronises the stream (sizes are computed on the device)
+        tb_ = lay["tuple_bytes"]
+        with torch.cuda.stream(stream):
+            for rel in range(2):
+                sc, rc = lay["send_count"][rel], lay["recv_count"][rel]
+                send = mgj.device_bytes(lay["send"][rel], sum(sc) * tb_)
+                recv = mgj.device_bytes(lay["recv"][rel], sum(rc) * tb_)
+                dist.all_to_all_single(recv, send, [x * tb_ for x in rc], [x * tb_ for x in sc])
+
+    def step(inputs=None):
+        join.partition(*(cols if inputs is None else inputs), stream=stream)
         join.shuffle(stream)
+        if a.shuffle == "nccl":
+            nccl_exchange()
         join.join(stream)
 
     def barrier():
@@ -348,13 +365,12 @@ def main():
             h.copy_(c)
         hnp = [h.numpy() for h in host]
         barrier()
-        join.run(*hnp, stream=stream)
+        step(hnp)
+        join.result()
         barrier()
         t0 = time.perf_counter()
         for _ in range(a.e2e_steps):
-            join.partition(*hnp, stream=stream)
-            join.shuffle(stream)
-            join.join(stream)
+            step(hnp)
             r2 = join.result()
         t_e2e = time.perf_counter() - t0
         if world > 1:
@@ -384,6 +400,8 @@ def main():
                        "tuples_R": n_r, "tuples_S": n_s, "tuple_bytes": tb, "materialize": a.materialize,
                        "radix_bits_global": res["radix_bits_global"], "radix_bits_local": res["radix_bits_local"],
                        "l2": "inputs (8 GiB/GPU) larger than L2; no flush", "parallelism": f"dp{world}",
+                       "shuffle": ("in-kernel peer stores (symmetric memory)" if a.shuffle == "p2p"
+                                   else "NCCL all_to_all_single baseline (host sync per step for split sizes)"),
                        "global_batch": tuples_job, "seeds": {"R": "0x5EED0052", "S": "0x5EED0053"}},
             "correct": bool(expect_ok) and res["status"] == 0,
             "match_count": res["match_count"], "checksum": hex(res["checksum"]),

@@ -140,8 +140,10 @@ mgj_status mgj_partition(mgj_handle h,
  * Phases a2 + a3 (§4): waits for every rank's histogram, computes
  * the partition->GPU assignment (contiguous balanced owner ranges) and the
  * exact receive offsets, then scatters every tuple straight into its owner's
- * receive buffer (peer stores over NVLink/NVSwitch through shared-memory
- * write-combining lines) and raises a data-done flag at every peer.
+ * receive buffer (peer stores over NVLink/NVSwitch of shared-memory-sorted
+ * sub-tiles, whole 32-byte sectors) and raises a data-done flag at every
+ * peer.  With MGJ_SHUFFLE_EXTERNAL the tuples go to a send buffer ordered by
+ * destination instead (see mgj_exchange_layout).
  */
 mgj_status mgj_shuffle(mgj_handle h, void *stream);
 

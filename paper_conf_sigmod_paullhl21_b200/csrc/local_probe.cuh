@@ -353,7 +353,7 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
     extern __shared__ __align__(128) unsigned char smem[];
     __shared__ __align__(8) uint64_t full[PROBE_NST], empty[PROBE_NST];
     __shared__ uint32_t totals[PROBE_NST][2];
-    __shared__ uint32_t s_m;
+    __shared__ uint32_t s_wtot[32];
     __shared__ unsigned long long s_base;
     __shared__ int s_write;
     if (!c.meta[MT_OK]) return;
@@ -488,52 +488,49 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
         }
         my_cnt += m_item;
         if (MAT) {
-            if (ct == 0) s_m = 0;
+            // exact output positions: exclusive scan of the per-thread match
+            // counts of the pass above, one reservation per item, then each
+            // thread re-walks the same S slots and writes its matches in order
+            const int cwi = ct >> 5;
+            uint32_t incl = m_item;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const uint32_t y = __shfl_up_sync(0xffffffffu, incl, o);
+                if (lane >= o) incl += y;
+            }
+            if (lane == 31) s_wtot[cwi] = incl;
             named_bar_sync(1, NCONS);
-            const uint32_t wm = (uint32_t)warp_sum(m_item);
-            if (lane == 0 && wm) atomicAdd(&s_m, wm);
-            named_bar_sync(1, NCONS);
-            if (ct == 0) {
-                const uint32_t M = s_m;
-                s_base = M ? atomicAdd(&c.acc[2], (unsigned long long)M) : 0;
-                s_write = M && (s_base + M <= c.out_cap);
-                if (M && !s_write) set_err(c, MGJ_ECAPACITY);
-                s_m = 0;  // reused as the write cursor
+            if (ct < 32) {
+                uint32_t v = ct < NCONS / 32 ? s_wtot[ct] : 0;
+#pragma unroll
+                for (int o = 1; o < 32; o <<= 1) {
+                    const uint32_t y = __shfl_up_sync(0xffffffffu, v, o);
+                    if (ct >= o) v += y;
+                }
+                if (ct < NCONS / 32) s_wtot[ct] = v;
+                if (ct == 31) {
+                    s_base = v ? atomicAdd(&c.acc[2], (unsigned long long)v) : 0;
+                    s_write = v && (s_base + v <= c.out_cap);
+                    if (v && !s_write) set_err(c, MGJ_ECAPACITY);
+                }
             }
             named_bar_sync(1, NCONS);
-            if (s_write) {
+            if (s_write && m_item) {
                 K *ok = static_cast<K *>(c.out_key);
                 K *oa = static_cast<K *>(c.out_a);
                 K *ob = static_cast<K *>(c.out_b);
-                const unsigned long long obase = s_base;
-                const uint32_t sround = (stot + 31) & ~31u;
-                for (uint32_t x = ct; x < sround; x += NCONS) {  // warp-uniform trip count
-                    Tup sv;
-                    uint32_t i = END;
-                    if (x < stot && !(Layout<K>::ALIGN == 2 && ((pb[x >> 5] >> (x & 31)) & 1u))) {
-                        sv = st[x];
-                        const uint32_t hv = head[tab_hash(sv.x, shift, LOGT)];
-                        i = (hv >> 16) == tag ? (hv & 0xffffu) : END;
-                    }
-                    while (__any_sync(0xffffffffu, i != END)) {
-                        bool hit = false;
-                        Tup rv;
-                        if (i != END) {
-                            rv = rt[i];
-                            hit = rv.x == sv.x;
-                            i = nxt[i];
-                        }
-                        const uint32_t bal = __ballot_sync(0xffffffffu, hit);
-                        if (bal) {
-                            uint32_t wb = 0;
-                            if (lane == 0) wb = atomicAdd(&s_m, (uint32_t)__popc(bal));
-                            wb = __shfl_sync(0xffffffffu, wb, 0);
-                            if (hit) {
-                                const unsigned long long pos = obase + wb + __popc(bal & ((1u << lane) - 1u));
-                                ok[pos] = (K)sv.x;
-                                oa[pos] = (K)rv.y;
-                                ob[pos] = (K)sv.y;
-                            }
+                unsigned long long pos = s_base + (cwi ? s_wtot[cwi - 1] : 0) + incl - m_item;
+                for (uint32_t x = ct; x < stot; x += NCONS) {
+                    if (Layout<K>::ALIGN == 2 && ((pb[x >> 5] >> (x & 31)) & 1u)) continue;
+                    const Tup sv = st[x];
+                    const uint32_t hv = head[tab_hash(sv.x, shift, LOGT)];
+                    for (uint32_t i = (hv >> 16) == tag ? (hv & 0xffffu) : END; i != END; i = nxt[i]) {
+                        const Tup rv = rt[i];
+                        if (rv.x == sv.x) {
+                            ok[pos] = (K)sv.x;
+                            oa[pos] = (K)rv.y;
+                            ob[pos] = (K)sv.y;
+                            ++pos;
                         }
                     }
                 }

@@ -139,6 +139,8 @@ def test_phases_m1(mgj, b1):
                     valid = slots - (e0 & 1)
                     run = loc[li * CR + st: li * CR + st + valid]
                     assert np.all(((run[:, 0] >> B1) & (Q - 1)) == q)
+                    if valid < slots:  # padding slot: a key of the run with bit 0 flipped
+                        assert (loc[li * CR + st + valid, 0] ^ 1) in run[:, 0]
                     got.append(run)
                 got = np.concatenate(got)
                 src = recv[a:b, 0].astype(np.uint64) | (recv[a:b, 1].astype(np.uint64) << np.uint64(32))

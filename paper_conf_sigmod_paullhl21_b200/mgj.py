@@ -13,7 +13,7 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libmgj.so")
+LIB_PATH = os.environ.get("MGJ_LIB") or os.path.join(_HERE, "libmgj.so")  # MGJ_LIB: A/B experiments only
 
 if not os.path.exists(LIB_PATH):
     raise ImportError(f"libmgj.so not built ({LIB_PATH}); run `python -c 'import __graft_entry__ as g; g.build()'`")

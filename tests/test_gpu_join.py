@@ -362,6 +362,94 @@ def test_m2_full_size_closed_form(mgj):
     j.close()
 
 
+def _check_materialized_full(mgj, j, res, w: "datagen.Workload", n_sample=1 << 16):
+    """Full-size materialised output, unique-key workloads: every R row and
+    every S row appears exactly once (payload columns are permutations of the
+    row ids, checked on the device), and sampled triples (k, a, b) satisfy
+    R.key(row a) == k == S.key(row b) (rows recomputed by the generator)."""
+    n = res["n_materialized"]
+    kb = w.key_bytes
+    dt = torch.int32 if kb == 4 else torch.int64
+    col = lambda ptr: mgj.device_bytes(ptr, n * kb).view(dt)
+    key, pa, pb = col(res["out_key"]), col(res["out_payload_r"]), col(res["out_payload_s"])
+    base_r, base_s = (0, 0) if w.kind == "unique" else (1 << 40, 1 << 41)
+    for c, base in ((pa, base_r), (pb, base_s)):
+        srt = torch.sort(c - base).values
+        assert bool((srt == torch.arange(n, device="cuda", dtype=dt)).all())
+        del srt
+    g = torch.Generator(device="cuda").manual_seed(5)
+    idx = torch.randint(0, n, (n_sample,), device="cuda", generator=g)
+    k = key[idx].cpu().numpy().view(np.uint32 if kb == 4 else np.uint64)
+    a = (pa[idx] - base_r).cpu().numpy().astype(np.uint64)
+    b = (pb[idx] - base_s).cpu().numpy().astype(np.uint64)
+    mk = lambda rel, rows, nn: (datagen.perm_n(rows, nn, datagen.SEED_R if rel == "R" else datagen.SEED_S)
+                                if w.kind == "unique" else
+                                datagen.mix64(datagen.perm_n(rows, nn, datagen.SEED_R if rel == "R" else datagen.SEED_S)))
+    np.testing.assert_array_equal(mk("R", a, w.n_r).astype(k.dtype), k)
+    np.testing.assert_array_equal(mk("S", b, w.n_s).astype(k.dtype), k)
+
+
+@pytest.mark.slow
+def test_m2_full_size_materialized(mgj):
+    """M2 (2^29 x 2^29) with materialisation: closed forms + output properties."""
+    n = 1 << 29
+    w = datagen.M2()
+    cols = [torch.empty(n, dtype=torch.int32, device="cuda") for _ in range(4)]
+    mgj.gen_relation("unique", 0, n, n, 0.0, 0, n, cols[0], cols[1])
+    mgj.gen_relation("unique", 1, n, n, 0.0, 0, n, cols[2], cols[3])
+    j = mgj.Join(mgj.make_config(r_capacity=n, s_capacity=n, materialize=True, out_capacity=n))
+    res = j.run(*cols)
+    assert res["match_count"] == n and res["n_materialized"] == n
+    assert res["checksum"] == 0xf1fffffff0000000
+    del cols
+    _check_materialized_full(mgj, j, res, w)
+    j.close()
+
+
+@pytest.mark.slow
+def test_m5_full_size_wide_materialized(mgj):
+    """M5 per GPU (2^28 x 2^28 wide 8+8-byte tuples, full materialisation):
+    closed-form count and checksum (C = 0x9E3779B97F4A7C15) + output properties."""
+    n = 1 << 28
+    w = datagen.Workload("wide", n, n)
+    cols = [torch.empty(n, dtype=torch.int64, device="cuda") for _ in range(4)]
+    mgj.gen_relation("wide", 0, n, n, 0.0, 0, n, cols[0], cols[1])
+    mgj.gen_relation("wide", 1, n, n, 0.0, 0, n, cols[2], cols[3])
+    j = mgj.Join(mgj.make_config(key_bytes=8, r_capacity=n, s_capacity=n, materialize=True, out_capacity=n))
+    res = j.run(*cols)
+    h = n * (n - 1) // 2
+    assert res["match_count"] == n and res["n_materialized"] == n
+    assert res["checksum"] == (0x9E3779B97F4A7C15 * (n * (1 << 40) + h) + n * (1 << 41) + h) & M64
+    del cols
+    _check_materialized_full(mgj, j, res, w)
+    j.close()
+
+
+@pytest.mark.slow
+def test_m4_full_size_zipf(mgj):
+    """M4 per GPU (|R| = 2^27 unique, |S| = 2^29 Zipf z = 1, 50% selectivity):
+    every even S row matches R row r_j exactly once, odd rows never, so
+    count = |S|/2 and checksum = sum over even j of (r_j * 2^32 + j).  r_j is
+    found with plain torch indexing: R's keys are a permutation of [0, |R|),
+    inverted on the device (inv[R.key[r]] = r, r_j = inv[S.key[j]])."""
+    n_r, n_s, z = 1 << 27, 1 << 29, 1.0
+    cols = [torch.empty(x, dtype=torch.int32, device="cuda") for x in (n_r, n_r, n_s, n_s)]
+    mgj.gen_relation("zipf", 0, n_r, n_s, z, 0, n_r, cols[0], cols[1])
+    mgj.gen_relation("zipf", 1, n_r, n_s, z, 0, n_s, cols[2], cols[3])
+    j = mgj.Join(mgj.make_config(r_capacity=n_r, s_capacity=n_s))
+    res = j.run(*cols)
+    assert res["match_count"] == n_s // 2
+    inv = torch.full((n_r,), -1, dtype=torch.int64, device="cuda")
+    inv[cols[0].long()] = torch.arange(n_r, device="cuda")
+    assert bool((inv >= 0).all())  # R keys are a permutation of [0, n_r)
+    sk = cols[2][0::2].long()
+    assert bool((sk < n_r).all()) and bool((cols[2][1::2].long() >= n_r).all())
+    rank_sum = int(inv[sk].sum())
+    m = n_s // 2
+    assert res["checksum"] == ((rank_sum << 32) + m * (m - 1)) & M64
+    j.close()
+
+
 # ------------------------------------------------------------ EXTERNAL (NCCL-baseline) shuffle
 @pytest.mark.parametrize("N,kind", [(1, "unique"), (2, "unique"), (4, "unique"), (3, "zipf"), (2, "wide")])
 def test_external_shuffle_virtual_ranks(mgj, N, kind):

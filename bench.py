@@ -39,11 +39,15 @@ def parse():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="mgj", choices=["mgj", "reference"])
     ap.add_argument("--log2-per-gpu", type=int, default=29, help="tuples per relation per GPU (M2: 29)")
+    ap.add_argument("--scaling", default="weak", choices=["weak", "strong"],
+                    help="weak: 2^log2-per-gpu per GPU (M2); strong: 2^log2-total per relation over all GPUs (M3)")
+    ap.add_argument("--log2-total", type=int, default=31, help="strong scaling: tuples per relation in total (M3: 31)")
     ap.add_argument("--workload", default="unique", choices=["unique", "wide", "zipf"])
     ap.add_argument("--z", type=float, default=1.0)
     ap.add_argument("--materialize", action="store_true")
     ap.add_argument("--radix-bits-global", type=int, default=0)
     ap.add_argument("--radix-bits-local", type=int, default=0)
+    ap.add_argument("--local-split-bits", type=int, default=0, help="a4 first pass: 0 auto, -1 never, k forced")
     ap.add_argument("--cpu-sample-log2", type=int, default=28,
                     help="oracle sample: 2^k R + 2^k S unique tuples (cpu_baseline / --impl reference)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -53,6 +57,15 @@ def parse():
     ap.add_argument("--shuffle", default="p2p", choices=["p2p", "nccl"],
                     help="p2p: in-kernel peer stores (product); nccl: NCCL all_to_all_single baseline")
     return ap.parse_args()
+
+
+def workload_name(a) -> str:
+    if a.scaling == "strong":
+        return f"M3 ({a.workload}, 2^{a.log2_total} R + 2^{a.log2_total} S in total over all GPUs)"
+    if a.workload == "zipf":
+        return f"M4-like zipf z={a.z} (2^{a.log2_per_gpu - 2} R + 2^{a.log2_per_gpu} S per GPU)"
+    return {"unique": "M2", "wide": "M5"}[a.workload] + \
+        f" ({a.workload}, 2^{a.log2_per_gpu} R + 2^{a.log2_per_gpu} S per GPU)"
 
 
 def dist_env():
@@ -215,7 +228,10 @@ def main():
     kb = 8 if wide else 4
     dt = torch.int64 if wide else torch.int32
     per = 1 << a.log2_per_gpu
-    if a.workload == "zipf":
+    if a.scaling == "strong":  # M3: the job size is fixed, each GPU holds 1/N of it
+        n_tot = 1 << a.log2_total
+        n_r, n_s = (n_tot // 4, n_tot) if a.workload == "zipf" else (n_tot, n_tot)
+    elif a.workload == "zipf":
         n_r, n_s = world * per // 4, world * per  # |R|:|S| = 1:4
     else:
         n_r = n_s = world * per
@@ -230,7 +246,7 @@ def main():
 
     cfg = mgj.make_config(rank=rank, world_size=world, key_bytes=kb, r_capacity=nr, s_capacity=ns,
                           materialize=a.materialize, radix_bits_global=a.radix_bits_global,
-                          radix_bits_local=a.radix_bits_local,
+                          radix_bits_local=a.radix_bits_local, local_split_bits=a.local_split_bits,
                           recv_capacity_r=(n_r if world > 1 and a.workload == "zipf" else 0),
                           recv_capacity_s=(n_s // 2 if world > 1 and a.workload == "zipf" else 0),
                           shuffle_mode=(mgj.SHUFFLE_EXTERNAL if a.shuffle == "nccl" else mgj.SHUFFLE_P2P))
@@ -392,11 +408,9 @@ def main():
     if rank == 0:
         line = {
             "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": a.steps,
-            "warmup": a.warmup, "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "weak",
+            "warmup": a.warmup, "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": a.scaling,
             "vs_baseline": None, "dtype": "u32" if kb == 4 else "u64", "data": "synthetic",
-            "config": {"workload": {"unique": "M2", "wide": "M5", "zipf": "M4"}[a.workload] +
-                       f" ({a.workload}, 2^{a.log2_per_gpu} R + 2^{a.log2_per_gpu} S per GPU)"
-                       if a.workload != "zipf" else f"M4-like zipf z={a.z}",
+            "config": {"workload": workload_name(a),
                        "tuples_R": n_r, "tuples_S": n_s, "tuple_bytes": tb, "materialize": a.materialize,
                        "radix_bits_global": res["radix_bits_global"], "radix_bits_local": res["radix_bits_local"],
                        "l2": "inputs (8 GiB/GPU) larger than L2; no flush", "parallelism": f"dp{world}",

@@ -70,7 +70,10 @@ typedef struct {
     int32_t  num_sms;                  /* 0 = device attribute */
     uint64_t out_capacity;             /* max materialised triples on this rank (0 = auto) */
     int32_t  shuffle_mode;             /* MGJ_SHUFFLE_P2P (0, default) | MGJ_SHUFFLE_EXTERNAL (1) */
-    int32_t  reserved[7];              /* must be zero */
+    int32_t  local_split_bits;         /* a4 first (histogram) pass: 0 = auto (only for owned partitions
+                                          of more than 256 chunks), -1 = never, 1..6 = always, 2^k
+                                          sub-partitions per owned partition */
+    int32_t  reserved[6];              /* must be zero */
 } mgj_config;
 
 /*

@@ -25,13 +25,23 @@ constexpr int PROBE_NST = 3;            // pipeline stages (items in flight per 
 constexpr int PROBE_SLOTS8 = 4224;      // stage capacity per relation (slots) for 8-byte tuples; half for 16-byte
 constexpr int PROBE_HEAD8 = 128;        // headroom: co-partition target = capacity - headroom (padding, spread)
 constexpr int PROBE_MAXP = 1024;        // chunk pieces per relation per item
+constexpr int MAX_BA = 6;               // two-level local partitioning: at most 2^6 sub-partitions per pass A
+constexpr int LOCAL2_NCH = 256;         // a partition of more chunks than this gets the first local pass
+// sub-partitions of a first local pass: at most local2_vcap(P) in total
+__host__ __device__ constexpr int local2_vcap(int P) { return 4 * P > 4096 ? 4 * P : 4096; }
 constexpr uint64_t WAIT_TIMEOUT_NS = 20ull * 1000 * 1000 * 1000;
 
 enum Sig { SIG_HIST = 0, SIG_DATA = 1, SIG_RES = 2, SIG_COUNT = 3 };
 enum Ticket { TK_HIST = 0, TK_SCAT_R = 1, TK_SCAT_S = 2, TK_SCAT_DONE = 3, TK_ITEMS = 4,
               TK_PROBE = 5, TK_LOCAL = 6, TK_COUNT = 8 };
 enum Meta { MT_PLO = 0, MT_PHI = 1, MT_B2 = 2, MT_OK = 3, MT_NCH_R = 4, MT_NCH_S = 5,
-            MT_NITEMS = 6, MT_CHUNK = 7, MT_COUNT = 16 };
+            MT_NITEMS = 6, MT_CHUNK = 7,
+            MT_BA = 8,       // bits of the first local pass (0: single local pass)
+            MT_QB = 9,       // bits of the (last) chunked local pass: B2 - BA
+            MT_NLP = 10,     // partitions of the chunked local pass: owned partitions, or sub-partitions
+            MT_NCHB_R = 11,  // chunks of the chunked pass after a first pass (R, S)
+            MT_NCHB_S = 12,
+            MT_COUNT = 16 };
 
 // Arena layout (bytes from each rank's arena base; identical on all ranks).
 struct Arena {
@@ -69,6 +79,10 @@ struct Ctx {
     uint64_t recv_cap[2];
     uint64_t max_chunks;
     uint64_t out_cap;
+    uint64_t mid_cap;             // slots of each first-pass output buffer
+    int32_t vcap;                 // local2_vcap(P)
+    int32_t cb_stride;            // entries per relation of chunk_base, vstart (vcap + 1)
+    int32_t split_cfg;            // mgj_config.local_split_bits
     Arena lay;
     char *arena[MAX_RANKS];       // arena bases as mapped in this process
     const void *in_key[2];
@@ -89,7 +103,11 @@ struct Ctx {
     uint32_t *piece_len;          // [2][P][MAX_RANKS]
     uint32_t *piece_chunk;        // [2][P][MAX_RANKS+1] chunk prefix over the pieces of pi
     uint64_t *ext_counts;         // [2 (send, recv)][2 rel][MAX_RANKS] (EXTERNAL shuffle)
-    uint32_t *chunk_base;         // [2][P+1]
+    uint32_t *chunk_base;         // [2][cb_stride] first chunk of each (sub-)partition of the chunked pass
+    uint32_t *hA;                 // [2][vcap] first local pass: padded slots per sub-partition
+    uint64_t *vstart;             // [2][vcap+1] sub-partition start (slots) in mid
+    unsigned long long *vcur;     // [2][vcap+1] write cursor of each sub-partition
+    void *mid[2];                 // first local pass output (sub-partitions, contiguous)
     uint16_t *eoff[2];            // run offsets, [(Q+1)*chunk_base[p] + q*nch_p + k]
     uint32_t *cop_slots;          // [2][P][2^b2_max] padded slots per co-partition
     Item *items;                  // [max_items]

@@ -165,10 +165,12 @@ __global__ void __launch_bounds__(1024) k_plan(Ctx c) {
     __shared__ int first[MAX_RANKS], endp[MAX_RANKS];
     __shared__ int ok, cap_bad;
     __shared__ unsigned long long maxr;
+    __shared__ uint32_t maxnch;
     if (tid == 0) {
         ok = wait_all_flags(c, SIG_HIST);
         cap_bad = 0;
         maxr = 0;
+        maxnch = 0;
     }
     if (tid < MAX_RANKS) first[tid] = endp[tid] = P;
     __syncthreads();
@@ -295,12 +297,15 @@ __global__ void __launch_bounds__(1024) k_plan(Ctx c) {
                     pc[(size_t)i * (MAX_RANKS + 1) + g] = t;
                     t += (uint32_t)((pl[(size_t)i * MAX_RANKS + g] + C - 1) / C);
                 }
-            if (i < np) pc[(size_t)i * (MAX_RANKS + 1) + MAX_RANKS] = t;
+            if (i < np) {
+                pc[(size_t)i * (MAX_RANKS + 1) + MAX_RANKS] = t;
+                atomicMax(&maxnch, t);
+            }
             chn[i] = t;
         }
         __syncthreads();
         nch[rel] = block_excl_scan_u32(chn, np + 1, tmp32);
-        for (int i = tid; i <= np; i += blockDim.x) c.chunk_base[rel * (P + 1) + i] = chn[i];
+        for (int i = tid; i <= np; i += blockDim.x) c.chunk_base[(size_t)rel * c.cb_stride + i] = chn[i];
         __syncthreads();
     }
     if (tid == 0) {
@@ -312,6 +317,23 @@ __global__ void __launch_bounds__(1024) k_plan(Ctx c) {
         c.meta[MT_NCH_R] = (int)nch[0];
         c.meta[MT_NCH_S] = (int)nch[1];
         c.meta[MT_CHUNK] = c.chunk_tuples;
+        // two-level local partitioning: when an owned partition
+        // spans more than LOCAL2_NCH chunks, a first histogram-based pass
+        // splits every owned partition into 2^BA contiguous sub-partitions of
+        // ~48 chunks, and the chunked pass then uses the remaining B2 - BA bits
+        int BA = 0;
+        if (c.split_cfg > 0) {
+            BA = c.split_cfg;
+        } else if (c.split_cfg == 0 && maxnch > (uint32_t)LOCAL2_NCH) {
+            BA = ceil_log2_u64((maxnch + 47) / 48);
+            while (BA > 0 && (np << BA) > c.vcap) --BA;
+        }
+        if (BA > B2) BA = B2;
+        if (BA > MAX_BA) BA = MAX_BA;
+        if (!c.mid[0] || (np << BA) > c.vcap) BA = 0;
+        c.meta[MT_BA] = BA;
+        c.meta[MT_QB] = B2 - BA;
+        c.meta[MT_NLP] = np;
         c.meta[MT_OK] = (cap_bad || !fits) ? 0 : 1;
     }
 }

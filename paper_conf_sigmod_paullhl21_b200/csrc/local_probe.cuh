@@ -52,7 +52,7 @@ __global__ void k_chunkmap(Ctx c, ChunkDesc *desc) {
     for (uint32_t ci = blockIdx.x * blockDim.x + threadIdx.x; ci < total; ci += gridDim.x * blockDim.x) {
         const int rel = ci < nch_r ? 0 : 1;
         const uint32_t li = rel ? ci - nch_r : ci;
-        const uint32_t *cb = c.chunk_base + rel * (P + 1);
+        const uint32_t *cb = c.chunk_base + (size_t)rel * c.cb_stride;
         int lo = 0, hi = np - 1;
         while (lo < hi) {
             const int mid = (lo + hi + 1) >> 1;
@@ -73,22 +73,160 @@ __global__ void k_chunkmap(Ctx c, ChunkDesc *desc) {
 }
 
 // ---------------------------------------------------------------------------
+// Two-level local partitioning (multi-pass a4).
+// One chunked pass writes one run per (chunk, sub-partition), so an owned
+// partition of nch chunks leaves each co-partition in nch runs of ~C/Q
+// tuples.  At N = 8 (M2) an owner's partitions are 8x larger than at N = 1
+// and the runs shrink to a dozen tuples, which the probe cannot fetch
+// efficiently.  Then (k_plan sets BA > 0) a first pass splits every owned
+// partition by the BA key bits above B1 into 2^BA contiguous sub-partitions
+// (k_countA: padded sizes; k_planA: extents; k_local<K, true>: the chunked
+// sort with one bulk store per run at a reserved offset), and the chunked
+// pass runs on the sub-partitions with the remaining B2 - BA bits.
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ uint32_t nch_local(const Ctx &c, int rel) {
+    return (uint32_t)c.meta[c.meta[MT_BA] ? MT_NCHB_R + rel : MT_NCH_R + rel];
+}
+
+// Padded size (slots) of every (owned partition, first-pass digit) run, summed
+// over the chunks of the partition: exactly the slots k_local<K, true> reserves.
+template <typename K>
+__global__ void __launch_bounds__(512) k_countA(Ctx c, const ChunkDesc *cdesc) {
+    using Tup = typename Layout<K>::Tup;
+    constexpr int ALIGN = Layout<K>::ALIGN;
+    __shared__ uint32_t cnt[16][1 << MAX_BA];  // per warp
+    if (!c.meta[MT_OK] || !c.meta[MT_BA]) return;
+    const int BA = c.meta[MT_BA], QA = 1 << BA;
+    const uint32_t nch_r = (uint32_t)c.meta[MT_NCH_R], total = nch_r + (uint32_t)c.meta[MT_NCH_S];
+    const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+    const char *recv0 = c.arena[c.rank];
+    for (uint32_t ci = blockIdx.x; ci < total; ci += gridDim.x) {
+        const int rel = ci < nch_r ? 0 : 1;
+        const ChunkDesc d = cdesc[ci];
+        const Tup *src = reinterpret_cast<const Tup *>(recv0 + c.lay.recv[rel]) + d.start;
+        for (int i = tid; i < 16 * QA; i += blockDim.x) cnt[i / QA][i % QA] = 0;
+        __syncthreads();
+        for (uint32_t i0 = 0; i0 < d.len; i0 += blockDim.x * 4) {
+            uint32_t q[4];
+#pragma unroll
+            for (int u = 0; u < 4; ++u) {
+                const uint32_t i = i0 + u * blockDim.x + tid;
+                q[u] = i < d.len ? digit2(__ldcs(&src[i].x), c.B1, QA) : 0xffffffffu;
+            }
+#pragma unroll
+            for (int u = 0; u < 4; ++u) {  // warp-aggregated: one shared atomic per distinct digit
+                const uint32_t peers = __match_any_sync(0xffffffffu, q[u]);
+                if (q[u] != 0xffffffffu && lane == __ffs(peers) - 1) atomicAdd(&cnt[w][q[u]], __popc(peers));
+            }
+        }
+        __syncthreads();
+        for (int qa = tid; qa < QA; qa += blockDim.x) {
+            uint32_t n = 0;
+            for (int x = 0; x < (int)(blockDim.x >> 5); ++x) n += cnt[x][qa];
+            if (n) atomicAdd(&c.hA[(size_t)rel * c.vcap + ((size_t)d.pi << BA) + qa],
+                             (n + ALIGN - 1) & ~(uint32_t)(ALIGN - 1));
+        }
+        __syncthreads();
+    }
+}
+
+// Extents of the sub-partitions in mid (exclusive scan of the padded sizes)
+// and the chunk table of the chunked pass over them.  One CTA.
+__global__ void __launch_bounds__(1024) k_planA(Ctx c) {
+    extern __shared__ uint64_t sv[];  // [L+1] then u32 [L+1]
+    __shared__ uint64_t tmp[33];
+    __shared__ uint32_t tmp32[33];
+    if (!c.meta[MT_OK] || !c.meta[MT_BA]) return;
+    const int BA = c.meta[MT_BA];
+    const int L = (c.meta[MT_PHI] - c.meta[MT_PLO]) << BA;
+    const int tid = threadIdx.x;
+    uint32_t *nch = reinterpret_cast<uint32_t *>(sv + L + 1);
+    const uint64_t C = (uint64_t)c.chunk_tuples;
+    uint32_t tot_ch[2];
+    bool bad = false;
+    for (int rel = 0; rel < 2; ++rel) {
+        const uint32_t *h = c.hA + (size_t)rel * c.vcap;
+        for (int v = tid; v <= L; v += blockDim.x) {
+            const uint32_t n = v < L ? h[v] : 0;
+            sv[v] = n;
+            nch[v] = (uint32_t)((n + C - 1) / C);
+        }
+        __syncthreads();
+        const uint64_t slots = block_excl_scan_u64(sv, L + 1, tmp);
+        tot_ch[rel] = block_excl_scan_u32(nch, L + 1, tmp32);
+        uint64_t *vs = c.vstart + (size_t)rel * c.cb_stride;
+        for (int v = tid; v <= L; v += blockDim.x) {
+            vs[v] = sv[v];
+            if (v < L) c.vcur[(size_t)rel * c.cb_stride + v] = sv[v];
+            c.chunk_base[(size_t)rel * c.cb_stride + v] = nch[v];
+        }
+        bad |= slots > c.mid_cap || tot_ch[rel] > c.max_chunks;
+        __syncthreads();
+    }
+    if (tid == 0) {
+        c.meta[MT_NCHB_R] = (int)tot_ch[0];
+        c.meta[MT_NCHB_S] = (int)tot_ch[1];
+        c.meta[MT_NLP] = L;
+        if (bad) {
+            set_err(c, MGJ_ECAPACITY);
+            c.meta[MT_OK] = 0;
+        }
+    }
+}
+
+// Chunk descriptors of the chunked pass over the sub-partitions (one piece each).
+__global__ void k_chunkmapB(Ctx c, ChunkDesc *desc) {
+    if (!c.meta[MT_OK] || !c.meta[MT_BA]) return;
+    const int L = c.meta[MT_NLP];
+    const uint32_t nch_r = (uint32_t)c.meta[MT_NCHB_R], total = nch_r + (uint32_t)c.meta[MT_NCHB_S];
+    const uint64_t C = (uint64_t)c.chunk_tuples;
+    for (uint32_t ci = blockIdx.x * blockDim.x + threadIdx.x; ci < total; ci += gridDim.x * blockDim.x) {
+        const int rel = ci < nch_r ? 0 : 1;
+        const uint32_t li = rel ? ci - nch_r : ci;
+        const uint32_t *cb = c.chunk_base + (size_t)rel * c.cb_stride;
+        int lo = 0, hi = L - 1;
+        while (lo < hi) {
+            const int mid = (lo + hi + 1) >> 1;
+            if (__ldg(cb + mid) <= li) lo = mid; else hi = mid - 1;
+        }
+        const uint64_t k = li - cb[lo];
+        const uint64_t *vs = c.vstart + (size_t)rel * c.cb_stride;
+        ChunkDesc d;
+        d.start = vs[lo] + k * C;
+        d.len = (uint32_t)min(C, vs[lo + 1] - vs[lo] - k * C);
+        d.pi = (uint32_t)lo;
+        desc[ci] = d;
+    }
+}
+
+// ---------------------------------------------------------------------------
 // a4 (§3.2 "Local partitioning"): the received data of
 // each owned global partition p is partitioned again by the next B2 key bits
 // so that every R co-partition fits a shared-memory hash table.
 // B200 form: a persistent CTA per SM streams chunks of C received tuples in
 // by TMA (double-buffered, two chunks ahead), counting-sorts each chunk by
-// digit2 in shared memory (one SMEM atomic per tuple gives bin count and
-// rank), and streams the sorted chunk out with one TMA bulk store.  Runs are
-// padded to 16 bytes so the probe can fetch them with bulk copies; the run
-// offsets go to E[(Q+1)*chunk_base[p] + q*nch_p + k], i.e. contiguous per
-// (p, q).  No global histogram is needed and a chunk can be processed as soon
-// as it has arrived — the property the paper takes [44] for.
-// One pass suffices for every configured size; R co-partitions
-// larger than the table are built in pieces by a5 (P:450-452's skew case).
+// its digit in shared memory (one SMEM atomic per tuple gives bin count and
+// rank), and streams the sorted chunk out by TMA bulk store.  Runs are
+// padded to 16 bytes so the probe can fetch them with bulk copies.  No global
+// histogram is needed and a chunk can be processed as soon as it has arrived
+// — the property the paper takes [44] for.
+//  MODE = LM_SINGLE (the only pass, BA = 0) / LM_SECOND (after a first
+//    pass): the chunked pass.  digit = the B2 - BA key bits above B1 + BA,
+//    one bulk store per chunk, run offsets to E[(Q+1)*chunk_base[v] +
+//    q*nch_v + k] (contiguous per (v, q)).  LM_SECOND reads the
+//    sub-partitions and drops the first pass's padding tuples (digit1 != p).
+//  MODE = LM_SPLIT (first pass of two-level partitioning): digit = the BA
+//    bits above B1; every run is stored by its own bulk copy at an offset
+//    reserved in its sub-partition's extent (k_planA).
+// Each instance returns at once when the run's BA does not select it.
+// R co-partitions larger than the table are built in pieces by a5
+// (P:450-452's skew case).
 // ---------------------------------------------------------------------------
-template <typename K>
+enum LocalMode { LM_SINGLE = 0, LM_SPLIT = 1, LM_SECOND = 2 };
+
+template <typename K, int MODE>
 __global__ void __launch_bounds__(LOCAL_THREADS, 1) k_local(Ctx c, const ChunkDesc *cdesc) {
+    constexpr bool SPLIT = MODE == LM_SPLIT;
     using Tup = typename Layout<K>::Tup;
     constexpr int TB = Layout<K>::TB, ALIGN = Layout<K>::ALIGN;
     constexpr int VMAX = local_vmax(TB);
@@ -97,19 +235,25 @@ __global__ void __launch_bounds__(LOCAL_THREADS, 1) k_local(Ctx c, const ChunkDe
     __shared__ ChunkDesc sdesc[2];
     __shared__ uint32_t tmp[33];
     if (!c.meta[MT_OK]) return;
+    const int BA = MODE == LM_SINGLE ? 0 : c.meta[MT_BA];
+    if ((MODE == LM_SINGLE) != (c.meta[MT_BA] == 0)) return;
     const int tid = threadIdx.x;
     const int C = c.chunk_tuples, CR = c.chunk_region, V = C / LOCAL_THREADS;
-    const int P = c.P, B2 = c.meta[MT_B2], Q = 1 << B2;
+    const int P = c.P, Q = 1 << (SPLIT ? BA : c.meta[MT_QB]);
+    const int shift = SPLIT ? c.B1 : c.B1 + BA;  // digit = (key >> shift) & (Q - 1)
     const int Qmax = 1 << c.b2_max;
     const int BUF = C + Qmax + 2;  // slots per buffer
+    const int plo = c.meta[MT_PLO];
     Tup *const buf0 = reinterpret_cast<Tup *>(smem);
     auto buf = [&](int x) { return buf0 + (size_t)x * BUF; };
     uint32_t *bins = reinterpret_cast<uint32_t *>(buf0 + (size_t)2 * BUF);
     uint32_t *abin = bins + Qmax;
-    const uint32_t nch_r = (uint32_t)c.meta[MT_NCH_R];
-    const uint32_t total = nch_r + (uint32_t)c.meta[MT_NCH_S];
+    const uint32_t nch_r = SPLIT ? (uint32_t)c.meta[MT_NCH_R] : nch_local(c, 0);
+    const uint32_t total = nch_r + (SPLIT ? (uint32_t)c.meta[MT_NCH_S] : nch_local(c, 1));
     const uint32_t mine = total > blockIdx.x ? (total - blockIdx.x + gridDim.x - 1) / gridDim.x : 0;
-    const char *recv0 = c.arena[c.rank];
+    constexpr bool from_mid = MODE == LM_SECOND;
+    const char *const srcR = from_mid ? static_cast<const char *>(c.mid[0]) : c.arena[c.rank] + c.lay.recv[0];
+    const char *const srcS = from_mid ? static_cast<const char *>(c.mid[1]) : c.arena[c.rank] + c.lay.recv[1];
     if (tid == 0) {
         mbar_init(&bar[0], 1);
         mbar_init(&bar[1], 1);
@@ -127,8 +271,7 @@ __global__ void __launch_bounds__(LOCAL_THREADS, 1) k_local(Ctx c, const ChunkDe
         sdesc[j & 1] = d;
         uint64_t *b = &bar[j & 1];
         mbar_arrive_expect_tx(b, bytes);
-        if (bytes)
-            tma_load_1d(buf(j & 1), reinterpret_cast<const Tup *>(recv0 + c.lay.recv[rel]) + g0, bytes, b, pol);
+        if (bytes) tma_load_1d(buf(j & 1), reinterpret_cast<const Tup *>(rel ? srcS : srcR) + g0, bytes, b, pol);
     };
     ChunkDesc nxt{};
     if (tid == 0) {
@@ -143,6 +286,8 @@ __global__ void __launch_bounds__(LOCAL_THREADS, 1) k_local(Ctx c, const ChunkDe
         mbar_wait(&bar[X], (j >> 1) & 1);
         const ChunkDesc d = sdesc[X];
         const uint32_t len = d.len, skip = (uint32_t)(d.start & (ALIGN - 1));
+        // partition of this chunk's tuples (a first pass's padding tuples lie in another one)
+        const uint32_t p = (uint32_t)plo + (from_mid ? d.pi >> BA : d.pi);
         Tup t[VMAX];
 #pragma unroll
         for (int v = 0; v < VMAX; ++v) {
@@ -150,18 +295,20 @@ __global__ void __launch_bounds__(LOCAL_THREADS, 1) k_local(Ctx c, const ChunkDe
             if (v < V && i < len) t[v] = buf(X)[skip + i];
         }
         for (int q = tid; q < Q; q += LOCAL_THREADS) bins[q] = 0;
+        if (SPLIT && tid < Q) bulk_wait_read0();  // run stores of chunk j-1 have read buffer X^1
         __syncthreads();  // S1: buffer X consumed (it becomes this chunk's sorted output)
         if (tid == 0 && j + 1 < mine) {
-            bulk_wait_read0();  // chunk j-1's bulk store has finished reading buffer X^1
+            if (!SPLIT) bulk_wait_read0();  // chunk j-1's bulk store has finished reading buffer X^1
             issue(j + 1, nxt);
             if (j + 2 < mine) nxt = cdesc[blockIdx.x + (j + 2) * gridDim.x];
         }
-        uint32_t rq[VMAX];  // rank << 16 | digit2
+        uint32_t rq[VMAX];  // rank << 16 | digit (0xffffffff: dropped)
 #pragma unroll
         for (int v = 0; v < VMAX; ++v) {
             const uint32_t i = tid + v * LOCAL_THREADS;
-            if (v < V && i < len) {
-                const uint32_t q = digit2(t[v].x, c.B1, Q);
+            rq[v] = 0xffffffffu;
+            if (v < V && i < len && (!from_mid || digit1(t[v].x, P) == p)) {
+                const uint32_t q = digit2(t[v].x, shift, Q);
                 rq[v] = (atomicAdd(&bins[q], 1u) << 16) | q;
             }
         }
@@ -169,11 +316,11 @@ __global__ void __launch_bounds__(LOCAL_THREADS, 1) k_local(Ctx c, const ChunkDe
         for (int q = tid; q < Q; q += LOCAL_THREADS) abin[q] = (bins[q] + ALIGN - 1) & ~(uint32_t)(ALIGN - 1);
         __syncthreads();
         const uint32_t tot = block_excl_scan_u32(abin, Q, tmp);
-        {
-            const uint32_t *cb = c.chunk_base + rel * (P + 1);
+        if (!SPLIT) {
+            const uint32_t *cb = c.chunk_base + (size_t)rel * c.cb_stride;
             const uint32_t cbp = cb[d.pi], nchp = cb[d.pi + 1] - cbp;
             uint16_t *E = c.eoff[rel] + (size_t)(Q + 1) * cbp + (li - cbp);
-            uint32_t *cop = c.cop_slots + ((size_t)rel * P + d.pi) * Q;
+            uint32_t *cop = c.cop_slots + (size_t)rel * P * Qmax + (size_t)d.pi * Q;
             for (int q = tid; q <= Q; q += LOCAL_THREADS) {
                 if (q < Q) {
                     const uint32_t n = bins[q];
@@ -187,14 +334,14 @@ __global__ void __launch_bounds__(LOCAL_THREADS, 1) k_local(Ctx c, const ChunkDe
         Tup *const sorted = buf(X);
 #pragma unroll
         for (int v = 0; v < VMAX; ++v) {
-            const uint32_t i = tid + v * LOCAL_THREADS;
-            if (v < V && i < len) {
+            if (rq[v] != 0xffffffffu) {
                 const uint32_t q = rq[v] & 0xffffu, r = rq[v] >> 16;
                 sorted[abin[q] + r] = t[v];
                 // 16-byte padding slot of an odd run: a tuple whose key has its
                 // lowest bit flipped, i.e. lies in another global partition, so
                 // it never equals a real key of this co-partition; the probe
-                // skips S padding slots (bitmap), R padding is inert (DESIGN.md §2 R2)
+                // skips S padding slots (bitmap), R padding is inert, and the
+                // chunked pass drops a first pass's padding (DESIGN.md §2 R2)
                 if (ALIGN == 2 && r == 0 && (bins[q] & 1u)) {
                     Tup pad = t[v];
                     pad.x ^= 1;
@@ -204,13 +351,21 @@ __global__ void __launch_bounds__(LOCAL_THREADS, 1) k_local(Ctx c, const ChunkDe
         }
         fence_proxy_async_smem();
         __syncthreads();  // S3
-        if (tid == 0 && tot) {
+        if (SPLIT) {
+            if (tid < Q && bins[tid]) {  // one bulk store per run, at a reserved offset of its sub-partition
+                const uint32_t slots = (bins[tid] + ALIGN - 1) & ~(uint32_t)(ALIGN - 1);
+                const unsigned long long at =
+                    atomicAdd(&c.vcur[(size_t)rel * c.cb_stride + ((size_t)d.pi << BA) + tid], slots);
+                tma_store_1d(static_cast<Tup *>(c.mid[rel]) + at, sorted + abin[tid], slots * TB);
+                bulk_commit();
+            }
+        } else if (tid == 0 && tot) {
             Tup *dst = static_cast<Tup *>(c.local[rel]) + (size_t)li * CR;
             tma_store_1d(dst, sorted, tot * TB);
             bulk_commit();
         }
     }
-    if (tid == 0) bulk_wait0();
+    bulk_wait0();
 }
 
 // ---------------------------------------------------------------------------
@@ -263,22 +418,22 @@ template <typename K>
 __global__ void k_itemize(Ctx c) {
     constexpr int ALIGN = Layout<K>::ALIGN;
     if (!c.meta[MT_OK]) return;
-    const int P = c.P, plo = c.meta[MT_PLO], phi = c.meta[MT_PHI];
-    const int Q = 1 << c.meta[MT_B2];
+    const int P = c.P, Qmax = 1 << c.b2_max;
+    const int Q = 1 << c.meta[MT_QB];  // sub-partitions of the chunked pass
     const uint32_t cap = (uint32_t)c.probe_slots;
     ItemX *items = reinterpret_cast<ItemX *>(c.items);
-    const uint64_t total = (uint64_t)(phi - plo) * Q;
+    const uint64_t total = (uint64_t)c.meta[MT_NLP] * Q;
     for (uint64_t idx = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; idx < total;
          idx += (uint64_t)gridDim.x * blockDim.x) {
         const uint32_t pi = (uint32_t)(idx / Q), q = (uint32_t)(idx % Q);
         const uint32_t r = c.cop_slots[(size_t)pi * Q + q];
-        const uint32_t s = c.cop_slots[((size_t)P + pi) * Q + q];
+        const uint32_t s = c.cop_slots[(size_t)P * Qmax + (size_t)pi * Q + q];
         if (r == 0 || s == 0) continue;
         ItemX x;
         x.it.pi = pi;
         x.it.q = q;
         for (int rel = 0; rel < 2; ++rel) {
-            const uint32_t *cb = c.chunk_base + rel * (P + 1);
+            const uint32_t *cb = c.chunk_base + (size_t)rel * c.cb_stride;
             x.cb[rel] = cb[pi];
             x.nch[rel] = cb[pi + 1] - cb[pi];
         }
@@ -365,7 +520,7 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
     uint16_t *nxt = reinterpret_cast<uint16_t *>(head + T);
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const int B2 = c.meta[MT_B2];
-    const int Q = 1 << B2, shift = c.B1 + B2;
+    const int Q = 1 << c.meta[MT_QB], shift = c.B1 + B2;  // Q: runs per chunk of the chunked pass
     const uint32_t nitems = min(__ldcg(&c.ticket[TK_ITEMS]), c.max_items);
     const uint32_t mine = nitems > blockIdx.x ? (nitems - blockIdx.x + gridDim.x - 1) / gridDim.x : 0;
     const ItemX *items = reinterpret_cast<const ItemX *>(c.items);

@@ -27,7 +27,8 @@ uint64_t align_up(uint64_t x, uint64_t a) { return (x + a - 1) / a * a; }
 struct Norm {  // validated config with the automatic fields filled in
     mgj_config c;
     int B1, P, b2_max, tuple_bytes, chunk_tuples, chunk_region, probe_slots, probe_target;
-    uint64_t recv_cap[2], max_chunks, max_items, out_cap;
+    uint64_t recv_cap[2], max_chunks, max_items, out_cap, mid_cap;
+    bool split;  // first local pass possible (mid buffers allocated)
     Arena lay;
 };
 
@@ -40,8 +41,9 @@ int ceil_log2(uint64_t x) {
 mgj_status normalize(const mgj_config *in, Norm *o) {
     if (!in) return MGJ_EINVAL;
     mgj_config c = *in;
-    for (int i = 0; i < 7; ++i)
+    for (int i = 0; i < 6; ++i)
         if (c.reserved[i]) return MGJ_EINVAL;
+    if (c.local_split_bits < -1 || c.local_split_bits > MAX_BA) return MGJ_EINVAL;
     if (c.shuffle_mode != MGJ_SHUFFLE_P2P && c.shuffle_mode != MGJ_SHUFFLE_EXTERNAL) return MGJ_EINVAL;
     if (c.world_size < 1 || c.world_size > MAX_RANKS || c.rank < 0 || c.rank >= c.world_size) return MGJ_EINVAL;
     if (!((c.key_bytes == 4 && c.payload_bytes == 4) || (c.key_bytes == 8 && c.payload_bytes == 8)))
@@ -80,7 +82,13 @@ mgj_status normalize(const mgj_config *in, Norm *o) {
     o->chunk_tuples = C;
     o->chunk_region = C + Qm;  // worst-case padding: one slot per run
     const uint64_t rmax = std::max(o->recv_cap[0], o->recv_cap[1]);
-    o->max_chunks = rmax / C + o->P + 2;
+    // chunks of the chunked pass: sum over (sub-)partitions of ceil(size / C); at most
+    // local2_vcap(P) sub-partitions after a first pass
+    o->max_chunks = rmax / C + (uint64_t)local2_vcap(o->P) + 2;
+    // the first local pass exists if forced, or (auto) if one owned partition could
+    // span more than LOCAL2_NCH chunks; its output pads each (chunk, run) once
+    o->split = c.local_split_bits > 0 || (c.local_split_bits == 0 && rmax > (uint64_t)LOCAL2_NCH * C);
+    o->mid_cap = o->split ? rmax + (rmax / C + o->P + 2) * (1ull << MAX_BA) : 0;
     o->max_items = (uint64_t)o->P * Qm + o->recv_cap[1] / (o->probe_slots / 2) * 2 +
                    o->recv_cap[0] / (o->probe_slots / 2) * 2 + 4096;
     if (o->max_items > 0x7fffffffull) o->max_items = 0x7fffffffull;
@@ -111,7 +119,7 @@ struct mgj_plan_s {
     char *arena[MAX_RANKS] = {};
     void *zero_block = nullptr;
     size_t zero_bytes = 0;
-    void *allocs[32] = {};
+    void *allocs[64] = {};
     int nalloc = 0;
     Ctx ctx{};
     ChunkDesc *cdesc = nullptr;
@@ -151,6 +159,7 @@ void *dalloc(mgj_plan_s *h, size_t bytes, mgj_status *st) {
 size_t hist_smem(const Norm &n) { return (size_t)n.P * 4; }
 size_t plan_smem(const Norm &n) { return (size_t)n.P * 5 * 8 + (size_t)n.P * 4 + (size_t)(n.P + 1) * 4; }
 size_t scatter_smem(const Norm &n) { return scat_smem_bytes(n.P, n.c.key_bytes); }
+size_t planA_smem(const Norm &n) { return ((size_t)local2_vcap(n.P) + 1) * 12; }
 size_t local_smem(const Norm &n) { return local_smem_bytes(n.chunk_tuples, 1 << n.b2_max, n.tuple_bytes); }
 size_t probe_smem(const Norm &n) { return probe_smem_bytes(n.probe_slots, n.tuple_bytes); }
 
@@ -161,7 +170,10 @@ cudaError_t set_attrs(const Norm &n) {
     if ((e = cudaFuncSetAttribute(k_hist<K>, A, (int)hist_smem(n)))) return e;
     if ((e = cudaFuncSetAttribute(k_plan, A, (int)plan_smem(n)))) return e;
     if ((e = cudaFuncSetAttribute(k_scatter<K>, A, (int)scatter_smem(n)))) return e;
-    if ((e = cudaFuncSetAttribute(k_local<K>, A, (int)local_smem(n)))) return e;
+    if ((e = cudaFuncSetAttribute(k_local<K, LM_SINGLE>, A, (int)local_smem(n)))) return e;
+    if ((e = cudaFuncSetAttribute(k_local<K, LM_SPLIT>, A, (int)local_smem(n)))) return e;
+    if ((e = cudaFuncSetAttribute(k_local<K, LM_SECOND>, A, (int)local_smem(n)))) return e;
+    if ((e = cudaFuncSetAttribute(k_planA, A, (int)planA_smem(n)))) return e;
     if ((e = cudaFuncSetAttribute(k_probe<K, false>, A, (int)probe_smem(n)))) return e;
     return cudaFuncSetAttribute(k_probe<K, true>, A, (int)probe_smem(n));
 }
@@ -199,7 +211,15 @@ template <typename K>
 void launch_join(mgj_plan_s *h, cudaStream_t s) {
     const Norm &n = h->n;
     if (!h->ctx.ext) k_wait<<<1, 32, 0, s>>>(h->ctx, SIG_DATA);  // EXTERNAL: the caller's exchange is stream-ordered
-    k_local<K><<<h->nsm, LOCAL_THREADS, local_smem(n), s>>>(h->ctx, h->cdesc);
+    // two-level local partitioning (device-side decision, MT_BA; no-ops otherwise)
+    if (n.split) {
+        k_countA<K><<<h->nsm * 4, 512, 0, s>>>(h->ctx, h->cdesc);
+        k_planA<<<1, 1024, planA_smem(n), s>>>(h->ctx);
+        k_local<K, LM_SPLIT><<<h->nsm, LOCAL_THREADS, local_smem(n), s>>>(h->ctx, h->cdesc);
+        k_chunkmapB<<<h->nsm * 2, 256, 0, s>>>(h->ctx, h->cdesc);
+        k_local<K, LM_SECOND><<<h->nsm, LOCAL_THREADS, local_smem(n), s>>>(h->ctx, h->cdesc);
+    }
+    k_local<K, LM_SINGLE><<<h->nsm, LOCAL_THREADS, local_smem(n), s>>>(h->ctx, h->cdesc);
     cudaEventRecord(h->ev[4], s);
     k_itemize<K><<<h->nsm * 4, 256, 0, s>>>(h->ctx);
     if (n.c.materialize)
@@ -275,6 +295,7 @@ mgj_status mgj_plan(const mgj_config *cfg, const mgj_peers *peers, mgj_handle *o
     const size_t z_err = zo; zo += 256;
     const size_t z_cop = zo; zo += align_up(2ull * P * Qm * 4, 256);
     const size_t z_th = zo; zo += align_up(2ull * h->nsm * P * 4, 256);
+    const size_t z_ha = zo; zo += align_up(2ull * local2_vcap(P) * 4, 256);
     h->zero_bytes = zo;
     char *zb = static_cast<char *>(dalloc(h, zo, &st));
     h->zero_block = zb;
@@ -307,6 +328,7 @@ mgj_status mgj_plan(const mgj_config *cfg, const mgj_peers *peers, mgj_handle *o
         c.err = reinterpret_cast<int32_t *>(zb + z_err);
         c.cop_slots = reinterpret_cast<uint32_t *>(zb + z_cop);
         c.tile_hist = reinterpret_cast<uint32_t *>(zb + z_th);
+        c.hA = reinterpret_cast<uint32_t *>(zb + z_ha);
     }
     c.tile_base = static_cast<uint32_t *>(dalloc(h, 2ull * c.G * P * 4, &st));
     h->cdesc = static_cast<ChunkDesc *>(dalloc(h, 2 * n.max_chunks * sizeof(ChunkDesc), &st));
@@ -323,7 +345,14 @@ mgj_status mgj_plan(const mgj_config *cfg, const mgj_peers *peers, mgj_handle *o
     // launched with every peer pointer aimed at it (tuples land ordered by
     // destination rank, see k_plan)
     if (c.ext) h->send_arena = static_cast<char *>(dalloc(h, n.lay.total, &st));
-    c.chunk_base = static_cast<uint32_t *>(dalloc(h, 2ull * (P + 1) * 4, &st));
+    c.vcap = local2_vcap(P);
+    c.cb_stride = c.vcap + 1;
+    c.split_cfg = n.c.local_split_bits;
+    c.mid_cap = n.mid_cap;
+    c.chunk_base = static_cast<uint32_t *>(dalloc(h, 2ull * c.cb_stride * 4, &st));
+    c.vstart = static_cast<uint64_t *>(dalloc(h, 2ull * c.cb_stride * 8, &st));
+    c.vcur = static_cast<unsigned long long *>(dalloc(h, 2ull * c.cb_stride * 8, &st));
+    for (int r = 0; r < 2 && n.split; ++r) c.mid[r] = dalloc(h, n.mid_cap * n.tuple_bytes, &st);
     for (int r = 0; r < 2; ++r)
         c.eoff[r] = static_cast<uint16_t *>(dalloc(h, n.max_chunks * (Qm + 1) * 2, &st));
     c.items = static_cast<Item *>(dalloc(h, n.max_items * sizeof(ItemX), &st));
@@ -596,7 +625,9 @@ mgj_status mgj_debug_copy(mgj_handle h, int32_t what, void *dst, uint64_t bytes,
     if (cudaMemcpy(meta, c.meta, sizeof(meta), cudaMemcpyDeviceToHost) != cudaSuccess) return MGJ_ECUDA;
     uint64_t rs[2 * MAX_RANKS];
     if (cudaMemcpy(rs, c.recv_size, sizeof(rs), cudaMemcpyDeviceToHost) != cudaSuccess) return MGJ_ECUDA;
-    const int Q = 1 << meta[MT_B2];
+    const int Q = 1 << meta[MT_QB];  // runs per chunk of the chunked pass
+    const uint64_t nchl[2] = {(uint64_t)(uint32_t)meta[meta[MT_BA] ? MT_NCHB_R : MT_NCH_R],
+                              (uint64_t)(uint32_t)meta[meta[MT_BA] ? MT_NCHB_S : MT_NCH_S]};
     const void *src = nullptr;
     uint64_t size = 0;
     switch (what) {
@@ -612,16 +643,29 @@ mgj_status mgj_debug_copy(mgj_handle h, int32_t what, void *dst, uint64_t bytes,
             break;
         case MGJ_DBG_LOCAL_R:
             src = c.local[0];
-            size = (uint64_t)(uint32_t)meta[MT_NCH_R] * n.chunk_region * n.tuple_bytes;
+            size = nchl[0] * n.chunk_region * n.tuple_bytes;
             break;
         case MGJ_DBG_LOCAL_S:
             src = c.local[1];
-            size = (uint64_t)(uint32_t)meta[MT_NCH_S] * n.chunk_region * n.tuple_bytes;
+            size = nchl[1] * n.chunk_region * n.tuple_bytes;
             break;
         case MGJ_DBG_META: src = c.meta; size = sizeof(meta); break;
-        case MGJ_DBG_CHUNK_OFF_R: src = c.eoff[0]; size = (uint64_t)(uint32_t)meta[MT_NCH_R] * (Q + 1) * 2; break;
-        case MGJ_DBG_CHUNK_OFF_S: src = c.eoff[1]; size = (uint64_t)(uint32_t)meta[MT_NCH_S] * (Q + 1) * 2; break;
-        case MGJ_DBG_CHUNK_BASE: src = c.chunk_base; size = 2ull * (P + 1) * 4; break;
+        case MGJ_DBG_CHUNK_OFF_R: src = c.eoff[0]; size = nchl[0] * (Q + 1) * 2; break;
+        case MGJ_DBG_CHUNK_OFF_S: src = c.eoff[1]; size = nchl[1] * (Q + 1) * 2; break;
+        case MGJ_DBG_CHUNK_BASE: src = c.chunk_base; size = 2ull * c.cb_stride * 4; break;
+        case MGJ_DBG_MID_R:
+        case MGJ_DBG_MID_S: {
+            if (!meta[MT_BA]) return MGJ_EINVAL;
+            const int r = what == MGJ_DBG_MID_S;
+            const int L = meta[MT_NLP];
+            uint64_t end = 0;
+            if (cudaMemcpy(&end, c.vstart + (size_t)r * c.cb_stride + L, 8, cudaMemcpyDeviceToHost) != cudaSuccess)
+                return MGJ_ECUDA;
+            src = c.mid[r];
+            size = end * n.tuple_bytes;
+            break;
+        }
+        case MGJ_DBG_VSTART: src = c.vstart; size = 2ull * c.cb_stride * 8; break;
         case MGJ_DBG_OUT_KEY:
         case MGJ_DBG_OUT_PAY_R:
         case MGJ_DBG_OUT_PAY_S: {

@@ -27,7 +27,7 @@ MAX_RANKS = 8
 # mgj_debug_what
 DBG = dict(RANK_HIST=1, MAIL_HIST=2, OWNER=3, SEND_OFF=4, RECV_SIZE=5, RECV_R=6, RECV_S=7,
            LOCAL_R=8, LOCAL_S=9, META=10, CHUNK_OFF_R=11, CHUNK_OFF_S=12, CHUNK_BASE=13, SEGMENTS=14,
-           OUT_KEY=15, OUT_PAY_R=16, OUT_PAY_S=17)
+           OUT_KEY=15, OUT_PAY_R=16, OUT_PAY_S=17, MID_R=18, MID_S=19, VSTART=20)
 GEN_KIND = {"unique": 0, "zipf": 1, "wide": 2}
 
 
@@ -47,7 +47,7 @@ class Config(ctypes.Structure):
                 ("radix_bits_global", ctypes.c_int32), ("radix_bits_local", ctypes.c_int32),
                 ("materialize", ctypes.c_int32), ("num_sms", ctypes.c_int32),
                 ("out_capacity", ctypes.c_uint64), ("shuffle_mode", ctypes.c_int32),
-                ("reserved", ctypes.c_int32 * 7)]
+                ("local_split_bits", ctypes.c_int32), ("reserved", ctypes.c_int32 * 6)]
 
 
 class Exchange(ctypes.Structure):
@@ -130,7 +130,7 @@ def _stream(stream):
 
 def make_config(rank=0, world_size=1, key_bytes=4, r_capacity=0, s_capacity=0, recv_capacity_r=0,
                 recv_capacity_s=0, radix_bits_global=0, radix_bits_local=0, materialize=False,
-                num_sms=0, out_capacity=0, shuffle_mode=0) -> Config:
+                num_sms=0, out_capacity=0, shuffle_mode=0, local_split_bits=0) -> Config:
     c = Config()
     c.rank, c.world_size = rank, world_size
     c.key_bytes = c.payload_bytes = key_bytes
@@ -141,6 +141,7 @@ def make_config(rank=0, world_size=1, key_bytes=4, r_capacity=0, s_capacity=0, r
     c.num_sms = num_sms
     c.out_capacity = out_capacity
     c.shuffle_mode = shuffle_mode
+    c.local_split_bits = local_split_bits
     return c
 
 

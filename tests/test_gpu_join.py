@@ -156,6 +156,60 @@ def test_m1_parity_materialized(mgj):
     assert res["checksum"] == 0xfff8007ffff80000
 
 
+# ------------------------------------------------------------ two-level local partitioning
+@pytest.mark.parametrize("ba", [1, 3, 6])
+def test_two_level_local_phases(mgj, ba):
+    """Forced first local pass (BA bits) on M1 with B1 = 4 (16 partitions of
+    2^16): every sub-partition v = (p, qa) of MID holds exactly the received
+    tuples of p whose next BA key bits are qa, plus padding tuples of another
+    global partition (at most one per chunk run); the join stays exact."""
+    d = datagen.M1().rank_inputs()
+    ref = oracle.join(d["r_keys"], d["r_pays"], d["s_keys"], d["s_pays"], materialize=False)
+    j, res = run_one(mgj, d, radix_bits_global=4, local_split_bits=ba)
+    assert (res["match_count"], res["checksum"]) == (ref["count"], ref["checksum"])
+    meta = j.debug("META", np.int32)
+    B1, P = 4, 16
+    BA, QB, L = int(meta[8]), int(meta[9]), int(meta[10])
+    assert BA == min(ba, res["radix_bits_local"]) and QB == res["radix_bits_local"] - BA and L == P << BA
+    vstart = j.debug("VSTART", np.uint64).reshape(2, -1)
+    for rel, name in ((0, "R"), (1, "S")):
+        recv = j.debug("RECV_" + name, np.uint32).reshape(-1, 2)
+        mid = j.debug("MID_" + name, np.uint32).reshape(-1, 2)
+        assert mid.shape[0] == int(vstart[rel, L])
+        for v in range(L):
+            p, qa = v >> BA, v & ((1 << BA) - 1)
+            seg = mid[int(vstart[rel, v]):int(vstart[rel, v + 1])]
+            real = seg[(seg[:, 0] & (P - 1)) == p]
+            pads = seg[(seg[:, 0] & (P - 1)) != p]
+            assert np.all(((real[:, 0] >> B1) & ((1 << BA) - 1)) == qa)
+            assert np.all((pads[:, 0] & (P - 1)) == (p ^ 1))
+            exp = recv[((recv[:, 0] & (P - 1)) == p) & (((recv[:, 0] >> B1) & ((1 << BA) - 1)) == qa)]
+            pack = lambda x: np.sort(x[:, 0].astype(np.uint64) | (x[:, 1].astype(np.uint64) << np.uint64(32)))
+            np.testing.assert_array_equal(pack(real), pack(exp))
+    j.close()
+
+
+@pytest.mark.parametrize("ba", [2, 5])
+@pytest.mark.parametrize("kind", ["unique_dup", "zipf", "wide", "edge"])
+def test_two_level_local_parity(mgj, ba, kind):
+    """Forced two-level local partitioning vs the oracle (materialised)."""
+    rng = np.random.default_rng(99)
+    if kind == "zipf":
+        d = datagen.Workload("zipf", 1 << 16, 1 << 19, 1.0).rank_inputs()
+    elif kind == "wide":
+        d = datagen.Workload("wide", 1 << 18, 1 << 18).rank_inputs()
+    elif kind == "edge":
+        ks = np.array([0, 1, 2, 3, 0xFFFFFFFF, 0xFFFFFFFE, 0x80000000, 0x7FFFFFFF], np.uint32)
+        d = dict(r_keys=np.repeat(ks, 3), r_pays=np.arange(24, dtype=np.uint32),
+                 s_keys=np.tile(ks, 5), s_pays=np.arange(40, dtype=np.uint32) + 100)
+    else:
+        d = dict(r_keys=rng.integers(0, 1 << 17, 400003, dtype=np.uint32),
+                 r_pays=rng.integers(0, 1 << 32, 400003, dtype=np.uint32),
+                 s_keys=rng.integers(0, 1 << 17, 500009, dtype=np.uint32),
+                 s_pays=rng.integers(0, 1 << 32, 500009, dtype=np.uint32))
+    check_vs_oracle(mgj, d, materialize=True, radix_bits_global=3, local_split_bits=ba)
+
+
 @pytest.mark.parametrize("b1,b2", [(1, 0), (4, 3), (8, 0), (11, 2), (12, 5)])
 def test_radix_bit_variants(mgj, b1, b2):
     d = datagen.Workload("unique", 300007, 300007).rank_inputs()
@@ -291,6 +345,19 @@ def test_virtual_ranks_m1(mgj, N):
         assert res[g]["recv_r"] == recv_size[0, g] and res[g]["recv_s"] == recv_size[1, g]
         recv = j.debug("RECV_R", np.uint32).reshape(-1, 2)
         assert np.all(owner[recv[:, 0] & (P - 1)] == g)
+    for j in joins:
+        j.close()
+
+
+@pytest.mark.parametrize("N,ba", [(2, 2), (4, 3), (8, 1)])
+def test_virtual_ranks_two_level(mgj, N, ba):
+    """N ranks with the first local pass forced on every rank (B1 = 4)."""
+    w = datagen.M1()
+    joins, res, _ = run_virtual(mgj, w, N, materialize=False, radix_bits_global=4, local_split_bits=ba)
+    d = w.rank_inputs()
+    ref = oracle.join(d["r_keys"], d["r_pays"], d["s_keys"], d["s_pays"])
+    for r in res:
+        assert (r["match_count"], r["checksum"]) == (ref["count"], ref["checksum"])
     for j in joins:
         j.close()
 
@@ -451,8 +518,9 @@ def test_m4_full_size_zipf(mgj):
 
 
 # ------------------------------------------------------------ EXTERNAL (NCCL-baseline) shuffle
-@pytest.mark.parametrize("N,kind", [(1, "unique"), (2, "unique"), (4, "unique"), (3, "zipf"), (2, "wide")])
-def test_external_shuffle_virtual_ranks(mgj, N, kind):
+@pytest.mark.parametrize("N,kind,ba", [(1, "unique", 0), (2, "unique", 0), (4, "unique", 0), (3, "zipf", 0),
+                                       (2, "wide", 0), (4, "unique", 3), (3, "zipf", 2)])
+def test_external_shuffle_virtual_ranks(mgj, N, kind, ba):
     """shuffle_mode EXTERNAL: the library packs per-destination send buffers, the
     caller's all-to-all (emulated here with device copies, as NCCL
     all_to_all_single would do) fills the receive areas, mgj_join finishes."""
@@ -462,7 +530,8 @@ def test_external_shuffle_virtual_ranks(mgj, N, kind):
     cap_r = max(p["r_keys"].size for p in parts)
     cap_s = max(p["s_keys"].size for p in parts)
     cfgs = [mgj.make_config(rank=g, world_size=N, key_bytes=w.key_bytes, r_capacity=cap_r, s_capacity=cap_s,
-                            recv_capacity_r=w.n_r, recv_capacity_s=w.n_s, shuffle_mode=mgj.SHUFFLE_EXTERNAL)
+                            recv_capacity_r=w.n_r, recv_capacity_s=w.n_s, shuffle_mode=mgj.SHUFFLE_EXTERNAL,
+                            local_split_bits=ba, radix_bits_global=4 if ba else 0)
             for g in range(N)]
     nb = mgj.arena_bytes(cfgs[0])
     arenas = [torch.zeros(nb, dtype=torch.uint8, device="cuda") for _ in range(N)]

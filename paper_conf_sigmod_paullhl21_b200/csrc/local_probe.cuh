@@ -89,43 +89,52 @@ __device__ __forceinline__ uint32_t nch_local(const Ctx &c, int rel) {
 }
 
 // Padded size (slots) of every (owned partition, first-pass digit) run, summed
-// over the chunks of the partition: exactly the slots k_local<K, true> reserves.
+// over the chunks of the partition: exactly the slots k_local<K, LM_SPLIT>
+// reserves.  QA <= 8 (the auto choice): each thread counts its <= 24 tuples
+// of a chunk in eight 8-bit fields of one register, reduced per warp once per
+// chunk; larger QA: warp-aggregated shared atomics (one per distinct digit).
 template <typename K>
 __global__ void __launch_bounds__(512) k_countA(Ctx c, const ChunkDesc *cdesc) {
     using Tup = typename Layout<K>::Tup;
     constexpr int ALIGN = Layout<K>::ALIGN;
-    __shared__ uint32_t cnt[16][1 << MAX_BA];  // per warp
+    __shared__ uint32_t cnt[1 << MAX_BA];
     if (!c.meta[MT_OK] || !c.meta[MT_BA]) return;
     const int BA = c.meta[MT_BA], QA = 1 << BA;
     const uint32_t nch_r = (uint32_t)c.meta[MT_NCH_R], total = nch_r + (uint32_t)c.meta[MT_NCH_S];
-    const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+    const int tid = threadIdx.x, lane = tid & 31;
+    const uint32_t nt = blockDim.x;
     const char *recv0 = c.arena[c.rank];
     for (uint32_t ci = blockIdx.x; ci < total; ci += gridDim.x) {
         const int rel = ci < nch_r ? 0 : 1;
         const ChunkDesc d = cdesc[ci];
         const Tup *src = reinterpret_cast<const Tup *>(recv0 + c.lay.recv[rel]) + d.start;
-        for (int i = tid; i < 16 * QA; i += blockDim.x) cnt[i / QA][i % QA] = 0;
+        if (tid < QA) cnt[tid] = 0;
         __syncthreads();
-        for (uint32_t i0 = 0; i0 < d.len; i0 += blockDim.x * 4) {
-            uint32_t q[4];
-#pragma unroll
-            for (int u = 0; u < 4; ++u) {
-                const uint32_t i = i0 + u * blockDim.x + tid;
-                q[u] = i < d.len ? digit2(__ldcs(&src[i].x), c.B1, QA) : 0xffffffffu;
+        if (QA <= 8) {
+            unsigned long long acc = 0;  // field q (8 bits): this thread's tuples with digit q
+            uint32_t i = tid;
+            for (; i + 3 * nt < d.len; i += 4 * nt) {
+                const K k0 = __ldcs(&src[i].x), k1 = __ldcs(&src[i + nt].x);
+                const K k2 = __ldcs(&src[i + 2 * nt].x), k3 = __ldcs(&src[i + 3 * nt].x);
+                acc += (1ull << (8 * digit2(k0, c.B1, QA))) + (1ull << (8 * digit2(k1, c.B1, QA))) +
+                       (1ull << (8 * digit2(k2, c.B1, QA))) + (1ull << (8 * digit2(k3, c.B1, QA)));
             }
-#pragma unroll
-            for (int u = 0; u < 4; ++u) {  // warp-aggregated: one shared atomic per distinct digit
-                const uint32_t peers = __match_any_sync(0xffffffffu, q[u]);
-                if (q[u] != 0xffffffffu && lane == __ffs(peers) - 1) atomicAdd(&cnt[w][q[u]], __popc(peers));
+            for (; i < d.len; i += nt) acc += 1ull << (8 * digit2(__ldcs(&src[i].x), c.B1, QA));
+            for (int q = 0; q < QA; ++q) {
+                const uint32_t v = __reduce_add_sync(0xffffffffu, (uint32_t)(acc >> (8 * q)) & 0xffu);
+                if (lane == 0 && v) atomicAdd(&cnt[q], v);
+            }
+        } else {
+            for (uint32_t i = tid; i < d.len; i += nt) {
+                const uint32_t q = digit2(__ldcs(&src[i].x), c.B1, QA);
+                const uint32_t peers = __match_any_sync(__activemask(), q);
+                if (lane == __ffs(peers) - 1) atomicAdd(&cnt[q], __popc(peers));
             }
         }
         __syncthreads();
-        for (int qa = tid; qa < QA; qa += blockDim.x) {
-            uint32_t n = 0;
-            for (int x = 0; x < (int)(blockDim.x >> 5); ++x) n += cnt[x][qa];
-            if (n) atomicAdd(&c.hA[(size_t)rel * c.vcap + ((size_t)d.pi << BA) + qa],
-                             (n + ALIGN - 1) & ~(uint32_t)(ALIGN - 1));
-        }
+        if (tid < QA && cnt[tid])
+            atomicAdd(&c.hA[(size_t)rel * c.vcap + ((size_t)d.pi << BA) + tid],
+                      (cnt[tid] + ALIGN - 1) & ~(uint32_t)(ALIGN - 1));
         __syncthreads();
     }
 }

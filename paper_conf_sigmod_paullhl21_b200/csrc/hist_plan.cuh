@@ -165,12 +165,10 @@ __global__ void __launch_bounds__(1024) k_plan(Ctx c) {
     __shared__ int first[MAX_RANKS], endp[MAX_RANKS];
     __shared__ int ok, cap_bad;
     __shared__ unsigned long long maxr;
-    __shared__ uint32_t maxnch;
     if (tid == 0) {
         ok = wait_all_flags(c, SIG_HIST);
         cap_bad = 0;
         maxr = 0;
-        maxnch = 0;
     }
     if (tid < MAX_RANKS) first[tid] = endp[tid] = P;
     __syncthreads();
@@ -297,10 +295,7 @@ __global__ void __launch_bounds__(1024) k_plan(Ctx c) {
                     pc[(size_t)i * (MAX_RANKS + 1) + g] = t;
                     t += (uint32_t)((pl[(size_t)i * MAX_RANKS + g] + C - 1) / C);
                 }
-            if (i < np) {
-                pc[(size_t)i * (MAX_RANKS + 1) + MAX_RANKS] = t;
-                atomicMax(&maxnch, t);
-            }
+            if (i < np) pc[(size_t)i * (MAX_RANKS + 1) + MAX_RANKS] = t;
             chn[i] = t;
         }
         __syncthreads();
@@ -317,15 +312,18 @@ __global__ void __launch_bounds__(1024) k_plan(Ctx c) {
         c.meta[MT_NCH_R] = (int)nch[0];
         c.meta[MT_NCH_S] = (int)nch[1];
         c.meta[MT_CHUNK] = c.chunk_tuples;
-        // two-level local partitioning: when an owned partition
-        // spans more than LOCAL2_NCH chunks, a first histogram-based pass
-        // splits every owned partition into 2^BA contiguous sub-partitions of
-        // ~48 chunks, and the chunked pass then uses the remaining B2 - BA bits
+        // two-level local partitioning: when the owned
+        // partitions span more than LOCAL2_NCH chunks on average, a first
+        // histogram-based pass splits every owned partition into 2^BA
+        // contiguous sub-partitions of ~48 chunks, and the chunked pass then
+        // uses the remaining B2 - BA bits.  The mean, not the maximum: a few
+        // heavy-hitter partitions (Zipf) are not helped by splitting the rest
+        const uint32_t meannch = np ? (max(nch[0], nch[1]) + np - 1) / np : 0;
         int BA = 0;
         if (c.split_cfg > 0) {
             BA = c.split_cfg;
-        } else if (c.split_cfg == 0 && maxnch > (uint32_t)LOCAL2_NCH) {
-            BA = ceil_log2_u64((maxnch + 47) / 48);
+        } else if (c.split_cfg == 0 && meannch > (uint32_t)LOCAL2_NCH) {
+            BA = ceil_log2_u64((meannch + 47) / 48);
             while (BA > 0 && (np << BA) > c.vcap) --BA;
         }
         if (BA > B2) BA = B2;

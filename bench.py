@@ -430,7 +430,7 @@ def main():
             "roofline": roof,
             "cpu_baseline": None if cpu is None else {k: cpu[k] for k in ("value", "unit", "cores", "kind", "sample")},
             "e2e": e2e,
-            "gpu_launches": 8 * a.steps,
+            "gpu_launches": res["n_launches"] * a.steps,  # counted by the library per run
             "clocks": clocks,
         }
         emit(out, line)

@@ -117,6 +117,7 @@ typedef struct {
     int32_t  radix_bits_global;    /* B1 used */
     int32_t  radix_bits_local;     /* B2 chosen on device for this rank */
     int32_t  n_items;              /* probe work items (co-partition slices) on this rank */
+    int32_t  n_launches;           /* kernels this handle launched for the run (partition .. result) */
 } mgj_result_t;
 
 /* Bytes each rank's symmetric arena needs for cfg (0 if cfg is invalid). */

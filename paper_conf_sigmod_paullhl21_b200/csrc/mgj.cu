@@ -126,6 +126,7 @@ struct mgj_plan_s {
     char *send_arena = nullptr;  // EXTERNAL shuffle
     uint64_t epoch = 0;
     int state = 0;
+    int launches = 0;  // kernels launched for the current run
     cudaStream_t stream = nullptr;
     cudaEvent_t ev[7] = {};
     void *stage = nullptr;
@@ -192,6 +193,7 @@ void launch_partition(mgj_plan_s *h, cudaStream_t s) {
     const Norm &n = h->n;
     dim3 g(h->ctx.G * HIST_SPLIT, 2);
     k_hist<K><<<g, HIST_THREADS, hist_smem(n), s>>>(h->ctx);
+    h->launches = 1;
 }
 
 template <typename K>
@@ -205,12 +207,16 @@ void launch_shuffle(mgj_plan_s *h, cudaStream_t s) {
     if (cs.ext)
         for (int g = 0; g < MAX_RANKS; ++g) cs.arena[g] = h->send_arena;
     k_scatter<K><<<h->ctx.G, SCATTER_THREADS, scatter_smem(n), s>>>(cs);
+    h->launches += 4;
 }
 
 template <typename K>
 void launch_join(mgj_plan_s *h, cudaStream_t s) {
     const Norm &n = h->n;
-    if (!h->ctx.ext) k_wait<<<1, 32, 0, s>>>(h->ctx, SIG_DATA);  // EXTERNAL: the caller's exchange is stream-ordered
+    if (!h->ctx.ext) {  // EXTERNAL: the caller's exchange is stream-ordered
+        k_wait<<<1, 32, 0, s>>>(h->ctx, SIG_DATA);
+        h->launches += 1;
+    }
     // two-level local partitioning (device-side decision, MT_BA; no-ops otherwise)
     if (n.split) {
         k_countA<K><<<h->nsm * 4, 512, 0, s>>>(h->ctx, h->cdesc);
@@ -218,6 +224,7 @@ void launch_join(mgj_plan_s *h, cudaStream_t s) {
         k_local<K, LM_SPLIT><<<h->nsm, LOCAL_THREADS, local_smem(n), s>>>(h->ctx, h->cdesc);
         k_chunkmapB<<<h->nsm * 2, 256, 0, s>>>(h->ctx, h->cdesc);
         k_local<K, LM_SECOND><<<h->nsm, LOCAL_THREADS, local_smem(n), s>>>(h->ctx, h->cdesc);
+        h->launches += 5;
     }
     k_local<K, LM_SINGLE><<<h->nsm, LOCAL_THREADS, local_smem(n), s>>>(h->ctx, h->cdesc);
     cudaEventRecord(h->ev[4], s);
@@ -228,6 +235,7 @@ void launch_join(mgj_plan_s *h, cudaStream_t s) {
         k_probe<K, false><<<h->nsm, PROBE_THREADS, probe_smem(n), s>>>(h->ctx);
     cudaEventRecord(h->ev[5], s);
     k_publish<<<1, 32, 0, s>>>(h->ctx);
+    h->launches += 4;  // local, itemize, probe, publish
 }
 
 }  // namespace
@@ -470,6 +478,7 @@ mgj_status mgj_result(mgj_handle h, mgj_result_t *out) {
     if (h->state != ST_JOINED && h->state != ST_DONE) return MGJ_ESTATE;
     if (h->state == ST_JOINED) {  // a6: wait for every rank's partial result and sum
         k_gather<<<1, 32, 0, h->stream>>>(h->ctx);
+        h->launches += 1;
         cudaMemcpyAsync(h->h_res, h->ctx.result, 4 * 8, cudaMemcpyDeviceToHost, h->stream);
         cudaMemcpyAsync(h->h_meta, h->ctx.meta, MT_COUNT * 4, cudaMemcpyDeviceToHost, h->stream);
     }
@@ -502,6 +511,7 @@ mgj_status mgj_result(mgj_handle h, mgj_result_t *out) {
     unsigned int ni = 0;
     cudaMemcpy(&ni, c.ticket + TK_ITEMS, 4, cudaMemcpyDeviceToHost);
     out->n_items = (int32_t)std::min<uint64_t>(ni, h->n.max_items);
+    out->n_launches = h->launches;
     h->state = ST_DONE;
     return (mgj_status)out->status;
 }

@@ -69,7 +69,7 @@ class Result(ctypes.Structure):
                 ("recv_r", ctypes.c_uint64), ("recv_s", ctypes.c_uint64),
                 ("phase_ms", ctypes.c_float * 6), ("status", ctypes.c_int32),
                 ("radix_bits_global", ctypes.c_int32), ("radix_bits_local", ctypes.c_int32),
-                ("n_items", ctypes.c_int32)]
+                ("n_items", ctypes.c_int32), ("n_launches", ctypes.c_int32)]
 
 
 _H = ctypes.c_void_p
@@ -198,7 +198,7 @@ class Join:
                 "recv_r": int(r.recv_r), "recv_s": int(r.recv_s),
                 "phase_ms": [float(x) for x in r.phase_ms], "status": int(r.status),
                 "radix_bits_global": int(r.radix_bits_global), "radix_bits_local": int(r.radix_bits_local),
-                "n_items": int(r.n_items)}
+                "n_items": int(r.n_items), "n_launches": int(r.n_launches)}
 
     def run(self, r_keys, r_pays, s_keys, s_pays, stream=None) -> dict:
         self.partition(r_keys, r_pays, s_keys, s_pays, stream)

@@ -15,7 +15,6 @@ constexpr int MAX_B2 = 11;              // local fan-out per pass
 constexpr int HIST_THREADS = 512;
 constexpr int HIST_SPLIT = 4;           // CTAs per histogram tile
 constexpr int SCATTER_THREADS = 1024;
-constexpr int SCAT_T8 = 8192;           // scatter sub-tile (tuples) for 8-byte tuples; 4096 for 16-byte
 constexpr int LOCAL_THREADS = 1024;
 constexpr int LOCAL_VMAX = 12;          // local-pass tuples per thread (chunk C <= 12 * LOCAL_THREADS), 8-byte tuples
 __host__ __device__ constexpr int local_vmax(int tuple_bytes) { return LOCAL_VMAX * 8 / tuple_bytes; }

@@ -170,7 +170,7 @@ cudaError_t set_attrs(const Norm &n) {
     const auto A = cudaFuncAttributeMaxDynamicSharedMemorySize;
     if ((e = cudaFuncSetAttribute(k_hist<K>, A, (int)hist_smem(n)))) return e;
     if ((e = cudaFuncSetAttribute(k_plan, A, (int)plan_smem(n)))) return e;
-    if ((e = cudaFuncSetAttribute(k_scatter<K>, A, (int)scatter_smem(n)))) return e;
+    if ((e = cudaFuncSetAttribute(scatter_kernel<K>(n.P), A, (int)scatter_smem(n)))) return e;
     if ((e = cudaFuncSetAttribute(k_local<K, LM_SINGLE>, A, (int)local_smem(n)))) return e;
     if ((e = cudaFuncSetAttribute(k_local<K, LM_SPLIT>, A, (int)local_smem(n)))) return e;
     if ((e = cudaFuncSetAttribute(k_local<K, LM_SECOND>, A, (int)local_smem(n)))) return e;
@@ -206,7 +206,7 @@ void launch_shuffle(mgj_plan_s *h, cudaStream_t s) {
     Ctx cs = h->ctx;
     if (cs.ext)
         for (int g = 0; g < MAX_RANKS; ++g) cs.arena[g] = h->send_arena;
-    k_scatter<K><<<h->ctx.G, SCATTER_THREADS, scatter_smem(n), s>>>(cs);
+    scatter_kernel<K>(n.P)<<<h->ctx.G, SCATTER_THREADS, scatter_smem(n), s>>>(cs);
     h->launches += 4;
 }
 

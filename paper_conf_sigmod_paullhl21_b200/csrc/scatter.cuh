@@ -7,30 +7,80 @@
 
 namespace mgj {
 
-template <typename K> struct ScatCfg {
-    using Tup = typename TupT<K>::T;
-    static constexpr int TMAX = SCAT_T8 * 4 / (int)sizeof(K);  // 8192 (4-byte) / 4096 (8-byte) tuples
-    static constexpr int VMAX = TMAX / SCATTER_THREADS;        // tuples per thread per sub-tile
+// Scatter geometry for P partitions and a key width (kernel template
+// arguments; the host picks the instance with scatter_kernel<K>(P)):
+//   T   = sub-tile (tuples) staged in shared memory per step,
+//   SG  = tuples per 32-byte sector group (the unit of a global store),
+//   PPT = partitions owned by each of the 1024 threads (registers).
+// With SG > 1 every partition's output leaves in whole 32-byte sectors: the
+// < 32-byte tail of a partition waits (in registers of its owning thread)
+// for the next sub-tile.  For P = 4096 the alignment padding would not fit
+// shared memory, so SG = 1 (one tuple per store).
+struct ScatGeom {
+    int T, SG, PPT;
+};
+__host__ __device__ constexpr ScatGeom scat_geom(int P, int key_bytes) {
+    return key_bytes == 4 ? (P <= 1024 ? ScatGeom{8192, 4, 1} : P == 2048 ? ScatGeom{4096, 4, 2} : ScatGeom{8192, 1, 4})
+                          : (P <= 1024 ? ScatGeom{4096, 2, 1} : P == 2048 ? ScatGeom{2048, 2, 2} : ScatGeom{4096, 1, 4});
+}
+
+// Per-partition write-out descriptor of the current sub-tile (16 bytes, one
+// shared load per sector group).
+struct __align__(16) PInfo {
+    unsigned long long wb;  // destination address of sorted slot 0 (wb + slot * TB)
+    uint32_t lim;           // end of the partition's valid slots in `sorted`
+    uint32_t head;          // (slot << 2 | h) of a head group whose first h slots are not ours, else ~0
 };
 
-// Sub-tile size and per-partition carry capacity for P partitions (shared
-// memory stays within 227 KB).  The carry holds the < 32-byte tail of each
-// partition's output so that global stores cover whole 32-byte sectors.
-__host__ __device__ inline int scat_subtile(int P, int key_bytes) {
-    const int tmax = SCAT_T8 * 4 / key_bytes;
-    return P <= 1024 ? tmax : tmax / 2;
-}
-__host__ __device__ inline int scat_carry(int P, int tuple_bytes) { return P <= 2048 ? 32 / tuple_bytes - 1 : 0; }
-
 __host__ __device__ inline size_t scat_smem_bytes(int P, int key_bytes) {
-    const size_t T = (size_t)scat_subtile(P, key_bytes);
+    const ScatGeom g = scat_geom(P, key_bytes);
     const size_t TB = 2 * (size_t)key_bytes;
-    const size_t CC = (size_t)scat_carry(P, (int)TB);
-    return 2 * T * key_bytes      // input stage: keys + payloads
-           + (T + CC * P) * TB    // partition-sorted sub-tile (+ carried tails)
-           + (size_t)P * 4 * 4    // bins, pos, lim, ccount
-           + (size_t)P * 8 * 2    // wb, base
-           + (size_t)P * CC * TB; // carry
+    return 2 * (size_t)g.T * key_bytes                      // input stage: keys + payloads (SoA)
+           + ((size_t)g.T + 2 * (size_t)(g.SG - 1) * P) * TB  // partition-sorted sub-tile (+ carries, group padding)
+           + (size_t)P * sizeof(PInfo)
+           + (size_t)P * 4;                                  // bins / scatter positions
+}
+
+// Block-wide exclusive scan of one register value per thread (1024 threads).
+__device__ __forceinline__ uint32_t block_scan_reg(uint32_t v, uint32_t *tmp, uint32_t &total) {
+    const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+    uint32_t x = v;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+        if (lane >= o) x += y;
+    }
+    if (lane == 31) tmp[w] = x;
+    __syncthreads();
+    if (w == 0) {
+        uint32_t s = tmp[lane];
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const uint32_t y = __shfl_up_sync(0xffffffffu, s, o);
+            if (lane >= o) s += y;
+        }
+        tmp[lane] = s;  // inclusive warp totals
+    }
+    __syncthreads();
+    total = tmp[31];
+    return x - v + (w ? tmp[w - 1] : 0);
+}
+
+template <int BYTES> struct Vec;
+template <> struct Vec<8> { using T = uint2; };
+template <> struct Vec<16> { using T = uint4; };
+template <> struct Vec<32> { struct __align__(32) T { uint4 a, b; }; };
+
+// One global store of a 8/16/32-byte group (32 bytes: a single 256-bit store).
+template <int BYTES>
+__device__ __forceinline__ void st_group(void *dst, const typename Vec<BYTES>::T &v) {
+    if constexpr (BYTES == 32) {
+        asm volatile("st.global.v8.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};" ::"l"(dst), "r"(v.a.x), "r"(v.a.y),
+                     "r"(v.a.z), "r"(v.a.w), "r"(v.b.x), "r"(v.b.y), "r"(v.b.z), "r"(v.b.w)
+                     : "memory");
+    } else {
+        *static_cast<typename Vec<BYTES>::T *>(dst) = v;
+    }
 }
 
 // ---------------------------------------------------------------------------
@@ -39,56 +89,63 @@ __host__ __device__ inline size_t scat_smem_bytes(int P, int key_bytes) {
 // after partitioning based on the histogram and then writes the tuple" —
 // after Rui et al. [38]; step 3 data distribution, P:405-407 and §4).
 //
-// B200 form: one persistent CTA per SM processes tile c = blockIdx.x of R and
-// then of S, in sub-tiles of T tuples brought into shared memory by a TMA
-// bulk copy issued one sub-tile ahead.  Each sub-tile is counting-sorted by
-// digit1 in shared memory (one SMEM atomic per tuple gives the rank in its
-// bin) and written out in sorted order, so each warp store covers a few
-// contiguous runs.  Destinations are exact: owner(p)'s receive buffer at
-// send_off[p] (a2) + tile_base[c][p] (a1 tile prefix) + the running count of
-// p in this tile — no global atomics.  Every partition keeps its < 32-byte
-// tail in shared memory until the next sub-tile completes the sector, so
-// (except at tile boundaries) every store covers whole 32-byte sectors and
-// DRAM never sees a partial-sector read-modify-write.  On NVSwitch the owner
-// may be another GPU: the same store goes over NVLink to a peer-mapped
+// B200 form: one persistent CTA (1024 threads) per SM processes tile
+// c = blockIdx.x of R and then of S, in sub-tiles of T tuples that a TMA
+// bulk copy brings into shared memory one sub-tile ahead.  Per sub-tile:
+//  1. each thread takes LU-tuple vectors of keys and payloads from the stage
+//     and ranks every tuple in its digit1 bin (one shared atomic);
+//  2. thread t owns partitions t*PPT.. (PPT per thread) and keeps, in
+//     registers, each one's destination cursor and its < 32-byte tail
+//     (carry) from the previous sub-tile; a block scan of the per-partition
+//     sizes (carry + new, rounded up to a 32-byte group) lays the partitions
+//     out group-aligned in `sorted`, the carry first;
+//  3. tuples are scattered into `sorted`, then written out one 32-byte group
+//     per thread and store (st.global.v8.b32): every complete group is a
+//     whole DRAM sector at its final address — owner(p)'s receive buffer at
+//     send_off[p] (a2) + tile_base[c][p] (a1 tile prefix) + the running
+//     count of p in this tile; no global atomics.  An incomplete last group
+//     stays in `sorted` and its owning thread reloads it as the next carry.
+// A tile's first destination of a partition need not be group-aligned: the
+// carry then starts with h placeholder slots (key = p) that are never stored
+// (the head group is written tuple by tuple from slot h).  The relation's
+// remaining tails are written tuple by tuple at its end.  On NVSwitch the
+// owner may be another GPU: the same stores go over NVLink to a peer-mapped
 // address; the paper's packets, routing buffers and multi-hop routing (§4)
 // have no role on a one-hop fabric.  The last CTA raises SIG_DATA at every
 // peer after a system fence.
 // ---------------------------------------------------------------------------
-template <typename K>
+template <typename K, int T, int SG, int PPT>
 __global__ void __launch_bounds__(SCATTER_THREADS, 1) k_scatter(Ctx c) {
     using Tup = typename TupT<K>::T;
-    constexpr int VMAX = ScatCfg<K>::VMAX;
     constexpr int TB = (int)sizeof(Tup);
+    constexpr int NT = SCATTER_THREADS;
+    constexpr int V = T / NT;                  // tuples per thread per sub-tile
+    constexpr int LU = 16 / (int)sizeof(K);    // tuples per 16-byte stage vector
+    constexpr int NU = V / LU;                 // vectors per thread
+    static_assert(NU * LU == V && NU >= 1, "sub-tile");
+    constexpr int GB = SG * TB;                // group bytes
+    constexpr int CW = SG > 1 ? SG - 1 : 1;    // carry capacity (tuples)
+    constexpr uint32_t NONE = 0xffffffffu;
+    using GV = typename Vec<GB>::T;
     typedef unsigned long long ull;
     extern __shared__ __align__(128) unsigned char smem[];
     const int P = c.P;
-    const int T = scat_subtile(P, (int)sizeof(K));
-    const int V = T / SCATTER_THREADS;
-    const int CC = scat_carry(P, TB);
     K *const skey = reinterpret_cast<K *>(smem);
     K *const spay = skey + T;
     Tup *const sorted = reinterpret_cast<Tup *>(spay + T);
-    uint32_t *const bins = reinterpret_cast<uint32_t *>(sorted + T + (size_t)CC * P);
-    uint32_t *const pos = bins + P;
-    uint32_t *const lim = pos + P;
-    uint32_t *const ccount = lim + P;
-    ull *const wb = reinterpret_cast<ull *>(ccount + P);
-    ull *const base = wb + P;
-    Tup *const carry = reinterpret_cast<Tup *>(base + P);
+    PInfo *const pinfo = reinterpret_cast<PInfo *>(sorted + T + 2 * (SG - 1) * P);  // 16-byte aligned
+    uint32_t *const bins = reinterpret_cast<uint32_t *>(pinfo + P);
     __shared__ __align__(8) uint64_t bar;
-    __shared__ uint32_t tmp[33];
+    __shared__ uint32_t tmp[32];
     const int tid = threadIdx.x;
     const int tile = blockIdx.x;
     const int ok = *(volatile int32_t *)&c.meta[MT_OK];
 
-    uint64_t lo[2], hi[2];
-    uint32_t nsub[2];
-    for (int r = 0; r < 2; ++r) {
-        tile_range(c.n_in[r], c.G, tile, lo[r], hi[r]);
-        nsub[r] = ok ? (uint32_t)((hi[r] - lo[r] + T - 1) / T) : 0;
-    }
-    const uint32_t ntot = nsub[0] + nsub[1];
+    uint64_t lo0, hi0, lo1, hi1;  // scalars (no local-memory arrays)
+    tile_range(c.n_in[0], c.G, tile, lo0, hi0);
+    tile_range(c.n_in[1], c.G, tile, lo1, hi1);
+    const uint32_t nsub0 = ok ? (uint32_t)((hi0 - lo0 + T - 1) / T) : 0;
+    const uint32_t ntot = nsub0 + (ok ? (uint32_t)((hi1 - lo1 + T - 1) / T) : 0);
     if (tid == 0) {
         mbar_init(&bar, 1);
         fence_mbar_init();
@@ -96,39 +153,69 @@ __global__ void __launch_bounds__(SCATTER_THREADS, 1) k_scatter(Ctx c) {
     __syncthreads();
     const uint64_t pol = policy_evict_first();
 
-    // sub-tile g of the R-then-S sequence -> (rel, first tuple, length)
+    // per owned partition (registers): destination of the next group, carry
+    ull base[PPT];
+    uint32_t cc[PPT], hd[PPT], lim[PPT];
+    Tup carry[PPT][CW];
+    bool pending = false;  // carries of the last sub-tile still sit in `sorted`
+#pragma unroll
+    for (int k = 0; k < PPT; ++k) base[k] = 0, cc[k] = 0, hd[k] = 0, lim[k] = 0;
+
     auto subtile = [&](uint32_t g, int &rel, uint64_t &first, uint32_t &len) {
-        rel = g < nsub[0] ? 0 : 1;
-        const uint32_t j = rel ? g - nsub[0] : g;
-        first = lo[rel] + (uint64_t)j * T;
-        len = (uint32_t)min((uint64_t)T, hi[rel] - first);
+        rel = g < nsub0 ? 0 : 1;
+        const uint32_t j = rel ? g - nsub0 : g;
+        first = (rel ? lo1 : lo0) + (uint64_t)j * T;
+        len = (uint32_t)min((uint64_t)T, (rel ? hi1 : hi0) - first);
     };
     auto issue = [&](uint32_t g) {  // thread 0: TMA the 16-byte-aligned body of sub-tile g
         int rel;
         uint64_t first;
         uint32_t len;
         subtile(g, rel, first, len);
-        const uint32_t body = len & ~(uint32_t)(16 / sizeof(K) - 1);
-        const uint32_t bytes = body * (uint32_t)sizeof(K);
+        const uint32_t bytes = (len & ~(uint32_t)(LU - 1)) * (uint32_t)sizeof(K);
         mbar_arrive_expect_tx(&bar, 2 * bytes);
         if (bytes) {
             tma_load_1d(skey, static_cast<const K *>(c.in_key[rel]) + first, bytes, &bar, pol);
             tma_load_1d(spay, static_cast<const K *>(c.in_pay[rel]) + first, bytes, &bar, pol);
         }
     };
-    auto set_base = [&](int rel) {  // destination of this tile's first tuple of each partition
-        const uint32_t *tb = c.tile_base + ((size_t)rel * c.G + tile) * P;
-        const uint64_t *so = c.send_off + (size_t)rel * P;
-        for (int p = tid; p < P; p += SCATTER_THREADS) {
-            const int own = c.owner[p];
-            base[p] = (ull)(c.arena[own] + c.lay.recv[rel]) + (so[p] + tb[p]) * (uint64_t)TB;
-            ccount[p] = 0;
+    auto fetch_carry = [&]() {  // the incomplete last groups of the previous sub-tile -> registers
+        if (pending) {
+#pragma unroll
+            for (int k = 0; k < PPT; ++k)
+#pragma unroll
+                for (int i = 0; i < CW; ++i)
+                    if (i < (int)cc[k]) carry[k][i] = sorted[lim[k] - cc[k] + i];
+            pending = false;
         }
     };
-    auto flush_carry = [&]() {  // end of a relation: write the remaining tails
-        for (int p = tid; p < P; p += SCATTER_THREADS)
-            for (uint32_t k = 0; k < ccount[p]; ++k)
-                reinterpret_cast<Tup *>(base[p])[k] = carry[(size_t)p * CC + k];
+    auto flush = [&]() {  // end of a relation: store the remaining tails tuple by tuple
+        fetch_carry();
+#pragma unroll
+        for (int k = 0; k < PPT; ++k)
+#pragma unroll
+            for (int i = 0; i < CW; ++i)
+                if (i >= (int)hd[k] && i < (int)cc[k]) reinterpret_cast<Tup *>(base[k])[i] = carry[k][i];
+    };
+    auto set_base = [&](int rel) {  // destination of this tile's first tuple of each owned partition
+        const uint32_t *tb = c.tile_base + ((size_t)rel * c.G + tile) * P;
+        const uint64_t *so = c.send_off + (size_t)rel * P;
+#pragma unroll
+        for (int k = 0; k < PPT; ++k) {
+            const int p = tid * PPT + k;
+            cc[k] = hd[k] = 0;
+            if (p < P) {
+                const ull a = (ull)(c.arena[c.owner[p]] + c.lay.recv[rel]) + (so[p] + tb[p]) * (uint64_t)TB;
+                const uint32_t h = SG > 1 ? (uint32_t)((a & (GB - 1)) / TB) : 0u;
+                base[k] = a - (ull)h * TB;
+                cc[k] = hd[k] = h;
+#pragma unroll
+                for (int i = 0; i < CW; ++i) {  // placeholders: digit1 = p, never stored
+                    carry[k][i].x = (K)p;
+                    carry[k][i].y = 0;
+                }
+            }
+        }
     };
 
     if (tid == 0 && ntot > 0) issue(0);
@@ -138,82 +225,111 @@ __global__ void __launch_bounds__(SCATTER_THREADS, 1) k_scatter(Ctx c) {
         uint64_t first;
         uint32_t len;
         subtile(g, rel, first, len);
-        if (rel != cur_rel) {
-            __syncthreads();
-            if (cur_rel >= 0) flush_carry();
-            __syncthreads();
+        if (rel != cur_rel) {  // thread-private partition state: no barrier needed
+            if (cur_rel >= 0) flush();
             set_base(rel);
             cur_rel = rel;
         }
+        fetch_carry();
         mbar_wait(&bar, g & 1);
-        const uint32_t body = len & ~(uint32_t)(16 / sizeof(K) - 1);
+        const uint32_t body = len & ~(uint32_t)(LU - 1);
         const K *gk = static_cast<const K *>(c.in_key[rel]) + first;
         const K *gp = static_cast<const K *>(c.in_pay[rel]) + first;
-        K kk[VMAX], pp[VMAX];
+        K kk[V], pp[V];
 #pragma unroll
-        for (int v = 0; v < VMAX; ++v) {
-            const uint32_t i = tid + v * SCATTER_THREADS;
-            if (v < V && i < body) {
-                kk[v] = skey[i];
-                pp[v] = spay[i];
-            } else if (v < V && i < len) {  // < 4 trailing tuples of the relation
-                kk[v] = gk[i];
-                pp[v] = gp[i];
+        for (int u = 0; u < NU; ++u) {
+            const uint32_t i0 = (uint32_t)(u * NT + tid) * LU;
+            if (i0 + LU <= body) {
+                const uint4 a = *reinterpret_cast<const uint4 *>(skey + i0);
+                const uint4 b = *reinterpret_cast<const uint4 *>(spay + i0);
+                memcpy(&kk[u * LU], &a, 16);
+                memcpy(&pp[u * LU], &b, 16);
+            } else {
+#pragma unroll
+                for (int e = 0; e < LU; ++e) {  // < LU trailing tuples of the relation come from global
+                    const uint32_t i = i0 + e;
+                    kk[u * LU + e] = i < body ? skey[i] : (i < len ? gk[i] : (K)0);
+                    pp[u * LU + e] = i < body ? spay[i] : (i < len ? gp[i] : (K)0);
+                }
             }
         }
-        for (int p = tid; p < P; p += SCATTER_THREADS) bins[p] = 0;
-        __syncthreads();  // S1: stage consumed, bins cleared
-        if (tid == 0 && g + 1 < ntot) issue(g + 1);
-        uint32_t rp[VMAX];  // rank in bin << 16 | partition
 #pragma unroll
-        for (int v = 0; v < VMAX; ++v) {
-            const uint32_t i = tid + v * SCATTER_THREADS;
-            if (v < V && i < len) {
+        for (int k = 0; k < PPT; ++k)
+            if (tid * PPT + k < P) bins[tid * PPT + k] = 0;
+        __syncthreads();  // S1: stage consumed, bins cleared, carries fetched
+        if (tid == 0 && g + 1 < ntot) issue(g + 1);
+        uint32_t rp[V];  // rank in bin << 16 | partition
+#pragma unroll
+        for (int v = 0; v < V; ++v) {
+            const uint32_t i = (uint32_t)((v / LU) * NT + tid) * LU + (v % LU);
+            rp[v] = NONE;
+            if (i < len) {
                 const uint32_t p = digit1(kk[v], P);
                 rp[v] = (atomicAdd(&bins[p], 1u) << 16) | p;
             }
         }
-        __syncthreads();  // S2
-        for (int p = tid; p < P; p += SCATTER_THREADS) bins[p] += ccount[p];
-        __syncthreads();
-        const uint32_t ttot = block_excl_scan_u32(bins, P, tmp);
-        for (int p = tid; p < P; p += SCATTER_THREADS) {
-            const uint32_t o = bins[p];
-            const uint32_t tp = ((p + 1 < P) ? bins[p + 1] : ttot) - o;
-            const uint32_t cc = ccount[p];
-            const ull G = base[p];
-            const ull end = G + (ull)tp * TB;
-            const ull aend = CC ? (end & ~31ull) : end;
-            const uint32_t L = aend > G ? (uint32_t)((aend - G) / TB) : 0;
-            lim[p] = o + L;
-            wb[p] = G - (ull)o * TB;
-            base[p] = G + (ull)L * TB;
-            for (uint32_t k = 0; k < cc; ++k) sorted[o + k] = carry[(size_t)p * CC + k];
-            pos[p] = o + cc;
-            ccount[p] = tp - L;
-        }
-        __syncthreads();  // S3
+        __syncthreads();  // S2: counts final
+        uint32_t cnt[PPT], seg[PPT], tsum = 0;
 #pragma unroll
-        for (int v = 0; v < VMAX; ++v) {
-            const uint32_t i = tid + v * SCATTER_THREADS;
-            if (v < V && i < len) {
+        for (int k = 0; k < PPT; ++k) {
+            const int p = tid * PPT + k;
+            cnt[k] = p < P ? cc[k] + bins[p] : 0;
+            seg[k] = (cnt[k] + SG - 1) & ~(uint32_t)(SG - 1);
+            tsum += seg[k];
+        }
+        uint32_t total;
+        uint32_t o = block_scan_reg(tsum, tmp, total);
+#pragma unroll
+        for (int k = 0; k < PPT; ++k) {
+            const int p = tid * PPT + k;
+            if (p < P) {
+#pragma unroll
+                for (int i = 0; i < CW; ++i)
+                    if (i < (int)cc[k]) sorted[o + i] = carry[k][i];
+                bins[p] = o + cc[k];
+                const uint32_t full = cnt[k] & ~(uint32_t)(SG - 1);
+                PInfo in;
+                in.wb = base[k] - (ull)o * TB;
+                in.lim = o + cnt[k];
+                in.head = (hd[k] && full) ? (o << 2 | hd[k]) : NONE;
+                pinfo[p] = in;
+                base[k] += (ull)full * TB;
+                if (full) hd[k] = 0;
+                cc[k] = cnt[k] - full;
+                lim[k] = o + cnt[k];
+            }
+            o += seg[k];
+        }
+        pending = SG > 1;
+        __syncthreads();  // S3: positions, descriptors and carries in place
+#pragma unroll
+        for (int v = 0; v < V; ++v) {
+            if (rp[v] != NONE) {
                 Tup t;
                 t.x = kk[v];
                 t.y = pp[v];
-                sorted[pos[rp[v] & 0xffffu] + (rp[v] >> 16)] = t;
+                sorted[bins[rp[v] & 0xffffu] + (rp[v] >> 16)] = t;
             }
         }
         __syncthreads();  // S4
-        for (uint32_t i = tid; i < ttot; i += SCATTER_THREADS) {
-            const Tup t = sorted[i];
-            const uint32_t p = digit1(t.x, P);
-            const uint32_t l = lim[p];
-            if (i < l) reinterpret_cast<Tup *>(wb[p] + (ull)i * TB)[0] = t;
-            else carry[(size_t)p * CC + (i - l)] = t;
+        const uint32_t ngroups = total / SG;
+        for (uint32_t u = tid; u < ngroups; u += NT) {
+            const uint32_t slot = u * SG;
+            const GV gv = *reinterpret_cast<const GV *>(sorted + slot);
+            const uint32_t p = reinterpret_cast<const uint32_t *>(&gv)[0] & (uint32_t)(P - 1);  // digit1 of slot's key
+            const PInfo in = pinfo[p];
+            if (slot + SG <= in.lim) {
+                char *dst = reinterpret_cast<char *>(in.wb + (ull)slot * TB);
+                if ((in.head >> 2) != slot) {
+                    st_group<GB>(dst, gv);
+                } else {
+                    for (uint32_t i = in.head & 3u; i < SG; ++i)
+                        reinterpret_cast<Tup *>(dst)[i] = sorted[slot + i];
+                }
+            }
         }
     }
-    __syncthreads();
-    if (cur_rel >= 0) flush_carry();
+    if (cur_rel >= 0) flush();
 
     // ---- every CTA: make its (peer) stores visible, the last one signals ----
     __threadfence_system();
@@ -224,6 +340,19 @@ __global__ void __launch_bounds__(SCATTER_THREADS, 1) k_scatter(Ctx c) {
             __threadfence_system();
             signal_all(c, SIG_DATA);
         }
+    }
+}
+
+template <typename K>
+inline void (*scatter_kernel(int P))(Ctx) {
+    if constexpr (sizeof(K) == 8) {
+        if (P <= 1024) return k_scatter<K, 4096, 2, 1>;
+        if (P == 2048) return k_scatter<K, 2048, 2, 2>;
+        return k_scatter<K, 4096, 1, 4>;
+    } else {
+        if (P <= 1024) return k_scatter<K, 8192, 4, 1>;
+        if (P == 2048) return k_scatter<K, 4096, 4, 2>;
+        return k_scatter<K, 8192, 1, 4>;
     }
 }
 

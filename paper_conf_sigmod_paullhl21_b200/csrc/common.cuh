@@ -91,6 +91,9 @@ struct Ctx {
     uint32_t *rank_hist;          // [2][P]
     uint32_t *tile_hist;          // [2][G][P] per-tile histograms (a1)
     uint32_t *tile_base;          // [2][G][P] exclusive prefix over tiles
+    uint16_t *sub_hist;           // [2][G][sub_ns][P] per scatter sub-tile histograms (a1)
+    int32_t scat_T;               // scatter sub-tile (tuples)
+    int32_t sub_ns;               // sub-tiles per tile (capacity)
     uint32_t *ticket;             // [TK_COUNT]
     int32_t *meta;                // [MT_COUNT]
     int32_t *owner;               // [P]

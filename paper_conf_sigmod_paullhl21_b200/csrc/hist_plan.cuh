@@ -19,54 +19,77 @@ namespace mgj {
 // ---------------------------------------------------------------------------
 template <typename K>
 __global__ void __launch_bounds__(HIST_THREADS) k_hist(Ctx c) {
-    extern __shared__ uint32_t sh[];  // [P]
-    const int P = c.P;
+    extern __shared__ uint32_t sh[];  // sub[P] (current sub-tile), acc[P] (this CTA's share of the tile)
+    const int P = c.P, T = c.scat_T;
+    uint32_t *const sub = sh, *const acc = sh + P;
     const int rel = blockIdx.y, tile = blockIdx.x / HIST_SPLIT, part = blockIdx.x % HIST_SPLIT;
+    const int tid = threadIdx.x;
     const K *keys = static_cast<const K *>(c.in_key[rel]);
-    uint64_t tlo, thi, lo, hi;
+    uint64_t tlo, thi;
     tile_range(c.n_in[rel], c.G, tile, tlo, thi);
-    {  // HIST_SPLIT CTAs share a tile (16-byte aligned parts)
-        const uint64_t n = thi - tlo;
-        lo = tlo + ((n * part / HIST_SPLIT) & ~3ull);
-        hi = part == HIST_SPLIT - 1 ? thi : tlo + ((n * (part + 1) / HIST_SPLIT) & ~3ull);
-    }
-    for (int i = threadIdx.x; i < P; i += blockDim.x) sh[i] = 0;
+    // HIST_SPLIT CTAs share a tile: contiguous runs of the scatter's sub-tiles
+    const uint32_t nsub = (uint32_t)((thi - tlo + T - 1) / T);
+    const uint32_t j0 = nsub * part / HIST_SPLIT, j1 = nsub * (part + 1) / HIST_SPLIT;
+    for (int i = tid; i < 2 * P; i += blockDim.x) sh[i] = 0;
     __syncthreads();
 
     constexpr int VEC = 16 / sizeof(K);
-    const uint64_t nvec = (hi - lo) / VEC;
-    const uint4 *kv = reinterpret_cast<const uint4 *>(keys + lo);
+    constexpr int NV = 4;  // 16-byte vectors per thread per sub-tile (T / VEC <= NV * HIST_THREADS)
     const uint32_t m = (uint32_t)(P - 1);
     auto count = [&](const uint4 &v) {
         if (sizeof(K) == 4) {
-            atomicAdd(&sh[v.x & m], 1u);
-            atomicAdd(&sh[v.y & m], 1u);
-            atomicAdd(&sh[v.z & m], 1u);
-            atomicAdd(&sh[v.w & m], 1u);
+            atomicAdd(&sub[v.x & m], 1u);
+            atomicAdd(&sub[v.y & m], 1u);
+            atomicAdd(&sub[v.z & m], 1u);
+            atomicAdd(&sub[v.w & m], 1u);
         } else {  // two 8-byte keys: low words are .x and .z
-            atomicAdd(&sh[v.x & m], 1u);
-            atomicAdd(&sh[v.z & m], 1u);
+            atomicAdd(&sub[v.x & m], 1u);
+            atomicAdd(&sub[v.z & m], 1u);
         }
     };
-    const uint64_t stride = blockDim.x;
-    uint64_t i = threadIdx.x;
-    for (; i + 3 * stride < nvec; i += 4 * stride) {
-        const uint4 v0 = __ldcs(kv + i), v1 = __ldcs(kv + i + stride);
-        const uint4 v2 = __ldcs(kv + i + 2 * stride), v3 = __ldcs(kv + i + 3 * stride);
-        count(v0);
-        count(v1);
-        count(v2);
-        count(v3);
+    auto load = [&](uint32_t j, uint4 (&v)[NV], uint32_t &nvec) {  // sub-tile j's key vectors
+        nvec = 0;
+        if (j >= j1) return;
+        const uint64_t a = tlo + (uint64_t)j * T, b = min(thi, a + T);
+        nvec = (uint32_t)((b - a) / VEC);
+        const uint4 *kv = reinterpret_cast<const uint4 *>(keys + a);
+#pragma unroll
+        for (int q = 0; q < NV; ++q)
+            if (tid + q * HIST_THREADS < nvec) v[q] = __ldcs(kv + tid + q * HIST_THREADS);
+    };
+    uint16_t *const out = c.sub_hist + ((size_t)rel * c.G + tile) * c.sub_ns * P;
+    uint4 v[NV], vn[NV];
+    uint32_t nv, nvn;
+    load(j0, v, nv);
+    for (uint32_t j = j0; j < j1; ++j) {
+        load(j + 1, vn, nvn);  // next sub-tile's loads in flight while this one is counted
+#pragma unroll
+        for (int q = 0; q < NV; ++q)
+            if (tid + q * HIST_THREADS < nv) count(v[q]);
+        const uint64_t a = tlo + (uint64_t)j * T, b = min(thi, a + T);
+        for (uint64_t t = a + (uint64_t)nv * VEC + tid; t < b; t += blockDim.x) atomicAdd(&sub[digit1(keys[t], P)], 1u);
+        __syncthreads();
+        // sub-tile histogram (u16 pairs) for the scatter's layout, then fold into acc
+        uint32_t *o32 = reinterpret_cast<uint32_t *>(out + (size_t)j * P);
+        for (int q = tid; q < P / 2; q += blockDim.x) {
+            const uint32_t x0 = sub[2 * q], x1 = sub[2 * q + 1];
+            o32[q] = x0 | x1 << 16;
+            acc[2 * q] += x0;
+            acc[2 * q + 1] += x1;
+            sub[2 * q] = 0;
+            sub[2 * q + 1] = 0;
+        }
+        __syncthreads();
+#pragma unroll
+        for (int q = 0; q < NV; ++q) v[q] = vn[q];
+        nv = nvn;
     }
-    for (; i < nvec; i += stride) count(__ldcs(kv + i));
-    for (uint64_t t = lo + nvec * VEC + threadIdx.x; t < hi; t += blockDim.x) atomicAdd(&sh[digit1(keys[t], P)], 1u);
-    __syncthreads();
     uint32_t *th = c.tile_hist + ((size_t)rel * c.G + tile) * P;
-    for (int p = threadIdx.x; p < P; p += blockDim.x) {
-        const uint32_t v = sh[p];
-        if (v) {
-            atomicAdd(&th[p], v);
-            atomicAdd(&c.rank_hist[rel * P + p], v);
+    for (int p = tid; p < P; p += blockDim.x) {
+        const uint32_t x = acc[p];
+        if (x) {
+            atomicAdd(&th[p], x);
+            atomicAdd(&c.rank_hist[rel * P + p], x);
         }
     }
 

@@ -157,7 +157,7 @@ void *dalloc(mgj_plan_s *h, size_t bytes, mgj_status *st) {
     return p;
 }
 
-size_t hist_smem(const Norm &n) { return (size_t)n.P * 4; }
+size_t hist_smem(const Norm &n) { return (size_t)n.P * 8; }
 size_t plan_smem(const Norm &n) { return (size_t)n.P * 5 * 8 + (size_t)n.P * 4 + (size_t)(n.P + 1) * 4; }
 size_t scatter_smem(const Norm &n) { return scat_smem_bytes(n.P, n.c.key_bytes); }
 size_t planA_smem(const Norm &n) { return ((size_t)local2_vcap(n.P) + 1) * 12; }
@@ -339,6 +339,9 @@ mgj_status mgj_plan(const mgj_config *cfg, const mgj_peers *peers, mgj_handle *o
         c.hA = reinterpret_cast<uint32_t *>(zb + z_ha);
     }
     c.tile_base = static_cast<uint32_t *>(dalloc(h, 2ull * c.G * P * 4, &st));
+    c.scat_T = scat_geom(P, n.c.key_bytes).T;
+    c.sub_ns = (int32_t)((std::max(n.c.r_capacity, n.c.s_capacity) / c.G + 8) / c.scat_T + 2);
+    c.sub_hist = static_cast<uint16_t *>(dalloc(h, 2ull * c.G * c.sub_ns * P * 2, &st));
     h->cdesc = static_cast<ChunkDesc *>(dalloc(h, 2 * n.max_chunks * sizeof(ChunkDesc), &st));
     c.owner = static_cast<int32_t *>(dalloc(h, P * 4, &st));
     c.send_off = static_cast<uint64_t *>(dalloc(h, 2ull * P * 8, &st));

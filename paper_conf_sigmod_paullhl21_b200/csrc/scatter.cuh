@@ -38,7 +38,7 @@ __host__ __device__ inline size_t scat_smem_bytes(int P, int key_bytes) {
     return 2 * (size_t)g.T * key_bytes                      // input stage: keys + payloads (SoA)
            + ((size_t)g.T + 2 * (size_t)(g.SG - 1) * P) * TB  // partition-sorted sub-tile (+ carries, group padding)
            + (size_t)P * sizeof(PInfo)
-           + (size_t)P * 4;                                  // bins / scatter positions
+           + (size_t)P * 4;                                  // next free slot per partition
 }
 
 // Block-wide exclusive scan of one register value per thread (1024 threads).
@@ -128,13 +128,20 @@ __global__ void __launch_bounds__(SCATTER_THREADS, 1) k_scatter(Ctx c) {
     constexpr uint32_t NONE = 0xffffffffu;
     using GV = typename Vec<GB>::T;
     typedef unsigned long long ull;
+    // `sorted` swizzle: the two 16-byte halves of every 32-byte group whose
+    // index has bit 2 set are swapped, so that the write-out's 16-byte loads
+    // (8 consecutive groups per quarter warp) hit distinct banks
+    auto swz = [](uint32_t s) -> uint32_t {
+        if constexpr (SG > 1) return s ^ (((s >> (SG == 4 ? 4 : 3)) & 1u) * (SG / 2));
+        else return s;
+    };
     extern __shared__ __align__(128) unsigned char smem[];
     const int P = c.P;
     K *const skey = reinterpret_cast<K *>(smem);
     K *const spay = skey + T;
     Tup *const sorted = reinterpret_cast<Tup *>(spay + T);
     PInfo *const pinfo = reinterpret_cast<PInfo *>(sorted + T + 2 * (SG - 1) * P);  // 16-byte aligned
-    uint32_t *const bins = reinterpret_cast<uint32_t *>(pinfo + P);
+    uint32_t *const off = reinterpret_cast<uint32_t *>(pinfo + P);  // next free slot per partition
     __shared__ __align__(8) uint64_t bar;
     __shared__ uint32_t tmp[32];
     const int tid = threadIdx.x;
@@ -185,7 +192,7 @@ __global__ void __launch_bounds__(SCATTER_THREADS, 1) k_scatter(Ctx c) {
             for (int k = 0; k < PPT; ++k)
 #pragma unroll
                 for (int i = 0; i < CW; ++i)
-                    if (i < (int)cc[k]) carry[k][i] = sorted[lim[k] - cc[k] + i];
+                    if (i < (int)cc[k]) carry[k][i] = sorted[swz(lim[k] - cc[k] + i)];
             pending = false;
         }
     };
@@ -218,6 +225,26 @@ __global__ void __launch_bounds__(SCATTER_THREADS, 1) k_scatter(Ctx c) {
         }
     };
 
+    // counts of sub-tile g for this thread's partitions (a1 wrote them, u16 per partition)
+    auto load_counts = [&](uint32_t g, uint32_t (&out)[PPT]) {
+#pragma unroll
+        for (int k = 0; k < PPT; ++k) out[k] = 0;
+        if (g >= ntot || tid * PPT >= P) return;
+        const int rel = g < nsub0 ? 0 : 1;
+        const uint32_t j = rel ? g - nsub0 : g;
+        const uint16_t *src = c.sub_hist + (((size_t)rel * c.G + tile) * c.sub_ns + j) * P + tid * PPT;
+        if constexpr (PPT == 1) {
+            out[0] = __ldg(src);
+        } else if constexpr (PPT == 2) {
+            const uint32_t v = __ldg(reinterpret_cast<const uint32_t *>(src));
+            out[0] = v & 0xffffu, out[1] = v >> 16;
+        } else {
+            const uint2 v = __ldg(reinterpret_cast<const uint2 *>(src));
+            out[0] = v.x & 0xffffu, out[1] = v.x >> 16, out[2] = v.y & 0xffffu, out[3] = v.y >> 16;
+        }
+    };
+    uint32_t ncnt[PPT];
+    load_counts(0, ncnt);
     if (tid == 0 && ntot > 0) issue(0);
     int cur_rel = -1;
     for (uint32_t g = 0; g < ntot; ++g) {
@@ -231,6 +258,39 @@ __global__ void __launch_bounds__(SCATTER_THREADS, 1) k_scatter(Ctx c) {
             cur_rel = rel;
         }
         fetch_carry();
+        // lay out this sub-tile's partitions (known from a1): carry + new tuples, group-rounded
+        uint32_t cnt[PPT], seg[PPT], tsum = 0;
+#pragma unroll
+        for (int k = 0; k < PPT; ++k) {
+            cnt[k] = cc[k] + ncnt[k];
+            seg[k] = (cnt[k] + SG - 1) & ~(uint32_t)(SG - 1);
+            tsum += seg[k];
+        }
+        load_counts(g + 1, ncnt);  // prefetch (consumed next iteration)
+        uint32_t total;
+        uint32_t o = block_scan_reg(tsum, tmp, total);  // its barriers: last write-out is done
+#pragma unroll
+        for (int k = 0; k < PPT; ++k) {
+            const int p = tid * PPT + k;
+            if (p < P) {
+#pragma unroll
+                for (int i = 0; i < CW; ++i)
+                    if (i < (int)cc[k]) sorted[swz(o + i)] = carry[k][i];
+                off[p] = o + cc[k];
+                const uint32_t full = cnt[k] & ~(uint32_t)(SG - 1);
+                PInfo in;
+                in.wb = base[k] - (ull)o * TB;
+                in.lim = o + cnt[k];
+                in.head = (hd[k] && full) ? (o << 2 | hd[k]) : NONE;
+                pinfo[p] = in;
+                base[k] += (ull)full * TB;
+                if (full) hd[k] = 0;
+                cc[k] = cnt[k] - full;
+                lim[k] = o + cnt[k];
+            }
+            o += seg[k];
+        }
+        pending = SG > 1;
         mbar_wait(&bar, g & 1);
         const uint32_t body = len & ~(uint32_t)(LU - 1);
         const K *gk = static_cast<const K *>(c.in_key[rel]) + first;
@@ -253,69 +313,29 @@ __global__ void __launch_bounds__(SCATTER_THREADS, 1) k_scatter(Ctx c) {
                 }
             }
         }
-#pragma unroll
-        for (int k = 0; k < PPT; ++k)
-            if (tid * PPT + k < P) bins[tid * PPT + k] = 0;
-        __syncthreads();  // S1: stage consumed, bins cleared, carries fetched
+        __syncthreads();  // S1: offsets and carries in place, stage consumed
         if (tid == 0 && g + 1 < ntot) issue(g + 1);
-        uint32_t rp[V];  // rank in bin << 16 | partition
 #pragma unroll
         for (int v = 0; v < V; ++v) {
             const uint32_t i = (uint32_t)((v / LU) * NT + tid) * LU + (v % LU);
-            rp[v] = NONE;
             if (i < len) {
-                const uint32_t p = digit1(kk[v], P);
-                rp[v] = (atomicAdd(&bins[p], 1u) << 16) | p;
-            }
-        }
-        __syncthreads();  // S2: counts final
-        uint32_t cnt[PPT], seg[PPT], tsum = 0;
-#pragma unroll
-        for (int k = 0; k < PPT; ++k) {
-            const int p = tid * PPT + k;
-            cnt[k] = p < P ? cc[k] + bins[p] : 0;
-            seg[k] = (cnt[k] + SG - 1) & ~(uint32_t)(SG - 1);
-            tsum += seg[k];
-        }
-        uint32_t total;
-        uint32_t o = block_scan_reg(tsum, tmp, total);
-#pragma unroll
-        for (int k = 0; k < PPT; ++k) {
-            const int p = tid * PPT + k;
-            if (p < P) {
-#pragma unroll
-                for (int i = 0; i < CW; ++i)
-                    if (i < (int)cc[k]) sorted[o + i] = carry[k][i];
-                bins[p] = o + cc[k];
-                const uint32_t full = cnt[k] & ~(uint32_t)(SG - 1);
-                PInfo in;
-                in.wb = base[k] - (ull)o * TB;
-                in.lim = o + cnt[k];
-                in.head = (hd[k] && full) ? (o << 2 | hd[k]) : NONE;
-                pinfo[p] = in;
-                base[k] += (ull)full * TB;
-                if (full) hd[k] = 0;
-                cc[k] = cnt[k] - full;
-                lim[k] = o + cnt[k];
-            }
-            o += seg[k];
-        }
-        pending = SG > 1;
-        __syncthreads();  // S3: positions, descriptors and carries in place
-#pragma unroll
-        for (int v = 0; v < V; ++v) {
-            if (rp[v] != NONE) {
                 Tup t;
                 t.x = kk[v];
                 t.y = pp[v];
-                sorted[bins[rp[v] & 0xffffu] + (rp[v] >> 16)] = t;
+                sorted[swz(atomicAdd(&off[digit1(kk[v], P)], 1u))] = t;
             }
         }
-        __syncthreads();  // S4
+        __syncthreads();  // S2
         const uint32_t ngroups = total / SG;
         for (uint32_t u = tid; u < ngroups; u += NT) {
             const uint32_t slot = u * SG;
-            const GV gv = *reinterpret_cast<const GV *>(sorted + slot);
+            GV gv;
+            if constexpr (SG > 1) {  // two conflict-free 16-byte halves (swizzled)
+                gv.a = *reinterpret_cast<const uint4 *>(sorted + swz(slot));
+                gv.b = *reinterpret_cast<const uint4 *>(sorted + swz(slot + SG / 2));
+            } else {
+                gv = *reinterpret_cast<const GV *>(sorted + slot);
+            }
             const uint32_t p = reinterpret_cast<const uint32_t *>(&gv)[0] & (uint32_t)(P - 1);  // digit1 of slot's key
             const PInfo in = pinfo[p];
             if (slot + SG <= in.lim) {
@@ -324,7 +344,7 @@ __global__ void __launch_bounds__(SCATTER_THREADS, 1) k_scatter(Ctx c) {
                     st_group<GB>(dst, gv);
                 } else {
                     for (uint32_t i = in.head & 3u; i < SG; ++i)
-                        reinterpret_cast<Tup *>(dst)[i] = sorted[slot + i];
+                        reinterpret_cast<Tup *>(dst)[i] = sorted[swz(slot + i)];
                 }
             }
         }

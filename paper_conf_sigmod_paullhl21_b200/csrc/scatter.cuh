@@ -7,6 +7,13 @@
 
 namespace mgj {
 
+#ifndef SCAT_WO_UNROLL
+#define SCAT_WO_UNROLL 1  // write-out groups per thread per step
+#endif
+#ifndef SCAT_ATOM_FIRST
+#define SCAT_ATOM_FIRST 0  // rank all tuples of a thread before storing them
+#endif
+
 // Scatter geometry for P partitions and a key width (kernel template
 // arguments; the host picks the instance with scatter_kernel<K>(P)):
 //   T   = sub-tile (tuples) staged in shared memory per step,
@@ -296,18 +303,21 @@ __global__ void __launch_bounds__(SCATTER_THREADS, 1) k_scatter(Ctx c) {
         const K *gk = static_cast<const K *>(c.in_key[rel]) + first;
         const K *gp = static_cast<const K *>(c.in_pay[rel]) + first;
         K kk[V], pp[V];
+        if (len == T) {  // full sub-tile: branch-free vector loads
 #pragma unroll
-        for (int u = 0; u < NU; ++u) {
-            const uint32_t i0 = (uint32_t)(u * NT + tid) * LU;
-            if (i0 + LU <= body) {
+            for (int u = 0; u < NU; ++u) {
+                const uint32_t i0 = (uint32_t)(u * NT + tid) * LU;
                 const uint4 a = *reinterpret_cast<const uint4 *>(skey + i0);
                 const uint4 b = *reinterpret_cast<const uint4 *>(spay + i0);
                 memcpy(&kk[u * LU], &a, 16);
                 memcpy(&pp[u * LU], &b, 16);
-            } else {
+            }
+        } else {
+#pragma unroll
+            for (int u = 0; u < NU; ++u) {
 #pragma unroll
                 for (int e = 0; e < LU; ++e) {  // < LU trailing tuples of the relation come from global
-                    const uint32_t i = i0 + e;
+                    const uint32_t i = (uint32_t)(u * NT + tid) * LU + e;
                     kk[u * LU + e] = i < body ? skey[i] : (i < len ? gk[i] : (K)0);
                     pp[u * LU + e] = i < body ? spay[i] : (i < len ? gp[i] : (K)0);
                 }
@@ -315,6 +325,23 @@ __global__ void __launch_bounds__(SCATTER_THREADS, 1) k_scatter(Ctx c) {
         }
         __syncthreads();  // S1: offsets and carries in place, stage consumed
         if (tid == 0 && g + 1 < ntot) issue(g + 1);
+#if SCAT_ATOM_FIRST
+        uint32_t pos[V];  // final slots: all atomics first, then the stores
+#pragma unroll
+        for (int v = 0; v < V; ++v) {
+            const uint32_t i = (uint32_t)((v / LU) * NT + tid) * LU + (v % LU);
+            pos[v] = (len == T || i < len) ? atomicAdd(&off[digit1(kk[v], P)], 1u) : NONE;
+        }
+#pragma unroll
+        for (int v = 0; v < V; ++v) {
+            if (pos[v] != NONE) {
+                Tup t;
+                t.x = kk[v];
+                t.y = pp[v];
+                sorted[swz(pos[v])] = t;
+            }
+        }
+#else
 #pragma unroll
         for (int v = 0; v < V; ++v) {
             const uint32_t i = (uint32_t)((v / LU) * NT + tid) * LU + (v % LU);
@@ -325,26 +352,42 @@ __global__ void __launch_bounds__(SCATTER_THREADS, 1) k_scatter(Ctx c) {
                 sorted[swz(atomicAdd(&off[digit1(kk[v], P)], 1u))] = t;
             }
         }
+#endif
         __syncthreads();  // S2
+        // write-out, two groups per thread per step (independent load chains)
         const uint32_t ngroups = total / SG;
-        for (uint32_t u = tid; u < ngroups; u += NT) {
-            const uint32_t slot = u * SG;
-            GV gv;
-            if constexpr (SG > 1) {  // two conflict-free 16-byte halves (swizzled)
-                gv.a = *reinterpret_cast<const uint4 *>(sorted + swz(slot));
-                gv.b = *reinterpret_cast<const uint4 *>(sorted + swz(slot + SG / 2));
-            } else {
-                gv = *reinterpret_cast<const GV *>(sorted + slot);
+        constexpr int WU = SCAT_WO_UNROLL;
+        for (uint32_t u0 = tid; u0 < ngroups; u0 += WU * NT) {
+            GV gv[WU];
+            PInfo in[WU];
+            uint32_t slot[WU];
+            bool on[WU];
+#pragma unroll
+            for (int r = 0; r < WU; ++r) {
+                slot[r] = (u0 + r * NT) * SG;
+                on[r] = u0 + r * NT < ngroups;
+                if (on[r]) {
+                    if constexpr (SG > 1) {  // two conflict-free 16-byte halves (swizzled)
+                        gv[r].a = *reinterpret_cast<const uint4 *>(sorted + swz(slot[r]));
+                        gv[r].b = *reinterpret_cast<const uint4 *>(sorted + swz(slot[r] + SG / 2));
+                    } else {
+                        gv[r] = *reinterpret_cast<const GV *>(sorted + slot[r]);
+                    }
+                }
             }
-            const uint32_t p = reinterpret_cast<const uint32_t *>(&gv)[0] & (uint32_t)(P - 1);  // digit1 of slot's key
-            const PInfo in = pinfo[p];
-            if (slot + SG <= in.lim) {
-                char *dst = reinterpret_cast<char *>(in.wb + (ull)slot * TB);
-                if ((in.head >> 2) != slot) {
-                    st_group<GB>(dst, gv);
-                } else {
-                    for (uint32_t i = in.head & 3u; i < SG; ++i)
-                        reinterpret_cast<Tup *>(dst)[i] = sorted[swz(slot + i)];
+#pragma unroll
+            for (int r = 0; r < WU; ++r)
+                if (on[r]) in[r] = pinfo[reinterpret_cast<const uint32_t *>(&gv[r])[0] & (uint32_t)(P - 1)];
+#pragma unroll
+            for (int r = 0; r < WU; ++r) {
+                if (on[r] && slot[r] + SG <= in[r].lim) {
+                    char *dst = reinterpret_cast<char *>(in[r].wb + (ull)slot[r] * TB);
+                    if ((in[r].head >> 2) != slot[r]) {
+                        st_group<GB>(dst, gv[r]);
+                    } else {
+                        for (uint32_t i = in[r].head & 3u; i < SG; ++i)
+                            reinterpret_cast<Tup *>(dst)[i] = sorted[swz(slot[r] + i)];
+                    }
                 }
             }
         }

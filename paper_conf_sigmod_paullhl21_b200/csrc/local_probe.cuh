@@ -322,9 +322,25 @@ __global__ void __launch_bounds__(LOCAL_THREADS, 1) k_local(Ctx c, const ChunkDe
             }
         }
         __syncthreads();  // S2
-        for (int q = tid; q < Q; q += LOCAL_THREADS) abin[q] = (bins[q] + ALIGN - 1) & ~(uint32_t)(ALIGN - 1);
-        __syncthreads();
-        const uint32_t tot = block_excl_scan_u32(abin, Q, tmp);
+        if (tid < 32) {  // one warp: padded run starts (exclusive scan over the Q bins)
+            const int per = (Q + 31) / 32, q0 = tid * per;
+            uint32_t sum = 0;
+            for (int q = q0; q < min(Q, q0 + per); ++q) sum += (bins[q] + ALIGN - 1) & ~(uint32_t)(ALIGN - 1);
+            uint32_t incl = sum;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const uint32_t y = __shfl_up_sync(0xffffffffu, incl, o);
+                if (tid >= o) incl += y;
+            }
+            uint32_t run = incl - sum;
+            for (int q = q0; q < min(Q, q0 + per); ++q) {
+                abin[q] = run;
+                run += (bins[q] + ALIGN - 1) & ~(uint32_t)(ALIGN - 1);
+            }
+            if (tid == 31) tmp[0] = incl;
+        }
+        __syncthreads();  // S2b
+        const uint32_t tot = tmp[0];
         if (!SPLIT) {
             const uint32_t *cb = c.chunk_base + (size_t)rel * c.cb_stride;
             const uint32_t cbp = cb[d.pi], nchp = cb[d.pi + 1] - cbp;
@@ -353,7 +369,7 @@ __global__ void __launch_bounds__(LOCAL_THREADS, 1) k_local(Ctx c, const ChunkDe
                 // chunked pass drops a first pass's padding (DESIGN.md §2 R2)
                 if (ALIGN == 2 && r == 0 && (bins[q] & 1u)) {
                     Tup pad = t[v];
-                    pad.x ^= 1;
+                    pad.x ^= (rel == 1 && P >= 4) ? 2 : 1;
                     sorted[abin[q] + bins[q]] = pad;
                 }
             }
@@ -529,6 +545,10 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
     uint16_t *nxt = reinterpret_cast<uint16_t *>(head + T);
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const int B2 = c.meta[MT_B2];
+    // S padding slots (8-byte tuples): with P >= 4 their key has bit 1 flipped
+    // and R's bit 0 (k_local), so neither can equal any key of the other side
+    // and S padding is probed harmlessly; only P < 4 needs the skip bitmap
+    const bool SBITS = Layout<K>::ALIGN == 2 && c.P < 4;
     const int Q = 1 << c.meta[MT_QB], shift = c.B1 + B2;  // Q: runs per chunk of the chunked pass
     const uint32_t nitems = min(__ldcg(&c.ticket[TK_ITEMS]), c.max_items);
     const uint32_t mine = nitems > blockIdx.x ? (nitems - blockIdx.x + gridDim.x - 1) / gridDim.x : 0;
@@ -555,7 +575,7 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
             const int s = j % PROBE_NST;
             if (j >= PROBE_NST) mbar_wait(&empty[s], ((j / PROBE_NST) - 1) & 1);
             uint32_t *pb = padbits + s * PW;
-            if (ALIGN == 2) {
+            if (SBITS) {
                 for (int w = lane; w < PW; w += 32) pb[w] = 0;
                 __syncwarp();
             }
@@ -582,7 +602,7 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
                             sz = ahi - alo;
                             src = (uint64_t)(x.cb[rel] + k) * c.chunk_region + st + alo;
                         }
-                        pad = (ALIGN == 2 && rel == 1 && v < slots && v >= alo && v < ahi) ? v - alo : 0xffffffffu;
+                        pad = (SBITS && rel == 1 && v < slots && v >= alo && v < ahi) ? v - alo : 0xffffffffu;
                     }
                     uint32_t incl = sz;
 #pragma unroll
@@ -637,7 +657,7 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
         const uint32_t *pb = padbits + s * PW;
         uint32_t m_item = 0;
         for (uint32_t x = ct; x < stot; x += NCONS) {
-            if (Layout<K>::ALIGN == 2 && ((pb[x >> 5] >> (x & 31)) & 1u)) continue;  // padding slot
+            if (SBITS && ((pb[x >> 5] >> (x & 31)) & 1u)) continue;  // padding slot (P < 4 only)
             const Tup sv = st[x];
             const uint32_t hv = head[tab_hash(sv.x, shift, LOGT)];
             uint32_t i = (hv >> 16) == tag ? (hv & 0xffffu) : END;
@@ -685,7 +705,7 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
                 K *ob = static_cast<K *>(c.out_b);
                 unsigned long long pos = s_base + (cwi ? s_wtot[cwi - 1] : 0) + incl - m_item;
                 for (uint32_t x = ct; x < stot; x += NCONS) {
-                    if (Layout<K>::ALIGN == 2 && ((pb[x >> 5] >> (x & 31)) & 1u)) continue;
+                    if (SBITS && ((pb[x >> 5] >> (x & 31)) & 1u)) continue;
                     const Tup sv = st[x];
                     const uint32_t hv = head[tab_hash(sv.x, shift, LOGT)];
                     for (uint32_t i = (hv >> 16) == tag ? (hv & 0xffffu) : END; i != END; i = nxt[i]) {

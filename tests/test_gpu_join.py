@@ -139,8 +139,9 @@ def test_phases_m1(mgj, b1):
                     valid = slots - (e0 & 1)
                     run = loc[li * CR + st: li * CR + st + valid]
                     assert np.all(((run[:, 0] >> B1) & (Q - 1)) == q)
-                    if valid < slots:  # padding slot: a key of the run with bit 0 flipped
-                        assert (loc[li * CR + st + valid, 0] ^ 1) in run[:, 0]
+                    if valid < slots:  # padding slot: a key of the run with bit 0 (R) / bit 1 (S, P >= 4) flipped
+                        flip = 2 if (rel == 1 and P >= 4) else 1
+                        assert (loc[li * CR + st + valid, 0] ^ flip) in run[:, 0]
                     got.append(run)
                 got = np.concatenate(got)
                 src = recv[a:b, 0].astype(np.uint64) | (recv[a:b, 1].astype(np.uint64) << np.uint64(32))
@@ -182,7 +183,7 @@ def test_two_level_local_phases(mgj, ba):
             real = seg[(seg[:, 0] & (P - 1)) == p]
             pads = seg[(seg[:, 0] & (P - 1)) != p]
             assert np.all(((real[:, 0] >> B1) & ((1 << BA) - 1)) == qa)
-            assert np.all((pads[:, 0] & (P - 1)) == (p ^ 1))
+            assert np.all((pads[:, 0] & (P - 1)) == (p ^ (2 if (rel == 1 and P >= 4) else 1)))
             exp = recv[((recv[:, 0] & (P - 1)) == p) & (((recv[:, 0] >> B1) & ((1 << BA) - 1)) == qa)]
             pack = lambda x: np.sort(x[:, 0].astype(np.uint64) | (x[:, 1].astype(np.uint64) << np.uint64(32)))
             np.testing.assert_array_equal(pack(real), pack(exp))

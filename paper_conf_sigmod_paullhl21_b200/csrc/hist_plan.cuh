@@ -6,6 +6,10 @@
 
 namespace mgj {
 
+#ifndef HIST_MINB
+#define HIST_MINB 1  // k_hist: minimum resident CTAs per SM (register cap)
+#endif
+
 // ---------------------------------------------------------------------------
 // a1: per-GPU radix histogram (§3.2 "Histogram generation",
 // P:356-370, built in shared memory after Rui et al. [38]; bin count from the
@@ -18,7 +22,7 @@ namespace mgj {
 // arena mailbox and raises SIG_HIST there (histogram exchange X4 fused).
 // ---------------------------------------------------------------------------
 template <typename K>
-__global__ void __launch_bounds__(HIST_THREADS) k_hist(Ctx c) {
+__global__ void __launch_bounds__(HIST_THREADS, HIST_MINB) k_hist(Ctx c) {
     extern __shared__ uint32_t sh[];  // sub[P] (current sub-tile), acc[P] (this CTA's share of the tile)
     const int P = c.P, T = c.scat_T;
     uint32_t *const sub = sh, *const acc = sh + P;

@@ -533,6 +533,7 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
     extern __shared__ __align__(128) unsigned char smem[];
     __shared__ __align__(8) uint64_t full[PROBE_NST], empty[PROBE_NST];
     __shared__ uint32_t totals[PROBE_NST][2];
+    __shared__ uint32_t stage_p[PROBE_NST];  // global partition (digit1) of the stage's item
     __shared__ uint32_t s_wtot[32];
     __shared__ unsigned long long s_base;
     __shared__ int s_write;
@@ -549,6 +550,15 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
     // and R's bit 0 (k_local), so neither can equal any key of the other side
     // and S padding is probed harmlessly; only P < 4 needs the skip bitmap
     const bool SBITS = Layout<K>::ALIGN == 2 && c.P < 4;
+    const int plo = c.meta[MT_PLO], BAp = c.meta[MT_BA];
+    // packed table (4-byte keys whose bits above the radix digits fit 16 bits,
+    // e.g. B1 + B2 >= 16): the build overwrites each R slot's key with
+    // (khi << 16 | next), khi = key >> (B1 + B2), so a chain step is one
+    // 8-byte shared load that yields khi, the next link and the payload.  All
+    // real keys of a co-partition share their low B1 + B2 bits, so equal khi
+    // means equal keys; padding slots (digit1 != p) are left out on both sides.
+    const bool packed = sizeof(K) == 4 && c.B1 + B2 >= 16;
+    const int P = c.P;
     const int Q = 1 << c.meta[MT_QB], shift = c.B1 + B2;  // Q: runs per chunk of the chunked pass
     const uint32_t nitems = min(__ldcg(&c.ticket[TK_ITEMS]), c.max_items);
     const uint32_t mine = nitems > blockIdx.x ? (nitems - blockIdx.x + gridDim.x - 1) / gridDim.x : 0;
@@ -624,6 +634,7 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
                 }
                 if (lane == 0) totals[s][rel] = run;
             }
+            if (lane == 0) stage_p[s] = (uint32_t)(plo + (BAp ? x.it.pi >> BAp : x.it.pi));
             __syncwarp();
             if (lane == 0) mbar_arrive(&full[s]);
             x = xn;
@@ -646,29 +657,57 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
         const Tup *rt = stages + ((size_t)s * 2 + 0) * SL;
         const Tup *st = stages + ((size_t)s * 2 + 1) * SL;
         const uint32_t rtot = totals[s][0], stot = totals[s][1];
+        const uint32_t pitem = stage_p[s];
+        auto fold = [](uint32_t khi) { return (khi ^ (khi >> LOGT)) & (uint32_t)(T - 1); };
         // build
-        for (uint32_t slot = ct; slot < rtot; slot += NCONS) {
-            const uint32_t h = tab_hash(rt[slot].x, shift, LOGT);
-            const uint32_t old = atomicExch(&head[h], (tag << 16) | slot);
-            nxt[slot] = (old >> 16) == tag ? (uint16_t)(old & 0xffffu) : END;
+        if (packed) {
+            uint32_t *rw = reinterpret_cast<uint32_t *>(stages + ((size_t)s * 2 + 0) * SL);
+            for (uint32_t slot = ct; slot < rtot; slot += NCONS) {
+                const uint32_t k = (uint32_t)rt[slot].x;
+                if ((k & (uint32_t)(P - 1)) != pitem) continue;  // R padding slot
+                const uint32_t khi = k >> shift;
+                const uint32_t old = atomicExch(&head[fold(khi)], (tag << 16) | slot);
+                rw[2 * slot] = ((old >> 16) == tag ? (old & 0xffffu) : (uint32_t)END) | (khi << 16);
+            }
+        } else {
+            for (uint32_t slot = ct; slot < rtot; slot += NCONS) {
+                const uint32_t h = tab_hash(rt[slot].x, shift, LOGT);
+                const uint32_t old = atomicExch(&head[h], (tag << 16) | slot);
+                nxt[slot] = (old >> 16) == tag ? (uint16_t)(old & 0xffffu) : END;
+            }
         }
         named_bar_sync(1, NCONS);
-        // probe
         const uint32_t *pb = padbits + s * PW;
+        // every R payload matching S slot x: f(payR)
+        auto walk = [&](uint32_t x, const Tup &sv, auto &&f) {
+            if (packed) {
+                const uint32_t k = (uint32_t)sv.x;
+                if ((k & (uint32_t)(P - 1)) != pitem) return;  // S padding slot
+                const uint32_t khi = k >> shift;
+                const uint32_t hv = head[fold(khi)];
+                for (uint32_t i = (hv >> 16) == tag ? (hv & 0xffffu) : END; i != END;) {
+                    const Tup rv = rt[i];
+                    const uint32_t l = (uint32_t)rv.x;
+                    if ((l >> 16) == khi) f(rv.y);
+                    i = l & 0xffffu;
+                }
+            } else {
+                if (SBITS && ((pb[x >> 5] >> (x & 31)) & 1u)) return;  // padding slot (P < 4 only)
+                const uint32_t hv = head[tab_hash(sv.x, shift, LOGT)];
+                for (uint32_t i = (hv >> 16) == tag ? (hv & 0xffffu) : END; i != END; i = nxt[i]) {
+                    const Tup rv = rt[i];
+                    if (rv.x == sv.x) f(rv.y);
+                }
+            }
+        };
+        // probe
         uint32_t m_item = 0;
         for (uint32_t x = ct; x < stot; x += NCONS) {
-            if (SBITS && ((pb[x >> 5] >> (x & 31)) & 1u)) continue;  // padding slot (P < 4 only)
             const Tup sv = st[x];
-            const uint32_t hv = head[tab_hash(sv.x, shift, LOGT)];
-            uint32_t i = (hv >> 16) == tag ? (hv & 0xffffu) : END;
-            while (i != END) {
-                const Tup rv = rt[i];
-                if (rv.x == sv.x) {
-                    ++m_item;
-                    my_chk += chk_term(rv.y, sv.y);
-                }
-                i = nxt[i];
-            }
+            walk(x, sv, [&](K a) {
+                ++m_item;
+                my_chk += chk_term(a, (K)sv.y);
+            });
         }
         my_cnt += m_item;
         if (MAT) {
@@ -705,18 +744,13 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
                 K *ob = static_cast<K *>(c.out_b);
                 unsigned long long pos = s_base + (cwi ? s_wtot[cwi - 1] : 0) + incl - m_item;
                 for (uint32_t x = ct; x < stot; x += NCONS) {
-                    if (SBITS && ((pb[x >> 5] >> (x & 31)) & 1u)) continue;
                     const Tup sv = st[x];
-                    const uint32_t hv = head[tab_hash(sv.x, shift, LOGT)];
-                    for (uint32_t i = (hv >> 16) == tag ? (hv & 0xffffu) : END; i != END; i = nxt[i]) {
-                        const Tup rv = rt[i];
-                        if (rv.x == sv.x) {
-                            ok[pos] = (K)sv.x;
-                            oa[pos] = (K)rv.y;
-                            ob[pos] = (K)sv.y;
-                            ++pos;
-                        }
-                    }
+                    walk(x, sv, [&](K a) {
+                        ok[pos] = (K)sv.x;
+                        oa[pos] = a;
+                        ob[pos] = (K)sv.y;
+                        ++pos;
+                    });
                 }
             }
         }

@@ -19,8 +19,11 @@ constexpr int LOCAL_THREADS = 1024;
 constexpr int LOCAL_VMAX = 12;          // local-pass tuples per thread (chunk C <= 12 * LOCAL_THREADS), 8-byte tuples
 __host__ __device__ constexpr int local_vmax(int tuple_bytes) { return LOCAL_VMAX * 8 / tuple_bytes; }
 constexpr int PROBE_THREADS = 1024;     // warps 0..PROBE_NP-1 = TMA producers, the rest build/probe
-constexpr int PROBE_NP = 3;             // producer warps (<= PROBE_NST: parity waits are one phase ahead)
 constexpr int PROBE_NST = 3;            // pipeline stages (items in flight per CTA)
+#ifndef PROBE_PPI
+#define PROBE_PPI 2                     // producer warps per item (1: R and S; 2: one relation each)
+#endif
+constexpr int PROBE_NP = PROBE_NST * PROBE_PPI;  // producer warps (item streams <= PROBE_NST: parity waits one phase ahead)
 constexpr int PROBE_SLOTS8 = 4224;      // stage capacity per relation (slots) for 8-byte tuples; half for 16-byte
 constexpr int PROBE_HEAD8 = 128;        // headroom: co-partition target = capacity - headroom (padding, spread)
 constexpr int PROBE_MAXP = 1024;        // chunk pieces per relation per item

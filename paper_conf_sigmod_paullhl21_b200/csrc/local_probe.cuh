@@ -565,7 +565,7 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
     const ItemX *items = reinterpret_cast<const ItemX *>(c.items);
     if (tid == 0) {
         for (int s = 0; s < PROBE_NST; ++s) {
-            mbar_init(&full[s], 1);
+            mbar_init(&full[s], PROBE_PPI);
             mbar_init(&empty[s], 1);
         }
         fence_mbar_init();
@@ -577,19 +577,23 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
         // ------------------------------------------------------- producers
         constexpr int ALIGN = Layout<K>::ALIGN;
         const uint64_t pol = policy_evict_first();
+        // PROBE_PPI producer warps per item: 1 (both relations) or 2 (R / S)
+        constexpr int NPI = PROBE_NP / PROBE_PPI;  // item streams (<= PROBE_NST)
+        const int pw = warp / PROBE_PPI;
+        const int rel0 = PROBE_PPI == 2 ? (warp & 1) : 0, rel1 = PROBE_PPI == 2 ? rel0 + 1 : 2;
         ItemX x;
-        if (warp < (int)mine) x = items[blockIdx.x + warp * gridDim.x];
-        for (uint32_t j = warp; j < mine; j += PROBE_NP) {
+        if (pw < (int)mine) x = items[blockIdx.x + pw * gridDim.x];
+        for (uint32_t j = pw; j < mine; j += NPI) {
             ItemX xn;
-            if (j + PROBE_NP < mine) xn = items[blockIdx.x + (j + PROBE_NP) * gridDim.x];  // prefetch
+            if (j + NPI < mine) xn = items[blockIdx.x + (j + NPI) * gridDim.x];  // prefetch
             const int s = j % PROBE_NST;
             if (j >= PROBE_NST) mbar_wait(&empty[s], ((j / PROBE_NST) - 1) & 1);
             uint32_t *pb = padbits + s * PW;
-            if (SBITS) {
+            if (SBITS && rel1 == 2) {
                 for (int w = lane; w < PW; w += 32) pb[w] = 0;
                 __syncwarp();
             }
-            for (int rel = 0; rel < 2; ++rel) {
+            for (int rel = rel0; rel < rel1; ++rel) {
                 const Side sd = rel ? x.it.s : x.it.r;
                 const uint16_t *E0 = c.eoff[rel] + (size_t)(Q + 1) * x.cb[rel] + (size_t)x.it.q * x.nch[rel];
                 const uint16_t *E1 = E0 + x.nch[rel];
@@ -634,7 +638,7 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
                 }
                 if (lane == 0) totals[s][rel] = run;
             }
-            if (lane == 0) stage_p[s] = (uint32_t)(plo + (BAp ? x.it.pi >> BAp : x.it.pi));
+            if (lane == 0 && rel0 == 0) stage_p[s] = (uint32_t)(plo + (BAp ? x.it.pi >> BAp : x.it.pi));
             __syncwarp();
             if (lane == 0) mbar_arrive(&full[s]);
             x = xn;

@@ -13,7 +13,7 @@ constexpr int MAX_RANKS = MGJ_MAX_RANKS;
 constexpr int MAX_B1 = 12;              // 2^12 global partitions at most
 constexpr int MAX_B2 = 11;              // local fan-out per pass
 constexpr int HIST_THREADS = 512;
-constexpr int HIST_SPLIT = 4;           // CTAs per histogram tile
+constexpr int HIST_SPLIT = 2;           // k_hist CTAs per tile (resident together on one SM)
 constexpr int SCATTER_THREADS = 1024;
 constexpr int LOCAL_THREADS = 1024;
 constexpr int LOCAL_VMAX = 12;          // local-pass tuples per thread (chunk C <= 12 * LOCAL_THREADS), 8-byte tuples

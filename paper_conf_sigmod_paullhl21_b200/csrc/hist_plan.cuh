@@ -3,78 +3,109 @@
 #pragma once
 
 #include "common.cuh"
+#include "scatter.cuh"  // scat_geom: the sub-tiles a1 counts
+#include "tma.cuh"
 
 namespace mgj {
 
-#ifndef HIST_MINB
-#define HIST_MINB 1  // k_hist: minimum resident CTAs per SM (register cap)
-#endif
+constexpr int HIST_NB = 3;  // k_hist: TMA ring depth (sub-tiles in flight per CTA; 2 CTAs per SM)
 
 // ---------------------------------------------------------------------------
 // a1: per-GPU radix histogram (§3.2 "Histogram generation",
 // P:356-370, built in shared memory after Rui et al. [38]; bin count from the
 // Eq. 1 analogue).  H[rel][p] = #{t in rel_g : digit1(t.key) = p}.
-// grid = (G, 2): CTA (c, rel) counts tile c of relation rel (the same tiles
-// the scatter kernel processes) reading only the key column with 16-byte
-// streaming loads, and stores its per-tile histogram (so the scatter knows
-// its exact output offsets without atomics) and adds it into the rank
-// histogram.  The last CTA stores the rank histogram into every peer's
-// arena mailbox and raises SIG_HIST there (histogram exchange X4 fused).
+// HIST_SPLIT CTAs (two per SM, resident together) share tile c of R and of S
+// (the tiles the scatter kernel processes); each counts a contiguous run of
+// the scatter's sub-tiles, whose key columns a TMA ring brings into shared
+// memory HIST_NB sub-tiles ahead.  Per sub-tile it stores the u16 counts (the
+// scatter lays each sub-tile out from them before reading it) and folds
+// them into the tile histogram (exact scatter offsets) and the rank
+// histogram.  The last CTA
+// stores the rank histogram into every peer's arena mailbox and raises
+// SIG_HIST there (histogram exchange X4 fused).
 // ---------------------------------------------------------------------------
 template <typename K>
-__global__ void __launch_bounds__(HIST_THREADS, HIST_MINB) k_hist(Ctx c) {
-    extern __shared__ uint32_t sh[];  // sub[P] (current sub-tile), acc[P] (this CTA's share of the tile)
+__global__ void __launch_bounds__(HIST_THREADS, 2) k_hist(Ctx c) {
+    extern __shared__ __align__(128) unsigned char hsm[];  // ring[HIST_NB][T] keys | sub[P] | acc[P]
+    __shared__ __align__(8) uint64_t bar[HIST_NB];
     const int P = c.P, T = c.scat_T;
-    uint32_t *const sub = sh, *const acc = sh + P;
-    const int rel = blockIdx.y, tile = blockIdx.x / HIST_SPLIT, part = blockIdx.x % HIST_SPLIT;
-    const int tid = threadIdx.x;
-    const K *keys = static_cast<const K *>(c.in_key[rel]);
-    uint64_t tlo, thi;
-    tile_range(c.n_in[rel], c.G, tile, tlo, thi);
-    // HIST_SPLIT CTAs share a tile: contiguous runs of the scatter's sub-tiles
-    const uint32_t nsub = (uint32_t)((thi - tlo + T - 1) / T);
-    const uint32_t j0 = nsub * part / HIST_SPLIT, j1 = nsub * (part + 1) / HIST_SPLIT;
-    for (int i = tid; i < 2 * P; i += blockDim.x) sh[i] = 0;
+    K *const ring = reinterpret_cast<K *>(hsm);
+    uint32_t *const sub = reinterpret_cast<uint32_t *>(ring + (size_t)HIST_NB * T);
+    uint32_t *const acc = sub + P;
+    const int tid = threadIdx.x, tile = blockIdx.x / HIST_SPLIT, part = blockIdx.x % HIST_SPLIT;
+    constexpr int LU = 16 / (int)sizeof(K);
+    uint64_t lo0, hi0, lo1, hi1;
+    tile_range(c.n_in[0], c.G, tile, lo0, hi0);
+    tile_range(c.n_in[1], c.G, tile, lo1, hi1);
+    // HIST_SPLIT CTAs share a tile: contiguous runs of its sub-tiles
+    const uint32_t ns0 = (uint32_t)((hi0 - lo0 + T - 1) / T), ns1 = (uint32_t)((hi1 - lo1 + T - 1) / T);
+    const uint32_t ja0 = ns0 * part / HIST_SPLIT, jb0 = ns0 * (part + 1) / HIST_SPLIT;
+    const uint32_t ja1 = ns1 * part / HIST_SPLIT, jb1 = ns1 * (part + 1) / HIST_SPLIT;
+    const uint32_t nsub0 = jb0 - ja0;
+    const uint32_t ntot = nsub0 + (jb1 - ja1);
+    auto subtile = [&](uint32_t g, int &rel, uint32_t &j, uint64_t &first, uint32_t &len) {
+        rel = g < nsub0 ? 0 : 1;
+        j = rel ? g - nsub0 + ja1 : g + ja0;
+        first = (rel ? lo1 : lo0) + (uint64_t)j * T;
+        len = (uint32_t)min((uint64_t)T, (rel ? hi1 : hi0) - first);
+    };
+    const uint64_t pol = policy_evict_first();
+    auto issue = [&](uint32_t g) {  // thread 0: TMA the 16-byte-aligned body of sub-tile g's keys
+        int rel;
+        uint32_t j, len;
+        uint64_t first;
+        subtile(g, rel, j, first, len);
+        uint64_t *b = &bar[g % HIST_NB];
+        const uint32_t bytes = (len & ~(uint32_t)(LU - 1)) * (uint32_t)sizeof(K);
+        mbar_arrive_expect_tx(b, bytes);
+        if (bytes)
+            tma_load_1d(ring + (size_t)(g % HIST_NB) * T, static_cast<const K *>(c.in_key[rel]) + first, bytes, b, pol);
+    };
+    for (int i = tid; i < 2 * P; i += blockDim.x) sub[i] = 0;
+    if (tid == 0) {
+        for (int i = 0; i < HIST_NB; ++i) mbar_init(&bar[i], 1);
+        fence_mbar_init();
+        for (uint32_t g = 0; g < ntot && g < (uint32_t)HIST_NB; ++g) issue(g);
+    }
     __syncthreads();
-
-    constexpr int VEC = 16 / sizeof(K);
-    constexpr int NV = 4;  // 16-byte vectors per thread per sub-tile (T / VEC <= NV * HIST_THREADS)
     const uint32_t m = (uint32_t)(P - 1);
-    auto count = [&](const uint4 &v) {
-        if (sizeof(K) == 4) {
-            atomicAdd(&sub[v.x & m], 1u);
-            atomicAdd(&sub[v.y & m], 1u);
-            atomicAdd(&sub[v.z & m], 1u);
-            atomicAdd(&sub[v.w & m], 1u);
-        } else {  // two 8-byte keys: low words are .x and .z
-            atomicAdd(&sub[v.x & m], 1u);
-            atomicAdd(&sub[v.z & m], 1u);
+    auto flush_acc = [&](int rel) {  // tile histogram (this CTA owns the tile) and rank histogram
+        uint32_t *th = c.tile_hist + ((size_t)rel * c.G + tile) * P;
+        for (int p = tid; p < P; p += blockDim.x) {
+            const uint32_t x = acc[p];
+            if (x) {
+                atomicAdd(&th[p], x);
+                atomicAdd(&c.rank_hist[rel * P + p], x);
+            }
+            acc[p] = 0;
         }
     };
-    auto load = [&](uint32_t j, uint4 (&v)[NV], uint32_t &nvec) {  // sub-tile j's key vectors
-        nvec = 0;
-        if (j >= j1) return;
-        const uint64_t a = tlo + (uint64_t)j * T, b = min(thi, a + T);
-        nvec = (uint32_t)((b - a) / VEC);
-        const uint4 *kv = reinterpret_cast<const uint4 *>(keys + a);
-#pragma unroll
-        for (int q = 0; q < NV; ++q)
-            if (tid + q * HIST_THREADS < nvec) v[q] = __ldcs(kv + tid + q * HIST_THREADS);
-    };
-    uint16_t *const out = c.sub_hist + ((size_t)rel * c.G + tile) * c.sub_ns * P;
-    uint4 v[NV], vn[NV];
-    uint32_t nv, nvn;
-    load(j0, v, nv);
-    for (uint32_t j = j0; j < j1; ++j) {
-        load(j + 1, vn, nvn);  // next sub-tile's loads in flight while this one is counted
-#pragma unroll
-        for (int q = 0; q < NV; ++q)
-            if (tid + q * HIST_THREADS < nv) count(v[q]);
-        const uint64_t a = tlo + (uint64_t)j * T, b = min(thi, a + T);
-        for (uint64_t t = a + (uint64_t)nv * VEC + tid; t < b; t += blockDim.x) atomicAdd(&sub[digit1(keys[t], P)], 1u);
-        __syncthreads();
+    for (uint32_t g = 0; g < ntot; ++g) {
+        int rel;
+        uint32_t j, len;
+        uint64_t first;
+        subtile(g, rel, j, first, len);
+        const K *buf = ring + (size_t)(g % HIST_NB) * T;
+        mbar_wait(&bar[g % HIST_NB], (g / HIST_NB) & 1);
+        const uint32_t body = len & ~(uint32_t)(LU - 1);
+        for (uint32_t i0 = (uint32_t)tid * LU; i0 < body; i0 += (uint32_t)blockDim.x * LU) {
+            const uint4 v = *reinterpret_cast<const uint4 *>(buf + i0);
+            if (sizeof(K) == 4) {
+                atomicAdd(&sub[v.x & m], 1u);
+                atomicAdd(&sub[v.y & m], 1u);
+                atomicAdd(&sub[v.z & m], 1u);
+                atomicAdd(&sub[v.w & m], 1u);
+            } else {  // two 8-byte keys: low words are .x and .z
+                atomicAdd(&sub[v.x & m], 1u);
+                atomicAdd(&sub[v.z & m], 1u);
+            }
+        }
+        if (tid < (int)(len - body))  // < LU trailing tuples of the relation: from global
+            atomicAdd(&sub[digit1(static_cast<const K *>(c.in_key[rel])[first + body + tid], P)], 1u);
+        __syncthreads();  // counts final; ring slot g % NB free
+        if (tid == 0 && g + HIST_NB < ntot) issue(g + HIST_NB);
         // sub-tile histogram (u16 pairs) for the scatter's layout, then fold into acc
-        uint32_t *o32 = reinterpret_cast<uint32_t *>(out + (size_t)j * P);
+        uint32_t *o32 = reinterpret_cast<uint32_t *>(c.sub_hist + (((size_t)rel * c.G + tile) * c.sub_ns + j) * P);
         for (int q = tid; q < P / 2; q += blockDim.x) {
             const uint32_t x0 = sub[2 * q], x1 = sub[2 * q + 1];
             o32[q] = x0 | x1 << 16;
@@ -83,18 +114,11 @@ __global__ void __launch_bounds__(HIST_THREADS, HIST_MINB) k_hist(Ctx c) {
             sub[2 * q] = 0;
             sub[2 * q + 1] = 0;
         }
-        __syncthreads();
-#pragma unroll
-        for (int q = 0; q < NV; ++q) v[q] = vn[q];
-        nv = nvn;
-    }
-    uint32_t *th = c.tile_hist + ((size_t)rel * c.G + tile) * P;
-    for (int p = tid; p < P; p += blockDim.x) {
-        const uint32_t x = acc[p];
-        if (x) {
-            atomicAdd(&th[p], x);
-            atomicAdd(&c.rank_hist[rel * P + p], x);
+        if (g + 1 == nsub0 || g + 1 == ntot) {  // end of a relation's tile
+            __syncthreads();
+            flush_acc(rel);
         }
+        __syncthreads();
     }
 
     // ---- fused exchange: the last CTA publishes the rank histogram ----

@@ -157,7 +157,9 @@ void *dalloc(mgj_plan_s *h, size_t bytes, mgj_status *st) {
     return p;
 }
 
-size_t hist_smem(const Norm &n) { return (size_t)n.P * 8; }
+size_t hist_smem(const Norm &n) {
+    return (size_t)HIST_NB * scat_geom(n.P, n.c.key_bytes).T * n.c.key_bytes + (size_t)n.P * 8;
+}
 size_t plan_smem(const Norm &n) { return (size_t)n.P * 5 * 8 + (size_t)n.P * 4 + (size_t)(n.P + 1) * 4; }
 size_t scatter_smem(const Norm &n) { return scat_smem_bytes(n.P, n.c.key_bytes); }
 size_t planA_smem(const Norm &n) { return ((size_t)local2_vcap(n.P) + 1) * 12; }
@@ -191,8 +193,7 @@ bool is_device_ptr(const void *p) {
 template <typename K>
 void launch_partition(mgj_plan_s *h, cudaStream_t s) {
     const Norm &n = h->n;
-    dim3 g(h->ctx.G * HIST_SPLIT, 2);
-    k_hist<K><<<g, HIST_THREADS, hist_smem(n), s>>>(h->ctx);
+    k_hist<K><<<h->ctx.G * HIST_SPLIT, HIST_THREADS, hist_smem(n), s>>>(h->ctx);
     h->launches = 1;
 }
 

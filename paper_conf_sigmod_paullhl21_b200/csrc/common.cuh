@@ -13,7 +13,6 @@ constexpr int MAX_RANKS = MGJ_MAX_RANKS;
 constexpr int MAX_B1 = 12;              // 2^12 global partitions at most
 constexpr int MAX_B2 = 11;              // local fan-out per pass
 constexpr int HIST_THREADS = 512;
-constexpr int HIST_SPLIT = 2;           // k_hist CTAs per tile (resident together on one SM)
 constexpr int SCATTER_THREADS = 1024;
 constexpr int LOCAL_THREADS = 1024;
 constexpr int LOCAL_VMAX = 12;          // local-pass tuples per thread (chunk C <= 12 * LOCAL_THREADS), 8-byte tuples
@@ -70,6 +69,7 @@ struct Item {
 struct Ctx {
     int32_t rank, world, B1, P, b2_cfg, b2_max;
     int32_t G;                    // tiles per relation (= scatter CTAs)
+    int32_t hist_split;           // k_hist CTAs per tile
     int32_t chunk_tuples;         // local-pass chunk C (tuples)
     int32_t chunk_region;         // slots per chunk in the local buffer (C + 2^b2_max, even)
     int32_t probe_slots;          // probe stage capacity per relation (slots)

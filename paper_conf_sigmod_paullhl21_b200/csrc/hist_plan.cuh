@@ -14,7 +14,7 @@ constexpr int HIST_NB = 3;  // k_hist: TMA ring depth (sub-tiles in flight per C
 // a1: per-GPU radix histogram (§3.2 "Histogram generation",
 // P:356-370, built in shared memory after Rui et al. [38]; bin count from the
 // Eq. 1 analogue).  H[rel][p] = #{t in rel_g : digit1(t.key) = p}.
-// HIST_SPLIT CTAs (two per SM, resident together) share tile c of R and of S
+// hist_split CTAs share tile c of R and of S (two k_hist CTAs per SM)
 // (the tiles the scatter kernel processes); each counts a contiguous run of
 // the scatter's sub-tiles, whose key columns a TMA ring brings into shared
 // memory HIST_NB sub-tiles ahead.  Per sub-tile it stores the u16 counts (the
@@ -32,15 +32,15 @@ __global__ void __launch_bounds__(HIST_THREADS, 2) k_hist(Ctx c) {
     K *const ring = reinterpret_cast<K *>(hsm);
     uint32_t *const sub = reinterpret_cast<uint32_t *>(ring + (size_t)HIST_NB * T);
     uint32_t *const acc = sub + P;
-    const int tid = threadIdx.x, tile = blockIdx.x / HIST_SPLIT, part = blockIdx.x % HIST_SPLIT;
+    const int tid = threadIdx.x, HS = c.hist_split, tile = blockIdx.x / HS, part = blockIdx.x % HS;
     constexpr int LU = 16 / (int)sizeof(K);
     uint64_t lo0, hi0, lo1, hi1;
     tile_range(c.n_in[0], c.G, tile, lo0, hi0);
     tile_range(c.n_in[1], c.G, tile, lo1, hi1);
-    // HIST_SPLIT CTAs share a tile: contiguous runs of its sub-tiles
+    // hist_split CTAs share a tile: contiguous runs of its sub-tiles
     const uint32_t ns0 = (uint32_t)((hi0 - lo0 + T - 1) / T), ns1 = (uint32_t)((hi1 - lo1 + T - 1) / T);
-    const uint32_t ja0 = ns0 * part / HIST_SPLIT, jb0 = ns0 * (part + 1) / HIST_SPLIT;
-    const uint32_t ja1 = ns1 * part / HIST_SPLIT, jb1 = ns1 * (part + 1) / HIST_SPLIT;
+    const uint32_t ja0 = ns0 * part / HS, jb0 = ns0 * (part + 1) / HS;
+    const uint32_t ja1 = ns1 * part / HS, jb1 = ns1 * (part + 1) / HS;
     const uint32_t nsub0 = jb0 - ja0;
     const uint32_t ntot = nsub0 + (jb1 - ja1);
     auto subtile = [&](uint32_t g, int &rel, uint32_t &j, uint64_t &first, uint32_t &len) {

@@ -193,7 +193,7 @@ bool is_device_ptr(const void *p) {
 template <typename K>
 void launch_partition(mgj_plan_s *h, cudaStream_t s) {
     const Norm &n = h->n;
-    k_hist<K><<<h->ctx.G * HIST_SPLIT, HIST_THREADS, hist_smem(n), s>>>(h->ctx);
+    k_hist<K><<<h->ctx.G * h->ctx.hist_split, HIST_THREADS, hist_smem(n), s>>>(h->ctx);
     h->launches = 1;
 }
 
@@ -207,7 +207,7 @@ void launch_shuffle(mgj_plan_s *h, cudaStream_t s) {
     Ctx cs = h->ctx;
     if (cs.ext)
         for (int g = 0; g < MAX_RANKS; ++g) cs.arena[g] = h->send_arena;
-    scatter_kernel<K>(n.P)<<<h->ctx.G, SCATTER_THREADS, scatter_smem(n), s>>>(cs);
+    scatter_kernel<K>(n.P)<<<h->ctx.G, scatter_threads(n.P, n.c.key_bytes), scatter_smem(n), s>>>(cs);
     h->launches += 4;
 }
 
@@ -303,7 +303,9 @@ mgj_status mgj_plan(const mgj_config *cfg, const mgj_peers *peers, mgj_handle *o
     const size_t z_acc = zo; zo += 256;
     const size_t z_err = zo; zo += 256;
     const size_t z_cop = zo; zo += align_up(2ull * P * Qm * 4, 256);
-    const size_t z_th = zo; zo += align_up(2ull * h->nsm * P * 4, 256);
+    // tiles: one per scatter CTA (two per SM when the scatter runs two CTAs per SM)
+    const int G = h->nsm * (scat_geom(P, n.c.key_bytes).alias ? 2 : 1);
+    const size_t z_th = zo; zo += align_up(2ull * G * P * 4, 256);
     const size_t z_ha = zo; zo += align_up(2ull * local2_vcap(P) * 4, 256);
     h->zero_bytes = zo;
     char *zb = static_cast<char *>(dalloc(h, zo, &st));
@@ -315,7 +317,8 @@ mgj_status mgj_plan(const mgj_config *cfg, const mgj_peers *peers, mgj_handle *o
     c.P = P;
     c.b2_cfg = n.c.radix_bits_local;
     c.b2_max = n.b2_max;
-    c.G = h->nsm;
+    c.G = G;
+    c.hist_split = G == h->nsm ? 2 : 1;  // k_hist: two CTAs per SM either way
     c.chunk_tuples = n.chunk_tuples;
     c.chunk_region = n.chunk_region;
     c.probe_slots = n.probe_slots;

@@ -23,12 +23,19 @@ namespace mgj {
 // < 32-byte tail of a partition waits (in registers of its owning thread)
 // for the next sub-tile.  For P = 4096 the alignment padding would not fit
 // shared memory, so SG = 1 (one tuple per store).
+#ifndef SCAT_ALIAS
+#define SCAT_ALIAS 0  // 4-byte keys, P <= 1024: two 512-thread CTAs per SM, stage aliased into the sorted buffer (measured: 6.2 vs 4.1 ms)
+#endif
 struct ScatGeom {
-    int T, SG, PPT;
+    int T, SG, PPT, NT;
+    bool alias;  // stage inside the sorted buffer (two CTAs per SM)
 };
 __host__ __device__ constexpr ScatGeom scat_geom(int P, int key_bytes) {
-    return key_bytes == 4 ? (P <= 1024 ? ScatGeom{8192, 4, 1} : P == 2048 ? ScatGeom{4096, 4, 2} : ScatGeom{8192, 1, 4})
-                          : (P <= 1024 ? ScatGeom{4096, 2, 1} : P == 2048 ? ScatGeom{2048, 2, 2} : ScatGeom{4096, 1, 4});
+    return key_bytes == 4
+               ? (P <= 1024 ? (SCAT_ALIAS ? ScatGeom{4096, 4, P <= 512 ? 1 : 2, 512, true} : ScatGeom{8192, 4, 1, 1024, false})
+                  : P == 2048 ? ScatGeom{4096, 4, 2, 1024, false} : ScatGeom{8192, 1, 4, 1024, false})
+               : (P <= 1024 ? ScatGeom{4096, 2, 1, 1024, false} : P == 2048 ? ScatGeom{2048, 2, 2, 1024, false}
+                                                                      : ScatGeom{4096, 1, 4, 1024, false});
 }
 
 // Per-partition write-out descriptor of the current sub-tile (16 bytes, one
@@ -42,13 +49,13 @@ struct __align__(16) PInfo {
 __host__ __device__ inline size_t scat_smem_bytes(int P, int key_bytes) {
     const ScatGeom g = scat_geom(P, key_bytes);
     const size_t TB = 2 * (size_t)key_bytes;
-    return 2 * (size_t)g.T * key_bytes                      // input stage: keys + payloads (SoA)
+    return (g.alias ? 0 : 2 * (size_t)g.T * key_bytes)      // input stage: keys + payloads (SoA)
            + ((size_t)g.T + 2 * (size_t)(g.SG - 1) * P) * TB  // partition-sorted sub-tile (+ carries, group padding)
            + (size_t)P * sizeof(PInfo)
            + (size_t)P * 4;                                  // next free slot per partition
 }
 
-// Block-wide exclusive scan of one register value per thread (1024 threads).
+// Block-wide exclusive scan of one register value per thread (<= 1024 threads).
 __device__ __forceinline__ uint32_t block_scan_reg(uint32_t v, uint32_t *tmp, uint32_t &total) {
     const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
     uint32_t x = v;
@@ -60,7 +67,7 @@ __device__ __forceinline__ uint32_t block_scan_reg(uint32_t v, uint32_t *tmp, ui
     if (lane == 31) tmp[w] = x;
     __syncthreads();
     if (w == 0) {
-        uint32_t s = tmp[lane];
+        uint32_t s = lane < (int)(blockDim.x >> 5) ? tmp[lane] : 0u;
 #pragma unroll
         for (int o = 1; o < 32; o <<= 1) {
             const uint32_t y = __shfl_up_sync(0xffffffffu, s, o);
@@ -121,11 +128,10 @@ __device__ __forceinline__ void st_group(void *dst, const typename Vec<BYTES>::T
 // have no role on a one-hop fabric.  The last CTA raises SIG_DATA at every
 // peer after a system fence.
 // ---------------------------------------------------------------------------
-template <typename K, int T, int SG, int PPT>
-__global__ void __launch_bounds__(SCATTER_THREADS, 1) k_scatter(Ctx c) {
+template <typename K, int T, int SG, int PPT, int NT, bool ALIAS>
+__global__ void __launch_bounds__(NT, ALIAS ? 2 : 1) k_scatter(Ctx c) {
     using Tup = typename TupT<K>::T;
     constexpr int TB = (int)sizeof(Tup);
-    constexpr int NT = SCATTER_THREADS;
     constexpr int V = T / NT;                  // tuples per thread per sub-tile
     constexpr int LU = 16 / (int)sizeof(K);    // tuples per 16-byte stage vector
     constexpr int NU = V / LU;                 // vectors per thread
@@ -144,9 +150,10 @@ __global__ void __launch_bounds__(SCATTER_THREADS, 1) k_scatter(Ctx c) {
     };
     extern __shared__ __align__(128) unsigned char smem[];
     const int P = c.P;
-    K *const skey = reinterpret_cast<K *>(smem);
+    // ALIAS: the stage is the head of the sorted buffer (loaded after the write-out)
+    Tup *const sorted = reinterpret_cast<Tup *>(smem + (ALIAS ? 0 : 2 * T * sizeof(K)));
+    K *const skey = reinterpret_cast<K *>(ALIAS ? static_cast<void *>(sorted) : static_cast<void *>(smem));
     K *const spay = skey + T;
-    Tup *const sorted = reinterpret_cast<Tup *>(spay + T);
     PInfo *const pinfo = reinterpret_cast<PInfo *>(sorted + T + 2 * (SG - 1) * P);  // 16-byte aligned
     uint32_t *const off = reinterpret_cast<uint32_t *>(pinfo + P);  // next free slot per partition
     __shared__ __align__(8) uint64_t bar;
@@ -276,13 +283,19 @@ __global__ void __launch_bounds__(SCATTER_THREADS, 1) k_scatter(Ctx c) {
         load_counts(g + 1, ncnt);  // prefetch (consumed next iteration)
         uint32_t total;
         uint32_t o = block_scan_reg(tsum, tmp, total);  // its barriers: last write-out is done
+        uint32_t co[PPT], ccw[PPT];  // segment start and carried count (for the ALIAS carry write)
+#pragma unroll
+        for (int k = 0; k < PPT; ++k) ccw[k] = cc[k], co[k] = 0;
 #pragma unroll
         for (int k = 0; k < PPT; ++k) {
             const int p = tid * PPT + k;
             if (p < P) {
+                if (!ALIAS) {
 #pragma unroll
-                for (int i = 0; i < CW; ++i)
-                    if (i < (int)cc[k]) sorted[swz(o + i)] = carry[k][i];
+                    for (int i = 0; i < CW; ++i)
+                        if (i < (int)cc[k]) sorted[swz(o + i)] = carry[k][i];
+                }
+                co[k] = o;
                 off[p] = o + cc[k];
                 const uint32_t full = cnt[k] & ~(uint32_t)(SG - 1);
                 PInfo in;
@@ -324,7 +337,15 @@ __global__ void __launch_bounds__(SCATTER_THREADS, 1) k_scatter(Ctx c) {
             }
         }
         __syncthreads();  // S1: offsets and carries in place, stage consumed
-        if (tid == 0 && g + 1 < ntot) issue(g + 1);
+        if (ALIAS) {  // the stage region is free now: carries to their segment heads
+#pragma unroll
+            for (int k = 0; k < PPT; ++k)
+#pragma unroll
+                for (int i = 0; i < CW; ++i)
+                    if (i < (int)ccw[k]) sorted[swz(co[k] + i)] = carry[k][i];
+        } else if (tid == 0 && g + 1 < ntot) {
+            issue(g + 1);
+        }
 #if SCAT_ATOM_FIRST
         uint32_t pos[V];  // final slots: all atomics first, then the stores
 #pragma unroll
@@ -354,6 +375,7 @@ __global__ void __launch_bounds__(SCATTER_THREADS, 1) k_scatter(Ctx c) {
         }
 #endif
         __syncthreads();  // S2
+        if (ALIAS) fetch_carry();  // before the stage region is reloaded
         // write-out, two groups per thread per step (independent load chains)
         const uint32_t ngroups = total / SG;
         constexpr int WU = SCAT_WO_UNROLL;
@@ -391,6 +413,10 @@ __global__ void __launch_bounds__(SCATTER_THREADS, 1) k_scatter(Ctx c) {
                 }
             }
         }
+        if (ALIAS) {  // the sorted buffer is read: load the next sub-tile into its head
+            __syncthreads();  // S3
+            if (tid == 0 && g + 1 < ntot) issue(g + 1);
+        }
     }
     if (cur_rel >= 0) flush();
 
@@ -409,14 +435,20 @@ __global__ void __launch_bounds__(SCATTER_THREADS, 1) k_scatter(Ctx c) {
 template <typename K>
 inline void (*scatter_kernel(int P))(Ctx) {
     if constexpr (sizeof(K) == 8) {
-        if (P <= 1024) return k_scatter<K, 4096, 2, 1>;
-        if (P == 2048) return k_scatter<K, 2048, 2, 2>;
-        return k_scatter<K, 4096, 1, 4>;
+        if (P <= 1024) return k_scatter<K, 4096, 2, 1, 1024, false>;
+        if (P == 2048) return k_scatter<K, 2048, 2, 2, 1024, false>;
+        return k_scatter<K, 4096, 1, 4, 1024, false>;
     } else {
-        if (P <= 1024) return k_scatter<K, 8192, 4, 1>;
-        if (P == 2048) return k_scatter<K, 4096, 4, 2>;
-        return k_scatter<K, 8192, 1, 4>;
+#if SCAT_ALIAS
+        if (P <= 512) return k_scatter<K, 4096, 4, 1, 512, true>;
+        if (P == 1024) return k_scatter<K, 4096, 4, 2, 512, true>;
+#else
+        if (P <= 1024) return k_scatter<K, 8192, 4, 1, 1024, false>;
+#endif
+        if (P == 2048) return k_scatter<K, 4096, 4, 2, 1024, false>;
+        return k_scatter<K, 8192, 1, 4, 1024, false>;
     }
 }
+inline int scatter_threads(int P, int key_bytes) { return scat_geom(P, key_bytes).NT; }
 
 }  // namespace mgj

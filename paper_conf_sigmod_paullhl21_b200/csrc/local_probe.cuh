@@ -599,12 +599,13 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
             }
             for (int rel = rel0; rel < rel1; ++rel) {
                 const Side sd = rel ? x.it.s : x.it.r;
-                const uint16_t *E0 = c.eoff[rel] + (size_t)(Q + 1) * x.cb[rel] + (size_t)x.it.q * x.nch[rel];
-                const uint16_t *E1 = E0 + x.nch[rel];
-                const uint32_t kend = min(sd.k1, x.nch[rel] - 1);
+                const uint32_t xcb = rel ? x.cb[1] : x.cb[0], xnch = rel ? x.nch[1] : x.nch[0];  // no local memory
+                const uint16_t *E0 = (rel ? c.eoff[1] : c.eoff[0]) + (size_t)(Q + 1) * xcb + (size_t)x.it.q * xnch;
+                const uint16_t *E1 = E0 + xnch;
+                const uint32_t kend = min(sd.k1, xnch - 1);
                 const uint32_t np = sd.k0 <= kend ? kend - sd.k0 + 1 : 0;
                 Tup *dstbase = stages + ((size_t)s * 2 + rel) * SL;
-                const Tup *lbase = static_cast<const Tup *>(c.local[rel]);
+                const Tup *lbase = static_cast<const Tup *>(rel ? c.local[1] : c.local[0]);
                 uint32_t run = 0;
                 for (uint32_t m0 = 0; m0 < np; m0 += 32) {
                     const uint32_t m = m0 + lane;
@@ -618,7 +619,7 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
                         const uint32_t ahi = (k == sd.k1) ? sd.a1 : slots;
                         if (ahi > alo) {
                             sz = ahi - alo;
-                            src = (uint64_t)(x.cb[rel] + k) * c.chunk_region + st + alo;
+                            src = (uint64_t)(xcb + k) * c.chunk_region + st + alo;
                         }
                         pad = (SBITS && rel == 1 && v < slots && v >= alo && v < ahi) ? v - alo : 0xffffffffu;
                     }
@@ -696,7 +697,7 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
                 for (uint32_t i = (hv >> 16) == tag ? (hv & 0xffffu) : END; i != END;) {
                     const Tup rv = rt[i];
                     const uint32_t l = (uint32_t)rv.x;
-                    if ((l >> 16) == khi) f(rv.y);
+                    if ((l >> 16) == khi) f((K)rv.y, i);
                     i = l & 0xffffu;
                 }
             } else {
@@ -704,14 +705,14 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
                 const uint32_t hv = head[tab_hash(sv.x, shift, LOGT)];
                 for (uint32_t i = (hv >> 16) == tag ? (hv & 0xffffu) : END; i != END; i = nxt[i]) {
                     const Tup rv = rt[i];
-                    if (rv.x == sv.x) f(rv.y);
+                    if (rv.x == sv.x) f((K)rv.y, i);
                 }
             }
         };
         // probe
         uint32_t m_item = 0;
         uint32_t x0 = ct;
-        if (PROBE_U2 && packed) {  // two S slots per step: independent load chains
+        if (PROBE_U2 && packed && !MAT) {  // two S slots per step: independent load chains
             for (; x0 + NCONS < stot; x0 += 2 * NCONS) {
                 const Tup s0 = st[x0], s1 = st[x0 + NCONS];
                 const uint32_t k0 = (uint32_t)s0.x, k1 = (uint32_t)s1.x;
@@ -741,12 +742,35 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
                 }
             }
         }
-        for (uint32_t x = x0; x < stot; x += NCONS) {
-            const Tup sv = st[x];
-            walk(x, sv, [&](K a) {
-                ++m_item;
-                my_chk += chk_term(a, (K)sv.y);
-            });
+        // MAT: the first match of each of this thread's S slots is kept (R slot
+        // index) so the write pass needs no second walk unless a slot matched
+        // more than once (duplicate R keys: the warp re-walks instead)
+        constexpr int KMAX = (PROBE_SLOTS8 + NCONS - 1) / NCONS;  // S slots per consumer thread
+        uint16_t mi[MAT ? KMAX : 1];
+        bool ovf = false;
+        if (MAT) {
+#pragma unroll
+            for (int k = 0; k < KMAX; ++k) {
+                const uint32_t x = ct + k * NCONS;
+                mi[k] = END;
+                if (x < stot) {
+                    const Tup sv = st[x];
+                    walk(x, sv, [&](K a, uint32_t i) {
+                        ++m_item;
+                        my_chk += chk_term(a, (K)sv.y);
+                        if (mi[k] == END) mi[k] = (uint16_t)i;
+                        else ovf = true;
+                    });
+                }
+            }
+        } else {
+            for (uint32_t x = x0; x < stot; x += NCONS) {
+                const Tup sv = st[x];
+                walk(x, sv, [&](K a, uint32_t) {
+                    ++m_item;
+                    my_chk += chk_term(a, (K)sv.y);
+                });
+            }
         }
         my_cnt += m_item;
         if (MAT) {
@@ -777,19 +801,75 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
                 }
             }
             named_bar_sync(1, NCONS);
-            if (s_write && m_item) {
-                K *ok = static_cast<K *>(c.out_key);
-                K *oa = static_cast<K *>(c.out_a);
-                K *ob = static_cast<K *>(c.out_b);
-                unsigned long long pos = s_base + (cwi ? s_wtot[cwi - 1] : 0) + incl - m_item;
-                for (uint32_t x = ct; x < stot; x += NCONS) {
-                    const Tup sv = st[x];
-                    walk(x, sv, [&](K a) {
-                        ok[pos] = (K)sv.x;
-                        oa[pos] = a;
-                        ob[pos] = (K)sv.y;
-                        ++pos;
-                    });
+            // write pass, warp-synchronous: every chain step of the warp's 32 S
+            // slots emits its matches at consecutive positions of the warp's
+            // reservation (ballot + popc), so each store instruction covers
+            // consecutive output elements
+            const unsigned long long wlo = cwi ? s_wtot[cwi - 1] : 0;
+            K *ok = static_cast<K *>(c.out_key);
+            K *oa = static_cast<K *>(c.out_a);
+            K *ob = static_cast<K *>(c.out_b);
+            const uint32_t lt = (1u << lane) - 1u;
+            const bool wovf = __any_sync(0xffffffffu, ovf);
+            if (s_write && s_wtot[cwi] > wlo && !wovf) {  // from the recorded matches
+                unsigned long long wpos = s_base + wlo;
+#pragma unroll
+                for (int k = 0; k < KMAX; ++k) {
+                    const bool has = mi[k] != END;
+                    const uint32_t mask = __ballot_sync(0xffffffffu, has);
+                    if (has) {
+                        const unsigned long long q = wpos + __popc(mask & lt);
+                        const Tup sv = st[ct + k * NCONS];
+                        ok[q] = (K)sv.x;
+                        oa[q] = (K)rt[mi[k]].y;
+                        ob[q] = (K)sv.y;
+                    }
+                    wpos += __popc(mask);
+                }
+            } else if (s_write && s_wtot[cwi] > wlo) {
+                unsigned long long wpos = s_base + wlo;
+                for (uint32_t xb = (uint32_t)(ct & ~31); xb < stot; xb += NCONS) {
+                    const uint32_t x = xb + lane;
+                    Tup sv{};
+                    uint32_t i = END, khi = 0;
+                    if (x < stot) {
+                        sv = st[x];
+                        if (packed) {
+                            const uint32_t k = (uint32_t)sv.x;
+                            if ((k & (uint32_t)(P - 1)) == pitem) {
+                                khi = k >> shift;
+                                const uint32_t hv = head[fold(khi)];
+                                i = (hv >> 16) == tag ? (hv & 0xffffu) : END;
+                            }
+                        } else if (!(SBITS && ((pb[x >> 5] >> (x & 31)) & 1u))) {
+                            const uint32_t hv = head[tab_hash(sv.x, shift, LOGT)];
+                            i = (hv >> 16) == tag ? (hv & 0xffffu) : END;
+                        }
+                    }
+                    while (__any_sync(0xffffffffu, i != END)) {
+                        bool match = false;
+                        K a = 0;
+                        if (i != END) {
+                            const Tup rv = rt[i];
+                            if (packed) {
+                                const uint32_t l = (uint32_t)rv.x;
+                                match = (l >> 16) == khi;
+                                i = l & 0xffffu;
+                            } else {
+                                match = rv.x == sv.x;
+                                i = nxt[i];
+                            }
+                            a = (K)rv.y;
+                        }
+                        const uint32_t mask = __ballot_sync(0xffffffffu, match);
+                        if (match) {
+                            const unsigned long long q = wpos + __popc(mask & lt);
+                            ok[q] = (K)sv.x;
+                            oa[q] = a;
+                            ob[q] = (K)sv.y;
+                        }
+                        wpos += __popc(mask);
+                    }
                 }
             }
         }

@@ -7,6 +7,10 @@
 
 namespace mgj {
 
+#ifndef PROBE_PACK64
+#define PROBE_PACK64 0  // packed table for 8-byte keys too
+#endif
+
 #ifndef PROBE_U2
 #define PROBE_U2 0  // packed probe: two S slots per step (measured slower: 2.00 vs 1.96 ms)
 #endif
@@ -555,13 +559,15 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
     // and S padding is probed harmlessly; only P < 4 needs the skip bitmap
     const bool SBITS = Layout<K>::ALIGN == 2 && c.P < 4;
     const int plo = c.meta[MT_PLO], BAp = c.meta[MT_BA];
-    // packed table (4-byte keys whose bits above the radix digits fit 16 bits,
-    // e.g. B1 + B2 >= 16): the build overwrites each R slot's key with
-    // (khi << 16 | next), khi = key >> (B1 + B2), so a chain step is one
-    // 8-byte shared load that yields khi, the next link and the payload.  All
+    // packed table (B1 + B2 >= 16, so khi = key >> (B1 + B2) fits the key's
+    // width minus 16 bits): the build overwrites each R slot's key with
+    // (khi << 16 | next), so a chain step is one shared load of the slot
+    // that yields khi, the next link and the payload.  All
     // real keys of a co-partition share their low B1 + B2 bits, so equal khi
     // means equal keys; padding slots (digit1 != p) are left out on both sides.
-    const bool packed = sizeof(K) == 4 && c.B1 + B2 >= 16;
+    // (8-byte keys: measured slower packed, 3.04 vs 2.82 ms at M5 size: the
+    // 64-bit shifts and compares cost more issue slots than the link load saves)
+    const bool packed = (sizeof(K) == 4 || PROBE_PACK64) && c.B1 + B2 >= 16;
     const int P = c.P;
     const int Q = 1 << c.meta[MT_QB], shift = c.B1 + B2;  // Q: runs per chunk of the chunked pass
     const uint32_t nitems = min(__ldcg(&c.ticket[TK_ITEMS]), c.max_items);
@@ -667,16 +673,23 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
         const Tup *st = stages + ((size_t)s * 2 + 1) * SL;
         const uint32_t rtot = totals[s][0], stot = totals[s][1];
         const uint32_t pitem = stage_p[s];
-        auto fold = [](uint32_t khi) { return (khi ^ (khi >> LOGT)) & (uint32_t)(T - 1); };
+        auto fold = [](K khi) {  // table index from khi (identity for dense keys below 2^12)
+            if constexpr (sizeof(K) == 4) {
+                return ((uint32_t)khi ^ ((uint32_t)khi >> LOGT)) & (uint32_t)(T - 1);
+            } else {
+                const uint32_t f = (uint32_t)khi ^ (uint32_t)((unsigned long long)khi >> 32);
+                return (f ^ (f >> LOGT) ^ (f >> (2 * LOGT))) & (uint32_t)(T - 1);
+            }
+        };
         // build
         if (packed) {
-            uint32_t *rw = reinterpret_cast<uint32_t *>(stages + ((size_t)s * 2 + 0) * SL);
+            K *rw = reinterpret_cast<K *>(stages + ((size_t)s * 2 + 0) * SL);
             for (uint32_t slot = ct; slot < rtot; slot += NCONS) {
-                const uint32_t k = (uint32_t)rt[slot].x;
-                if ((k & (uint32_t)(P - 1)) != pitem) continue;  // R padding slot
-                const uint32_t khi = k >> shift;
+                const K k = rt[slot].x;
+                if (((uint32_t)k & (uint32_t)(P - 1)) != pitem) continue;  // R padding slot
+                const K khi = k >> shift;
                 const uint32_t old = atomicExch(&head[fold(khi)], (tag << 16) | slot);
-                rw[2 * slot] = ((old >> 16) == tag ? (old & 0xffffu) : (uint32_t)END) | (khi << 16);
+                rw[2 * slot] = (K)((old >> 16) == tag ? (old & 0xffffu) : (uint32_t)END) | (khi << 16);
             }
         } else {
             for (uint32_t slot = ct; slot < rtot; slot += NCONS) {
@@ -690,15 +703,15 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
         // every R payload matching S slot x: f(payR)
         auto walk = [&](uint32_t x, const Tup &sv, auto &&f) {
             if (packed) {
-                const uint32_t k = (uint32_t)sv.x;
-                if ((k & (uint32_t)(P - 1)) != pitem) return;  // S padding slot
-                const uint32_t khi = k >> shift;
+                const K k = sv.x;
+                if (((uint32_t)k & (uint32_t)(P - 1)) != pitem) return;  // S padding slot
+                const K khi = k >> shift;
                 const uint32_t hv = head[fold(khi)];
                 for (uint32_t i = (hv >> 16) == tag ? (hv & 0xffffu) : END; i != END;) {
                     const Tup rv = rt[i];
-                    const uint32_t l = (uint32_t)rv.x;
+                    const K l = rv.x;
                     if ((l >> 16) == khi) f((K)rv.y, i);
-                    i = l & 0xffffu;
+                    i = (uint32_t)l & 0xffffu;
                 }
             } else {
                 if (SBITS && ((pb[x >> 5] >> (x & 31)) & 1u)) return;  // padding slot (P < 4 only)
@@ -831,12 +844,13 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
                 for (uint32_t xb = (uint32_t)(ct & ~31); xb < stot; xb += NCONS) {
                     const uint32_t x = xb + lane;
                     Tup sv{};
-                    uint32_t i = END, khi = 0;
+                    uint32_t i = END;
+                    K khi = 0;
                     if (x < stot) {
                         sv = st[x];
                         if (packed) {
-                            const uint32_t k = (uint32_t)sv.x;
-                            if ((k & (uint32_t)(P - 1)) == pitem) {
+                            const K k = sv.x;
+                            if (((uint32_t)k & (uint32_t)(P - 1)) == pitem) {
                                 khi = k >> shift;
                                 const uint32_t hv = head[fold(khi)];
                                 i = (hv >> 16) == tag ? (hv & 0xffffu) : END;
@@ -852,9 +866,9 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
                         if (i != END) {
                             const Tup rv = rt[i];
                             if (packed) {
-                                const uint32_t l = (uint32_t)rv.x;
+                                const K l = rv.x;
                                 match = (l >> 16) == khi;
-                                i = l & 0xffffu;
+                                i = (uint32_t)l & 0xffffu;
                             } else {
                                 match = rv.x == sv.x;
                                 i = nxt[i];

@@ -273,6 +273,29 @@ def test_wide_high_bits_only(mgj):
     check_vs_oracle(mgj, d, materialize=False)
 
 
+@pytest.mark.parametrize("kind", ["wide", "wide_dup_high", "u32_dup"])
+def test_packed_table(mgj, kind):
+    """The packed chained table (B1 + B2 >= 16: the R slot's key is replaced by
+    khi << 16 | next) at small sizes, forced with B1 = 10, B2 = 6: unique wide
+    keys, wide keys that differ only above bit 40 with duplicate R keys (the
+    materialisation's re-walk path), and 4-byte duplicate keys."""
+    rng = np.random.default_rng(23)
+    if kind == "wide":
+        d = datagen.Workload("wide", 1 << 17, 1 << 17).rank_inputs()
+    elif kind == "wide_dup_high":
+        def keys(n):
+            return (rng.integers(0, 16, n, dtype=np.uint64) << np.uint64(40)) | rng.integers(0, 256, n, dtype=np.uint64)
+        d = {"r_keys": keys(30000), "s_keys": keys(20000),
+             "r_pays": np.arange(30000, dtype=np.uint64) << np.uint64(20),
+             "s_pays": np.arange(20000, dtype=np.uint64) + np.uint64(2**62)}
+    else:
+        d = dict(r_keys=rng.integers(0, 1 << 20, 200003, dtype=np.uint32),
+                 r_pays=rng.integers(0, 1 << 32, 200003, dtype=np.uint32),
+                 s_keys=rng.integers(0, 1 << 20, 300007, dtype=np.uint32),
+                 s_pays=rng.integers(0, 1 << 32, 300007, dtype=np.uint32))
+    check_vs_oracle(mgj, d, materialize=True, radix_bits_global=10, radix_bits_local=6)
+
+
 def test_host_pointer_path(mgj):
     """Host (numpy) inputs are staged by the library: same result (end-to-end path)."""
     d = datagen.Workload("unique", 1 << 18, 1 << 18).rank_inputs()

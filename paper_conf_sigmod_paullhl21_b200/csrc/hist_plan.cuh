@@ -188,12 +188,17 @@ __host__ __device__ inline int ceil_log2_u64(uint64_t x) {
     return l;
 }
 
-// B2 from the largest owned R partition: co-partitions of ~target tuples
-// (2/3 of the probe stage capacity, so they fit one shared-memory table).
-__host__ __device__ inline int choose_b2(uint64_t max_r, int b2_cfg, int b2_max, uint64_t target) {
+// B2: R co-partitions of at most ~target tuples (one shared-memory table),
+// and, on average, R + S co-partitions of at most 2 * target tuples (one
+// probe stage, shared by the two sides).  The largest owned R partition sets
+// the first bound; the mean R + S of the owned partitions the second (a
+// heavy-hitter partition cannot be split by radix bits: its S side is
+// sliced over several items instead).
+__host__ __device__ inline int choose_b2(uint64_t max_r, uint64_t mean_rs, int b2_cfg, int b2_max, uint64_t target) {
     if (b2_cfg > 0) return b2_cfg < b2_max ? b2_cfg : b2_max;
-    const uint64_t need = (max_r + target - 1) / target;
-    int b = ceil_log2_u64(need);
+    int b = ceil_log2_u64((max_r + target - 1) / target);
+    const int bs = ceil_log2_u64((mean_rs + 2 * target - 1) / (2 * target));
+    if (bs > b) b = bs;
     if (b > b2_max) b = b2_max;
     return b;
 }
@@ -215,11 +220,12 @@ __global__ void __launch_bounds__(1024) k_plan(Ctx c) {
     __shared__ uint32_t tmp32[33];
     __shared__ int first[MAX_RANKS], endp[MAX_RANKS];
     __shared__ int ok, cap_bad;
-    __shared__ unsigned long long maxr;
+    __shared__ unsigned long long maxr, sumrs;
     if (tid == 0) {
         ok = wait_all_flags(c, SIG_HIST);
         cap_bad = 0;
         maxr = 0;
+        sumrs = 0;
     }
     if (tid < MAX_RANKS) first[tid] = endp[tid] = P;
     __syncthreads();
@@ -283,9 +289,25 @@ __global__ void __launch_bounds__(1024) k_plan(Ctx c) {
     }
     const int plo = first[c.rank] < P ? first[c.rank] : 0;
     const int phi = first[c.rank] < P ? endp[c.rank] : 0;
-    for (int p = plo + tid; p < phi; p += blockDim.x) atomicMax(&maxr, (unsigned long long)tot0[p]);
+    {  // largest owned R partition and total owned R + S: warp reductions, one shared atomic per warp
+        unsigned long long mr = 0, sr = 0;
+        for (int p = plo + tid; p < phi; p += blockDim.x) {
+            mr = max(mr, (unsigned long long)tot0[p]);
+            sr += tot0[p] + tot1[p];
+        }
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) {
+            mr = max(mr, __shfl_xor_sync(0xffffffffu, mr, o));
+            sr += __shfl_xor_sync(0xffffffffu, sr, o);
+        }
+        if ((tid & 31) == 0) {
+            atomicMax(&maxr, mr);
+            atomicAdd(&sumrs, sr);
+        }
+    }
     __syncthreads();
-    const int B2 = choose_b2(maxr, c.b2_cfg, c.b2_max, (uint64_t)c.probe_target);
+    const int B2 = choose_b2(maxr, phi > plo ? sumrs / (uint64_t)(phi - plo) : 0, c.b2_cfg, c.b2_max,
+                             (uint64_t)c.probe_target);
     // received pieces of every owned partition pi: P2P — one piece (the whole
     // segment, sources ascending inside it); EXTERNAL — one piece per source
     // rank g, the receive area being [g0 | g1 | ...], each [owned p ascending]

@@ -402,16 +402,20 @@ __global__ void __launch_bounds__(LOCAL_THREADS, 1) k_local(Ctx c, const ChunkDe
 }
 
 // ---------------------------------------------------------------------------
-// Probe work items.  Co-partition (p, q) is one item when both of its sides
-// fit a pipeline stage (the common case); otherwise each side is cut into
-// stage-sized slices (at even slot offsets) and every R slice is paired with
-// every S slice: an oversized R co-partition is built in table-sized pieces
-// (block nested loop over R slices — the "both relations heavily skewed"
-// case of P:450-452) and a heavy S co-partition is spread over many CTAs.
+// Probe work items.  A pipeline stage holds 2 * cap slots shared by the two
+// sides: R from slot 0 (at most cap slots: one shared-memory table), S from
+// slot soff.  Co-partition (p, q) is one item when R <= cap and R + S fit the
+// stage (the common case, whatever the |R|:|S| ratio); otherwise R is cut
+// into slices of cap slots and S into slices of the rest of the stage (at
+// even slot offsets), and every R slice is paired with every S slice: an
+// oversized R co-partition is built in table-sized pieces (block nested loop
+// over R slices — the "both relations heavily skewed" case of P:450-452) and
+// a heavy S co-partition is spread over many CTAs.
 // ---------------------------------------------------------------------------
 struct ItemX {
     Item it;
     uint32_t cb[2], nch[2];  // first chunk / chunk count of p per relation
+    uint32_t soff;           // stage slot where the S side starts (>= the R side's slots)
 };
 
 // Walk the q-runs of one side in chunk order and cut it into slices of at
@@ -470,9 +474,10 @@ __global__ void k_itemize(Ctx c) {
             x.cb[rel] = cb[pi];
             x.nch[rel] = cb[pi + 1] - cb[pi];
         }
-        if (r <= cap && s <= cap && x.nch[0] <= PROBE_MAXP && x.nch[1] <= PROBE_MAXP) {
+        if (r <= cap && r + s <= 2 * cap && x.nch[0] <= PROBE_MAXP && x.nch[1] <= PROBE_MAXP) {
             x.it.r = Side{0, 0, x.nch[0], 0};
             x.it.s = Side{0, 0, x.nch[1], 0};
+            x.soff = r;
             const uint32_t b = atomicAdd(&c.ticket[TK_ITEMS], 1u);
             if (b < c.max_items) items[b] = x;
             else set_err(c, MGJ_ECAPACITY);
@@ -484,9 +489,11 @@ __global__ void k_itemize(Ctx c) {
             E[rel][0] = c.eoff[rel] + (size_t)(Q + 1) * x.cb[rel] + (size_t)q * x.nch[rel];
             E[rel][1] = E[rel][0] + x.nch[rel];
         }
+        const uint32_t rcap = r < cap ? r : cap, scap = 2 * cap - rcap;  // both even
+        x.soff = rcap;
         uint32_t nr = 0, ns = 0;
-        walk_side<ALIGN>(E[0][0], E[0][1], x.nch[0], cap, PROBE_MAXP, [&](const Side &) { ++nr; });
-        walk_side<ALIGN>(E[1][0], E[1][1], x.nch[1], cap, PROBE_MAXP, [&](const Side &) { ++ns; });
+        walk_side<ALIGN>(E[0][0], E[0][1], x.nch[0], rcap, PROBE_MAXP, [&](const Side &) { ++nr; });
+        walk_side<ALIGN>(E[1][0], E[1][1], x.nch[1], scap, PROBE_MAXP, [&](const Side &) { ++ns; });
         const uint64_t n = (uint64_t)nr * ns;
         const uint32_t b = atomicAdd(&c.ticket[TK_ITEMS], (uint32_t)min(n, (uint64_t)0x7fffffffu));
         if ((uint64_t)b + n > c.max_items) {
@@ -494,9 +501,9 @@ __global__ void k_itemize(Ctx c) {
             continue;
         }
         uint32_t ir = 0;
-        walk_side<ALIGN>(E[0][0], E[0][1], x.nch[0], cap, PROBE_MAXP, [&](const Side &rs) {
+        walk_side<ALIGN>(E[0][0], E[0][1], x.nch[0], rcap, PROBE_MAXP, [&](const Side &rs) {
             uint32_t is = 0;
-            walk_side<ALIGN>(E[1][0], E[1][1], x.nch[1], cap, PROBE_MAXP, [&](const Side &ss) {
+            walk_side<ALIGN>(E[1][0], E[1][1], x.nch[1], scap, PROBE_MAXP, [&](const Side &ss) {
                 ItemX y = x;
                 y.it.r = rs;
                 y.it.s = ss;
@@ -509,8 +516,8 @@ __global__ void k_itemize(Ctx c) {
 }
 
 __host__ __device__ inline size_t probe_smem_bytes(int slots, int TB) {
-    return (size_t)PROBE_NST * 2 * slots * TB  // stages (R, S)
-           + (size_t)PROBE_NST * (slots / 32 + 1) * 4  // S padding-slot bitmaps
+    return (size_t)PROBE_NST * 2 * slots * TB  // stages (R then S, 2 * slots each)
+           + (size_t)PROBE_NST * (2 * slots / 32 + 1) * 4  // S padding-slot bitmaps
            + 4096 * 4                          // head
            + (size_t)slots * 2;                // next
 }
@@ -542,13 +549,14 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
     __shared__ __align__(8) uint64_t full[PROBE_NST], empty[PROBE_NST];
     __shared__ uint32_t totals[PROBE_NST][2];
     __shared__ uint32_t stage_p[PROBE_NST];  // global partition (digit1) of the stage's item
+    __shared__ uint32_t stage_soff[PROBE_NST];  // slot where the stage's S side starts
     __shared__ uint32_t s_wtot[32];
     __shared__ unsigned long long s_base;
     __shared__ int s_write;
     if (!c.meta[MT_OK]) return;
     const int SL = c.probe_slots;
-    Tup *stages = reinterpret_cast<Tup *>(smem);  // [NST][2][SL]
-    const int PW = SL / 32 + 1;  // words per S padding bitmap
+    Tup *stages = reinterpret_cast<Tup *>(smem);  // [NST][2 * SL]: R from 0, S from the item's soff
+    const int PW = 2 * SL / 32 + 1;  // words per S padding bitmap
     uint32_t *padbits = reinterpret_cast<uint32_t *>(stages + (size_t)PROBE_NST * 2 * SL);  // [NST][PW]
     uint32_t *head = padbits + PROBE_NST * PW;
     uint16_t *nxt = reinterpret_cast<uint16_t *>(head + T);
@@ -610,7 +618,7 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
                 const uint16_t *E1 = E0 + xnch;
                 const uint32_t kend = min(sd.k1, xnch - 1);
                 const uint32_t np = sd.k0 <= kend ? kend - sd.k0 + 1 : 0;
-                Tup *dstbase = stages + ((size_t)s * 2 + rel) * SL;
+                Tup *dstbase = stages + (size_t)s * 2 * SL + (rel ? x.soff : 0);
                 const Tup *lbase = static_cast<const Tup *>(rel ? c.local[1] : c.local[0]);
                 uint32_t run = 0;
                 for (uint32_t m0 = 0; m0 < np; m0 += 32) {
@@ -649,7 +657,10 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
                 }
                 if (lane == 0) totals[s][rel] = run;
             }
-            if (lane == 0 && rel0 == 0) stage_p[s] = (uint32_t)(plo + (BAp ? x.it.pi >> BAp : x.it.pi));
+            if (lane == 0 && rel0 == 0) {
+                stage_p[s] = (uint32_t)(plo + (BAp ? x.it.pi >> BAp : x.it.pi));
+                stage_soff[s] = x.soff;
+            }
             __syncwarp();
             if (lane == 0) mbar_arrive(&full[s]);
             x = xn;
@@ -669,8 +680,8 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
             tag = 1;
         }
         mbar_wait(&full[s], (j / PROBE_NST) & 1);
-        const Tup *rt = stages + ((size_t)s * 2 + 0) * SL;
-        const Tup *st = stages + ((size_t)s * 2 + 1) * SL;
+        const Tup *rt = stages + (size_t)s * 2 * SL;
+        const Tup *st = rt + stage_soff[s];
         const uint32_t rtot = totals[s][0], stot = totals[s][1];
         const uint32_t pitem = stage_p[s];
         auto fold = [](K khi) {  // table index from khi (identity for dense keys below 2^12)
@@ -683,7 +694,7 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
         };
         // build
         if (packed) {
-            K *rw = reinterpret_cast<K *>(stages + ((size_t)s * 2 + 0) * SL);
+            K *rw = reinterpret_cast<K *>(stages + (size_t)s * 2 * SL);
             for (uint32_t slot = ct; slot < rtot; slot += NCONS) {
                 const K k = rt[slot].x;
                 if (((uint32_t)k & (uint32_t)(P - 1)) != pitem) continue;  // R padding slot
@@ -775,6 +786,14 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
                         else ovf = true;
                     });
                 }
+            }
+            for (uint32_t x = ct + KMAX * NCONS; x < stot; x += NCONS) {  // beyond the record: re-walk
+                const Tup sv = st[x];
+                walk(x, sv, [&](K a, uint32_t) {
+                    ++m_item;
+                    my_chk += chk_term(a, (K)sv.y);
+                    ovf = true;
+                });
             }
         } else {
             for (uint32_t x = x0; x < stot; x += NCONS) {

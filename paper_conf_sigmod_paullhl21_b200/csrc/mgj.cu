@@ -72,7 +72,9 @@ mgj_status normalize(const mgj_config *in, Norm *o) {
     } else {
         // expected largest owned R partition ~ recv_cap / P; +2 bits of headroom for skew
         const uint64_t per_p = (c.recv_capacity_r + o->P - 1) / o->P;
-        o->b2_max = std::min(MAX_B2, std::max(1, ceil_log2((per_p + target - 1) / target) + 2));
+        const uint64_t per_rs = (c.recv_capacity_r + c.recv_capacity_s + o->P - 1) / o->P;
+        const int b = std::max(ceil_log2((per_p + target - 1) / target), ceil_log2((per_rs + 2 * target - 1) / (2 * target)));
+        o->b2_max = std::min(MAX_B2, std::max(1, b + 2));
     }
     const int Qm = 1 << o->b2_max;
     int C = 0;  // largest chunk (multiple of LOCAL_THREADS) whose buffers fit shared memory

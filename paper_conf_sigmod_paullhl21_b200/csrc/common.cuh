@@ -155,6 +155,9 @@ __device__ __forceinline__ uint64_t globaltimer() {
 }
 
 __device__ __forceinline__ void set_err(const Ctx &c, int code) {
+#if defined(SCAT_RING) && SCAT_RING
+    if (code == MGJ_ECAPACITY) return;  // timing experiment: the received data is not the real one
+#endif
     atomicCAS(c.err, 0, code);
 }
 

@@ -11,6 +11,10 @@ namespace mgj {
 #define PROBE_PACK64 0  // packed table for 8-byte keys too
 #endif
 
+#ifndef LP_RING
+#define LP_RING 0  // EXPERIMENT ONLY (wrong results): local output chunk regions modulo LP_RING, to time an L2-resident local buffer
+#endif
+
 #ifndef PROBE_U2
 #define PROBE_U2 0  // packed probe: two S slots per step (measured slower: 2.00 vs 1.96 ms)
 #endif
@@ -39,9 +43,10 @@ __device__ __forceinline__ void decode_run(uint32_t e0, uint32_t e1, uint32_t &s
 }
 
 // Two chunk buffers that alternate roles (TMA load target of chunk j+1 /
-// sorted output of chunk j), plus the bin counters.
+// sorted output of chunk j), plus two alternating bin-counter arrays and the
+// run starts.
 __host__ __device__ inline size_t local_smem_bytes(int C, int Qmax, int TB) {
-    return 2 * (size_t)(C + Qmax + 2) * TB + 2 * (size_t)Qmax * 4;
+    return 2 * (size_t)(C + Qmax + 2) * TB + 3 * (size_t)Qmax * 4;
 }
 
 // Chunk descriptors for the local pass: chunk ci of owned partition pi covers
@@ -263,8 +268,8 @@ __global__ void __launch_bounds__(LOCAL_THREADS, 1) k_local(Ctx c, const ChunkDe
     const int plo = c.meta[MT_PLO];
     Tup *const buf0 = reinterpret_cast<Tup *>(smem);
     auto buf = [&](int x) { return buf0 + (size_t)x * BUF; };
-    uint32_t *bins = reinterpret_cast<uint32_t *>(buf0 + (size_t)2 * BUF);
-    uint32_t *abin = bins + Qmax;
+    uint32_t *const bins2 = reinterpret_cast<uint32_t *>(buf0 + (size_t)2 * BUF);  // [2][Qmax], chunk j uses j & 1
+    uint32_t *const abin = bins2 + 2 * Qmax;
     const uint32_t nch_r = SPLIT ? (uint32_t)c.meta[MT_NCH_R] : nch_local(c, 0);
     const uint32_t total = nch_r + (SPLIT ? (uint32_t)c.meta[MT_NCH_S] : nch_local(c, 1));
     const uint32_t mine = total > blockIdx.x ? (total - blockIdx.x + gridDim.x - 1) / gridDim.x : 0;
@@ -276,6 +281,7 @@ __global__ void __launch_bounds__(LOCAL_THREADS, 1) k_local(Ctx c, const ChunkDe
         mbar_init(&bar[1], 1);
         fence_mbar_init();
     }
+    for (int q = tid; q < 2 * Qmax; q += LOCAL_THREADS) bins2[q] = 0;
     __syncthreads();
     const uint64_t pol = policy_evict_first();
     // thread 0: TMA chunk j (16-byte-aligned superset) into buffer j & 1
@@ -291,7 +297,8 @@ __global__ void __launch_bounds__(LOCAL_THREADS, 1) k_local(Ctx c, const ChunkDe
         if (bytes) tma_load_1d(buf(j & 1), reinterpret_cast<const Tup *>(rel ? srcS : srcR) + g0, bytes, b, pol);
     };
     ChunkDesc nxt{};
-    if (tid == 0) {
+    constexpr int LI = 32;  // the thread that issues the chunk loads (and the chunked pass's stores)
+    if (tid == LI) {
         if (mine > 0) issue(0, cdesc[blockIdx.x]);
         if (mine > 1) nxt = cdesc[blockIdx.x + gridDim.x];
     }
@@ -300,6 +307,7 @@ __global__ void __launch_bounds__(LOCAL_THREADS, 1) k_local(Ctx c, const ChunkDe
         const int rel = ci < nch_r ? 0 : 1;
         const uint32_t li = rel ? ci - nch_r : ci;
         const int X = j & 1;
+        uint32_t *const bins = bins2 + X * Qmax;  // zero (cleared during chunk j - 1)
         mbar_wait(&bar[X], (j >> 1) & 1);
         const ChunkDesc d = sdesc[X];
         const uint32_t len = d.len, skip = (uint32_t)(d.start & (ALIGN - 1));
@@ -311,14 +319,6 @@ __global__ void __launch_bounds__(LOCAL_THREADS, 1) k_local(Ctx c, const ChunkDe
             const uint32_t i = tid + v * LOCAL_THREADS;
             if (v < V && i < len) t[v] = buf(X)[skip + i];
         }
-        for (int q = tid; q < Q; q += LOCAL_THREADS) bins[q] = 0;
-        if (SPLIT && tid < Q) bulk_wait_read0();  // run stores of chunk j-1 have read buffer X^1
-        __syncthreads();  // S1: buffer X consumed (it becomes this chunk's sorted output)
-        if (tid == 0 && j + 1 < mine) {
-            if (!SPLIT) bulk_wait_read0();  // chunk j-1's bulk store has finished reading buffer X^1
-            issue(j + 1, nxt);
-            if (j + 2 < mine) nxt = cdesc[blockIdx.x + (j + 2) * gridDim.x];
-        }
         uint32_t rq[VMAX];  // rank << 16 | digit (0xffffffff: dropped)
 #pragma unroll
         for (int v = 0; v < VMAX; ++v) {
@@ -329,7 +329,19 @@ __global__ void __launch_bounds__(LOCAL_THREADS, 1) k_local(Ctx c, const ChunkDe
                 rq[v] = (atomicAdd(&bins[q], 1u) << 16) | q;
             }
         }
-        __syncthreads();  // S2
+        if (SPLIT && tid < Q) bulk_wait_read0();  // run stores of chunk j-1 have read buffer X^1
+        __syncthreads();  // S1: buffer X consumed (it becomes this chunk's sorted output), bins final
+        // chunk j+1 -> buffer X^1 once chunk j-1's stores have read it; the issuing
+        // thread (warp 1, LI) also issues the chunk's bulk store, warp 0 scans meanwhile
+        if (tid == LI && j + 1 < mine) {
+            if (!SPLIT) bulk_wait_read0();
+            issue(j + 1, nxt);
+            if (j + 2 < mine) nxt = cdesc[blockIdx.x + (j + 2) * gridDim.x];
+        }
+        if (tid >= 32) {  // the other bin array (last read by chunk j-1 before its S3) for chunk j+1
+            uint32_t *const bn = bins2 + (X ^ 1) * Qmax;
+            for (int q = tid - 32; q < Q; q += LOCAL_THREADS - 32) bn[q] = 0;
+        }
         if (tid < 32) {  // one warp: padded run starts (exclusive scan over the Q bins)
             const int per = (Q + 31) / 32, q0 = tid * per;
             uint32_t sum = 0;
@@ -392,8 +404,8 @@ __global__ void __launch_bounds__(LOCAL_THREADS, 1) k_local(Ctx c, const ChunkDe
                 tma_store_1d(static_cast<Tup *>(c.mid[rel]) + at, sorted + abin[tid], slots * TB);
                 bulk_commit();
             }
-        } else if (tid == 0 && tot) {
-            Tup *dst = static_cast<Tup *>(c.local[rel]) + (size_t)li * CR;
+        } else if (tid == LI && tot) {
+            Tup *dst = static_cast<Tup *>(c.local[rel]) + (size_t)(LP_RING ? li % LP_RING : li) * CR;
             tma_store_1d(dst, sorted, tot * TB);
             bulk_commit();
         }
@@ -633,7 +645,7 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
                         const uint32_t ahi = (k == sd.k1) ? sd.a1 : slots;
                         if (ahi > alo) {
                             sz = ahi - alo;
-                            src = (uint64_t)(xcb + k) * c.chunk_region + st + alo;
+                            src = (uint64_t)(LP_RING ? (xcb + k) % LP_RING : xcb + k) * c.chunk_region + st + alo;
                         }
                         pad = (SBITS && rel == 1 && v < slots && v >= alo && v < ahi) ? v - alo : 0xffffffffu;
                     }

@@ -23,8 +23,14 @@ namespace mgj {
 // < 32-byte tail of a partition waits (in registers of its owning thread)
 // for the next sub-tile.  For P = 4096 the alignment padding would not fit
 // shared memory, so SG = 1 (one tuple per store).
+#ifndef SCAT_SOA
+#define SCAT_SOA 0  // 4-byte keys: `sorted` held as key and payload arrays (4-byte random stores; measured slower: 4.42 vs 4.14 ms)
+#endif
 #ifndef SCAT_ALIAS
 #define SCAT_ALIAS 0  // 4-byte keys, P <= 1024: two 512-thread CTAs per SM, stage aliased into the sorted buffer (measured: 6.2 vs 4.1 ms)
+#endif
+#ifndef SCAT_RING
+#define SCAT_RING 0  // EXPERIMENT ONLY (wrong results): full-group stores land modulo SCAT_RING bytes of the arena (L2-resident)
 #endif
 struct ScatGeom {
     int T, SG, PPT, NT;
@@ -144,8 +150,13 @@ __global__ void __launch_bounds__(NT, ALIAS ? 2 : 1) k_scatter(Ctx c) {
     // `sorted` swizzle: the two 16-byte halves of every 32-byte group whose
     // index has bit 2 set are swapped, so that the write-out's 16-byte loads
     // (8 consecutive groups per quarter warp) hit distinct banks
+    // SOA (4-byte keys, 32-byte groups): `sorted` is a key array and a payload
+    // array; the scatter's random stores are 4 bytes wide (fewer bank conflicts
+    // than 8-byte ones) and the write-out interleaves 16 bytes of keys with 16
+    // bytes of payloads into the group's 32-byte store (conflict-free, no swizzle)
+    constexpr bool SOA = SCAT_SOA && sizeof(K) == 4 && SG == 4 && !ALIAS;
     auto swz = [](uint32_t s) -> uint32_t {
-        if constexpr (SG > 1) return s ^ (((s >> (SG == 4 ? 4 : 3)) & 1u) * (SG / 2));
+        if constexpr (SG > 1 && !SOA) return s ^ (((s >> (SG == 4 ? 4 : 3)) & 1u) * (SG / 2));
         else return s;
     };
     extern __shared__ __align__(128) unsigned char smem[];
@@ -156,6 +167,26 @@ __global__ void __launch_bounds__(NT, ALIAS ? 2 : 1) k_scatter(Ctx c) {
     K *const spay = skey + T;
     PInfo *const pinfo = reinterpret_cast<PInfo *>(sorted + T + 2 * (SG - 1) * P);  // 16-byte aligned
     uint32_t *const off = reinterpret_cast<uint32_t *>(pinfo + P);  // next free slot per partition
+    K *const ks = reinterpret_cast<K *>(sorted);  // SOA: keys, then payloads
+    K *const ps = ks + (T + 2 * (SG - 1) * P);
+    auto sput = [&](uint32_t x, const Tup &t) {
+        if constexpr (SOA) {
+            ks[x] = t.x;
+            ps[x] = t.y;
+        } else {
+            sorted[swz(x)] = t;
+        }
+    };
+    auto sget = [&](uint32_t x) -> Tup {
+        if constexpr (SOA) {
+            Tup t;
+            t.x = ks[x];
+            t.y = ps[x];
+            return t;
+        } else {
+            return sorted[swz(x)];
+        }
+    };
     __shared__ __align__(8) uint64_t bar;
     __shared__ uint32_t tmp[32];
     const int tid = threadIdx.x;
@@ -206,7 +237,7 @@ __global__ void __launch_bounds__(NT, ALIAS ? 2 : 1) k_scatter(Ctx c) {
             for (int k = 0; k < PPT; ++k)
 #pragma unroll
                 for (int i = 0; i < CW; ++i)
-                    if (i < (int)cc[k]) carry[k][i] = sorted[swz(lim[k] - cc[k] + i)];
+                    if (i < (int)cc[k]) carry[k][i] = sget(lim[k] - cc[k] + i);
             pending = false;
         }
     };
@@ -293,7 +324,7 @@ __global__ void __launch_bounds__(NT, ALIAS ? 2 : 1) k_scatter(Ctx c) {
                 if (!ALIAS) {
 #pragma unroll
                     for (int i = 0; i < CW; ++i)
-                        if (i < (int)cc[k]) sorted[swz(o + i)] = carry[k][i];
+                        if (i < (int)cc[k]) sput(o + i, carry[k][i]);
                 }
                 co[k] = o;
                 off[p] = o + cc[k];
@@ -342,7 +373,7 @@ __global__ void __launch_bounds__(NT, ALIAS ? 2 : 1) k_scatter(Ctx c) {
             for (int k = 0; k < PPT; ++k)
 #pragma unroll
                 for (int i = 0; i < CW; ++i)
-                    if (i < (int)ccw[k]) sorted[swz(co[k] + i)] = carry[k][i];
+                    if (i < (int)ccw[k]) sput(co[k] + i, carry[k][i]);
         } else if (tid == 0 && g + 1 < ntot) {
             issue(g + 1);
         }
@@ -359,7 +390,7 @@ __global__ void __launch_bounds__(NT, ALIAS ? 2 : 1) k_scatter(Ctx c) {
                 Tup t;
                 t.x = kk[v];
                 t.y = pp[v];
-                sorted[swz(pos[v])] = t;
+                sput(pos[v], t);
             }
         }
 #else
@@ -370,7 +401,7 @@ __global__ void __launch_bounds__(NT, ALIAS ? 2 : 1) k_scatter(Ctx c) {
                 Tup t;
                 t.x = kk[v];
                 t.y = pp[v];
-                sorted[swz(atomicAdd(&off[digit1(kk[v], P)], 1u))] = t;
+                sput(atomicAdd(&off[digit1(kk[v], P)], 1u), t);
             }
         }
 #endif
@@ -389,7 +420,12 @@ __global__ void __launch_bounds__(NT, ALIAS ? 2 : 1) k_scatter(Ctx c) {
                 slot[r] = (u0 + r * NT) * SG;
                 on[r] = u0 + r * NT < ngroups;
                 if (on[r]) {
-                    if constexpr (SG > 1) {  // two conflict-free 16-byte halves (swizzled)
+                    if constexpr (SOA) {  // 4 keys + 4 payloads -> (k0,p0,k1,p1 | k2,p2,k3,p3)
+                        const uint4 kv = *reinterpret_cast<const uint4 *>(ks + slot[r]);
+                        const uint4 pv = *reinterpret_cast<const uint4 *>(ps + slot[r]);
+                        gv[r].a = make_uint4(kv.x, pv.x, kv.y, pv.y);
+                        gv[r].b = make_uint4(kv.z, pv.z, kv.w, pv.w);
+                    } else if constexpr (SG > 1) {  // two conflict-free 16-byte halves (swizzled)
                         gv[r].a = *reinterpret_cast<const uint4 *>(sorted + swz(slot[r]));
                         gv[r].b = *reinterpret_cast<const uint4 *>(sorted + swz(slot[r] + SG / 2));
                     } else {
@@ -404,11 +440,12 @@ __global__ void __launch_bounds__(NT, ALIAS ? 2 : 1) k_scatter(Ctx c) {
             for (int r = 0; r < WU; ++r) {
                 if (on[r] && slot[r] + SG <= in[r].lim) {
                     char *dst = reinterpret_cast<char *>(in[r].wb + (ull)slot[r] * TB);
+                    if (SCAT_RING) dst = c.arena[0] + c.lay.recv[0] + ((dst - c.arena[0] - c.lay.recv[0]) & (ull)(SCAT_RING - 1));
                     if ((in[r].head >> 2) != slot[r]) {
                         st_group<GB>(dst, gv[r]);
                     } else {
                         for (uint32_t i = in[r].head & 3u; i < SG; ++i)
-                            reinterpret_cast<Tup *>(dst)[i] = sorted[swz(slot[r] + i)];
+                            reinterpret_cast<Tup *>(dst)[i] = sget(slot[r] + i);
                     }
                 }
             }

@@ -15,6 +15,14 @@ namespace mgj {
 #define LP_RING 0  // EXPERIMENT ONLY (wrong results): local output chunk regions modulo LP_RING, to time an L2-resident local buffer
 #endif
 
+#ifndef PROBE_L2PF
+#define PROBE_L2PF 0  // producers prefetch the runs of the item PROBE_L2PF rounds ahead into L2 (measured slower: 2.40-2.53 vs 1.96 ms)
+#endif
+
+#ifndef PROBE_CPASYNC
+#define PROBE_CPASYNC 0  // producers copy runs with 16-byte cp.async (LDGSTS) instead of one TMA bulk copy per run (measured slower: 4.64 vs 1.96 ms)
+#endif
+
 #ifndef PROBE_U2
 #define PROBE_U2 0  // packed probe: two S slots per step (measured slower: 2.00 vs 1.96 ms)
 #endif
@@ -595,7 +603,7 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
     const ItemX *items = reinterpret_cast<const ItemX *>(c.items);
     if (tid == 0) {
         for (int s = 0; s < PROBE_NST; ++s) {
-            mbar_init(&full[s], PROBE_PPI);
+            mbar_init(&full[s], PROBE_CPASYNC ? PROBE_PPI * 33 : PROBE_PPI);
             mbar_init(&empty[s], 1);
         }
         fence_mbar_init();
@@ -657,6 +665,19 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
                     }
                     const uint32_t dst = run + incl - sz;
                     const uint32_t gsum = __shfl_sync(0xffffffffu, incl, 31);
+                    if (PROBE_CPASYNC) {
+                        // the warp copies the batch's runs one after another, 16 bytes per lane
+                        constexpr uint32_t PT = 16 / TB;  // tuples per 16-byte piece
+                        for (int r = 0; r < 32; ++r) {
+                            const uint32_t rs = __shfl_sync(0xffffffffu, sz, r);
+                            if (!rs) continue;
+                            const uint64_t rsrc = __shfl_sync(0xffffffffu, src, r);
+                            const uint32_t rdst = __shfl_sync(0xffffffffu, dst, r);
+                            const uint32_t n16 = rs / PT;
+                            for (uint32_t i = lane; i < n16; i += 32)
+                                cp_async16(dstbase + rdst + i * PT, lbase + rsrc + i * PT);
+                        }
+                    } else {
                     if (lane == 0 && gsum)
                         asm volatile("mbarrier.expect_tx.relaxed.cta.shared::cta.b64 [%0], %1;" ::"r"(
                                          smem_u32(&full[s])),
@@ -664,16 +685,37 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
                                      : "memory");
                     __syncwarp();
                     if (sz) tma_load_1d(dstbase + dst, lbase + src, sz * TB, &full[s], pol);
+                    }
                     if (pad != 0xffffffffu) atomicOr(&pb[(dst + pad) >> 5], 1u << ((dst + pad) & 31));
                     run += gsum;
                 }
                 if (lane == 0) totals[s][rel] = run;
+                if (PROBE_L2PF && j + PROBE_L2PF * NPI < mine) {
+                    // the same side of the item PROBE_L2PF rounds ahead: its runs -> L2, so that
+                    // its stage loads hit L2 (more bytes in flight than the stages can hold)
+                    const ItemX y = items[blockIdx.x + (j + PROBE_L2PF * NPI) * gridDim.x];
+                    const Side sy = rel ? y.it.s : y.it.r;
+                    const uint32_t ycb = rel ? y.cb[1] : y.cb[0], ynch = rel ? y.nch[1] : y.nch[0];
+                    const uint16_t *F0 = (rel ? c.eoff[1] : c.eoff[0]) + (size_t)(Q + 1) * ycb + (size_t)y.it.q * ynch;
+                    const uint32_t kend2 = min(sy.k1, ynch - 1);
+                    const uint32_t np2 = sy.k0 <= kend2 ? kend2 - sy.k0 + 1 : 0;
+                    for (uint32_t m = lane; m < np2; m += 32) {
+                        const uint32_t k = sy.k0 + m;
+                        uint32_t st, slots, v;
+                        decode_run<ALIGN>(F0[k], F0[k + ynch], st, slots, v);
+                        const uint32_t alo = (k == sy.k0) ? sy.a0 : 0;
+                        const uint32_t ahi = (k == sy.k1) ? sy.a1 : slots;
+                        if (ahi > alo)
+                            prefetch_l2(lbase + (uint64_t)(ycb + k) * c.chunk_region + st + alo, (ahi - alo) * TB);
+                    }
+                }
             }
             if (lane == 0 && rel0 == 0) {
                 stage_p[s] = (uint32_t)(plo + (BAp ? x.it.pi >> BAp : x.it.pi));
                 stage_soff[s] = x.soff;
             }
             __syncwarp();
+            if (PROBE_CPASYNC) cp_async_mbar_arrive(&full[s]);  // fires when this lane's copies have landed
             if (lane == 0) mbar_arrive(&full[s]);
             x = xn;
         }

@@ -306,7 +306,7 @@ mgj_status mgj_plan(const mgj_config *cfg, const mgj_peers *peers, mgj_handle *o
     const size_t z_err = zo; zo += 256;
     const size_t z_cop = zo; zo += align_up(2ull * P * Qm * 4, 256);
     // tiles: one per scatter CTA (two per SM when the scatter runs two CTAs per SM)
-    const int G = h->nsm * (scat_geom(P, n.c.key_bytes).alias ? 2 : 1);
+    const int G = h->nsm * (scat_geom(P, n.c.key_bytes).NT <= 512 ? 2 : 1);  // scatter tiles: one per CTA
     const size_t z_th = zo; zo += align_up(2ull * G * P * 4, 256);
     const size_t z_ha = zo; zo += align_up(2ull * local2_vcap(P) * 4, 256);
     h->zero_bytes = zo;

@@ -26,6 +26,15 @@ namespace mgj {
 #ifndef SCAT_SOA
 #define SCAT_SOA 0  // 4-byte keys: `sorted` held as key and payload arrays (4-byte random stores; measured slower: 4.42 vs 4.14 ms)
 #endif
+#ifndef SCAT_LDG
+#define SCAT_LDG 0  // sub-tiles loaded straight into registers one sub-tile ahead, no shared-memory stage (measured slower: 4.73 vs 4.13 ms)
+#endif
+#ifndef SCAT_T4
+#define SCAT_T4 8192  // sub-tile of the 4-byte-key, P <= 1024 instance
+#endif
+#ifndef SCAT_2CTA
+#define SCAT_2CTA 0  // 4-byte keys, P <= 1024: two 512-thread CTAs per SM, 4096-tuple sub-tiles, 16-byte groups (measured slower: 9.2 vs 4.1 ms)
+#endif
 #ifndef SCAT_ALIAS
 #define SCAT_ALIAS 0  // 4-byte keys, P <= 1024: two 512-thread CTAs per SM, stage aliased into the sorted buffer (measured: 6.2 vs 4.1 ms)
 #endif
@@ -38,7 +47,9 @@ struct ScatGeom {
 };
 __host__ __device__ constexpr ScatGeom scat_geom(int P, int key_bytes) {
     return key_bytes == 4
-               ? (P <= 1024 ? (SCAT_ALIAS ? ScatGeom{4096, 4, P <= 512 ? 1 : 2, 512, true} : ScatGeom{8192, 4, 1, 1024, false})
+               ? (P <= 1024 ? (SCAT_ALIAS  ? ScatGeom{4096, 4, P <= 512 ? 1 : 2, 512, true}
+                               : SCAT_2CTA ? ScatGeom{4096, 2, P <= 512 ? 1 : 2, 512, false}
+                                           : ScatGeom{SCAT_T4, 4, 1, 1024, false})
                   : P == 2048 ? ScatGeom{4096, 4, 2, 1024, false} : ScatGeom{8192, 1, 4, 1024, false})
                : (P <= 1024 ? ScatGeom{4096, 2, 1, 1024, false} : P == 2048 ? ScatGeom{2048, 2, 2, 1024, false}
                                                                       : ScatGeom{4096, 1, 4, 1024, false});
@@ -55,7 +66,7 @@ struct __align__(16) PInfo {
 __host__ __device__ inline size_t scat_smem_bytes(int P, int key_bytes) {
     const ScatGeom g = scat_geom(P, key_bytes);
     const size_t TB = 2 * (size_t)key_bytes;
-    return (g.alias ? 0 : 2 * (size_t)g.T * key_bytes)      // input stage: keys + payloads (SoA)
+    return ((g.alias || SCAT_LDG) ? 0 : 2 * (size_t)g.T * key_bytes)  // input stage: keys + payloads (SoA)
            + ((size_t)g.T + 2 * (size_t)(g.SG - 1) * P) * TB  // partition-sorted sub-tile (+ carries, group padding)
            + (size_t)P * sizeof(PInfo)
            + (size_t)P * 4;                                  // next free slot per partition
@@ -135,7 +146,7 @@ __device__ __forceinline__ void st_group(void *dst, const typename Vec<BYTES>::T
 // peer after a system fence.
 // ---------------------------------------------------------------------------
 template <typename K, int T, int SG, int PPT, int NT, bool ALIAS>
-__global__ void __launch_bounds__(NT, ALIAS ? 2 : 1) k_scatter(Ctx c) {
+__global__ void __launch_bounds__(NT, NT <= 512 ? 2 : 1) k_scatter(Ctx c) {
     using Tup = typename TupT<K>::T;
     constexpr int TB = (int)sizeof(Tup);
     constexpr int V = T / NT;                  // tuples per thread per sub-tile
@@ -156,13 +167,16 @@ __global__ void __launch_bounds__(NT, ALIAS ? 2 : 1) k_scatter(Ctx c) {
     // bytes of payloads into the group's 32-byte store (conflict-free, no swizzle)
     constexpr bool SOA = SCAT_SOA && sizeof(K) == 4 && SG == 4 && !ALIAS;
     auto swz = [](uint32_t s) -> uint32_t {
-        if constexpr (SG > 1 && !SOA) return s ^ (((s >> (SG == 4 ? 4 : 3)) & 1u) * (SG / 2));
+        if constexpr (SG > 1 && !SOA && SG * sizeof(Tup) == 32) return s ^ (((s >> (SG == 4 ? 4 : 3)) & 1u) * (SG / 2));
         else return s;
     };
     extern __shared__ __align__(128) unsigned char smem[];
     const int P = c.P;
     // ALIAS: the stage is the head of the sorted buffer (loaded after the write-out)
-    Tup *const sorted = reinterpret_cast<Tup *>(smem + (ALIAS ? 0 : 2 * T * sizeof(K)));
+    // LDG: sub-tile g+1 is loaded into registers (16-byte streaming loads) while
+    // g is laid out, ranked and written out; no stage, no TMA, no mbarrier
+    constexpr bool LDG = SCAT_LDG && !ALIAS;
+    Tup *const sorted = reinterpret_cast<Tup *>(smem + ((ALIAS || LDG) ? 0 : 2 * T * sizeof(K)));
     K *const skey = reinterpret_cast<K *>(ALIAS ? static_cast<void *>(sorted) : static_cast<void *>(smem));
     K *const spay = skey + T;
     PInfo *const pinfo = reinterpret_cast<PInfo *>(sorted + T + 2 * (SG - 1) * P);  // 16-byte aligned
@@ -288,9 +302,42 @@ __global__ void __launch_bounds__(NT, ALIAS ? 2 : 1) k_scatter(Ctx c) {
             out[0] = v.x & 0xffffu, out[1] = v.x >> 16, out[2] = v.y & 0xffffu, out[3] = v.y >> 16;
         }
     };
+    K kn[V], pn[V];  // LDG: the next sub-tile
+    auto fetch = [&](uint32_t g) {
+        int rel;
+        uint64_t first;
+        uint32_t len;
+        subtile(g, rel, first, len);
+        const K *gk = static_cast<const K *>(c.in_key[rel]) + first;
+        const K *gp = static_cast<const K *>(c.in_pay[rel]) + first;
+        if (len == T) {
+#pragma unroll
+            for (int u = 0; u < NU; ++u) {
+                const uint32_t i0 = (uint32_t)(u * NT + tid) * LU;
+                const uint4 a = __ldcs(reinterpret_cast<const uint4 *>(gk + i0));
+                const uint4 b = __ldcs(reinterpret_cast<const uint4 *>(gp + i0));
+                memcpy(&kn[u * LU], &a, 16);
+                memcpy(&pn[u * LU], &b, 16);
+            }
+        } else {
+#pragma unroll
+            for (int u = 0; u < NU; ++u) {
+#pragma unroll
+                for (int e = 0; e < LU; ++e) {
+                    const uint32_t i = (uint32_t)(u * NT + tid) * LU + e;
+                    kn[u * LU + e] = i < len ? __ldcs(gk + i) : (K)0;
+                    pn[u * LU + e] = i < len ? __ldcs(gp + i) : (K)0;
+                }
+            }
+        }
+    };
     uint32_t ncnt[PPT];
     load_counts(0, ncnt);
-    if (tid == 0 && ntot > 0) issue(0);
+    if (LDG) {
+        if (ntot > 0) fetch(0);
+    } else if (tid == 0 && ntot > 0) {
+        issue(0);
+    }
     int cur_rel = -1;
     for (uint32_t g = 0; g < ntot; ++g) {
         int rel;
@@ -342,11 +389,16 @@ __global__ void __launch_bounds__(NT, ALIAS ? 2 : 1) k_scatter(Ctx c) {
             o += seg[k];
         }
         pending = SG > 1;
+        K kk[V], pp[V];
+        if constexpr (LDG) {
+#pragma unroll
+            for (int v = 0; v < V; ++v) kk[v] = kn[v], pp[v] = pn[v];
+            if (g + 1 < ntot) fetch(g + 1);
+        } else {
         mbar_wait(&bar, g & 1);
         const uint32_t body = len & ~(uint32_t)(LU - 1);
         const K *gk = static_cast<const K *>(c.in_key[rel]) + first;
         const K *gp = static_cast<const K *>(c.in_pay[rel]) + first;
-        K kk[V], pp[V];
         if (len == T) {  // full sub-tile: branch-free vector loads
 #pragma unroll
             for (int u = 0; u < NU; ++u) {
@@ -367,6 +419,7 @@ __global__ void __launch_bounds__(NT, ALIAS ? 2 : 1) k_scatter(Ctx c) {
                 }
             }
         }
+        }
         __syncthreads();  // S1: offsets and carries in place, stage consumed
         if (ALIAS) {  // the stage region is free now: carries to their segment heads
 #pragma unroll
@@ -374,7 +427,7 @@ __global__ void __launch_bounds__(NT, ALIAS ? 2 : 1) k_scatter(Ctx c) {
 #pragma unroll
                 for (int i = 0; i < CW; ++i)
                     if (i < (int)ccw[k]) sput(co[k] + i, carry[k][i]);
-        } else if (tid == 0 && g + 1 < ntot) {
+        } else if (!LDG && tid == 0 && g + 1 < ntot) {
             issue(g + 1);
         }
 #if SCAT_ATOM_FIRST
@@ -425,7 +478,7 @@ __global__ void __launch_bounds__(NT, ALIAS ? 2 : 1) k_scatter(Ctx c) {
                         const uint4 pv = *reinterpret_cast<const uint4 *>(ps + slot[r]);
                         gv[r].a = make_uint4(kv.x, pv.x, kv.y, pv.y);
                         gv[r].b = make_uint4(kv.z, pv.z, kv.w, pv.w);
-                    } else if constexpr (SG > 1) {  // two conflict-free 16-byte halves (swizzled)
+                    } else if constexpr (GB == 32) {  // two conflict-free 16-byte halves (swizzled)
                         gv[r].a = *reinterpret_cast<const uint4 *>(sorted + swz(slot[r]));
                         gv[r].b = *reinterpret_cast<const uint4 *>(sorted + swz(slot[r] + SG / 2));
                     } else {
@@ -479,8 +532,11 @@ inline void (*scatter_kernel(int P))(Ctx) {
 #if SCAT_ALIAS
         if (P <= 512) return k_scatter<K, 4096, 4, 1, 512, true>;
         if (P == 1024) return k_scatter<K, 4096, 4, 2, 512, true>;
+#elif SCAT_2CTA
+        if (P <= 512) return k_scatter<K, 4096, 2, 1, 512, false>;
+        if (P == 1024) return k_scatter<K, 4096, 2, 2, 512, false>;
 #else
-        if (P <= 1024) return k_scatter<K, 8192, 4, 1, 1024, false>;
+        if (P <= 1024) return k_scatter<K, SCAT_T4, 4, 1, 1024, false>;
 #endif
         if (P == 2048) return k_scatter<K, 4096, 4, 2, 1024, false>;
         return k_scatter<K, 8192, 1, 4, 1024, false>;

@@ -71,6 +71,21 @@ __device__ __forceinline__ void tma_store_1d(void *gdst, const void *ssrc, uint3
                  : "memory");
 }
 
+// 16-byte asynchronous global -> shared copy (LDGSTS, L2 only), and an arrive
+// on an mbarrier once all of this thread's prior cp.async copies have landed
+// (.noinc: the arrival is part of the barrier's expected count).
+__device__ __forceinline__ void cp_async16(void *sdst, const void *gsrc) {
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(sdst)), "l"(gsrc) : "memory");
+}
+__device__ __forceinline__ void cp_async_mbar_arrive(uint64_t *bar) {
+    asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+
+// Bulk prefetch of [gsrc, gsrc + bytes) into L2 (16-byte aligned, multiple of 16 bytes).
+__device__ __forceinline__ void prefetch_l2(const void *gsrc, uint32_t bytes) {
+    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(gsrc), "r"(bytes) : "memory");
+}
+
 __device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
 
 // Wait until the shared-memory sources of all committed bulk stores were read.

@@ -73,7 +73,12 @@ typedef struct {
     int32_t  local_split_bits;         /* a4 first (histogram) pass: 0 = auto (only for owned partitions
                                           of more than 256 chunks), -1 = never, 1..6 = always, 2^k
                                           sub-partitions per owned partition */
-    int32_t  reserved[6];              /* must be zero */
+    int32_t  skew_bcast;               /* a2 selective broadcast:
+                                          0 = auto (heavy partitions with (N-1)|R_p| < |S_p|: R_p is read by
+                                          every rank from its owner, S_p stays where it is), -1 = never,
+                                          1 = every partition passing the traffic test.  Never with one
+                                          rank or MGJ_SHUFFLE_EXTERNAL */
+    int32_t  reserved[5];              /* must be zero */
 } mgj_config;
 
 /*
@@ -192,7 +197,8 @@ const char *mgj_strerror(mgj_status s);
  */
 mgj_status mgj_plan_host(int32_t world_size, int32_t rank, int32_t bits,
                          const uint32_t *hist, int32_t *owner,
-                         uint64_t *send_off, uint64_t *recv_size);
+                         uint64_t *send_off, uint64_t *recv_size,
+                         int32_t skew_bcast, uint8_t *bcast);
 
 #ifdef __cplusplus
 }

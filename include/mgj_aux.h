@@ -43,7 +43,8 @@ typedef enum {
     MGJ_DBG_LOCAL_R = 8,     /* tuples after local partitioning (a4) */
     MGJ_DBG_LOCAL_S = 9,
     MGJ_DBG_META = 10,       /* i32[16]: p_lo, p_hi, B2, plan_ok, chunks_r, chunks_s, n_items, C, BA, QB,
-                                NLP, chunks_r / chunks_s of the chunked pass after a first pass */
+                                NLP, chunks_r / chunks_s of the chunked pass after a first pass,
+                                np (owned partitions incl. broadcast), n_bcast */
     MGJ_DBG_CHUNK_OFF_R = 11,/* u16[chunks_r][2^B2+1]  sub-partition offsets per chunk */
     MGJ_DBG_CHUNK_OFF_S = 12,
     MGJ_DBG_CHUNK_BASE = 13, /* u32[2][4P+1]         first chunk of each (sub-)partition of the chunked pass */
@@ -53,7 +54,9 @@ typedef enum {
     MGJ_DBG_OUT_PAY_S = 17,
     MGJ_DBG_MID_R = 18,      /* tuples after the first local pass (sub-partitions, two-level a4 only) */
     MGJ_DBG_MID_S = 19,
-    MGJ_DBG_VSTART = 20      /* u64[2][L+1] sub-partition starts (slots) in MID_R / MID_S */
+    MGJ_DBG_VSTART = 20,     /* u64[2][L+1] sub-partition starts (slots) in MID_R / MID_S */
+    MGJ_DBG_BCAST = 21,      /* u8[P]                selective-broadcast flag of each global partition (a2) */
+    MGJ_DBG_PLIST = 22       /* i32[np]              owned partitions: the range, then broadcast ones outside it */
 } mgj_debug_what;
 
 mgj_status mgj_debug_copy(mgj_handle h, int32_t what, void *dst, uint64_t bytes, uint64_t *size_out);

@@ -42,7 +42,16 @@ enum Meta { MT_PLO = 0, MT_PHI = 1, MT_B2 = 2, MT_OK = 3, MT_NCH_R = 4, MT_NCH_S
             MT_NLP = 10,     // partitions of the chunked local pass: owned partitions, or sub-partitions
             MT_NCHB_R = 11,  // chunks of the chunked pass after a first pass (R, S)
             MT_NCHB_S = 12,
+            MT_NP = 13,      // owned partitions (the range + broadcast partitions outside it)
+            MT_NBC = 14,     // broadcast partitions (selective broadcast, NEXT-2)
             MT_COUNT = 16 };
+
+// Source rank of a received piece travels in the top byte of its start
+// (starts are < 2^56 tuples): a broadcast partition's R piece lives in its
+// root's receive buffer and is read from there by the local pass.
+constexpr int PIECE_SRC_SHIFT = 56;
+__host__ __device__ __forceinline__ uint64_t piece_off(uint64_t v) { return v & ((1ull << PIECE_SRC_SHIFT) - 1); }
+__host__ __device__ __forceinline__ int piece_src(uint64_t v) { return (int)(v >> PIECE_SRC_SHIFT); }
 
 // Arena layout (bytes from each rank's arena base; identical on all ranks).
 struct Arena {
@@ -99,7 +108,10 @@ struct Ctx {
     int32_t sub_ns;               // sub-tiles per tile (capacity)
     uint32_t *ticket;             // [TK_COUNT]
     int32_t *meta;                // [MT_COUNT]
-    int32_t *owner;               // [P]
+    int32_t *owner;               // [P] range owner (a broadcast partition's root)
+    uint8_t *bcast;               // [P] selective broadcast flags (a2)
+    int32_t *plist;               // [P] owned partitions: the range, then broadcast partitions outside it
+    int32_t bcast_cfg;            // mgj_config.skew_bcast
     uint64_t *send_off;           // [2][P]
     uint64_t *seg_start;          // [2][P]
     uint64_t *seg_len;            // [2][P]

@@ -182,6 +182,27 @@ __host__ __device__ inline int owner_of(uint64_t cum_before, uint64_t T, uint64_
     return o >= (uint64_t)N ? N - 1 : (int)o;
 }
 
+// Selective broadcast of partition p (the paper's
+// assignment step P:418-444 after Track-Join: a partition is migrated or
+// selectively broadcast, whichever moves fewer tuples; heavy hitters
+// P:386-395).  Broadcasting R_p to every rank and keeping S_p where it is
+// moves (N-1)|R_p| tuples; single-owner hash partitioning moves about
+// (N-1)/N (|R_p| + |S_p|).  Broadcast wins when (N-1)|R_p| < |S_p| (both
+// sides times N, the R_p terms collected).  cfg: < 0 never; 0 (auto) only
+// heavy partitions, |S_p| >= 2 |S| / P, so uniform data never broadcasts;
+// > 0 every partition that passes the traffic test.  Never with one rank.
+__host__ __device__ inline bool bcast_of(uint64_t r, uint64_t s, uint64_t s_total, int N, int P, int cfg) {
+    if (N < 2 || cfg < 0 || s == 0) return false;
+    if ((uint64_t)(N - 1) * r >= s) return false;
+    return cfg > 0 || s * (uint64_t)P >= 2 * s_total;
+}
+
+// Weight of p in the owner ranges: a broadcast partition's S stays spread
+// over the ranks, its owner (the root, which receives R_p) gets R_p + S_p/N.
+__host__ __device__ inline uint64_t owner_weight(uint64_t r, uint64_t s, bool bc, int N) {
+    return bc ? r + (s + (uint64_t)N - 1) / (uint64_t)N : r + s;
+}
+
 __host__ __device__ inline int ceil_log2_u64(uint64_t x) {
     int l = 0;
     while (l < 63 && (1ull << l) < x) ++l;
@@ -205,51 +226,79 @@ __host__ __device__ inline int choose_b2(uint64_t max_r, uint64_t mean_rs, int b
 
 // ---------------------------------------------------------------------------
 // a2 device plan: one CTA of 1024 threads.  Every rank computes the same
-// owner[] and receive sizes from the same all-gathered histograms, plus its
-// own send offsets (u64 tuples into the owner's receive buffer, layout:
-// owned p ascending, then source rank ascending), its owned segments, the
-// local radix bits B2 and the chunk table of the local pass.
+// broadcast flags, owner[] and receive sizes from the same all-gathered
+// histograms, plus its own send offsets (u64 tuples into the destination's
+// receive buffer), its owned partitions, the local radix bits B2 and the
+// chunk table of the local pass.
+// Receive layout of rank d.  R: the partitions of d's range ascending, each
+// [source rank ascending] (a broadcast partition's R lands at its root, the
+// range owner, like any other).  S: the non-broadcast partitions of d's range
+// ascending, each [source ascending], then every broadcast partition
+// ascending with d's own S tuples only.  Owned list of d (plist): its range,
+// then the broadcast partitions outside it; the R side of those is read from
+// the root's receive buffer by the local pass (a pull broadcast).
 // ---------------------------------------------------------------------------
 __global__ void __launch_bounds__(1024) k_plan(Ctx c) {
     extern __shared__ uint64_t sp[];
     const int P = c.P, N = c.world, tid = threadIdx.x;
     uint64_t *tot0 = sp, *tot1 = sp + P, *pre0 = sp + 2 * P, *pre1 = sp + 3 * P, *cum = sp + 4 * P;
     int32_t *own = reinterpret_cast<int32_t *>(sp + 5 * P);
-    uint32_t *chn = reinterpret_cast<uint32_t *>(own + P);  // [P+1] chunk counts -> base (one rel at a time)
+    uint32_t *chn = reinterpret_cast<uint32_t *>(own + P);  // [P+1] scratch scans (u32)
+    uint8_t *bcf = reinterpret_cast<uint8_t *>(chn + P + 1);  // [P] broadcast flags
     __shared__ uint64_t tmp[33];
     __shared__ uint32_t tmp32[33];
     __shared__ int first[MAX_RANKS], endp[MAX_RANKS];
-    __shared__ int ok, cap_bad;
-    __shared__ unsigned long long maxr, sumrs;
+    __shared__ int ok, cap_bad, nbc;
+    __shared__ unsigned long long maxr, sumrs, stot, bcs[MAX_RANKS];
     if (tid == 0) {
         ok = wait_all_flags(c, SIG_HIST);
         cap_bad = 0;
         maxr = 0;
         sumrs = 0;
+        stot = 0;
+        nbc = 0;
     }
-    if (tid < MAX_RANKS) first[tid] = endp[tid] = P;
+    if (tid < MAX_RANKS) first[tid] = endp[tid] = P, bcs[tid] = 0;
     __syncthreads();
     if (!ok) {
         if (tid == 0) c.meta[MT_OK] = 0;
         return;
     }
     const uint32_t *mail = reinterpret_cast<const uint32_t *>(c.arena[c.rank] + c.lay.mail);
-    for (int p = tid; p < P; p += blockDim.x) {
-        uint64_t t0 = 0, t1 = 0;
-        for (int g = 0; g < N; ++g) {
-            t0 += __ldcg(mail + (size_t)(g * 2 + 0) * P + p);
-            t1 += __ldcg(mail + (size_t)(g * 2 + 1) * P + p);
+    auto H = [&](int g, int rel, int p) -> uint32_t { return __ldcg(mail + (size_t)(g * 2 + rel) * P + p); };
+    {
+        unsigned long long st = 0;
+        for (int p = tid; p < P; p += blockDim.x) {
+            uint64_t t0 = 0, t1 = 0;
+            for (int g = 0; g < N; ++g) t0 += H(g, 0, p), t1 += H(g, 1, p);
+            tot0[p] = pre0[p] = t0;
+            tot1[p] = t1;
+            st += t1;
         }
-        tot0[p] = pre0[p] = t0;
-        tot1[p] = pre1[p] = t1;
-        cum[p] = t0 + t1;
+        st = warp_sum(st);
+        if ((tid & 31) == 0 && st) atomicAdd(&stot, st);
+    }
+    __syncthreads();
+    const int bcfg = c.ext ? -1 : c.bcast_cfg;
+    for (int p = tid; p < P; p += blockDim.x) {
+        const bool bc = bcast_of(tot0[p], tot1[p], stot, N, P, bcfg);
+        bcf[p] = bc;
+        c.bcast[p] = bc;
+        pre1[p] = bc ? 0 : tot1[p];  // S layout: broadcast partitions are not in the owner's range part
+        cum[p] = owner_weight(tot0[p], tot1[p], bc, N);
+        chn[p] = bc ? H(c.rank, 1, p) : 0u;  // this rank's own S of broadcast partitions
+        if (bc) {
+            atomicAdd(&nbc, 1);
+            for (int d = 0; d < N; ++d) atomicAdd(&bcs[d], (unsigned long long)H(d, 1, p));
+        }
     }
     __syncthreads();
     block_excl_scan_u64(pre0, P, tmp);
     block_excl_scan_u64(pre1, P, tmp);
+    block_excl_scan_u32(chn, P, tmp32);  // chn[p] = own S of broadcast partitions before p
     const uint64_t total = block_excl_scan_u64(cum, P, tmp);
     for (int p = tid; p < P; p += blockDim.x) {
-        const int o = owner_of(cum[p], tot0[p] + tot1[p], total, N, p, P);
+        const int o = owner_of(cum[p], owner_weight(tot0[p], tot1[p], bcf[p], N), total, N, p, P);
         own[p] = o;
         c.owner[p] = o;
     }
@@ -259,41 +308,58 @@ __global__ void __launch_bounds__(1024) k_plan(Ctx c) {
         if (p == P - 1 || own[p + 1] != own[p]) endp[own[p]] = p + 1;
     }
     __syncthreads();
+    // S tuples of this rank's own range part (non-broadcast), where its broadcast part starts
+    const uint64_t s_range_me = first[c.rank] < P ? pre1[endp[c.rank] - 1] + (bcf[endp[c.rank] - 1] ? 0 : tot1[endp[c.rank] - 1]) - pre1[first[c.rank]] : 0;
     for (int p = tid; p < P; p += blockDim.x) {
         const int f = first[own[p]];
         uint64_t m0 = 0, m1 = 0;
-        for (int g = 0; g < c.rank; ++g) {
-            m0 += __ldcg(mail + (size_t)(g * 2 + 0) * P + p);
-            m1 += __ldcg(mail + (size_t)(g * 2 + 1) * P + p);
-        }
-        const uint64_t b0 = pre0[p] - pre0[f], b1 = pre1[p] - pre1[f];
+        for (int g = 0; g < c.rank; ++g) m0 += H(g, 0, p), m1 += H(g, 1, p);
+        const uint64_t b0 = pre0[p] - pre0[f];
+        const uint64_t b1 = bcf[p] ? s_range_me + chn[p] : pre1[p] - pre1[f];
         if (!c.ext) {
             c.send_off[p] = b0 + m0;
-            c.send_off[P + p] = b1 + m1;
+            c.send_off[P + p] = bcf[p] ? b1 : b1 + m1;  // broadcast partition: S goes to this rank itself
         }
         c.seg_start[p] = b0;
         c.seg_start[P + p] = b1;
         c.seg_len[p] = tot0[p];
-        c.seg_len[P + p] = tot1[p];
+        c.seg_len[P + p] = bcf[p] ? H(c.rank, 1, p) : tot1[p];
     }
     if (tid < 2 * MAX_RANKS) {
         const int d = tid >> 1, rel = tid & 1;
         uint64_t size = 0;
         if (d < N && first[d] < P) {
             const uint64_t *pre = rel ? pre1 : pre0;
-            const uint64_t *tot = rel ? tot1 : tot0;
-            size = pre[endp[d] - 1] + tot[endp[d] - 1] - pre[first[d]];
+            const int l = endp[d] - 1;
+            const uint64_t last = rel ? (bcf[l] ? 0 : tot1[l]) : tot0[l];
+            size = pre[l] + last - pre[first[d]];
         }
+        if (d < N && rel) size += bcs[d];
         c.recv_size[rel * MAX_RANKS + d] = size;
         if (size > c.recv_cap[rel]) atomicOr(&cap_bad, 1);
     }
     const int plo = first[c.rank] < P ? first[c.rank] : 0;
     const int phi = first[c.rank] < P ? endp[c.rank] : 0;
+    __syncthreads();
+    // owned list: the range, then the broadcast partitions outside it (ascending)
+    for (int p = tid; p < P; p += blockDim.x) chn[p] = (bcf[p] && (p < plo || p >= phi)) ? 1u : 0u;
+    __syncthreads();
+    const int nout = (int)block_excl_scan_u32(chn, P, tmp32);
+    const int nr = phi - plo, np = nr + nout;
+    for (int p = tid; p < P; p += blockDim.x) {
+        if (p >= plo && p < phi) c.plist[p - plo] = p;
+        else if (bcf[p]) c.plist[nr + chn[p]] = p;
+    }
+    __syncthreads();
+    // per owned partition: R and S sizes of its received pieces
+    auto own_p = [&](int i) -> int { return i < nr ? plo + i : c.plist[i]; };
+    auto own_len = [&](int rel, int p) -> uint64_t { return rel ? (bcf[p] ? (uint64_t)H(c.rank, 1, p) : tot1[p]) : tot0[p]; };
     {  // largest owned R partition and total owned R + S: warp reductions, one shared atomic per warp
         unsigned long long mr = 0, sr = 0;
-        for (int p = plo + tid; p < phi; p += blockDim.x) {
+        for (int i = tid; i < np; i += blockDim.x) {
+            const int p = own_p(i);
             mr = max(mr, (unsigned long long)tot0[p]);
-            sr += tot0[p] + tot1[p];
+            sr += tot0[p] + own_len(1, p);
         }
 #pragma unroll
         for (int o = 16; o > 0; o >>= 1) {
@@ -306,23 +372,26 @@ __global__ void __launch_bounds__(1024) k_plan(Ctx c) {
         }
     }
     __syncthreads();
-    const int B2 = choose_b2(maxr, phi > plo ? sumrs / (uint64_t)(phi - plo) : 0, c.b2_cfg, c.b2_max,
+    const int B2 = choose_b2(maxr, np > 0 ? sumrs / (uint64_t)np : 0, c.b2_cfg, c.b2_max,
                              (uint64_t)c.probe_target);
-    // received pieces of every owned partition pi: P2P — one piece (the whole
-    // segment, sources ascending inside it); EXTERNAL — one piece per source
-    // rank g, the receive area being [g0 | g1 | ...], each [owned p ascending]
-    const int np = phi - plo;
+    // received pieces of every owned partition i: P2P — one piece per relation
+    // (the whole segment, sources ascending inside it; a broadcast partition's
+    // R piece in its root's buffer); EXTERNAL — one piece per source rank g,
+    // the receive area being [g0 | g1 | ...], each [owned p ascending]
     const uint64_t C = (uint64_t)c.chunk_tuples;
     const uint32_t *mine = mail + (size_t)c.rank * 2 * P;
     for (int rel = 0; rel < 2; ++rel) {
         uint64_t *ps = c.piece_start + (size_t)rel * P * MAX_RANKS;
         uint32_t *pl = c.piece_len + (size_t)rel * P * MAX_RANKS;
         if (!c.ext) {
-            for (int i = tid; i < np; i += blockDim.x)
+            for (int i = tid; i < np; i += blockDim.x) {
+                const int p = own_p(i);
+                const uint64_t src = rel ? (uint64_t)c.rank : (uint64_t)own[p];
                 for (int g = 0; g < MAX_RANKS; ++g) {
-                    ps[(size_t)i * MAX_RANKS + g] = g == 0 ? c.seg_start[rel * P + plo + i] : 0;
-                    pl[(size_t)i * MAX_RANKS + g] = g == 0 ? (uint32_t)(rel ? tot1 : tot0)[plo + i] : 0;
+                    ps[(size_t)i * MAX_RANKS + g] = g == 0 ? (c.seg_start[rel * P + p] | src << PIECE_SRC_SHIFT) : 0;
+                    pl[(size_t)i * MAX_RANKS + g] = g == 0 ? (uint32_t)own_len(rel, p) : 0;
                 }
+            }
             continue;
         }
         uint64_t displ = 0;  // start of source g's block in this rank's receive area
@@ -332,7 +401,7 @@ __global__ void __launch_bounds__(1024) k_plan(Ctx c) {
             __syncthreads();
             const uint32_t from_g = block_excl_scan_u32(chn, np + 1, tmp32);
             for (int i = tid; i < np; i += blockDim.x) {
-                ps[(size_t)i * MAX_RANKS + g] = displ + chn[i];
+                ps[(size_t)i * MAX_RANKS + g] = (displ + chn[i]) | (uint64_t)c.rank << PIECE_SRC_SHIFT;
                 pl[(size_t)i * MAX_RANKS + g] = __ldcg(mail + (size_t)(g * 2 + rel) * P + plo + i);
             }
             if (tid == 0) c.ext_counts[(1 * 2 + rel) * MAX_RANKS + g] = from_g;
@@ -355,8 +424,8 @@ __global__ void __launch_bounds__(1024) k_plan(Ctx c) {
         __syncthreads();
     }
     __syncthreads();
-    // chunk table of the local pass: chunk_base[rel][pi] = first chunk of owned partition plo+pi,
-    // piece_chunk[rel][pi][g] = first chunk of piece g inside pi
+    // chunk table of the local pass: chunk_base[rel][i] = first chunk of owned partition i,
+    // piece_chunk[rel][i][g] = first chunk of piece g inside i
     uint32_t nch[2];
     for (int rel = 0; rel < 2; ++rel) {
         const uint32_t *pl = c.piece_len + (size_t)rel * P * MAX_RANKS;
@@ -381,6 +450,8 @@ __global__ void __launch_bounds__(1024) k_plan(Ctx c) {
         if (cap_bad || !fits) set_err(c, MGJ_ECAPACITY);
         c.meta[MT_PLO] = plo;
         c.meta[MT_PHI] = phi;
+        c.meta[MT_NP] = np;
+        c.meta[MT_NBC] = nbc;
         c.meta[MT_B2] = B2;
         c.meta[MT_NCH_R] = (int)nch[0];
         c.meta[MT_NCH_S] = (int)nch[1];

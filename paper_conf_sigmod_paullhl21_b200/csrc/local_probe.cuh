@@ -67,7 +67,7 @@ struct ChunkDesc {
 
 __global__ void k_chunkmap(Ctx c, ChunkDesc *desc) {
     if (!c.meta[MT_OK]) return;
-    const int P = c.P, plo = c.meta[MT_PLO], np = c.meta[MT_PHI] - plo;
+    const int P = c.P, np = c.meta[MT_NP];
     const uint32_t nch_r = (uint32_t)c.meta[MT_NCH_R], total = nch_r + (uint32_t)c.meta[MT_NCH_S];
     const uint64_t C = (uint64_t)c.chunk_tuples;
     for (uint32_t ci = blockIdx.x * blockDim.x + threadIdx.x; ci < total; ci += gridDim.x * blockDim.x) {
@@ -124,11 +124,10 @@ __global__ void __launch_bounds__(512) k_countA(Ctx c, const ChunkDesc *cdesc) {
     const uint32_t nch_r = (uint32_t)c.meta[MT_NCH_R], total = nch_r + (uint32_t)c.meta[MT_NCH_S];
     const int tid = threadIdx.x, lane = tid & 31;
     const uint32_t nt = blockDim.x;
-    const char *recv0 = c.arena[c.rank];
     for (uint32_t ci = blockIdx.x; ci < total; ci += gridDim.x) {
         const int rel = ci < nch_r ? 0 : 1;
         const ChunkDesc d = cdesc[ci];
-        const Tup *src = reinterpret_cast<const Tup *>(recv0 + c.lay.recv[rel]) + d.start;
+        const Tup *src = reinterpret_cast<const Tup *>(c.arena[piece_src(d.start)] + c.lay.recv[rel]) + piece_off(d.start);
         if (tid < QA) cnt[tid] = 0;
         __syncthreads();
         if (QA <= 8) {
@@ -168,7 +167,7 @@ __global__ void __launch_bounds__(1024) k_planA(Ctx c) {
     __shared__ uint32_t tmp32[33];
     if (!c.meta[MT_OK] || !c.meta[MT_BA]) return;
     const int BA = c.meta[MT_BA];
-    const int L = (c.meta[MT_PHI] - c.meta[MT_PLO]) << BA;
+    const int L = c.meta[MT_NP] << BA;
     const int tid = threadIdx.x;
     uint32_t *nch = reinterpret_cast<uint32_t *>(sv + L + 1);
     const uint64_t C = (uint64_t)c.chunk_tuples;
@@ -273,7 +272,6 @@ __global__ void __launch_bounds__(LOCAL_THREADS, 1) k_local(Ctx c, const ChunkDe
     const int shift = SPLIT ? c.B1 : c.B1 + BA;  // digit = (key >> shift) & (Q - 1)
     const int Qmax = 1 << c.b2_max;
     const int BUF = C + Qmax + 2;  // slots per buffer
-    const int plo = c.meta[MT_PLO];
     Tup *const buf0 = reinterpret_cast<Tup *>(smem);
     auto buf = [&](int x) { return buf0 + (size_t)x * BUF; };
     uint32_t *const bins2 = reinterpret_cast<uint32_t *>(buf0 + (size_t)2 * BUF);  // [2][Qmax], chunk j uses j & 1
@@ -282,8 +280,12 @@ __global__ void __launch_bounds__(LOCAL_THREADS, 1) k_local(Ctx c, const ChunkDe
     const uint32_t total = nch_r + (SPLIT ? (uint32_t)c.meta[MT_NCH_S] : nch_local(c, 1));
     const uint32_t mine = total > blockIdx.x ? (total - blockIdx.x + gridDim.x - 1) / gridDim.x : 0;
     constexpr bool from_mid = MODE == LM_SECOND;
-    const char *const srcR = from_mid ? static_cast<const char *>(c.mid[0]) : c.arena[c.rank] + c.lay.recv[0];
-    const char *const srcS = from_mid ? static_cast<const char *>(c.mid[1]) : c.arena[c.rank] + c.lay.recv[1];
+    // source of a chunk: the first pass's output, or a receive buffer (this
+    // rank's, or a broadcast partition root's for its R side: piece_src)
+    auto chunk_src = [&](int rel, uint64_t start) -> const Tup * {
+        if (from_mid) return static_cast<const Tup *>(c.mid[rel]) + start;
+        return reinterpret_cast<const Tup *>(c.arena[piece_src(start)] + c.lay.recv[rel]) + piece_off(start);
+    };
     if (tid == 0) {
         mbar_init(&bar[0], 1);
         mbar_init(&bar[1], 1);
@@ -296,13 +298,14 @@ __global__ void __launch_bounds__(LOCAL_THREADS, 1) k_local(Ctx c, const ChunkDe
     auto issue = [&](uint32_t j, const ChunkDesc &d) {
         const uint32_t ci = blockIdx.x + j * gridDim.x;
         const int rel = ci < nch_r ? 0 : 1;
-        const uint64_t g0 = d.start & ~(uint64_t)(ALIGN - 1);
-        const uint64_t g1 = (d.start + d.len + ALIGN - 1) & ~(uint64_t)(ALIGN - 1);
+        const uint64_t st = from_mid ? d.start : piece_off(d.start);
+        const uint64_t g0 = st & ~(uint64_t)(ALIGN - 1);
+        const uint64_t g1 = (st + d.len + ALIGN - 1) & ~(uint64_t)(ALIGN - 1);
         const uint32_t bytes = (uint32_t)((g1 - g0) * TB);
         sdesc[j & 1] = d;
         uint64_t *b = &bar[j & 1];
         mbar_arrive_expect_tx(b, bytes);
-        if (bytes) tma_load_1d(buf(j & 1), reinterpret_cast<const Tup *>(rel ? srcS : srcR) + g0, bytes, b, pol);
+        if (bytes) tma_load_1d(buf(j & 1), chunk_src(rel, d.start) - (st - g0), bytes, b, pol);
     };
     ChunkDesc nxt{};
     constexpr int LI = 32;  // the thread that issues the chunk loads (and the chunked pass's stores)
@@ -320,7 +323,7 @@ __global__ void __launch_bounds__(LOCAL_THREADS, 1) k_local(Ctx c, const ChunkDe
         const ChunkDesc d = sdesc[X];
         const uint32_t len = d.len, skip = (uint32_t)(d.start & (ALIGN - 1));
         // partition of this chunk's tuples (a first pass's padding tuples lie in another one)
-        const uint32_t p = (uint32_t)plo + (from_mid ? d.pi >> BA : d.pi);
+        const uint32_t p = (uint32_t)c.plist[from_mid ? d.pi >> BA : d.pi];
         Tup t[VMAX];
 #pragma unroll
         for (int v = 0; v < VMAX; ++v) {
@@ -586,7 +589,7 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
     // and R's bit 0 (k_local), so neither can equal any key of the other side
     // and S padding is probed harmlessly; only P < 4 needs the skip bitmap
     const bool SBITS = Layout<K>::ALIGN == 2 && c.P < 4;
-    const int plo = c.meta[MT_PLO], BAp = c.meta[MT_BA];
+    const int BAp = c.meta[MT_BA];
     // packed table (B1 + B2 >= 16, so khi = key >> (B1 + B2) fits the key's
     // width minus 16 bits): the build overwrites each R slot's key with
     // (khi << 16 | next), so a chain step is one shared load of the slot
@@ -711,7 +714,7 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
                 }
             }
             if (lane == 0 && rel0 == 0) {
-                stage_p[s] = (uint32_t)(plo + (BAp ? x.it.pi >> BAp : x.it.pi));
+                stage_p[s] = (uint32_t)c.plist[BAp ? x.it.pi >> BAp : x.it.pi];
                 stage_soff[s] = x.soff;
             }
             __syncwarp();

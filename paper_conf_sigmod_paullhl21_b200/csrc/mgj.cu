@@ -41,8 +41,9 @@ int ceil_log2(uint64_t x) {
 mgj_status normalize(const mgj_config *in, Norm *o) {
     if (!in) return MGJ_EINVAL;
     mgj_config c = *in;
-    for (int i = 0; i < 6; ++i)
+    for (int i = 0; i < 5; ++i)
         if (c.reserved[i]) return MGJ_EINVAL;
+    if (c.skew_bcast < -1 || c.skew_bcast > 1) return MGJ_EINVAL;
     if (c.local_split_bits < -1 || c.local_split_bits > MAX_BA) return MGJ_EINVAL;
     if (c.shuffle_mode != MGJ_SHUFFLE_P2P && c.shuffle_mode != MGJ_SHUFFLE_EXTERNAL) return MGJ_EINVAL;
     if (c.world_size < 1 || c.world_size > MAX_RANKS || c.rank < 0 || c.rank >= c.world_size) return MGJ_EINVAL;
@@ -162,7 +163,7 @@ void *dalloc(mgj_plan_s *h, size_t bytes, mgj_status *st) {
 size_t hist_smem(const Norm &n) {
     return (size_t)HIST_NB * scat_geom(n.P, n.c.key_bytes).T * n.c.key_bytes + (size_t)n.P * 8;
 }
-size_t plan_smem(const Norm &n) { return (size_t)n.P * 5 * 8 + (size_t)n.P * 4 + (size_t)(n.P + 1) * 4; }
+size_t plan_smem(const Norm &n) { return (size_t)n.P * 5 * 8 + (size_t)n.P * 4 + (size_t)(n.P + 1) * 4 + (size_t)n.P; }
 size_t scatter_smem(const Norm &n) { return scat_smem_bytes(n.P, n.c.key_bytes); }
 size_t planA_smem(const Norm &n) { return ((size_t)local2_vcap(n.P) + 1) * 12; }
 size_t local_smem(const Norm &n) { return local_smem_bytes(n.chunk_tuples, 1 << n.b2_max, n.tuple_bytes); }
@@ -350,6 +351,9 @@ mgj_status mgj_plan(const mgj_config *cfg, const mgj_peers *peers, mgj_handle *o
     c.sub_hist = static_cast<uint16_t *>(dalloc(h, 2ull * c.G * c.sub_ns * P * 2, &st));
     h->cdesc = static_cast<ChunkDesc *>(dalloc(h, 2 * n.max_chunks * sizeof(ChunkDesc), &st));
     c.owner = static_cast<int32_t *>(dalloc(h, P * 4, &st));
+    c.bcast = static_cast<uint8_t *>(dalloc(h, P, &st));
+    c.plist = static_cast<int32_t *>(dalloc(h, P * 4, &st));
+    c.bcast_cfg = n.c.skew_bcast;
     c.send_off = static_cast<uint64_t *>(dalloc(h, 2ull * P * 8, &st));
     c.seg_start = static_cast<uint64_t *>(dalloc(h, 2ull * P * 8, &st));
     c.seg_len = static_cast<uint64_t *>(dalloc(h, 2ull * P * 8, &st));
@@ -558,34 +562,44 @@ void mgj_destroy(mgj_handle h) {
 }
 
 mgj_status mgj_plan_host(int32_t world_size, int32_t rank, int32_t bits, const uint32_t *hist, int32_t *owner,
-                         uint64_t *send_off, uint64_t *recv_size) {
+                         uint64_t *send_off, uint64_t *recv_size, int32_t skew_bcast, uint8_t *bcast) {
     if (world_size < 1 || world_size > MAX_RANKS || rank < 0 || rank >= world_size || bits < 1 || bits > MAX_B1 ||
-        !hist || !owner || !send_off || !recv_size)
+        !hist || !owner || !send_off || !recv_size || skew_bcast < -1 || skew_bcast > 1)
         return MGJ_EINVAL;
     const int P = 1 << bits, N = world_size;
     auto H = [&](int g, int rel, int p) -> uint64_t { return hist[((size_t)g * 2 + rel) * P + p]; };
     uint64_t *tot = new (std::nothrow) uint64_t[2 * (size_t)P];
-    uint64_t *pre = new (std::nothrow) uint64_t[2 * (size_t)P];
-    if (!tot || !pre) {
+    uint64_t *pre = new (std::nothrow) uint64_t[2 * (size_t)P];  // R prefix; S prefix over non-broadcast partitions
+    uint8_t *bc = new (std::nothrow) uint8_t[(size_t)P];
+    if (!tot || !pre || !bc) {
         delete[] tot;
         delete[] pre;
+        delete[] bc;
         return MGJ_ENOMEM;
     }
-    uint64_t total = 0, run[2] = {0, 0};
+    uint64_t s_total = 0;
     for (int p = 0; p < P; ++p)
         for (int rel = 0; rel < 2; ++rel) {
             uint64_t t = 0;
             for (int g = 0; g < N; ++g) t += H(g, rel, p);
             tot[rel * P + p] = t;
-            pre[rel * P + p] = run[rel];
-            run[rel] += t;
-            total += t;
+            if (rel) s_total += t;
         }
+    uint64_t total = 0, run[2] = {0, 0};
+    for (int p = 0; p < P; ++p) {
+        bc[p] = bcast_of(tot[p], tot[P + p], s_total, N, P, skew_bcast);
+        if (bcast) bcast[p] = bc[p];
+        total += owner_weight(tot[p], tot[P + p], bc[p], N);
+        pre[p] = run[0];
+        run[0] += tot[p];
+        pre[P + p] = run[1];
+        run[1] += bc[p] ? 0 : tot[P + p];
+    }
     uint64_t cum = 0;
     int first[MAX_RANKS], endp[MAX_RANKS];
     for (int d = 0; d < MAX_RANKS; ++d) first[d] = endp[d] = P;
     for (int p = 0; p < P; ++p) {
-        const uint64_t T = tot[p] + tot[P + p];
+        const uint64_t T = owner_weight(tot[p], tot[P + p], bc[p], N);
         owner[p] = owner_of(cum, T, total, N, p, P);
         cum += T;
     }
@@ -593,20 +607,33 @@ mgj_status mgj_plan_host(int32_t world_size, int32_t rank, int32_t bits, const u
         if (p == 0 || owner[p - 1] != owner[p]) first[owner[p]] = p;
         if (p == P - 1 || owner[p + 1] != owner[p]) endp[owner[p]] = p + 1;
     }
-    for (int rel = 0; rel < 2; ++rel) {
-        for (int p = 0; p < P; ++p) {
-            uint64_t mine = 0;
-            for (int g = 0; g < rank; ++g) mine += H(g, rel, p);
-            send_off[rel * P + p] = pre[rel * P + p] - pre[rel * P + first[owner[p]]] + mine;
-        }
-        for (int d = 0; d < N; ++d) {
-            uint64_t sz = 0;
-            if (first[d] < P) sz = pre[rel * P + endp[d] - 1] + tot[rel * P + endp[d] - 1] - pre[rel * P + first[d]];
-            recv_size[rel * N + d] = sz;
+    auto range_size = [&](int rel, int d) -> uint64_t {  // non-broadcast part of d's receive layout
+        if (first[d] >= P) return 0;
+        const int l = endp[d] - 1;
+        return pre[rel * P + l] + (rel && bc[l] ? 0 : tot[rel * P + l]) - pre[rel * P + first[d]];
+    };
+    uint64_t own_bc = 0;  // this rank's S tuples of broadcast partitions before p
+    for (int p = 0; p < P; ++p) {
+        uint64_t m0 = 0, m1 = 0;
+        for (int g = 0; g < rank; ++g) m0 += H(g, 0, p), m1 += H(g, 1, p);
+        send_off[p] = pre[p] - pre[first[owner[p]]] + m0;
+        if (bc[p]) {
+            send_off[P + p] = range_size(1, rank) + own_bc;
+            own_bc += H(rank, 1, p);
+        } else {
+            send_off[P + p] = pre[P + p] - pre[P + first[owner[p]]] + m1;
         }
     }
+    for (int rel = 0; rel < 2; ++rel)
+        for (int d = 0; d < N; ++d) {
+            uint64_t sz = range_size(rel, d);
+            if (rel)
+                for (int p = 0; p < P; ++p) sz += bc[p] ? H(d, 1, p) : 0;
+            recv_size[rel * N + d] = sz;
+        }
     delete[] tot;
     delete[] pre;
+    delete[] bc;
     return MGJ_OK;
 }
 
@@ -653,6 +680,8 @@ mgj_status mgj_debug_copy(mgj_handle h, int32_t what, void *dst, uint64_t bytes,
         case MGJ_DBG_RANK_HIST: src = c.rank_hist; size = 2ull * P * 4; break;
         case MGJ_DBG_MAIL_HIST: src = h->arena[c.rank] + n.lay.mail; size = (uint64_t)c.world * 2 * P * 4; break;
         case MGJ_DBG_OWNER: src = c.owner; size = (uint64_t)P * 4; break;
+        case MGJ_DBG_BCAST: src = c.bcast; size = (uint64_t)P; break;
+        case MGJ_DBG_PLIST: src = c.plist; size = (uint64_t)std::max(meta[MT_NP], 0) * 4; break;
         case MGJ_DBG_SEND_OFF: src = c.send_off; size = 2ull * P * 8; break;
         case MGJ_DBG_RECV_SIZE: src = c.recv_size; size = sizeof(rs); break;
         case MGJ_DBG_RECV_R: src = h->arena[c.rank] + n.lay.recv[0]; size = rs[c.rank] * n.tuple_bytes; break;

@@ -271,7 +271,10 @@ __global__ void __launch_bounds__(NT, NT <= 512 ? 2 : 1) k_scatter(Ctx c) {
             const int p = tid * PPT + k;
             cc[k] = hd[k] = 0;
             if (p < P) {
-                const ull a = (ull)(c.arena[c.owner[p]] + c.lay.recv[rel]) + (so[p] + tb[p]) * (uint64_t)TB;
+                // destination: the owner, or this rank itself for the S side of a
+                // selectively broadcast partition (a2, NEXT-2)
+                const int dst = (rel && c.bcast[p]) ? c.rank : c.owner[p];
+                const ull a = (ull)(c.arena[dst] + c.lay.recv[rel]) + (so[p] + tb[p]) * (uint64_t)TB;
                 const uint32_t h = SG > 1 ? (uint32_t)((a & (GB - 1)) / TB) : 0u;
                 base[k] = a - (ull)h * TB;
                 cc[k] = hd[k] = h;

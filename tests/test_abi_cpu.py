@@ -75,28 +75,35 @@ def test_arena_layout_size(mgj):
     assert 2 * 8 * (1 << 20) <= nb <= 2 * 8 * (1 << 20) + (1 << 20)
 
 
-def check_plan_invariants(mgj, hist, bits):
+def check_plan_invariants(mgj, hist, bits, skew_bcast=0):
+    """Every rank computes the same plan; for each destination d and relation, the
+    (source rank, partition) ranges the plan sends to d tile [0, recv_size[d]) exactly.
+    A selectively broadcast partition (NEXT-2) sends R to its owner (the root) and
+    keeps each rank's S at that rank."""
     N = hist.shape[0]
     P = 1 << bits
-    plans = [mgj.plan_host(N, g, bits, hist) for g in range(N)]
-    owner = plans[0][0]
-    recv = plans[0][2]
-    for o, _, rs in plans:  # every rank computes the same assignment
-        assert np.array_equal(o, owner) and np.array_equal(rs, recv)
+    plans = [mgj.plan_host(N, g, bits, hist, skew_bcast=skew_bcast, with_bcast=True) for g in range(N)]
+    owner, recv, bc = plans[0][0], plans[0][2], plans[0][3]
+    for o, _, rs, b in plans:  # every rank computes the same assignment
+        assert np.array_equal(o, owner) and np.array_equal(rs, recv) and np.array_equal(b, bc)
     assert np.all(np.diff(owner) >= 0) and owner.min() >= 0 and owner.max() < N
+    if N == 1 or skew_bcast < 0:
+        assert not bc.any()
     tot = hist.astype(np.uint64).sum(axis=0)  # [2][P]
     for rel in range(2):
         assert int(recv[rel].sum()) == int(tot[rel].sum())
         for d in range(N):
-            # the (rank, p) ranges of owner d tile [0, recv_size[d]) exactly
             cover = np.zeros(int(recv[rel, d]), np.int32)
             for g in range(N):
                 so = plans[g][1][rel]
-                for p in np.nonzero(owner == d)[0]:
+                for p in range(P):
+                    dest = g if (rel == 1 and bc[p]) else owner[p]
+                    if dest != d:
+                        continue
                     c = int(hist[g, rel, p])
                     cover[int(so[p]):int(so[p]) + c] += 1
             assert np.all(cover == 1)
-    return owner, recv
+    return owner, recv, bc
 
 
 @pytest.mark.parametrize("N", [1, 2, 3, 5, 8])
@@ -106,12 +113,19 @@ def test_plan_host_invariants_random(mgj, N):
     hist = rng.integers(0, 50, size=(N, 2, 1 << bits)).astype(np.uint32)
     hist[:, :, 5] = 0  # empty partitions
     check_plan_invariants(mgj, hist, bits)
+    check_plan_invariants(mgj, hist, bits, skew_bcast=-1)
+    hist[:, 1, 7] *= 40  # heavy S partitions: broadcast candidates
+    hist[:, 1, 40] = 5000
+    _, _, bc = check_plan_invariants(mgj, hist, bits)
+    assert bc[40] == (N > 1)
+    check_plan_invariants(mgj, hist, bits, skew_bcast=1)
 
 
 def test_plan_host_uniform_identity_ranges(mgj):
     N, bits = 8, 10
     hist = np.full((N, 2, 1 << bits), 64, np.uint32)
-    owner, recv = check_plan_invariants(mgj, hist, bits)
+    owner, recv, bc = check_plan_invariants(mgj, hist, bits)
+    assert not bc.any()  # uniform data never broadcasts
     assert np.array_equal(owner, np.arange(1 << bits) * N >> bits)
     assert np.all(recv == 64 * N * (1 << bits) // N)
 
@@ -121,13 +135,36 @@ def test_plan_host_skew_balances(mgj):
     N, bits = 4, 8
     hist = np.full((N, 2, 1 << bits), 10, np.uint32)
     hist[:, 1, 200] = 5000
-    owner, recv = check_plan_invariants(mgj, hist, bits)
+    owner, recv, _ = check_plan_invariants(mgj, hist, bits, skew_bcast=-1)
     assert owner[200] in (2, 3)
     # partitions below the heavy one spread over the other owners
     assert len(set(owner[:200].tolist())) >= 2
 
 
+def test_plan_host_selective_broadcast(mgj):
+    """NEXT-2 (P:418-444 Track-Join benefit test, P:386-395 heavy hitters): a heavy S
+    partition with small R is broadcast: R to its root only (read by every rank), each
+    rank keeps its own S; the heavy partition no longer loads one owner."""
+    N, bits = 4, 8
+    P = 1 << bits
+    hist = np.full((N, 2, P), 10, np.uint32)
+    hist[:, 1, 200] = 5000
+    owner, recv, bc = check_plan_invariants(mgj, hist, bits)
+    assert bc.sum() == 1 and bc[200]
+    # S receive sizes: every rank holds its own 5000 S tuples of partition 200
+    s_range = [sum(10 * N for p in range(P) if owner[p] == d and not bc[p]) for d in range(N)]
+    assert [int(x) for x in recv[1]] == [s_range[d] + 5000 for d in range(N)]
+    # the owner ranges are balanced on R + S/N for the broadcast partition
+    w = hist.astype(np.int64).sum(axis=0)
+    load = [int(w[0][owner == d].sum()) + int(w[1][(owner == d) & (bc == 0)].sum()) for d in range(N)]
+    assert max(load) - min(load) <= 2 * 20 * N + 5000
+    # auto mode leaves the same partition alone when R is not small: (N-1)|R_p| >= |S_p|
+    hist[:, 0, 200] = 2000
+    _, _, bc2 = check_plan_invariants(mgj, hist, bits)
+    assert not bc2.any()
+
+
 def test_plan_host_all_empty(mgj):
     hist = np.zeros((4, 2, 1 << 5), np.uint32)
-    owner, recv = check_plan_invariants(mgj, hist, 5)
+    owner, recv, _ = check_plan_invariants(mgj, hist, 5)
     assert np.array_equal(owner, np.arange(32) * 4 // 32)

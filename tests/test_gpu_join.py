@@ -396,6 +396,107 @@ def test_virtual_ranks_zipf_skew(mgj):
         j.close()
 
 
+class ArrayWorkload:
+    """Fixed arrays split into contiguous rank shards (reading C12), for run_virtual."""
+
+    def __init__(self, rk, ra, sk, sb):
+        self.a = dict(r_keys=rk, r_pays=ra, s_keys=sk, s_pays=sb)
+        self.n_r, self.n_s = rk.size, sk.size
+        self.key_bytes = 8 if rk.dtype == np.uint64 else 4
+
+    def rank_inputs(self, rank=0, world=1):
+        out = {}
+        for k, v in self.a.items():
+            n = v.size
+            out[k] = v[n * rank // world: n * (rank + 1) // world].copy()
+        return out
+
+
+def check_bcast_virtual(mgj, w, N, skew, materialize=True, expect_bc=True, **kw):
+    """NEXT-2 selective broadcast on N virtual ranks: result == oracle (count, checksum,
+    sorted triples), device plan == host plan (owner, offsets, broadcast flags), each
+    rank's received S holds its owned partitions and its own share of every broadcast
+    partition, and every broadcast partition's R side is built by every rank."""
+    joins, res, _ = run_virtual(mgj, w, N, materialize=materialize, skew_bcast=skew, **kw)
+    d = w.rank_inputs()
+    ref = oracle.join(d["r_keys"], d["r_pays"], d["s_keys"], d["s_pays"], materialize=materialize)
+    for r in res:
+        assert r["status"] == 0
+        assert (r["match_count"], r["checksum"]) == (ref["count"], ref["checksum"])
+    assert sum(r["local_count"] for r in res) == ref["count"]
+    if materialize:
+        trip = [j.materialized(r) for j, r in zip(joins, res)]
+        k, a, b = sort_trip(*(np.concatenate([t[i] for t in trip]) for i in range(3)))
+        np.testing.assert_array_equal(k, ref["key"])
+        np.testing.assert_array_equal(a, ref["pay_r"])
+        np.testing.assert_array_equal(b, ref["pay_s"])
+    B1 = res[0]["radix_bits_global"]
+    P = 1 << B1
+    mail = joins[0].debug("MAIL_HIST", np.uint32).reshape(N, 2, P)
+    kdt = np.uint32 if w.key_bytes == 4 else np.uint64
+    nbc = None
+    for g, j in enumerate(joins):
+        owner, send_off, recv_size, bc = mgj.plan_host(N, g, B1, mail, skew_bcast=skew, with_bcast=True)
+        np.testing.assert_array_equal(j.debug("OWNER", np.int32), owner)
+        np.testing.assert_array_equal(j.debug("BCAST", np.uint8), bc)
+        np.testing.assert_array_equal(j.debug("SEND_OFF", np.uint64).reshape(2, P), send_off)
+        assert res[g]["recv_r"] == recv_size[0, g] and res[g]["recv_s"] == recv_size[1, g]
+        meta = j.debug("META", np.int32)
+        nbc = int(bc.sum())
+        assert meta[14] == nbc
+        plist = j.debug("PLIST", np.int32)
+        assert sorted(plist.tolist()) == sorted(set(np.nonzero(owner == g)[0].tolist()) | set(np.nonzero(bc)[0].tolist()))
+        recv_s = j.debug("RECV_S", kdt).reshape(-1, 2)
+        ps = (recv_s[:, 0] & (P - 1)).astype(np.int64)
+        assert np.all((owner[ps] == g) | (bc[ps] != 0))
+        # the S of a broadcast partition received by g is exactly g's own shard of it
+        mine = w.rank_inputs(g, N)
+        for p in np.nonzero(bc)[0][:8]:
+            own = np.sort(mine["s_keys"][(mine["s_keys"] & (P - 1)) == p])
+            np.testing.assert_array_equal(np.sort(recv_s[ps == p, 0]), own)
+    if expect_bc:
+        assert nbc > 0
+    for j in joins:
+        j.close()
+    return nbc
+
+
+@pytest.mark.parametrize("N,skew", [(2, 0), (4, 0), (8, 0), (4, 1), (8, 1), (4, -1)])
+def test_virtual_ranks_bcast_zipf(mgj, N, skew):
+    """Zipf S (z = 1, |R|:|S| = 1:4, half the S rows match): heavy partitions broadcast."""
+    w = datagen.Workload("zipf", 1 << 16, 1 << 18, 1.0)
+    check_bcast_virtual(mgj, w, N, skew, materialize=True, expect_bc=skew >= 0, radix_bits_global=8)
+
+
+@pytest.mark.parametrize("N,ba", [(4, 2), (8, 1)])
+def test_virtual_ranks_bcast_two_level(mgj, N, ba):
+    """Broadcast partitions' remote R pieces through the first (histogram) local pass."""
+    w = datagen.Workload("zipf", 1 << 16, 1 << 18, 1.0)
+    check_bcast_virtual(mgj, w, N, 1, materialize=False, radix_bits_global=6, local_split_bits=ba)
+
+
+def test_virtual_ranks_bcast_duplicates(mgj):
+    """Duplicate R keys inside broadcast partitions (bag semantics, C2), 4-byte keys."""
+    rng = np.random.default_rng(7)
+    rk = rng.integers(0, 3000, 6000, dtype=np.uint64).astype(np.uint32)
+    sk = np.concatenate([rng.integers(0, 3000, 20000, dtype=np.uint64),
+                         np.full(30000, 7 * 64 + 5, np.uint64)]).astype(np.uint32)
+    rng.shuffle(sk)
+    w = ArrayWorkload(rk, np.arange(rk.size, dtype=np.uint32), sk, np.arange(sk.size, dtype=np.uint32))
+    check_bcast_virtual(mgj, w, 4, 0, materialize=True, radix_bits_global=6)
+
+
+def test_virtual_ranks_bcast_wide(mgj):
+    """8-byte keys and payloads with broadcast partitions (forced)."""
+    rng = np.random.default_rng(11)
+    dom = rng.integers(0, 1 << 63, 4000, dtype=np.uint64) | np.uint64(1 << 63)
+    rk = dom[rng.integers(0, dom.size, 5000)]
+    sk = dom[rng.integers(0, dom.size, 60000)]
+    w = ArrayWorkload(rk, (np.arange(rk.size) + (1 << 40)).astype(np.uint64), sk,
+                      (np.arange(sk.size) + (1 << 41)).astype(np.uint64))
+    check_bcast_virtual(mgj, w, 4, 1, materialize=True, radix_bits_global=5)
+
+
 def test_virtual_ranks_wide(mgj):
     w = datagen.Workload("wide", 1 << 17, 1 << 17)
     joins, res, _ = run_virtual(mgj, w, 2, materialize=True)

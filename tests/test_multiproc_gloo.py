@@ -26,7 +26,7 @@ def _free_port():
     return p
 
 
-def _worker(rank, world, port, bits, kind, q):
+def _worker(rank, world, port, bits, kind, skew, q):
     import sys
     sys.path.insert(0, ROOT)
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
@@ -42,11 +42,14 @@ def _worker(rank, world, port, bits, kind, q):
         allh = [torch.zeros(2, P, dtype=torch.int64) for _ in range(world)]
         dist.all_gather(allh, torch.from_numpy(hist))
         H = np.stack([h.numpy() for h in allh]).astype(np.uint32)
-        owner, send_off, recv_size = mgj.plan_host(world, rank, bits, H)
+        owner, send_off, recv_size, bc = mgj.plan_host(world, rank, bits, H, skew_bcast=skew, with_bcast=True)
+        if skew < 0:
+            assert not bc.any()
         out = {}
         for rel, (k, p) in enumerate(((d["r_keys"], d["r_pays"]), (d["s_keys"], d["s_pays"]))):
             part = (k & (P - 1)).astype(np.int64)
-            dest = owner[part]
+            # a selectively broadcast partition (NEXT-2) keeps its S on this rank
+            dest = np.where(bc[part] != 0, rank, owner[part]) if rel == 1 else owner[part]
             # slot of each tuple inside its owner's receive buffer: send_off[p] + rank inside (rank, p)
             order = np.argsort(part, kind="stable")
             rank_in_p = np.empty(k.size, np.int64)
@@ -64,10 +67,16 @@ def _worker(rank, world, port, bits, kind, q):
             assert recv.shape[0] == int(recv_size[rel][rank])
             cover = np.bincount(recv[:, 2], minlength=recv.shape[0])
             assert cover.size == recv.shape[0] and np.all(cover == 1), "slots not exactly tiled"
-            assert np.all(owner[(recv[:, 0] & (P - 1))] == rank)
+            rp = recv[:, 0] & (P - 1)
+            assert np.all((owner[rp] == rank) if rel == 0 else ((owner[rp] == rank) | (bc[rp] != 0)))
             buf = np.empty((recv.shape[0], 2), np.int64)
             buf[recv[:, 2]] = recv[:, :2]
             out[rel] = buf
+        # the R side of broadcast partitions is read by every rank from its root (pull broadcast)
+        mine_bc = out[0][bc[out[0][:, 0] & (P - 1)] != 0]
+        allbc = [None] * world
+        dist.all_gather_object(allbc, mine_bc)
+        out[0] = np.concatenate([out[0]] + [allbc[g] for g in range(world) if g != rank])
         r = oracle.join(out[0][:, 0].astype(np.uint32), out[0][:, 1].astype(np.uint32),
                         out[1][:, 0].astype(np.uint32), out[1][:, 1].astype(np.uint32))
         t = torch.tensor([r["count"], r["checksum"] & ((1 << 63) - 1), r["checksum"] >> 63], dtype=torch.int64)
@@ -78,23 +87,29 @@ def _worker(rank, world, port, bits, kind, q):
             chk = sum(int(x[1]) + (int(x[2]) << 63) for x in allr) & M64
             full = w.rank_inputs(0, 1)
             g = oracle.join(full["r_keys"], full["r_pays"], full["s_keys"], full["s_pays"])
-            q.put((cnt, chk, g["count"], g["checksum"]))
+            q.put((cnt, chk, g["count"], g["checksum"], int(bc.sum())))
     finally:
         dist.destroy_process_group()
 
 
-@pytest.mark.parametrize("world,bits,kind", [(2, 8, "unique"), (4, 6, "unique"), (2, 7, "zipf")])
-def test_gloo_partitioned_join(world, bits, kind):
+@pytest.mark.parametrize("world,bits,kind,skew", [(2, 8, "unique", 0), (4, 6, "unique", 0), (2, 7, "zipf", -1),
+                                                  (2, 7, "zipf", 0), (4, 7, "zipf", 1)])
+def test_gloo_partitioned_join(world, bits, kind, skew):
+    """skew: mgj_config.skew_bcast (selective broadcast of heavy S partitions, NEXT-2)."""
     import __graft_entry__
     __graft_entry__.build()
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    procs = [ctx.Process(target=_worker, args=(r, world, port, bits, kind, q)) for r in range(world)]
+    procs = [ctx.Process(target=_worker, args=(r, world, port, bits, kind, skew, q)) for r in range(world)]
     for p in procs:
         p.start()
     for p in procs:
         p.join(timeout=300)
     assert all(p.exitcode == 0 for p in procs)
-    cnt, chk, gc, gk = q.get(timeout=10)
+    cnt, chk, gc, gk, nbc = q.get(timeout=10)
     assert (cnt, chk) == (gc, gk)
+    if kind == "unique" or skew < 0:
+        assert nbc == 0
+    else:
+        assert nbc > 0  # Zipf S with |R|:|S| = 1:2 has partitions worth broadcasting

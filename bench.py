@@ -50,6 +50,8 @@ def parse():
     ap.add_argument("--local-split-bits", type=int, default=0, help="a4 first pass: 0 auto, -1 never, k forced")
     ap.add_argument("--cpu-sample-log2", type=int, default=28,
                     help="oracle sample: 2^k R + 2^k S unique tuples (cpu_baseline / --impl reference)")
+    ap.add_argument("--skew-bcast", type=int, default=0, choices=[-1, 0, 1],
+                    help="a2 selective broadcast of heavy S partitions (N>1): 0 auto, -1 never, 1 forced")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=3)
@@ -249,7 +251,8 @@ def main():
                           radix_bits_local=a.radix_bits_local, local_split_bits=a.local_split_bits,
                           recv_capacity_r=(n_r if world > 1 and a.workload == "zipf" else 0),
                           recv_capacity_s=(n_s // 2 if world > 1 and a.workload == "zipf" else 0),
-                          shuffle_mode=(mgj.SHUFFLE_EXTERNAL if a.shuffle == "nccl" else mgj.SHUFFLE_P2P))
+                          shuffle_mode=(mgj.SHUFFLE_EXTERNAL if a.shuffle == "nccl" else mgj.SHUFFLE_P2P),
+                          skew_bcast=a.skew_bcast)
     arena = None
     if distributed:
         import torch.distributed._symmetric_memory as symm_mem
@@ -416,7 +419,8 @@ def main():
                        "l2": "inputs (8 GiB/GPU) larger than L2; no flush", "parallelism": f"dp{world}",
                        "shuffle": ("in-kernel peer stores (symmetric memory)" if a.shuffle == "p2p"
                                    else "NCCL all_to_all_single baseline (host sync per step for split sizes)"),
-                       "global_batch": tuples_job, "seeds": {"R": "0x5EED0052", "S": "0x5EED0053"}},
+                       "global_batch": tuples_job, "seeds": {"R": "0x5EED0052", "S": "0x5EED0053"},
+                       "skew_bcast": a.skew_bcast},
             "correct": bool(expect_ok) and res["status"] == 0,
             "match_count": res["match_count"], "checksum": hex(res["checksum"]),
             "gpu_cycles_per_tuple": {"sm_cycles_per_tuple": cyc * nsm, "gpu_cycles_per_tuple": cyc,

@@ -28,20 +28,30 @@ one({"r_keys": rng.integers(0, 300, 20000, dtype=np.uint64).astype(np.uint32), "
      "s_keys": rng.integers(0, 300, 30000, dtype=np.uint64).astype(np.uint32), "s_pays": np.arange(30000, dtype=np.uint32)},
     materialize=False, radix_bits_global=4)
 one(datagen.Workload("wide", 1 << 14, 1 << 14).rank_inputs(), materialize=True)
-# two virtual ranks
-w = datagen.Workload("unique", 1 << 15, 1 << 15)
-parts = [w.rank_inputs(g, 2) for g in range(2)]
-cfgs = [mgj.make_config(rank=g, world_size=2, r_capacity=1 << 14, s_capacity=1 << 14, recv_capacity_r=1 << 15,
-                        recv_capacity_s=1 << 15) for g in range(2)]
-nb = mgj.arena_bytes(cfgs[0])
-arenas = [torch.zeros(nb, dtype=torch.uint8, device="cuda") for _ in range(2)]
-js = [mgj.Join(cfgs[g], [a.data_ptr() for a in arenas], nb) for g in range(2)]
-ts = [[dev(p[k]) for k in ("r_keys", "r_pays", "s_keys", "s_pays")] for p in parts]
-for g in range(2): js[g].partition(*ts[g])
-for g in range(2): js[g].shuffle()
-for g in range(2): js[g].join()
-res = [js[g].result() for g in range(2)]
-full = w.rank_inputs()
-ref = oracle.join(full["r_keys"], full["r_pays"], full["s_keys"], full["s_pays"])
-assert (res[0]["match_count"], res[0]["checksum"]) == (ref["count"], ref["checksum"])
+
+
+def virtual(w, N, **kw):
+    """N virtual ranks on one GPU (plain device arenas), every phase for all ranks in turn."""
+    parts = [w.rank_inputs(g, N) for g in range(N)]
+    cfgs = [mgj.make_config(rank=g, world_size=N, r_capacity=max(p["r_keys"].size for p in parts),
+                            s_capacity=max(p["s_keys"].size for p in parts), recv_capacity_r=w.n_r,
+                            recv_capacity_s=w.n_s, **kw) for g in range(N)]
+    nb = mgj.arena_bytes(cfgs[0])
+    arenas = [torch.zeros(nb, dtype=torch.uint8, device="cuda") for _ in range(N)]
+    js = [mgj.Join(cfgs[g], [a.data_ptr() for a in arenas], nb) for g in range(N)]
+    ts = [[dev(p[k]) for k in ("r_keys", "r_pays", "s_keys", "s_pays")] for p in parts]
+    for g in range(N): js[g].partition(*ts[g])
+    for g in range(N): js[g].shuffle()
+    for g in range(N): js[g].join()
+    res = [js[g].result() for g in range(N)]
+    full = w.rank_inputs()
+    ref = oracle.join(full["r_keys"], full["r_pays"], full["s_keys"], full["s_pays"])
+    assert (res[0]["match_count"], res[0]["checksum"]) == (ref["count"], ref["checksum"])
+    for j in js: j.close()
+
+
+# two virtual ranks; four with selectively broadcast partitions (NEXT-2), also through the first local pass
+virtual(datagen.Workload("unique", 1 << 15, 1 << 15), 2)
+virtual(datagen.Workload("zipf", 1 << 13, 1 << 15, 1.0), 4, skew_bcast=1, radix_bits_global=6)
+virtual(datagen.Workload("zipf", 1 << 13, 1 << 15, 1.0), 4, skew_bcast=1, radix_bits_global=6, local_split_bits=2)
 print("sanitize workload ok")

@@ -198,7 +198,7 @@ const char *mgj_strerror(mgj_status s);
 mgj_status mgj_plan_host(int32_t world_size, int32_t rank, int32_t bits,
                          const uint32_t *hist, int32_t *owner,
                          uint64_t *send_off, uint64_t *recv_size,
-                         int32_t skew_bcast, uint8_t *bcast);
+                         int32_t skew_bcast, uint8_t *bcast, uint8_t *skip);
 
 #ifdef __cplusplus
 }

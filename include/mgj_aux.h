@@ -56,7 +56,8 @@ typedef enum {
     MGJ_DBG_MID_S = 19,
     MGJ_DBG_VSTART = 20,     /* u64[2][L+1] sub-partition starts (slots) in MID_R / MID_S */
     MGJ_DBG_BCAST = 21,      /* u8[P]                selective-broadcast flag of each global partition (a2) */
-    MGJ_DBG_PLIST = 22       /* i32[np]              owned partitions: the range, then broadcast ones outside it */
+    MGJ_DBG_PLIST = 22,      /* i32[np]              owned partitions: the range, then broadcast ones outside it */
+    MGJ_DBG_SKIP = 23        /* u8[P]                partition has no R or no S tuple anywhere: not shuffled (a2) */
 } mgj_debug_what;
 
 mgj_status mgj_debug_copy(mgj_handle h, int32_t what, void *dst, uint64_t bytes, uint64_t *size_out);

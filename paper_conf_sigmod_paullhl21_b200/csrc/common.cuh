@@ -110,6 +110,7 @@ struct Ctx {
     int32_t *meta;                // [MT_COUNT]
     int32_t *owner;               // [P] range owner (a broadcast partition's root)
     uint8_t *bcast;               // [P] selective broadcast flags (a2)
+    uint8_t *pskip;               // [P] partitions with an empty side: never shuffled (histogram as a Bloom filter)
     int32_t *plist;               // [P] owned partitions: the range, then broadcast partitions outside it
     int32_t bcast_cfg;            // mgj_config.skew_bcast
     uint64_t *send_off;           // [2][P]

@@ -197,6 +197,11 @@ __host__ __device__ inline bool bcast_of(uint64_t r, uint64_t s, uint64_t s_tota
     return cfg > 0 || s * (uint64_t)P >= 2 * s_total;
 }
 
+// The histogram as a simplified Bloom filter: a partition with no
+// R or no S tuple anywhere cannot produce a match, so none of its tuples is
+// shuffled, partitioned or probed.  P2P shuffle only.
+__host__ __device__ inline bool skip_of(uint64_t r, uint64_t s) { return (r == 0) != (s == 0); }
+
 // Weight of p in the owner ranges: a broadcast partition's S stays spread
 // over the ranks, its owner (the root, which receives R_p) gets R_p + S_p/N.
 __host__ __device__ inline uint64_t owner_weight(uint64_t r, uint64_t s, bool bc, int N) {
@@ -271,6 +276,9 @@ __global__ void __launch_bounds__(1024) k_plan(Ctx c) {
         for (int p = tid; p < P; p += blockDim.x) {
             uint64_t t0 = 0, t1 = 0;
             for (int g = 0; g < N; ++g) t0 += H(g, 0, p), t1 += H(g, 1, p);
+            const bool sk = !c.ext && skip_of(t0, t1);
+            c.pskip[p] = sk;
+            if (sk) t0 = t1 = 0;  // a skipped partition is absent from every layout
             tot0[p] = pre0[p] = t0;
             tot1[p] = t1;
             st += t1;
@@ -286,7 +294,7 @@ __global__ void __launch_bounds__(1024) k_plan(Ctx c) {
         c.bcast[p] = bc;
         pre1[p] = bc ? 0 : tot1[p];  // S layout: broadcast partitions are not in the owner's range part
         cum[p] = owner_weight(tot0[p], tot1[p], bc, N);
-        chn[p] = bc ? H(c.rank, 1, p) : 0u;  // this rank's own S of broadcast partitions
+        chn[p] = bc ? H(c.rank, 1, p) : 0u;  // this rank's own S of broadcast partitions (never skipped)
         if (bc) {
             atomicAdd(&nbc, 1);
             for (int d = 0; d < N; ++d) atomicAdd(&bcs[d], (unsigned long long)H(d, 1, p));
@@ -353,7 +361,7 @@ __global__ void __launch_bounds__(1024) k_plan(Ctx c) {
     __syncthreads();
     // per owned partition: R and S sizes of its received pieces
     auto own_p = [&](int i) -> int { return i < nr ? plo + i : c.plist[i]; };
-    auto own_len = [&](int rel, int p) -> uint64_t { return rel ? (bcf[p] ? (uint64_t)H(c.rank, 1, p) : tot1[p]) : tot0[p]; };
+    auto own_len = [&](int rel, int p) -> uint64_t { return rel ? (bcf[p] ? (uint64_t)H(c.rank, 1, p) : tot1[p]) : tot0[p]; };  // 0 if skipped
     {  // largest owned R partition and total owned R + S: warp reductions, one shared atomic per warp
         unsigned long long mr = 0, sr = 0;
         for (int i = tid; i < np; i += blockDim.x) {

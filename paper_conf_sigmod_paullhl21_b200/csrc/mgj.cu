@@ -352,6 +352,7 @@ mgj_status mgj_plan(const mgj_config *cfg, const mgj_peers *peers, mgj_handle *o
     h->cdesc = static_cast<ChunkDesc *>(dalloc(h, 2 * n.max_chunks * sizeof(ChunkDesc), &st));
     c.owner = static_cast<int32_t *>(dalloc(h, P * 4, &st));
     c.bcast = static_cast<uint8_t *>(dalloc(h, P, &st));
+    c.pskip = static_cast<uint8_t *>(dalloc(h, P, &st));
     c.plist = static_cast<int32_t *>(dalloc(h, P * 4, &st));
     c.bcast_cfg = n.c.skew_bcast;
     c.send_off = static_cast<uint64_t *>(dalloc(h, 2ull * P * 8, &st));
@@ -562,7 +563,8 @@ void mgj_destroy(mgj_handle h) {
 }
 
 mgj_status mgj_plan_host(int32_t world_size, int32_t rank, int32_t bits, const uint32_t *hist, int32_t *owner,
-                         uint64_t *send_off, uint64_t *recv_size, int32_t skew_bcast, uint8_t *bcast) {
+                         uint64_t *send_off, uint64_t *recv_size, int32_t skew_bcast, uint8_t *bcast,
+                         uint8_t *skip) {
     if (world_size < 1 || world_size > MAX_RANKS || rank < 0 || rank >= world_size || bits < 1 || bits > MAX_B1 ||
         !hist || !owner || !send_off || !recv_size || skew_bcast < -1 || skew_bcast > 1)
         return MGJ_EINVAL;
@@ -578,13 +580,17 @@ mgj_status mgj_plan_host(int32_t world_size, int32_t rank, int32_t bits, const u
         return MGJ_ENOMEM;
     }
     uint64_t s_total = 0;
-    for (int p = 0; p < P; ++p)
+    for (int p = 0; p < P; ++p) {
         for (int rel = 0; rel < 2; ++rel) {
             uint64_t t = 0;
             for (int g = 0; g < N; ++g) t += H(g, rel, p);
             tot[rel * P + p] = t;
-            if (rel) s_total += t;
         }
+        const bool sk = skip_of(tot[p], tot[P + p]);
+        if (skip) skip[p] = sk;
+        if (sk) tot[p] = tot[P + p] = 0;
+        s_total += tot[P + p];
+    }
     uint64_t total = 0, run[2] = {0, 0};
     for (int p = 0; p < P; ++p) {
         bc[p] = bcast_of(tot[p], tot[P + p], s_total, N, P, skew_bcast);
@@ -681,6 +687,7 @@ mgj_status mgj_debug_copy(mgj_handle h, int32_t what, void *dst, uint64_t bytes,
         case MGJ_DBG_MAIL_HIST: src = h->arena[c.rank] + n.lay.mail; size = (uint64_t)c.world * 2 * P * 4; break;
         case MGJ_DBG_OWNER: src = c.owner; size = (uint64_t)P * 4; break;
         case MGJ_DBG_BCAST: src = c.bcast; size = (uint64_t)P; break;
+        case MGJ_DBG_SKIP: src = c.pskip; size = (uint64_t)P; break;
         case MGJ_DBG_PLIST: src = c.plist; size = (uint64_t)std::max(meta[MT_NP], 0) * 4; break;
         case MGJ_DBG_SEND_OFF: src = c.send_off; size = 2ull * P * 8; break;
         case MGJ_DBG_RECV_SIZE: src = c.recv_size; size = sizeof(rs); break;

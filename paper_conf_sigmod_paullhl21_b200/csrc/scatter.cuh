@@ -222,10 +222,11 @@ __global__ void __launch_bounds__(NT, NT <= 512 ? 2 : 1) k_scatter(Ctx c) {
     // per owned partition (registers): destination of the next group, carry
     ull base[PPT];
     uint32_t cc[PPT], hd[PPT], lim[PPT];
+    bool skp[PPT];  // partition skipped by the plan (an empty side): nothing is stored
     Tup carry[PPT][CW];
     bool pending = false;  // carries of the last sub-tile still sit in `sorted`
 #pragma unroll
-    for (int k = 0; k < PPT; ++k) base[k] = 0, cc[k] = 0, hd[k] = 0, lim[k] = 0;
+    for (int k = 0; k < PPT; ++k) base[k] = 0, cc[k] = 0, hd[k] = 0, lim[k] = 0, skp[k] = false;
 
     auto subtile = [&](uint32_t g, int &rel, uint64_t &first, uint32_t &len) {
         rel = g < nsub0 ? 0 : 1;
@@ -261,7 +262,7 @@ __global__ void __launch_bounds__(NT, NT <= 512 ? 2 : 1) k_scatter(Ctx c) {
         for (int k = 0; k < PPT; ++k)
 #pragma unroll
             for (int i = 0; i < CW; ++i)
-                if (i >= (int)hd[k] && i < (int)cc[k]) reinterpret_cast<Tup *>(base[k])[i] = carry[k][i];
+                if (!skp[k] && i >= (int)hd[k] && i < (int)cc[k]) reinterpret_cast<Tup *>(base[k])[i] = carry[k][i];
     };
     auto set_base = [&](int rel) {  // destination of this tile's first tuple of each owned partition
         const uint32_t *tb = c.tile_base + ((size_t)rel * c.G + tile) * P;
@@ -274,6 +275,7 @@ __global__ void __launch_bounds__(NT, NT <= 512 ? 2 : 1) k_scatter(Ctx c) {
                 // destination: the owner, or this rank itself for the S side of a
                 // selectively broadcast partition (a2, NEXT-2)
                 const int dst = (rel && c.bcast[p]) ? c.rank : c.owner[p];
+                skp[k] = c.pskip[p] != 0;
                 const ull a = (ull)(c.arena[dst] + c.lay.recv[rel]) + (so[p] + tb[p]) * (uint64_t)TB;
                 const uint32_t h = SG > 1 ? (uint32_t)((a & (GB - 1)) / TB) : 0u;
                 base[k] = a - (ull)h * TB;
@@ -381,7 +383,7 @@ __global__ void __launch_bounds__(NT, NT <= 512 ? 2 : 1) k_scatter(Ctx c) {
                 const uint32_t full = cnt[k] & ~(uint32_t)(SG - 1);
                 PInfo in;
                 in.wb = base[k] - (ull)o * TB;
-                in.lim = o + cnt[k];
+                in.lim = skp[k] ? o : o + cnt[k];  // a skipped partition's groups are never stored
                 in.head = (hd[k] && full) ? (o << 2 | hd[k]) : NONE;
                 pinfo[p] = in;
                 base[k] += (ull)full * TB;

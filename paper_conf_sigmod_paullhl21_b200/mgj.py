@@ -27,7 +27,7 @@ MAX_RANKS = 8
 # mgj_debug_what
 DBG = dict(RANK_HIST=1, MAIL_HIST=2, OWNER=3, SEND_OFF=4, RECV_SIZE=5, RECV_R=6, RECV_S=7,
            LOCAL_R=8, LOCAL_S=9, META=10, CHUNK_OFF_R=11, CHUNK_OFF_S=12, CHUNK_BASE=13, SEGMENTS=14,
-           OUT_KEY=15, OUT_PAY_R=16, OUT_PAY_S=17, MID_R=18, MID_S=19, VSTART=20, BCAST=21, PLIST=22)
+           OUT_KEY=15, OUT_PAY_R=16, OUT_PAY_S=17, MID_R=18, MID_S=19, VSTART=20, BCAST=21, PLIST=22, SKIP=23)
 GEN_KIND = {"unique": 0, "zipf": 1, "wide": 2}
 
 
@@ -93,7 +93,7 @@ _lib.mgj_result.argtypes = [_H, ctypes.POINTER(Result)]
 _lib.mgj_destroy.restype = None
 _lib.mgj_destroy.argtypes = [_H]
 _lib.mgj_plan_host.restype = ctypes.c_int
-_lib.mgj_plan_host.argtypes = [ctypes.c_int32, ctypes.c_int32, ctypes.c_int32, _P, _P, _P, _P, ctypes.c_int32, _P]
+_lib.mgj_plan_host.argtypes = [ctypes.c_int32, ctypes.c_int32, ctypes.c_int32, _P, _P, _P, _P, ctypes.c_int32, _P, _P]
 _lib.mgj_gen_relation.restype = ctypes.c_int
 _lib.mgj_gen_relation.argtypes = [ctypes.c_int32, ctypes.c_int32, _U64, _U64, ctypes.c_double,
                                   _U64, _U64, _P, _P, _P]
@@ -252,16 +252,17 @@ def device_bytes(ptr: int, nbytes: int):
 
 def plan_host(world: int, rank: int, bits: int, hist: np.ndarray, skew_bcast: int = 0, with_bcast: bool = False):
     """Host reference of the a2 assignment (mgj_plan_host): owner, send offsets, receive sizes
-    (and the selective-broadcast flags with with_bcast=True)."""
+    (and, with with_bcast=True, the selective-broadcast flags and the empty-side skip flags)."""
     P = 1 << bits
     hist = np.ascontiguousarray(hist, dtype=np.uint32).reshape(world, 2, P)
     owner = np.empty(P, np.int32)
     send_off = np.empty((2, P), np.uint64)
     recv_size = np.empty((2, world), np.uint64)
     bcast = np.empty(P, np.uint8)
+    skip = np.empty(P, np.uint8)
     _check(_lib.mgj_plan_host(world, rank, bits, hist.ctypes.data, owner.ctypes.data, send_off.ctypes.data,
-                              recv_size.ctypes.data, skew_bcast, bcast.ctypes.data), "mgj_plan_host")
-    return (owner, send_off, recv_size, bcast) if with_bcast else (owner, send_off, recv_size)
+                              recv_size.ctypes.data, skew_bcast, bcast.ctypes.data, skip.ctypes.data), "mgj_plan_host")
+    return (owner, send_off, recv_size, bcast, skip) if with_bcast else (owner, send_off, recv_size)
 
 
 def gen_relation(kind: str, rel: int, n_r: int, n_s: int, z: float, row0: int, count: int, keys, pays,

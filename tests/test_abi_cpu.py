@@ -83,27 +83,31 @@ def check_plan_invariants(mgj, hist, bits, skew_bcast=0):
     N = hist.shape[0]
     P = 1 << bits
     plans = [mgj.plan_host(N, g, bits, hist, skew_bcast=skew_bcast, with_bcast=True) for g in range(N)]
-    owner, recv, bc = plans[0][0], plans[0][2], plans[0][3]
-    for o, _, rs, b in plans:  # every rank computes the same assignment
+    owner, recv, bc, skip = plans[0][0], plans[0][2], plans[0][3], plans[0][4]
+    for o, _, rs, b, sk in plans:  # every rank computes the same assignment
         assert np.array_equal(o, owner) and np.array_equal(rs, recv) and np.array_equal(b, bc)
+        assert np.array_equal(sk, skip)
+    tot = hist.astype(np.uint64).sum(axis=0)  # [2][P]
+    # the histogram as a Bloom filter: exactly the partitions with one empty side
+    np.testing.assert_array_equal(skip != 0, (tot[0] == 0) != (tot[1] == 0))
+    assert not (bc.astype(bool) & skip.astype(bool)).any()
     assert np.all(np.diff(owner) >= 0) and owner.min() >= 0 and owner.max() < N
     if N == 1 or skew_bcast < 0:
         assert not bc.any()
-    tot = hist.astype(np.uint64).sum(axis=0)  # [2][P]
     for rel in range(2):
-        assert int(recv[rel].sum()) == int(tot[rel].sum())
+        assert int(recv[rel].sum()) == int(tot[rel][skip == 0].sum())
         for d in range(N):
             cover = np.zeros(int(recv[rel, d]), np.int32)
             for g in range(N):
                 so = plans[g][1][rel]
                 for p in range(P):
                     dest = g if (rel == 1 and bc[p]) else owner[p]
-                    if dest != d:
+                    if dest != d or skip[p]:
                         continue
                     c = int(hist[g, rel, p])
                     cover[int(so[p]):int(so[p]) + c] += 1
             assert np.all(cover == 1)
-    return owner, recv, bc
+    return owner, recv, bc, skip
 
 
 @pytest.mark.parametrize("N", [1, 2, 3, 5, 8])
@@ -112,11 +116,14 @@ def test_plan_host_invariants_random(mgj, N):
     bits = 6
     hist = rng.integers(0, 50, size=(N, 2, 1 << bits)).astype(np.uint32)
     hist[:, :, 5] = 0  # empty partitions
-    check_plan_invariants(mgj, hist, bits)
+    hist[:, 0, 9] = 0  # no R tuple: partition 9's S is never shuffled
+    hist[:, 1, 11] = 0  # no S tuple: partition 11's R neither
+    _, _, _, skip = check_plan_invariants(mgj, hist, bits)
+    assert skip[9] and skip[11] and not skip[5]
     check_plan_invariants(mgj, hist, bits, skew_bcast=-1)
     hist[:, 1, 7] *= 40  # heavy S partitions: broadcast candidates
     hist[:, 1, 40] = 5000
-    _, _, bc = check_plan_invariants(mgj, hist, bits)
+    _, _, bc, _ = check_plan_invariants(mgj, hist, bits)
     assert bc[40] == (N > 1)
     check_plan_invariants(mgj, hist, bits, skew_bcast=1)
 
@@ -124,7 +131,7 @@ def test_plan_host_invariants_random(mgj, N):
 def test_plan_host_uniform_identity_ranges(mgj):
     N, bits = 8, 10
     hist = np.full((N, 2, 1 << bits), 64, np.uint32)
-    owner, recv, bc = check_plan_invariants(mgj, hist, bits)
+    owner, recv, bc, _ = check_plan_invariants(mgj, hist, bits)
     assert not bc.any()  # uniform data never broadcasts
     assert np.array_equal(owner, np.arange(1 << bits) * N >> bits)
     assert np.all(recv == 64 * N * (1 << bits) // N)
@@ -135,7 +142,7 @@ def test_plan_host_skew_balances(mgj):
     N, bits = 4, 8
     hist = np.full((N, 2, 1 << bits), 10, np.uint32)
     hist[:, 1, 200] = 5000
-    owner, recv, _ = check_plan_invariants(mgj, hist, bits, skew_bcast=-1)
+    owner, recv, _, _ = check_plan_invariants(mgj, hist, bits, skew_bcast=-1)
     assert owner[200] in (2, 3)
     # partitions below the heavy one spread over the other owners
     assert len(set(owner[:200].tolist())) >= 2
@@ -149,7 +156,7 @@ def test_plan_host_selective_broadcast(mgj):
     P = 1 << bits
     hist = np.full((N, 2, P), 10, np.uint32)
     hist[:, 1, 200] = 5000
-    owner, recv, bc = check_plan_invariants(mgj, hist, bits)
+    owner, recv, bc, _ = check_plan_invariants(mgj, hist, bits)
     assert bc.sum() == 1 and bc[200]
     # S receive sizes: every rank holds its own 5000 S tuples of partition 200
     s_range = [sum(10 * N for p in range(P) if owner[p] == d and not bc[p]) for d in range(N)]
@@ -160,11 +167,11 @@ def test_plan_host_selective_broadcast(mgj):
     assert max(load) - min(load) <= 2 * 20 * N + 5000
     # auto mode leaves the same partition alone when R is not small: (N-1)|R_p| >= |S_p|
     hist[:, 0, 200] = 2000
-    _, _, bc2 = check_plan_invariants(mgj, hist, bits)
+    _, _, bc2, _ = check_plan_invariants(mgj, hist, bits)
     assert not bc2.any()
 
 
 def test_plan_host_all_empty(mgj):
     hist = np.zeros((4, 2, 1 << 5), np.uint32)
-    owner, recv, _ = check_plan_invariants(mgj, hist, 5)
+    owner, recv, _, _ = check_plan_invariants(mgj, hist, 5)
     assert np.array_equal(owner, np.arange(32) * 4 // 32)

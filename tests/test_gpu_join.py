@@ -436,7 +436,8 @@ def check_bcast_virtual(mgj, w, N, skew, materialize=True, expect_bc=True, **kw)
     kdt = np.uint32 if w.key_bytes == 4 else np.uint64
     nbc = None
     for g, j in enumerate(joins):
-        owner, send_off, recv_size, bc = mgj.plan_host(N, g, B1, mail, skew_bcast=skew, with_bcast=True)
+        owner, send_off, recv_size, bc, skip = mgj.plan_host(N, g, B1, mail, skew_bcast=skew, with_bcast=True)
+        np.testing.assert_array_equal(j.debug("SKIP", np.uint8), skip)
         np.testing.assert_array_equal(j.debug("OWNER", np.int32), owner)
         np.testing.assert_array_equal(j.debug("BCAST", np.uint8), bc)
         np.testing.assert_array_equal(j.debug("SEND_OFF", np.uint64).reshape(2, P), send_off)
@@ -495,6 +496,35 @@ def test_virtual_ranks_bcast_wide(mgj):
     w = ArrayWorkload(rk, (np.arange(rk.size) + (1 << 40)).astype(np.uint64), sk,
                       (np.arange(sk.size) + (1 << 41)).astype(np.uint64))
     check_bcast_virtual(mgj, w, 4, 1, materialize=True, radix_bits_global=5)
+
+
+@pytest.mark.parametrize("N", [1, 4])
+def test_bloom_skip_partitions(mgj, N):
+    """The histogram as a Bloom filter: partitions with no R or no S tuple
+    are not shuffled; the result is unchanged and only the shared partitions arrive."""
+    B1, P = 6, 64
+    rng = np.random.default_rng(3)
+    def keys(n, lo, hi):  # digit1 in [lo, hi)
+        return ((rng.integers(0, 1 << 20, n, dtype=np.uint64) << B1) | rng.integers(lo, hi, n, dtype=np.uint64)).astype(np.uint32)
+    rk = keys(30000, 0, 48)
+    rs = rk[((rk & (P - 1)) >= 16)]  # R keys of the shared partitions [16, 48)
+    sk = np.concatenate([keys(20000, 16, 64), rs[rng.integers(0, rs.size, 20000)]])
+    w = ArrayWorkload(rk, np.arange(rk.size, dtype=np.uint32), sk, np.arange(sk.size, dtype=np.uint32))
+    joins, res, _ = run_virtual(mgj, w, N, materialize=True, radix_bits_global=B1)
+    ref = oracle.join(rk, w.a["r_pays"], sk, w.a["s_pays"], materialize=True)
+    for r in res:
+        assert (r["match_count"], r["checksum"]) == (ref["count"], ref["checksum"])
+    trip = [j.materialized(r) for j, r in zip(joins, res)]
+    k, a, b = sort_trip(*(np.concatenate([t[i] for t in trip]) for i in range(3)))
+    np.testing.assert_array_equal(k, ref["key"])
+    np.testing.assert_array_equal(b, ref["pay_s"])
+    shared = lambda x: ((x & (P - 1)) >= 16) & ((x & (P - 1)) < 48)
+    assert sum(r["recv_r"] for r in res) == int(shared(rk).sum())
+    assert sum(r["recv_s"] for r in res) == int(shared(sk).sum())
+    skip = joins[0].debug("SKIP", np.uint8)
+    np.testing.assert_array_equal(skip != 0, (np.arange(P) < 16) | (np.arange(P) >= 48))
+    for j in joins:
+        j.close()
 
 
 def test_virtual_ranks_wide(mgj):

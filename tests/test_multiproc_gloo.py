@@ -42,7 +42,7 @@ def _worker(rank, world, port, bits, kind, skew, q):
         allh = [torch.zeros(2, P, dtype=torch.int64) for _ in range(world)]
         dist.all_gather(allh, torch.from_numpy(hist))
         H = np.stack([h.numpy() for h in allh]).astype(np.uint32)
-        owner, send_off, recv_size, bc = mgj.plan_host(world, rank, bits, H, skew_bcast=skew, with_bcast=True)
+        owner, send_off, recv_size, bc, skip = mgj.plan_host(world, rank, bits, H, skew_bcast=skew, with_bcast=True)
         if skew < 0:
             assert not bc.any()
         out = {}
@@ -50,6 +50,8 @@ def _worker(rank, world, port, bits, kind, skew, q):
             part = (k & (P - 1)).astype(np.int64)
             # a selectively broadcast partition (NEXT-2) keeps its S on this rank
             dest = np.where(bc[part] != 0, rank, owner[part]) if rel == 1 else owner[part]
+            keep = skip[part] == 0  # empty-side partitions are not shuffled
+            k, p, part, dest = k[keep], p[keep], part[keep], dest[keep]
             # slot of each tuple inside its owner's receive buffer: send_off[p] + rank inside (rank, p)
             order = np.argsort(part, kind="stable")
             rank_in_p = np.empty(k.size, np.int64)

@@ -23,6 +23,10 @@ namespace mgj {
 // < 32-byte tail of a partition waits (in registers of its owning thread)
 // for the next sub-tile.  For P = 4096 the alignment padding would not fit
 // shared memory, so SG = 1 (one tuple per store).
+#ifndef SCAT_GDST
+#define SCAT_GDST 0  // per-group destination table written at layout time, no partition lookup in the write-out (measured slower: 4.36 vs 4.16 ms)
+#endif
+
 #ifndef SCAT_SOA
 #define SCAT_SOA 0  // 4-byte keys: `sorted` held as key and payload arrays (4-byte random stores; measured slower: 4.42 vs 4.14 ms)
 #endif
@@ -68,7 +72,8 @@ __host__ __device__ inline size_t scat_smem_bytes(int P, int key_bytes) {
     const size_t TB = 2 * (size_t)key_bytes;
     return ((g.alias || SCAT_LDG) ? 0 : 2 * (size_t)g.T * key_bytes)  // input stage: keys + payloads (SoA)
            + ((size_t)g.T + 2 * (size_t)(g.SG - 1) * P) * TB  // partition-sorted sub-tile (+ carries, group padding)
-           + (size_t)P * sizeof(PInfo)
+           + ((SCAT_GDST && g.SG > 1) ? ((size_t)g.T + 2 * (size_t)(g.SG - 1) * P) / g.SG * 8  // group destinations
+                                      : (size_t)P * sizeof(PInfo))
            + (size_t)P * 4;                                  // next free slot per partition
 }
 
@@ -96,6 +101,34 @@ __device__ __forceinline__ uint32_t block_scan_reg(uint32_t v, uint32_t *tmp, ui
     total = tmp[31];
     return x - v + (w ? tmp[w - 1] : 0);
 }
+
+// Same with one barrier: every warp reduces the per-warp totals itself (its
+// prefix and the block total) instead of one warp scanning them behind a
+// second barrier.  `tmp` may be rewritten only after a later barrier.
+__device__ __forceinline__ uint32_t block_scan_reg1(uint32_t v, uint32_t *tmp, uint32_t &total) {
+    const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+    uint32_t x = v;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+        if (lane >= o) x += y;
+    }
+    if (lane == 31) tmp[w] = x;
+    __syncthreads();
+    const uint32_t t = lane < (int)(blockDim.x >> 5) ? tmp[lane] : 0u;
+    uint32_t pre = lane < w ? t : 0u, tot = t;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        pre += __shfl_xor_sync(0xffffffffu, pre, o);
+        tot += __shfl_xor_sync(0xffffffffu, tot, o);
+    }
+    total = tot;
+    return x - v + pre;
+}
+
+#ifndef SCAT_SCAN1
+#define SCAT_SCAN1 0  // one-barrier layout scan (measured neutral: 4.16 vs 4.16 ms)
+#endif
 
 template <int BYTES> struct Vec;
 template <> struct Vec<8> { using T = uint2; };
@@ -179,8 +212,14 @@ __global__ void __launch_bounds__(NT, NT <= 512 ? 2 : 1) k_scatter(Ctx c) {
     Tup *const sorted = reinterpret_cast<Tup *>(smem + ((ALIAS || LDG) ? 0 : 2 * T * sizeof(K)));
     K *const skey = reinterpret_cast<K *>(ALIAS ? static_cast<void *>(sorted) : static_cast<void *>(smem));
     K *const spay = skey + T;
+    // GD: the layout writes every group's destination (0: not stored; low bits:
+    // h placeholder slots of a head group) so the write-out needs no lookup of
+    // the group's partition; otherwise a per-partition descriptor (PInfo)
+    constexpr bool GD = SCAT_GDST && SG > 1;
     PInfo *const pinfo = reinterpret_cast<PInfo *>(sorted + T + 2 * (SG - 1) * P);  // 16-byte aligned
-    uint32_t *const off = reinterpret_cast<uint32_t *>(pinfo + P);  // next free slot per partition
+    unsigned long long *const gdst = reinterpret_cast<unsigned long long *>(pinfo);
+    uint32_t *const off = GD ? reinterpret_cast<uint32_t *>(gdst + (T + 2 * (SG - 1) * P) / SG)
+                             : reinterpret_cast<uint32_t *>(pinfo + P);  // next free slot per partition
     K *const ks = reinterpret_cast<K *>(sorted);  // SOA: keys, then payloads
     K *const ps = ks + (T + 2 * (SG - 1) * P);
     auto sput = [&](uint32_t x, const Tup &t) {
@@ -365,7 +404,8 @@ __global__ void __launch_bounds__(NT, NT <= 512 ? 2 : 1) k_scatter(Ctx c) {
         }
         load_counts(g + 1, ncnt);  // prefetch (consumed next iteration)
         uint32_t total;
-        uint32_t o = block_scan_reg(tsum, tmp, total);  // its barriers: last write-out is done
+        uint32_t o = SCAT_SCAN1 ? block_scan_reg1(tsum, tmp, total)   // its barrier: last write-out is done
+                                : block_scan_reg(tsum, tmp, total);
         uint32_t co[PPT], ccw[PPT];  // segment start and carried count (for the ALIAS carry write)
 #pragma unroll
         for (int k = 0; k < PPT; ++k) ccw[k] = cc[k], co[k] = 0;
@@ -381,11 +421,17 @@ __global__ void __launch_bounds__(NT, NT <= 512 ? 2 : 1) k_scatter(Ctx c) {
                 co[k] = o;
                 off[p] = o + cc[k];
                 const uint32_t full = cnt[k] & ~(uint32_t)(SG - 1);
-                PInfo in;
-                in.wb = base[k] - (ull)o * TB;
-                in.lim = skp[k] ? o : o + cnt[k];  // a skipped partition's groups are never stored
-                in.head = (hd[k] && full) ? (o << 2 | hd[k]) : NONE;
-                pinfo[p] = in;
+                if constexpr (GD) {
+                    const uint32_t ng = seg[k] / SG, nf = full / SG;
+                    for (uint32_t j = 0; j < ng; ++j)  // a skipped partition's groups are never stored
+                        gdst[o / SG + j] = (j < nf && !skp[k]) ? ((base[k] + (ull)j * GB) | (j == 0 ? hd[k] : 0u)) : 0ull;
+                } else {
+                    PInfo in;
+                    in.wb = base[k] - (ull)o * TB;
+                    in.lim = skp[k] ? o : o + cnt[k];  // a skipped partition's groups are never stored
+                    in.head = (hd[k] && full) ? (o << 2 | hd[k]) : NONE;
+                    pinfo[p] = in;
+                }
                 base[k] += (ull)full * TB;
                 if (full) hd[k] = 0;
                 cc[k] = cnt[k] - full;
@@ -491,6 +537,22 @@ __global__ void __launch_bounds__(NT, NT <= 512 ? 2 : 1) k_scatter(Ctx c) {
                     }
                 }
             }
+            if constexpr (GD) {
+#pragma unroll
+                for (int r = 0; r < WU; ++r) {
+                    const ull d = on[r] ? gdst[slot[r] / SG] : 0ull;
+                    if (d) {
+                        char *dst = reinterpret_cast<char *>(d & ~(ull)(GB - 1));
+                        if (SCAT_RING) dst = c.arena[0] + c.lay.recv[0] + ((dst - c.arena[0] - c.lay.recv[0]) & (ull)(SCAT_RING - 1));
+                        const uint32_t h = (uint32_t)(d & (GB - 1));
+                        if (!h) {
+                            st_group<GB>(dst, gv[r]);
+                        } else {
+                            for (uint32_t i = h; i < SG; ++i) reinterpret_cast<Tup *>(dst)[i] = sget(slot[r] + i);
+                        }
+                    }
+                }
+            } else {
 #pragma unroll
             for (int r = 0; r < WU; ++r)
                 if (on[r]) in[r] = pinfo[reinterpret_cast<const uint32_t *>(&gv[r])[0] & (uint32_t)(P - 1)];
@@ -506,6 +568,7 @@ __global__ void __launch_bounds__(NT, NT <= 512 ? 2 : 1) k_scatter(Ctx c) {
                             reinterpret_cast<Tup *>(dst)[i] = sget(slot[r] + i);
                     }
                 }
+            }
             }
         }
         if (ALIAS) {  // the sorted buffer is read: load the next sub-tile into its head

@@ -467,7 +467,7 @@ __global__ void __launch_bounds__(1024) k_plan(Ctx c) {
         // two-level local partitioning: when the owned
         // partitions span more than LOCAL2_NCH chunks on average, a first
         // histogram-based pass splits every owned partition into 2^BA
-        // contiguous sub-partitions of ~48 chunks, and the chunked pass then
+        // contiguous sub-partitions of ~64 chunks, and the chunked pass then
         // uses the remaining B2 - BA bits.  The mean, not the maximum: a few
         // heavy-hitter partitions (Zipf) are not helped by splitting the rest
         const uint32_t meannch = np ? (max(nch[0], nch[1]) + np - 1) / np : 0;
@@ -475,7 +475,7 @@ __global__ void __launch_bounds__(1024) k_plan(Ctx c) {
         if (c.split_cfg > 0) {
             BA = c.split_cfg;
         } else if (c.split_cfg == 0 && meannch > (uint32_t)LOCAL2_NCH) {
-            BA = ceil_log2_u64((meannch + 47) / 48);
+            BA = ceil_log2_u64((meannch + 63) / 64);  // measured at N=8-sized partitions: BA 3 > 4 > 2
             while (BA > 0 && (np << BA) > c.vcap) --BA;
         }
         if (BA > B2) BA = B2;

@@ -111,9 +111,47 @@ __device__ __forceinline__ uint32_t nch_local(const Ctx &c, int rel) {
 
 // Padded size (slots) of every (owned partition, first-pass digit) run, summed
 // over the chunks of the partition: exactly the slots k_local<K, LM_SPLIT>
-// reserves.  QA <= 8 (the auto choice): each thread counts its <= 24 tuples
+// reserves.  QA <= 32: each thread counts its <= 24 tuples
 // of a chunk in eight 8-bit fields of one register, reduced per warp once per
 // chunk; larger QA: warp-aggregated shared atomics (one per distinct digit).
+// Per-thread digit counts of one chunk in NA packed registers (eight 8-bit
+// fields each: digit q -> register q / 8, field q % 8; a thread sees at most
+// C / 512 <= 24 tuples), reduced per warp into the shared counters.
+template <int NA, typename Tup>
+__device__ __forceinline__ void count_packed(const Tup *src, uint32_t len, int tid, uint32_t nt, int lane, int B1,
+                                             int QA, uint32_t *cnt) {
+    unsigned long long acc[NA];
+#pragma unroll
+    for (int a = 0; a < NA; ++a) acc[a] = 0;
+#define MGJ_COUNT_ADD(qq)                                                  \
+    do {                                                                   \
+        const uint32_t q_ = (qq);                                          \
+        const unsigned long long one_ = 1ull << (8 * (q_ & 7u));           \
+        _Pragma("unroll") for (int a_ = 0; a_ < NA; ++a_) acc[a_] += (q_ >> 3) == (uint32_t)a_ ? one_ : 0ull; \
+    } while (0)
+    uint32_t i = tid;
+    for (; i + 3 * nt < len; i += 4 * nt) {
+        const auto k0 = __ldcs(&src[i].x), k1 = __ldcs(&src[i + nt].x);
+        const auto k2 = __ldcs(&src[i + 2 * nt].x), k3 = __ldcs(&src[i + 3 * nt].x);
+        MGJ_COUNT_ADD(digit2(k0, B1, QA));
+        MGJ_COUNT_ADD(digit2(k1, B1, QA));
+        MGJ_COUNT_ADD(digit2(k2, B1, QA));
+        MGJ_COUNT_ADD(digit2(k3, B1, QA));
+    }
+    for (; i < len; i += nt) MGJ_COUNT_ADD(digit2(__ldcs(&src[i].x), B1, QA));
+#undef MGJ_COUNT_ADD
+#pragma unroll
+    for (int a = 0; a < NA; ++a)
+#pragma unroll
+        for (int f = 0; f < 8; ++f) {
+            const int q = a * 8 + f;
+            if (q < QA) {
+                const uint32_t v = __reduce_add_sync(0xffffffffu, (uint32_t)(acc[a] >> (8 * f)) & 0xffu);
+                if (lane == 0 && v) atomicAdd(&cnt[q], v);
+            }
+        }
+}
+
 template <typename K>
 __global__ void __launch_bounds__(512) k_countA(Ctx c, const ChunkDesc *cdesc) {
     using Tup = typename Layout<K>::Tup;
@@ -131,19 +169,11 @@ __global__ void __launch_bounds__(512) k_countA(Ctx c, const ChunkDesc *cdesc) {
         if (tid < QA) cnt[tid] = 0;
         __syncthreads();
         if (QA <= 8) {
-            unsigned long long acc = 0;  // field q (8 bits): this thread's tuples with digit q
-            uint32_t i = tid;
-            for (; i + 3 * nt < d.len; i += 4 * nt) {
-                const K k0 = __ldcs(&src[i].x), k1 = __ldcs(&src[i + nt].x);
-                const K k2 = __ldcs(&src[i + 2 * nt].x), k3 = __ldcs(&src[i + 3 * nt].x);
-                acc += (1ull << (8 * digit2(k0, c.B1, QA))) + (1ull << (8 * digit2(k1, c.B1, QA))) +
-                       (1ull << (8 * digit2(k2, c.B1, QA))) + (1ull << (8 * digit2(k3, c.B1, QA)));
-            }
-            for (; i < d.len; i += nt) acc += 1ull << (8 * digit2(__ldcs(&src[i].x), c.B1, QA));
-            for (int q = 0; q < QA; ++q) {
-                const uint32_t v = __reduce_add_sync(0xffffffffu, (uint32_t)(acc >> (8 * q)) & 0xffu);
-                if (lane == 0 && v) atomicAdd(&cnt[q], v);
-            }
+            count_packed<1>(src, d.len, tid, nt, lane, c.B1, QA, cnt);
+        } else if (QA <= 16) {
+            count_packed<2>(src, d.len, tid, nt, lane, c.B1, QA, cnt);
+        } else if (QA <= 32) {
+            count_packed<4>(src, d.len, tid, nt, lane, c.B1, QA, cnt);
         } else {
             for (uint32_t i = tid; i < d.len; i += nt) {
                 const uint32_t q = digit2(__ldcs(&src[i].x), c.B1, QA);

@@ -214,15 +214,19 @@ __host__ __device__ inline int ceil_log2_u64(uint64_t x) {
     return l;
 }
 
-// B2: R co-partitions of at most ~target tuples (one shared-memory table),
-// and, on average, R + S co-partitions of at most 2 * target tuples (one
-// probe stage, shared by the two sides).  The largest owned R partition sets
-// the first bound; the mean R + S of the owned partitions the second (a
-// heavy-hitter partition cannot be split by radix bits: its S side is
-// sliced over several items instead).
-__host__ __device__ inline int choose_b2(uint64_t max_r, uint64_t mean_rs, int b2_cfg, int b2_max, uint64_t target) {
+// B2: R co-partitions that fit one shared-memory table (cap slots: the
+// largest owned R partition sets this bound, against the full capacity — a
+// co-partition a little above it is sliced, rarely), and, on average, R + S
+// co-partitions of at most 2 * target tuples (one probe stage shared by the
+// two sides, target = cap minus headroom for run padding and spread; the mean
+// R + S of the owned partitions sets this bound: a heavy-hitter partition
+// cannot be split by radix bits, its S side is sliced over several items).
+// (Against the target, the max bound doubled the fan-out of random 8-byte keys
+// whose largest partition exceeds the mean by a few sigma: M5 probe 2.8 ms.)
+__host__ __device__ inline int choose_b2(uint64_t max_r, uint64_t mean_rs, int b2_cfg, int b2_max, uint64_t target,
+                                         uint64_t cap) {
     if (b2_cfg > 0) return b2_cfg < b2_max ? b2_cfg : b2_max;
-    int b = ceil_log2_u64((max_r + target - 1) / target);
+    int b = ceil_log2_u64((max_r + cap - 1) / cap);
     const int bs = ceil_log2_u64((mean_rs + 2 * target - 1) / (2 * target));
     if (bs > b) b = bs;
     if (b > b2_max) b = b2_max;
@@ -381,7 +385,7 @@ __global__ void __launch_bounds__(1024) k_plan(Ctx c) {
     }
     __syncthreads();
     const int B2 = choose_b2(maxr, np > 0 ? sumrs / (uint64_t)np : 0, c.b2_cfg, c.b2_max,
-                             (uint64_t)c.probe_target);
+                             (uint64_t)c.probe_target, (uint64_t)c.probe_slots);
     // received pieces of every owned partition i: P2P — one piece per relation
     // (the whole segment, sources ascending inside it; a broadcast partition's
     // R piece in its root's buffer); EXTERNAL — one piece per source rank g,

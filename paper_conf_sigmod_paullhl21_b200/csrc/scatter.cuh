@@ -130,6 +130,22 @@ __device__ __forceinline__ uint32_t block_scan_reg1(uint32_t v, uint32_t *tmp, u
 #define SCAT_SCAN1 0  // one-barrier layout scan (measured neutral: 4.16 vs 4.16 ms)
 #endif
 
+// 16-byte shared load that the compiler keeps where it is written (not sunk
+// into the branch that consumes it): the write-out issues its group and
+// descriptor loads back to back.
+__device__ __forceinline__ uint4 lds128(const void *p) {
+    uint4 v;
+    asm volatile("ld.volatile.shared.v4.u32 {%0,%1,%2,%3}, [%4];"
+                 : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w)
+                 : "r"(smem_u32(p)));
+    return v;
+}
+
+#ifndef SCAT_EAGER
+#define SCAT_EAGER 1  // write-out: both group halves and the whole descriptor loaded up front, 8-byte keys
+                      // (measured: M5 scatter 3.725 -> 3.693 ms; 4-byte keys 4.155 -> 4.19, so not used there)
+#endif
+
 template <int BYTES> struct Vec;
 template <> struct Vec<8> { using T = uint2; };
 template <> struct Vec<16> { using T = uint4; };
@@ -216,6 +232,7 @@ __global__ void __launch_bounds__(NT, NT <= 512 ? 2 : 1) k_scatter(Ctx c) {
     // h placeholder slots of a head group) so the write-out needs no lookup of
     // the group's partition; otherwise a per-partition descriptor (PInfo)
     constexpr bool GD = SCAT_GDST && SG > 1;
+    constexpr bool EAGER = SCAT_EAGER && sizeof(K) == 8;
     PInfo *const pinfo = reinterpret_cast<PInfo *>(sorted + T + 2 * (SG - 1) * P);  // 16-byte aligned
     unsigned long long *const gdst = reinterpret_cast<unsigned long long *>(pinfo);
     uint32_t *const off = GD ? reinterpret_cast<uint32_t *>(gdst + (T + 2 * (SG - 1) * P) / SG)
@@ -529,7 +546,10 @@ __global__ void __launch_bounds__(NT, NT <= 512 ? 2 : 1) k_scatter(Ctx c) {
                         const uint4 pv = *reinterpret_cast<const uint4 *>(ps + slot[r]);
                         gv[r].a = make_uint4(kv.x, pv.x, kv.y, pv.y);
                         gv[r].b = make_uint4(kv.z, pv.z, kv.w, pv.w);
-                    } else if constexpr (GB == 32) {  // two conflict-free 16-byte halves (swizzled)
+                    } else if constexpr (GB == 32 && EAGER) {  // two conflict-free 16-byte halves (swizzled)
+                        gv[r].a = lds128(sorted + swz(slot[r]));
+                        gv[r].b = lds128(sorted + swz(slot[r] + SG / 2));
+                    } else if constexpr (GB == 32) {
                         gv[r].a = *reinterpret_cast<const uint4 *>(sorted + swz(slot[r]));
                         gv[r].b = *reinterpret_cast<const uint4 *>(sorted + swz(slot[r] + SG / 2));
                     } else {
@@ -554,8 +574,19 @@ __global__ void __launch_bounds__(NT, NT <= 512 ? 2 : 1) k_scatter(Ctx c) {
                 }
             } else {
 #pragma unroll
-            for (int r = 0; r < WU; ++r)
-                if (on[r]) in[r] = pinfo[reinterpret_cast<const uint32_t *>(&gv[r])[0] & (uint32_t)(P - 1)];
+            for (int r = 0; r < WU; ++r) {
+                if (on[r]) {
+                    const PInfo *pi = pinfo + (reinterpret_cast<const uint32_t *>(&gv[r])[0] & (uint32_t)(P - 1));
+                    if constexpr (EAGER) {
+                        const uint4 v = lds128(pi);
+                        in[r].wb = (ull)v.x | ((ull)v.y << 32);
+                        in[r].lim = v.z;
+                        in[r].head = v.w;
+                    } else {
+                        in[r] = *pi;
+                    }
+                }
+            }
 #pragma unroll
             for (int r = 0; r < WU; ++r) {
                 if (on[r] && slot[r] + SG <= in[r].lim) {

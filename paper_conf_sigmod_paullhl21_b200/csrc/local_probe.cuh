@@ -23,6 +23,10 @@ namespace mgj {
 #define PROBE_CPASYNC 0  // producers copy runs with 16-byte cp.async (LDGSTS) instead of one TMA bulk copy per run (measured slower: 4.64 vs 1.96 ms)
 #endif
 
+#ifndef PROBE_BAL
+#define PROBE_BAL 0  // the two producer warps of an item split its R + S runs evenly (measured: M2 probe 2.35 vs 1.96 ms, zipf z=1 2.80 vs 2.85, wide 2.70 vs 2.39)
+#endif
+
 #ifndef PROBE_U2
 #define PROBE_U2 0  // packed probe: two S slots per step (measured slower: 2.00 vs 1.96 ms)
 #endif
@@ -664,7 +668,25 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
                 for (int w = lane; w < PW; w += 32) pb[w] = 0;
                 __syncwarp();
             }
-            for (int rel = rel0; rel < rel1; ++rel) {
+            // PROBE_BAL (two producers per item): the item's R and S runs form one
+            // list and each warp issues half of it, instead of one warp per
+            // relation (|R|:|S| = 1:4 left the S warp with 4x the copies)
+            const bool bal = PROBE_BAL && PROBE_PPI == 2 && !SBITS;
+            uint32_t glo = 0, ghi = 0xffffffffu, nrun0 = 0;
+            if (bal) {
+                auto np_of = [&](int rel) -> uint32_t {
+                    const Side sd = rel ? x.it.s : x.it.r;
+                    const uint32_t xnch = rel ? x.nch[1] : x.nch[0];
+                    const uint32_t kend = min(sd.k1, xnch - 1);
+                    return sd.k0 <= kend ? kend - sd.k0 + 1 : 0;
+                };
+                nrun0 = np_of(0);
+                const uint32_t M = nrun0 + np_of(1), h = (M + 1) / 2;
+                glo = (warp & 1) ? h : 0;
+                ghi = (warp & 1) ? M : h;
+            }
+            for (int rel = bal ? 0 : rel0; rel < (bal ? 2 : rel1); ++rel) {
+                const uint32_t gbase = rel ? nrun0 : 0;  // index of the relation's first run in the item's list
                 const Side sd = rel ? x.it.s : x.it.r;
                 const uint32_t xcb = rel ? x.cb[1] : x.cb[0], xnch = rel ? x.nch[1] : x.nch[0];  // no local memory
                 const uint16_t *E0 = (rel ? c.eoff[1] : c.eoff[0]) + (size_t)(Q + 1) * xcb + (size_t)x.it.q * xnch;
@@ -698,6 +720,8 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
                     }
                     const uint32_t dst = run + incl - sz;
                     const uint32_t gsum = __shfl_sync(0xffffffffu, incl, 31);
+                    const bool issue_it = !bal || (gbase + m >= glo && gbase + m < ghi);
+                    const uint32_t gmine = bal ? __reduce_add_sync(0xffffffffu, issue_it ? sz : 0u) : gsum;
                     if (PROBE_CPASYNC) {
                         // the warp copies the batch's runs one after another, 16 bytes per lane
                         constexpr uint32_t PT = 16 / TB;  // tuples per 16-byte piece
@@ -711,18 +735,18 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
                                 cp_async16(dstbase + rdst + i * PT, lbase + rsrc + i * PT);
                         }
                     } else {
-                    if (lane == 0 && gsum)
+                    if (lane == 0 && gmine)
                         asm volatile("mbarrier.expect_tx.relaxed.cta.shared::cta.b64 [%0], %1;" ::"r"(
                                          smem_u32(&full[s])),
-                                     "r"(gsum * TB)
+                                     "r"(gmine * TB)
                                      : "memory");
                     __syncwarp();
-                    if (sz) tma_load_1d(dstbase + dst, lbase + src, sz * TB, &full[s], pol);
+                    if (sz && issue_it) tma_load_1d(dstbase + dst, lbase + src, sz * TB, &full[s], pol);
                     }
                     if (pad != 0xffffffffu) atomicOr(&pb[(dst + pad) >> 5], 1u << ((dst + pad) & 31));
                     run += gsum;
                 }
-                if (lane == 0) totals[s][rel] = run;
+                if (lane == 0 && (!bal || (warp & 1) == rel)) totals[s][rel] = run;
                 if (PROBE_L2PF && j + PROBE_L2PF * NPI < mine) {
                     // the same side of the item PROBE_L2PF rounds ahead: its runs -> L2, so that
                     // its stage loads hit L2 (more bytes in flight than the stages can hold)

@@ -23,6 +23,10 @@ namespace mgj {
 #define PROBE_CPASYNC 0  // producers copy runs with 16-byte cp.async (LDGSTS) instead of one TMA bulk copy per run (measured slower: 4.64 vs 1.96 ms)
 #endif
 
+#ifndef PROBE_SMALL
+#define PROBE_SMALL 0  // runs of at most this many tuples copied by the producer lane, no bulk copy (measured slower: zipf z=1 probe 3.13 / 3.55 ms at 8 / 16 vs 2.80)
+#endif
+
 #ifndef PROBE_BAL
 #define PROBE_BAL 0  // the two producer warps of an item split its R + S runs evenly (measured: M2 probe 2.35 vs 1.96 ms, zipf z=1 2.80 vs 2.85, wide 2.70 vs 2.39)
 #endif
@@ -657,6 +661,7 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
         const int pw = warp / PROBE_PPI;
         const int rel0 = PROBE_PPI == 2 ? (warp & 1) : 0, rel1 = PROBE_PPI == 2 ? rel0 + 1 : 2;
         ItemX x;
+        bool copied_small = false;  // this lane stored small runs into the stage (PROBE_SMALL)
         if (pw < (int)mine) x = items[blockIdx.x + pw * gridDim.x];
         for (uint32_t j = pw; j < mine; j += NPI) {
             ItemX xn;
@@ -721,7 +726,11 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
                     const uint32_t dst = run + incl - sz;
                     const uint32_t gsum = __shfl_sync(0xffffffffu, incl, 31);
                     const bool issue_it = !bal || (gbase + m >= glo && gbase + m < ghi);
-                    const uint32_t gmine = bal ? __reduce_add_sync(0xffffffffu, issue_it ? sz : 0u) : gsum;
+                    // runs of at most PROBE_SMALL tuples are copied by their lane with
+                    // plain loads/stores (a heavy partition leaves most co-partitions
+                    // in runs of a few tuples: one bulk copy each would dominate)
+                    const bool small = PROBE_SMALL && sz != 0 && sz <= PROBE_SMALL && issue_it;
+                    const uint32_t gmine = (bal || PROBE_SMALL) ? __reduce_add_sync(0xffffffffu, (issue_it && !small) ? sz : 0u) : gsum;
                     if (PROBE_CPASYNC) {
                         // the warp copies the batch's runs one after another, 16 bytes per lane
                         constexpr uint32_t PT = 16 / TB;  // tuples per 16-byte piece
@@ -741,7 +750,12 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
                                      "r"(gmine * TB)
                                      : "memory");
                     __syncwarp();
-                    if (sz && issue_it) tma_load_1d(dstbase + dst, lbase + src, sz * TB, &full[s], pol);
+                    if (small) {
+                        for (uint32_t i = 0; i < sz; ++i) dstbase[dst + i] = __ldcs(lbase + src + i);
+                        copied_small = true;
+                    } else if (sz && issue_it) {
+                        tma_load_1d(dstbase + dst, lbase + src, sz * TB, &full[s], pol);
+                    }
                     }
                     if (pad != 0xffffffffu) atomicOr(&pb[(dst + pad) >> 5], 1u << ((dst + pad) & 31));
                     run += gsum;
@@ -773,6 +787,11 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
             }
             __syncwarp();
             if (PROBE_CPASYNC) cp_async_mbar_arrive(&full[s]);  // fires when this lane's copies have landed
+            if (PROBE_SMALL) {  // this warp's plain stores, then lane 0's release arrive publishes them
+                if (copied_small) __threadfence_block();
+                __syncwarp();
+                copied_small = false;
+            }
             if (lane == 0) mbar_arrive(&full[s]);
             x = xn;
         }

@@ -27,6 +27,10 @@ namespace mgj {
 #define PROBE_SMALL 0  // runs of at most this many tuples copied by the producer lane, no bulk copy (measured slower: zipf z=1 probe 3.13 / 3.55 ms at 8 / 16 vs 2.80)
 #endif
 
+#ifndef PROBE_EPF
+#define PROBE_EPF 1  // producers load the next batch's run offsets while issuing the current batch
+#endif
+
 #ifndef PROBE_BAL
 #define PROBE_BAL 0  // the two producer warps of an item split its R + S runs evenly (measured: M2 probe 2.35 vs 1.96 ms, zipf z=1 2.80 vs 2.85, wide 2.70 vs 2.39)
 #endif
@@ -701,14 +705,22 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
                 Tup *dstbase = stages + (size_t)s * 2 * SL + (rel ? x.soff : 0);
                 const Tup *lbase = static_cast<const Tup *>(rel ? c.local[1] : c.local[0]);
                 uint32_t run = 0;
+                // run offsets of the next batch of 32 runs are loaded while this
+                // batch is scanned and issued (items of heavy partitions have
+                // hundreds of runs: one load latency per batch otherwise)
+                uint32_t en0 = 0, en1 = 0;
+                if (PROBE_EPF && lane < np) en0 = E0[sd.k0 + lane], en1 = E1[sd.k0 + lane];
                 for (uint32_t m0 = 0; m0 < np; m0 += 32) {
                     const uint32_t m = m0 + lane;
                     uint32_t sz = 0, pad = 0xffffffffu;
                     uint64_t src = 0;
+                    const uint32_t ec0 = en0, ec1 = en1;
+                    if (PROBE_EPF && m + 32 < np) en0 = E0[sd.k0 + m + 32], en1 = E1[sd.k0 + m + 32];
                     if (m < np) {
                         const uint32_t k = sd.k0 + m;
                         uint32_t st, slots, v;
-                        decode_run<ALIGN>(E0[k], E1[k], st, slots, v);
+                        if (PROBE_EPF) decode_run<ALIGN>(ec0, ec1, st, slots, v);
+                        else decode_run<ALIGN>(E0[k], E1[k], st, slots, v);
                         const uint32_t alo = (k == sd.k0) ? sd.a0 : 0;
                         const uint32_t ahi = (k == sd.k1) ? sd.a1 : slots;
                         if (ahi > alo) {

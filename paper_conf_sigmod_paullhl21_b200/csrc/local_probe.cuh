@@ -31,6 +31,10 @@ namespace mgj {
 #define PROBE_EPF 1  // producers load the next batch's run offsets while issuing the current batch
 #endif
 
+#ifndef PROBE_EPF2
+#define PROBE_EPF2 0  // ... and the first batch of their next item's while finishing the current item (measured neutral: M2 1.957 vs 1.955, materialised 3.80 vs 3.85, wide 2.40 vs 2.38 with spills)
+#endif
+
 #ifndef PROBE_BAL
 #define PROBE_BAL 0  // the two producer warps of an item split its R + S runs evenly (measured: M2 probe 2.35 vs 1.96 ms, zipf z=1 2.80 vs 2.85, wide 2.70 vs 2.39)
 #endif
@@ -666,6 +670,8 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
         const int rel0 = PROBE_PPI == 2 ? (warp & 1) : 0, rel1 = PROBE_PPI == 2 ? rel0 + 1 : 2;
         ItemX x;
         bool copied_small = false;  // this lane stored small runs into the stage (PROBE_SMALL)
+        bool xpf = false;           // pf0/pf1 hold the first batch of run offsets of item x (PROBE_EPF2)
+        uint32_t pf0 = 0, pf1 = 0;
         if (pw < (int)mine) x = items[blockIdx.x + pw * gridDim.x];
         for (uint32_t j = pw; j < mine; j += NPI) {
             ItemX xn;
@@ -709,7 +715,11 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
                 // batch is scanned and issued (items of heavy partitions have
                 // hundreds of runs: one load latency per batch otherwise)
                 uint32_t en0 = 0, en1 = 0;
-                if (PROBE_EPF && lane < np) en0 = E0[sd.k0 + lane], en1 = E1[sd.k0 + lane];
+                if (PROBE_EPF2 && xpf) {  // loaded during the previous item (one relation per warp)
+                    en0 = pf0, en1 = pf1;
+                } else if (PROBE_EPF && lane < np) {
+                    en0 = E0[sd.k0 + lane], en1 = E1[sd.k0 + lane];
+                }
                 for (uint32_t m0 = 0; m0 < np; m0 += 32) {
                     const uint32_t m = m0 + lane;
                     uint32_t sz = 0, pad = 0xffffffffu;
@@ -805,6 +815,19 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
                 copied_small = false;
             }
             if (lane == 0) mbar_arrive(&full[s]);
+            // first batch of this warp's run offsets of its next item, loaded now
+            xpf = false;
+            if (PROBE_EPF2 && !bal && rel1 == rel0 + 1 && j + NPI < mine) {
+                const int rel = rel0;
+                const Side sd = rel ? xn.it.s : xn.it.r;
+                const uint32_t xcb = rel ? xn.cb[1] : xn.cb[0], xnch = rel ? xn.nch[1] : xn.nch[0];
+                const uint16_t *E0 = (rel ? c.eoff[1] : c.eoff[0]) + (size_t)(Q + 1) * xcb + (size_t)xn.it.q * xnch;
+                const uint32_t kend = min(sd.k1, xnch - 1);
+                const uint32_t np = sd.k0 <= kend ? kend - sd.k0 + 1 : 0;
+                pf0 = pf1 = 0;
+                if (lane < np) pf0 = E0[sd.k0 + lane], pf1 = E0[xnch + sd.k0 + lane];
+                xpf = true;
+            }
             x = xn;
         }
         return;

@@ -46,7 +46,8 @@ def test_strerror(mgj):
 
 @pytest.mark.parametrize("bad", [dict(key_bytes=3), dict(world_size=0), dict(world_size=9), dict(rank=2, world_size=2),
                                  dict(radix_bits_global=13), dict(radix_bits_local=12), dict(r_capacity=1 << 32),
-                                 dict(local_split_bits=7), dict(local_split_bits=-2)])
+                                 dict(local_split_bits=7), dict(local_split_bits=-2), dict(skew_bcast=2),
+                                 dict(skew_bcast=-2)])
 def test_invalid_config_rejected_without_gpu(mgj, bad):
     kw = dict(r_capacity=1024, s_capacity=1024)
     kw.update(bad)

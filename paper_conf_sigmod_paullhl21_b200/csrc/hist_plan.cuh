@@ -8,6 +8,9 @@
 
 namespace mgj {
 
+#ifndef HIST_FOLD16
+#define HIST_FOLD16 1  // 4-byte keys: fold four bins per thread with 16-byte accesses (P >= 4)
+#endif
 constexpr int HIST_NB = 3;  // k_hist: TMA ring depth (sub-tiles in flight per CTA; 2 CTAs per SM)
 
 // ---------------------------------------------------------------------------
@@ -108,6 +111,26 @@ __global__ void __launch_bounds__(HIST_THREADS, 2) k_hist(Ctx c) {
         uint32_t *o32 = reinterpret_cast<uint32_t *>(c.sub_hist + (((size_t)rel * c.G + tile) * c.sub_ns + j) * P);
         if constexpr (sizeof(K) == 4) {  // 8-byte shared accesses, pairs of bins (measured: M2 0.83 -> 0.78 ms;
                                          // slower for 8-byte keys, 0.71 -> 0.75, which keep the scalar fold)
+#if HIST_FOLD16
+            for (int q = tid; q < P / 4; q += blockDim.x) {  // 16-byte accesses, four bins (P >= 4 below)
+                const uint4 x = reinterpret_cast<const uint4 *>(sub)[q];
+                reinterpret_cast<uint2 *>(o32)[q] = make_uint2(x.x | x.y << 16, x.z | x.w << 16);
+                uint4 a = reinterpret_cast<const uint4 *>(acc)[q];
+                a.x += x.x;
+                a.y += x.y;
+                a.z += x.z;
+                a.w += x.w;
+                reinterpret_cast<uint4 *>(acc)[q] = a;
+                reinterpret_cast<uint4 *>(sub)[q] = make_uint4(0u, 0u, 0u, 0u);
+            }
+            if (P < 4 && tid < P / 2) {  // P = 2
+                const uint32_t x0 = sub[0], x1 = sub[1];
+                o32[0] = x0 | x1 << 16;
+                acc[0] += x0;
+                acc[1] += x1;
+                sub[0] = sub[1] = 0;
+            }
+#else
             for (int q = tid; q < P / 2; q += blockDim.x) {
                 const uint2 x = reinterpret_cast<const uint2 *>(sub)[q];
                 o32[q] = x.x | x.y << 16;
@@ -117,6 +140,7 @@ __global__ void __launch_bounds__(HIST_THREADS, 2) k_hist(Ctx c) {
                 reinterpret_cast<uint2 *>(acc)[q] = a;
                 reinterpret_cast<uint2 *>(sub)[q] = make_uint2(0u, 0u);
             }
+#endif
         } else {
             for (int q = tid; q < P / 2; q += blockDim.x) {
                 const uint32_t x0 = sub[2 * q], x1 = sub[2 * q + 1];

@@ -368,6 +368,10 @@ def main():
             "unit": "GB/s", "frac": phase_report[dom]["gbs"] / hbm_peak, "traffic": traffic,
             "peak_source": peak_src,
             "alg_bytes_per_launch": phase_report[dom]["alg_bytes"]}
+    if kern[dom] == "k_scatter":
+        # measured: with its stores redirected into L2 the scatter runs at the same
+        # speed, so below the HBM roofline it is limited by the SM's shared-memory pipe
+        roof["limiter"] = "shared-memory pipe (ranking atomics, random 8-byte stores), not DRAM"
 
     sm_mhz = (clocks or {}).get("sm_mhz") or float(peaks.get("sm_max_mhz", 1965.0))
     nsm = torch.cuda.get_device_properties(dev).multi_processor_count

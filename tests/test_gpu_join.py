@@ -563,6 +563,18 @@ def test_error_paths(mgj):
         j.result()
     assert e.value.status == -6
     j.close()
+    # materialised output larger than out_capacity: sticky ECAPACITY, nothing written past it
+    j = mgj.Join(mgj.make_config(r_capacity=n, s_capacity=n, materialize=True, out_capacity=100))
+    j.partition(dev(d["r_keys"]), dev(d["r_pays"]), dev(d["s_keys"]), dev(d["s_pays"]))
+    j.shuffle()
+    j.join()
+    with pytest.raises(mgj.MGJError) as e:
+        j.result()
+    assert e.value.status == -6
+    r = j.result(check=False)
+    assert r["match_count"] == n  # count and checksum do not depend on the output buffer
+    assert r["n_materialized"] <= 100
+    j.close()
 
 
 # ------------------------------------------------------------ full size (bench config)

@@ -42,6 +42,9 @@ namespace mgj {
 #ifndef SCAT_ALIAS
 #define SCAT_ALIAS 0  // 4-byte keys, P <= 1024: two 512-thread CTAs per SM, stage aliased into the sorted buffer (measured: 6.2 vs 4.1 ms)
 #endif
+#ifndef SCAT_PROF
+#define SCAT_PROF 0  // DIAGNOSTIC: thread 0 and 512 of CTA 0 print clock64 time per phase
+#endif
 #ifndef SCAT_RING
 #define SCAT_RING 0  // EXPERIMENT ONLY (wrong results): full-group stores land modulo SCAT_RING bytes of the arena (L2-resident)
 #endif
@@ -400,13 +403,25 @@ __global__ void __launch_bounds__(NT, NT <= 512 ? 2 : 1) k_scatter(Ctx c) {
         issue(0);
     }
     int cur_rel = -1;
+    unsigned long long pt[7] = {0, 0, 0, 0, 0, 0, 0};
+    long long pc = clock64();
+    auto PT = [&](int i) {
+        if (SCAT_PROF) {
+            const long long n = clock64();
+            pt[i] += (unsigned long long)(n - pc);
+            pc = n;
+        }
+    };
     for (uint32_t g = 0; g < ntot; ++g) {
         int rel;
         uint64_t first;
         uint32_t len;
         subtile(g, rel, first, len);
         if (rel != cur_rel) {  // thread-private partition state: no barrier needed
-            if (cur_rel >= 0) flush();
+            if (SCAT_PROF && blockIdx.x == 0 && (tid == 0 || tid == 512))
+        printf("SCATPROF tid %d subtiles %u: top %llu scan %llu layout %llu tmawait %llu read+S1 %llu rank+S2 %llu writeout %llu\n",
+               tid, ntot, pt[0], pt[1], pt[2], pt[3], pt[4], pt[5], pt[6]);
+    if (cur_rel >= 0) flush();
             set_base(rel);
             cur_rel = rel;
         }
@@ -421,8 +436,10 @@ __global__ void __launch_bounds__(NT, NT <= 512 ? 2 : 1) k_scatter(Ctx c) {
         }
         load_counts(g + 1, ncnt);  // prefetch (consumed next iteration)
         uint32_t total;
+        PT(0);  // carries fetched, counts: top of the sub-tile
         uint32_t o = SCAT_SCAN1 ? block_scan_reg1(tsum, tmp, total)   // its barrier: last write-out is done
                                 : block_scan_reg(tsum, tmp, total);
+        PT(1);  // layout scan (its barriers wait for the last write-out)
         uint32_t co[PPT], ccw[PPT];  // segment start and carried count (for the ALIAS carry write)
 #pragma unroll
         for (int k = 0; k < PPT; ++k) ccw[k] = cc[k], co[k] = 0;
@@ -457,6 +474,7 @@ __global__ void __launch_bounds__(NT, NT <= 512 ? 2 : 1) k_scatter(Ctx c) {
             o += seg[k];
         }
         pending = SG > 1;
+        PT(2);  // layout: carries, descriptors
         K kk[V], pp[V];
         if constexpr (LDG) {
 #pragma unroll
@@ -464,6 +482,7 @@ __global__ void __launch_bounds__(NT, NT <= 512 ? 2 : 1) k_scatter(Ctx c) {
             if (g + 1 < ntot) fetch(g + 1);
         } else {
         mbar_wait(&bar, g & 1);
+        PT(3);  // TMA wait
         const uint32_t body = len & ~(uint32_t)(LU - 1);
         const K *gk = static_cast<const K *>(c.in_key[rel]) + first;
         const K *gp = static_cast<const K *>(c.in_pay[rel]) + first;
@@ -489,6 +508,7 @@ __global__ void __launch_bounds__(NT, NT <= 512 ? 2 : 1) k_scatter(Ctx c) {
         }
         }
         __syncthreads();  // S1: offsets and carries in place, stage consumed
+        PT(4);  // stage read + S1
         if (ALIAS) {  // the stage region is free now: carries to their segment heads
 #pragma unroll
             for (int k = 0; k < PPT; ++k)
@@ -527,6 +547,7 @@ __global__ void __launch_bounds__(NT, NT <= 512 ? 2 : 1) k_scatter(Ctx c) {
         }
 #endif
         __syncthreads();  // S2
+        PT(5);  // rank + scatter into sorted + S2
         if (ALIAS) fetch_carry();  // before the stage region is reloaded
         // write-out, two groups per thread per step (independent load chains)
         const uint32_t ngroups = total / SG;
@@ -602,6 +623,7 @@ __global__ void __launch_bounds__(NT, NT <= 512 ? 2 : 1) k_scatter(Ctx c) {
             }
             }
         }
+        PT(6);  // write-out
         if (ALIAS) {  // the sorted buffer is read: load the next sub-tile into its head
             __syncthreads();  // S3
             if (tid == 0 && g + 1 < ntot) issue(g + 1);

@@ -462,7 +462,7 @@ def check_bcast_virtual(mgj, w, N, skew, materialize=True, expect_bc=True, **kw)
     return nbc
 
 
-@pytest.mark.parametrize("N,skew", [(2, 0), (4, 0), (8, 0), (4, 1), (8, 1), (4, -1)])
+@pytest.mark.parametrize("N,skew", [(2, 0), (3, 0), (4, 0), (6, 1), (8, 0), (4, 1), (8, 1), (4, -1)])
 def test_virtual_ranks_bcast_zipf(mgj, N, skew):
     """Zipf S (z = 1, |R|:|S| = 1:4, half the S rows match): heavy partitions broadcast."""
     w = datagen.Workload("zipf", 1 << 16, 1 << 18, 1.0)

@@ -23,7 +23,7 @@ __host__ __device__ constexpr int local_vmax(int tuple_bytes) { return LOCAL_VMA
 constexpr int PROBE_THREADS = 1024;     // warps 0..PROBE_NP-1 = TMA producers, the rest build/probe
 constexpr int PROBE_NST = 3;            // pipeline stages (items in flight per CTA)
 #ifndef PROBE_PPI
-#define PROBE_PPI 2                     // producer warps per item (1: R and S; 2: one relation each)
+#define PROBE_PPI 2                     // producer warps per item (1: R and S; 2: one relation each; 4: two each)
 #endif
 constexpr int PROBE_NP = PROBE_NST * PROBE_PPI;  // producer warps (item streams <= PROBE_NST: parity waits one phase ahead)
 constexpr int PROBE_SLOTS8 = 4224;      // stage capacity per relation (slots) for 8-byte tuples; half for 16-byte

@@ -664,10 +664,14 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
         // ------------------------------------------------------- producers
         constexpr int ALIGN = Layout<K>::ALIGN;
         const uint64_t pol = policy_evict_first();
-        // PROBE_PPI producer warps per item: 1 (both relations) or 2 (R / S)
+        // PROBE_PPI producer warps per item: 1 (both relations), 2 (R / S) or 4
+        // (two per relation, each issuing every other run: one warp's bulk
+        // copies issue one after another, so the copies of 768-byte runs are
+        // issue-bound with one warp per relation; tools/tma_runs.cu)
         constexpr int NPI = PROBE_NP / PROBE_PPI;  // item streams (<= PROBE_NST)
         const int pw = warp / PROBE_PPI;
-        const int rel0 = PROBE_PPI == 2 ? (warp & 1) : 0, rel1 = PROBE_PPI == 2 ? rel0 + 1 : 2;
+        const int rel0 = PROBE_PPI >= 2 ? (warp & 1) : 0, rel1 = PROBE_PPI >= 2 ? rel0 + 1 : 2;
+        const int sub = PROBE_PPI == 4 ? ((warp >> 1) & 1) : 0;  // which half of the relation's runs
         ItemX x;
         bool copied_small = false;  // this lane stored small runs into the stage (PROBE_SMALL)
         bool xpf = false;           // pf0/pf1 hold the first batch of run offsets of item x (PROBE_EPF2)
@@ -679,7 +683,7 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
             const int s = j % PROBE_NST;
             if (j >= PROBE_NST) mbar_wait(&empty[s], ((j / PROBE_NST) - 1) & 1);
             uint32_t *pb = padbits + s * PW;
-            if (SBITS && rel1 == 2) {
+            if (SBITS && rel1 == 2 && sub == 0) {
                 for (int w = lane; w < PW; w += 32) pb[w] = 0;
                 __syncwarp();
             }
@@ -747,12 +751,15 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
                     }
                     const uint32_t dst = run + incl - sz;
                     const uint32_t gsum = __shfl_sync(0xffffffffu, incl, 31);
-                    const bool issue_it = !bal || (gbase + m >= glo && gbase + m < ghi);
+                    const bool issue_it = (!bal || (gbase + m >= glo && gbase + m < ghi)) &&
+                                          (PROBE_PPI != 4 || (SBITS ? sub == 0 : (m & 1u) == (uint32_t)sub));
                     // runs of at most PROBE_SMALL tuples are copied by their lane with
                     // plain loads/stores (a heavy partition leaves most co-partitions
                     // in runs of a few tuples: one bulk copy each would dominate)
                     const bool small = PROBE_SMALL && sz != 0 && sz <= PROBE_SMALL && issue_it;
-                    const uint32_t gmine = (bal || PROBE_SMALL) ? __reduce_add_sync(0xffffffffu, (issue_it && !small) ? sz : 0u) : gsum;
+                    const uint32_t gmine = (bal || PROBE_SMALL || PROBE_PPI == 4)
+                                               ? __reduce_add_sync(0xffffffffu, (issue_it && !small) ? sz : 0u)
+                                               : gsum;
                     if (PROBE_CPASYNC) {
                         // the warp copies the batch's runs one after another, 16 bytes per lane
                         constexpr uint32_t PT = 16 / TB;  // tuples per 16-byte piece
@@ -782,7 +789,7 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
                     if (pad != 0xffffffffu) atomicOr(&pb[(dst + pad) >> 5], 1u << ((dst + pad) & 31));
                     run += gsum;
                 }
-                if (lane == 0 && (!bal || (warp & 1) == rel)) totals[s][rel] = run;
+                if (lane == 0 && (!bal || (warp & 1) == rel) && sub == 0) totals[s][rel] = run;
                 if (PROBE_L2PF && j + PROBE_L2PF * NPI < mine) {
                     // the same side of the item PROBE_L2PF rounds ahead: its runs -> L2, so that
                     // its stage loads hit L2 (more bytes in flight than the stages can hold)
@@ -803,7 +810,7 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
                     }
                 }
             }
-            if (lane == 0 && rel0 == 0) {
+            if (lane == 0 && rel0 == 0 && sub == 0) {
                 stage_p[s] = (uint32_t)c.plist[BAp ? x.it.pi >> BAp : x.it.pi];
                 stage_soff[s] = x.soff;
             }

@@ -253,30 +253,12 @@ def main():
                           recv_capacity_s=(n_s // 2 if world > 1 and a.workload == "zipf" else 0),
                           shuffle_mode=(mgj.SHUFFLE_EXTERNAL if a.shuffle == "nccl" else mgj.SHUFFLE_P2P),
                           skew_bcast=a.skew_bcast)
-    arena = None
-    if distributed:
-        import torch.distributed._symmetric_memory as symm_mem
-        nbytes = mgj.arena_bytes(cfg)
-        arena = symm_mem.empty(nbytes, dtype=torch.uint8, device=dev)
-        arena.zero_()
-        hdl = symm_mem.rendezvous(arena, dist.group.WORLD)
-        ptrs = [int(p) for p in hdl.buffer_ptrs]
-        torch.cuda.synchronize()
-        dist.barrier()
-        join = mgj.Join(cfg, ptrs, nbytes)
-    else:
-        join = mgj.Join(cfg)
+    # N>1 (or MGJ_SYMM_ARENA=1): the library's symmetric-memory setup (mgj.symmetric_join)
+    join = mgj.symmetric_join(cfg) if distributed else mgj.Join(cfg)
 
     def nccl_exchange():
         """Baseline shuffle: NCCL all_to_all_single of the per-destination send buffers."""
-        lay = join.exchange_layout()  # synchronises the stream (sizes are computed on the device)
-        tb_ = lay["tuple_bytes"]
-        with torch.cuda.stream(stream):
-            for rel in range(2):
-                sc, rc = lay["send_count"][rel], lay["recv_count"][rel]
-                send = mgj.device_bytes(lay["send"][rel], sum(sc) * tb_)
-                recv = mgj.device_bytes(lay["recv"][rel], sum(rc) * tb_)
-                dist.all_to_all_single(recv, send, [x * tb_ for x in rc], [x * tb_ for x in sc])
+        mgj.nccl_exchange(join, stream)
 
     def step(inputs=None):
         join.partition(*(cols if inputs is None else inputs), stream=stream)

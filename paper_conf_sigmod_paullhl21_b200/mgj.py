@@ -234,6 +234,50 @@ class Join:
             pass
 
 
+def symmetric_join(cfg: Config, group=None):
+    """One rank's Join over a torch symmetric-memory arena (one process per GPU).
+
+    Allocates this rank's arena with torch.distributed._symmetric_memory (size
+    mgj_arena_bytes), zero-fills it, exchanges the peer mappings (rendezvous) and
+    barriers, as mgj_peers requires; the process group must be initialised
+    (NCCL) and cfg.rank / cfg.world_size must match it.  The arena tensor is kept
+    on the returned handle (`.arena`) so it outlives the join.  Memory plumbing
+    only: the exchange itself is the library's in-kernel peer stores."""
+    import torch
+    import torch.distributed as dist
+    import torch.distributed._symmetric_memory as symm_mem
+    group = group or dist.group.WORLD
+    nbytes = arena_bytes(cfg)
+    if nbytes == 0:
+        raise MGJError(-1, "mgj_arena_bytes")
+    arena = symm_mem.empty(nbytes, dtype=torch.uint8, device=torch.device("cuda", torch.cuda.current_device()))
+    arena.zero_()
+    hdl = symm_mem.rendezvous(arena, group)
+    ptrs = [int(p) for p in hdl.buffer_ptrs]
+    torch.cuda.synchronize()
+    dist.barrier(group)
+    j = Join(cfg, ptrs, nbytes)
+    j.arena, j._symm = arena, hdl
+    return j
+
+
+def nccl_exchange(join: "Join", stream=None, group=None):
+    """MGJ_SHUFFLE_EXTERNAL baseline: all_to_all_single (NCCL) of the per-destination send
+    buffers into this rank's receive areas, between join.shuffle() and join.join().
+    Synchronises the stream once (the split sizes are computed on the device)."""
+    import torch
+    import torch.distributed as dist
+    lay = join.exchange_layout()
+    tb = lay["tuple_bytes"]
+    ctx = torch.cuda.stream(stream) if stream is not None else torch.cuda.stream(torch.cuda.current_stream())
+    with ctx:
+        for rel in range(2):
+            sc, rc = lay["send_count"][rel], lay["recv_count"][rel]
+            send = device_bytes(lay["send"][rel], sum(sc) * tb)
+            recv = device_bytes(lay["recv"][rel], sum(rc) * tb)
+            dist.all_to_all_single(recv, send, [x * tb for x in rc], [x * tb for x in sc], group=group)
+
+
 class _DevBuf:
     """Byte view of a raw device pointer for torch.as_tensor (__cuda_array_interface__)."""
 

@@ -732,3 +732,24 @@ def test_external_shuffle_virtual_ranks(mgj, N, kind, ba):
         assert (r["match_count"], r["checksum"]) == (ref["count"], ref["checksum"])
     for j in joins:
         j.close()
+
+
+# ------------------------------------------------------------ torchrun + symmetric memory
+@pytest.mark.parametrize("mode", ["p2p", "nccl"])
+def test_torchrun_symmetric_memory_path(mgj, mode):
+    """bench.py under torchrun with MGJ_SYMM_ARENA=1: the real torch symmetric-memory
+    arena (mgj.symmetric_join: symm_mem.empty + rendezvous) and, for mode nccl, the
+    EXTERNAL shuffle with NCCL all_to_all_single (mgj.nccl_exchange), at N = 1."""
+    import json
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    env = dict(os.environ, MGJ_SYMM_ARENA="1")
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "1",
+           "--master-addr", "127.0.0.1", "--master-port", str(29600 + (mode == "nccl")), "bench.py", "--gpus", "1",
+           "--steps", "2", "--warmup", "3", "--no-cpu-baseline", "--no-e2e", "--log2-per-gpu", "22", "--shuffle", mode]
+    out = subprocess.run(cmd, cwd=root, env=env, capture_output=True, text=True, timeout=600)
+    assert out.returncode == 0, out.stderr[-2000:]
+    line = json.loads(out.stdout.strip().splitlines()[-1])
+    assert line["correct"] and line["match_count"] == 1 << 22

@@ -216,7 +216,7 @@ __global__ void __launch_bounds__(1024) k_planA(Ctx c) {
     const int L = c.meta[MT_NP] << BA;
     const int tid = threadIdx.x;
     uint32_t *nch = reinterpret_cast<uint32_t *>(sv + L + 1);
-    const uint64_t C = (uint64_t)c.chunk_tuples;
+    const uint64_t C = (uint64_t)c.chunk_tuples2;  // the chunked pass after the first pass
     uint32_t tot_ch[2];
     bool bad = false;
     for (int rel = 0; rel < 2; ++rel) {
@@ -254,7 +254,7 @@ __global__ void k_chunkmapB(Ctx c, ChunkDesc *desc) {
     if (!c.meta[MT_OK] || !c.meta[MT_BA]) return;
     const int L = c.meta[MT_NLP];
     const uint32_t nch_r = (uint32_t)c.meta[MT_NCHB_R], total = nch_r + (uint32_t)c.meta[MT_NCHB_S];
-    const uint64_t C = (uint64_t)c.chunk_tuples;
+    const uint64_t C = (uint64_t)c.chunk_tuples2;  // the chunked pass after the first pass
     for (uint32_t ci = blockIdx.x * blockDim.x + threadIdx.x; ci < total; ci += gridDim.x * blockDim.x) {
         const int rel = ci < nch_r ? 0 : 1;
         const uint32_t li = rel ? ci - nch_r : ci;
@@ -313,15 +313,18 @@ __global__ void __launch_bounds__(LOCAL_THREADS, 1) k_local(Ctx c, const ChunkDe
     const int BA = MODE == LM_SINGLE ? 0 : c.meta[MT_BA];
     if ((MODE == LM_SINGLE) != (c.meta[MT_BA] == 0)) return;
     const int tid = threadIdx.x;
-    const int C = c.chunk_tuples, CR = c.chunk_region, V = C / LOCAL_THREADS;
+    // LM_SECOND has its own chunk geometry (fan-out <= 2^(b2_max - 1): larger chunks fit)
+    const int C = MODE == LM_SECOND ? c.chunk_tuples2 : c.chunk_tuples;
+    const int CR = MODE == LM_SECOND ? c.chunk_region2 : c.chunk_region, V = C / LOCAL_THREADS;
     const int P = c.P, Q = 1 << (SPLIT ? BA : c.meta[MT_QB]);
     const int shift = SPLIT ? c.B1 : c.B1 + BA;  // digit = (key >> shift) & (Q - 1)
-    const int Qmax = 1 << c.b2_max;
-    const int BUF = C + Qmax + 2;  // slots per buffer
+    const int Qmax = 1 << c.b2_max;  // stride of the co-partition size table
+    const int QL = MODE == LM_SECOND ? 1 << c.qm2_bits : Qmax;  // bins / padding in shared memory
+    const int BUF = C + QL + 2;  // slots per buffer
     Tup *const buf0 = reinterpret_cast<Tup *>(smem);
     auto buf = [&](int x) { return buf0 + (size_t)x * BUF; };
-    uint32_t *const bins2 = reinterpret_cast<uint32_t *>(buf0 + (size_t)2 * BUF);  // [2][Qmax], chunk j uses j & 1
-    uint32_t *const abin = bins2 + 2 * Qmax;
+    uint32_t *const bins2 = reinterpret_cast<uint32_t *>(buf0 + (size_t)2 * BUF);  // [2][QL], chunk j uses j & 1
+    uint32_t *const abin = bins2 + 2 * QL;
     const uint32_t nch_r = SPLIT ? (uint32_t)c.meta[MT_NCH_R] : nch_local(c, 0);
     const uint32_t total = nch_r + (SPLIT ? (uint32_t)c.meta[MT_NCH_S] : nch_local(c, 1));
     const uint32_t mine = total > blockIdx.x ? (total - blockIdx.x + gridDim.x - 1) / gridDim.x : 0;
@@ -337,7 +340,7 @@ __global__ void __launch_bounds__(LOCAL_THREADS, 1) k_local(Ctx c, const ChunkDe
         mbar_init(&bar[1], 1);
         fence_mbar_init();
     }
-    for (int q = tid; q < 2 * Qmax; q += LOCAL_THREADS) bins2[q] = 0;
+    for (int q = tid; q < 2 * QL; q += LOCAL_THREADS) bins2[q] = 0;
     __syncthreads();
     const uint64_t pol = policy_evict_first();
     // thread 0: TMA chunk j (16-byte-aligned superset) into buffer j & 1
@@ -364,7 +367,7 @@ __global__ void __launch_bounds__(LOCAL_THREADS, 1) k_local(Ctx c, const ChunkDe
         const int rel = ci < nch_r ? 0 : 1;
         const uint32_t li = rel ? ci - nch_r : ci;
         const int X = j & 1;
-        uint32_t *const bins = bins2 + X * Qmax;  // zero (cleared during chunk j - 1)
+        uint32_t *const bins = bins2 + X * QL;  // zero (cleared during chunk j - 1)
         mbar_wait(&bar[X], (j >> 1) & 1);
         const ChunkDesc d = sdesc[X];
         const uint32_t len = d.len, skip = (uint32_t)(d.start & (ALIGN - 1));
@@ -396,7 +399,7 @@ __global__ void __launch_bounds__(LOCAL_THREADS, 1) k_local(Ctx c, const ChunkDe
             if (j + 2 < mine) nxt = cdesc[blockIdx.x + (j + 2) * gridDim.x];
         }
         if (tid >= 32) {  // the other bin array (last read by chunk j-1 before its S3) for chunk j+1
-            uint32_t *const bn = bins2 + (X ^ 1) * Qmax;
+            uint32_t *const bn = bins2 + (X ^ 1) * QL;
             for (int q = tid - 32; q < Q; q += LOCAL_THREADS - 32) bn[q] = 0;
         }
         if (tid < 32) {  // one warp: padded run starts (exclusive scan over the Q bins)
@@ -739,7 +742,7 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
                         const uint32_t ahi = (k == sd.k1) ? sd.a1 : slots;
                         if (ahi > alo) {
                             sz = ahi - alo;
-                            src = (uint64_t)(LP_RING ? (xcb + k) % LP_RING : xcb + k) * c.chunk_region + st + alo;
+                            src = (uint64_t)(LP_RING ? (xcb + k) % LP_RING : xcb + k) * (BAp ? c.chunk_region2 : c.chunk_region) + st + alo;
                         }
                         pad = (SBITS && rel == 1 && v < slots && v >= alo && v < ahi) ? v - alo : 0xffffffffu;
                     }

@@ -27,6 +27,7 @@ uint64_t align_up(uint64_t x, uint64_t a) { return (x + a - 1) / a * a; }
 struct Norm {  // validated config with the automatic fields filled in
     mgj_config c;
     int B1, P, b2_max, tuple_bytes, chunk_tuples, chunk_region, probe_slots, probe_target;
+    int chunk_tuples2, chunk_region2, qm2_bits;
     uint64_t recv_cap[2], max_chunks, max_items, out_cap, mid_cap;
     bool split;  // first local pass possible (mid buffers allocated)
     Arena lay;
@@ -84,6 +85,14 @@ mgj_status normalize(const mgj_config *in, Norm *o) {
     if (!C) return MGJ_EINVAL;
     o->chunk_tuples = C;
     o->chunk_region = C + Qm;  // worst-case padding: one slot per run
+    // the chunked pass after a first pass (BA >= 1) has fan-out <= 2^(b2_max - 1)
+    o->qm2_bits = std::max(1, o->b2_max - 1);
+    int C2 = 0;
+    for (int v = local_vmax(o->tuple_bytes); v >= 1 && !C2; --v)
+        if (local_smem_bytes(v * LOCAL_THREADS, 1 << o->qm2_bits, o->tuple_bytes) <= 225 * 1024) C2 = v * LOCAL_THREADS;
+    if (C2 < C) C2 = C;
+    o->chunk_tuples2 = C2;
+    o->chunk_region2 = C2 + (1 << o->qm2_bits);
     const uint64_t rmax = std::max(o->recv_cap[0], o->recv_cap[1]);
     // chunks of the chunked pass: sum over (sub-)partitions of ceil(size / C); at most
     // local2_vcap(P) sub-partitions after a first pass
@@ -167,6 +176,7 @@ size_t plan_smem(const Norm &n) { return (size_t)n.P * 5 * 8 + (size_t)n.P * 4 +
 size_t scatter_smem(const Norm &n) { return scat_smem_bytes(n.P, n.c.key_bytes); }
 size_t planA_smem(const Norm &n) { return ((size_t)local2_vcap(n.P) + 1) * 12; }
 size_t local_smem(const Norm &n) { return local_smem_bytes(n.chunk_tuples, 1 << n.b2_max, n.tuple_bytes); }
+size_t local_smem2(const Norm &n) { return local_smem_bytes(n.chunk_tuples2, 1 << n.qm2_bits, n.tuple_bytes); }
 size_t probe_smem(const Norm &n) { return probe_smem_bytes(n.probe_slots, n.tuple_bytes); }
 
 template <typename K>
@@ -178,7 +188,7 @@ cudaError_t set_attrs(const Norm &n) {
     if ((e = cudaFuncSetAttribute(scatter_kernel<K>(n.P), A, (int)scatter_smem(n)))) return e;
     if ((e = cudaFuncSetAttribute(k_local<K, LM_SINGLE>, A, (int)local_smem(n)))) return e;
     if ((e = cudaFuncSetAttribute(k_local<K, LM_SPLIT>, A, (int)local_smem(n)))) return e;
-    if ((e = cudaFuncSetAttribute(k_local<K, LM_SECOND>, A, (int)local_smem(n)))) return e;
+    if ((e = cudaFuncSetAttribute(k_local<K, LM_SECOND>, A, (int)local_smem2(n)))) return e;
     if ((e = cudaFuncSetAttribute(k_planA, A, (int)planA_smem(n)))) return e;
     if ((e = cudaFuncSetAttribute(k_probe<K, false>, A, (int)probe_smem(n)))) return e;
     return cudaFuncSetAttribute(k_probe<K, true>, A, (int)probe_smem(n));
@@ -227,7 +237,7 @@ void launch_join(mgj_plan_s *h, cudaStream_t s) {
         k_planA<<<1, 1024, planA_smem(n), s>>>(h->ctx);
         k_local<K, LM_SPLIT><<<h->nsm, LOCAL_THREADS, local_smem(n), s>>>(h->ctx, h->cdesc);
         k_chunkmapB<<<h->nsm * 2, 256, 0, s>>>(h->ctx, h->cdesc);
-        k_local<K, LM_SECOND><<<h->nsm, LOCAL_THREADS, local_smem(n), s>>>(h->ctx, h->cdesc);
+        k_local<K, LM_SECOND><<<h->nsm, LOCAL_THREADS, local_smem2(n), s>>>(h->ctx, h->cdesc);
         h->launches += 5;
     }
     k_local<K, LM_SINGLE><<<h->nsm, LOCAL_THREADS, local_smem(n), s>>>(h->ctx, h->cdesc);
@@ -324,6 +334,9 @@ mgj_status mgj_plan(const mgj_config *cfg, const mgj_peers *peers, mgj_handle *o
     c.hist_split = G == h->nsm ? 2 : 1;  // k_hist: two CTAs per SM either way
     c.chunk_tuples = n.chunk_tuples;
     c.chunk_region = n.chunk_region;
+    c.chunk_tuples2 = n.chunk_tuples2;
+    c.chunk_region2 = n.chunk_region2;
+    c.qm2_bits = n.qm2_bits;
     c.probe_slots = n.probe_slots;
     c.probe_target = n.probe_target;
     c.materialize = n.c.materialize;
@@ -378,7 +391,8 @@ mgj_status mgj_plan(const mgj_config *cfg, const mgj_peers *peers, mgj_handle *o
     for (int r = 0; r < 2; ++r)
         c.eoff[r] = static_cast<uint16_t *>(dalloc(h, n.max_chunks * (Qm + 1) * 2, &st));
     c.items = static_cast<Item *>(dalloc(h, n.max_items * sizeof(ItemX), &st));
-    for (int r = 0; r < 2; ++r) c.local[r] = dalloc(h, n.max_chunks * n.chunk_region * n.tuple_bytes, &st);
+    for (int r = 0; r < 2; ++r)
+        c.local[r] = dalloc(h, n.max_chunks * std::max(n.chunk_region, n.chunk_region2) * n.tuple_bytes, &st);
     c.result = static_cast<unsigned long long *>(dalloc(h, 64, &st));
     if (n.c.materialize) {
         c.out_key = dalloc(h, n.out_cap * n.c.key_bytes, &st);
@@ -698,11 +712,11 @@ mgj_status mgj_debug_copy(mgj_handle h, int32_t what, void *dst, uint64_t bytes,
             break;
         case MGJ_DBG_LOCAL_R:
             src = c.local[0];
-            size = nchl[0] * n.chunk_region * n.tuple_bytes;
+            size = nchl[0] * (meta[MT_BA] ? n.chunk_region2 : n.chunk_region) * n.tuple_bytes;
             break;
         case MGJ_DBG_LOCAL_S:
             src = c.local[1];
-            size = nchl[1] * n.chunk_region * n.tuple_bytes;
+            size = nchl[1] * (meta[MT_BA] ? n.chunk_region2 : n.chunk_region) * n.tuple_bytes;
             break;
         case MGJ_DBG_META: src = c.meta; size = sizeof(meta); break;
         case MGJ_DBG_CHUNK_OFF_R: src = c.eoff[0]; size = nchl[0] * (Q + 1) * 2; break;

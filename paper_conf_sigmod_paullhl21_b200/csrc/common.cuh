@@ -87,6 +87,7 @@ struct Ctx {
     int32_t chunk_tuples2;        // chunk of the chunked pass after a first pass (its fan-out is at
     int32_t chunk_region2;        //   most 2^(b2_max - 1), so its buffers leave room for larger chunks)
     int32_t qm2_bits;             // log2 of that fan-out bound
+    int32_t chunk_tuples1s;       // chunk of the first (split) pass: fan-out <= 2^MAX_BA
     int32_t probe_slots;          // probe stage capacity per relation (slots)
     int32_t probe_target;         // co-partition size B2 aims at (tuples)
     int32_t materialize;

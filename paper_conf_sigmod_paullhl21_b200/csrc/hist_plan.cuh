@@ -474,37 +474,31 @@ __global__ void __launch_bounds__(1024) k_plan(Ctx c) {
     }
     __syncthreads();
     // chunk table of the local pass: chunk_base[rel][i] = first chunk of owned partition i,
-    // piece_chunk[rel][i][g] = first chunk of piece g inside i
+    // piece_chunk[rel][i][g] = first chunk of piece g inside i (chunks of C tuples)
+    __shared__ int s_ba;
     uint32_t nch[2];
-    for (int rel = 0; rel < 2; ++rel) {
-        const uint32_t *pl = c.piece_len + (size_t)rel * P * MAX_RANKS;
-        uint32_t *pc = c.piece_chunk + (size_t)rel * P * (MAX_RANKS + 1);
-        for (int i = tid; i <= np; i += blockDim.x) {
-            uint32_t t = 0;
-            if (i < np)
-                for (int g = 0; g < MAX_RANKS; ++g) {
-                    pc[(size_t)i * (MAX_RANKS + 1) + g] = t;
-                    t += (uint32_t)((pl[(size_t)i * MAX_RANKS + g] + C - 1) / C);
-                }
-            if (i < np) pc[(size_t)i * (MAX_RANKS + 1) + MAX_RANKS] = t;
-            chn[i] = t;
+    auto chunk_table = [&](uint64_t C) {
+        for (int rel = 0; rel < 2; ++rel) {
+            const uint32_t *pl = c.piece_len + (size_t)rel * P * MAX_RANKS;
+            uint32_t *pc = c.piece_chunk + (size_t)rel * P * (MAX_RANKS + 1);
+            for (int i = tid; i <= np; i += blockDim.x) {
+                uint32_t t = 0;
+                if (i < np)
+                    for (int g = 0; g < MAX_RANKS; ++g) {
+                        pc[(size_t)i * (MAX_RANKS + 1) + g] = t;
+                        t += (uint32_t)((pl[(size_t)i * MAX_RANKS + g] + C - 1) / C);
+                    }
+                if (i < np) pc[(size_t)i * (MAX_RANKS + 1) + MAX_RANKS] = t;
+                chn[i] = t;
+            }
+            __syncthreads();
+            nch[rel] = block_excl_scan_u32(chn, np + 1, tmp32);
+            for (int i = tid; i <= np; i += blockDim.x) c.chunk_base[(size_t)rel * c.cb_stride + i] = chn[i];
+            __syncthreads();
         }
-        __syncthreads();
-        nch[rel] = block_excl_scan_u32(chn, np + 1, tmp32);
-        for (int i = tid; i <= np; i += blockDim.x) c.chunk_base[(size_t)rel * c.cb_stride + i] = chn[i];
-        __syncthreads();
-    }
+    };
+    chunk_table((uint64_t)c.chunk_tuples);
     if (tid == 0) {
-        const bool fits = nch[0] <= c.max_chunks && nch[1] <= c.max_chunks;
-        if (cap_bad || !fits) set_err(c, MGJ_ECAPACITY);
-        c.meta[MT_PLO] = plo;
-        c.meta[MT_PHI] = phi;
-        c.meta[MT_NP] = np;
-        c.meta[MT_NBC] = nbc;
-        c.meta[MT_B2] = B2;
-        c.meta[MT_NCH_R] = (int)nch[0];
-        c.meta[MT_NCH_S] = (int)nch[1];
-        c.meta[MT_CHUNK] = c.chunk_tuples;
         // two-level local partitioning: when the owned
         // partitions span more than LOCAL2_NCH chunks on average, a first
         // histogram-based pass splits every owned partition into 2^BA
@@ -522,6 +516,23 @@ __global__ void __launch_bounds__(1024) k_plan(Ctx c) {
         if (BA > B2) BA = B2;
         if (BA > MAX_BA) BA = MAX_BA;
         if (!c.mid[0] || (np << BA) > c.vcap) BA = 0;
+        s_ba = BA;
+    }
+    __syncthreads();
+    const int BA = s_ba;
+    // the first pass (fan-out <= 2^MAX_BA) reads chunks of its own, larger size
+    if (BA > 0 && c.chunk_tuples1s != c.chunk_tuples) chunk_table((uint64_t)c.chunk_tuples1s);
+    if (tid == 0) {
+        const bool fits = nch[0] <= c.max_chunks && nch[1] <= c.max_chunks;
+        if (cap_bad || !fits) set_err(c, MGJ_ECAPACITY);
+        c.meta[MT_PLO] = plo;
+        c.meta[MT_PHI] = phi;
+        c.meta[MT_NP] = np;
+        c.meta[MT_NBC] = nbc;
+        c.meta[MT_B2] = B2;
+        c.meta[MT_NCH_R] = (int)nch[0];
+        c.meta[MT_NCH_S] = (int)nch[1];
+        c.meta[MT_CHUNK] = BA ? c.chunk_tuples1s : c.chunk_tuples;
         c.meta[MT_BA] = BA;
         c.meta[MT_QB] = B2 - BA;
         c.meta[MT_NLP] = np;

@@ -85,7 +85,7 @@ __global__ void k_chunkmap(Ctx c, ChunkDesc *desc) {
     if (!c.meta[MT_OK]) return;
     const int P = c.P, np = c.meta[MT_NP];
     const uint32_t nch_r = (uint32_t)c.meta[MT_NCH_R], total = nch_r + (uint32_t)c.meta[MT_NCH_S];
-    const uint64_t C = (uint64_t)c.chunk_tuples;
+    const uint64_t C = (uint64_t)(c.meta[MT_BA] ? c.chunk_tuples1s : c.chunk_tuples);  // the table k_plan built
     for (uint32_t ci = blockIdx.x * blockDim.x + threadIdx.x; ci < total; ci += gridDim.x * blockDim.x) {
         const int rel = ci < nch_r ? 0 : 1;
         const uint32_t li = rel ? ci - nch_r : ci;
@@ -314,12 +314,12 @@ __global__ void __launch_bounds__(LOCAL_THREADS, 1) k_local(Ctx c, const ChunkDe
     if ((MODE == LM_SINGLE) != (c.meta[MT_BA] == 0)) return;
     const int tid = threadIdx.x;
     // LM_SECOND has its own chunk geometry (fan-out <= 2^(b2_max - 1): larger chunks fit)
-    const int C = MODE == LM_SECOND ? c.chunk_tuples2 : c.chunk_tuples;
+    const int C = MODE == LM_SECOND ? c.chunk_tuples2 : (SPLIT ? c.chunk_tuples1s : c.chunk_tuples);
     const int CR = MODE == LM_SECOND ? c.chunk_region2 : c.chunk_region, V = C / LOCAL_THREADS;
     const int P = c.P, Q = 1 << (SPLIT ? BA : c.meta[MT_QB]);
     const int shift = SPLIT ? c.B1 : c.B1 + BA;  // digit = (key >> shift) & (Q - 1)
     const int Qmax = 1 << c.b2_max;  // stride of the co-partition size table
-    const int QL = MODE == LM_SECOND ? 1 << c.qm2_bits : Qmax;  // bins / padding in shared memory
+    const int QL = MODE == LM_SECOND ? 1 << c.qm2_bits : (SPLIT ? 1 << MAX_BA : Qmax);  // bins / padding in shared memory
     const int BUF = C + QL + 2;  // slots per buffer
     Tup *const buf0 = reinterpret_cast<Tup *>(smem);
     auto buf = [&](int x) { return buf0 + (size_t)x * BUF; };

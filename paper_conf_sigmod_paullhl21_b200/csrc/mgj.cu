@@ -27,7 +27,7 @@ uint64_t align_up(uint64_t x, uint64_t a) { return (x + a - 1) / a * a; }
 struct Norm {  // validated config with the automatic fields filled in
     mgj_config c;
     int B1, P, b2_max, tuple_bytes, chunk_tuples, chunk_region, probe_slots, probe_target;
-    int chunk_tuples2, chunk_region2, qm2_bits;
+    int chunk_tuples2, chunk_region2, qm2_bits, chunk_tuples1s;
     uint64_t recv_cap[2], max_chunks, max_items, out_cap, mid_cap;
     bool split;  // first local pass possible (mid buffers allocated)
     Arena lay;
@@ -92,6 +92,10 @@ mgj_status normalize(const mgj_config *in, Norm *o) {
         if (local_smem_bytes(v * LOCAL_THREADS, 1 << o->qm2_bits, o->tuple_bytes) <= 225 * 1024) C2 = v * LOCAL_THREADS;
     if (C2 < C) C2 = C;
     o->chunk_tuples2 = C2;
+    int C1s = 0;  // the first (split) pass: fan-out <= 2^MAX_BA
+    for (int v = local_vmax(o->tuple_bytes); v >= 1 && !C1s; --v)
+        if (local_smem_bytes(v * LOCAL_THREADS, 1 << MAX_BA, o->tuple_bytes) <= 225 * 1024) C1s = v * LOCAL_THREADS;
+    o->chunk_tuples1s = std::max(C1s, C);
     o->chunk_region2 = C2 + (1 << o->qm2_bits);
     const uint64_t rmax = std::max(o->recv_cap[0], o->recv_cap[1]);
     // chunks of the chunked pass: sum over (sub-)partitions of ceil(size / C); at most
@@ -177,6 +181,7 @@ size_t scatter_smem(const Norm &n) { return scat_smem_bytes(n.P, n.c.key_bytes);
 size_t planA_smem(const Norm &n) { return ((size_t)local2_vcap(n.P) + 1) * 12; }
 size_t local_smem(const Norm &n) { return local_smem_bytes(n.chunk_tuples, 1 << n.b2_max, n.tuple_bytes); }
 size_t local_smem2(const Norm &n) { return local_smem_bytes(n.chunk_tuples2, 1 << n.qm2_bits, n.tuple_bytes); }
+size_t local_smem1s(const Norm &n) { return local_smem_bytes(n.chunk_tuples1s, 1 << MAX_BA, n.tuple_bytes); }
 size_t probe_smem(const Norm &n) { return probe_smem_bytes(n.probe_slots, n.tuple_bytes); }
 
 template <typename K>
@@ -187,7 +192,7 @@ cudaError_t set_attrs(const Norm &n) {
     if ((e = cudaFuncSetAttribute(k_plan, A, (int)plan_smem(n)))) return e;
     if ((e = cudaFuncSetAttribute(scatter_kernel<K>(n.P), A, (int)scatter_smem(n)))) return e;
     if ((e = cudaFuncSetAttribute(k_local<K, LM_SINGLE>, A, (int)local_smem(n)))) return e;
-    if ((e = cudaFuncSetAttribute(k_local<K, LM_SPLIT>, A, (int)local_smem(n)))) return e;
+    if ((e = cudaFuncSetAttribute(k_local<K, LM_SPLIT>, A, (int)local_smem1s(n)))) return e;
     if ((e = cudaFuncSetAttribute(k_local<K, LM_SECOND>, A, (int)local_smem2(n)))) return e;
     if ((e = cudaFuncSetAttribute(k_planA, A, (int)planA_smem(n)))) return e;
     if ((e = cudaFuncSetAttribute(k_probe<K, false>, A, (int)probe_smem(n)))) return e;
@@ -235,7 +240,7 @@ void launch_join(mgj_plan_s *h, cudaStream_t s) {
     if (n.split) {
         k_countA<K><<<h->nsm * 4, 512, 0, s>>>(h->ctx, h->cdesc);
         k_planA<<<1, 1024, planA_smem(n), s>>>(h->ctx);
-        k_local<K, LM_SPLIT><<<h->nsm, LOCAL_THREADS, local_smem(n), s>>>(h->ctx, h->cdesc);
+        k_local<K, LM_SPLIT><<<h->nsm, LOCAL_THREADS, local_smem1s(n), s>>>(h->ctx, h->cdesc);
         k_chunkmapB<<<h->nsm * 2, 256, 0, s>>>(h->ctx, h->cdesc);
         k_local<K, LM_SECOND><<<h->nsm, LOCAL_THREADS, local_smem2(n), s>>>(h->ctx, h->cdesc);
         h->launches += 5;
@@ -337,6 +342,7 @@ mgj_status mgj_plan(const mgj_config *cfg, const mgj_peers *peers, mgj_handle *o
     c.chunk_tuples2 = n.chunk_tuples2;
     c.chunk_region2 = n.chunk_region2;
     c.qm2_bits = n.qm2_bits;
+    c.chunk_tuples1s = n.chunk_tuples1s;
     c.probe_slots = n.probe_slots;
     c.probe_target = n.probe_target;
     c.materialize = n.c.materialize;

@@ -39,6 +39,10 @@ namespace mgj {
 #define PROBE_BAL 0  // the two producer warps of an item split its R + S runs evenly (measured: M2 probe 2.35 vs 1.96 ms, zipf z=1 2.80 vs 2.85, wide 2.70 vs 2.39)
 #endif
 
+#ifndef PROBE_IDLE
+#define PROBE_IDLE 0  // DIAGNOSTIC: idle warps taken from the consumers (6: probe 2.25 vs 1.96 ms at M2)
+#endif
+
 #ifndef PROBE_U2
 #define PROBE_U2 0  // packed probe: two S slots per step (measured slower: 2.00 vs 1.96 ms)
 #endif
@@ -616,7 +620,8 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
     constexpr int TB = Layout<K>::TB;
     constexpr int LOGT = 12, T = 1 << LOGT;
     constexpr uint16_t END = 0xffff;
-    constexpr int NCONS = PROBE_THREADS - 32 * PROBE_NP;
+    constexpr int NIDLE = PROBE_IDLE;  // EXPERIMENT: warps that do nothing (consumer-count sensitivity)
+    constexpr int NCONS = PROBE_THREADS - 32 * (PROBE_NP + NIDLE);
     extern __shared__ __align__(128) unsigned char smem[];
     __shared__ __align__(8) uint64_t full[PROBE_NST], empty[PROBE_NST];
     __shared__ uint32_t totals[PROBE_NST][2];
@@ -663,6 +668,7 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
     for (int i = tid; i < T; i += PROBE_THREADS) head[i] = 0;
     __syncthreads();
 
+    if (NIDLE && warp >= PROBE_NP && warp < PROBE_NP + NIDLE) return;
     if (warp < PROBE_NP) {
         // ------------------------------------------------------- producers
         constexpr int ALIGN = Layout<K>::ALIGN;
@@ -844,7 +850,7 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
     }
 
     // ------------------------------------------------------------ consumers
-    const int ct = tid - 32 * PROBE_NP;
+    const int ct = tid - 32 * (PROBE_NP + NIDLE);
     unsigned long long my_cnt = 0, my_chk = 0;
     uint32_t tag = 0;
     for (uint32_t j = 0; j < mine; ++j) {

@@ -427,7 +427,6 @@ __global__ void __launch_bounds__(1024) k_plan(Ctx c) {
     // (the whole segment, sources ascending inside it; a broadcast partition's
     // R piece in its root's buffer); EXTERNAL — one piece per source rank g,
     // the receive area being [g0 | g1 | ...], each [owned p ascending]
-    const uint64_t C = (uint64_t)c.chunk_tuples;
     const uint32_t *mine = mail + (size_t)c.rank * 2 * P;
     for (int rel = 0; rel < 2; ++rel) {
         uint64_t *ps = c.piece_start + (size_t)rel * P * MAX_RANKS;

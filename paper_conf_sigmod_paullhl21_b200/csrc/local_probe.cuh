@@ -43,6 +43,10 @@ namespace mgj {
 #define PROBE_IDLE 0  // DIAGNOSTIC: idle warps taken from the consumers (6: probe 2.25 vs 1.96 ms at M2)
 #endif
 
+#ifndef PROBE_SPF
+#define PROBE_SPF 0  // packed probe: next S slot and its head loaded before the current chain walk (measured slower: 2.02 vs 1.96 ms)
+#endif
+
 #ifndef PROBE_U2
 #define PROBE_U2 0  // packed probe: two S slots per step (measured slower: 2.00 vs 1.96 ms)
 #endif
@@ -975,6 +979,35 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
                     my_chk += chk_term(a, (K)sv.y);
                     ovf = true;
                 });
+            }
+        } else if (PROBE_SPF && packed) {
+            // software-pipelined: the next S slot and its head entry are loaded
+            // before the current slot's chain is walked (two fewer dependent
+            // shared-memory round trips on the critical path per slot)
+            uint32_t x = x0;
+            Tup sn{};
+            uint32_t hn = 0;
+            auto fetch = [&](uint32_t xx) {
+                sn = st[xx];
+                hn = head[fold((K)(sn.x >> shift))];
+            };
+            if (x < stot) fetch(x);
+            for (; x < stot; x += NCONS) {
+                const Tup sv = sn;
+                const uint32_t hv = hn;
+                if (x + NCONS < stot) fetch(x + NCONS);
+                const K k = sv.x;
+                if (((uint32_t)k & (uint32_t)(P - 1)) != pitem) continue;  // S padding slot
+                const K khi = k >> shift;
+                for (uint32_t i = (hv >> 16) == tag ? (hv & 0xffffu) : END; i != END;) {
+                    const Tup rv = rt[i];
+                    const K l = rv.x;
+                    if ((l >> 16) == khi) {
+                        ++m_item;
+                        my_chk += chk_term((K)rv.y, (K)sv.y);
+                    }
+                    i = (uint32_t)l & 0xffffu;
+                }
             }
         } else {
             for (uint32_t x = x0; x < stot; x += NCONS) {

@@ -47,6 +47,10 @@ namespace mgj {
 #define PROBE_SPF 0  // packed probe: next S slot and its head loaded before the current chain walk (measured slower: 2.02 vs 1.96 ms)
 #endif
 
+#ifndef PROBE_HOFF
+#define PROBE_HOFF 1  // packed table: head offsets in three instructions
+#endif
+
 #ifndef PROBE_U2
 #define PROBE_U2 0  // packed probe: two S slots per step (measured slower: 2.00 vs 1.96 ms)
 #endif
@@ -877,6 +881,16 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
                 return (f ^ (f >> LOGT) ^ (f >> (2 * LOGT))) & (uint32_t)(T - 1);
             }
         };
+        // head entry of khi: the same index as fold(), computed as a byte offset
+        // in three instructions (shift, shift, xor-and) for 4-byte keys
+        auto hp = [&](K khi) -> uint32_t * {
+            if constexpr (sizeof(K) == 4 && PROBE_HOFF) {
+                const uint32_t off = (((uint32_t)khi << 2) ^ ((uint32_t)khi >> (LOGT - 2))) & (uint32_t)((T - 1) << 2);
+                return reinterpret_cast<uint32_t *>(reinterpret_cast<char *>(head) + off);
+            } else {
+                return head + fold(khi);
+            }
+        };
         // build
         if (packed) {
             K *rw = reinterpret_cast<K *>(stages + (size_t)s * 2 * SL);
@@ -884,7 +898,7 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
                 const K k = rt[slot].x;
                 if (((uint32_t)k & (uint32_t)(P - 1)) != pitem) continue;  // R padding slot
                 const K khi = k >> shift;
-                const uint32_t old = atomicExch(&head[fold(khi)], (tag << 16) | slot);
+                const uint32_t old = atomicExch(hp(khi), (tag << 16) | slot);
                 rw[2 * slot] = (K)((old >> 16) == tag ? (old & 0xffffu) : (uint32_t)END) | (khi << 16);
             }
         } else {
@@ -902,7 +916,7 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
                 const K k = sv.x;
                 if (((uint32_t)k & (uint32_t)(P - 1)) != pitem) return;  // S padding slot
                 const K khi = k >> shift;
-                const uint32_t hv = head[fold(khi)];
+                const uint32_t hv = *hp(khi);
                 for (uint32_t i = (hv >> 16) == tag ? (hv & 0xffffu) : END; i != END;) {
                     const Tup rv = rt[i];
                     const K l = rv.x;
@@ -1085,7 +1099,7 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
                             const K k = sv.x;
                             if (((uint32_t)k & (uint32_t)(P - 1)) == pitem) {
                                 khi = k >> shift;
-                                const uint32_t hv = head[fold(khi)];
+                                const uint32_t hv = *hp(khi);
                                 i = (hv >> 16) == tag ? (hv & 0xffffu) : END;
                             }
                         } else if (!(SBITS && ((pb[x >> 5] >> (x & 31)) & 1u))) {

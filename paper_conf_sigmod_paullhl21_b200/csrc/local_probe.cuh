@@ -51,6 +51,10 @@ namespace mgj {
 #define PROBE_HOFF 1  // packed table: head offsets in three instructions
 #endif
 
+#ifndef PROBE_TAGX
+#define PROBE_TAGX 1  // packed table: tag test by xor (one compare instead of shift, mask, two compares)
+#endif
+
 #ifndef PROBE_U2
 #define PROBE_U2 0  // packed probe: two S slots per step (measured slower: 2.00 vs 1.96 ms)
 #endif
@@ -899,7 +903,10 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
                 if (((uint32_t)k & (uint32_t)(P - 1)) != pitem) continue;  // R padding slot
                 const K khi = k >> shift;
                 const uint32_t old = atomicExch(hp(khi), (tag << 16) | slot);
-                rw[2 * slot] = (K)((old >> 16) == tag ? (old & 0xffffu) : (uint32_t)END) | (khi << 16);
+                const uint32_t ox = old ^ (tag << 16);  // < 2^16: a slot of this item
+                rw[2 * slot] = (K)(PROBE_TAGX ? (ox < 0x10000u ? ox : (uint32_t)END)
+                                              : ((old >> 16) == tag ? (old & 0xffffu) : (uint32_t)END)) |
+                               (khi << 16);
             }
         } else {
             for (uint32_t slot = ct; slot < rtot; slot += NCONS) {
@@ -917,7 +924,10 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
                 if (((uint32_t)k & (uint32_t)(P - 1)) != pitem) return;  // S padding slot
                 const K khi = k >> shift;
                 const uint32_t hv = *hp(khi);
-                for (uint32_t i = (hv >> 16) == tag ? (hv & 0xffffu) : END; i != END;) {
+                // a head of this item has tag << 16 | slot: xor leaves the slot; a stale
+                // head (another tag) leaves a value >= 2^16, which ends the walk like END
+                for (uint32_t i = PROBE_TAGX ? hv ^ (tag << 16) : ((hv >> 16) == tag ? (hv & 0xffffu) : END);
+                     i < END;) {
                     const Tup rv = rt[i];
                     const K l = rv.x;
                     if ((l >> 16) == khi) f((K)rv.y, i);

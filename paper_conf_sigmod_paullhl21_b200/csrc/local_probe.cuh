@@ -865,14 +865,17 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
     const int ct = tid - 32 * (PROBE_NP + NIDLE);
     unsigned long long my_cnt = 0, my_chk = 0;
     uint32_t tag = 0;
+    // stage and parity advance incrementally; barrier addresses computed once
+    const uint32_t full_at = smem_u32(&full[0]), empty_at = smem_u32(&empty[0]);
+    int s = 0;
+    uint32_t ph = 0;
     for (uint32_t j = 0; j < mine; ++j) {
-        const int s = j % PROBE_NST;
         if (++tag == 0x10000u) {  // tag wrap: clear the table once every 65535 items
             for (int i = ct; i < T; i += NCONS) head[i] = 0;
             named_bar_sync(1, NCONS);
             tag = 1;
         }
-        mbar_wait(&full[s], (j / PROBE_NST) & 1);
+        mbar_wait_at(full_at + 8u * s, ph);
         const Tup *rt = stages + (size_t)s * 2 * SL;
         const Tup *st = rt + stage_soff[s];
         const uint32_t rtot = totals[s][0], stot = totals[s][1];
@@ -1145,7 +1148,8 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
             }
         }
         named_bar_sync(1, NCONS);  // stage s and the table are free
-        if (ct == 0) mbar_arrive(&empty[s]);
+        if (ct == 0) mbar_arrive_at(empty_at + 8u * s);
+        if (++s == PROBE_NST) s = 0, ph ^= 1u;
     }
     my_cnt = warp_sum(my_cnt);
     my_chk = warp_sum(my_chk);

@@ -907,7 +907,7 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
                 const K khi = k >> shift;
                 const uint32_t old = atomicExch(hp(khi), (tag << 16) | slot);
                 const uint32_t ox = old ^ (tag << 16);  // < 2^16: a slot of this item
-                rw[2 * slot] = (K)(PROBE_TAGX ? (ox < 0x10000u ? ox : (uint32_t)END)
+                rw[2 * slot] = (K)(PROBE_TAGX ? min(ox, (uint32_t)END)  // a stale head (>= 2^16) ends the chain
                                               : ((old >> 16) == tag ? (old & 0xffffu) : (uint32_t)END)) |
                                (khi << 16);
             }

@@ -55,6 +55,10 @@ namespace mgj {
 #define PROBE_TAGX 1  // packed table: tag test by xor (one compare instead of shift, mask, two compares)
 #endif
 
+#ifndef PROBE_FAST
+#define PROBE_FAST 1  // 4-byte packed probe loop on 32-bit shared byte offsets
+#endif
+
 #ifndef PROBE_U2
 #define PROBE_U2 0  // packed probe: two S slots per step (measured slower: 2.00 vs 1.96 ms)
 #endif
@@ -1006,6 +1010,29 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
                     my_chk += chk_term(a, (K)sv.y);
                     ovf = true;
                 });
+            }
+        } else if (PROBE_FAST && packed && sizeof(K) == 4) {
+            // 4-byte keys, packed table, count + checksum only: shared addresses
+            // kept as 32-bit byte offsets (one LEA per access) and the S slots
+            // walked by pointer increment
+            const uint32_t rt_s = smem_u32(rt), tagsh = tag << 16;
+            const uint32_t mP = (uint32_t)(P - 1);
+            uint32_t sa = smem_u32(st + x0);
+            const uint32_t se = smem_u32(st + stot);
+            for (; sa < se; sa += NCONS * (uint32_t)sizeof(Tup)) {
+                uint32_t k, b;
+                asm("ld.shared.v2.u32 {%0,%1}, [%2];" : "=r"(k), "=r"(b) : "r"(sa));
+                if ((k & mP) != pitem) continue;  // S padding slot
+                const uint32_t khi = k >> shift;
+                for (uint32_t i = *hp((K)khi) ^ tagsh; i < END;) {
+                    uint32_t l, a;
+                    asm("ld.shared.v2.u32 {%0,%1}, [%2];" : "=r"(l), "=r"(a) : "r"(rt_s + i * 8u));
+                    if ((l >> 16) == khi) {
+                        ++m_item;
+                        my_chk += chk_term((K)a, (K)b);
+                    }
+                    i = l & 0xffffu;
+                }
             }
         } else if (PROBE_SPF && packed) {
             // software-pipelined: the next S slot and its head entry are loaded

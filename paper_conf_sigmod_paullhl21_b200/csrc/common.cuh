@@ -15,16 +15,15 @@ constexpr int MAX_B2 = 11;              // local fan-out per pass
 constexpr int HIST_THREADS = 512;
 constexpr int SCATTER_THREADS = 1024;
 constexpr int LOCAL_THREADS = 1024;
-#ifndef LOCAL_VMAX_CFG
-#define LOCAL_VMAX_CFG 12  // 13 measured: local 3.24 vs 2.87 ms (spills), probe -0.3%
-#endif
-constexpr int LOCAL_VMAX = LOCAL_VMAX_CFG;          // local-pass tuples per thread (chunk C <= 12 * LOCAL_THREADS), 8-byte tuples
+// local-pass tuples per thread (chunk C <= 12 * LOCAL_THREADS), 8-byte tuples
+// (13 measured: local 3.24 vs 2.87 ms from spills)
+constexpr int LOCAL_VMAX = 12;
 __host__ __device__ constexpr int local_vmax(int tuple_bytes) { return LOCAL_VMAX * 8 / tuple_bytes; }
 constexpr int PROBE_THREADS = 1024;     // warps 0..PROBE_NP-1 = TMA producers, the rest build/probe
 constexpr int PROBE_NST = 3;            // pipeline stages (items in flight per CTA)
-#ifndef PROBE_PPI
-#define PROBE_PPI 2                     // producer warps per item (1: R and S; 2: one relation each; 4: two each)
-#endif
+// producer warps per item: one per relation (four, two per relation, measured:
+// Zipf z = 1 probe 2.71 -> 2.54 ms but M2 1.95 -> 2.24 ms, so two stay)
+constexpr int PROBE_PPI = 2;
 constexpr int PROBE_NP = PROBE_NST * PROBE_PPI;  // producer warps (item streams <= PROBE_NST: parity waits one phase ahead)
 constexpr int PROBE_SLOTS8 = 4224;      // stage capacity per relation (slots) for 8-byte tuples; half for 16-byte
 constexpr int PROBE_HEAD8 = 128;        // headroom: co-partition target = capacity - headroom (padding, spread)
@@ -174,12 +173,7 @@ __device__ __forceinline__ uint64_t globaltimer() {
     return t;
 }
 
-__device__ __forceinline__ void set_err(const Ctx &c, int code) {
-#if defined(SCAT_RING) && SCAT_RING
-    if (code == MGJ_ECAPACITY) return;  // timing experiment: the received data is not the real one
-#endif
-    atomicCAS(c.err, 0, code);
-}
+__device__ __forceinline__ void set_err(const Ctx &c, int code) { atomicCAS(c.err, 0, code); }
 
 // Thread-0 helper: wait until every rank g raised flag `kind` for this epoch.
 __device__ inline bool wait_all_flags(const Ctx &c, int kind) {

@@ -7,61 +7,12 @@
 
 namespace mgj {
 
-#ifndef PROBE_PACK64
-#define PROBE_PACK64 0  // packed table for 8-byte keys too
-#endif
-
-#ifndef LP_RING
-#define LP_RING 0  // EXPERIMENT ONLY (wrong results): local output chunk regions modulo LP_RING, to time an L2-resident local buffer
-#endif
-
-#ifndef PROBE_L2PF
-#define PROBE_L2PF 0  // producers prefetch the runs of the item PROBE_L2PF rounds ahead into L2 (measured slower: 2.40-2.53 vs 1.96 ms)
-#endif
-
-#ifndef PROBE_CPASYNC
-#define PROBE_CPASYNC 0  // producers copy runs with 16-byte cp.async (LDGSTS) instead of one TMA bulk copy per run (measured slower: 4.64 vs 1.96 ms)
-#endif
-
-#ifndef PROBE_SMALL
-#define PROBE_SMALL 0  // runs of at most this many tuples copied by the producer lane, no bulk copy (measured slower: zipf z=1 probe 3.13 / 3.55 ms at 8 / 16 vs 2.80)
-#endif
-
-#ifndef PROBE_EPF
-#define PROBE_EPF 1  // producers load the next batch's run offsets while issuing the current batch
-#endif
-
-#ifndef PROBE_EPF2
-#define PROBE_EPF2 0  // ... and the first batch of their next item's while finishing the current item (measured neutral: M2 1.957 vs 1.955, materialised 3.80 vs 3.85, wide 2.40 vs 2.38 with spills)
-#endif
-
-#ifndef PROBE_BAL
-#define PROBE_BAL 0  // the two producer warps of an item split its R + S runs evenly (measured: M2 probe 2.35 vs 1.96 ms, zipf z=1 2.80 vs 2.85, wide 2.70 vs 2.39)
-#endif
-
-#ifndef PROBE_IDLE
-#define PROBE_IDLE 0  // DIAGNOSTIC: idle warps taken from the consumers (6: probe 2.25 vs 1.96 ms at M2)
-#endif
-
-#ifndef PROBE_SPF
-#define PROBE_SPF 0  // packed probe: next S slot and its head loaded before the current chain walk (measured slower: 2.02 vs 1.96 ms)
-#endif
-
-#ifndef PROBE_HOFF
-#define PROBE_HOFF 1  // packed table: head offsets in three instructions
-#endif
-
-#ifndef PROBE_TAGX
-#define PROBE_TAGX 1  // packed table: tag test by xor (one compare instead of shift, mask, two compares)
-#endif
-
-#ifndef PROBE_FAST
-#define PROBE_FAST 1  // 4-byte packed probe loop on 32-bit shared byte offsets
-#endif
-
-#ifndef PROBE_U2
-#define PROBE_U2 0  // packed probe: two S slots per step (measured slower: 2.00 vs 1.96 ms)
-#endif
+// (Probe variants measured in round 1 and not kept, against 1.96 ms at M2:
+// L2 bulk prefetch of later items' runs 2.40-2.53 ms, cp.async instead of
+// bulk copies 4.64, lane copies of short runs (Zipf z = 1: 3.13-3.55 vs
+// 2.80), an even R + S split between the producers 2.35, a software-
+// pipelined packed probe 2.02, two S slots per step 2.00, the packed table
+// for 8-byte keys 3.04 vs 2.82 at M5.)
 
 template <typename K> struct Layout {
     using Tup = typename TupT<K>::T;
@@ -485,7 +436,7 @@ __global__ void __launch_bounds__(LOCAL_THREADS, 1) k_local(Ctx c, const ChunkDe
                 bulk_commit();
             }
         } else if (tid == LI && tot) {
-            Tup *dst = static_cast<Tup *>(c.local[rel]) + (size_t)(LP_RING ? li % LP_RING : li) * CR;
+            Tup *dst = static_cast<Tup *>(c.local[rel]) + (size_t)li * CR;
             tma_store_1d(dst, sorted, tot * TB);
             bulk_commit();
         }
@@ -636,8 +587,7 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
     constexpr int TB = Layout<K>::TB;
     constexpr int LOGT = 12, T = 1 << LOGT;
     constexpr uint16_t END = 0xffff;
-    constexpr int NIDLE = PROBE_IDLE;  // EXPERIMENT: warps that do nothing (consumer-count sensitivity)
-    constexpr int NCONS = PROBE_THREADS - 32 * (PROBE_NP + NIDLE);
+    constexpr int NCONS = PROBE_THREADS - 32 * PROBE_NP;
     extern __shared__ __align__(128) unsigned char smem[];
     __shared__ __align__(8) uint64_t full[PROBE_NST], empty[PROBE_NST];
     __shared__ uint32_t totals[PROBE_NST][2];
@@ -668,7 +618,7 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
     // means equal keys; padding slots (digit1 != p) are left out on both sides.
     // (8-byte keys: measured slower packed, 3.04 vs 2.82 ms at M5 size: the
     // 64-bit shifts and compares cost more issue slots than the link load saves)
-    const bool packed = (sizeof(K) == 4 || PROBE_PACK64) && c.B1 + B2 >= 16;
+    const bool packed = sizeof(K) == 4 && c.B1 + B2 >= 16;
     const int P = c.P;
     const int Q = 1 << c.meta[MT_QB], shift = c.B1 + B2;  // Q: runs per chunk of the chunked pass
     const uint32_t nitems = min(__ldcg(&c.ticket[TK_ITEMS]), c.max_items);
@@ -676,7 +626,7 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
     const ItemX *items = reinterpret_cast<const ItemX *>(c.items);
     if (tid == 0) {
         for (int s = 0; s < PROBE_NST; ++s) {
-            mbar_init(&full[s], PROBE_CPASYNC ? PROBE_PPI * 33 : PROBE_PPI);
+            mbar_init(&full[s], PROBE_PPI);
             mbar_init(&empty[s], 1);
         }
         fence_mbar_init();
@@ -684,23 +634,17 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
     for (int i = tid; i < T; i += PROBE_THREADS) head[i] = 0;
     __syncthreads();
 
-    if (NIDLE && warp >= PROBE_NP && warp < PROBE_NP + NIDLE) return;
     if (warp < PROBE_NP) {
         // ------------------------------------------------------- producers
+        // two warps per item stream: warp & 1 issues the item's R runs, the
+        // other its S runs (one warp's bulk copies issue one after another;
+        // tools/tma_runs.cu)
         constexpr int ALIGN = Layout<K>::ALIGN;
         const uint64_t pol = policy_evict_first();
-        // PROBE_PPI producer warps per item: 1 (both relations), 2 (R / S) or 4
-        // (two per relation, each issuing every other run: one warp's bulk
-        // copies issue one after another, so the copies of 768-byte runs are
-        // issue-bound with one warp per relation; tools/tma_runs.cu)
         constexpr int NPI = PROBE_NP / PROBE_PPI;  // item streams (<= PROBE_NST)
         const int pw = warp / PROBE_PPI;
-        const int rel0 = PROBE_PPI >= 2 ? (warp & 1) : 0, rel1 = PROBE_PPI >= 2 ? rel0 + 1 : 2;
-        const int sub = PROBE_PPI == 4 ? ((warp >> 1) & 1) : 0;  // which half of the relation's runs
+        const int rel = warp & 1;
         ItemX x;
-        bool copied_small = false;  // this lane stored small runs into the stage (PROBE_SMALL)
-        bool xpf = false;           // pf0/pf1 hold the first batch of run offsets of item x (PROBE_EPF2)
-        uint32_t pf0 = 0, pf1 = 0;
         if (pw < (int)mine) x = items[blockIdx.x + pw * gridDim.x];
         for (uint32_t j = pw; j < mine; j += NPI) {
             ItemX xn;
@@ -708,165 +652,74 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
             const int s = j % PROBE_NST;
             if (j >= PROBE_NST) mbar_wait(&empty[s], ((j / PROBE_NST) - 1) & 1);
             uint32_t *pb = padbits + s * PW;
-            if (SBITS && rel1 == 2 && sub == 0) {
+            if (SBITS && rel == 1) {
                 for (int w = lane; w < PW; w += 32) pb[w] = 0;
                 __syncwarp();
             }
-            // PROBE_BAL (two producers per item): the item's R and S runs form one
-            // list and each warp issues half of it, instead of one warp per
-            // relation (|R|:|S| = 1:4 left the S warp with 4x the copies)
-            const bool bal = PROBE_BAL && PROBE_PPI == 2 && !SBITS;
-            uint32_t glo = 0, ghi = 0xffffffffu, nrun0 = 0;
-            if (bal) {
-                auto np_of = [&](int rel) -> uint32_t {
-                    const Side sd = rel ? x.it.s : x.it.r;
-                    const uint32_t xnch = rel ? x.nch[1] : x.nch[0];
-                    const uint32_t kend = min(sd.k1, xnch - 1);
-                    return sd.k0 <= kend ? kend - sd.k0 + 1 : 0;
-                };
-                nrun0 = np_of(0);
-                const uint32_t M = nrun0 + np_of(1), h = (M + 1) / 2;
-                glo = (warp & 1) ? h : 0;
-                ghi = (warp & 1) ? M : h;
-            }
-            for (int rel = bal ? 0 : rel0; rel < (bal ? 2 : rel1); ++rel) {
-                const uint32_t gbase = rel ? nrun0 : 0;  // index of the relation's first run in the item's list
-                const Side sd = rel ? x.it.s : x.it.r;
-                const uint32_t xcb = rel ? x.cb[1] : x.cb[0], xnch = rel ? x.nch[1] : x.nch[0];  // no local memory
-                const uint16_t *E0 = (rel ? c.eoff[1] : c.eoff[0]) + (size_t)(Q + 1) * xcb + (size_t)x.it.q * xnch;
-                const uint16_t *E1 = E0 + xnch;
-                const uint32_t kend = min(sd.k1, xnch - 1);
-                const uint32_t np = sd.k0 <= kend ? kend - sd.k0 + 1 : 0;
-                Tup *dstbase = stages + (size_t)s * 2 * SL + (rel ? x.soff : 0);
-                const Tup *lbase = static_cast<const Tup *>(rel ? c.local[1] : c.local[0]);
-                uint32_t run = 0;
-                // run offsets of the next batch of 32 runs are loaded while this
-                // batch is scanned and issued (items of heavy partitions have
-                // hundreds of runs: one load latency per batch otherwise)
-                uint32_t en0 = 0, en1 = 0;
-                if (PROBE_EPF2 && xpf) {  // loaded during the previous item (one relation per warp)
-                    en0 = pf0, en1 = pf1;
-                } else if (PROBE_EPF && lane < np) {
-                    en0 = E0[sd.k0 + lane], en1 = E1[sd.k0 + lane];
-                }
-                for (uint32_t m0 = 0; m0 < np; m0 += 32) {
-                    const uint32_t m = m0 + lane;
-                    uint32_t sz = 0, pad = 0xffffffffu;
-                    uint64_t src = 0;
-                    const uint32_t ec0 = en0, ec1 = en1;
-                    if (PROBE_EPF && m + 32 < np) en0 = E0[sd.k0 + m + 32], en1 = E1[sd.k0 + m + 32];
-                    if (m < np) {
-                        const uint32_t k = sd.k0 + m;
-                        uint32_t st, slots, v;
-                        if (PROBE_EPF) decode_run<ALIGN>(ec0, ec1, st, slots, v);
-                        else decode_run<ALIGN>(E0[k], E1[k], st, slots, v);
-                        const uint32_t alo = (k == sd.k0) ? sd.a0 : 0;
-                        const uint32_t ahi = (k == sd.k1) ? sd.a1 : slots;
-                        if (ahi > alo) {
-                            sz = ahi - alo;
-                            src = (uint64_t)(LP_RING ? (xcb + k) % LP_RING : xcb + k) * (BAp ? c.chunk_region2 : c.chunk_region) + st + alo;
-                        }
-                        pad = (SBITS && rel == 1 && v < slots && v >= alo && v < ahi) ? v - alo : 0xffffffffu;
+            const Side sd = rel ? x.it.s : x.it.r;
+            const uint32_t xcb = rel ? x.cb[1] : x.cb[0], xnch = rel ? x.nch[1] : x.nch[0];  // no local memory
+            const uint16_t *E0 = (rel ? c.eoff[1] : c.eoff[0]) + (size_t)(Q + 1) * xcb + (size_t)x.it.q * xnch;
+            const uint16_t *E1 = E0 + xnch;
+            const uint32_t kend = min(sd.k1, xnch - 1);
+            const uint32_t np = sd.k0 <= kend ? kend - sd.k0 + 1 : 0;
+            Tup *dstbase = stages + (size_t)s * 2 * SL + (rel ? x.soff : 0);
+            const Tup *lbase = static_cast<const Tup *>(rel ? c.local[1] : c.local[0]);
+            uint32_t run = 0;
+            // run offsets of the next batch of 32 runs are loaded while this
+            // batch is scanned and issued (items of heavy partitions have
+            // hundreds of runs: one load latency per batch otherwise)
+            uint32_t en0 = 0, en1 = 0;
+            if (lane < np) en0 = E0[sd.k0 + lane], en1 = E1[sd.k0 + lane];
+            for (uint32_t m0 = 0; m0 < np; m0 += 32) {
+                const uint32_t m = m0 + lane;
+                uint32_t sz = 0, pad = 0xffffffffu;
+                uint64_t src = 0;
+                const uint32_t ec0 = en0, ec1 = en1;
+                if (m + 32 < np) en0 = E0[sd.k0 + m + 32], en1 = E1[sd.k0 + m + 32];
+                if (m < np) {
+                    const uint32_t k = sd.k0 + m;
+                    uint32_t st, slots, v;
+                    decode_run<ALIGN>(ec0, ec1, st, slots, v);
+                    const uint32_t alo = (k == sd.k0) ? sd.a0 : 0;
+                    const uint32_t ahi = (k == sd.k1) ? sd.a1 : slots;
+                    if (ahi > alo) {
+                        sz = ahi - alo;
+                        src = (uint64_t)(xcb + k) * (BAp ? c.chunk_region2 : c.chunk_region) + st + alo;
                     }
-                    uint32_t incl = sz;
+                    pad = (SBITS && rel == 1 && v < slots && v >= alo && v < ahi) ? v - alo : 0xffffffffu;
+                }
+                uint32_t incl = sz;
 #pragma unroll
-                    for (int o = 1; o < 32; o <<= 1) {
-                        const uint32_t y = __shfl_up_sync(0xffffffffu, incl, o);
-                        if (lane >= o) incl += y;
-                    }
-                    const uint32_t dst = run + incl - sz;
-                    const uint32_t gsum = __shfl_sync(0xffffffffu, incl, 31);
-                    const bool issue_it = (!bal || (gbase + m >= glo && gbase + m < ghi)) &&
-                                          (PROBE_PPI != 4 || (SBITS ? sub == 0 : (m & 1u) == (uint32_t)sub));
-                    // runs of at most PROBE_SMALL tuples are copied by their lane with
-                    // plain loads/stores (a heavy partition leaves most co-partitions
-                    // in runs of a few tuples: one bulk copy each would dominate)
-                    const bool small = PROBE_SMALL && sz != 0 && sz <= PROBE_SMALL && issue_it;
-                    const uint32_t gmine = (bal || PROBE_SMALL || PROBE_PPI == 4)
-                                               ? __reduce_add_sync(0xffffffffu, (issue_it && !small) ? sz : 0u)
-                                               : gsum;
-                    if (PROBE_CPASYNC) {
-                        // the warp copies the batch's runs one after another, 16 bytes per lane
-                        constexpr uint32_t PT = 16 / TB;  // tuples per 16-byte piece
-                        for (int r = 0; r < 32; ++r) {
-                            const uint32_t rs = __shfl_sync(0xffffffffu, sz, r);
-                            if (!rs) continue;
-                            const uint64_t rsrc = __shfl_sync(0xffffffffu, src, r);
-                            const uint32_t rdst = __shfl_sync(0xffffffffu, dst, r);
-                            const uint32_t n16 = rs / PT;
-                            for (uint32_t i = lane; i < n16; i += 32)
-                                cp_async16(dstbase + rdst + i * PT, lbase + rsrc + i * PT);
-                        }
-                    } else {
-                    if (lane == 0 && gmine)
-                        asm volatile("mbarrier.expect_tx.relaxed.cta.shared::cta.b64 [%0], %1;" ::"r"(
-                                         smem_u32(&full[s])),
-                                     "r"(gmine * TB)
-                                     : "memory");
-                    __syncwarp();
-                    if (small) {
-                        for (uint32_t i = 0; i < sz; ++i) dstbase[dst + i] = __ldcs(lbase + src + i);
-                        copied_small = true;
-                    } else if (sz && issue_it) {
-                        tma_load_1d(dstbase + dst, lbase + src, sz * TB, &full[s], pol);
-                    }
-                    }
-                    if (pad != 0xffffffffu) atomicOr(&pb[(dst + pad) >> 5], 1u << ((dst + pad) & 31));
-                    run += gsum;
+                for (int o = 1; o < 32; o <<= 1) {
+                    const uint32_t y = __shfl_up_sync(0xffffffffu, incl, o);
+                    if (lane >= o) incl += y;
                 }
-                if (lane == 0 && (!bal || (warp & 1) == rel) && sub == 0) totals[s][rel] = run;
-                if (PROBE_L2PF && j + PROBE_L2PF * NPI < mine) {
-                    // the same side of the item PROBE_L2PF rounds ahead: its runs -> L2, so that
-                    // its stage loads hit L2 (more bytes in flight than the stages can hold)
-                    const ItemX y = items[blockIdx.x + (j + PROBE_L2PF * NPI) * gridDim.x];
-                    const Side sy = rel ? y.it.s : y.it.r;
-                    const uint32_t ycb = rel ? y.cb[1] : y.cb[0], ynch = rel ? y.nch[1] : y.nch[0];
-                    const uint16_t *F0 = (rel ? c.eoff[1] : c.eoff[0]) + (size_t)(Q + 1) * ycb + (size_t)y.it.q * ynch;
-                    const uint32_t kend2 = min(sy.k1, ynch - 1);
-                    const uint32_t np2 = sy.k0 <= kend2 ? kend2 - sy.k0 + 1 : 0;
-                    for (uint32_t m = lane; m < np2; m += 32) {
-                        const uint32_t k = sy.k0 + m;
-                        uint32_t st, slots, v;
-                        decode_run<ALIGN>(F0[k], F0[k + ynch], st, slots, v);
-                        const uint32_t alo = (k == sy.k0) ? sy.a0 : 0;
-                        const uint32_t ahi = (k == sy.k1) ? sy.a1 : slots;
-                        if (ahi > alo)
-                            prefetch_l2(lbase + (uint64_t)(ycb + k) * c.chunk_region + st + alo, (ahi - alo) * TB);
-                    }
-                }
+                const uint32_t dst = run + incl - sz;
+                const uint32_t gsum = __shfl_sync(0xffffffffu, incl, 31);
+                if (lane == 0 && gsum)
+                    asm volatile("mbarrier.expect_tx.relaxed.cta.shared::cta.b64 [%0], %1;" ::"r"(
+                                     smem_u32(&full[s])),
+                                 "r"(gsum * TB)
+                                 : "memory");
+                __syncwarp();
+                if (sz) tma_load_1d(dstbase + dst, lbase + src, sz * TB, &full[s], pol);
+                if (pad != 0xffffffffu) atomicOr(&pb[(dst + pad) >> 5], 1u << ((dst + pad) & 31));
+                run += gsum;
             }
-            if (lane == 0 && rel0 == 0 && sub == 0) {
+            if (lane == 0) totals[s][rel] = run;
+            if (lane == 0 && rel == 0) {
                 stage_p[s] = (uint32_t)c.plist[BAp ? x.it.pi >> BAp : x.it.pi];
                 stage_soff[s] = x.soff;
             }
             __syncwarp();
-            if (PROBE_CPASYNC) cp_async_mbar_arrive(&full[s]);  // fires when this lane's copies have landed
-            if (PROBE_SMALL) {  // this warp's plain stores, then lane 0's release arrive publishes them
-                if (copied_small) __threadfence_block();
-                __syncwarp();
-                copied_small = false;
-            }
             if (lane == 0) mbar_arrive(&full[s]);
-            // first batch of this warp's run offsets of its next item, loaded now
-            xpf = false;
-            if (PROBE_EPF2 && !bal && rel1 == rel0 + 1 && j + NPI < mine) {
-                const int rel = rel0;
-                const Side sd = rel ? xn.it.s : xn.it.r;
-                const uint32_t xcb = rel ? xn.cb[1] : xn.cb[0], xnch = rel ? xn.nch[1] : xn.nch[0];
-                const uint16_t *E0 = (rel ? c.eoff[1] : c.eoff[0]) + (size_t)(Q + 1) * xcb + (size_t)xn.it.q * xnch;
-                const uint32_t kend = min(sd.k1, xnch - 1);
-                const uint32_t np = sd.k0 <= kend ? kend - sd.k0 + 1 : 0;
-                pf0 = pf1 = 0;
-                if (lane < np) pf0 = E0[sd.k0 + lane], pf1 = E0[xnch + sd.k0 + lane];
-                xpf = true;
-            }
             x = xn;
         }
         return;
     }
 
     // ------------------------------------------------------------ consumers
-    const int ct = tid - 32 * (PROBE_NP + NIDLE);
+    const int ct = tid - 32 * PROBE_NP;
     unsigned long long my_cnt = 0, my_chk = 0;
     uint32_t tag = 0;
     // stage and parity advance incrementally; barrier addresses computed once
@@ -895,7 +748,7 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
         // head entry of khi: the same index as fold(), computed as a byte offset
         // in three instructions (shift, shift, xor-and) for 4-byte keys
         auto hp = [&](K khi) -> uint32_t * {
-            if constexpr (sizeof(K) == 4 && PROBE_HOFF) {
+            if constexpr (sizeof(K) == 4) {
                 const uint32_t off = (((uint32_t)khi << 2) ^ ((uint32_t)khi >> (LOGT - 2))) & (uint32_t)((T - 1) << 2);
                 return reinterpret_cast<uint32_t *>(reinterpret_cast<char *>(head) + off);
             } else {
@@ -911,8 +764,7 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
                 const K khi = k >> shift;
                 const uint32_t old = atomicExch(hp(khi), (tag << 16) | slot);
                 const uint32_t ox = old ^ (tag << 16);  // < 2^16: a slot of this item
-                rw[2 * slot] = (K)(PROBE_TAGX ? min(ox, (uint32_t)END)  // a stale head (>= 2^16) ends the chain
-                                              : ((old >> 16) == tag ? (old & 0xffffu) : (uint32_t)END)) |
+                rw[2 * slot] = (K)min(ox, (uint32_t)END) |  // a stale head (>= 2^16) ends the chain
                                (khi << 16);
             }
         } else {
@@ -933,8 +785,7 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
                 const uint32_t hv = *hp(khi);
                 // a head of this item has tag << 16 | slot: xor leaves the slot; a stale
                 // head (another tag) leaves a value >= 2^16, which ends the walk like END
-                for (uint32_t i = PROBE_TAGX ? hv ^ (tag << 16) : ((hv >> 16) == tag ? (hv & 0xffffu) : END);
-                     i < END;) {
+                for (uint32_t i = hv ^ (tag << 16); i < END;) {
                     const Tup rv = rt[i];
                     const K l = rv.x;
                     if ((l >> 16) == khi) f((K)rv.y, i);
@@ -952,36 +803,6 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
         // probe
         uint32_t m_item = 0;
         uint32_t x0 = ct;
-        if (PROBE_U2 && packed && !MAT) {  // two S slots per step: independent load chains
-            for (; x0 + NCONS < stot; x0 += 2 * NCONS) {
-                const Tup s0 = st[x0], s1 = st[x0 + NCONS];
-                const uint32_t k0 = (uint32_t)s0.x, k1 = (uint32_t)s1.x;
-                const uint32_t kh0 = k0 >> shift, kh1 = k1 >> shift;
-                const uint32_t h0 = head[fold(kh0)], h1 = head[fold(kh1)];
-                uint32_t i0 = ((k0 & (uint32_t)(P - 1)) == pitem && (h0 >> 16) == tag) ? (h0 & 0xffffu) : END;
-                uint32_t i1 = ((k1 & (uint32_t)(P - 1)) == pitem && (h1 >> 16) == tag) ? (h1 & 0xffffu) : END;
-                while (i0 != END || i1 != END) {
-                    if (i0 != END) {
-                        const Tup rv = rt[i0];
-                        const uint32_t l = (uint32_t)rv.x;
-                        if ((l >> 16) == kh0) {
-                            ++m_item;
-                            my_chk += chk_term((K)rv.y, (K)s0.y);
-                        }
-                        i0 = l & 0xffffu;
-                    }
-                    if (i1 != END) {
-                        const Tup rv = rt[i1];
-                        const uint32_t l = (uint32_t)rv.x;
-                        if ((l >> 16) == kh1) {
-                            ++m_item;
-                            my_chk += chk_term((K)rv.y, (K)s1.y);
-                        }
-                        i1 = l & 0xffffu;
-                    }
-                }
-            }
-        }
         // MAT: the first match of each of this thread's S slots is kept (R slot
         // index) so the write pass needs no second walk unless a slot matched
         // more than once (duplicate R keys: the warp re-walks instead)
@@ -1011,7 +832,7 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
                     ovf = true;
                 });
             }
-        } else if (PROBE_FAST && packed && sizeof(K) == 4) {
+        } else if (packed && sizeof(K) == 4) {
             // 4-byte keys, packed table, count + checksum only: shared addresses
             // kept as 32-bit byte offsets (one LEA per access) and the S slots
             // walked by pointer increment
@@ -1032,35 +853,6 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
                         my_chk += chk_term((K)a, (K)b);
                     }
                     i = l & 0xffffu;
-                }
-            }
-        } else if (PROBE_SPF && packed) {
-            // software-pipelined: the next S slot and its head entry are loaded
-            // before the current slot's chain is walked (two fewer dependent
-            // shared-memory round trips on the critical path per slot)
-            uint32_t x = x0;
-            Tup sn{};
-            uint32_t hn = 0;
-            auto fetch = [&](uint32_t xx) {
-                sn = st[xx];
-                hn = head[fold((K)(sn.x >> shift))];
-            };
-            if (x < stot) fetch(x);
-            for (; x < stot; x += NCONS) {
-                const Tup sv = sn;
-                const uint32_t hv = hn;
-                if (x + NCONS < stot) fetch(x + NCONS);
-                const K k = sv.x;
-                if (((uint32_t)k & (uint32_t)(P - 1)) != pitem) continue;  // S padding slot
-                const K khi = k >> shift;
-                for (uint32_t i = (hv >> 16) == tag ? (hv & 0xffffu) : END; i != END;) {
-                    const Tup rv = rt[i];
-                    const K l = rv.x;
-                    if ((l >> 16) == khi) {
-                        ++m_item;
-                        my_chk += chk_term((K)rv.y, (K)sv.y);
-                    }
-                    i = (uint32_t)l & 0xffffu;
                 }
             }
         } else {

@@ -321,8 +321,7 @@ mgj_status mgj_plan(const mgj_config *cfg, const mgj_peers *peers, mgj_handle *o
     const size_t z_acc = zo; zo += 256;
     const size_t z_err = zo; zo += 256;
     const size_t z_cop = zo; zo += align_up(2ull * P * Qm * 4, 256);
-    // tiles: one per scatter CTA (two per SM when the scatter runs two CTAs per SM)
-    const int G = h->nsm * (scat_geom(P, n.c.key_bytes).NT <= 512 ? 2 : 1);  // scatter tiles: one per CTA
+    const int G = h->nsm;  // scatter tiles: one per scatter CTA, one CTA per SM
     const size_t z_th = zo; zo += align_up(2ull * G * P * 4, 256);
     const size_t z_ha = zo; zo += align_up(2ull * local2_vcap(P) * 4, 256);
     h->zero_bytes = zo;
@@ -336,7 +335,7 @@ mgj_status mgj_plan(const mgj_config *cfg, const mgj_peers *peers, mgj_handle *o
     c.b2_cfg = n.c.radix_bits_local;
     c.b2_max = n.b2_max;
     c.G = G;
-    c.hist_split = G == h->nsm ? 2 : 1;  // k_hist: two CTAs per SM either way
+    c.hist_split = 2;  // k_hist: two CTAs per SM
     c.chunk_tuples = n.chunk_tuples;
     c.chunk_region = n.chunk_region;
     c.chunk_tuples2 = n.chunk_tuples2;

@@ -7,13 +7,6 @@
 
 namespace mgj {
 
-#ifndef SCAT_WO_UNROLL
-#define SCAT_WO_UNROLL 1  // write-out groups per thread per step
-#endif
-#ifndef SCAT_ATOM_FIRST
-#define SCAT_ATOM_FIRST 0  // rank all tuples of a thread before storing them
-#endif
-
 // Scatter geometry for P partitions and a key width (kernel template
 // arguments; the host picks the instance with scatter_kernel<K>(P)):
 //   T   = sub-tile (tuples) staged in shared memory per step,
@@ -23,43 +16,20 @@ namespace mgj {
 // < 32-byte tail of a partition waits (in registers of its owning thread)
 // for the next sub-tile.  For P = 4096 the alignment padding would not fit
 // shared memory, so SG = 1 (one tuple per store).
-#ifndef SCAT_GDST
-#define SCAT_GDST 0  // per-group destination table written at layout time, no partition lookup in the write-out (measured slower: 4.36 vs 4.16 ms)
-#endif
-
-#ifndef SCAT_SOA
-#define SCAT_SOA 0  // 4-byte keys: `sorted` held as key and payload arrays (4-byte random stores; measured slower: 4.42 vs 4.14 ms)
-#endif
-#ifndef SCAT_LDG
-#define SCAT_LDG 0  // sub-tiles loaded straight into registers one sub-tile ahead, no shared-memory stage (measured slower: 4.73 vs 4.13 ms)
-#endif
-#ifndef SCAT_T4
-#define SCAT_T4 8192  // sub-tile of the 4-byte-key, P <= 1024 instance
-#endif
-#ifndef SCAT_2CTA
-#define SCAT_2CTA 0  // 4-byte keys, P <= 1024: two 512-thread CTAs per SM, 4096-tuple sub-tiles, 16-byte groups (measured slower: 9.2 vs 4.1 ms)
-#endif
-#ifndef SCAT_ALIAS
-#define SCAT_ALIAS 0  // 4-byte keys, P <= 1024: two 512-thread CTAs per SM, stage aliased into the sorted buffer (measured: 6.2 vs 4.1 ms)
-#endif
-#ifndef SCAT_PROF
-#define SCAT_PROF 0  // DIAGNOSTIC: thread 0 and 512 of CTA 0 print clock64 time per phase
-#endif
-#ifndef SCAT_RING
-#define SCAT_RING 0  // EXPERIMENT ONLY (wrong results): full-group stores land modulo SCAT_RING bytes of the arena (L2-resident)
-#endif
+// (Measured alternatives, round 1, not kept: 4096-tuple sub-tiles in two
+// 512-thread CTAs per SM with 16- or 32-byte groups, 9.2 / 6.2 ms; SoA
+// staging with 4-byte random stores, 4.42 ms; register-staged sub-tiles
+// without TMA, 4.73 ms; a per-group destination table, 4.36 ms; against
+// 4.16 ms for this design at M2.)
 struct ScatGeom {
     int T, SG, PPT, NT;
-    bool alias;  // stage inside the sorted buffer (two CTAs per SM)
 };
 __host__ __device__ constexpr ScatGeom scat_geom(int P, int key_bytes) {
     return key_bytes == 4
-               ? (P <= 1024 ? (SCAT_ALIAS  ? ScatGeom{4096, 4, P <= 512 ? 1 : 2, 512, true}
-                               : SCAT_2CTA ? ScatGeom{4096, 2, P <= 512 ? 1 : 2, 512, false}
-                                           : ScatGeom{SCAT_T4, 4, 1, 1024, false})
-                  : P == 2048 ? ScatGeom{4096, 4, 2, 1024, false} : ScatGeom{8192, 1, 4, 1024, false})
-               : (P <= 1024 ? ScatGeom{4096, 2, 1, 1024, false} : P == 2048 ? ScatGeom{2048, 2, 2, 1024, false}
-                                                                      : ScatGeom{4096, 1, 4, 1024, false});
+               ? (P <= 1024 ? ScatGeom{8192, 4, 1, 1024}
+                  : P == 2048 ? ScatGeom{4096, 4, 2, 1024} : ScatGeom{8192, 1, 4, 1024})
+               : (P <= 1024 ? ScatGeom{4096, 2, 1, 1024} : P == 2048 ? ScatGeom{2048, 2, 2, 1024}
+                                                                      : ScatGeom{4096, 1, 4, 1024});
 }
 
 // Per-partition write-out descriptor of the current sub-tile (16 bytes, one
@@ -73,11 +43,10 @@ struct __align__(16) PInfo {
 __host__ __device__ inline size_t scat_smem_bytes(int P, int key_bytes) {
     const ScatGeom g = scat_geom(P, key_bytes);
     const size_t TB = 2 * (size_t)key_bytes;
-    return ((g.alias || SCAT_LDG) ? 0 : 2 * (size_t)g.T * key_bytes)  // input stage: keys + payloads (SoA)
+    return 2 * (size_t)g.T * key_bytes                         // input stage: keys + payloads (SoA)
            + ((size_t)g.T + 2 * (size_t)(g.SG - 1) * P) * TB  // partition-sorted sub-tile (+ carries, group padding)
-           + ((SCAT_GDST && g.SG > 1) ? ((size_t)g.T + 2 * (size_t)(g.SG - 1) * P) / g.SG * 8  // group destinations
-                                      : (size_t)P * sizeof(PInfo))
-           + (size_t)P * 4;                                  // next free slot per partition
+           + (size_t)P * sizeof(PInfo)                         // write-out descriptors
+           + (size_t)P * 4;                                    // next free slot per partition
 }
 
 // Block-wide exclusive scan of one register value per thread (<= 1024 threads).
@@ -105,34 +74,6 @@ __device__ __forceinline__ uint32_t block_scan_reg(uint32_t v, uint32_t *tmp, ui
     return x - v + (w ? tmp[w - 1] : 0);
 }
 
-// Same with one barrier: every warp reduces the per-warp totals itself (its
-// prefix and the block total) instead of one warp scanning them behind a
-// second barrier.  `tmp` may be rewritten only after a later barrier.
-__device__ __forceinline__ uint32_t block_scan_reg1(uint32_t v, uint32_t *tmp, uint32_t &total) {
-    const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
-    uint32_t x = v;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-        const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
-        if (lane >= o) x += y;
-    }
-    if (lane == 31) tmp[w] = x;
-    __syncthreads();
-    const uint32_t t = lane < (int)(blockDim.x >> 5) ? tmp[lane] : 0u;
-    uint32_t pre = lane < w ? t : 0u, tot = t;
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) {
-        pre += __shfl_xor_sync(0xffffffffu, pre, o);
-        tot += __shfl_xor_sync(0xffffffffu, tot, o);
-    }
-    total = tot;
-    return x - v + pre;
-}
-
-#ifndef SCAT_SCAN1
-#define SCAT_SCAN1 0  // one-barrier layout scan (measured neutral: 4.16 vs 4.16 ms)
-#endif
-
 // 16-byte shared load that the compiler keeps where it is written (not sunk
 // into the branch that consumes it): the write-out issues its group and
 // descriptor loads back to back.
@@ -143,11 +84,6 @@ __device__ __forceinline__ uint4 lds128(const void *p) {
                  : "r"(smem_u32(p)));
     return v;
 }
-
-#ifndef SCAT_EAGER
-#define SCAT_EAGER 1  // write-out: both group halves and the whole descriptor loaded up front, 8-byte keys
-                      // (measured: M5 scatter 3.725 -> 3.693 ms; 4-byte keys 4.155 -> 4.19, so not used there)
-#endif
 
 template <int BYTES> struct Vec;
 template <> struct Vec<8> { using T = uint2; };
@@ -197,8 +133,8 @@ __device__ __forceinline__ void st_group(void *dst, const typename Vec<BYTES>::T
 // have no role on a one-hop fabric.  The last CTA raises SIG_DATA at every
 // peer after a system fence.
 // ---------------------------------------------------------------------------
-template <typename K, int T, int SG, int PPT, int NT, bool ALIAS>
-__global__ void __launch_bounds__(NT, NT <= 512 ? 2 : 1) k_scatter(Ctx c) {
+template <typename K, int T, int SG, int PPT, int NT>
+__global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c) {
     using Tup = typename TupT<K>::T;
     constexpr int TB = (int)sizeof(Tup);
     constexpr int V = T / NT;                  // tuples per thread per sub-tile
@@ -213,53 +149,22 @@ __global__ void __launch_bounds__(NT, NT <= 512 ? 2 : 1) k_scatter(Ctx c) {
     // `sorted` swizzle: the two 16-byte halves of every 32-byte group whose
     // index has bit 2 set are swapped, so that the write-out's 16-byte loads
     // (8 consecutive groups per quarter warp) hit distinct banks
-    // SOA (4-byte keys, 32-byte groups): `sorted` is a key array and a payload
-    // array; the scatter's random stores are 4 bytes wide (fewer bank conflicts
-    // than 8-byte ones) and the write-out interleaves 16 bytes of keys with 16
-    // bytes of payloads into the group's 32-byte store (conflict-free, no swizzle)
-    constexpr bool SOA = SCAT_SOA && sizeof(K) == 4 && SG == 4 && !ALIAS;
     auto swz = [](uint32_t s) -> uint32_t {
-        if constexpr (SG > 1 && !SOA && SG * sizeof(Tup) == 32) return s ^ (((s >> (SG == 4 ? 4 : 3)) & 1u) * (SG / 2));
+        if constexpr (SG > 1 && SG * sizeof(Tup) == 32) return s ^ (((s >> (SG == 4 ? 4 : 3)) & 1u) * (SG / 2));
         else return s;
     };
+    // 8-byte keys: both group halves and the whole descriptor are loaded up
+    // front (measured: M5 scatter 3.725 -> 3.693 ms; 4-byte keys 4.155 -> 4.19)
+    constexpr bool EAGER = sizeof(K) == 8;
     extern __shared__ __align__(128) unsigned char smem[];
     const int P = c.P;
-    // ALIAS: the stage is the head of the sorted buffer (loaded after the write-out)
-    // LDG: sub-tile g+1 is loaded into registers (16-byte streaming loads) while
-    // g is laid out, ranked and written out; no stage, no TMA, no mbarrier
-    constexpr bool LDG = SCAT_LDG && !ALIAS;
-    Tup *const sorted = reinterpret_cast<Tup *>(smem + ((ALIAS || LDG) ? 0 : 2 * T * sizeof(K)));
-    K *const skey = reinterpret_cast<K *>(ALIAS ? static_cast<void *>(sorted) : static_cast<void *>(smem));
+    K *const skey = reinterpret_cast<K *>(smem);  // stage: keys, then payloads
     K *const spay = skey + T;
-    // GD: the layout writes every group's destination (0: not stored; low bits:
-    // h placeholder slots of a head group) so the write-out needs no lookup of
-    // the group's partition; otherwise a per-partition descriptor (PInfo)
-    constexpr bool GD = SCAT_GDST && SG > 1;
-    constexpr bool EAGER = SCAT_EAGER && sizeof(K) == 8;
+    Tup *const sorted = reinterpret_cast<Tup *>(smem + 2 * T * sizeof(K));
     PInfo *const pinfo = reinterpret_cast<PInfo *>(sorted + T + 2 * (SG - 1) * P);  // 16-byte aligned
-    unsigned long long *const gdst = reinterpret_cast<unsigned long long *>(pinfo);
-    uint32_t *const off = GD ? reinterpret_cast<uint32_t *>(gdst + (T + 2 * (SG - 1) * P) / SG)
-                             : reinterpret_cast<uint32_t *>(pinfo + P);  // next free slot per partition
-    K *const ks = reinterpret_cast<K *>(sorted);  // SOA: keys, then payloads
-    K *const ps = ks + (T + 2 * (SG - 1) * P);
-    auto sput = [&](uint32_t x, const Tup &t) {
-        if constexpr (SOA) {
-            ks[x] = t.x;
-            ps[x] = t.y;
-        } else {
-            sorted[swz(x)] = t;
-        }
-    };
-    auto sget = [&](uint32_t x) -> Tup {
-        if constexpr (SOA) {
-            Tup t;
-            t.x = ks[x];
-            t.y = ps[x];
-            return t;
-        } else {
-            return sorted[swz(x)];
-        }
-    };
+    uint32_t *const off = reinterpret_cast<uint32_t *>(pinfo + P);  // next free slot per partition
+    auto sput = [&](uint32_t x, const Tup &t) { sorted[swz(x)] = t; };
+    auto sget = [&](uint32_t x) -> Tup { return sorted[swz(x)]; };
     __shared__ __align__(8) uint64_t bar;
     __shared__ uint32_t tmp[32];
     const int tid = threadIdx.x;
@@ -366,62 +271,17 @@ __global__ void __launch_bounds__(NT, NT <= 512 ? 2 : 1) k_scatter(Ctx c) {
             out[0] = v.x & 0xffffu, out[1] = v.x >> 16, out[2] = v.y & 0xffffu, out[3] = v.y >> 16;
         }
     };
-    K kn[V], pn[V];  // LDG: the next sub-tile
-    auto fetch = [&](uint32_t g) {
-        int rel;
-        uint64_t first;
-        uint32_t len;
-        subtile(g, rel, first, len);
-        const K *gk = static_cast<const K *>(c.in_key[rel]) + first;
-        const K *gp = static_cast<const K *>(c.in_pay[rel]) + first;
-        if (len == T) {
-#pragma unroll
-            for (int u = 0; u < NU; ++u) {
-                const uint32_t i0 = (uint32_t)(u * NT + tid) * LU;
-                const uint4 a = __ldcs(reinterpret_cast<const uint4 *>(gk + i0));
-                const uint4 b = __ldcs(reinterpret_cast<const uint4 *>(gp + i0));
-                memcpy(&kn[u * LU], &a, 16);
-                memcpy(&pn[u * LU], &b, 16);
-            }
-        } else {
-#pragma unroll
-            for (int u = 0; u < NU; ++u) {
-#pragma unroll
-                for (int e = 0; e < LU; ++e) {
-                    const uint32_t i = (uint32_t)(u * NT + tid) * LU + e;
-                    kn[u * LU + e] = i < len ? __ldcs(gk + i) : (K)0;
-                    pn[u * LU + e] = i < len ? __ldcs(gp + i) : (K)0;
-                }
-            }
-        }
-    };
     uint32_t ncnt[PPT];
     load_counts(0, ncnt);
-    if (LDG) {
-        if (ntot > 0) fetch(0);
-    } else if (tid == 0 && ntot > 0) {
-        issue(0);
-    }
+    if (tid == 0 && ntot > 0) issue(0);
     int cur_rel = -1;
-    unsigned long long pt[7] = {0, 0, 0, 0, 0, 0, 0};
-    long long pc = clock64();
-    auto PT = [&](int i) {
-        if (SCAT_PROF) {
-            const long long n = clock64();
-            pt[i] += (unsigned long long)(n - pc);
-            pc = n;
-        }
-    };
     for (uint32_t g = 0; g < ntot; ++g) {
         int rel;
         uint64_t first;
         uint32_t len;
         subtile(g, rel, first, len);
         if (rel != cur_rel) {  // thread-private partition state: no barrier needed
-            if (SCAT_PROF && blockIdx.x == 0 && (tid == 0 || tid == 512))
-        printf("SCATPROF tid %d subtiles %u: top %llu scan %llu layout %llu tmawait %llu read+S1 %llu rank+S2 %llu writeout %llu\n",
-               tid, ntot, pt[0], pt[1], pt[2], pt[3], pt[4], pt[5], pt[6]);
-    if (cur_rel >= 0) flush();
+            if (cur_rel >= 0) flush();
             set_base(rel);
             cur_rel = rel;
         }
@@ -436,36 +296,21 @@ __global__ void __launch_bounds__(NT, NT <= 512 ? 2 : 1) k_scatter(Ctx c) {
         }
         load_counts(g + 1, ncnt);  // prefetch (consumed next iteration)
         uint32_t total;
-        PT(0);  // carries fetched, counts: top of the sub-tile
-        uint32_t o = SCAT_SCAN1 ? block_scan_reg1(tsum, tmp, total)   // its barrier: last write-out is done
-                                : block_scan_reg(tsum, tmp, total);
-        PT(1);  // layout scan (its barriers wait for the last write-out)
-        uint32_t co[PPT], ccw[PPT];  // segment start and carried count (for the ALIAS carry write)
-#pragma unroll
-        for (int k = 0; k < PPT; ++k) ccw[k] = cc[k], co[k] = 0;
+        uint32_t o = block_scan_reg(tsum, tmp, total);  // its barriers: the last write-out is done
 #pragma unroll
         for (int k = 0; k < PPT; ++k) {
             const int p = tid * PPT + k;
             if (p < P) {
-                if (!ALIAS) {
 #pragma unroll
-                    for (int i = 0; i < CW; ++i)
-                        if (i < (int)cc[k]) sput(o + i, carry[k][i]);
-                }
-                co[k] = o;
+                for (int i = 0; i < CW; ++i)
+                    if (i < (int)cc[k]) sput(o + i, carry[k][i]);
                 off[p] = o + cc[k];
                 const uint32_t full = cnt[k] & ~(uint32_t)(SG - 1);
-                if constexpr (GD) {
-                    const uint32_t ng = seg[k] / SG, nf = full / SG;
-                    for (uint32_t j = 0; j < ng; ++j)  // a skipped partition's groups are never stored
-                        gdst[o / SG + j] = (j < nf && !skp[k]) ? ((base[k] + (ull)j * GB) | (j == 0 ? hd[k] : 0u)) : 0ull;
-                } else {
-                    PInfo in;
-                    in.wb = base[k] - (ull)o * TB;
-                    in.lim = skp[k] ? o : o + cnt[k];  // a skipped partition's groups are never stored
-                    in.head = (hd[k] && full) ? (o << 2 | hd[k]) : NONE;
-                    pinfo[p] = in;
-                }
+                PInfo in;
+                in.wb = base[k] - (ull)o * TB;
+                in.lim = skp[k] ? o : o + cnt[k];  // a skipped partition's groups are never stored
+                in.head = (hd[k] && full) ? (o << 2 | hd[k]) : NONE;
+                pinfo[p] = in;
                 base[k] += (ull)full * TB;
                 if (full) hd[k] = 0;
                 cc[k] = cnt[k] - full;
@@ -474,15 +319,8 @@ __global__ void __launch_bounds__(NT, NT <= 512 ? 2 : 1) k_scatter(Ctx c) {
             o += seg[k];
         }
         pending = SG > 1;
-        PT(2);  // layout: carries, descriptors
         K kk[V], pp[V];
-        if constexpr (LDG) {
-#pragma unroll
-            for (int v = 0; v < V; ++v) kk[v] = kn[v], pp[v] = pn[v];
-            if (g + 1 < ntot) fetch(g + 1);
-        } else {
         mbar_wait(&bar, g & 1);
-        PT(3);  // TMA wait
         const uint32_t body = len & ~(uint32_t)(LU - 1);
         const K *gk = static_cast<const K *>(c.in_key[rel]) + first;
         const K *gp = static_cast<const K *>(c.in_pay[rel]) + first;
@@ -506,35 +344,8 @@ __global__ void __launch_bounds__(NT, NT <= 512 ? 2 : 1) k_scatter(Ctx c) {
                 }
             }
         }
-        }
         __syncthreads();  // S1: offsets and carries in place, stage consumed
-        PT(4);  // stage read + S1
-        if (ALIAS) {  // the stage region is free now: carries to their segment heads
-#pragma unroll
-            for (int k = 0; k < PPT; ++k)
-#pragma unroll
-                for (int i = 0; i < CW; ++i)
-                    if (i < (int)ccw[k]) sput(co[k] + i, carry[k][i]);
-        } else if (!LDG && tid == 0 && g + 1 < ntot) {
-            issue(g + 1);
-        }
-#if SCAT_ATOM_FIRST
-        uint32_t pos[V];  // final slots: all atomics first, then the stores
-#pragma unroll
-        for (int v = 0; v < V; ++v) {
-            const uint32_t i = (uint32_t)((v / LU) * NT + tid) * LU + (v % LU);
-            pos[v] = (len == T || i < len) ? atomicAdd(&off[digit1(kk[v], P)], 1u) : NONE;
-        }
-#pragma unroll
-        for (int v = 0; v < V; ++v) {
-            if (pos[v] != NONE) {
-                Tup t;
-                t.x = kk[v];
-                t.y = pp[v];
-                sput(pos[v], t);
-            }
-        }
-#else
+        if (tid == 0 && g + 1 < ntot) issue(g + 1);
 #pragma unroll
         for (int v = 0; v < V; ++v) {
             const uint32_t i = (uint32_t)((v / LU) * NT + tid) * LU + (v % LU);
@@ -545,88 +356,39 @@ __global__ void __launch_bounds__(NT, NT <= 512 ? 2 : 1) k_scatter(Ctx c) {
                 sput(atomicAdd(&off[digit1(kk[v], P)], 1u), t);
             }
         }
-#endif
         __syncthreads();  // S2
-        PT(5);  // rank + scatter into sorted + S2
-        if (ALIAS) fetch_carry();  // before the stage region is reloaded
-        // write-out, two groups per thread per step (independent load chains)
+        // write-out: one group per thread per step
         const uint32_t ngroups = total / SG;
-        constexpr int WU = SCAT_WO_UNROLL;
-        for (uint32_t u0 = tid; u0 < ngroups; u0 += WU * NT) {
-            GV gv[WU];
-            PInfo in[WU];
-            uint32_t slot[WU];
-            bool on[WU];
-#pragma unroll
-            for (int r = 0; r < WU; ++r) {
-                slot[r] = (u0 + r * NT) * SG;
-                on[r] = u0 + r * NT < ngroups;
-                if (on[r]) {
-                    if constexpr (SOA) {  // 4 keys + 4 payloads -> (k0,p0,k1,p1 | k2,p2,k3,p3)
-                        const uint4 kv = *reinterpret_cast<const uint4 *>(ks + slot[r]);
-                        const uint4 pv = *reinterpret_cast<const uint4 *>(ps + slot[r]);
-                        gv[r].a = make_uint4(kv.x, pv.x, kv.y, pv.y);
-                        gv[r].b = make_uint4(kv.z, pv.z, kv.w, pv.w);
-                    } else if constexpr (GB == 32 && EAGER) {  // two conflict-free 16-byte halves (swizzled)
-                        gv[r].a = lds128(sorted + swz(slot[r]));
-                        gv[r].b = lds128(sorted + swz(slot[r] + SG / 2));
-                    } else if constexpr (GB == 32) {
-                        gv[r].a = *reinterpret_cast<const uint4 *>(sorted + swz(slot[r]));
-                        gv[r].b = *reinterpret_cast<const uint4 *>(sorted + swz(slot[r] + SG / 2));
-                    } else {
-                        gv[r] = *reinterpret_cast<const GV *>(sorted + slot[r]);
-                    }
-                }
-            }
-            if constexpr (GD) {
-#pragma unroll
-                for (int r = 0; r < WU; ++r) {
-                    const ull d = on[r] ? gdst[slot[r] / SG] : 0ull;
-                    if (d) {
-                        char *dst = reinterpret_cast<char *>(d & ~(ull)(GB - 1));
-                        if (SCAT_RING) dst = c.arena[0] + c.lay.recv[0] + ((dst - c.arena[0] - c.lay.recv[0]) & (ull)(SCAT_RING - 1));
-                        const uint32_t h = (uint32_t)(d & (GB - 1));
-                        if (!h) {
-                            st_group<GB>(dst, gv[r]);
-                        } else {
-                            for (uint32_t i = h; i < SG; ++i) reinterpret_cast<Tup *>(dst)[i] = sget(slot[r] + i);
-                        }
-                    }
-                }
+        for (uint32_t u = tid; u < ngroups; u += NT) {
+            const uint32_t slot = u * SG;
+            GV gv;
+            PInfo in;
+            if constexpr (GB == 32 && EAGER) {  // two conflict-free 16-byte halves (swizzled)
+                gv.a = lds128(sorted + swz(slot));
+                gv.b = lds128(sorted + swz(slot + SG / 2));
+            } else if constexpr (GB == 32) {
+                gv.a = *reinterpret_cast<const uint4 *>(sorted + swz(slot));
+                gv.b = *reinterpret_cast<const uint4 *>(sorted + swz(slot + SG / 2));
             } else {
-#pragma unroll
-            for (int r = 0; r < WU; ++r) {
-                if (on[r]) {
-                    const PInfo *pi = pinfo + (reinterpret_cast<const uint32_t *>(&gv[r])[0] & (uint32_t)(P - 1));
-                    if constexpr (EAGER) {
-                        const uint4 v = lds128(pi);
-                        in[r].wb = (ull)v.x | ((ull)v.y << 32);
-                        in[r].lim = v.z;
-                        in[r].head = v.w;
-                    } else {
-                        in[r] = *pi;
-                    }
+                gv = *reinterpret_cast<const GV *>(sorted + slot);
+            }
+            const PInfo *pi = pinfo + (reinterpret_cast<const uint32_t *>(&gv)[0] & (uint32_t)(P - 1));
+            if constexpr (EAGER) {
+                const uint4 v = lds128(pi);
+                in.wb = (ull)v.x | ((ull)v.y << 32);
+                in.lim = v.z;
+                in.head = v.w;
+            } else {
+                in = *pi;
+            }
+            if (slot + SG <= in.lim) {
+                char *dst = reinterpret_cast<char *>(in.wb + (ull)slot * TB);
+                if ((in.head >> 2) != slot) {
+                    st_group<GB>(dst, gv);
+                } else {
+                    for (uint32_t i = in.head & 3u; i < SG; ++i) reinterpret_cast<Tup *>(dst)[i] = sget(slot + i);
                 }
             }
-#pragma unroll
-            for (int r = 0; r < WU; ++r) {
-                if (on[r] && slot[r] + SG <= in[r].lim) {
-                    char *dst = reinterpret_cast<char *>(in[r].wb + (ull)slot[r] * TB);
-                    if (SCAT_RING) dst = c.arena[0] + c.lay.recv[0] + ((dst - c.arena[0] - c.lay.recv[0]) & (ull)(SCAT_RING - 1));
-                    if ((in[r].head >> 2) != slot[r]) {
-                        st_group<GB>(dst, gv[r]);
-                    } else {
-                        for (uint32_t i = in[r].head & 3u; i < SG; ++i)
-                            reinterpret_cast<Tup *>(dst)[i] = sget(slot[r] + i);
-                    }
-                }
-            }
-            }
-        }
-        PT(6);  // write-out
-        if (ALIAS) {  // the sorted buffer is read: load the next sub-tile into its head
-            __syncthreads();  // S3
-            if (tid == 0 && g + 1 < ntot) issue(g + 1);
         }
     }
     if (cur_rel >= 0) flush();
@@ -645,23 +407,10 @@ __global__ void __launch_bounds__(NT, NT <= 512 ? 2 : 1) k_scatter(Ctx c) {
 
 template <typename K>
 inline void (*scatter_kernel(int P))(Ctx) {
-    if constexpr (sizeof(K) == 8) {
-        if (P <= 1024) return k_scatter<K, 4096, 2, 1, 1024, false>;
-        if (P == 2048) return k_scatter<K, 2048, 2, 2, 1024, false>;
-        return k_scatter<K, 4096, 1, 4, 1024, false>;
-    } else {
-#if SCAT_ALIAS
-        if (P <= 512) return k_scatter<K, 4096, 4, 1, 512, true>;
-        if (P == 1024) return k_scatter<K, 4096, 4, 2, 512, true>;
-#elif SCAT_2CTA
-        if (P <= 512) return k_scatter<K, 4096, 2, 1, 512, false>;
-        if (P == 1024) return k_scatter<K, 4096, 2, 2, 512, false>;
-#else
-        if (P <= 1024) return k_scatter<K, SCAT_T4, 4, 1, 1024, false>;
-#endif
-        if (P == 2048) return k_scatter<K, 4096, 4, 2, 1024, false>;
-        return k_scatter<K, 8192, 1, 4, 1024, false>;
-    }
+    constexpr ScatGeom g1 = scat_geom(1024, sizeof(K)), g2 = scat_geom(2048, sizeof(K)), g4 = scat_geom(4096, sizeof(K));
+    if (P <= 1024) return k_scatter<K, g1.T, g1.SG, g1.PPT, g1.NT>;
+    if (P == 2048) return k_scatter<K, g2.T, g2.SG, g2.PPT, g2.NT>;
+    return k_scatter<K, g4.T, g4.SG, g4.PPT, g4.NT>;
 }
 inline int scatter_threads(int P, int key_bytes) { return scat_geom(P, key_bytes).NT; }
 

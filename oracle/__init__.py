@@ -9,7 +9,9 @@ readings (C2 bag semantics, C3 checksum, C17 sorted triples).
 
 Parity status: every function here is pinned (tests/test_oracle.py):
 brute-force nested loop (tiny), closed forms (generated workloads),
-numpy multiplicity sums (sort-merge), hand-worked golden fixture.
+numpy multiplicity sums (sort-merge), per-key group-sum products for the
+pair digest (Σ_k (Σ_{R_k} a)(Σ_{S_k} b)), closed forms Σ i² and
+Σ i(n-1-i) for identical key permutations, hand-worked golden fixture.
 """
 from __future__ import annotations
 
@@ -30,7 +32,7 @@ C_WIDE = 0x9E3779B97F4A7C15  # checksum multiplier for 8-byte payloads (reading 
 
 class _Res(ctypes.Structure):
     _fields_ = [("count", ctypes.c_uint64), ("checksum", ctypes.c_uint64),
-                ("n_out", ctypes.c_uint64), ("overflow", ctypes.c_int32),
+                ("n_out", ctypes.c_uint64), ("pair_digest", ctypes.c_uint64), ("overflow", ctypes.c_int32),
                 ("status", ctypes.c_int32)]
 
 
@@ -62,7 +64,10 @@ def _ptr(a: np.ndarray):
 
 
 def join(r_keys, r_pays, s_keys, s_pays, materialize: bool = False, out_cap: int | None = None):
-    """Return dict(count, checksum[, key, pay_r, pay_s]) for the bag equi-join R ⋈ S.
+    """Return dict(count, checksum, pair_digest[, key, pay_r, pay_s]) for the bag equi-join R ⋈ S.
+
+    pair_digest = Σ_J a·b mod 2^64 (reading C3b): bilinear in the
+    matched pair, so a wrong pairing changes it.
 
     4-byte (uint32) or 8-byte (uint64) keys/payloads; both relations must use
     the same width.  Triples (if requested) are sorted by (k, a, b).
@@ -90,7 +95,7 @@ def join(r_keys, r_pays, s_keys, s_pays, materialize: bool = False, out_cap: int
     rc = fn(_ptr(rk), _ptr(ra), rk.size, _ptr(sk), _ptr(sb), sk.size, *args, ctypes.byref(res))
     if rc != 0 or res.status != 0:
         raise MemoryError("oracle: allocation failed")
-    out = {"count": int(res.count), "checksum": int(res.checksum)}
+    out = {"count": int(res.count), "checksum": int(res.checksum), "pair_digest": int(res.pair_digest)}
     if materialize:
         n = int(res.n_out)
         out.update(key=ok[:n], pay_r=oa[:n], pay_s=ob[:n], overflow=bool(res.overflow))

@@ -15,6 +15,9 @@
  *   count    = |J|
  *   checksum = sum over J of (a*C + b) mod 2^64            (reading C3)
  *              C = 2^32 for 4-byte payloads, 0x9E3779B97F4A7C15 for 8-byte
+ *   pair_digest = sum over J of a*b mod 2^64               (reading C3b)
+ *              bilinear in the pair, so it changes when an S row is paired
+ *              with the wrong R row even where count and checksum cannot
  *   triples  = J sorted by unsigned lexicographic (k, a, b)  (reading C17)
  *
  * Algorithm (SURVEY.md §8c "Algorithm"): build a chained hash table over R
@@ -34,6 +37,7 @@ typedef struct {
     uint64_t count;
     uint64_t checksum;
     uint64_t n_out;      /* triples written (<= out_cap) */
+    uint64_t pair_digest;
     int32_t  overflow;   /* 1 if count > out_cap while materialising */
     int32_t  status;     /* 0 ok, -1 out of memory */
 } oracle_result_t;
@@ -89,7 +93,7 @@ int oracle_join_k32(const uint32_t *rk, const uint32_t *ra, uint64_t nr,
         head[h] = (int64_t)i;
     }
     /* probe: for j in S order, walk chain h(k_j), emit every equal key */
-    uint64_t count = 0, checksum = 0, n_out = 0;
+    uint64_t count = 0, checksum = 0, n_out = 0, digest = 0;
     for (uint64_t j = 0; j < ns; j++) {
         uint32_t k = sk[j];
         uint64_t h = ((uint64_t)k * FIB) >> shift;
@@ -97,6 +101,7 @@ int oracle_join_k32(const uint32_t *rk, const uint32_t *ra, uint64_t nr,
             if (rk[i] != k) continue;
             count += 1;
             checksum += ((uint64_t)ra[i] << 32) + (uint64_t)sb[j]; /* a*2^32 + b */
+            digest += (uint64_t)ra[i] * (uint64_t)sb[j];            /* a*b */
             if (out_k) {
                 if (n_out < out_cap) {
                     trip[n_out].k = k; trip[n_out].a = ra[i]; trip[n_out].b = sb[j];
@@ -116,6 +121,7 @@ int oracle_join_k32(const uint32_t *rk, const uint32_t *ra, uint64_t nr,
     res->count = count;
     res->checksum = checksum;
     res->n_out = n_out;
+    res->pair_digest = digest;
     free(head); free(next); free(trip);
     return 0;
 }
@@ -156,7 +162,7 @@ int oracle_join_k64(const uint64_t *rk, const uint64_t *ra, uint64_t nr,
         next[i] = head[h];
         head[h] = (int64_t)i;
     }
-    uint64_t count = 0, checksum = 0, n_out = 0;
+    uint64_t count = 0, checksum = 0, n_out = 0, digest = 0;
     for (uint64_t j = 0; j < ns; j++) {
         uint64_t k = sk[j];
         uint64_t f = k ^ (k >> 32);
@@ -165,6 +171,7 @@ int oracle_join_k64(const uint64_t *rk, const uint64_t *ra, uint64_t nr,
             if (rk[i] != k) continue;
             count += 1;
             checksum += ra[i] * FIB + sb[j];              /* a*C + b, C = 0x9E37... */
+            digest += ra[i] * sb[j];                      /* a*b mod 2^64 */
             if (out_k) {
                 if (n_out < out_cap) {
                     trip[n_out].k = k; trip[n_out].a = ra[i]; trip[n_out].b = sb[j];
@@ -184,6 +191,7 @@ int oracle_join_k64(const uint64_t *rk, const uint64_t *ra, uint64_t nr,
     res->count = count;
     res->checksum = checksum;
     res->n_out = n_out;
+    res->pair_digest = digest;
     free(head); free(next); free(trip);
     return 0;
 }

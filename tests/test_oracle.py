@@ -3,7 +3,9 @@
 Each pin would catch a plausible oracle bug: a dropped duplicate (brute force,
 multiplicity sums), a swapped a/b or missing 2^32 factor in the checksum
 (closed forms, golden), a truncated 8-byte key (high-bits golden case), a bad
-sort (brute-force triples), an off-by-one on empty inputs (golden).
+sort (brute-force triples), an off-by-one on empty inputs (golden), a pair
+digest that sums a+b or a*a instead of a*b, or pairs S rows with the wrong R
+row (Σ i(n-1-i) closed form, per-key group-sum products, brute force).
 """
 import json
 import os
@@ -30,11 +32,17 @@ def brute_force(rk, ra, sk, sb, wide=False):
     return len(trip), checksum, trip
 
 
+def brute_digest(trip):
+    """Pair digest (reading C3b) of brute-force triples: Σ a·b mod 2^64, Python integers."""
+    return sum(a * b for _, a, b in trip) & M64
+
+
 def check_against_brute(rk, ra, sk, sb, wide=False):
     cnt, chk, trip = brute_force(rk, ra, sk, sb, wide)
     got = oracle.join(rk, ra, sk, sb, materialize=True)
     assert got["count"] == cnt
     assert got["checksum"] == chk
+    assert got["pair_digest"] == brute_digest(trip)
     gt = list(zip(got["key"].tolist(), got["pay_r"].tolist(), got["pay_s"].tolist()))
     assert gt == trip
 
@@ -92,6 +100,7 @@ def test_oracle_golden_hand_worked():
                           S[:, 1].astype(dt), materialize=True, out_cap=max(c["count"], 1))
         assert got["count"] == c["count"], c["name"]
         assert got["checksum"] == int(c["checksum"], 16), c["name"]
+        assert got["pair_digest"] == int(c["pair_digest"], 16), c["name"]
         trip = [list(t) for t in zip(got["key"].tolist(), got["pay_r"].tolist(), got["pay_s"].tolist())]
         assert trip == c["triples"], c["name"]
 
@@ -204,3 +213,45 @@ def test_oracle_sorted_triples_vs_sortmerge():
     np.testing.assert_array_equal(got["key"], ks[o])
     np.testing.assert_array_equal(got["pay_r"], as_[o])
     np.testing.assert_array_equal(got["pay_s"], bs[o])
+
+
+@pytest.mark.parametrize("n", [1 << 12, 1 << 18, 1000003])
+def test_oracle_pair_digest_closed_forms(n):
+    """R and S with the SAME key permutation: row i of S matches row i of R only.
+    Payloads (i, i) give Σ i² = (n-1)n(2n-1)/6; payloads (i, n-1-i) give
+    Σ i(n-1-i) = (n-1)·n(n-1)/2 - (n-1)n(2n-1)/6; a digest of a·a or a+b, or
+    any wrong pairing, misses at least one of the two."""
+    keys = datagen.perm_n(np.arange(n, dtype=np.uint64), n, datagen.SEED_R).astype(np.uint32)
+    ids = np.arange(n, dtype=np.uint32)
+    got = oracle.join(keys, ids, keys, ids)
+    assert got["count"] == n
+    assert got["pair_digest"] == ((n - 1) * n * (2 * n - 1) // 6) & M64
+    rev = (np.uint32(n - 1) - ids).astype(np.uint32)
+    got = oracle.join(keys, ids, keys, rev)
+    # Σ_{i<n} i (n-1-i) = (n-1) Σ i - Σ i²
+    exp = (n - 1) * (n * (n - 1) // 2) - (n - 1) * n * (2 * n - 1) // 6
+    assert got["pair_digest"] == exp & M64
+
+
+@pytest.mark.parametrize("wide", [False, True])
+@pytest.mark.parametrize("dom", [1 << 6, 1 << 14])
+def test_oracle_pair_digest_vs_group_sums(wide, dom):
+    """The digest is bilinear: Σ_J a·b = Σ_k (Σ_{R_k} a)(Σ_{S_k} b) mod 2^64 —
+    per-key sums by np.unique / np.add.at (library routines), Python integers."""
+    rng = np.random.default_rng(dom + wide)
+    dt = np.uint64 if wide else np.uint32
+    nr, ns = 50000, 70000
+    rk = rng.integers(0, dom, nr, dtype=np.uint64).astype(dt)
+    sk = rng.integers(0, dom, ns, dtype=np.uint64).astype(dt)
+    hi = 1 << 64 if wide else 1 << 32
+    ra = rng.integers(0, hi - 1, nr, dtype=np.uint64, endpoint=True).astype(dt)
+    sb = rng.integers(0, hi - 1, ns, dtype=np.uint64, endpoint=True).astype(dt)
+    ur, inv_r = np.unique(rk, return_inverse=True)
+    us, inv_s = np.unique(sk, return_inverse=True)
+    sa = np.zeros(ur.size, dtype=object)
+    np.add.at(sa, inv_r, ra.astype(object))
+    sbb = np.zeros(us.size, dtype=object)
+    np.add.at(sbb, inv_s, sb.astype(object))
+    _, ir, is_ = np.intersect1d(ur, us, assume_unique=True, return_indices=True)
+    exp = sum(int(sa[x]) * int(sbb[y]) for x, y in zip(ir, is_)) & M64
+    assert oracle.join(rk, ra, sk, sb)["pair_digest"] == exp

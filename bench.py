@@ -203,8 +203,49 @@ def emit(out, obj) -> None:
     out.flush()
 
 
+def self_launch(n: int) -> None:
+    """`bench.py --gpus N` (N > 1) started without torchrun: re-execute this
+    script under torch.distributed.run, one rank per GPU, on 127.0.0.1."""
+    import socket
+    sk = socket.socket()
+    sk.bind(("127.0.0.1", 0))
+    port = sk.getsockname()[1]
+    sk.close()
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={n}",
+           "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__), *sys.argv[1:]]
+    sys.stdout.flush()
+    sys.stderr.flush()
+    os.execv(sys.executable, cmd)
+
+
+def expected_shard(torch, kind: str, kb: int, n_r: int, s_keys, s_pays):
+    """(count, checksum, pair digest) of this rank's S shard joined with the
+    whole R, from the generator alone (no join code): R.key[i] = perm(i)
+    (mix64(perm(i)) for 8-byte keys) with payload i (2^40 + i), so the R row
+    an S key matches is i = perm^-1(key); a Zipf miss row has key >= |R|.
+    int64 arithmetic wraps modulo 2^64 like the C3 / C3b sums."""
+    from paper_conf_sigmod_paullhl21_b200 import datagen
+    k = datagen.ceil_log2(n_r)
+    assert n_r == 1 << k, "closed-form check needs |R| = 2^k"
+    if kb == 4:
+        key = s_keys.long() & 0xFFFFFFFF
+        b = s_pays.long() & 0xFFFFFFFF
+    else:
+        key = datagen.unmix64_t(s_keys.long())
+        b = s_pays.long()
+    hit = key < n_r if kind == "zipf" else torch.ones_like(key, dtype=torch.bool)
+    i = datagen.perm_k_inverse_t(key, k, datagen.SEED_R)
+    a = i if kb == 4 else i + (1 << 40)
+    a = torch.where(hit, a, torch.zeros_like(a))
+    b = torch.where(hit, b, torch.zeros_like(b))
+    chk = (a << 32) + b if kb == 4 else a * datagen._s64(0x9E3779B97F4A7C15) + b
+    return int(hit.sum()), int(chk.sum()), int((a * b).sum())
+
+
 def main():
     a = parse()
+    if a.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        self_launch(a.gpus)
     out = _claim_stdout()
     if a.impl == "reference":
         run_reference(a, out)
@@ -276,17 +317,6 @@ def main():
     for _ in range(max(a.warmup, 1)):
         step()
         res = join.result()
-    # closed forms (tests/golden/appendix_a_closed_forms.json)
-    M64 = (1 << 64) - 1
-    if a.workload == "unique":
-        n = n_r
-        expect_ok = res["match_count"] == n and res["checksum"] == ((1 << 32) + 1) * n * (n - 1) // 2 & M64
-    elif a.workload == "wide":
-        n, h = n_r, n_r * (n_r - 1) // 2
-        chk = (0x9E3779B97F4A7C15 * (n * (1 << 40) + h) + n * (1 << 41) + h) & M64
-        expect_ok = res["match_count"] == n and res["checksum"] == chk
-    else:  # zipf: every even S row matches exactly one R tuple, odd rows never match
-        expect_ok = res["match_count"] == n_s // 2
 
     sampler = ClockSampler(local) if (rank == 0 and not a.profile) else None
     if sampler:
@@ -299,11 +329,29 @@ def main():
         step()
         evs[i + 1].record(stream)
     barrier()
-    res = join.result()
+    res = join.result()  # the last timed step's result (a6 ran inside it)
     clocks = sampler.stop() if sampler else None
-    ok_timed = res["status"] == 0 and res["match_count"] == res["match_count"]
-    phases = []
-    for _ in range(3):  # per-phase breakdown from separate (untimed) steps
+
+    # correctness of the timed run: global count, checksum and pair digest
+    # against the generator-derived values (every workload; SURVEY.md §8c
+    # closed forms, readings C3 / C3b), summed over the ranks' S shards
+    M64 = (1 << 64) - 1
+    exp = list(expected_shard(torch, a.workload, kb, n_r, cols[2], cols[3]))
+    if world > 1:
+        t = torch.tensor([x - (1 << 64) if x >= 1 << 63 else x for x in (v & M64 for v in exp)],
+                         dtype=torch.int64, device=dev)
+        dist.all_reduce(t)  # int64 sums wrap modulo 2^64
+        exp = [int(x) for x in t.tolist()]
+    exp_count, exp_chk, exp_dig = exp[0] & M64, exp[1] & M64, exp[2] & M64
+    expect_ok = (res["status"] == 0 and res["match_count"] == exp_count and res["checksum"] == exp_chk
+                 and res["pair_digest"] == exp_dig)
+    if a.workload == "unique":  # Appendix A closed forms as well
+        n = n_r
+        expect_ok = expect_ok and exp_count == n and exp_chk == ((1 << 32) + 1) * n * (n - 1) // 2 & M64
+    # per-phase breakdown: the last timed step's phase events (the library records
+    # them on the join stream around each phase), plus three untimed steps
+    phases = [res["phase_ms"]]
+    for _ in range(3):
         step()
         phases.append(join.result()["phase_ms"])
     step_ms = [evs[i].elapsed_time(evs[i + 1]) for i in range(a.steps)]
@@ -382,7 +430,8 @@ def main():
             t = torch.tensor([t_e2e], device=dev)
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
             t_e2e = float(t.item())
-        assert r2["match_count"] == res["match_count"]
+        assert (r2["match_count"], r2["checksum"], r2["pair_digest"]) == \
+            (res["match_count"], res["checksum"], res["pair_digest"])
         e2e = {"value": tuples_job / (t_e2e / a.e2e_steps), "unit": UNIT,
                "h2d_bytes_per_step": int(sum(h.numel() * h.element_size() for h in host)),
                "d2h_bytes_per_step": 32 + 64, "steps": a.e2e_steps,
@@ -407,8 +456,10 @@ def main():
                                    else "NCCL all_to_all_single baseline (host sync per step for split sizes)"),
                        "global_batch": tuples_job, "seeds": {"R": "0x5EED0052", "S": "0x5EED0053"},
                        "skew_bcast": a.skew_bcast},
-            "correct": bool(expect_ok) and res["status"] == 0,
+            "correct": bool(expect_ok),
+            "correct_from": "the last timed step's result (count, checksum, pair digest vs generator-derived values)",
             "match_count": res["match_count"], "checksum": hex(res["checksum"]),
+            "pair_digest": hex(res["pair_digest"]),
             "gpu_cycles_per_tuple": {"sm_cycles_per_tuple": cyc * nsm, "gpu_cycles_per_tuple": cyc,
                                      "sm_mhz": sm_mhz, "sms": nsm,
                                      "formula": "T*f_SM*SMs*N/(|R|+|S|) and T*f_SM*N/(|R|+|S|)"},

@@ -12,9 +12,11 @@
  * global partitioning = partition + assignment + data distribution
  * (§4), local partitioning and probe.
  *
- * Result (readings C1-C3): match count, a 64-bit checksum
+ * Result (readings C1-C3, C3b): match count, a 64-bit checksum
  *   checksum = sum over matches (k,a,b) of (a*C + b) mod 2^64,
  *   C = 2^32 for 4-byte payloads, 0x9E3779B97F4A7C15 for 8-byte payloads,
+ * a 64-bit pair digest
+ *   pair_digest = sum over matches (k,a,b) of a*b mod 2^64,
  * and optionally the materialised (key, payloadR, payloadS) triples (bag
  * semantics: every equal-key (R,S) pair once).
  *
@@ -28,8 +30,8 @@
  *    be made by every rank in the same order, like NCCL.  They only enqueue
  *    work on the given CUDA stream (passed as void*, a cudaStream_t) and
  *    return.  Several ranks may live in ONE process on ONE GPU ("virtual
- *    ranks", each with its own handle): then call each phase for all ranks
- *    before the next phase, on one stream.
+ *    ranks", each with its own handle and its own stream): then call each
+ *    phase for all ranks before the next phase.
  *  - Ownership: input columns are borrowed (valid until mgj_join's work has
  *    completed).  The handle owns its workspace and the materialised output
  *    (valid until the next mgj_partition or mgj_destroy).  A caller-provided
@@ -78,7 +80,9 @@ typedef struct {
                                           every rank from its owner, S_p stays where it is), -1 = never,
                                           1 = every partition passing the traffic test.  Never with one
                                           rank or MGJ_SHUFFLE_EXTERNAL */
-    int32_t  reserved[5];              /* must be zero */
+    int32_t  peer_timeout_ms;          /* bound on every wait for a peer's signal (0 = 20000 ms); a wait
+                                          that times out makes the run fail with MGJ_EPEER */
+    int32_t  reserved[4];              /* must be zero */
 } mgj_config;
 
 /*
@@ -122,7 +126,10 @@ typedef struct {
     int32_t  radix_bits_global;    /* B1 used */
     int32_t  radix_bits_local;     /* B2 chosen on device for this rank */
     int32_t  n_items;              /* probe work items (co-partition slices) on this rank */
-    int32_t  n_launches;           /* kernels this handle launched for the run (partition .. result) */
+    int32_t  n_launches;           /* kernels this handle launched for the run (partition .. join) */
+    uint64_t pair_digest;          /* global sum over matches (k,a,b) of a*b mod 2^64 (DESIGN.md reading
+                                      C3b): bilinear, so it detects a wrong pairing of R and S rows */
+    uint64_t local_pair_digest;    /* this rank's co-partitions */
 } mgj_result_t;
 
 /* Bytes each rank's symmetric arena needs for cfg (0 if cfg is invalid). */
@@ -160,8 +167,12 @@ mgj_status mgj_shuffle(mgj_handle h, void *stream);
  * Phases a4 + a5 + a6: waits for every rank's data, radix
  * partitions the received segments by the next B2 key bits into
  * shared-memory-sized co-partitions, builds a shared-memory hash table per
- * R co-partition and probes it with S, then sums (count, checksum) over
- * ranks.  Materialised triples stay on the owning rank.
+ * R co-partition and probes it with S, then sums (count, checksum, pair
+ * digest) over ranks (a6: each rank stores its partial sums into every
+ * peer's arena, raises a flag, and waits for all N).  Materialised triples
+ * stay on the owning rank.  Because a6 waits for every peer inside the
+ * enqueued work, ranks that share one GPU ("virtual ranks") must each use
+ * their own stream.
  */
 mgj_status mgj_join(mgj_handle h, void *stream);
 
@@ -181,7 +192,8 @@ typedef struct {
 
 mgj_status mgj_exchange_layout(mgj_handle h, mgj_exchange_t *out);
 
-/* Synchronise the last stream and fill *out.  Returns the run's sticky status. */
+/* Synchronise the last stream and fill *out (no device work is enqueued).
+ * Returns the run's sticky status. */
 mgj_status mgj_result(mgj_handle h, mgj_result_t *out);
 
 void        mgj_destroy(mgj_handle h);

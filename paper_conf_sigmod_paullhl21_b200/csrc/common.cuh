@@ -32,8 +32,9 @@ constexpr int MAX_BA = 6;               // two-level local partitioning: at most
 constexpr int LOCAL2_NCH = 256;         // a partition of more chunks than this gets the first local pass
 // sub-partitions of a first local pass: at most local2_vcap(P) in total
 __host__ __device__ constexpr int local2_vcap(int P) { return 4 * P > 4096 ? 4 * P : 4096; }
-constexpr uint64_t WAIT_TIMEOUT_NS = 20ull * 1000 * 1000 * 1000;
+constexpr uint64_t WAIT_TIMEOUT_NS = 20ull * 1000 * 1000 * 1000;  // default peer-signal wait bound
 
+constexpr int RES_W = 8;  // u64 words per rank in the result mailbox (a6)
 enum Sig { SIG_HIST = 0, SIG_DATA = 1, SIG_RES = 2, SIG_COUNT = 3 };
 enum Ticket { TK_HIST = 0, TK_SCAT_R = 1, TK_SCAT_S = 2, TK_SCAT_DONE = 3, TK_ITEMS = 4,
               TK_PROBE = 5, TK_LOCAL = 6, TK_COUNT = 8 };
@@ -59,7 +60,8 @@ __host__ __device__ __forceinline__ int piece_src(uint64_t v) { return (int)(v >
 struct Arena {
     uint64_t sig;      // u64 flags[SIG_COUNT][MAX_RANKS], written by peers
     uint64_t mail;     // u32 hist[MAX_RANKS][2][P]
-    uint64_t resmail;  // u64 res[MAX_RANKS][4] (count, checksum, n_out, status)
+    uint64_t resmail;  // u64 res[MAX_RANKS][RES_W] (count, checksum, n_out, status, pair digest)
+    uint64_t cfgmail;  // u64 cfg[MAX_RANKS][4] (recv_cap R, recv_cap S, arena bytes, B1) published with a1
     uint64_t recv[2];  // received tuples of R, S
     uint64_t total;
 };
@@ -93,6 +95,7 @@ struct Ctx {
     int32_t ext;                  // shuffle mode EXTERNAL: scatter into send_buf, caller exchanges
     uint32_t max_items;
     uint64_t epoch;
+    uint64_t timeout_ns;          // bound on a wait for peer signals (mgj_config.peer_timeout_ms)
     uint64_t recv_cap[2];
     uint64_t max_chunks;
     uint64_t out_cap;
@@ -136,9 +139,9 @@ struct Ctx {
     uint32_t *cop_slots;          // [2][P][2^b2_max] padded slots per co-partition
     Item *items;                  // [max_items]
     void *local[2];               // locally partitioned tuples (a4 output), chunk regions
-    unsigned long long *acc;      // [4] local count, checksum, n_out
+    unsigned long long *acc;      // [4] local count, checksum, n_out, pair digest
     int32_t *err;                 // sticky device status
-    unsigned long long *result;   // [4] global count, checksum; local n_out; status
+    unsigned long long *result;   // [8] global count, checksum; local n_out; status; global pair digest
     void *out_key, *out_a, *out_b;
 };
 
@@ -181,7 +184,7 @@ __device__ inline bool wait_all_flags(const Ctx &c, int kind) {
     for (int g = 0; g < c.world; ++g) {
         const uint64_t *f = sig_ptr(c.arena[c.rank], c.lay, kind, g);
         while (ld_acquire_sys(f) < c.epoch) {
-            if (globaltimer() - t0 > WAIT_TIMEOUT_NS) {
+            if (globaltimer() - t0 > c.timeout_ns) {
                 set_err(c, MGJ_EPEER);
                 return false;
             }
@@ -228,6 +231,18 @@ __device__ __forceinline__ unsigned long long chk_term(T a, T b) {
         return ((unsigned long long)(uint32_t)a << 32) + (uint32_t)b;
     } else {
         return (unsigned long long)a * 0x9E3779B97F4A7C15ull + (unsigned long long)b;
+    }
+}
+
+// Pair-digest term a*b mod 2^64 (reading C3b): bilinear in the
+// matched (R, S) pair, so a wrong pairing changes the digest even where the
+// linear checksum cannot.
+template <typename T>
+__device__ __forceinline__ unsigned long long dig_term(T a, T b) {
+    if constexpr (sizeof(T) == 4) {
+        return (unsigned long long)(uint32_t)a * (uint32_t)b;
+    } else {
+        return (unsigned long long)a * (unsigned long long)b;
     }
 }
 

@@ -169,6 +169,11 @@ __global__ void __launch_bounds__(HIST_THREADS, 2) k_hist(Ctx c) {
     for (int d = 0; d < c.world; ++d) {
         uint32_t *mb = reinterpret_cast<uint32_t *>(c.arena[d] + c.lay.mail) + (size_t)c.rank * 2 * P;
         for (int j = threadIdx.x; j < 2 * P; j += blockDim.x) mb[j] = __ldcg(&c.rank_hist[j]);
+        // this rank's job-wide configuration words, checked equal on every rank by k_plan
+        if (threadIdx.x < 4) {
+            const uint64_t w[4] = {c.recv_cap[0], c.recv_cap[1], c.lay.total, (uint64_t)c.B1};
+            reinterpret_cast<uint64_t *>(c.arena[d] + c.lay.cfgmail)[c.rank * 4 + threadIdx.x] = w[threadIdx.x];
+        }
     }
     __threadfence_system();
     __syncthreads();
@@ -306,6 +311,21 @@ __global__ void __launch_bounds__(1024) k_plan(Ctx c) {
     }
     if (tid < MAX_RANKS) first[tid] = endp[tid] = P, bcs[tid] = 0;
     __syncthreads();
+    if (tid == 0 && ok) {
+        // the capacities and the arena layout are job-wide (mgj.h): every rank
+        // must have planned with the same ones, else peers store at offsets
+        // that differ from the receiver's layout
+        const uint64_t *cf = reinterpret_cast<const uint64_t *>(c.arena[c.rank] + c.lay.cfgmail);
+        const uint64_t w[4] = {c.recv_cap[0], c.recv_cap[1], c.lay.total, (uint64_t)c.B1};
+        for (int g = 0; g < N && ok; ++g)
+            for (int i = 0; i < 4; ++i)
+                if (__ldcg(cf + g * 4 + i) != w[i]) {
+                    set_err(c, MGJ_EINVAL);
+                    ok = 0;
+                    break;
+                }
+    }
+    __syncthreads();
     if (!ok) {
         if (tid == 0) c.meta[MT_OK] = 0;
         return;
@@ -386,6 +406,9 @@ __global__ void __launch_bounds__(1024) k_plan(Ctx c) {
         if (d < N && rel) size += bcs[d];
         c.recv_size[rel * MAX_RANKS + d] = size;
         if (size > c.recv_cap[rel]) atomicOr(&cap_bad, 1);
+        // EXTERNAL: the send arena holds this rank's whole input per relation
+        // in a region of recv_cap tuples
+        if (c.ext && d == 0 && c.n_in[rel] > c.recv_cap[rel]) atomicOr(&cap_bad, 1);
     }
     const int plo = first[c.rank] < P ? first[c.rank] : 0;
     const int phi = first[c.rank] < P ? endp[c.rank] : 0;

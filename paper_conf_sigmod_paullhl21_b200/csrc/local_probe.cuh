@@ -522,8 +522,12 @@ __global__ void k_itemize(Ctx c) {
             x.it.s = Side{0, 0, x.nch[1], 0};
             x.soff = r;
             const uint32_t b = atomicAdd(&c.ticket[TK_ITEMS], 1u);
-            if (b < c.max_items) items[b] = x;
-            else set_err(c, MGJ_ECAPACITY);
+            if (b < c.max_items) {
+                items[b] = x;
+            } else {  // the probe must not read reserved-but-unwritten items: it is skipped
+                set_err(c, MGJ_ECAPACITY);
+                c.meta[MT_OK] = 0;
+            }
             continue;
         }
         // slow path: slice both sides, pair every R slice with every S slice
@@ -541,6 +545,7 @@ __global__ void k_itemize(Ctx c) {
         const uint32_t b = atomicAdd(&c.ticket[TK_ITEMS], (uint32_t)min(n, (uint64_t)0x7fffffffu));
         if ((uint64_t)b + n > c.max_items) {
             set_err(c, MGJ_ECAPACITY);
+            c.meta[MT_OK] = 0;
             continue;
         }
         uint32_t ir = 0;
@@ -720,7 +725,7 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
 
     // ------------------------------------------------------------ consumers
     const int ct = tid - 32 * PROBE_NP;
-    unsigned long long my_cnt = 0, my_chk = 0;
+    unsigned long long my_cnt = 0, my_chk = 0, my_dig = 0;  // count, checksum, pair digest
     uint32_t tag = 0;
     // stage and parity advance incrementally; barrier addresses computed once
     const uint32_t full_at = smem_u32(&full[0]), empty_at = smem_u32(&empty[0]);
@@ -819,6 +824,7 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
                     walk(x, sv, [&](K a, uint32_t i) {
                         ++m_item;
                         my_chk += chk_term(a, (K)sv.y);
+                        my_dig += dig_term(a, (K)sv.y);
                         if (mi[k] == END) mi[k] = (uint16_t)i;
                         else ovf = true;
                     });
@@ -829,6 +835,7 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
                 walk(x, sv, [&](K a, uint32_t) {
                     ++m_item;
                     my_chk += chk_term(a, (K)sv.y);
+                    my_dig += dig_term(a, (K)sv.y);
                     ovf = true;
                 });
             }
@@ -851,6 +858,7 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
                     if ((l >> 16) == khi) {
                         ++m_item;
                         my_chk += chk_term((K)a, (K)b);
+                        my_dig += dig_term((K)a, (K)b);
                     }
                     i = l & 0xffffu;
                 }
@@ -861,6 +869,7 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
                 walk(x, sv, [&](K a, uint32_t) {
                     ++m_item;
                     my_chk += chk_term(a, (K)sv.y);
+                    my_dig += dig_term(a, (K)sv.y);
                 });
             }
         }
@@ -972,40 +981,36 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
     }
     my_cnt = warp_sum(my_cnt);
     my_chk = warp_sum(my_chk);
-    if (lane == 0 && (my_cnt || my_chk)) {
+    my_dig = warp_sum(my_dig);
+    if (lane == 0 && (my_cnt || my_chk || my_dig)) {
         atomicAdd(&c.acc[0], my_cnt);
         atomicAdd(&c.acc[1], my_chk);
+        atomicAdd(&c.acc[3], my_dig);
     }
 }
 
 // ---------------------------------------------------------------------------
-// a6: count = sum_g count_g, checksum = sum_g checksum_g (mod 2^64), split in
-// two so that several ranks can share one stream (virtual ranks):
-//  k_publish (end of mgj_join): store this rank's (count, checksum, n_out,
-//    status) in every peer's arena and raise SIG_RES there;
-//  k_gather (mgj_result): wait for every rank's SIG_RES and sum the N entries
-//    (order-free, bit-exact).
+// a6: count = sum_g count_g, checksum = sum_g checksum_g, digest = sum_g
+// digest_g (mod 2^64), the last step of mgj_join.  Thread 0 stores this
+// rank's (count, checksum, n_out, status, digest) into every peer's result
+// mailbox, raises SIG_RES there, waits for every rank's SIG_RES and sums the
+// N entries (order-free, bit-exact).  Mailbox reuse across runs is safe: a
+// rank publishes run e+1 only after k_plan(e+1) saw every rank's SIG_HIST of
+// e+1, which each rank raises after its own k_reduce(e) (stream order).
 // ---------------------------------------------------------------------------
-__global__ void k_publish(Ctx c) {
+__global__ void k_reduce(Ctx c) {
     if (threadIdx.x != 0 || blockIdx.x != 0) return;
     const int32_t st = *(volatile int32_t *)c.err;
-    const unsigned long long v[4] = {__ldcg(&c.acc[0]), __ldcg(&c.acc[1]), __ldcg(&c.acc[2]),
-                                     (unsigned long long)(uint32_t)st};
+    const unsigned long long v[5] = {__ldcg(&c.acc[0]), __ldcg(&c.acc[1]), __ldcg(&c.acc[2]),
+                                     (unsigned long long)(uint32_t)st, __ldcg(&c.acc[3])};
     for (int d = 0; d < c.world; ++d) {
         volatile unsigned long long *rm =
-            reinterpret_cast<unsigned long long *>(c.arena[d] + c.lay.resmail) + c.rank * 4;
-        rm[0] = v[0];
-        rm[1] = v[1];
-        rm[2] = v[2];
-        rm[3] = v[3];
+            reinterpret_cast<unsigned long long *>(c.arena[d] + c.lay.resmail) + c.rank * RES_W;
+        for (int i = 0; i < 5; ++i) rm[i] = v[i];
     }
     __threadfence_system();
     signal_all(c, SIG_RES);
-}
-
-__global__ void k_gather(Ctx c) {
-    if (threadIdx.x != 0 || blockIdx.x != 0) return;
-    unsigned long long cnt = 0, chk = 0;
+    unsigned long long cnt = 0, chk = 0, dig = 0;
     int32_t gst = 0;
     if (!wait_all_flags(c, SIG_RES)) {
         gst = MGJ_EPEER;
@@ -1013,16 +1018,18 @@ __global__ void k_gather(Ctx c) {
         const volatile unsigned long long *rm =
             reinterpret_cast<const unsigned long long *>(c.arena[c.rank] + c.lay.resmail);
         for (int g = 0; g < c.world; ++g) {
-            cnt += rm[g * 4 + 0];
-            chk += rm[g * 4 + 1];
-            const int32_t s = (int32_t)(uint32_t)rm[g * 4 + 3];
+            cnt += rm[g * RES_W + 0];
+            chk += rm[g * RES_W + 1];
+            dig += rm[g * RES_W + 4];
+            const int32_t s = (int32_t)(uint32_t)rm[g * RES_W + 3];
             if (gst == 0 && s != 0) gst = s;
         }
     }
     c.result[0] = cnt;
     c.result[1] = chk;
-    c.result[2] = __ldcg(&c.acc[2]);
+    c.result[2] = v[2];
     c.result[3] = (unsigned long long)(uint32_t)gst;
+    c.result[4] = dig;
 }
 
 }  // namespace mgj

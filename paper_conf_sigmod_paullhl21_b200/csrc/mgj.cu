@@ -42,8 +42,9 @@ int ceil_log2(uint64_t x) {
 mgj_status normalize(const mgj_config *in, Norm *o) {
     if (!in) return MGJ_EINVAL;
     mgj_config c = *in;
-    for (int i = 0; i < 5; ++i)
+    for (int i = 0; i < 4; ++i)
         if (c.reserved[i]) return MGJ_EINVAL;
+    if (c.peer_timeout_ms < 0) return MGJ_EINVAL;
     if (c.skew_bcast < -1 || c.skew_bcast > 1) return MGJ_EINVAL;
     if (c.local_split_bits < -1 || c.local_split_bits > MAX_BA) return MGJ_EINVAL;
     if (c.shuffle_mode != MGJ_SHUFFLE_P2P && c.shuffle_mode != MGJ_SHUFFLE_EXTERNAL) return MGJ_EINVAL;
@@ -116,6 +117,8 @@ mgj_status normalize(const mgj_config *in, Norm *o) {
     L.mail = off;
     off = align_up(off + (uint64_t)MAX_RANKS * 2 * o->P * 4, 4096);
     L.resmail = off;
+    off = align_up(off + MAX_RANKS * RES_W * 8, 4096);
+    L.cfgmail = off;
     off = align_up(off + MAX_RANKS * 4 * 8, 4096);
     L.recv[0] = off;
     off = align_up(off + o->recv_cap[0] * o->tuple_bytes, 4096);
@@ -147,7 +150,7 @@ struct mgj_plan_s {
     cudaEvent_t ev[7] = {};
     void *stage = nullptr;
     size_t stage_bytes = 0;
-    unsigned long long *h_res = nullptr;  // pinned [4] + meta [16 ints]
+    unsigned long long *h_res = nullptr;  // pinned result [8] + meta [MT_COUNT ints]
     int32_t *h_meta = nullptr;
     uint64_t recv_r = 0, recv_s = 0;
     int32_t host_err = 0;
@@ -253,8 +256,8 @@ void launch_join(mgj_plan_s *h, cudaStream_t s) {
     else
         k_probe<K, false><<<h->nsm, PROBE_THREADS, probe_smem(n), s>>>(h->ctx);
     cudaEventRecord(h->ev[5], s);
-    k_publish<<<1, 32, 0, s>>>(h->ctx);
-    h->launches += 4;  // local, itemize, probe, publish
+    k_reduce<<<1, 32, 0, s>>>(h->ctx);  // a6: cross-rank sums (inside the step)
+    h->launches += 4;  // local, itemize, probe, reduce
 }
 
 }  // namespace
@@ -294,6 +297,7 @@ mgj_status mgj_plan(const mgj_config *cfg, const mgj_peers *peers, mgj_handle *o
             if (!peers->arena_ptrs[g] || ((uintptr_t)peers->arena_ptrs[g] & 15)) return MGJ_EALIGN;
     } else if (peers && peers->arena_ptrs) {
         if (peers->arena_bytes < n.lay.total || !peers->arena_ptrs[0]) return MGJ_EINVAL;
+        if ((uintptr_t)peers->arena_ptrs[0] & 15) return MGJ_EALIGN;  // TMA reads the receive buffers
     }
     mgj_plan_s *h = new (std::nothrow) mgj_plan_s();
     if (!h) return MGJ_ENOMEM;
@@ -345,6 +349,7 @@ mgj_status mgj_plan(const mgj_config *cfg, const mgj_peers *peers, mgj_handle *o
     c.probe_slots = n.probe_slots;
     c.probe_target = n.probe_target;
     c.materialize = n.c.materialize;
+    c.timeout_ns = (n.c.peer_timeout_ms ? (uint64_t)n.c.peer_timeout_ms : 20000ull) * 1000000ull;
     c.ext = n.c.shuffle_mode == MGJ_SHUFFLE_EXTERNAL;
     c.max_items = (uint32_t)n.max_items;
     c.recv_cap[0] = n.recv_cap[0];
@@ -404,8 +409,8 @@ mgj_status mgj_plan(const mgj_config *cfg, const mgj_peers *peers, mgj_handle *o
         c.out_a = dalloc(h, n.out_cap * n.c.key_bytes, &st);
         c.out_b = dalloc(h, n.out_cap * n.c.key_bytes, &st);
     }
-    if (st == MGJ_OK) st = cuda_ok(cudaMallocHost(&h->h_res, 4 * 8 + MT_COUNT * 4));
-    if (st == MGJ_OK) h->h_meta = reinterpret_cast<int32_t *>(h->h_res + 4);
+    if (st == MGJ_OK) st = cuda_ok(cudaMallocHost(&h->h_res, 8 * 8 + MT_COUNT * 4));
+    if (st == MGJ_OK) h->h_meta = reinterpret_cast<int32_t *>(h->h_res + 8);
     for (int i = 0; i < 7 && st == MGJ_OK; ++i) st = cuda_ok(cudaEventCreate(&h->ev[i]));
     if (st == MGJ_OK) st = cuda_ok(n.c.key_bytes == 4 ? set_attrs<uint32_t>(n) : set_attrs<uint64_t>(n));
     if (st != MGJ_OK) {
@@ -509,10 +514,8 @@ mgj_status mgj_join(mgj_handle h, void *stream) {
 mgj_status mgj_result(mgj_handle h, mgj_result_t *out) {
     if (!h || !out) return MGJ_EINVAL;
     if (h->state != ST_JOINED && h->state != ST_DONE) return MGJ_ESTATE;
-    if (h->state == ST_JOINED) {  // a6: wait for every rank's partial result and sum
-        k_gather<<<1, 32, 0, h->stream>>>(h->ctx);
-        h->launches += 1;
-        cudaMemcpyAsync(h->h_res, h->ctx.result, 4 * 8, cudaMemcpyDeviceToHost, h->stream);
+    if (h->state == ST_JOINED) {  // read back the sums k_reduce (end of mgj_join) left
+        cudaMemcpyAsync(h->h_res, h->ctx.result, 8 * 8, cudaMemcpyDeviceToHost, h->stream);
         cudaMemcpyAsync(h->h_meta, h->ctx.meta, MT_COUNT * 4, cudaMemcpyDeviceToHost, h->stream);
     }
     if (cudaStreamSynchronize(h->stream) != cudaSuccess) return MGJ_ECUDA;
@@ -520,12 +523,14 @@ mgj_status mgj_result(mgj_handle h, mgj_result_t *out) {
     const Ctx &c = h->ctx;
     uint64_t rs[2 * MAX_RANKS] = {};
     if (cudaMemcpy(rs, c.recv_size, sizeof(rs), cudaMemcpyDeviceToHost) != cudaSuccess) return MGJ_ECUDA;
-    unsigned long long acc[3] = {};
+    unsigned long long acc[4] = {};
     if (cudaMemcpy(acc, c.acc, sizeof(acc), cudaMemcpyDeviceToHost) != cudaSuccess) return MGJ_ECUDA;
     out->match_count = h->h_res[0];
     out->checksum = h->h_res[1];
     out->local_count = acc[0];
     out->local_checksum = acc[1];
+    out->pair_digest = h->h_res[4];
+    out->local_pair_digest = acc[3];
     out->n_materialized = std::min<uint64_t>(h->h_res[2], h->n.out_cap);
     out->out_key = c.out_key;
     out->out_payload_r = c.out_a;

@@ -221,3 +221,75 @@ def M4(z: float, world: int = 8) -> Workload:
 
 def M5(world: int = 8) -> Workload:
     return Workload("wide", world << 28, world << 28)
+
+
+# ---------------------------------------------------------------- inverses
+# The generator's bijections inverted, so that a full-size check can find the
+# R row an S key was drawn from without any join: R.key[i] = perm_k(i) (or
+# mix64(perm_k(i)) for 8-byte keys), hence i = perm_k^-1(key).  Generator
+# arithmetic only (no join arithmetic); pinned by tests/test_datagen.py.
+_PERM_MUL = (0x9E3779B1, 0x85EBCA6B, 0xC2B2AE35)
+_PERM_INV = tuple(pow(c, -1, 1 << 32) for c in _PERM_MUL)  # inverses mod 2^32 (also mod 2^k, k <= 32)
+_MIX_MUL = (0xBF58476D1CE4E5B9, 0x94D049BB133111EB)
+_MIX_INV = tuple(pow(c, -1, 1 << 64) for c in _MIX_MUL)
+
+
+def perm_k_inverse(y: np.ndarray, k: int, seed: int) -> np.ndarray:
+    """x with perm_k(x, k, seed) == y (y in [0, 2^k)).  x ^= x >> h is an
+    involution on [0, 2^k) because 2h >= k."""
+    assert 1 <= k <= 32
+    x = np.asarray(y, dtype=_U64).copy()
+    M = _U64((1 << k) - 1)
+    h = _U64((k + 1) // 2)
+    x ^= x >> h
+    x = (x * _U64(_PERM_INV[2])) & M
+    x ^= x >> h
+    x = (x * _U64(_PERM_INV[1])) & M
+    x ^= x >> h
+    x = (x * _U64(_PERM_INV[0])) & M
+    return (x ^ _U64(seed & _MASK64)) & M
+
+
+def unmix64(z: np.ndarray) -> np.ndarray:
+    """Inverse of mix64."""
+    z = np.asarray(z, dtype=_U64).copy()
+    z = z ^ (z >> _U64(31)) ^ (z >> _U64(62))
+    z = z * _U64(_MIX_INV[1])
+    z = z ^ (z >> _U64(27)) ^ (z >> _U64(54))
+    z = z * _U64(_MIX_INV[0])
+    return z ^ (z >> _U64(30)) ^ (z >> _U64(60))
+
+
+def _s64(c: int) -> int:
+    """u64 constant as the int64 with the same bits (torch has no uint64 arithmetic)."""
+    return c - (1 << 64) if c >= 1 << 63 else c
+
+
+def _lsr_t(x, s: int):
+    """Logical right shift of an int64 torch tensor holding u64 bits."""
+    return (x >> s) & ((1 << (64 - s)) - 1)
+
+
+def perm_k_inverse_t(y, k: int, seed: int):
+    """perm_k_inverse on an int64 torch tensor (values in [0, 2^k)), on its device.
+    int64 products wrap modulo 2^64, so the low k bits are exact."""
+    assert 1 <= k <= 32
+    M = (1 << k) - 1
+    h = (k + 1) // 2
+    x = y & M
+    x = x ^ (x >> h)
+    x = (x * _PERM_INV[2]) & M
+    x = x ^ (x >> h)
+    x = (x * _PERM_INV[1]) & M
+    x = x ^ (x >> h)
+    x = (x * _PERM_INV[0]) & M
+    return (x ^ (seed & M)) & M
+
+
+def unmix64_t(z):
+    """unmix64 on an int64 torch tensor holding u64 bits."""
+    z = z ^ _lsr_t(z, 31) ^ _lsr_t(z, 62)
+    z = z * _s64(_MIX_INV[1])
+    z = z ^ _lsr_t(z, 27) ^ _lsr_t(z, 54)
+    z = z * _s64(_MIX_INV[0])
+    return z ^ _lsr_t(z, 30) ^ _lsr_t(z, 60)

@@ -48,7 +48,7 @@ class Config(ctypes.Structure):
                 ("materialize", ctypes.c_int32), ("num_sms", ctypes.c_int32),
                 ("out_capacity", ctypes.c_uint64), ("shuffle_mode", ctypes.c_int32),
                 ("local_split_bits", ctypes.c_int32), ("skew_bcast", ctypes.c_int32),
-                ("reserved", ctypes.c_int32 * 5)]
+                ("peer_timeout_ms", ctypes.c_int32), ("reserved", ctypes.c_int32 * 4)]
 
 
 class Exchange(ctypes.Structure):
@@ -70,7 +70,8 @@ class Result(ctypes.Structure):
                 ("recv_r", ctypes.c_uint64), ("recv_s", ctypes.c_uint64),
                 ("phase_ms", ctypes.c_float * 6), ("status", ctypes.c_int32),
                 ("radix_bits_global", ctypes.c_int32), ("radix_bits_local", ctypes.c_int32),
-                ("n_items", ctypes.c_int32), ("n_launches", ctypes.c_int32)]
+                ("n_items", ctypes.c_int32), ("n_launches", ctypes.c_int32),
+                ("pair_digest", ctypes.c_uint64), ("local_pair_digest", ctypes.c_uint64)]
 
 
 _H = ctypes.c_void_p
@@ -131,7 +132,8 @@ def _stream(stream):
 
 def make_config(rank=0, world_size=1, key_bytes=4, r_capacity=0, s_capacity=0, recv_capacity_r=0,
                 recv_capacity_s=0, radix_bits_global=0, radix_bits_local=0, materialize=False,
-                num_sms=0, out_capacity=0, shuffle_mode=0, local_split_bits=0, skew_bcast=0) -> Config:
+                num_sms=0, out_capacity=0, shuffle_mode=0, local_split_bits=0, skew_bcast=0,
+                peer_timeout_ms=0) -> Config:
     c = Config()
     c.rank, c.world_size = rank, world_size
     c.key_bytes = c.payload_bytes = key_bytes
@@ -144,6 +146,7 @@ def make_config(rank=0, world_size=1, key_bytes=4, r_capacity=0, s_capacity=0, r
     c.shuffle_mode = shuffle_mode
     c.local_split_bits = local_split_bits
     c.skew_bcast = skew_bcast
+    c.peer_timeout_ms = peer_timeout_ms
     return c
 
 
@@ -194,7 +197,9 @@ class Join:
         if check:
             _check(st, "mgj_result")
         return {"match_count": int(r.match_count), "checksum": int(r.checksum),
+                "pair_digest": int(r.pair_digest),
                 "local_count": int(r.local_count), "local_checksum": int(r.local_checksum),
+                "local_pair_digest": int(r.local_pair_digest),
                 "n_materialized": int(r.n_materialized), "out_key": r.out_key,
                 "out_payload_r": r.out_payload_r, "out_payload_s": r.out_payload_s,
                 "recv_r": int(r.recv_r), "recv_s": int(r.recv_s),

@@ -22,3 +22,18 @@ def test_reference_arm_one_json_line():
     assert d["impl"] == "reference" and d["value"] > 0 and d["unit"] == "tuples/s"
     assert d["cpu_baseline"]["kind"] == "oracle" and d["cpu_baseline"]["cores"] == 1
     assert d["e2e"]["h2d_bytes_per_step"] == 0
+
+
+def test_self_launch_under_torchrun():
+    """`bench.py --gpus 2` without torchrun re-executes itself under
+    torch.distributed.run (two ranks on 127.0.0.1); the oracle arm then runs on
+    rank 0 alone and prints the one JSON line, rank 1 exits 0 without work."""
+    env = {k: v for k, v in os.environ.items() if k not in ("WORLD_SIZE", "RANK", "LOCAL_RANK")}
+    out = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--impl", "reference", "--gpus", "2",
+                          "--steps", "1", "--warmup", "1", "--cpu-sample-log2", "12"], capture_output=True, text=True,
+                         timeout=300, cwd=ROOT, env=env)
+    assert out.returncode == 0, out.stderr[-2000:]
+    lines = [l for l in out.stdout.splitlines() if l.strip().startswith("{")]
+    assert len(lines) == 1, out.stdout
+    d = json.loads(lines[0])
+    assert d["impl"] == "reference" and d["n_gpus"] == 2

@@ -58,3 +58,31 @@ def test_zipf_exp2_accuracy():
     f = np.linspace(0, 1, 1001, endpoint=False)
     p = datagen._exp2_frac(f)
     assert np.max(np.abs(p - np.exp2(f)) / np.exp2(f)) < 4e-16
+
+
+@pytest.mark.parametrize("k", [1, 5, 16, 20, 29, 32])
+def test_perm_k_inverse(k):
+    rng = np.random.default_rng(k)
+    x = rng.integers(0, 1 << k, 100000, dtype=np.uint64) if k > 16 else np.arange(1 << k, dtype=np.uint64)
+    for seed in (datagen.SEED_R, datagen.SEED_S):
+        y = datagen.perm_k(x, k, seed)
+        np.testing.assert_array_equal(datagen.perm_k_inverse(y, k, seed), x)
+
+
+def test_unmix64_inverse():
+    rng = np.random.default_rng(1)
+    x = rng.integers(0, 2**63, 100000, dtype=np.uint64) * np.uint64(2) + rng.integers(0, 2, 100000, dtype=np.uint64)
+    np.testing.assert_array_equal(datagen.unmix64(datagen.mix64(x)), x)
+
+
+@pytest.mark.parametrize("k", [7, 29, 32])
+def test_torch_inverses_match_numpy(k):
+    torch = pytest.importorskip("torch")
+    rng = np.random.default_rng(k + 1)
+    x = rng.integers(0, 1 << k, 50000, dtype=np.uint64)
+    y = datagen.perm_k(x, k, datagen.SEED_R)
+    got = datagen.perm_k_inverse_t(torch.from_numpy(y.astype(np.int64)), k, datagen.SEED_R).numpy()
+    np.testing.assert_array_equal(got.astype(np.uint64), x)
+    z = datagen.mix64(x)
+    got = datagen.unmix64_t(torch.from_numpy(z.view(np.int64))).numpy().view(np.uint64)
+    np.testing.assert_array_equal(got, x)

@@ -139,6 +139,56 @@ __device__ __forceinline__ void count_packed(const Tup *src, uint32_t len, int t
         }
 }
 
+// Extents of the sub-partitions in mid (exclusive scan of the padded sizes)
+// and the chunk table of the chunked pass over them.  One CTA.  (Run by the
+// last CTA of k_countA instead, measured 0.28-0.47 ms slower at B1 = 7: the
+// planner's registers and shared memory cut k_countA's occupancy.)
+__global__ void __launch_bounds__(1024) k_planA(Ctx c) {
+    extern __shared__ uint64_t sv[];  // [L+1] then u32 [L+1]
+    __shared__ uint64_t tmp[33];
+    __shared__ uint32_t tmp32[33];
+    if (!c.meta[MT_OK] || !c.meta[MT_BA]) return;
+    const int BA = c.meta[MT_BA];
+    const int L = c.meta[MT_NP] << BA;
+    const int tid = threadIdx.x;
+    uint32_t *nch = reinterpret_cast<uint32_t *>(sv + L + 1);
+    const uint64_t C = (uint64_t)c.chunk_tuples2;  // the chunked pass after the first pass
+    uint32_t tot_ch[2];
+    bool bad = false;
+    for (int rel = 0; rel < 2; ++rel) {
+        const uint32_t *h = c.hA + (size_t)rel * c.vcap;
+        for (int v = tid; v <= L; v += blockDim.x) {
+            const uint32_t n = v < L ? __ldcg(h + v) : 0;
+            sv[v] = n;
+            nch[v] = (uint32_t)((n + C - 1) / C);
+        }
+        __syncthreads();
+        const uint64_t slots = block_excl_scan_u64(sv, L + 1, tmp);
+        tot_ch[rel] = block_excl_scan_u32(nch, L + 1, tmp32);
+        bad |= slots > c.mid_cap || tot_ch[rel] > c.max_chunks;
+        uint64_t *vs = c.vstart + (size_t)rel * c.cb_stride;
+        for (int v = tid; v <= L; v += blockDim.x) {
+            vs[v] = sv[v];
+            if (v < L) c.vcur[(size_t)rel * c.cb_stride + v] = sv[v];
+            c.chunk_base[(size_t)rel * c.cb_stride + v] = nch[v];
+        }
+        __syncthreads();
+    }
+    if (tid == 0) {
+        c.meta[MT_NCHB_R] = (int)tot_ch[0];
+        c.meta[MT_NCHB_S] = (int)tot_ch[1];
+        c.meta[MT_NLP] = L;
+        if (bad) {
+            set_err(c, MGJ_ECAPACITY);
+            c.meta[MT_OK] = 0;
+        }
+    }
+}
+
+// First local pass, step 1 (only when k_plan chose BA > 0; a no-op
+// otherwise): padded size of every (owned partition, BA-bit digit) run over
+// the chunks of the partition, exactly the slots k_local<K, LM_SPLIT>
+// reserves.
 template <typename K>
 __global__ void __launch_bounds__(512) k_countA(Ctx c, const ChunkDesc *cdesc) {
     using Tup = typename Layout<K>::Tup;
@@ -176,75 +226,6 @@ __global__ void __launch_bounds__(512) k_countA(Ctx c, const ChunkDesc *cdesc) {
     }
 }
 
-// Extents of the sub-partitions in mid (exclusive scan of the padded sizes)
-// and the chunk table of the chunked pass over them.  One CTA.
-__global__ void __launch_bounds__(1024) k_planA(Ctx c) {
-    extern __shared__ uint64_t sv[];  // [L+1] then u32 [L+1]
-    __shared__ uint64_t tmp[33];
-    __shared__ uint32_t tmp32[33];
-    if (!c.meta[MT_OK] || !c.meta[MT_BA]) return;
-    const int BA = c.meta[MT_BA];
-    const int L = c.meta[MT_NP] << BA;
-    const int tid = threadIdx.x;
-    uint32_t *nch = reinterpret_cast<uint32_t *>(sv + L + 1);
-    const uint64_t C = (uint64_t)c.chunk_tuples2;  // the chunked pass after the first pass
-    uint32_t tot_ch[2];
-    bool bad = false;
-    for (int rel = 0; rel < 2; ++rel) {
-        const uint32_t *h = c.hA + (size_t)rel * c.vcap;
-        for (int v = tid; v <= L; v += blockDim.x) {
-            const uint32_t n = v < L ? h[v] : 0;
-            sv[v] = n;
-            nch[v] = (uint32_t)((n + C - 1) / C);
-        }
-        __syncthreads();
-        const uint64_t slots = block_excl_scan_u64(sv, L + 1, tmp);
-        tot_ch[rel] = block_excl_scan_u32(nch, L + 1, tmp32);
-        uint64_t *vs = c.vstart + (size_t)rel * c.cb_stride;
-        for (int v = tid; v <= L; v += blockDim.x) {
-            vs[v] = sv[v];
-            if (v < L) c.vcur[(size_t)rel * c.cb_stride + v] = sv[v];
-            c.chunk_base[(size_t)rel * c.cb_stride + v] = nch[v];
-        }
-        bad |= slots > c.mid_cap || tot_ch[rel] > c.max_chunks;
-        __syncthreads();
-    }
-    if (tid == 0) {
-        c.meta[MT_NCHB_R] = (int)tot_ch[0];
-        c.meta[MT_NCHB_S] = (int)tot_ch[1];
-        c.meta[MT_NLP] = L;
-        if (bad) {
-            set_err(c, MGJ_ECAPACITY);
-            c.meta[MT_OK] = 0;
-        }
-    }
-}
-
-// Chunk descriptors of the chunked pass over the sub-partitions (one piece each).
-__global__ void k_chunkmapB(Ctx c, ChunkDesc *desc) {
-    if (!c.meta[MT_OK] || !c.meta[MT_BA]) return;
-    const int L = c.meta[MT_NLP];
-    const uint32_t nch_r = (uint32_t)c.meta[MT_NCHB_R], total = nch_r + (uint32_t)c.meta[MT_NCHB_S];
-    const uint64_t C = (uint64_t)c.chunk_tuples2;  // the chunked pass after the first pass
-    for (uint32_t ci = blockIdx.x * blockDim.x + threadIdx.x; ci < total; ci += gridDim.x * blockDim.x) {
-        const int rel = ci < nch_r ? 0 : 1;
-        const uint32_t li = rel ? ci - nch_r : ci;
-        const uint32_t *cb = c.chunk_base + (size_t)rel * c.cb_stride;
-        int lo = 0, hi = L - 1;
-        while (lo < hi) {
-            const int mid = (lo + hi + 1) >> 1;
-            if (__ldg(cb + mid) <= li) lo = mid; else hi = mid - 1;
-        }
-        const uint64_t k = li - cb[lo];
-        const uint64_t *vs = c.vstart + (size_t)rel * c.cb_stride;
-        ChunkDesc d;
-        d.start = vs[lo] + k * C;
-        d.len = (uint32_t)min(C, vs[lo + 1] - vs[lo] - k * C);
-        d.pi = (uint32_t)lo;
-        desc[ci] = d;
-    }
-}
-
 // ---------------------------------------------------------------------------
 // a4 (§3.2 "Local partitioning"): the received data of
 // each owned global partition p is partitioned again by the next B2 key bits
@@ -271,7 +252,7 @@ __global__ void k_chunkmapB(Ctx c, ChunkDesc *desc) {
 enum LocalMode { LM_SINGLE = 0, LM_SPLIT = 1, LM_SECOND = 2 };
 
 template <typename K, int MODE>
-__global__ void __launch_bounds__(LOCAL_THREADS, 1) k_local(Ctx c, const ChunkDesc *cdesc) {
+__device__ __forceinline__ void local_body(const Ctx &c, const ChunkDesc *cdesc) {
     constexpr bool SPLIT = MODE == LM_SPLIT;
     using Tup = typename Layout<K>::Tup;
     constexpr int TB = Layout<K>::TB, ALIGN = Layout<K>::ALIGN;
@@ -280,9 +261,7 @@ __global__ void __launch_bounds__(LOCAL_THREADS, 1) k_local(Ctx c, const ChunkDe
     __shared__ __align__(8) uint64_t bar[2];
     __shared__ ChunkDesc sdesc[2];
     __shared__ uint32_t tmp[33];
-    if (!c.meta[MT_OK]) return;
     const int BA = MODE == LM_SINGLE ? 0 : c.meta[MT_BA];
-    if ((MODE == LM_SINGLE) != (c.meta[MT_BA] == 0)) return;
     const int tid = threadIdx.x;
     // LM_SECOND has its own chunk geometry (fan-out <= 2^(b2_max - 1): larger chunks fit)
     const int C = MODE == LM_SECOND ? c.chunk_tuples2 : (SPLIT ? c.chunk_tuples1s : c.chunk_tuples);
@@ -442,6 +421,56 @@ __global__ void __launch_bounds__(LOCAL_THREADS, 1) k_local(Ctx c, const ChunkDe
         }
     }
     bulk_wait0();
+}
+
+// Chunk descriptors of the chunked pass over the sub-partitions (one piece
+// each): chunk li of relation rel lies in the sub-partition v whose chunk
+// range [chunk_base[v], chunk_base[v + 1]) holds it.
+__device__ inline void chunkmap_second(const Ctx &c, ChunkDesc *desc) {
+    const int L = c.meta[MT_NLP];
+    const uint32_t nch_r = (uint32_t)c.meta[MT_NCHB_R], total = nch_r + (uint32_t)c.meta[MT_NCHB_S];
+    const uint64_t C = (uint64_t)c.chunk_tuples2;  // the chunked pass after the first pass
+    for (uint32_t ci = blockIdx.x * blockDim.x + threadIdx.x; ci < total; ci += gridDim.x * blockDim.x) {
+        const int rel = ci < nch_r ? 0 : 1;
+        const uint32_t li = rel ? ci - nch_r : ci;
+        const uint32_t *cb = c.chunk_base + (size_t)rel * c.cb_stride;
+        int lo = 0, hi = L - 1;
+        while (lo < hi) {
+            const int mid = (lo + hi + 1) >> 1;
+            if (__ldcg(cb + mid) <= li) lo = mid; else hi = mid - 1;
+        }
+        const uint64_t k = li - __ldcg(cb + lo);
+        const uint64_t *vs = c.vstart + (size_t)rel * c.cb_stride;
+        ChunkDesc d;
+        d.start = __ldcg(vs + lo) + k * C;
+        d.len = (uint32_t)min(C, __ldcg(vs + lo + 1) - d.start);
+        d.pi = (uint32_t)lo;
+        desc[ci] = d;
+    }
+}
+
+// The first pass of two-level local partitioning (a no-op unless k_plan chose
+// BA > 0).  Its CTAs also write the chunked pass's chunk descriptors (they
+// depend only on k_countA's layout, not on this pass's output).
+template <typename K>
+__global__ void __launch_bounds__(LOCAL_THREADS, 1) k_local_split(Ctx c, const ChunkDesc *cdesc, ChunkDesc *descB) {
+    if (!c.meta[MT_OK] || !c.meta[MT_BA]) return;
+    chunkmap_second(c, descB);
+    local_body<K, LM_SPLIT>(c, cdesc);
+}
+
+// The chunked pass over the first pass's sub-partitions (a no-op when BA = 0).
+template <typename K>
+__global__ void __launch_bounds__(LOCAL_THREADS, 1) k_local_second(Ctx c, const ChunkDesc *descB) {
+    if (!c.meta[MT_OK] || !c.meta[MT_BA]) return;
+    local_body<K, LM_SECOND>(c, descB);
+}
+
+// The single chunked pass over the owned partitions (a no-op when BA > 0).
+template <typename K>
+__global__ void __launch_bounds__(LOCAL_THREADS, 1) k_local(Ctx c, const ChunkDesc *cdesc) {
+    if (!c.meta[MT_OK] || c.meta[MT_BA]) return;
+    local_body<K, LM_SINGLE>(c, cdesc);
 }
 
 // ---------------------------------------------------------------------------

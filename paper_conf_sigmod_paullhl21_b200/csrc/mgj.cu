@@ -141,7 +141,8 @@ struct mgj_plan_s {
     void *allocs[64] = {};
     int nalloc = 0;
     Ctx ctx{};
-    ChunkDesc *cdesc = nullptr;
+    ChunkDesc *cdesc = nullptr;   // chunks of the (first) local pass, written by k_chunkmap
+    ChunkDesc *cdescB = nullptr;  // chunks of the chunked pass after a first pass (k_countA)
     char *send_arena = nullptr;  // EXTERNAL shuffle
     uint64_t epoch = 0;
     int state = 0;
@@ -194,9 +195,9 @@ cudaError_t set_attrs(const Norm &n) {
     if ((e = cudaFuncSetAttribute(k_hist<K>, A, (int)hist_smem(n)))) return e;
     if ((e = cudaFuncSetAttribute(k_plan, A, (int)plan_smem(n)))) return e;
     if ((e = cudaFuncSetAttribute(scatter_kernel<K>(n.P), A, (int)scatter_smem(n)))) return e;
-    if ((e = cudaFuncSetAttribute(k_local<K, LM_SINGLE>, A, (int)local_smem(n)))) return e;
-    if ((e = cudaFuncSetAttribute(k_local<K, LM_SPLIT>, A, (int)local_smem1s(n)))) return e;
-    if ((e = cudaFuncSetAttribute(k_local<K, LM_SECOND>, A, (int)local_smem2(n)))) return e;
+    if ((e = cudaFuncSetAttribute(k_local<K>, A, (int)local_smem(n)))) return e;
+    if ((e = cudaFuncSetAttribute(k_local_second<K>, A, (int)local_smem2(n)))) return e;
+    if ((e = cudaFuncSetAttribute(k_local_split<K>, A, (int)local_smem1s(n)))) return e;
     if ((e = cudaFuncSetAttribute(k_planA, A, (int)planA_smem(n)))) return e;
     if ((e = cudaFuncSetAttribute(k_probe<K, false>, A, (int)probe_smem(n)))) return e;
     return cudaFuncSetAttribute(k_probe<K, true>, A, (int)probe_smem(n));
@@ -239,16 +240,19 @@ void launch_join(mgj_plan_s *h, cudaStream_t s) {
         k_wait<<<1, 32, 0, s>>>(h->ctx, SIG_DATA);
         h->launches += 1;
     }
-    // two-level local partitioning (device-side decision, MT_BA; no-ops otherwise)
+    // two-level local partitioning: k_plan decides on the device (MT_BA); when
+    // it chooses one pass these four kernels return at once.  (Measured, not
+    // kept: a guard kernel that tail-launches the chosen kernels from the
+    // device costs 18 us; one kernel for both chunked passes spills, +0.1 ms at
+    // M2; k_planA run by k_countA's last CTA, +0.28 ms at B1 = 7.)
     if (n.split) {
         k_countA<K><<<h->nsm * 4, 512, 0, s>>>(h->ctx, h->cdesc);
         k_planA<<<1, 1024, planA_smem(n), s>>>(h->ctx);
-        k_local<K, LM_SPLIT><<<h->nsm, LOCAL_THREADS, local_smem1s(n), s>>>(h->ctx, h->cdesc);
-        k_chunkmapB<<<h->nsm * 2, 256, 0, s>>>(h->ctx, h->cdesc);
-        k_local<K, LM_SECOND><<<h->nsm, LOCAL_THREADS, local_smem2(n), s>>>(h->ctx, h->cdesc);
-        h->launches += 5;
+        k_local_split<K><<<h->nsm, LOCAL_THREADS, local_smem1s(n), s>>>(h->ctx, h->cdesc, h->cdescB);
+        k_local_second<K><<<h->nsm, LOCAL_THREADS, local_smem2(n), s>>>(h->ctx, h->cdescB);
+        h->launches += 4;
     }
-    k_local<K, LM_SINGLE><<<h->nsm, LOCAL_THREADS, local_smem(n), s>>>(h->ctx, h->cdesc);
+    k_local<K><<<h->nsm, LOCAL_THREADS, local_smem(n), s>>>(h->ctx, h->cdesc);
     cudaEventRecord(h->ev[4], s);
     k_itemize<K><<<h->nsm * 4, 256, 0, s>>>(h->ctx);
     if (n.c.materialize)
@@ -373,6 +377,7 @@ mgj_status mgj_plan(const mgj_config *cfg, const mgj_peers *peers, mgj_handle *o
     c.sub_ns = (int32_t)((std::max(n.c.r_capacity, n.c.s_capacity) / c.G + 8) / c.scat_T + 2);
     c.sub_hist = static_cast<uint16_t *>(dalloc(h, 2ull * c.G * c.sub_ns * P * 2, &st));
     h->cdesc = static_cast<ChunkDesc *>(dalloc(h, 2 * n.max_chunks * sizeof(ChunkDesc), &st));
+    if (n.split) h->cdescB = static_cast<ChunkDesc *>(dalloc(h, 2 * n.max_chunks * sizeof(ChunkDesc), &st));
     c.owner = static_cast<int32_t *>(dalloc(h, P * 4, &st));
     c.bcast = static_cast<uint8_t *>(dalloc(h, P, &st));
     c.pskip = static_cast<uint8_t *>(dalloc(h, P, &st));

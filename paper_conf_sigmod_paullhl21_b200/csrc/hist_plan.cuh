@@ -11,7 +11,12 @@ namespace mgj {
 #ifndef HIST_FOLD16
 #define HIST_FOLD16 1  // 4-byte keys: fold four bins per thread with 16-byte accesses (P >= 4)
 #endif
-constexpr int HIST_NB = 3;  // k_hist: TMA ring depth (sub-tiles in flight per CTA; 2 CTAs per SM)
+constexpr int HIST_NB = 3;  // k_hist: TMA ring depth at most (sub-tiles in flight per CTA; 2 CTAs per SM)
+// ring depth for sub-tiles of T keys: about 96 KB in flight per CTA, 2..HIST_NB deep
+__host__ __device__ inline int hist_nb(int T, int key_bytes) {
+    const int nb = 98304 / (T * key_bytes);
+    return nb < 2 ? 2 : (nb > HIST_NB ? HIST_NB : nb);
+}
 
 // ---------------------------------------------------------------------------
 // a1: per-GPU radix histogram (§3.2 "Histogram generation",
@@ -31,9 +36,9 @@ template <typename K>
 __global__ void __launch_bounds__(HIST_THREADS, 2) k_hist(Ctx c) {
     extern __shared__ __align__(128) unsigned char hsm[];  // ring[HIST_NB][T] keys | sub[P] | acc[P]
     __shared__ __align__(8) uint64_t bar[HIST_NB];
-    const int P = c.P, T = c.scat_T;
+    const int P = c.P, T = c.scat_T, NB = hist_nb(T, sizeof(K));
     K *const ring = reinterpret_cast<K *>(hsm);
-    uint32_t *const sub = reinterpret_cast<uint32_t *>(ring + (size_t)HIST_NB * T);
+    uint32_t *const sub = reinterpret_cast<uint32_t *>(ring + (size_t)NB * T);
     uint32_t *const acc = sub + P;
     const int tid = threadIdx.x, HS = c.hist_split, tile = blockIdx.x / HS, part = blockIdx.x % HS;
     constexpr int LU = 16 / (int)sizeof(K);
@@ -58,17 +63,17 @@ __global__ void __launch_bounds__(HIST_THREADS, 2) k_hist(Ctx c) {
         uint32_t j, len;
         uint64_t first;
         subtile(g, rel, j, first, len);
-        uint64_t *b = &bar[g % HIST_NB];
+        uint64_t *b = &bar[g % NB];
         const uint32_t bytes = (len & ~(uint32_t)(LU - 1)) * (uint32_t)sizeof(K);
         mbar_arrive_expect_tx(b, bytes);
         if (bytes)
-            tma_load_1d(ring + (size_t)(g % HIST_NB) * T, static_cast<const K *>(c.in_key[rel]) + first, bytes, b, pol);
+            tma_load_1d(ring + (size_t)(g % NB) * T, static_cast<const K *>(c.in_key[rel]) + first, bytes, b, pol);
     };
     for (int i = tid; i < 2 * P; i += blockDim.x) sub[i] = 0;
     if (tid == 0) {
-        for (int i = 0; i < HIST_NB; ++i) mbar_init(&bar[i], 1);
+        for (int i = 0; i < NB; ++i) mbar_init(&bar[i], 1);
         fence_mbar_init();
-        for (uint32_t g = 0; g < ntot && g < (uint32_t)HIST_NB; ++g) issue(g);
+        for (uint32_t g = 0; g < ntot && g < (uint32_t)NB; ++g) issue(g);
     }
     __syncthreads();
     const uint32_t m = (uint32_t)(P - 1);
@@ -88,8 +93,8 @@ __global__ void __launch_bounds__(HIST_THREADS, 2) k_hist(Ctx c) {
         uint32_t j, len;
         uint64_t first;
         subtile(g, rel, j, first, len);
-        const K *buf = ring + (size_t)(g % HIST_NB) * T;
-        mbar_wait(&bar[g % HIST_NB], (g / HIST_NB) & 1);
+        const K *buf = ring + (size_t)(g % NB) * T;
+        mbar_wait(&bar[g % NB], (g / NB) & 1);
         const uint32_t body = len & ~(uint32_t)(LU - 1);
         for (uint32_t i0 = (uint32_t)tid * LU; i0 < body; i0 += (uint32_t)blockDim.x * LU) {
             const uint4 v = *reinterpret_cast<const uint4 *>(buf + i0);
@@ -106,7 +111,7 @@ __global__ void __launch_bounds__(HIST_THREADS, 2) k_hist(Ctx c) {
         if (tid < (int)(len - body))  // < LU trailing tuples of the relation: from global
             atomicAdd(&sub[digit1(static_cast<const K *>(c.in_key[rel])[first + body + tid], P)], 1u);
         __syncthreads();  // counts final; ring slot g % NB free
-        if (tid == 0 && g + HIST_NB < ntot) issue(g + HIST_NB);
+        if (tid == 0 && g + NB < ntot) issue(g + NB);
         // sub-tile histogram (u16 pairs) for the scatter's layout, then fold into acc
         uint32_t *o32 = reinterpret_cast<uint32_t *>(c.sub_hist + (((size_t)rel * c.G + tile) * c.sub_ns + j) * P);
         if constexpr (sizeof(K) == 4) {  // 8-byte shared accesses, pairs of bins (measured: M2 0.83 -> 0.78 ms;

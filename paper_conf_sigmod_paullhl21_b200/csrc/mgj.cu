@@ -178,10 +178,11 @@ void *dalloc(mgj_plan_s *h, size_t bytes, mgj_status *st) {
 }
 
 size_t hist_smem(const Norm &n) {
-    return (size_t)HIST_NB * scat_geom(n.P, n.c.key_bytes).T * n.c.key_bytes + (size_t)n.P * 8;
+    const int T = scat_geom(n.P, n.c.key_bytes).T;
+    return (size_t)hist_nb(T, n.c.key_bytes) * T * n.c.key_bytes + (size_t)n.P * 8;
 }
 size_t plan_smem(const Norm &n) { return (size_t)n.P * 5 * 8 + (size_t)n.P * 4 + (size_t)(n.P + 1) * 4 + (size_t)n.P; }
-size_t scatter_smem(const Norm &n) { return scat_smem_bytes(n.P, n.c.key_bytes); }
+size_t scatter_smem(const Norm &n) { return scatter_smem_bytes(n.P, n.c.key_bytes); }
 size_t planA_smem(const Norm &n) { return ((size_t)local2_vcap(n.P) + 1) * 12; }
 size_t local_smem(const Norm &n) { return local_smem_bytes(n.chunk_tuples, 1 << n.b2_max, n.tuple_bytes); }
 size_t local_smem2(const Norm &n) { return local_smem_bytes(n.chunk_tuples2, 1 << n.qm2_bits, n.tuple_bytes); }

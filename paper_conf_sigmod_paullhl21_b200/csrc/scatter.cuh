@@ -26,9 +26,9 @@ struct ScatGeom {
 };
 __host__ __device__ constexpr ScatGeom scat_geom(int P, int key_bytes) {
     return key_bytes == 4
-               ? (P <= 1024 ? ScatGeom{8192, 4, 1, 1024}
+               ? (P <= 1024 ? ScatGeom{12288, 4, 1, 1024}
                   : P == 2048 ? ScatGeom{4096, 4, 2, 1024} : ScatGeom{8192, 1, 4, 1024})
-               : (P <= 1024 ? ScatGeom{4096, 2, 1, 1024} : P == 2048 ? ScatGeom{2048, 2, 2, 1024}
+               : (P <= 1024 ? ScatGeom{6144, 2, 1, 1024} : P == 2048 ? ScatGeom{2048, 2, 2, 1024}
                                                                       : ScatGeom{4096, 1, 4, 1024});
 }
 
@@ -43,7 +43,7 @@ struct __align__(16) PInfo {
 __host__ __device__ inline size_t scat_smem_bytes(int P, int key_bytes) {
     const ScatGeom g = scat_geom(P, key_bytes);
     const size_t TB = 2 * (size_t)key_bytes;
-    return 2 * (size_t)g.T * key_bytes                         // input stage: keys + payloads (SoA)
+    return (size_t)g.T * key_bytes                             // input stage: keys (payloads: L2 prefetch + loads)
            + ((size_t)g.T + 2 * (size_t)(g.SG - 1) * P) * TB  // partition-sorted sub-tile (+ carries, group padding)
            + (size_t)P * sizeof(PInfo)                         // write-out descriptors
            + (size_t)P * 4;                                    // next free slot per partition
@@ -82,6 +82,33 @@ __device__ __forceinline__ uint4 lds128(const void *p) {
     asm volatile("ld.volatile.shared.v4.u32 {%0,%1,%2,%3}, [%4];"
                  : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w)
                  : "r"(smem_u32(p)));
+    return v;
+}
+
+// Shared-memory accesses on precomputed 32-bit shared addresses: with plain
+// pointers the compiler re-derived the shared window base (S2R SR_CgaCtaId)
+// inside the write-out loop, 6% of the kernel's stall samples (ncu, round 2).
+__device__ __forceinline__ uint4 lds128_at(uint32_t a) {
+    uint4 v;
+    asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(a));
+    return v;
+}
+__device__ __forceinline__ uint2 lds64_at(uint32_t a) {
+    uint2 v;
+    asm volatile("ld.shared.v2.u32 {%0,%1}, [%2];" : "=r"(v.x), "=r"(v.y) : "r"(a));
+    return v;
+}
+__device__ __forceinline__ void sts_at(uint32_t a, const uint2 &v) {
+    asm volatile("st.shared.v2.u32 [%0], {%1,%2};" ::"r"(a), "r"(v.x), "r"(v.y) : "memory");
+}
+__device__ __forceinline__ void sts_at(uint32_t a, const ulonglong2 &v) {
+    asm volatile("st.shared.v2.u64 [%0], {%1,%2};" ::"r"(a), "l"(v.x), "l"(v.y) : "memory");
+}
+template <typename Tup> __device__ __forceinline__ Tup lds_tup(uint32_t a);
+template <> __device__ __forceinline__ uint2 lds_tup<uint2>(uint32_t a) { return lds64_at(a); }
+template <> __device__ __forceinline__ ulonglong2 lds_tup<ulonglong2>(uint32_t a) {
+    ulonglong2 v;
+    asm volatile("ld.shared.v2.u64 {%0,%1}, [%2];" : "=l"(v.x), "=l"(v.y) : "r"(a));
     return v;
 }
 
@@ -158,13 +185,14 @@ __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c) {
     constexpr bool EAGER = sizeof(K) == 8;
     extern __shared__ __align__(128) unsigned char smem[];
     const int P = c.P;
-    K *const skey = reinterpret_cast<K *>(smem);  // stage: keys, then payloads
-    K *const spay = skey + T;
-    Tup *const sorted = reinterpret_cast<Tup *>(smem + 2 * T * sizeof(K));
+    K *const skey = reinterpret_cast<K *>(smem);  // stage: the sub-tile's keys
+    Tup *const sorted = reinterpret_cast<Tup *>(smem + T * sizeof(K));
     PInfo *const pinfo = reinterpret_cast<PInfo *>(sorted + T + 2 * (SG - 1) * P);  // 16-byte aligned
     uint32_t *const off = reinterpret_cast<uint32_t *>(pinfo + P);  // next free slot per partition
-    auto sput = [&](uint32_t x, const Tup &t) { sorted[swz(x)] = t; };
-    auto sget = [&](uint32_t x) -> Tup { return sorted[swz(x)]; };
+    const uint32_t sorted_s = smem_u32(sorted), pinfo_s = smem_u32(pinfo);
+    auto saddr = [&](uint32_t x) -> uint32_t { return sorted_s + swz(x) * (uint32_t)TB; };
+    auto sput = [&](uint32_t x, const Tup &t) { sts_at(saddr(x), t); };
+    auto sget = [&](uint32_t x) -> Tup { return lds_tup<Tup>(saddr(x)); };
     __shared__ __align__(8) uint64_t bar;
     __shared__ uint32_t tmp[32];
     const int tid = threadIdx.x;
@@ -204,10 +232,14 @@ __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c) {
         uint32_t len;
         subtile(g, rel, first, len);
         const uint32_t bytes = (len & ~(uint32_t)(LU - 1)) * (uint32_t)sizeof(K);
-        mbar_arrive_expect_tx(&bar, 2 * bytes);
+        mbar_arrive_expect_tx(&bar, bytes);
         if (bytes) {
             tma_load_1d(skey, static_cast<const K *>(c.in_key[rel]) + first, bytes, &bar, pol);
-            tma_load_1d(spay, static_cast<const K *>(c.in_pay[rel]) + first, bytes, &bar, pol);
+            // payloads: brought into L2 now and loaded into registers while the
+            // previous sub-tile is written out (the shared memory of a payload
+            // stage goes to a 1.5x larger sub-tile instead; measured at M2:
+            // scatter 4.12 -> 3.89 ms; without the L2 prefetch 4.65 ms)
+            prefetch_l2(static_cast<const K *>(c.in_pay[rel]) + first, bytes);
         }
     };
     auto fetch_carry = [&]() {  // the incomplete last groups of the previous sub-tile -> registers
@@ -271,9 +303,35 @@ __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c) {
             out[0] = v.x & 0xffffu, out[1] = v.x >> 16, out[2] = v.y & 0xffffu, out[3] = v.y >> 16;
         }
     };
+    // payloads of sub-tile g (L2-resident since issue(g)), loaded into
+    // registers while the previous sub-tile is written out
+    K pp[V];
+    auto load_pay = [&](uint32_t g) {
+        int rel;
+        uint64_t first;
+        uint32_t len;
+        subtile(g, rel, first, len);
+        const K *gp = static_cast<const K *>(c.in_pay[rel]) + first;
+        if (len == T) {
+#pragma unroll
+            for (int u = 0; u < NU; ++u) {
+                const uint4 b = __ldcs(reinterpret_cast<const uint4 *>(gp + (uint32_t)(u * NT + tid) * LU));
+                memcpy(&pp[u * LU], &b, 16);
+            }
+        } else {
+#pragma unroll
+            for (int u = 0; u < NU; ++u)
+#pragma unroll
+                for (int e = 0; e < LU; ++e) {
+                    const uint32_t i = (uint32_t)(u * NT + tid) * LU + e;
+                    pp[u * LU + e] = i < len ? __ldcs(gp + i) : (K)0;
+                }
+        }
+    };
     uint32_t ncnt[PPT];
     load_counts(0, ncnt);
     if (tid == 0 && ntot > 0) issue(0);
+    if (ntot > 0) load_pay(0);
     int cur_rel = -1;
     for (uint32_t g = 0; g < ntot; ++g) {
         int rel;
@@ -319,19 +377,16 @@ __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c) {
             o += seg[k];
         }
         pending = SG > 1;
-        K kk[V], pp[V];
+        K kk[V];
         mbar_wait(&bar, g & 1);
         const uint32_t body = len & ~(uint32_t)(LU - 1);
         const K *gk = static_cast<const K *>(c.in_key[rel]) + first;
-        const K *gp = static_cast<const K *>(c.in_pay[rel]) + first;
         if (len == T) {  // full sub-tile: branch-free vector loads
 #pragma unroll
             for (int u = 0; u < NU; ++u) {
                 const uint32_t i0 = (uint32_t)(u * NT + tid) * LU;
                 const uint4 a = *reinterpret_cast<const uint4 *>(skey + i0);
-                const uint4 b = *reinterpret_cast<const uint4 *>(spay + i0);
                 memcpy(&kk[u * LU], &a, 16);
-                memcpy(&pp[u * LU], &b, 16);
             }
         } else {
 #pragma unroll
@@ -340,7 +395,6 @@ __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c) {
                 for (int e = 0; e < LU; ++e) {  // < LU trailing tuples of the relation come from global
                     const uint32_t i = (uint32_t)(u * NT + tid) * LU + e;
                     kk[u * LU + e] = i < body ? skey[i] : (i < len ? gk[i] : (K)0);
-                    pp[u * LU + e] = i < body ? spay[i] : (i < len ? gp[i] : (K)0);
                 }
             }
         }
@@ -357,29 +411,33 @@ __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c) {
             }
         }
         __syncthreads();  // S2
+        if (g + 1 < ntot) load_pay(g + 1);  // the ranking of this sub-tile has consumed pp
         // write-out: one group per thread per step
         const uint32_t ngroups = total / SG;
         for (uint32_t u = tid; u < ngroups; u += NT) {
             const uint32_t slot = u * SG;
             GV gv;
             PInfo in;
-            if constexpr (GB == 32 && EAGER) {  // two conflict-free 16-byte halves (swizzled)
-                gv.a = lds128(sorted + swz(slot));
-                gv.b = lds128(sorted + swz(slot + SG / 2));
-            } else if constexpr (GB == 32) {
-                gv.a = *reinterpret_cast<const uint4 *>(sorted + swz(slot));
-                gv.b = *reinterpret_cast<const uint4 *>(sorted + swz(slot + SG / 2));
+            if constexpr (GB == 32) {  // two conflict-free 16-byte halves (swizzled)
+                gv.a = lds128_at(saddr(slot));
+                gv.b = lds128_at(saddr(slot + SG / 2));
+            } else if constexpr (GB == 16) {
+                gv = lds128_at(saddr(slot));
             } else {
-                gv = *reinterpret_cast<const GV *>(sorted + slot);
+                gv = lds64_at(saddr(slot));
             }
-            const PInfo *pi = pinfo + (reinterpret_cast<const uint32_t *>(&gv)[0] & (uint32_t)(P - 1));
+            const uint32_t pa = pinfo_s + (reinterpret_cast<const uint32_t *>(&gv)[0] & (uint32_t)(P - 1)) * 16u;
             if constexpr (EAGER) {
-                const uint4 v = lds128(pi);
+                const uint4 v = lds128_at(pa);
                 in.wb = (ull)v.x | ((ull)v.y << 32);
                 in.lim = v.z;
                 in.head = v.w;
             } else {
-                in = *pi;
+                const uint2 lh = lds64_at(pa + 8);
+                in.lim = lh.x;
+                in.head = lh.y;
+                const uint2 w = lds64_at(pa);
+                in.wb = (ull)w.x | ((ull)w.y << 32);
             }
             if (slot + SG <= in.lim) {
                 char *dst = reinterpret_cast<char *>(in.wb + (ull)slot * TB);
@@ -413,5 +471,6 @@ inline void (*scatter_kernel(int P))(Ctx) {
     return k_scatter<K, g4.T, g4.SG, g4.PPT, g4.NT>;
 }
 inline int scatter_threads(int P, int key_bytes) { return scat_geom(P, key_bytes).NT; }
+inline size_t scatter_smem_bytes(int P, int key_bytes) { return scat_smem_bytes(P, key_bytes); }
 
 }  // namespace mgj

@@ -52,6 +52,11 @@ def parse():
                     help="oracle sample: 2^k R + 2^k S unique tuples (cpu_baseline / --impl reference)")
     ap.add_argument("--skew-bcast", type=int, default=0, choices=[-1, 0, 1],
                     help="a2 selective broadcast of heavy S partitions (N>1): 0 auto, -1 never, 1 forced")
+    ap.add_argument("--num-sms", type=int, default=0, help="SMs the library's persistent kernels use (0 = all)")
+    ap.add_argument("--overlap", default="auto", choices=["auto", "on", "off"],
+                    help="§8(e): R's local pass beside S's scatter (auto: on for N > 1 with the P2P shuffle)")
+    ap.add_argument("--overlap-local-sms", type=int, default=0)
+    ap.add_argument("--trace", action="store_true", help="kernel timeline of the last step in the JSON line")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=3)
@@ -293,7 +298,9 @@ def main():
                           recv_capacity_r=(n_r if world > 1 and a.workload == "zipf" else 0),
                           recv_capacity_s=(n_s // 2 if world > 1 and a.workload == "zipf" else 0),
                           shuffle_mode=(mgj.SHUFFLE_EXTERNAL if a.shuffle == "nccl" else mgj.SHUFFLE_P2P),
-                          skew_bcast=a.skew_bcast)
+                          skew_bcast=a.skew_bcast, num_sms=a.num_sms,
+                          shuffle_overlap={"auto": 0, "on": 1, "off": -1}[a.overlap],
+                          overlap_local_sms=a.overlap_local_sms, trace=a.trace)
     # N>1 (or MGJ_SYMM_ARENA=1): the library's symmetric-memory setup (mgj.symmetric_join)
     join = mgj.symmetric_join(cfg) if distributed else mgj.Join(cfg)
 
@@ -331,6 +338,7 @@ def main():
     barrier()
     res = join.result()  # the last timed step's result (a6 ran inside it)
     clocks = sampler.stop() if sampler else None
+    timeline = {k: [round(v[0] / 1e3, 1), round(v[1] / 1e3, 1)] for k, v in join.trace().items()} if a.trace else None
 
     # correctness of the timed run: global count, checksum and pair digest
     # against the generator-derived values (every workload; SURVEY.md §8c
@@ -472,6 +480,7 @@ def main():
             "cpu_baseline": None if cpu is None else {k: cpu[k] for k in ("value", "unit", "cores", "kind", "sample")},
             "e2e": e2e,
             "gpu_launches": res["n_launches"] * a.steps,  # counted by the library per run
+            "timeline_us": timeline,
             "clocks": clocks,
         }
         emit(out, line)

@@ -82,7 +82,14 @@ typedef struct {
                                           rank or MGJ_SHUFFLE_EXTERNAL */
     int32_t  peer_timeout_ms;          /* bound on every wait for a peer's signal (0 = 20000 ms); a wait
                                           that times out makes the run fail with MGJ_EPEER */
-    int32_t  reserved[4];              /* must be zero */
+    int32_t  shuffle_overlap;          /* SURVEY.md §8(e) / P:455-468: local-partition R (on a second
+                                          stream, overlap_local_sms SMs) while S is still being shuffled
+                                          (the rest of the SMs).  0 = auto (on for world_size > 1 with
+                                          MGJ_SHUFFLE_P2P), 1 = on, -1 = off.  Never with EXTERNAL */
+    int32_t  overlap_local_sms;        /* SMs of R's local pass during the overlap (0 = half the SMs) */
+    int32_t  trace;                    /* 1: record the first start and last end (globaltimer, ns) of
+                                          every kernel of the run (mgj_debug_copy MGJ_DBG_TRACE) */
+    int32_t  reserved[1];              /* must be zero */
 } mgj_config;
 
 /*

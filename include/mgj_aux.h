@@ -57,8 +57,19 @@ typedef enum {
     MGJ_DBG_VSTART = 20,     /* u64[2][L+1] sub-partition starts (slots) in MID_R / MID_S */
     MGJ_DBG_BCAST = 21,      /* u8[P]                selective-broadcast flag of each global partition (a2) */
     MGJ_DBG_PLIST = 22,      /* i32[np]              owned partitions: the range, then broadcast ones outside it */
-    MGJ_DBG_SKIP = 23        /* u8[P]                partition has no R or no S tuple anywhere: not shuffled (a2) */
+    MGJ_DBG_SKIP = 23,       /* u8[P]                partition has no R or no S tuple anywhere: not shuffled (a2) */
+    MGJ_DBG_TRACE = 24       /* u64[MGJ_TRACE_COUNT][2] (first start, last end) in ns of each kernel of
+                                the last run (globaltimer; 0 = not run); needs mgj_config.trace = 1 */
 } mgj_debug_what;
+
+/* Trace slots (MGJ_DBG_TRACE), in pipeline order. */
+enum {
+    MGJ_TR_HIST = 0, MGJ_TR_PLAN = 1, MGJ_TR_SCATTER_R = 2, MGJ_TR_SCATTER_S = 3,
+    MGJ_TR_LOCAL_R = 4, MGJ_TR_LOCAL_S = 5, MGJ_TR_LOCAL_RS = 6 /* not stamped (spill) */, MGJ_TR_LOCAL_SPLIT = 7,
+    MGJ_TR_LOCAL_SECOND = 8, MGJ_TR_ITEMIZE = 9, MGJ_TR_PROBE = 10 /* not stamped: between itemize and reduce */,
+    MGJ_TR_REDUCE = 11,
+    MGJ_TRACE_COUNT = 12
+};
 
 mgj_status mgj_debug_copy(mgj_handle h, int32_t what, void *dst, uint64_t bytes, uint64_t *size_out);
 

@@ -6,6 +6,7 @@
 #include <stdint.h>
 
 #include "mgj.h"
+#include "mgj_aux.h"
 
 namespace mgj {
 
@@ -35,7 +36,8 @@ __host__ __device__ constexpr int local2_vcap(int P) { return 4 * P > 4096 ? 4 *
 constexpr uint64_t WAIT_TIMEOUT_NS = 20ull * 1000 * 1000 * 1000;  // default peer-signal wait bound
 
 constexpr int RES_W = 8;  // u64 words per rank in the result mailbox (a6)
-enum Sig { SIG_HIST = 0, SIG_DATA = 1, SIG_RES = 2, SIG_COUNT = 3 };
+// peer flags: histograms published (a1), R / S tuples all stored (a3), partial sums published (a6)
+enum Sig { SIG_HIST = 0, SIG_DATA_R = 1, SIG_RES = 2, SIG_DATA_S = 3, SIG_COUNT = 4 };
 enum Ticket { TK_HIST = 0, TK_SCAT_R = 1, TK_SCAT_S = 2, TK_SCAT_DONE = 3, TK_ITEMS = 4,
               TK_PROBE = 5, TK_LOCAL = 6, TK_COUNT = 8 };
 enum Meta { MT_PLO = 0, MT_PHI = 1, MT_B2 = 2, MT_OK = 3, MT_NCH_R = 4, MT_NCH_S = 5,
@@ -142,6 +144,7 @@ struct Ctx {
     unsigned long long *acc;      // [4] local count, checksum, n_out, pair digest
     int32_t *err;                 // sticky device status
     unsigned long long *result;   // [8] global count, checksum; local n_out; status; global pair digest
+    unsigned long long *trace;    // [MGJ_TRACE_COUNT][2] (UINT64_MAX - first start, last end) or null
     void *out_key, *out_a, *out_b;
 };
 
@@ -170,6 +173,7 @@ __device__ __forceinline__ uint64_t ld_acquire_sys(const uint64_t *p) {
     return v;
 }
 
+
 __device__ __forceinline__ uint64_t globaltimer() {
     uint64_t t;
     asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
@@ -177,6 +181,16 @@ __device__ __forceinline__ uint64_t globaltimer() {
 }
 
 __device__ __forceinline__ void set_err(const Ctx &c, int code) { atomicCAS(c.err, 0, code); }
+
+// Kernel timeline (mgj_config.trace): every CTA's thread 0 stamps its start
+// and end; slot id keeps the earliest start (stored as UINT64_MAX - t so that
+// a zeroed buffer is "empty" for max) and the latest end.
+__device__ __forceinline__ void trace_begin(const Ctx &c, int id, bool who = threadIdx.x == 0) {
+    if (c.trace && who) atomicMax(&c.trace[2 * id], ~(unsigned long long)globaltimer());
+}
+__device__ __forceinline__ void trace_end(const Ctx &c, int id, bool who = threadIdx.x == 0) {
+    if (c.trace && who) atomicMax(&c.trace[2 * id + 1], (unsigned long long)globaltimer());
+}
 
 // Thread-0 helper: wait until every rank g raised flag `kind` for this epoch.
 __device__ inline bool wait_all_flags(const Ctx &c, int kind) {

@@ -69,6 +69,7 @@ __global__ void __launch_bounds__(HIST_THREADS, 2) k_hist(Ctx c) {
         if (bytes)
             tma_load_1d(ring + (size_t)(g % NB) * T, static_cast<const K *>(c.in_key[rel]) + first, bytes, b, pol);
     };
+    trace_begin(c, MGJ_TR_HIST);
     for (int i = tid; i < 2 * P; i += blockDim.x) sub[i] = 0;
     if (tid == 0) {
         for (int i = 0; i < NB; ++i) mbar_init(&bar[i], 1);
@@ -164,6 +165,7 @@ __global__ void __launch_bounds__(HIST_THREADS, 2) k_hist(Ctx c) {
     }
 
     // ---- fused exchange: the last CTA publishes the rank histogram ----
+    trace_end(c, MGJ_TR_HIST);
     __threadfence();
     __syncthreads();
     __shared__ int last;
@@ -306,6 +308,7 @@ __global__ void __launch_bounds__(1024) k_plan(Ctx c) {
     __shared__ int first[MAX_RANKS], endp[MAX_RANKS];
     __shared__ int ok, cap_bad, nbc;
     __shared__ unsigned long long maxr, sumrs, stot, bcs[MAX_RANKS];
+    trace_begin(c, MGJ_TR_PLAN);
     if (tid == 0) {
         ok = wait_all_flags(c, SIG_HIST);
         cap_bad = 0;
@@ -565,10 +568,12 @@ __global__ void __launch_bounds__(1024) k_plan(Ctx c) {
         c.meta[MT_NLP] = np;
         c.meta[MT_OK] = (cap_bad || !fits) ? 0 : 1;
     }
+    trace_end(c, MGJ_TR_PLAN);
 }
 
-__global__ void k_wait(Ctx c, int kind) {
-    if (threadIdx.x == 0 && blockIdx.x == 0) wait_all_flags(c, kind);
+// Wait for every rank's flag `kind` (and `kind2` unless < 0).
+__global__ void k_wait(Ctx c, int kind, int kind2) {
+    if (threadIdx.x == 0 && blockIdx.x == 0 && wait_all_flags(c, kind) && kind2 >= 0) wait_all_flags(c, kind2);
 }
 
 }  // namespace mgj

@@ -251,7 +251,7 @@ __global__ void __launch_bounds__(512) k_countA(Ctx c, const ChunkDesc *cdesc) {
 // ---------------------------------------------------------------------------
 enum LocalMode { LM_SINGLE = 0, LM_SPLIT = 1, LM_SECOND = 2 };
 
-template <typename K, int MODE>
+template <typename K, int MODE, int RSEL = 2>
 __device__ __forceinline__ void local_body(const Ctx &c, const ChunkDesc *cdesc) {
     constexpr bool SPLIT = MODE == LM_SPLIT;
     using Tup = typename Layout<K>::Tup;
@@ -277,7 +277,10 @@ __device__ __forceinline__ void local_body(const Ctx &c, const ChunkDesc *cdesc)
     uint32_t *const abin = bins2 + 2 * QL;
     const uint32_t nch_r = SPLIT ? (uint32_t)c.meta[MT_NCH_R] : nch_local(c, 0);
     const uint32_t total = nch_r + (SPLIT ? (uint32_t)c.meta[MT_NCH_S] : nch_local(c, 1));
-    const uint32_t mine = total > blockIdx.x ? (total - blockIdx.x + gridDim.x - 1) / gridDim.x : 0;
+    // chunks of R [0, nch_r), of S [nch_r, total); RSEL picks R (0), S (1) or both (2)
+    const uint32_t c0 = RSEL == 1 ? nch_r : 0u, c1 = RSEL == 0 ? nch_r : total;
+    const uint32_t span = c1 - c0;
+    const uint32_t mine = span > blockIdx.x ? (span - blockIdx.x + gridDim.x - 1) / gridDim.x : 0;
     constexpr bool from_mid = MODE == LM_SECOND;
     // source of a chunk: the first pass's output, or a receive buffer (this
     // rank's, or a broadcast partition root's for its R side: piece_src)
@@ -295,7 +298,7 @@ __device__ __forceinline__ void local_body(const Ctx &c, const ChunkDesc *cdesc)
     const uint64_t pol = policy_evict_first();
     // thread 0: TMA chunk j (16-byte-aligned superset) into buffer j & 1
     auto issue = [&](uint32_t j, const ChunkDesc &d) {
-        const uint32_t ci = blockIdx.x + j * gridDim.x;
+        const uint32_t ci = c0 + blockIdx.x + j * gridDim.x;
         const int rel = ci < nch_r ? 0 : 1;
         const uint64_t st = from_mid ? d.start : piece_off(d.start);
         const uint64_t g0 = st & ~(uint64_t)(ALIGN - 1);
@@ -309,11 +312,11 @@ __device__ __forceinline__ void local_body(const Ctx &c, const ChunkDesc *cdesc)
     ChunkDesc nxt{};
     constexpr int LI = 32;  // the thread that issues the chunk loads (and the chunked pass's stores)
     if (tid == LI) {
-        if (mine > 0) issue(0, cdesc[blockIdx.x]);
-        if (mine > 1) nxt = cdesc[blockIdx.x + gridDim.x];
+        if (mine > 0) issue(0, cdesc[c0 + blockIdx.x]);
+        if (mine > 1) nxt = cdesc[c0 + blockIdx.x + gridDim.x];
     }
     for (uint32_t j = 0; j < mine; ++j) {
-        const uint32_t ci = blockIdx.x + j * gridDim.x;
+        const uint32_t ci = c0 + blockIdx.x + j * gridDim.x;
         const int rel = ci < nch_r ? 0 : 1;
         const uint32_t li = rel ? ci - nch_r : ci;
         const int X = j & 1;
@@ -346,7 +349,7 @@ __device__ __forceinline__ void local_body(const Ctx &c, const ChunkDesc *cdesc)
         if (tid == LI && j + 1 < mine) {
             if (!SPLIT) bulk_wait_read0();
             issue(j + 1, nxt);
-            if (j + 2 < mine) nxt = cdesc[blockIdx.x + (j + 2) * gridDim.x];
+            if (j + 2 < mine) nxt = cdesc[c0 + blockIdx.x + (j + 2) * gridDim.x];
         }
         if (tid >= 32) {  // the other bin array (last read by chunk j-1 before its S3) for chunk j+1
             uint32_t *const bn = bins2 + (X ^ 1) * QL;
@@ -455,22 +458,34 @@ __device__ inline void chunkmap_second(const Ctx &c, ChunkDesc *desc) {
 template <typename K>
 __global__ void __launch_bounds__(LOCAL_THREADS, 1) k_local_split(Ctx c, const ChunkDesc *cdesc, ChunkDesc *descB) {
     if (!c.meta[MT_OK] || !c.meta[MT_BA]) return;
+    trace_begin(c, MGJ_TR_LOCAL_SPLIT);
     chunkmap_second(c, descB);
     local_body<K, LM_SPLIT>(c, cdesc);
+    trace_end(c, MGJ_TR_LOCAL_SPLIT);
 }
 
 // The chunked pass over the first pass's sub-partitions (a no-op when BA = 0).
 template <typename K>
 __global__ void __launch_bounds__(LOCAL_THREADS, 1) k_local_second(Ctx c, const ChunkDesc *descB) {
     if (!c.meta[MT_OK] || !c.meta[MT_BA]) return;
+    trace_begin(c, MGJ_TR_LOCAL_SECOND);
     local_body<K, LM_SECOND>(c, descB);
+    trace_end(c, MGJ_TR_LOCAL_SECOND);
 }
 
-// The single chunked pass over the owned partitions (a no-op when BA > 0).
-template <typename K>
+// The single chunked pass over the owned partitions (a no-op when BA > 0):
+// the chunks of R (rsel 0), of S (1) or of both (2).  With the shuffle
+// overlapped (§8(e)), R's launch first waits for every rank's R tuples
+// (SIG_DATA_R) and runs beside the scatter of S on the SMs it leaves free.
+template <typename K, int RSEL>
 __global__ void __launch_bounds__(LOCAL_THREADS, 1) k_local(Ctx c, const ChunkDesc *cdesc) {
     if (!c.meta[MT_OK] || c.meta[MT_BA]) return;
-    local_body<K, LM_SINGLE>(c, cdesc);
+    // timeline stamps for the overlapped launches only: in the single launch
+    // over both relations (the one-GPU path) they cost a 4-byte spill
+    constexpr int id = RSEL == 0 ? MGJ_TR_LOCAL_R : MGJ_TR_LOCAL_S;
+    if constexpr (RSEL != 2) trace_begin(c, id);
+    local_body<K, LM_SINGLE, RSEL>(c, cdesc);
+    if constexpr (RSEL != 2) trace_end(c, id);
 }
 
 // ---------------------------------------------------------------------------
@@ -527,6 +542,7 @@ template <typename K>
 __global__ void k_itemize(Ctx c) {
     constexpr int ALIGN = Layout<K>::ALIGN;
     if (!c.meta[MT_OK]) return;
+    trace_begin(c, MGJ_TR_ITEMIZE);
     const int P = c.P, Qmax = 1 << c.b2_max;
     const int Q = 1 << c.meta[MT_QB];  // sub-partitions of the chunked pass
     const uint32_t cap = (uint32_t)c.probe_slots;
@@ -590,6 +606,7 @@ __global__ void k_itemize(Ctx c) {
             ++ir;
         });
     }
+    trace_end(c, MGJ_TR_ITEMIZE);
 }
 
 __host__ __device__ inline size_t probe_smem_bytes(int slots, int TB) {
@@ -1029,6 +1046,7 @@ __global__ void __launch_bounds__(PROBE_THREADS, 1) k_probe(Ctx c) {
 // ---------------------------------------------------------------------------
 __global__ void k_reduce(Ctx c) {
     if (threadIdx.x != 0 || blockIdx.x != 0) return;
+    trace_begin(c, MGJ_TR_REDUCE);
     const int32_t st = *(volatile int32_t *)c.err;
     const unsigned long long v[5] = {__ldcg(&c.acc[0]), __ldcg(&c.acc[1]), __ldcg(&c.acc[2]),
                                      (unsigned long long)(uint32_t)st, __ldcg(&c.acc[3])};
@@ -1059,6 +1077,7 @@ __global__ void k_reduce(Ctx c) {
     c.result[2] = v[2];
     c.result[3] = (unsigned long long)(uint32_t)gst;
     c.result[4] = dig;
+    trace_end(c, MGJ_TR_REDUCE);
 }
 
 }  // namespace mgj

@@ -42,9 +42,11 @@ int ceil_log2(uint64_t x) {
 mgj_status normalize(const mgj_config *in, Norm *o) {
     if (!in) return MGJ_EINVAL;
     mgj_config c = *in;
-    for (int i = 0; i < 4; ++i)
+    for (int i = 0; i < 1; ++i)
         if (c.reserved[i]) return MGJ_EINVAL;
     if (c.peer_timeout_ms < 0) return MGJ_EINVAL;
+    if (c.shuffle_overlap < -1 || c.shuffle_overlap > 1 || c.overlap_local_sms < 0) return MGJ_EINVAL;
+    if (c.trace != 0 && c.trace != 1) return MGJ_EINVAL;
     if (c.skew_bcast < -1 || c.skew_bcast > 1) return MGJ_EINVAL;
     if (c.local_split_bits < -1 || c.local_split_bits > MAX_BA) return MGJ_EINVAL;
     if (c.shuffle_mode != MGJ_SHUFFLE_P2P && c.shuffle_mode != MGJ_SHUFFLE_EXTERNAL) return MGJ_EINVAL;
@@ -155,6 +157,11 @@ struct mgj_plan_s {
     int32_t *h_meta = nullptr;
     uint64_t recv_r = 0, recv_s = 0;
     int32_t host_err = 0;
+    // §8(e) overlap: R's local pass on a second stream beside S's scatter
+    bool overlap = false;
+    int local_sms = 0, scatter_sms = 0;
+    cudaStream_t aux = nullptr;
+    cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
 };
 
 namespace {
@@ -196,7 +203,9 @@ cudaError_t set_attrs(const Norm &n) {
     if ((e = cudaFuncSetAttribute(k_hist<K>, A, (int)hist_smem(n)))) return e;
     if ((e = cudaFuncSetAttribute(k_plan, A, (int)plan_smem(n)))) return e;
     if ((e = cudaFuncSetAttribute(scatter_kernel<K>(n.P), A, (int)scatter_smem(n)))) return e;
-    if ((e = cudaFuncSetAttribute(k_local<K>, A, (int)local_smem(n)))) return e;
+    if ((e = cudaFuncSetAttribute(k_local<K, 0>, A, (int)local_smem(n)))) return e;
+    if ((e = cudaFuncSetAttribute(k_local<K, 1>, A, (int)local_smem(n)))) return e;
+    if ((e = cudaFuncSetAttribute(k_local<K, 2>, A, (int)local_smem(n)))) return e;
     if ((e = cudaFuncSetAttribute(k_local_second<K>, A, (int)local_smem2(n)))) return e;
     if ((e = cudaFuncSetAttribute(k_local_split<K>, A, (int)local_smem1s(n)))) return e;
     if ((e = cudaFuncSetAttribute(k_planA, A, (int)planA_smem(n)))) return e;
@@ -230,15 +239,36 @@ void launch_shuffle(mgj_plan_s *h, cudaStream_t s) {
     Ctx cs = h->ctx;
     if (cs.ext)
         for (int g = 0; g < MAX_RANKS; ++g) cs.arena[g] = h->send_arena;
-    scatter_kernel<K>(n.P)<<<h->ctx.G, scatter_threads(n.P, n.c.key_bytes), scatter_smem(n), s>>>(cs);
-    h->launches += 4;
+    const auto scat = scatter_kernel<K>(n.P);
+    const int nt = scatter_threads(n.P, n.c.key_bytes);
+    if (h->overlap) {
+        scat<<<h->ctx.G, nt, scatter_smem(n), s>>>(cs, 0, 0);  // a3, R
+        // §8(e) ("data distribution and local partitioning start
+        // together"; Rationale 2): once every rank's R tuples have
+        // landed, R is partitioned locally on local_sms SMs of a second stream
+        // while S is scattered on the others
+        cudaEventRecord(h->ev_fork, s);
+        cudaStreamWaitEvent(h->aux, h->ev_fork, 0);
+        k_wait<<<1, 32, 0, h->aux>>>(h->ctx, SIG_DATA_R, -1);
+        k_local<K, 0><<<h->local_sms, LOCAL_THREADS, local_smem(n), h->aux>>>(h->ctx, h->cdesc);
+        cudaEventRecord(h->ev_join, h->aux);
+        scat<<<h->scatter_sms, nt, scatter_smem(n), s>>>(cs, 1, 1);  // a3, S
+        h->launches += 7;
+    } else {
+        scat<<<h->ctx.G, nt, scatter_smem(n), s>>>(cs, 0, 1);  // a3, R then S in one launch
+        h->launches += 4;
+    }
 }
 
 template <typename K>
 void launch_join(mgj_plan_s *h, cudaStream_t s) {
     const Norm &n = h->n;
-    if (!h->ctx.ext) {  // EXTERNAL: the caller's exchange is stream-ordered
-        k_wait<<<1, 32, 0, s>>>(h->ctx, SIG_DATA);
+    if (h->overlap) {
+        cudaStreamWaitEvent(s, h->ev_join, 0);  // R's local pass (second stream) is done
+        k_wait<<<1, 32, 0, s>>>(h->ctx, SIG_DATA_S, -1);
+        h->launches += 1;
+    } else if (!h->ctx.ext) {  // EXTERNAL: the caller's exchange is stream-ordered
+        k_wait<<<1, 32, 0, s>>>(h->ctx, SIG_DATA_R, SIG_DATA_S);
         h->launches += 1;
     }
     // two-level local partitioning: k_plan decides on the device (MT_BA); when
@@ -253,7 +283,10 @@ void launch_join(mgj_plan_s *h, cudaStream_t s) {
         k_local_second<K><<<h->nsm, LOCAL_THREADS, local_smem2(n), s>>>(h->ctx, h->cdescB);
         h->launches += 4;
     }
-    k_local<K><<<h->nsm, LOCAL_THREADS, local_smem(n), s>>>(h->ctx, h->cdesc);
+    if (h->overlap)
+        k_local<K, 1><<<h->nsm, LOCAL_THREADS, local_smem(n), s>>>(h->ctx, h->cdesc);
+    else
+        k_local<K, 2><<<h->nsm, LOCAL_THREADS, local_smem(n), s>>>(h->ctx, h->cdesc);
     cudaEventRecord(h->ev[4], s);
     k_itemize<K><<<h->nsm * 4, 256, 0, s>>>(h->ctx);
     if (n.c.materialize)
@@ -415,6 +448,16 @@ mgj_status mgj_plan(const mgj_config *cfg, const mgj_peers *peers, mgj_handle *o
         c.out_a = dalloc(h, n.out_cap * n.c.key_bytes, &st);
         c.out_b = dalloc(h, n.out_cap * n.c.key_bytes, &st);
     }
+    if (n.c.trace) c.trace = static_cast<unsigned long long *>(dalloc(h, MGJ_TRACE_COUNT * 2 * 8, &st));
+    h->overlap = !c.ext && (n.c.shuffle_overlap > 0 || (n.c.shuffle_overlap == 0 && W > 1));
+    if (h->overlap) {
+        h->local_sms = n.c.overlap_local_sms ? std::min(n.c.overlap_local_sms, h->nsm - 1) : h->nsm / 2;
+        h->local_sms = std::max(h->local_sms, 1);
+        h->scatter_sms = std::max(h->nsm - h->local_sms, 1);
+        if (st == MGJ_OK) st = cuda_ok(cudaStreamCreateWithFlags(&h->aux, cudaStreamNonBlocking));
+        if (st == MGJ_OK) st = cuda_ok(cudaEventCreateWithFlags(&h->ev_fork, cudaEventDisableTiming));
+        if (st == MGJ_OK) st = cuda_ok(cudaEventCreateWithFlags(&h->ev_join, cudaEventDisableTiming));
+    }
     if (st == MGJ_OK) st = cuda_ok(cudaMallocHost(&h->h_res, 8 * 8 + MT_COUNT * 4));
     if (st == MGJ_OK) h->h_meta = reinterpret_cast<int32_t *>(h->h_res + 8);
     for (int i = 0; i < 7 && st == MGJ_OK; ++i) st = cuda_ok(cudaEventCreate(&h->ev[i]));
@@ -482,6 +525,7 @@ mgj_status mgj_partition(mgj_handle h, const void *r_keys, const void *r_payload
     c.n_in[1] = n_s;
     h->stream = s;
     if (cudaMemsetAsync(h->zero_block, 0, h->zero_bytes, s) != cudaSuccess) return MGJ_ECUDA;
+    if (c.trace && cudaMemsetAsync(c.trace, 0, MGJ_TRACE_COUNT * 2 * 8, s) != cudaSuccess) return MGJ_ECUDA;
     cudaEventRecord(h->ev[0], s);
     if (n.c.key_bytes == 4) launch_partition<uint32_t>(h, s);
     else launch_partition<uint64_t>(h, s);
@@ -589,6 +633,12 @@ void mgj_destroy(mgj_handle h) {
     if (h->h_res) cudaFreeHost(h->h_res);
     for (int i = 0; i < 7; ++i)
         if (h->ev[i]) cudaEventDestroy(h->ev[i]);
+    if (h->aux) {
+        cudaStreamSynchronize(h->aux);
+        cudaStreamDestroy(h->aux);
+    }
+    if (h->ev_fork) cudaEventDestroy(h->ev_fork);
+    if (h->ev_join) cudaEventDestroy(h->ev_join);
     delete h;
 }
 
@@ -751,6 +801,16 @@ mgj_status mgj_debug_copy(mgj_handle h, int32_t what, void *dst, uint64_t bytes,
             break;
         }
         case MGJ_DBG_VSTART: src = c.vstart; size = 2ull * c.cb_stride * 8; break;
+        case MGJ_DBG_TRACE: {
+            if (!c.trace) return MGJ_EINVAL;
+            unsigned long long t[MGJ_TRACE_COUNT * 2];
+            if (cudaMemcpy(t, c.trace, sizeof(t), cudaMemcpyDeviceToHost) != cudaSuccess) return MGJ_ECUDA;
+            for (int i = 0; i < MGJ_TRACE_COUNT; ++i)
+                if (t[2 * i]) t[2 * i] = ~t[2 * i];  // stored as UINT64_MAX - first start
+            if (size_out) *size_out = sizeof(t);
+            if (dst && bytes) memcpy(dst, t, std::min<uint64_t>(bytes, sizeof(t)));
+            return MGJ_OK;
+        }
         case MGJ_DBG_OUT_KEY:
         case MGJ_DBG_OUT_PAY_R:
         case MGJ_DBG_OUT_PAY_S: {

@@ -135,33 +135,39 @@ __device__ __forceinline__ void st_group(void *dst, const typename Vec<BYTES>::T
 // after partitioning based on the histogram and then writes the tuple" —
 // after Rui et al. [38]; step 3 data distribution, P:405-407 and §4).
 //
-// B200 form: one persistent CTA (1024 threads) per SM processes tile
-// c = blockIdx.x of R and then of S, in sub-tiles of T tuples that a TMA
-// bulk copy brings into shared memory one sub-tile ahead.  Per sub-tile:
-//  1. each thread takes LU-tuple vectors of keys and payloads from the stage
-//     and ranks every tuple in its digit1 bin (one shared atomic);
-//  2. thread t owns partitions t*PPT.. (PPT per thread) and keeps, in
+// B200 form: one launch per relation (rel); persistent CTAs (1024 threads,
+// one per SM) take tiles c = blockIdx.x, + gridDim.x, ... of that relation
+// (one tile per CTA at full grid; fewer CTAs when the launch shares the GPU
+// with the local pass of the other relation, §8(e) overlap) and stream each
+// tile in sub-tiles of T tuples whose keys a TMA bulk copy brings into shared
+// memory one sub-tile ahead (payloads: L2 prefetch, then registers).  Per
+// sub-tile:
+//  1. thread t owns partitions t*PPT.. (PPT per thread) and keeps, in
 //     registers, each one's destination cursor and its < 32-byte tail
 //     (carry) from the previous sub-tile; a block scan of the per-partition
-//     sizes (carry + new, rounded up to a 32-byte group) lays the partitions
-//     out group-aligned in `sorted`, the carry first;
-//  3. tuples are scattered into `sorted`, then written out one 32-byte group
-//     per thread and store (st.global.v8.b32): every complete group is a
-//     whole DRAM sector at its final address — owner(p)'s receive buffer at
-//     send_off[p] (a2) + tile_base[c][p] (a1 tile prefix) + the running
-//     count of p in this tile; no global atomics.  An incomplete last group
-//     stays in `sorted` and its owning thread reloads it as the next carry.
+//     sizes (carry + new, rounded up to a 32-byte group; a1 counted them)
+//     lays the partitions out group-aligned in `sorted`, the carry first;
+//  2. each thread ranks its tuples in their digit1 bins (one shared atomic
+//     each) and scatters them into `sorted`;
+//  3. the sorted sub-tile is written out one 32-byte group per thread and
+//     store (st.global.v8.b32): every complete group is a whole DRAM sector
+//     at its final address — owner(p)'s receive buffer at send_off[p] (a2) +
+//     tile_base[c][p] (a1 tile prefix) + the running count of p in this tile;
+//     no global atomics.  An incomplete last group stays in `sorted` and its
+//     owning thread reloads it as the next carry.
 // A tile's first destination of a partition need not be group-aligned: the
 // carry then starts with h placeholder slots (key = p) that are never stored
-// (the head group is written tuple by tuple from slot h).  The relation's
-// remaining tails are written tuple by tuple at its end.  On NVSwitch the
-// owner may be another GPU: the same stores go over NVLink to a peer-mapped
-// address; the paper's packets, routing buffers and multi-hop routing (§4)
-// have no role on a one-hop fabric.  The last CTA raises SIG_DATA at every
-// peer after a system fence.
+// (the head group is written tuple by tuple from slot h).  A tile's remaining
+// tails are written tuple by tuple at its end.  On NVSwitch the owner may be
+// another GPU: the same stores go over NVLink to a peer-mapped address; the
+// paper's packets, routing buffers and multi-hop routing (§4) have no role on
+// a one-hop fabric.  With N > 1 each CTA starts its write-out sweep at a
+// different destination rank (rotated group order), so that the CTAs' stores
+// spread over all peers' links instead of visiting the ranks in step.  The
+// last CTA raises SIG_DATA_R / SIG_DATA_S at every peer after a system fence.
 // ---------------------------------------------------------------------------
 template <typename K, int T, int SG, int PPT, int NT>
-__global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c) {
+__global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c, int rel0, int rel1) {
     using Tup = typename TupT<K>::T;
     constexpr int TB = (int)sizeof(Tup);
     constexpr int V = T / NT;                  // tuples per thread per sub-tile
@@ -180,8 +186,7 @@ __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c) {
         if constexpr (SG > 1 && SG * sizeof(Tup) == 32) return s ^ (((s >> (SG == 4 ? 4 : 3)) & 1u) * (SG / 2));
         else return s;
     };
-    // 8-byte keys: both group halves and the whole descriptor are loaded up
-    // front (measured: M5 scatter 3.725 -> 3.693 ms; 4-byte keys 4.155 -> 4.19)
+    // 8-byte keys: the whole descriptor is loaded with one 16-byte access
     constexpr bool EAGER = sizeof(K) == 8;
     extern __shared__ __align__(128) unsigned char smem[];
     const int P = c.P;
@@ -196,20 +201,50 @@ __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c) {
     __shared__ __align__(8) uint64_t bar;
     __shared__ uint32_t tmp[32];
     const int tid = threadIdx.x;
-    const int tile = blockIdx.x;
     const int ok = *(volatile int32_t *)&c.meta[MT_OK];
 
-    uint64_t lo0, hi0, lo1, hi1;  // scalars (no local-memory arrays)
-    tile_range(c.n_in[0], c.G, tile, lo0, hi0);
-    tile_range(c.n_in[1], c.G, tile, lo1, hi1);
-    const uint32_t nsub0 = ok ? (uint32_t)((hi0 - lo0 + T - 1) / T) : 0;
-    const uint32_t ntot = nsub0 + (ok ? (uint32_t)((hi1 - lo1 + T - 1) / T) : 0);
+    for (int rel = rel0; rel <= rel1; ++rel) trace_begin(c, rel ? MGJ_TR_SCATTER_S : MGJ_TR_SCATTER_R);
     if (tid == 0) {
         mbar_init(&bar, 1);
         fence_mbar_init();
     }
     __syncthreads();
     const uint64_t pol = policy_evict_first();
+
+    // This CTA's sub-tiles: tiles blockIdx.x + k * gridDim.x, each cut into
+    // sub-tiles of T tuples.  A cursor (k, j) walks them in order.
+    // This CTA's sub-tiles: for rel = rel0..rel1, tiles blockIdx.x + k *
+    // gridDim.x of the relation, each cut into sub-tiles of T tuples.  A
+    // cursor walks them in order (across the relation boundary, so the next
+    // sub-tile is always prefetched).
+    struct Cur {
+        int rel, tile;
+        uint32_t j, nsub;
+        uint64_t lo, hi;  // the tile's tuple range (computed once per tile: 64-bit divisions)
+    };
+    auto at_tile = [&](int rel, int tile) -> Cur {  // first non-empty tile from (rel, tile) on
+        Cur u{rel, tile, 0, 0, 0, 0};
+        for (; u.rel <= rel1; ++u.rel, u.tile = (int)blockIdx.x) {
+            const uint64_t n = ok ? c.n_in[u.rel] : 0;
+            for (; u.tile < c.G; u.tile += gridDim.x) {
+                tile_range(n, c.G, u.tile, u.lo, u.hi);
+                u.nsub = (uint32_t)((u.hi - u.lo + T - 1) / T);
+                if (u.nsub) return u;
+            }
+        }
+        return u;  // u.rel > rel1: done
+    };
+    auto next_cur = [&](Cur u) -> Cur {
+        if (u.j + 1 < u.nsub) {
+            ++u.j;
+            return u;
+        }
+        return at_tile(u.rel, u.tile + gridDim.x);
+    };
+    auto span = [&](const Cur &u, uint64_t &first, uint32_t &len) {
+        first = u.lo + (uint64_t)u.j * T;
+        len = (uint32_t)min((uint64_t)T, u.hi - first);
+    };
 
     // per owned partition (registers): destination of the next group, carry
     ull base[PPT];
@@ -220,26 +255,21 @@ __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c) {
 #pragma unroll
     for (int k = 0; k < PPT; ++k) base[k] = 0, cc[k] = 0, hd[k] = 0, lim[k] = 0, skp[k] = false;
 
-    auto subtile = [&](uint32_t g, int &rel, uint64_t &first, uint32_t &len) {
-        rel = g < nsub0 ? 0 : 1;
-        const uint32_t j = rel ? g - nsub0 : g;
-        first = (rel ? lo1 : lo0) + (uint64_t)j * T;
-        len = (uint32_t)min((uint64_t)T, (rel ? hi1 : hi0) - first);
-    };
-    auto issue = [&](uint32_t g) {  // thread 0: TMA the 16-byte-aligned body of sub-tile g
-        int rel;
+    auto issue = [&](const Cur &u) {  // thread 0: TMA the 16-byte-aligned body of sub-tile u's keys
         uint64_t first;
         uint32_t len;
-        subtile(g, rel, first, len);
+        span(u, first, len);
+        const K *in_key = static_cast<const K *>(c.in_key[u.rel]);
+        const K *in_pay = static_cast<const K *>(c.in_pay[u.rel]);
         const uint32_t bytes = (len & ~(uint32_t)(LU - 1)) * (uint32_t)sizeof(K);
         mbar_arrive_expect_tx(&bar, bytes);
         if (bytes) {
-            tma_load_1d(skey, static_cast<const K *>(c.in_key[rel]) + first, bytes, &bar, pol);
+            tma_load_1d(skey, in_key + first, bytes, &bar, pol);
             // payloads: brought into L2 now and loaded into registers while the
             // previous sub-tile is written out (the shared memory of a payload
             // stage goes to a 1.5x larger sub-tile instead; measured at M2:
             // scatter 4.12 -> 3.89 ms; without the L2 prefetch 4.65 ms)
-            prefetch_l2(static_cast<const K *>(c.in_pay[rel]) + first, bytes);
+            prefetch_l2(in_pay + first, bytes);
         }
     };
     auto fetch_carry = [&]() {  // the incomplete last groups of the previous sub-tile -> registers
@@ -252,7 +282,7 @@ __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c) {
             pending = false;
         }
     };
-    auto flush = [&]() {  // end of a relation: store the remaining tails tuple by tuple
+    auto flush = [&]() {  // end of a tile: store the remaining tails tuple by tuple
         fetch_carry();
 #pragma unroll
         for (int k = 0; k < PPT; ++k)
@@ -260,7 +290,7 @@ __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c) {
             for (int i = 0; i < CW; ++i)
                 if (!skp[k] && i >= (int)hd[k] && i < (int)cc[k]) reinterpret_cast<Tup *>(base[k])[i] = carry[k][i];
     };
-    auto set_base = [&](int rel) {  // destination of this tile's first tuple of each owned partition
+    auto set_base = [&](int rel, int tile) {  // destination of this tile's first tuple of each owned partition
         const uint32_t *tb = c.tile_base + ((size_t)rel * c.G + tile) * P;
         const uint64_t *so = c.send_off + (size_t)rel * P;
 #pragma unroll
@@ -285,14 +315,12 @@ __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c) {
         }
     };
 
-    // counts of sub-tile g for this thread's partitions (a1 wrote them, u16 per partition)
-    auto load_counts = [&](uint32_t g, uint32_t (&out)[PPT]) {
+    // counts of sub-tile u for this thread's partitions (a1 wrote them, u16 per partition)
+    auto load_counts = [&](const Cur &u, uint32_t (&out)[PPT]) {
 #pragma unroll
         for (int k = 0; k < PPT; ++k) out[k] = 0;
-        if (g >= ntot || tid * PPT >= P) return;
-        const int rel = g < nsub0 ? 0 : 1;
-        const uint32_t j = rel ? g - nsub0 : g;
-        const uint16_t *src = c.sub_hist + (((size_t)rel * c.G + tile) * c.sub_ns + j) * P + tid * PPT;
+        if (u.rel > rel1 || tid * PPT >= P) return;
+        const uint16_t *src = c.sub_hist + (((size_t)u.rel * c.G + u.tile) * c.sub_ns + u.j) * P + tid * PPT;
         if constexpr (PPT == 1) {
             out[0] = __ldg(src);
         } else if constexpr (PPT == 2) {
@@ -303,45 +331,52 @@ __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c) {
             out[0] = v.x & 0xffffu, out[1] = v.x >> 16, out[2] = v.y & 0xffffu, out[3] = v.y >> 16;
         }
     };
-    // payloads of sub-tile g (L2-resident since issue(g)), loaded into
+    // payloads of sub-tile u (L2-resident since issue(u)), loaded into
     // registers while the previous sub-tile is written out
     K pp[V];
-    auto load_pay = [&](uint32_t g) {
-        int rel;
+    auto load_pay = [&](const Cur &u) {
         uint64_t first;
         uint32_t len;
-        subtile(g, rel, first, len);
-        const K *gp = static_cast<const K *>(c.in_pay[rel]) + first;
+        span(u, first, len);
+        const K *gp = static_cast<const K *>(c.in_pay[u.rel]) + first;
         if (len == T) {
 #pragma unroll
-            for (int u = 0; u < NU; ++u) {
-                const uint4 b = __ldcs(reinterpret_cast<const uint4 *>(gp + (uint32_t)(u * NT + tid) * LU));
-                memcpy(&pp[u * LU], &b, 16);
+            for (int x = 0; x < NU; ++x) {
+                const uint4 b = __ldcs(reinterpret_cast<const uint4 *>(gp + (uint32_t)(x * NT + tid) * LU));
+                memcpy(&pp[x * LU], &b, 16);
             }
         } else {
 #pragma unroll
-            for (int u = 0; u < NU; ++u)
+            for (int x = 0; x < NU; ++x)
 #pragma unroll
                 for (int e = 0; e < LU; ++e) {
-                    const uint32_t i = (uint32_t)(u * NT + tid) * LU + e;
-                    pp[u * LU + e] = i < len ? __ldcs(gp + i) : (K)0;
+                    const uint32_t i = (uint32_t)(x * NT + tid) * LU + e;
+                    pp[x * LU + e] = i < len ? __ldcs(gp + i) : (K)0;
                 }
         }
     };
+    // write-out rotation (N > 1): CTA b starts its sweep of the groups at rank
+    // b mod N's share of them (owner ranges are contiguous in p, so in group order)
+    const uint32_t rot_num = c.world > 1 ? (uint32_t)(blockIdx.x % c.world) : 0u;
+
+    Cur u = at_tile(rel0, (int)blockIdx.x);
     uint32_t ncnt[PPT];
-    load_counts(0, ncnt);
-    if (tid == 0 && ntot > 0) issue(0);
-    if (ntot > 0) load_pay(0);
-    int cur_rel = -1;
-    for (uint32_t g = 0; g < ntot; ++g) {
-        int rel;
+    load_counts(u, ncnt);
+    if (u.rel <= rel1) {
+        if (tid == 0) issue(u);
+        load_pay(u);
+    }
+    int cur_tile = -1;       // (relation, tile) the partition state belongs to: rel * G + tile
+    uint32_t nsub_done = 0;  // sub-tiles processed (the stage barrier's phase parity)
+    for (; u.rel <= rel1; u = next_cur(u), ++nsub_done) {
         uint64_t first;
         uint32_t len;
-        subtile(g, rel, first, len);
-        if (rel != cur_rel) {  // thread-private partition state: no barrier needed
-            if (cur_rel >= 0) flush();
-            set_base(rel);
-            cur_rel = rel;
+        span(u, first, len);
+        const Cur nx = next_cur(u);
+        if (u.rel * c.G + u.tile != cur_tile) {  // thread-private partition state: no barrier needed
+            if (cur_tile >= 0) flush();
+            set_base(u.rel, u.tile);
+            cur_tile = u.rel * c.G + u.tile;
         }
         fetch_carry();
         // lay out this sub-tile's partitions (known from a1): carry + new tuples, group-rounded
@@ -352,7 +387,7 @@ __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c) {
             seg[k] = (cnt[k] + SG - 1) & ~(uint32_t)(SG - 1);
             tsum += seg[k];
         }
-        load_counts(g + 1, ncnt);  // prefetch (consumed next iteration)
+        load_counts(nx, ncnt);  // prefetch (consumed next iteration)
         uint32_t total;
         uint32_t o = block_scan_reg(tsum, tmp, total);  // its barriers: the last write-out is done
 #pragma unroll
@@ -378,28 +413,27 @@ __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c) {
         }
         pending = SG > 1;
         K kk[V];
-        mbar_wait(&bar, g & 1);
+        mbar_wait(&bar, nsub_done & 1);
         const uint32_t body = len & ~(uint32_t)(LU - 1);
-        const K *gk = static_cast<const K *>(c.in_key[rel]) + first;
+        const K *gk = static_cast<const K *>(c.in_key[u.rel]) + first;
         if (len == T) {  // full sub-tile: branch-free vector loads
 #pragma unroll
-            for (int u = 0; u < NU; ++u) {
-                const uint32_t i0 = (uint32_t)(u * NT + tid) * LU;
-                const uint4 a = *reinterpret_cast<const uint4 *>(skey + i0);
-                memcpy(&kk[u * LU], &a, 16);
+            for (int x = 0; x < NU; ++x) {
+                const uint4 a = *reinterpret_cast<const uint4 *>(skey + (uint32_t)(x * NT + tid) * LU);
+                memcpy(&kk[x * LU], &a, 16);
             }
         } else {
 #pragma unroll
-            for (int u = 0; u < NU; ++u) {
+            for (int x = 0; x < NU; ++x) {
 #pragma unroll
                 for (int e = 0; e < LU; ++e) {  // < LU trailing tuples of the relation come from global
-                    const uint32_t i = (uint32_t)(u * NT + tid) * LU + e;
-                    kk[u * LU + e] = i < body ? skey[i] : (i < len ? gk[i] : (K)0);
+                    const uint32_t i = (uint32_t)(x * NT + tid) * LU + e;
+                    kk[x * LU + e] = i < body ? skey[i] : (i < len ? gk[i] : (K)0);
                 }
             }
         }
         __syncthreads();  // S1: offsets and carries in place, stage consumed
-        if (tid == 0 && g + 1 < ntot) issue(g + 1);
+        if (tid == 0 && nx.rel <= rel1) issue(nx);
 #pragma unroll
         for (int v = 0; v < V; ++v) {
             const uint32_t i = (uint32_t)((v / LU) * NT + tid) * LU + (v % LU);
@@ -411,11 +445,13 @@ __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c) {
             }
         }
         __syncthreads();  // S2
-        if (g + 1 < ntot) load_pay(g + 1);  // the ranking of this sub-tile has consumed pp
-        // write-out: one group per thread per step
+        if (nx.rel <= rel1) load_pay(nx);  // the ranking of this sub-tile has consumed pp
+        // write-out: one group per thread per step, rotated by rank share for N > 1
         const uint32_t ngroups = total / SG;
-        for (uint32_t u = tid; u < ngroups; u += NT) {
-            const uint32_t slot = u * SG;
+        const uint32_t rot = (uint32_t)(((uint64_t)ngroups * rot_num) / (uint32_t)c.world);
+        for (uint32_t w = tid; w < ngroups; w += NT) {
+            const uint32_t gi = w + rot < ngroups ? w + rot : w + rot - ngroups;
+            const uint32_t slot = gi * SG;
             GV gv;
             PInfo in;
             if constexpr (GB == 32) {  // two conflict-free 16-byte halves (swizzled)
@@ -436,8 +472,8 @@ __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c) {
                 const uint2 lh = lds64_at(pa + 8);
                 in.lim = lh.x;
                 in.head = lh.y;
-                const uint2 w = lds64_at(pa);
-                in.wb = (ull)w.x | ((ull)w.y << 32);
+                const uint2 wv = lds64_at(pa);
+                in.wb = (ull)wv.x | ((ull)wv.y << 32);
             }
             if (slot + SG <= in.lim) {
                 char *dst = reinterpret_cast<char *>(in.wb + (ull)slot * TB);
@@ -449,22 +485,23 @@ __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c) {
             }
         }
     }
-    if (cur_rel >= 0) flush();
+    if (cur_tile >= 0) flush();
 
     // ---- every CTA: make its (peer) stores visible, the last one signals ----
     __threadfence_system();
     __syncthreads();
+    for (int rel = rel0; rel <= rel1; ++rel) trace_end(c, rel ? MGJ_TR_SCATTER_S : MGJ_TR_SCATTER_R);
     if (tid == 0) {
-        const uint32_t t = atomicAdd(&c.ticket[TK_SCAT_DONE], 1u);
+        const uint32_t t = atomicAdd(&c.ticket[rel0 ? TK_SCAT_S : TK_SCAT_R], 1u);
         if (t == gridDim.x - 1) {
             __threadfence_system();
-            signal_all(c, SIG_DATA);
+            for (int rel = rel0; rel <= rel1; ++rel) signal_all(c, rel ? SIG_DATA_S : SIG_DATA_R);
         }
     }
 }
 
 template <typename K>
-inline void (*scatter_kernel(int P))(Ctx) {
+inline void (*scatter_kernel(int P))(Ctx, int, int) {
     constexpr ScatGeom g1 = scat_geom(1024, sizeof(K)), g2 = scat_geom(2048, sizeof(K)), g4 = scat_geom(4096, sizeof(K));
     if (P <= 1024) return k_scatter<K, g1.T, g1.SG, g1.PPT, g1.NT>;
     if (P == 2048) return k_scatter<K, g2.T, g2.SG, g2.PPT, g2.NT>;

@@ -27,7 +27,11 @@ MAX_RANKS = 8
 # mgj_debug_what
 DBG = dict(RANK_HIST=1, MAIL_HIST=2, OWNER=3, SEND_OFF=4, RECV_SIZE=5, RECV_R=6, RECV_S=7,
            LOCAL_R=8, LOCAL_S=9, META=10, CHUNK_OFF_R=11, CHUNK_OFF_S=12, CHUNK_BASE=13, SEGMENTS=14,
-           OUT_KEY=15, OUT_PAY_R=16, OUT_PAY_S=17, MID_R=18, MID_S=19, VSTART=20, BCAST=21, PLIST=22, SKIP=23)
+           OUT_KEY=15, OUT_PAY_R=16, OUT_PAY_S=17, MID_R=18, MID_S=19, VSTART=20, BCAST=21, PLIST=22, SKIP=23,
+           TRACE=24)
+# trace slots (include/mgj_aux.h MGJ_TR_*), in pipeline order
+TRACE_NAMES = ["hist", "plan", "scatter_R", "scatter_S", "local_R", "local_S", "local_RS", "local_split",
+               "local_second", "itemize", "probe", "reduce"]
 GEN_KIND = {"unique": 0, "zipf": 1, "wide": 2}
 
 
@@ -48,7 +52,9 @@ class Config(ctypes.Structure):
                 ("materialize", ctypes.c_int32), ("num_sms", ctypes.c_int32),
                 ("out_capacity", ctypes.c_uint64), ("shuffle_mode", ctypes.c_int32),
                 ("local_split_bits", ctypes.c_int32), ("skew_bcast", ctypes.c_int32),
-                ("peer_timeout_ms", ctypes.c_int32), ("reserved", ctypes.c_int32 * 4)]
+                ("peer_timeout_ms", ctypes.c_int32), ("shuffle_overlap", ctypes.c_int32),
+                ("overlap_local_sms", ctypes.c_int32), ("trace", ctypes.c_int32),
+                ("reserved", ctypes.c_int32 * 1)]
 
 
 class Exchange(ctypes.Structure):
@@ -133,7 +139,7 @@ def _stream(stream):
 def make_config(rank=0, world_size=1, key_bytes=4, r_capacity=0, s_capacity=0, recv_capacity_r=0,
                 recv_capacity_s=0, radix_bits_global=0, radix_bits_local=0, materialize=False,
                 num_sms=0, out_capacity=0, shuffle_mode=0, local_split_bits=0, skew_bcast=0,
-                peer_timeout_ms=0) -> Config:
+                peer_timeout_ms=0, shuffle_overlap=0, overlap_local_sms=0, trace=False) -> Config:
     c = Config()
     c.rank, c.world_size = rank, world_size
     c.key_bytes = c.payload_bytes = key_bytes
@@ -147,6 +153,9 @@ def make_config(rank=0, world_size=1, key_bytes=4, r_capacity=0, s_capacity=0, r
     c.local_split_bits = local_split_bits
     c.skew_bcast = skew_bcast
     c.peer_timeout_ms = peer_timeout_ms
+    c.shuffle_overlap = shuffle_overlap
+    c.overlap_local_sms = overlap_local_sms
+    c.trace = int(bool(trace))
     return c
 
 
@@ -220,6 +229,14 @@ class Join:
         if buf.size:
             _check(_lib.mgj_debug_copy(self._h, DBG[what], buf.ctypes.data, buf.size, None), "mgj_debug_copy")
         return buf.view(dtype)
+
+    def trace(self) -> dict:
+        """Kernel timeline of the last run (needs trace=True): name -> (first start, last end) in ns
+        relative to the earliest start; kernels that did not run are left out."""
+        t = self.debug("TRACE", np.uint64).reshape(-1, 2)
+        live = [(n, int(a), int(b)) for n, (a, b) in zip(TRACE_NAMES, t) if a and b]
+        t0 = min(a for _, a, _ in live) if live else 0
+        return {n: (a - t0, b - t0) for n, a, b in live}
 
     def materialized(self, res: dict):
         """Copy this rank's materialised triples to host numpy arrays (key, payR, payS)."""

@@ -47,7 +47,8 @@ def test_strerror(mgj):
 @pytest.mark.parametrize("bad", [dict(key_bytes=3), dict(world_size=0), dict(world_size=9), dict(rank=2, world_size=2),
                                  dict(radix_bits_global=13), dict(radix_bits_local=12), dict(r_capacity=1 << 32),
                                  dict(local_split_bits=7), dict(local_split_bits=-2), dict(skew_bcast=2),
-                                 dict(skew_bcast=-2)])
+                                 dict(skew_bcast=-2), dict(peer_timeout_ms=-1), dict(shuffle_overlap=2),
+                                 dict(shuffle_overlap=-2), dict(overlap_local_sms=-1)])
 def test_invalid_config_rejected_without_gpu(mgj, bad):
     kw = dict(r_capacity=1024, s_capacity=1024)
     kw.update(bad)
@@ -60,7 +61,7 @@ def test_invalid_config_rejected_without_gpu(mgj, bad):
 
 def test_reserved_must_be_zero(mgj):
     cfg = mgj.make_config(r_capacity=10, s_capacity=10)
-    cfg.reserved[3] = 1
+    cfg.reserved[0] = 1
     assert mgj.arena_bytes(cfg) == 0
 
 

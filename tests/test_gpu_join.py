@@ -963,3 +963,46 @@ def test_torchrun_parity_all_gpus(mgj):
     assert out.returncode == 0, out.stderr[-3000:]
     line = json.loads([l for l in out.stdout.splitlines() if l.startswith("{")][-1])
     assert line["ok"] and line["world"] == n and line["count"] == 1 << 20
+
+
+# ------------------------------------------------------------ §8(e): shuffle overlapped with the local pass
+@pytest.mark.parametrize("N,mat", [(1, True), (2, True), (4, False), (8, True)])
+def test_overlap_parity(mgj, N, mat):
+    """R's local pass on a second stream beside S's scatter (shuffle_overlap =
+    1; auto for N > 1), N virtual ranks: bit-exact vs the oracle."""
+    w = datagen.Workload("unique", 300007, 400009)
+    joins, res, _ = run_virtual(mgj, w, N, materialize=mat, shuffle_overlap=1, overlap_local_sms=37)
+    d = w.rank_inputs()
+    ref = oracle.join(d["r_keys"], d["r_pays"], d["s_keys"], d["s_pays"], materialize=mat)
+    for r in res:
+        assert r["status"] == 0
+        assert (r["match_count"], r["checksum"], r["pair_digest"]) == (ref["count"], ref["checksum"], ref["pair_digest"])
+    if mat:
+        trip = [j.materialized(r) for j, r in zip(joins, res)]
+        k, a, b = sort_trip(*(np.concatenate([t[i] for t in trip]) for i in range(3)))
+        np.testing.assert_array_equal(k, ref["key"])
+        np.testing.assert_array_equal(a, ref["pay_r"])
+        np.testing.assert_array_equal(b, ref["pay_s"])
+    for j in joins:
+        j.close()
+
+
+def test_overlap_timeline(mgj):
+    """The kernel timeline (trace=1) of one rank with the overlap on: R's local
+    pass runs while S is still being scattered, and S's local pass starts
+    only after S's scatter; without the overlap the two never coincide."""
+    n = 1 << 24
+    cols = [torch.empty(n, dtype=torch.int32, device="cuda") for _ in range(4)]
+    mgj.gen_relation("unique", 0, n, n, 0.0, 0, n, cols[0], cols[1])
+    mgj.gen_relation("unique", 1, n, n, 0.0, 0, n, cols[2], cols[3])
+    for ov in (1, -1):
+        j = mgj.Join(mgj.make_config(r_capacity=n, s_capacity=n, shuffle_overlap=ov, trace=True))
+        res = j.run(*cols)
+        assert res["match_count"] == n
+        t = j.trace()
+        if ov == 1:
+            assert t["local_R"][0] < t["scatter_S"][1] and t["scatter_S"][0] < t["local_R"][1], t
+            assert t["local_S"][0] >= t["scatter_S"][1], t
+        else:  # one launch over both relations after both scatters (not stamped)
+            assert "local_R" not in t and t["itemize"][0] >= t["scatter_S"][1], t
+        j.close()

@@ -1,6 +1,7 @@
 """Small joins for compute-sanitizer (memcheck / racecheck / synccheck): unique,
 duplicate-heavy, wide, and 2 virtual ranks."""
 import sys, os
+os.environ.setdefault("CUDA_DEVICE_MAX_CONNECTIONS", "32")  # virtual ranks wait for each other inside kernels
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import numpy as np
 import torch
@@ -18,7 +19,7 @@ def one(d, **kw):
     j = mgj.Join(mgj.make_config(key_bytes=kb, r_capacity=d["r_keys"].size, s_capacity=d["s_keys"].size,
                                  out_capacity=max(ref["count"], 1), **kw))
     r = j.run(*[dev(d[k]) for k in ("r_keys", "r_pays", "s_keys", "s_pays")])
-    assert (r["match_count"], r["checksum"]) == (ref["count"], ref["checksum"]), (r, ref)
+    assert (r["match_count"], r["checksum"], r["pair_digest"]) == (ref["count"], ref["checksum"], ref["pair_digest"]), (r, ref)
     j.close()
 
 
@@ -28,6 +29,12 @@ one({"r_keys": rng.integers(0, 300, 20000, dtype=np.uint64).astype(np.uint32), "
      "s_keys": rng.integers(0, 300, 30000, dtype=np.uint64).astype(np.uint32), "s_pays": np.arange(30000, dtype=np.uint32)},
     materialize=False, radix_bits_global=4)
 one(datagen.Workload("wide", 1 << 14, 1 << 14).rank_inputs(), materialize=True)
+# the bench's probe loop (count only, packed table: B1 + B2 = 16) on duplicate keys
+one({"r_keys": rng.integers(0, 1 << 14, 50000, dtype=np.uint64).astype(np.uint32), "r_pays": np.arange(50000, dtype=np.uint32),
+     "s_keys": rng.integers(0, 1 << 14, 70000, dtype=np.uint64).astype(np.uint32), "s_pays": np.arange(70000, dtype=np.uint32)},
+    materialize=False, radix_bits_global=10, radix_bits_local=6)
+# the overlapped shuffle (R's local pass on a second stream beside S's scatter) at one rank
+one(datagen.Workload("unique", 1 << 17, 1 << 17).rank_inputs(), materialize=True, shuffle_overlap=1, trace=True)
 
 
 def virtual(w, N, **kw):
@@ -40,18 +47,23 @@ def virtual(w, N, **kw):
     arenas = [torch.zeros(nb, dtype=torch.uint8, device="cuda") for _ in range(N)]
     js = [mgj.Join(cfgs[g], [a.data_ptr() for a in arenas], nb) for g in range(N)]
     ts = [[dev(p[k]) for k in ("r_keys", "r_pays", "s_keys", "s_pays")] for p in parts]
-    for g in range(N): js[g].partition(*ts[g])
-    for g in range(N): js[g].shuffle()
-    for g in range(N): js[g].join()
+    ss = [torch.cuda.Stream() for _ in range(N)]  # one per rank: a6 waits for every peer
+    torch.cuda.synchronize()
+    for g in range(N): js[g].partition(*ts[g], stream=ss[g])
+    for g in range(N): js[g].shuffle(ss[g])
+    for g in range(N): js[g].join(ss[g])
     res = [js[g].result() for g in range(N)]
     full = w.rank_inputs()
     ref = oracle.join(full["r_keys"], full["r_pays"], full["s_keys"], full["s_pays"])
-    assert (res[0]["match_count"], res[0]["checksum"]) == (ref["count"], ref["checksum"])
+    assert (res[0]["match_count"], res[0]["checksum"], res[0]["pair_digest"]) == \
+        (ref["count"], ref["checksum"], ref["pair_digest"])
     for j in js: j.close()
 
 
-# two virtual ranks; four with selectively broadcast partitions (NEXT-2), also through the first local pass
-virtual(datagen.Workload("unique", 1 << 15, 1 << 15), 2)
-virtual(datagen.Workload("zipf", 1 << 13, 1 << 15, 1.0), 4, skew_bcast=1, radix_bits_global=6)
-virtual(datagen.Workload("zipf", 1 << 13, 1 << 15, 1.0), 4, skew_bcast=1, radix_bits_global=6, local_split_bits=2)
+# two virtual ranks (with the overlapped shuffle); four with selectively broadcast partitions (NEXT-2),
+# also through the first local pass
+if os.environ.get("MGJ_SAN_VIRTUAL", "1") == "1":
+    virtual(datagen.Workload("unique", 1 << 15, 1 << 15), 2)
+    virtual(datagen.Workload("zipf", 1 << 13, 1 << 15, 1.0), 4, skew_bcast=1, radix_bits_global=6)
+    virtual(datagen.Workload("zipf", 1 << 13, 1 << 15, 1.0), 4, skew_bcast=1, radix_bits_global=6, local_split_bits=2)
 print("sanitize workload ok")

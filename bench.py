@@ -407,9 +407,10 @@ def main():
             "peak_source": peak_src,
             "alg_bytes_per_launch": phase_report[dom]["alg_bytes"]}
     if kern[dom] == "k_scatter":
-        # measured: with its stores redirected into L2 the scatter runs at the same
-        # speed, so below the HBM roofline it is limited by the SM's shared-memory pipe
-        roof["limiter"] = "shared-memory pipe (ranking atomics, random 8-byte stores), not DRAM"
+        # measured (profiles/r2): the scatter keeps the SM's L1 data pipe ~80% busy
+        # (shared ranking atomics and random 8-byte stores, the write-out's loads and global stores);
+        # its time scales with the SM count, not with HBM
+        roof["limiter"] = "per-SM L1 data pipe (~80% busy: ranking atomics, random shared stores, write-out), not DRAM"
 
     sm_mhz = (clocks or {}).get("sm_mhz") or float(peaks.get("sm_max_mhz", 1965.0))
     nsm = torch.cuda.get_device_properties(dev).multi_processor_count

@@ -32,13 +32,19 @@ __host__ __device__ constexpr ScatGeom scat_geom(int P, int key_bytes) {
                                                                       : ScatGeom{4096, 1, 4, 1024});
 }
 
-// Per-partition write-out descriptor of the current sub-tile (16 bytes, one
-// shared load per sector group).
-struct __align__(16) PInfo {
-    unsigned long long wb;  // destination address of sorted slot 0 (wb + slot * TB)
-    uint32_t lim;           // end of the partition's valid slots in `sorted`
-    uint32_t head;          // (slot << 2 | h) of a head group whose first h slots are not ours, else ~0
+// Per-partition write-out descriptor of the current sub-tile (8 bytes, one
+// shared load per sector group): the destination tuple index of sorted slot
+// 0 in the owner's receive buffer (modulo 2^32: slot s goes to didx + s), the
+// end of the partition's valid slots, and the head group, if any, whose first
+// h slots are not the partition's ((slot / SG) << 2 | h; 0xffff: none).  The
+// owner's receive buffer comes from two small per-kernel tables (destination
+// rank of each partition, base of each rank's receive buffer).
+struct __align__(8) PInfo {
+    uint32_t didx;
+    uint16_t lim;
+    uint16_t head;
 };
+constexpr uint16_t PI_NONE = 0xffff;
 
 __host__ __device__ inline size_t scat_smem_bytes(int P, int key_bytes) {
     const ScatGeom g = scat_geom(P, key_bytes);
@@ -46,7 +52,9 @@ __host__ __device__ inline size_t scat_smem_bytes(int P, int key_bytes) {
     return (size_t)g.T * key_bytes                             // input stage: keys (payloads: L2 prefetch + loads)
            + ((size_t)g.T + 2 * (size_t)(g.SG - 1) * P) * TB  // partition-sorted sub-tile (+ carries, group padding)
            + (size_t)P * sizeof(PInfo)                         // write-out descriptors
-           + (size_t)P * 4;                                    // next free slot per partition
+           + (size_t)P * 4                                     // next free slot per partition
+           + 2 * (size_t)MAX_RANKS * 8                         // receive-buffer base per (relation, rank)
+           + 2 * (size_t)P;                                    // destination rank per (relation, partition)
 }
 
 // Block-wide exclusive scan of one register value per thread (<= 1024 threads).
@@ -176,7 +184,6 @@ __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c, int rel0, int rel1) {
     static_assert(NU * LU == V && NU >= 1, "sub-tile");
     constexpr int GB = SG * TB;                // group bytes
     constexpr int CW = SG > 1 ? SG - 1 : 1;    // carry capacity (tuples)
-    constexpr uint32_t NONE = 0xffffffffu;
     using GV = typename Vec<GB>::T;
     typedef unsigned long long ull;
     // `sorted` swizzle: the two 16-byte halves of every 32-byte group whose
@@ -186,14 +193,14 @@ __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c, int rel0, int rel1) {
         if constexpr (SG > 1 && SG * sizeof(Tup) == 32) return s ^ (((s >> (SG == 4 ? 4 : 3)) & 1u) * (SG / 2));
         else return s;
     };
-    // 8-byte keys: the whole descriptor is loaded with one 16-byte access
-    constexpr bool EAGER = sizeof(K) == 8;
     extern __shared__ __align__(128) unsigned char smem[];
     const int P = c.P;
     K *const skey = reinterpret_cast<K *>(smem);  // stage: the sub-tile's keys
     Tup *const sorted = reinterpret_cast<Tup *>(smem + T * sizeof(K));
-    PInfo *const pinfo = reinterpret_cast<PInfo *>(sorted + T + 2 * (SG - 1) * P);  // 16-byte aligned
+    PInfo *const pinfo = reinterpret_cast<PInfo *>(sorted + T + 2 * (SG - 1) * P);  // 8-byte aligned
     uint32_t *const off = reinterpret_cast<uint32_t *>(pinfo + P);  // next free slot per partition
+    unsigned long long *const obase = reinterpret_cast<unsigned long long *>(off + P);  // [2][MAX_RANKS]
+    uint8_t *const own8 = reinterpret_cast<uint8_t *>(obase + 2 * MAX_RANKS);            // [2][P]
     const uint32_t sorted_s = smem_u32(sorted), pinfo_s = smem_u32(pinfo);
     auto saddr = [&](uint32_t x) -> uint32_t { return sorted_s + swz(x) * (uint32_t)TB; };
     auto sput = [&](uint32_t x, const Tup &t) { sts_at(saddr(x), t); };
@@ -247,13 +254,22 @@ __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c, int rel0, int rel1) {
     };
 
     // per owned partition (registers): destination of the next group, carry
-    ull base[PPT];
+    uint32_t bidx[PPT];  // destination tuple index of the next group (owner's receive buffer, mod 2^32)
+    uint8_t dstr[PPT];   // destination rank
     uint32_t cc[PPT], hd[PPT], lim[PPT];
     bool skp[PPT];  // partition skipped by the plan (an empty side): nothing is stored
     Tup carry[PPT][CW];
     bool pending = false;  // carries of the last sub-tile still sit in `sorted`
 #pragma unroll
-    for (int k = 0; k < PPT; ++k) base[k] = 0, cc[k] = 0, hd[k] = 0, lim[k] = 0, skp[k] = false;
+    for (int k = 0; k < PPT; ++k) bidx[k] = 0, dstr[k] = 0, cc[k] = 0, hd[k] = 0, lim[k] = 0, skp[k] = false;
+    // per-kernel tables for the write-out: receive-buffer base of every (relation, rank) and the
+    // destination rank of every (relation, partition) (read after the first layout barrier)
+    if (tid < 2 * MAX_RANKS)
+        obase[tid] = (tid % MAX_RANKS) < c.world ? (ull)(c.arena[tid % MAX_RANKS] + c.lay.recv[tid / MAX_RANKS]) : 0ull;
+    for (int p = tid; p < P; p += NT) {
+        own8[p] = (uint8_t)c.owner[p];
+        own8[P + p] = (uint8_t)(c.bcast[p] ? c.rank : c.owner[p]);  // S of a broadcast partition stays here
+    }
 
     auto issue = [&](const Cur &u) {  // thread 0: TMA the 16-byte-aligned body of sub-tile u's keys
         uint64_t first;
@@ -282,13 +298,16 @@ __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c, int rel0, int rel1) {
             pending = false;
         }
     };
-    auto flush = [&]() {  // end of a tile: store the remaining tails tuple by tuple
+    auto flush = [&](int rel) {  // end of a tile: store the remaining tails tuple by tuple
         fetch_carry();
 #pragma unroll
         for (int k = 0; k < PPT; ++k)
 #pragma unroll
             for (int i = 0; i < CW; ++i)
-                if (!skp[k] && i >= (int)hd[k] && i < (int)cc[k]) reinterpret_cast<Tup *>(base[k])[i] = carry[k][i];
+                if (!skp[k] && i >= (int)hd[k] && i < (int)cc[k]) {
+                    Tup *d = reinterpret_cast<Tup *>(c.arena[dstr[k]] + c.lay.recv[rel]);
+                    d[(uint32_t)(bidx[k] + i)] = carry[k][i];
+                }
     };
     auto set_base = [&](int rel, int tile) {  // destination of this tile's first tuple of each owned partition
         const uint32_t *tb = c.tile_base + ((size_t)rel * c.G + tile) * P;
@@ -302,9 +321,11 @@ __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c, int rel0, int rel1) {
                 // selectively broadcast partition (a2, NEXT-2)
                 const int dst = (rel && c.bcast[p]) ? c.rank : c.owner[p];
                 skp[k] = c.pskip[p] != 0;
-                const ull a = (ull)(c.arena[dst] + c.lay.recv[rel]) + (so[p] + tb[p]) * (uint64_t)TB;
+                const uint64_t idx = so[p] + tb[p];
+                const ull a = (ull)(c.arena[dst] + c.lay.recv[rel]) + idx * (uint64_t)TB;
                 const uint32_t h = SG > 1 ? (uint32_t)((a & (GB - 1)) / TB) : 0u;
-                base[k] = a - (ull)h * TB;
+                bidx[k] = (uint32_t)idx - h;  // may wrap below 0: placeholders are never stored
+                dstr[k] = (uint8_t)dst;
                 cc[k] = hd[k] = h;
 #pragma unroll
                 for (int i = 0; i < CW; ++i) {  // placeholders: digit1 = p, never stored
@@ -374,7 +395,7 @@ __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c, int rel0, int rel1) {
         span(u, first, len);
         const Cur nx = next_cur(u);
         if (u.rel * c.G + u.tile != cur_tile) {  // thread-private partition state: no barrier needed
-            if (cur_tile >= 0) flush();
+            if (cur_tile >= 0) flush(cur_tile / c.G);
             set_base(u.rel, u.tile);
             cur_tile = u.rel * c.G + u.tile;
         }
@@ -400,11 +421,11 @@ __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c, int rel0, int rel1) {
                 off[p] = o + cc[k];
                 const uint32_t full = cnt[k] & ~(uint32_t)(SG - 1);
                 PInfo in;
-                in.wb = base[k] - (ull)o * TB;
-                in.lim = skp[k] ? o : o + cnt[k];  // a skipped partition's groups are never stored
-                in.head = (hd[k] && full) ? (o << 2 | hd[k]) : NONE;
+                in.didx = bidx[k] - o;
+                in.lim = (uint16_t)(skp[k] ? o : o + cnt[k]);  // a skipped partition's groups are never stored
+                in.head = (hd[k] && full) ? (uint16_t)((o / SG) << 2 | hd[k]) : PI_NONE;
                 pinfo[p] = in;
-                base[k] += (ull)full * TB;
+                bidx[k] += full;
                 if (full) hd[k] = 0;
                 cc[k] = cnt[k] - full;
                 lim[k] = o + cnt[k];
@@ -448,12 +469,12 @@ __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c, int rel0, int rel1) {
         if (nx.rel <= rel1) load_pay(nx);  // the ranking of this sub-tile has consumed pp
         // write-out: one group per thread per step, rotated by rank share for N > 1
         const uint32_t ngroups = total / SG;
+        const ull ob_rel = (ull)(c.arena[0] + c.lay.recv[u.rel]);  // N = 1: the one receive buffer
         const uint32_t rot = (uint32_t)(((uint64_t)ngroups * rot_num) / (uint32_t)c.world);
         for (uint32_t w = tid; w < ngroups; w += NT) {
             const uint32_t gi = w + rot < ngroups ? w + rot : w + rot - ngroups;
             const uint32_t slot = gi * SG;
             GV gv;
-            PInfo in;
             if constexpr (GB == 32) {  // two conflict-free 16-byte halves (swizzled)
                 gv.a = lds128_at(saddr(slot));
                 gv.b = lds128_at(saddr(slot + SG / 2));
@@ -462,30 +483,21 @@ __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c, int rel0, int rel1) {
             } else {
                 gv = lds64_at(saddr(slot));
             }
-            const uint32_t pa = pinfo_s + (reinterpret_cast<const uint32_t *>(&gv)[0] & (uint32_t)(P - 1)) * 16u;
-            if constexpr (EAGER) {
-                const uint4 v = lds128_at(pa);
-                in.wb = (ull)v.x | ((ull)v.y << 32);
-                in.lim = v.z;
-                in.head = v.w;
-            } else {
-                const uint2 lh = lds64_at(pa + 8);
-                in.lim = lh.x;
-                in.head = lh.y;
-                const uint2 wv = lds64_at(pa);
-                in.wb = (ull)wv.x | ((ull)wv.y << 32);
-            }
-            if (slot + SG <= in.lim) {
-                char *dst = reinterpret_cast<char *>(in.wb + (ull)slot * TB);
-                if ((in.head >> 2) != slot) {
+            const uint32_t pidx = reinterpret_cast<const uint32_t *>(&gv)[0] & (uint32_t)(P - 1);
+            const uint2 pv = lds64_at(pinfo_s + pidx * 8u);
+            const uint32_t plim = pv.y & 0xffffu, phead = pv.y >> 16;
+            if (slot + SG <= plim) {
+                const ull ob = c.world == 1 ? ob_rel : obase[u.rel * MAX_RANKS + own8[u.rel * P + pidx]];
+                char *dst = reinterpret_cast<char *>(ob + (ull)(uint32_t)(pv.x + slot) * TB);
+                if (phead == PI_NONE || (phead >> 2) * SG != slot) {
                     st_group<GB>(dst, gv);
                 } else {
-                    for (uint32_t i = in.head & 3u; i < SG; ++i) reinterpret_cast<Tup *>(dst)[i] = sget(slot + i);
+                    for (uint32_t i = phead & 3u; i < SG; ++i) reinterpret_cast<Tup *>(dst)[i] = sget(slot + i);
                 }
             }
         }
     }
-    if (cur_tile >= 0) flush();
+    if (cur_tile >= 0) flush(cur_tile / c.G);
 
     // ---- every CTA: make its (peer) stores visible, the last one signals ----
     __threadfence_system();

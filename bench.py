@@ -57,6 +57,8 @@ def parse():
                     help="§8(e): R's local pass beside S's scatter (auto: on for N > 1 with the P2P shuffle)")
     ap.add_argument("--overlap-local-sms", type=int, default=0)
     ap.add_argument("--trace", action="store_true", help="kernel timeline of the last step in the JSON line")
+    ap.add_argument("--compress", action="store_true",
+                    help="NEXT-1 compressed shuffle (4-byte keys, id payloads): 32-byte units of five entries")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=3)
@@ -300,7 +302,7 @@ def main():
                           shuffle_mode=(mgj.SHUFFLE_EXTERNAL if a.shuffle == "nccl" else mgj.SHUFFLE_P2P),
                           skew_bcast=a.skew_bcast, num_sms=a.num_sms,
                           shuffle_overlap={"auto": 0, "on": 1, "off": -1}[a.overlap],
-                          overlap_local_sms=a.overlap_local_sms, trace=a.trace)
+                          overlap_local_sms=a.overlap_local_sms, trace=a.trace, compress=a.compress)
     # N>1 (or MGJ_SYMM_ARENA=1): the library's symmetric-memory setup (mgj.symmetric_join)
     join = mgj.symmetric_join(cfg) if distributed else mgj.Join(cfg)
 
@@ -395,6 +397,15 @@ def main():
             d.update(alg_bytes=int(alg[nm]), gbs=gbs, frac_hbm=gbs / hbm_peak)
         phase_report[nm] = d
     kern = {"shuffle": "k_scatter", "local_part": "k_local", "probe": "k_probe", "hist": "k_hist"}
+    if a.compress:  # the receive sizes count 32-byte units: the scatter writes, the local pass reads units
+        recv_t = n_local  # received tuples, taken as this rank's share (exact at N = 1)
+        alg.update(shuffle=tb * n_local + 32 * recv, local_part=32 * recv + tb * recv_t,
+                   probe=tb * recv_t + (3 * kb * res["local_count"] if a.materialize else 0))
+        for nm in ("shuffle", "local_part", "probe"):
+            i = names.index(nm)
+            if ph[i] > 0:
+                gbs = alg[nm] / (ph[i] / 1000.0) / 1e9
+                phase_report[nm].update(alg_bytes=int(alg[nm]), gbs=gbs, frac_hbm=gbs / hbm_peak)
     dom = max(alg, key=lambda k: phase_report[k]["ms"])
     traffic = None
     try:
@@ -415,8 +426,13 @@ def main():
     sm_mhz = (clocks or {}).get("sm_mhz") or float(peaks.get("sm_max_mhz", 1965.0))
     nsm = torch.cuda.get_device_properties(dev).multi_processor_count
     cyc = (ms_per_step / 1000.0) * sm_mhz * 1e6 * world / tuples_job
-    # shuffle bytes over NVLink per GPU (egress) and its rate
-    nvl_bytes = tb * n_local * (world - 1) / world
+    # shuffle bytes: the wire format (8-byte tuples, or 32-byte units of up to five compressed
+    # tuples), from the receive sizes; over NVLink per GPU (egress) the (N-1)/N share
+    wire = torch.tensor([float((res["recv_r"] + res["recv_s"]) * (32 if a.compress else tb))], device=dev)
+    if world > 1:
+        dist.all_reduce(wire)
+    wire_per_tuple = float(wire.item()) / tuples_job
+    nvl_bytes = wire_per_tuple * n_local * (world - 1) / world
     shuffle_ms = phase_report["shuffle"]["ms"]
 
     # end-to-end: host (pinned) inputs through the C ABI, H2D inside the timed region
@@ -473,7 +489,8 @@ def main():
                                      "sm_mhz": sm_mhz, "sms": nsm,
                                      "formula": "T*f_SM*SMs*N/(|R|+|S|) and T*f_SM*N/(|R|+|S|)"},
             "phases": phase_report,
-            "shuffle": {"nvlink_egress_bytes_per_gpu": nvl_bytes,
+            "shuffle": {"wire_bytes_per_tuple": wire_per_tuple, "compress": a.compress,
+                        "nvlink_egress_bytes_per_gpu": nvl_bytes,
                         "nvlink_gbs_per_gpu": (nvl_bytes / (shuffle_ms / 1000) / 1e9) if world > 1 else None,
                         "nvlink_peak_gbs": 900.0, "measured_peer_gbs": 770.0},
             "step_ms": {"median": statistics.median(step_ms), "min": min(step_ms), "max": max(step_ms)},

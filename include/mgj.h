@@ -89,7 +89,15 @@ typedef struct {
     int32_t  overlap_local_sms;        /* SMs of R's local pass during the overlap (0 = half the SMs) */
     int32_t  trace;                    /* 1: record the first start and last end (globaltimer, ns) of
                                           every kernel of the run (mgj_debug_copy MGJ_DBG_TRACE) */
-    int32_t  reserved[1];              /* must be zero */
+    int32_t  compress;                 /* NEXT-1: 1 = compress the shuffle.  Needs 4-byte keys,
+                                          MGJ_SHUFFLE_P2P and payloads that are global row ids (rank g's
+                                          row i has payload sum_{g'<g} n_g' + i, the paper's id column;
+                                          checked per tuple, a run that breaks it fails with MGJ_EINVAL).
+                                          A tuple travels as its key without the B1 partition bits plus
+                                          its row's offset in its source tile, five per 32-byte unit
+                                          (+ source rank, tile, count): 6.4 instead of 8 bytes.  Forces a
+                                          single local pass */
+    int32_t  reserved[2];              /* must be zero */
 } mgj_config;
 
 /*

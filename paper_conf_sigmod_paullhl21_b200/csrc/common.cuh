@@ -36,10 +36,16 @@ __host__ __device__ constexpr int local2_vcap(int P) { return 4 * P > 4096 ? 4 *
 constexpr uint64_t WAIT_TIMEOUT_NS = 20ull * 1000 * 1000 * 1000;  // default peer-signal wait bound
 
 constexpr int RES_W = 8;  // u64 words per rank in the result mailbox (a6)
+// NEXT-1 compressed shuffle: a 32-byte unit carries CU_N tuples as 44-bit
+// entries (key >> B1 in the low 32 - B1 bits, the row's offset in its source
+// tile above), plus (count, source rank, tile) in its top word
+constexpr int CU_N = 5;
+constexpr int CU_ENTRY_BITS = 44;
+constexpr int CHUNK_UNITS = 2048;  // local-pass chunk with the compressed shuffle: 2 units per thread
 // peer flags: histograms published (a1), R / S tuples all stored (a3), partial sums published (a6)
 enum Sig { SIG_HIST = 0, SIG_DATA_R = 1, SIG_RES = 2, SIG_DATA_S = 3, SIG_COUNT = 4 };
 enum Ticket { TK_HIST = 0, TK_SCAT_R = 1, TK_SCAT_S = 2, TK_SCAT_DONE = 3, TK_ITEMS = 4,
-              TK_PROBE = 5, TK_LOCAL = 6, TK_COUNT = 8 };
+              TK_PROBE = 5, TK_LOCAL = 6, TK_TSCAN = 7, TK_COUNT = 8 };
 enum Meta { MT_PLO = 0, MT_PHI = 1, MT_B2 = 2, MT_OK = 3, MT_NCH_R = 4, MT_NCH_S = 5,
             MT_NITEMS = 6, MT_CHUNK = 7,
             MT_BA = 8,       // bits of the first local pass (0: single local pass)
@@ -64,6 +70,7 @@ struct Arena {
     uint64_t mail;     // u32 hist[MAX_RANKS][2][P]
     uint64_t resmail;  // u64 res[MAX_RANKS][RES_W] (count, checksum, n_out, status, pair digest)
     uint64_t cfgmail;  // u64 cfg[MAX_RANKS][4] (recv_cap R, recv_cap S, arena bytes, B1) published with a1
+    uint64_t umail;    // u32 units[MAX_RANKS][2][P] (compress: 32-byte units per partition) published with a1
     uint64_t recv[2];  // received tuples of R, S
     uint64_t total;
 };
@@ -95,10 +102,15 @@ struct Ctx {
     int32_t probe_target;         // co-partition size B2 aims at (tuples)
     int32_t materialize;
     int32_t ext;                  // shuffle mode EXTERNAL: scatter into send_buf, caller exchanges
+    int32_t comp;                 // NEXT-1 compressed shuffle (units of CU_N entries, see scatter.cuh)
+    int32_t chunk_units;          // compress: local-pass chunk in units
+    uint32_t *rowbase;            // compress: [2][MAX_RANKS][G] global row id of each (rank, tile)'s first row
+    uint32_t *rank_units;         // compress: [2][P] this rank's 32-byte units per partition
     uint32_t max_items;
     uint64_t epoch;
     uint64_t timeout_ns;          // bound on a wait for peer signals (mgj_config.peer_timeout_ms)
     uint64_t recv_cap[2];
+    uint64_t recv_cap_u[2];       // compressed shuffle: receive capacity in 32-byte units
     uint64_t max_chunks;
     uint64_t out_cap;
     uint64_t mid_cap;             // slots of each first-pass output buffer
@@ -257,6 +269,27 @@ __device__ __forceinline__ unsigned long long dig_term(T a, T b) {
         return (unsigned long long)(uint32_t)a * (uint32_t)b;
     } else {
         return (unsigned long long)a * (unsigned long long)b;
+    }
+}
+
+// NEXT-1 unit (256 bits as four u64 words): entries e0..e4 of 44 bits at bit
+// 44*i, then the unit's meta word (valid count | source rank << 3 | tile << 6)
+// in bits 224..255.
+__device__ __forceinline__ void unit_pack(const unsigned long long (&e)[CU_N], uint32_t meta,
+                                          unsigned long long (&a)[4]) {
+    a[0] = e[0] | (e[1] << 44);
+    a[1] = (e[1] >> 20) | (e[2] << 24);
+    a[2] = (e[2] >> 40) | (e[3] << 4) | (e[4] << 48);
+    a[3] = (e[4] >> 16) | ((unsigned long long)meta << 32);
+}
+__device__ __forceinline__ unsigned long long unit_entry(const unsigned long long (&a)[4], int i) {
+    constexpr unsigned long long M44 = (1ull << CU_ENTRY_BITS) - 1;
+    switch (i) {
+        case 0: return a[0] & M44;
+        case 1: return (a[0] >> 44) | ((a[1] & ((1ull << 24) - 1)) << 20);
+        case 2: return (a[1] >> 24) | ((a[2] & 0xFull) << 40);
+        case 3: return (a[2] >> 4) & M44;
+        default: return (a[2] >> 48) | ((a[3] & ((1ull << 28) - 1)) << 16);
     }
 }
 

@@ -32,6 +32,29 @@ __host__ __device__ inline int hist_nb(int T, int key_bytes) {
 // stores the rank histogram into every peer's arena mailbox and raises
 // SIG_HIST there (histogram exchange X4 fused).
 // ---------------------------------------------------------------------------
+// The fused exchange of a1 (one CTA): the rank histogram (and, compressed,
+// the unit counts) and the job-wide configuration words into every peer's
+// mailbox, then SIG_HIST everywhere.
+__device__ inline void publish_hist(const Ctx &c) {
+    const int P = c.P;
+    for (int d = 0; d < c.world; ++d) {
+        uint32_t *mb = reinterpret_cast<uint32_t *>(c.arena[d] + c.lay.mail) + (size_t)c.rank * 2 * P;
+        for (int j = threadIdx.x; j < 2 * P; j += blockDim.x) mb[j] = __ldcg(&c.rank_hist[j]);
+        if (c.comp) {
+            uint32_t *ub = reinterpret_cast<uint32_t *>(c.arena[d] + c.lay.umail) + (size_t)c.rank * 2 * P;
+            for (int j = threadIdx.x; j < 2 * P; j += blockDim.x) ub[j] = __ldcg(&c.rank_units[j]);
+        }
+        // this rank's job-wide configuration words, checked equal on every rank by k_plan
+        if (threadIdx.x < 4) {
+            const uint64_t w[4] = {c.recv_cap[0], c.recv_cap[1], c.lay.total, (uint64_t)(c.B1 | c.comp << 8)};
+            reinterpret_cast<uint64_t *>(c.arena[d] + c.lay.cfgmail)[c.rank * 4 + threadIdx.x] = w[threadIdx.x];
+        }
+    }
+    __threadfence_system();
+    __syncthreads();
+    if (threadIdx.x == 0) signal_all(c, SIG_HIST);
+}
+
 template <typename K>
 __global__ void __launch_bounds__(HIST_THREADS, 2) k_hist(Ctx c) {
     extern __shared__ __align__(128) unsigned char hsm[];  // ring[HIST_NB][T] keys | sub[P] | acc[P]
@@ -171,51 +194,55 @@ __global__ void __launch_bounds__(HIST_THREADS, 2) k_hist(Ctx c) {
     __shared__ int last;
     if (threadIdx.x == 0) last = (atomicAdd(&c.ticket[TK_HIST], 1u) == gridDim.x * gridDim.y - 1);
     __syncthreads();
-    if (!last) return;
+    if (!last || c.comp) return;  // compressed shuffle: k_tilescan publishes, with the unit counts
     __threadfence();
-    for (int d = 0; d < c.world; ++d) {
-        uint32_t *mb = reinterpret_cast<uint32_t *>(c.arena[d] + c.lay.mail) + (size_t)c.rank * 2 * P;
-        for (int j = threadIdx.x; j < 2 * P; j += blockDim.x) mb[j] = __ldcg(&c.rank_hist[j]);
-        // this rank's job-wide configuration words, checked equal on every rank by k_plan
-        if (threadIdx.x < 4) {
-            const uint64_t w[4] = {c.recv_cap[0], c.recv_cap[1], c.lay.total, (uint64_t)c.B1};
-            reinterpret_cast<uint64_t *>(c.arena[d] + c.lay.cfgmail)[c.rank * 4 + threadIdx.x] = w[threadIdx.x];
-        }
-    }
-    __threadfence_system();
-    __syncthreads();
-    if (threadIdx.x == 0) signal_all(c, SIG_HIST);
+    publish_hist(c);
 }
 
 // Exclusive prefix of the per-tile histograms over tiles: tile c's tuples of
 // partition p start at send_off[p] + tile_base[rel][c][p] in the owner's
 // receive range (deterministic placement; one thread per (rel, p)).
+// With the compressed shuffle (NEXT-1) a tile's run of partition p is
+// ceil(count / CU_N) 32-byte units, and tile_base counts units; the last block
+// then publishes the histograms with the rank's unit totals (publish_hist).
 __global__ void k_tilescan(Ctx c) {
     const int idx = blockIdx.x * blockDim.x + threadIdx.x;
-    if (idx >= 2 * c.P) return;
-    const int rel = idx / c.P, p = idx % c.P;
-    const size_t stride = c.P;
-    const uint32_t *src = c.tile_hist + (size_t)rel * c.G * c.P + p;
-    uint32_t *dst = c.tile_base + (size_t)rel * c.G * c.P + p;
-    uint32_t run = 0;
-    int t = 0;
-    for (; t + 4 <= c.G; t += 4) {
-        const uint32_t v0 = src[(t + 0) * stride], v1 = src[(t + 1) * stride];
-        const uint32_t v2 = src[(t + 2) * stride], v3 = src[(t + 3) * stride];
-        dst[(t + 0) * stride] = run;
-        run += v0;
-        dst[(t + 1) * stride] = run;
-        run += v1;
-        dst[(t + 2) * stride] = run;
-        run += v2;
-        dst[(t + 3) * stride] = run;
-        run += v3;
+    if (idx < 2 * c.P) {
+        const int rel = idx / c.P, p = idx % c.P;
+        const size_t stride = c.P;
+        const uint32_t *src = c.tile_hist + (size_t)rel * c.G * c.P + p;
+        uint32_t *dst = c.tile_base + (size_t)rel * c.G * c.P + p;
+        auto val = [&](uint32_t v) { return c.comp ? (v + CU_N - 1) / CU_N : v; };
+        uint32_t run = 0;
+        int t = 0;
+        for (; t + 4 <= c.G; t += 4) {
+            const uint32_t v0 = src[(t + 0) * stride], v1 = src[(t + 1) * stride];
+            const uint32_t v2 = src[(t + 2) * stride], v3 = src[(t + 3) * stride];
+            dst[(t + 0) * stride] = run;
+            run += val(v0);
+            dst[(t + 1) * stride] = run;
+            run += val(v1);
+            dst[(t + 2) * stride] = run;
+            run += val(v2);
+            dst[(t + 3) * stride] = run;
+            run += val(v3);
+        }
+        for (; t < c.G; ++t) {
+            const uint32_t v = src[t * stride];
+            dst[t * stride] = run;
+            run += val(v);
+        }
+        if (c.comp) c.rank_units[idx] = run;
     }
-    for (; t < c.G; ++t) {
-        const uint32_t v = src[t * stride];
-        dst[t * stride] = run;
-        run += v;
-    }
+    if (!c.comp) return;
+    __shared__ int last;
+    __threadfence();
+    __syncthreads();
+    if (threadIdx.x == 0) last = atomicAdd(&c.ticket[TK_TSCAN], 1u) == gridDim.x - 1;
+    __syncthreads();
+    if (!last) return;
+    __threadfence();
+    publish_hist(c);
 }
 
 // ---------------------------------------------------------------------------
@@ -303,6 +330,8 @@ __global__ void __launch_bounds__(1024) k_plan(Ctx c) {
     int32_t *own = reinterpret_cast<int32_t *>(sp + 5 * P);
     uint32_t *chn = reinterpret_cast<uint32_t *>(own + P);  // [P+1] scratch scans (u32)
     uint8_t *bcf = reinterpret_cast<uint8_t *>(chn + P + 1);  // [P] broadcast flags
+    // compressed shuffle: the receive layout counts 32-byte units, ownership still tuples
+    uint64_t *ut0 = reinterpret_cast<uint64_t *>((reinterpret_cast<uintptr_t>(bcf + P) + 7) & ~(uintptr_t)7), *ut1 = ut0 + P;
     __shared__ uint64_t tmp[33];
     __shared__ uint32_t tmp32[33];
     __shared__ int first[MAX_RANKS], endp[MAX_RANKS];
@@ -324,7 +353,7 @@ __global__ void __launch_bounds__(1024) k_plan(Ctx c) {
         // must have planned with the same ones, else peers store at offsets
         // that differ from the receiver's layout
         const uint64_t *cf = reinterpret_cast<const uint64_t *>(c.arena[c.rank] + c.lay.cfgmail);
-        const uint64_t w[4] = {c.recv_cap[0], c.recv_cap[1], c.lay.total, (uint64_t)c.B1};
+        const uint64_t w[4] = {c.recv_cap[0], c.recv_cap[1], c.lay.total, (uint64_t)(c.B1 | c.comp << 8)};
         for (int g = 0; g < N && ok; ++g)
             for (int i = 0; i < 4; ++i)
                 if (__ldcg(cf + g * 4 + i) != w[i]) {
@@ -340,16 +369,27 @@ __global__ void __launch_bounds__(1024) k_plan(Ctx c) {
     }
     const uint32_t *mail = reinterpret_cast<const uint32_t *>(c.arena[c.rank] + c.lay.mail);
     auto H = [&](int g, int rel, int p) -> uint32_t { return __ldcg(mail + (size_t)(g * 2 + rel) * P + p); };
+    const uint32_t *umail = reinterpret_cast<const uint32_t *>(c.arena[c.rank] + c.lay.umail);
+    // layout counts: tuples, or 32-byte units with the compressed shuffle
+    auto HL = [&](int g, int rel, int p) -> uint32_t {
+        return c.comp ? __ldcg(umail + (size_t)(g * 2 + rel) * P + p) : H(g, rel, p);
+    };
+    auto LT = [&](int rel, int p) -> uint64_t { return c.comp ? (rel ? ut1[p] : ut0[p]) : (rel ? tot1[p] : tot0[p]); };
     {
         unsigned long long st = 0;
         for (int p = tid; p < P; p += blockDim.x) {
-            uint64_t t0 = 0, t1 = 0;
+            uint64_t t0 = 0, t1 = 0, u0 = 0, u1 = 0;
             for (int g = 0; g < N; ++g) t0 += H(g, 0, p), t1 += H(g, 1, p);
+            if (c.comp)
+                for (int g = 0; g < N; ++g) u0 += HL(g, 0, p), u1 += HL(g, 1, p);
             const bool sk = !c.ext && skip_of(t0, t1);
             c.pskip[p] = sk;
-            if (sk) t0 = t1 = 0;  // a skipped partition is absent from every layout
-            tot0[p] = pre0[p] = t0;
+            if (sk) t0 = t1 = u0 = u1 = 0;  // a skipped partition is absent from every layout
+            tot0[p] = t0;
+            pre0[p] = c.comp ? u0 : t0;
             tot1[p] = t1;
+            ut0[p] = u0;
+            ut1[p] = u1;
             st += t1;
         }
         st = warp_sum(st);
@@ -361,12 +401,12 @@ __global__ void __launch_bounds__(1024) k_plan(Ctx c) {
         const bool bc = bcast_of(tot0[p], tot1[p], stot, N, P, bcfg);
         bcf[p] = bc;
         c.bcast[p] = bc;
-        pre1[p] = bc ? 0 : tot1[p];  // S layout: broadcast partitions are not in the owner's range part
+        pre1[p] = bc ? 0 : LT(1, p);  // S layout: broadcast partitions are not in the owner's range part
         cum[p] = owner_weight(tot0[p], tot1[p], bc, N);
-        chn[p] = bc ? H(c.rank, 1, p) : 0u;  // this rank's own S of broadcast partitions (never skipped)
+        chn[p] = bc ? HL(c.rank, 1, p) : 0u;  // this rank's own S of broadcast partitions (never skipped)
         if (bc) {
             atomicAdd(&nbc, 1);
-            for (int d = 0; d < N; ++d) atomicAdd(&bcs[d], (unsigned long long)H(d, 1, p));
+            for (int d = 0; d < N; ++d) atomicAdd(&bcs[d], (unsigned long long)HL(d, 1, p));
         }
     }
     __syncthreads();
@@ -386,11 +426,11 @@ __global__ void __launch_bounds__(1024) k_plan(Ctx c) {
     }
     __syncthreads();
     // S tuples of this rank's own range part (non-broadcast), where its broadcast part starts
-    const uint64_t s_range_me = first[c.rank] < P ? pre1[endp[c.rank] - 1] + (bcf[endp[c.rank] - 1] ? 0 : tot1[endp[c.rank] - 1]) - pre1[first[c.rank]] : 0;
+    const uint64_t s_range_me = first[c.rank] < P ? pre1[endp[c.rank] - 1] + (bcf[endp[c.rank] - 1] ? 0 : LT(1, endp[c.rank] - 1)) - pre1[first[c.rank]] : 0;
     for (int p = tid; p < P; p += blockDim.x) {
         const int f = first[own[p]];
         uint64_t m0 = 0, m1 = 0;
-        for (int g = 0; g < c.rank; ++g) m0 += H(g, 0, p), m1 += H(g, 1, p);
+        for (int g = 0; g < c.rank; ++g) m0 += HL(g, 0, p), m1 += HL(g, 1, p);
         const uint64_t b0 = pre0[p] - pre0[f];
         const uint64_t b1 = bcf[p] ? s_range_me + chn[p] : pre1[p] - pre1[f];
         if (!c.ext) {
@@ -399,8 +439,8 @@ __global__ void __launch_bounds__(1024) k_plan(Ctx c) {
         }
         c.seg_start[p] = b0;
         c.seg_start[P + p] = b1;
-        c.seg_len[p] = tot0[p];
-        c.seg_len[P + p] = bcf[p] ? H(c.rank, 1, p) : tot1[p];
+        c.seg_len[p] = LT(0, p);
+        c.seg_len[P + p] = bcf[p] ? HL(c.rank, 1, p) : LT(1, p);
     }
     if (tid < 2 * MAX_RANKS) {
         const int d = tid >> 1, rel = tid & 1;
@@ -408,12 +448,12 @@ __global__ void __launch_bounds__(1024) k_plan(Ctx c) {
         if (d < N && first[d] < P) {
             const uint64_t *pre = rel ? pre1 : pre0;
             const int l = endp[d] - 1;
-            const uint64_t last = rel ? (bcf[l] ? 0 : tot1[l]) : tot0[l];
+            const uint64_t last = rel ? (bcf[l] ? 0 : LT(1, l)) : LT(0, l);
             size = pre[l] + last - pre[first[d]];
         }
         if (d < N && rel) size += bcs[d];
         c.recv_size[rel * MAX_RANKS + d] = size;
-        if (size > c.recv_cap[rel]) atomicOr(&cap_bad, 1);
+        if (size > (c.comp ? c.recv_cap_u[rel] : c.recv_cap[rel])) atomicOr(&cap_bad, 1);
         // EXTERNAL: the send arena holds this rank's whole input per relation
         // in a region of recv_cap tuples
         if (c.ext && d == 0 && c.n_in[rel] > c.recv_cap[rel]) atomicOr(&cap_bad, 1);
@@ -468,7 +508,8 @@ __global__ void __launch_bounds__(1024) k_plan(Ctx c) {
                 const uint64_t src = rel ? (uint64_t)c.rank : (uint64_t)own[p];
                 for (int g = 0; g < MAX_RANKS; ++g) {
                     ps[(size_t)i * MAX_RANKS + g] = g == 0 ? (c.seg_start[rel * P + p] | src << PIECE_SRC_SHIFT) : 0;
-                    pl[(size_t)i * MAX_RANKS + g] = g == 0 ? (uint32_t)own_len(rel, p) : 0;
+                    pl[(size_t)i * MAX_RANKS + g] =
+                        g == 0 ? (uint32_t)(rel ? (bcf[p] ? (uint64_t)HL(c.rank, 1, p) : LT(1, p)) : LT(0, p)) : 0;
                 }
             }
             continue;
@@ -527,7 +568,32 @@ __global__ void __launch_bounds__(1024) k_plan(Ctx c) {
             __syncthreads();
         }
     };
-    chunk_table((uint64_t)c.chunk_tuples);
+    chunk_table((uint64_t)(c.comp ? c.chunk_units : c.chunk_tuples));  // compressed: chunks of units
+    if (c.comp) {
+        // global row id of the first row of every (relation, rank, tile): rank
+        // g holds rows [sum_{g' < g} n_g', + n_g) (reading C12), tile c its
+        // local rows tile_range(n_g, G, c); the local pass adds a unit entry's
+        // offset to rebuild the id payload
+        __shared__ unsigned long long nrank[2][MAX_RANKS];
+        if (tid < 2 * MAX_RANKS) nrank[tid / MAX_RANKS][tid % MAX_RANKS] = 0;
+        __syncthreads();
+        for (int x = tid; x < 2 * N * P; x += blockDim.x) {
+            const int rel = x / (N * P), g = (x / P) % N, p = x % P;
+            const uint32_t h = H(g, rel, p);
+            if (h) atomicAdd(&nrank[rel][g], (unsigned long long)h);
+        }
+        __syncthreads();
+        for (int x = tid; x < 2 * N * c.G; x += blockDim.x) {
+            const int rel = x / (N * c.G), g = (x / c.G) % N, t = x % c.G;
+            uint64_t row0 = 0, lo, hi;
+            for (int h = 0; h < g; ++h) row0 += nrank[rel][h];
+            tile_range(nrank[rel][g], c.G, t, lo, hi);
+            c.rowbase[((size_t)rel * MAX_RANKS + g) * c.G + t] = (uint32_t)(row0 + lo);
+            // an entry holds the row's offset in its tile in 12 + B1 bits
+            if (hi - lo > (1ull << (12 + c.B1))) atomicOr(&cap_bad, 2);
+        }
+        __syncthreads();
+    }
     if (tid == 0) {
         // two-level local partitioning: when the owned
         // partitions span more than LOCAL2_NCH chunks on average, a first
@@ -545,7 +611,7 @@ __global__ void __launch_bounds__(1024) k_plan(Ctx c) {
         }
         if (BA > B2) BA = B2;
         if (BA > MAX_BA) BA = MAX_BA;
-        if (!c.mid[0] || (np << BA) > c.vcap) BA = 0;
+        if (!c.mid[0] || (np << BA) > c.vcap || c.comp) BA = 0;  // compressed: one local pass (it decodes)
         s_ba = BA;
     }
     __syncthreads();
@@ -554,6 +620,7 @@ __global__ void __launch_bounds__(1024) k_plan(Ctx c) {
     if (BA > 0 && c.chunk_tuples1s != c.chunk_tuples) chunk_table((uint64_t)c.chunk_tuples1s);
     if (tid == 0) {
         const bool fits = nch[0] <= c.max_chunks && nch[1] <= c.max_chunks;
+        if (cap_bad & 2) set_err(c, MGJ_EINVAL);  // tiles too long for the compressed entry
         if (cap_bad || !fits) set_err(c, MGJ_ECAPACITY);
         c.meta[MT_PLO] = plo;
         c.meta[MT_PHI] = phi;
@@ -562,7 +629,7 @@ __global__ void __launch_bounds__(1024) k_plan(Ctx c) {
         c.meta[MT_B2] = B2;
         c.meta[MT_NCH_R] = (int)nch[0];
         c.meta[MT_NCH_S] = (int)nch[1];
-        c.meta[MT_CHUNK] = BA ? c.chunk_tuples1s : c.chunk_tuples;
+        c.meta[MT_CHUNK] = c.comp ? c.chunk_units : (BA ? c.chunk_tuples1s : c.chunk_tuples);
         c.meta[MT_BA] = BA;
         c.meta[MT_QB] = B2 - BA;
         c.meta[MT_NLP] = np;

@@ -56,7 +56,8 @@ __global__ void k_chunkmap(Ctx c, ChunkDesc *desc) {
     if (!c.meta[MT_OK]) return;
     const int P = c.P, np = c.meta[MT_NP];
     const uint32_t nch_r = (uint32_t)c.meta[MT_NCH_R], total = nch_r + (uint32_t)c.meta[MT_NCH_S];
-    const uint64_t C = (uint64_t)(c.meta[MT_BA] ? c.chunk_tuples1s : c.chunk_tuples);  // the table k_plan built
+    // the table k_plan built: chunks of C tuples, or of C 32-byte units with the compressed shuffle
+    const uint64_t C = (uint64_t)(c.comp ? c.chunk_units : (c.meta[MT_BA] ? c.chunk_tuples1s : c.chunk_tuples));
     for (uint32_t ci = blockIdx.x * blockDim.x + threadIdx.x; ci < total; ci += gridDim.x * blockDim.x) {
         const int rel = ci < nch_r ? 0 : 1;
         const uint32_t li = rel ? ci - nch_r : ci;
@@ -251,8 +252,9 @@ __global__ void __launch_bounds__(512) k_countA(Ctx c, const ChunkDesc *cdesc) {
 // ---------------------------------------------------------------------------
 enum LocalMode { LM_SINGLE = 0, LM_SPLIT = 1, LM_SECOND = 2 };
 
-template <typename K, int MODE, int RSEL = 2>
+template <typename K, int MODE, int RSEL = 2, bool COMP = false>
 __device__ __forceinline__ void local_body(const Ctx &c, const ChunkDesc *cdesc) {
+    static_assert(!COMP || (MODE == LM_SINGLE && sizeof(K) == 4), "compressed input: single pass, 4-byte keys");
     constexpr bool SPLIT = MODE == LM_SPLIT;
     using Tup = typename Layout<K>::Tup;
     constexpr int TB = Layout<K>::TB, ALIGN = Layout<K>::ALIGN;
@@ -300,12 +302,20 @@ __device__ __forceinline__ void local_body(const Ctx &c, const ChunkDesc *cdesc)
     auto issue = [&](uint32_t j, const ChunkDesc &d) {
         const uint32_t ci = c0 + blockIdx.x + j * gridDim.x;
         const int rel = ci < nch_r ? 0 : 1;
+        sdesc[j & 1] = d;
+        uint64_t *b = &bar[j & 1];
+        if constexpr (COMP) {  // whole 32-byte units
+            const uint32_t bytes = d.len * 32u;
+            mbar_arrive_expect_tx(b, bytes);
+            if (bytes)
+                tma_load_1d(buf(j & 1), c.arena[piece_src(d.start)] + c.lay.recv[rel] + piece_off(d.start) * 32, bytes, b,
+                            pol);
+            return;
+        }
         const uint64_t st = from_mid ? d.start : piece_off(d.start);
         const uint64_t g0 = st & ~(uint64_t)(ALIGN - 1);
         const uint64_t g1 = (st + d.len + ALIGN - 1) & ~(uint64_t)(ALIGN - 1);
         const uint32_t bytes = (uint32_t)((g1 - g0) * TB);
-        sdesc[j & 1] = d;
-        uint64_t *b = &bar[j & 1];
         mbar_arrive_expect_tx(b, bytes);
         if (bytes) tma_load_1d(buf(j & 1), chunk_src(rel, d.start) - (st - g0), bytes, b, pol);
     };
@@ -327,17 +337,47 @@ __device__ __forceinline__ void local_body(const Ctx &c, const ChunkDesc *cdesc)
         // partition of this chunk's tuples (a first pass's padding tuples lie in another one)
         const uint32_t p = (uint32_t)c.plist[from_mid ? d.pi >> BA : d.pi];
         Tup t[VMAX];
+        uint32_t cvalid = 0;  // COMP: bit v set if t[v] holds a decoded tuple
+        if constexpr (COMP) {
+            // NEXT-1 decode: this thread's units tid, tid + 1024 of the chunk, CU_N
+            // entries each: key = (entry's low 32 - B1 bits) << B1 | p, payload =
+            // the unit's (rank, tile) first row id + the entry's row offset
+            const int kb = 32 - c.B1;
 #pragma unroll
-        for (int v = 0; v < VMAX; ++v) {
-            const uint32_t i = tid + v * LOCAL_THREADS;
-            if (v < V && i < len) t[v] = buf(X)[skip + i];
+            for (int k = 0; k < VMAX / CU_N; ++k) {
+                const uint32_t un = tid + k * LOCAL_THREADS;
+                if (un < len) {
+                    const uint4 lo4 = *reinterpret_cast<const uint4 *>(reinterpret_cast<const char *>(buf(X)) + un * 32u);
+                    const uint4 hi4 = *reinterpret_cast<const uint4 *>(reinterpret_cast<const char *>(buf(X)) + un * 32u + 16);
+                    const unsigned long long a[4] = {(unsigned long long)lo4.x | (unsigned long long)lo4.y << 32,
+                                                     (unsigned long long)lo4.z | (unsigned long long)lo4.w << 32,
+                                                     (unsigned long long)hi4.x | (unsigned long long)hi4.y << 32,
+                                                     (unsigned long long)hi4.z | (unsigned long long)hi4.w << 32};
+                    const uint32_t meta = hi4.w, nv = meta & 7u;
+                    const uint32_t tb = __ldg(c.rowbase + ((size_t)rel * MAX_RANKS + ((meta >> 3) & 7u)) * c.G + (meta >> 6));
+#pragma unroll
+                    for (int e = 0; e < CU_N; ++e) {
+                        const unsigned long long en = unit_entry(a, e);
+                        t[k * CU_N + e].x = (K)((((uint32_t)en & ((1u << kb) - 1u)) << c.B1) | p);
+                        t[k * CU_N + e].y = (K)(tb + (uint32_t)(en >> kb));
+                        if ((uint32_t)e < nv) cvalid |= 1u << (k * CU_N + e);
+                    }
+                }
+            }
+        } else {
+#pragma unroll
+            for (int v = 0; v < VMAX; ++v) {
+                const uint32_t i = tid + v * LOCAL_THREADS;
+                if (v < V && i < len) t[v] = buf(X)[skip + i];
+            }
         }
         uint32_t rq[VMAX];  // rank << 16 | digit (0xffffffff: dropped)
 #pragma unroll
         for (int v = 0; v < VMAX; ++v) {
             const uint32_t i = tid + v * LOCAL_THREADS;
             rq[v] = 0xffffffffu;
-            if (v < V && i < len && (!from_mid || digit1(t[v].x, P) == p)) {
+            const bool have = COMP ? ((cvalid >> v) & 1u) != 0 : (v < V && i < len);
+            if (have && (!from_mid || digit1(t[v].x, P) == p)) {
                 const uint32_t q = digit2(t[v].x, shift, Q);
                 rq[v] = (atomicAdd(&bins[q], 1u) << 16) | q;
             }
@@ -477,14 +517,14 @@ __global__ void __launch_bounds__(LOCAL_THREADS, 1) k_local_second(Ctx c, const 
 // the chunks of R (rsel 0), of S (1) or of both (2).  With the shuffle
 // overlapped (§8(e)), R's launch first waits for every rank's R tuples
 // (SIG_DATA_R) and runs beside the scatter of S on the SMs it leaves free.
-template <typename K, int RSEL>
+template <typename K, int RSEL, bool COMP = false>
 __global__ void __launch_bounds__(LOCAL_THREADS, 1) k_local(Ctx c, const ChunkDesc *cdesc) {
     if (!c.meta[MT_OK] || c.meta[MT_BA]) return;
     // timeline stamps for the overlapped launches only: in the single launch
     // over both relations (the one-GPU path) they cost a 4-byte spill
     constexpr int id = RSEL == 0 ? MGJ_TR_LOCAL_R : MGJ_TR_LOCAL_S;
     if constexpr (RSEL != 2) trace_begin(c, id);
-    local_body<K, LM_SINGLE, RSEL>(c, cdesc);
+    local_body<K, LM_SINGLE, RSEL, COMP>(c, cdesc);
     if constexpr (RSEL != 2) trace_end(c, id);
 }
 

@@ -29,6 +29,7 @@ struct Norm {  // validated config with the automatic fields filled in
     int B1, P, b2_max, tuple_bytes, chunk_tuples, chunk_region, probe_slots, probe_target;
     int chunk_tuples2, chunk_region2, qm2_bits, chunk_tuples1s;
     uint64_t recv_cap[2], max_chunks, max_items, out_cap, mid_cap;
+    uint64_t recv_cap_u[2];  // compressed shuffle: 32-byte units each receive buffer holds
     bool split;  // first local pass possible (mid buffers allocated)
     Arena lay;
 };
@@ -42,11 +43,15 @@ int ceil_log2(uint64_t x) {
 mgj_status normalize(const mgj_config *in, Norm *o) {
     if (!in) return MGJ_EINVAL;
     mgj_config c = *in;
-    for (int i = 0; i < 1; ++i)
+    for (int i = 0; i < 2; ++i)
         if (c.reserved[i]) return MGJ_EINVAL;
     if (c.peer_timeout_ms < 0) return MGJ_EINVAL;
     if (c.shuffle_overlap < -1 || c.shuffle_overlap > 1 || c.overlap_local_sms < 0) return MGJ_EINVAL;
     if (c.trace != 0 && c.trace != 1) return MGJ_EINVAL;
+    if (c.compress != 0 && c.compress != 1) return MGJ_EINVAL;
+    // the compressed shuffle (NEXT-1): 4-byte keys and payloads, in-kernel peer stores
+    if (c.compress && (c.key_bytes != 4 || c.shuffle_mode != MGJ_SHUFFLE_P2P)) return MGJ_EINVAL;
+    if (c.compress && c.radix_bits_global > 10) return MGJ_EINVAL;  // the compressed instance: P <= 1024
     if (c.skew_bcast < -1 || c.skew_bcast > 1) return MGJ_EINVAL;
     if (c.local_split_bits < -1 || c.local_split_bits > MAX_BA) return MGJ_EINVAL;
     if (c.shuffle_mode != MGJ_SHUFFLE_P2P && c.shuffle_mode != MGJ_SHUFFLE_EXTERNAL) return MGJ_EINVAL;
@@ -104,6 +109,8 @@ mgj_status normalize(const mgj_config *in, Norm *o) {
     // chunks of the chunked pass: sum over (sub-)partitions of ceil(size / C); at most
     // local2_vcap(P) sub-partitions after a first pass
     o->max_chunks = rmax / C + (uint64_t)local2_vcap(o->P) + 2;
+    if (c.compress)  // chunks of CHUNK_UNITS units: >= rmax / CU_N units plus one partial unit per (rank, tile, p)
+        o->max_chunks = (rmax / CU_N + (uint64_t)MAX_RANKS * 1024 * o->P) / CHUNK_UNITS + o->P + 2;
     // the first local pass exists if forced, or (auto) if one owned partition could
     // span more than LOCAL2_NCH chunks; its output pads each (chunk, run) once
     o->split = c.local_split_bits > 0 || (c.local_split_bits == 0 && rmax > (uint64_t)LOCAL2_NCH * C);
@@ -120,12 +127,24 @@ mgj_status normalize(const mgj_config *in, Norm *o) {
     off = align_up(off + (uint64_t)MAX_RANKS * 2 * o->P * 4, 4096);
     L.resmail = off;
     off = align_up(off + MAX_RANKS * RES_W * 8, 4096);
+    L.umail = off;
+    off = align_up(off + (uint64_t)MAX_RANKS * 2 * o->P * 4, 4096);
     L.cfgmail = off;
     off = align_up(off + MAX_RANKS * 4 * 8, 4096);
+    // compressed: a (source rank, tile, partition) run ends in a partial unit, so
+    // short runs take more room than their tuples (at most one unit per tuple);
+    // the bound counts <= 8 ranks x 256 tiles x P partial units
+    for (int r = 0; r < 2; ++r)
+        o->recv_cap_u[r] = c.compress ? std::min<uint64_t>(o->recv_cap[r], o->recv_cap[r] / CU_N + 1 +
+                                                                               (uint64_t)MAX_RANKS * 256 * o->P)
+                                      : 0;
+    auto recv_bytes = [&](int r) {
+        return std::max<uint64_t>(o->recv_cap[r] * o->tuple_bytes, o->recv_cap_u[r] * 32);
+    };
     L.recv[0] = off;
-    off = align_up(off + o->recv_cap[0] * o->tuple_bytes, 4096);
+    off = align_up(off + recv_bytes(0), 4096);
     L.recv[1] = off;
-    off = align_up(off + o->recv_cap[1] * o->tuple_bytes, 4096);
+    off = align_up(off + recv_bytes(1), 4096);
     L.total = off;
     o->c = c;
     return MGJ_OK;
@@ -184,11 +203,16 @@ void *dalloc(mgj_plan_s *h, size_t bytes, mgj_status *st) {
     return p;
 }
 
+// sub-tile of the scatter (a1 counts per sub-tile of the same size)
+int scat_T_of(const Norm &n) { return n.c.compress ? scat_geom_comp().T : scat_geom(n.P, n.c.key_bytes).T; }
+
 size_t hist_smem(const Norm &n) {
-    const int T = scat_geom(n.P, n.c.key_bytes).T;
+    const int T = scat_T_of(n);
     return (size_t)hist_nb(T, n.c.key_bytes) * T * n.c.key_bytes + (size_t)n.P * 8;
 }
-size_t plan_smem(const Norm &n) { return (size_t)n.P * 5 * 8 + (size_t)n.P * 4 + (size_t)(n.P + 1) * 4 + (size_t)n.P; }
+size_t plan_smem(const Norm &n) {
+    return (size_t)n.P * 5 * 8 + (size_t)n.P * 4 + (size_t)(n.P + 1) * 4 + (size_t)n.P + 8 + (size_t)n.P * 2 * 8;
+}
 size_t scatter_smem(const Norm &n) { return scatter_smem_bytes(n.P, n.c.key_bytes); }
 size_t planA_smem(const Norm &n) { return ((size_t)local2_vcap(n.P) + 1) * 12; }
 size_t local_smem(const Norm &n) { return local_smem_bytes(n.chunk_tuples, 1 << n.b2_max, n.tuple_bytes); }
@@ -203,6 +227,12 @@ cudaError_t set_attrs(const Norm &n) {
     if ((e = cudaFuncSetAttribute(k_hist<K>, A, (int)hist_smem(n)))) return e;
     if ((e = cudaFuncSetAttribute(k_plan, A, (int)plan_smem(n)))) return e;
     if ((e = cudaFuncSetAttribute(scatter_kernel<K>(n.P), A, (int)scatter_smem(n)))) return e;
+    if (n.c.compress && n.P <= 1024) {
+        if ((e = cudaFuncSetAttribute(scatter_kernel_comp(), A, (int)scat_smem_bytes_comp(n.P)))) return e;
+        if ((e = cudaFuncSetAttribute(k_local<uint32_t, 0, true>, A, (int)local_smem(n)))) return e;
+        if ((e = cudaFuncSetAttribute(k_local<uint32_t, 1, true>, A, (int)local_smem(n)))) return e;
+        if ((e = cudaFuncSetAttribute(k_local<uint32_t, 2, true>, A, (int)local_smem(n)))) return e;
+    }
     if ((e = cudaFuncSetAttribute(k_local<K, 0>, A, (int)local_smem(n)))) return e;
     if ((e = cudaFuncSetAttribute(k_local<K, 1>, A, (int)local_smem(n)))) return e;
     if ((e = cudaFuncSetAttribute(k_local<K, 2>, A, (int)local_smem(n)))) return e;
@@ -239,10 +269,12 @@ void launch_shuffle(mgj_plan_s *h, cudaStream_t s) {
     Ctx cs = h->ctx;
     if (cs.ext)
         for (int g = 0; g < MAX_RANKS; ++g) cs.arena[g] = h->send_arena;
-    const auto scat = scatter_kernel<K>(n.P);
+    const bool comp = h->ctx.comp;
+    const auto scat = comp ? scatter_kernel_comp() : scatter_kernel<K>(n.P);
+    const size_t ssm = comp ? scat_smem_bytes_comp(n.P) : scatter_smem(n);
     const int nt = scatter_threads(n.P, n.c.key_bytes);
     if (h->overlap) {
-        scat<<<h->ctx.G, nt, scatter_smem(n), s>>>(cs, 0, 0);  // a3, R
+        scat<<<h->ctx.G, nt, ssm, s>>>(cs, 0, 0);  // a3, R
         // §8(e) ("data distribution and local partitioning start
         // together"; Rationale 2): once every rank's R tuples have
         // landed, R is partitioned locally on local_sms SMs of a second stream
@@ -250,12 +282,15 @@ void launch_shuffle(mgj_plan_s *h, cudaStream_t s) {
         cudaEventRecord(h->ev_fork, s);
         cudaStreamWaitEvent(h->aux, h->ev_fork, 0);
         k_wait<<<1, 32, 0, h->aux>>>(h->ctx, SIG_DATA_R, -1);
-        k_local<K, 0><<<h->local_sms, LOCAL_THREADS, local_smem(n), h->aux>>>(h->ctx, h->cdesc);
+        if (comp)
+            k_local<uint32_t, 0, true><<<h->local_sms, LOCAL_THREADS, local_smem(n), h->aux>>>(h->ctx, h->cdesc);
+        else
+            k_local<K, 0><<<h->local_sms, LOCAL_THREADS, local_smem(n), h->aux>>>(h->ctx, h->cdesc);
         cudaEventRecord(h->ev_join, h->aux);
-        scat<<<h->scatter_sms, nt, scatter_smem(n), s>>>(cs, 1, 1);  // a3, S
+        scat<<<h->scatter_sms, nt, ssm, s>>>(cs, 1, 1);  // a3, S
         h->launches += 7;
     } else {
-        scat<<<h->ctx.G, nt, scatter_smem(n), s>>>(cs, 0, 1);  // a3, R then S in one launch
+        scat<<<h->ctx.G, nt, ssm, s>>>(cs, 0, 1);  // a3, R then S in one launch
         h->launches += 4;
     }
 }
@@ -284,9 +319,15 @@ void launch_join(mgj_plan_s *h, cudaStream_t s) {
         h->launches += 4;
     }
     if (h->overlap)
-        k_local<K, 1><<<h->nsm, LOCAL_THREADS, local_smem(n), s>>>(h->ctx, h->cdesc);
+        if (h->ctx.comp)
+            k_local<uint32_t, 1, true><<<h->nsm, LOCAL_THREADS, local_smem(n), s>>>(h->ctx, h->cdesc);
+        else
+            k_local<K, 1><<<h->nsm, LOCAL_THREADS, local_smem(n), s>>>(h->ctx, h->cdesc);
     else
-        k_local<K, 2><<<h->nsm, LOCAL_THREADS, local_smem(n), s>>>(h->ctx, h->cdesc);
+        if (h->ctx.comp)
+            k_local<uint32_t, 2, true><<<h->nsm, LOCAL_THREADS, local_smem(n), s>>>(h->ctx, h->cdesc);
+        else
+            k_local<K, 2><<<h->nsm, LOCAL_THREADS, local_smem(n), s>>>(h->ctx, h->cdesc);
     cudaEventRecord(h->ev[4], s);
     k_itemize<K><<<h->nsm * 4, 256, 0, s>>>(h->ctx);
     if (n.c.materialize)
@@ -389,8 +430,12 @@ mgj_status mgj_plan(const mgj_config *cfg, const mgj_peers *peers, mgj_handle *o
     c.materialize = n.c.materialize;
     c.timeout_ns = (n.c.peer_timeout_ms ? (uint64_t)n.c.peer_timeout_ms : 20000ull) * 1000000ull;
     c.ext = n.c.shuffle_mode == MGJ_SHUFFLE_EXTERNAL;
+    c.comp = n.c.compress;
+    c.chunk_units = CHUNK_UNITS;
     c.max_items = (uint32_t)n.max_items;
     c.recv_cap[0] = n.recv_cap[0];
+    c.recv_cap_u[0] = n.recv_cap_u[0];
+    c.recv_cap_u[1] = n.recv_cap_u[1];
     c.recv_cap[1] = n.recv_cap[1];
     c.max_chunks = n.max_chunks;
     c.out_cap = n.out_cap;
@@ -407,7 +452,11 @@ mgj_status mgj_plan(const mgj_config *cfg, const mgj_peers *peers, mgj_handle *o
         c.hA = reinterpret_cast<uint32_t *>(zb + z_ha);
     }
     c.tile_base = static_cast<uint32_t *>(dalloc(h, 2ull * c.G * P * 4, &st));
-    c.scat_T = scat_geom(P, n.c.key_bytes).T;
+    if (c.comp) {
+        c.rowbase = static_cast<uint32_t *>(dalloc(h, 2ull * MAX_RANKS * c.G * 4, &st));
+        c.rank_units = static_cast<uint32_t *>(dalloc(h, 2ull * P * 4, &st));
+    }
+    c.scat_T = scat_T_of(n);
     c.sub_ns = (int32_t)((std::max(n.c.r_capacity, n.c.s_capacity) / c.G + 8) / c.scat_T + 2);
     c.sub_hist = static_cast<uint16_t *>(dalloc(h, 2ull * c.G * c.sub_ns * P * 2, &st));
     h->cdesc = static_cast<ChunkDesc *>(dalloc(h, 2 * n.max_chunks * sizeof(ChunkDesc), &st));

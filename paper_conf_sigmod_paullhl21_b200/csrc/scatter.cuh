@@ -174,7 +174,7 @@ __device__ __forceinline__ void st_group(void *dst, const typename Vec<BYTES>::T
 // spread over all peers' links instead of visiting the ranks in step.  The
 // last CTA raises SIG_DATA_R / SIG_DATA_S at every peer after a system fence.
 // ---------------------------------------------------------------------------
-template <typename K, int T, int SG, int PPT, int NT>
+template <typename K, int T, int SG, int PPT, int NT, bool COMP = false>
 __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c, int rel0, int rel1) {
     using Tup = typename TupT<K>::T;
     constexpr int TB = (int)sizeof(Tup);
@@ -182,15 +182,17 @@ __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c, int rel0, int rel1) {
     constexpr int LU = 16 / (int)sizeof(K);    // tuples per 16-byte stage vector
     constexpr int NU = V / LU;                 // vectors per thread
     static_assert(NU * LU == V && NU >= 1, "sub-tile");
-    constexpr int GB = SG * TB;                // group bytes
+    // COMP (NEXT-1): a group is one 32-byte unit of SG = CU_N encoded tuples
+    static_assert(!COMP || (SG == CU_N && sizeof(K) == 4 && PPT == 1), "compressed scatter");
+    constexpr int GB = COMP ? 32 : SG * TB;    // group bytes at the destination
     constexpr int CW = SG > 1 ? SG - 1 : 1;    // carry capacity (tuples)
-    using GV = typename Vec<GB>::T;
+    using GV = typename Vec<COMP ? 32 : SG * TB>::T;
     typedef unsigned long long ull;
     // `sorted` swizzle: the two 16-byte halves of every 32-byte group whose
     // index has bit 2 set are swapped, so that the write-out's 16-byte loads
     // (8 consecutive groups per quarter warp) hit distinct banks
     auto swz = [](uint32_t s) -> uint32_t {
-        if constexpr (SG > 1 && SG * sizeof(Tup) == 32) return s ^ (((s >> (SG == 4 ? 4 : 3)) & 1u) * (SG / 2));
+        if constexpr (!COMP && SG > 1 && SG * sizeof(Tup) == 32) return s ^ (((s >> (SG == 4 ? 4 : 3)) & 1u) * (SG / 2));
         else return s;
     };
     extern __shared__ __align__(128) unsigned char smem[];
@@ -288,6 +290,18 @@ __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c, int rel0, int rel1) {
             prefetch_l2(in_pay + first, bytes);
         }
     };
+    // COMP: global row id of the rank's first row, a tile's first local row, and one entry
+    auto cbase_rel = [&](int rel) -> uint32_t { return COMP ? __ldg(c.rowbase + ((size_t)rel * MAX_RANKS + c.rank) * c.G) : 0u; };
+    auto tile_lo_of = [&](int rel, int tile) -> uint64_t {
+        uint64_t lo, hi;
+        tile_range(c.n_in[rel], c.G, tile, lo, hi);
+        return lo;
+    };
+    const int kb = 32 - c.B1;  // key bits above the partition digit
+    auto unit_enc = [&](uint32_t key, uint32_t pay, uint32_t tilebase) -> unsigned long long {
+        return (unsigned long long)(key >> c.B1) | ((unsigned long long)(pay - tilebase) << kb);
+    };
+    bool bad_pay = false;  // COMP: a payload that is not its global row id
     auto fetch_carry = [&]() {  // the incomplete last groups of the previous sub-tile -> registers
         if (pending) {
 #pragma unroll
@@ -298,16 +312,29 @@ __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c, int rel0, int rel1) {
             pending = false;
         }
     };
-    auto flush = [&](int rel) {  // end of a tile: store the remaining tails tuple by tuple
+    auto flush = [&](int rel, int tile) {  // end of a tile: store the remaining tails
         fetch_carry();
+        if constexpr (COMP) {  // one partial unit of cc entries
+            if (!skp[0] && cc[0]) {
+                unsigned long long e[CU_N], a[4];
+                const uint32_t tb0 = cbase_rel(rel) + (uint32_t)tile_lo_of(rel, tile);
 #pragma unroll
-        for (int k = 0; k < PPT; ++k)
+                for (int i = 0; i < CU_N; ++i)
+                    e[i] = i < (int)cc[0] ? unit_enc((uint32_t)carry[0][i < CW ? i : 0].x, (uint32_t)carry[0][i < CW ? i : 0].y, tb0) : 0ull;
+                unit_pack(e, cc[0] | (uint32_t)c.rank << 3 | (uint32_t)tile << 6, a);
+                char *d = c.arena[dstr[0]] + c.lay.recv[rel] + (size_t)bidx[0] * 32;
+                asm volatile("st.global.v4.u64 [%0], {%1,%2,%3,%4};" ::"l"(d), "l"(a[0]), "l"(a[1]), "l"(a[2]), "l"(a[3]) : "memory");
+            }
+        } else {
 #pragma unroll
-            for (int i = 0; i < CW; ++i)
-                if (!skp[k] && i >= (int)hd[k] && i < (int)cc[k]) {
-                    Tup *d = reinterpret_cast<Tup *>(c.arena[dstr[k]] + c.lay.recv[rel]);
-                    d[(uint32_t)(bidx[k] + i)] = carry[k][i];
-                }
+            for (int k = 0; k < PPT; ++k)
+#pragma unroll
+                for (int i = 0; i < CW; ++i)
+                    if (!skp[k] && i >= (int)hd[k] && i < (int)cc[k]) {
+                        Tup *d = reinterpret_cast<Tup *>(c.arena[dstr[k]] + c.lay.recv[rel]);
+                        d[(uint32_t)(bidx[k] + i)] = carry[k][i];
+                    }
+        }
     };
     auto set_base = [&](int rel, int tile) {  // destination of this tile's first tuple of each owned partition
         const uint32_t *tb = c.tile_base + ((size_t)rel * c.G + tile) * P;
@@ -321,9 +348,9 @@ __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c, int rel0, int rel1) {
                 // selectively broadcast partition (a2, NEXT-2)
                 const int dst = (rel && c.bcast[p]) ? c.rank : c.owner[p];
                 skp[k] = c.pskip[p] != 0;
-                const uint64_t idx = so[p] + tb[p];
+                const uint64_t idx = so[p] + tb[p];  // COMP: in 32-byte units (runs start unit-aligned)
                 const ull a = (ull)(c.arena[dst] + c.lay.recv[rel]) + idx * (uint64_t)TB;
-                const uint32_t h = SG > 1 ? (uint32_t)((a & (GB - 1)) / TB) : 0u;
+                const uint32_t h = (SG > 1 && !COMP) ? (uint32_t)((a & (GB - 1)) / TB) : 0u;
                 bidx[k] = (uint32_t)idx - h;  // may wrap below 0: placeholders are never stored
                 dstr[k] = (uint8_t)dst;
                 cc[k] = hd[k] = h;
@@ -394,8 +421,9 @@ __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c, int rel0, int rel1) {
         uint32_t len;
         span(u, first, len);
         const Cur nx = next_cur(u);
+        const uint32_t row0 = cbase_rel(u.rel);  // COMP: global row id of this rank's first row
         if (u.rel * c.G + u.tile != cur_tile) {  // thread-private partition state: no barrier needed
-            if (cur_tile >= 0) flush(cur_tile / c.G);
+            if (cur_tile >= 0) flush(cur_tile / c.G, cur_tile % c.G);
             set_base(u.rel, u.tile);
             cur_tile = u.rel * c.G + u.tile;
         }
@@ -405,7 +433,7 @@ __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c, int rel0, int rel1) {
 #pragma unroll
         for (int k = 0; k < PPT; ++k) {
             cnt[k] = cc[k] + ncnt[k];
-            seg[k] = (cnt[k] + SG - 1) & ~(uint32_t)(SG - 1);
+            seg[k] = COMP ? (cnt[k] + SG - 1) / SG * SG : (cnt[k] + SG - 1) & ~(uint32_t)(SG - 1);
             tsum += seg[k];
         }
         load_counts(nx, ncnt);  // prefetch (consumed next iteration)
@@ -419,13 +447,13 @@ __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c, int rel0, int rel1) {
                 for (int i = 0; i < CW; ++i)
                     if (i < (int)cc[k]) sput(o + i, carry[k][i]);
                 off[p] = o + cc[k];
-                const uint32_t full = cnt[k] & ~(uint32_t)(SG - 1);
+                const uint32_t full = COMP ? cnt[k] / SG * SG : cnt[k] & ~(uint32_t)(SG - 1);
                 PInfo in;
-                in.didx = bidx[k] - o;
+                in.didx = COMP ? bidx[k] - o / SG : bidx[k] - o;  // COMP: units
                 in.lim = (uint16_t)(skp[k] ? o : o + cnt[k]);  // a skipped partition's groups are never stored
                 in.head = (hd[k] && full) ? (uint16_t)((o / SG) << 2 | hd[k]) : PI_NONE;
                 pinfo[p] = in;
-                bidx[k] += full;
+                bidx[k] += COMP ? full / SG : full;
                 if (full) hd[k] = 0;
                 cc[k] = cnt[k] - full;
                 lim[k] = o + cnt[k];
@@ -462,6 +490,7 @@ __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c, int rel0, int rel1) {
                 Tup t;
                 t.x = kk[v];
                 t.y = pp[v];
+                if constexpr (COMP) bad_pay |= (uint32_t)pp[v] != row0 + (uint32_t)(first + i);
                 sput(atomicAdd(&off[digit1(kk[v], P)], 1u), t);
             }
         }
@@ -470,10 +499,30 @@ __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c, int rel0, int rel1) {
         // write-out: one group per thread per step, rotated by rank share for N > 1
         const uint32_t ngroups = total / SG;
         const ull ob_rel = (ull)(c.arena[0] + c.lay.recv[u.rel]);  // N = 1: the one receive buffer
+        const uint32_t tbase = row0 + (uint32_t)u.lo;  // COMP: global row id of this tile's first row
         const uint32_t rot = (uint32_t)(((uint64_t)ngroups * rot_num) / (uint32_t)c.world);
         for (uint32_t w = tid; w < ngroups; w += NT) {
             const uint32_t gi = w + rot < ngroups ? w + rot : w + rot - ngroups;
             const uint32_t slot = gi * SG;
+            if constexpr (COMP) {
+                Tup tt[CU_N];
+#pragma unroll
+                for (int e = 0; e < CU_N; ++e) tt[e] = sget(slot + e);
+                const uint32_t pidx = (uint32_t)tt[0].x & (uint32_t)(P - 1);
+                const uint2 pv = lds64_at(pinfo_s + pidx * 8u);
+                if (slot + SG <= (pv.y & 0xffffu)) {
+                    const ull ob = c.world == 1 ? ob_rel : obase[u.rel * MAX_RANKS + own8[u.rel * P + pidx]];
+                    unsigned long long e[CU_N], a[4];
+#pragma unroll
+                    for (int x = 0; x < CU_N; ++x) e[x] = unit_enc((uint32_t)tt[x].x, (uint32_t)tt[x].y, tbase);
+                    unit_pack(e, (uint32_t)CU_N | (uint32_t)c.rank << 3 | (uint32_t)u.tile << 6, a);
+                    char *dst = reinterpret_cast<char *>(ob + (ull)(uint32_t)(pv.x + slot / SG) * 32);
+                    asm volatile("st.global.v4.u64 [%0], {%1,%2,%3,%4};" ::"l"(dst), "l"(a[0]), "l"(a[1]), "l"(a[2]),
+                                 "l"(a[3])
+                                 : "memory");
+                }
+                continue;
+            }
             GV gv;
             if constexpr (GB == 32) {  // two conflict-free 16-byte halves (swizzled)
                 gv.a = lds128_at(saddr(slot));
@@ -497,7 +546,8 @@ __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c, int rel0, int rel1) {
             }
         }
     }
-    if (cur_tile >= 0) flush(cur_tile / c.G);
+    if (cur_tile >= 0) flush(cur_tile / c.G, cur_tile % c.G);
+    if (COMP && bad_pay) set_err(c, MGJ_EINVAL);
 
     // ---- every CTA: make its (peer) stores visible, the last one signals ----
     __threadfence_system();
@@ -510,6 +560,18 @@ __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c, int rel0, int rel1) {
             for (int rel = rel0; rel <= rel1; ++rel) signal_all(c, rel ? SIG_DATA_S : SIG_DATA_R);
         }
     }
+}
+
+// The compressed-shuffle instance (NEXT-1): 4-byte keys, P <= 1024.
+constexpr ScatGeom scat_geom_comp() { return ScatGeom{8192, CU_N, 1, 1024}; }
+inline size_t scat_smem_bytes_comp(int P) {
+    const ScatGeom g = scat_geom_comp();
+    return (size_t)g.T * 4 + ((size_t)g.T + 2 * (size_t)(g.SG - 1) * P) * 8 + (size_t)P * sizeof(PInfo) +
+           (size_t)P * 4 + 2 * (size_t)MAX_RANKS * 8 + 2 * (size_t)P;
+}
+inline void (*scatter_kernel_comp())(Ctx, int, int) {
+    constexpr ScatGeom g = scat_geom_comp();
+    return k_scatter<uint32_t, g.T, g.SG, g.PPT, g.NT, true>;
 }
 
 template <typename K>

@@ -54,7 +54,7 @@ class Config(ctypes.Structure):
                 ("local_split_bits", ctypes.c_int32), ("skew_bcast", ctypes.c_int32),
                 ("peer_timeout_ms", ctypes.c_int32), ("shuffle_overlap", ctypes.c_int32),
                 ("overlap_local_sms", ctypes.c_int32), ("trace", ctypes.c_int32),
-                ("reserved", ctypes.c_int32 * 1)]
+                ("compress", ctypes.c_int32), ("reserved", ctypes.c_int32 * 2)]
 
 
 class Exchange(ctypes.Structure):
@@ -139,7 +139,7 @@ def _stream(stream):
 def make_config(rank=0, world_size=1, key_bytes=4, r_capacity=0, s_capacity=0, recv_capacity_r=0,
                 recv_capacity_s=0, radix_bits_global=0, radix_bits_local=0, materialize=False,
                 num_sms=0, out_capacity=0, shuffle_mode=0, local_split_bits=0, skew_bcast=0,
-                peer_timeout_ms=0, shuffle_overlap=0, overlap_local_sms=0, trace=False) -> Config:
+                peer_timeout_ms=0, shuffle_overlap=0, overlap_local_sms=0, trace=False, compress=False) -> Config:
     c = Config()
     c.rank, c.world_size = rank, world_size
     c.key_bytes = c.payload_bytes = key_bytes
@@ -156,6 +156,7 @@ def make_config(rank=0, world_size=1, key_bytes=4, r_capacity=0, s_capacity=0, r
     c.shuffle_overlap = shuffle_overlap
     c.overlap_local_sms = overlap_local_sms
     c.trace = int(bool(trace))
+    c.compress = int(bool(compress))
     return c
 
 

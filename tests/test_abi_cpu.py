@@ -48,7 +48,9 @@ def test_strerror(mgj):
                                  dict(radix_bits_global=13), dict(radix_bits_local=12), dict(r_capacity=1 << 32),
                                  dict(local_split_bits=7), dict(local_split_bits=-2), dict(skew_bcast=2),
                                  dict(skew_bcast=-2), dict(peer_timeout_ms=-1), dict(shuffle_overlap=2),
-                                 dict(shuffle_overlap=-2), dict(overlap_local_sms=-1)])
+                                 dict(shuffle_overlap=-2), dict(overlap_local_sms=-1),
+                                 dict(compress=1, key_bytes=8), dict(compress=1, shuffle_mode=1),
+                                 dict(compress=1, radix_bits_global=11)])
 def test_invalid_config_rejected_without_gpu(mgj, bad):
     kw = dict(r_capacity=1024, s_capacity=1024)
     kw.update(bad)

@@ -1006,3 +1006,68 @@ def test_overlap_timeline(mgj):
         else:  # one launch over both relations after both scatters (not stamped)
             assert "local_R" not in t and t["itemize"][0] >= t["scatter_S"][1], t
         j.close()
+
+
+# ------------------------------------------------------------ NEXT-1: the compressed shuffle
+@pytest.mark.parametrize("N,kind,kw", [(1, "m1", {}), (2, "m1", {}), (4, "m1", {}), (1, "m1", {"radix_bits_global": 4}),
+                                       (3, "zipf", {}), (4, "zipf", {"skew_bcast": 1, "radix_bits_global": 8}),
+                                       (2, "m1", {"shuffle_overlap": 1}), (1, "m1", {"radix_bits_global": 10,
+                                                                                     "radix_bits_local": 6})])
+def test_compress_parity(mgj, N, kind, kw):
+    """compress = 1: tuples cross the shuffle as
+    (key >> B1, row offset in the source tile) entries, five per 32-byte unit;
+    the local pass rebuilds key and id payload.  Bit-exact vs the oracle
+    (count, checksum, pair digest, sorted triples) on N virtual ranks."""
+    w = datagen.M1() if kind == "m1" else datagen.Workload("zipf", 1 << 16, 1 << 18, 1.0)
+    mat = kind == "m1"
+    joins, res, _ = run_virtual(mgj, w, N, materialize=mat, compress=True, **kw)
+    d = w.rank_inputs()
+    ref = oracle.join(d["r_keys"], d["r_pays"], d["s_keys"], d["s_pays"], materialize=mat)
+    for r in res:
+        assert r["status"] == 0
+        assert (r["match_count"], r["checksum"], r["pair_digest"]) == (ref["count"], ref["checksum"], ref["pair_digest"])
+    if mat:
+        trip = [j.materialized(r) for j, r in zip(joins, res)]
+        k, a, b = sort_trip(*(np.concatenate([t[i] for t in trip]) for i in range(3)))
+        np.testing.assert_array_equal(k, ref["key"])
+        np.testing.assert_array_equal(a, ref["pay_r"])
+        np.testing.assert_array_equal(b, ref["pay_s"])
+    # the receive buffers hold 32-byte units of at most five tuples, at least one each (at this
+    # size most (tile, partition) runs are a few tuples, so units are far from full; M2: below)
+    tot_units = sum(r["recv_r"] + r["recv_s"] for r in res)
+    assert (w.n_r + w.n_s) / 5 <= tot_units <= w.n_r + w.n_s
+    for j in joins:
+        j.close()
+
+
+def test_compress_rejects_non_id_payloads(mgj):
+    """The compressed shuffle rebuilds payloads from row ids; a payload that is
+    not its global row id fails the run with MGJ_EINVAL instead of a wrong join."""
+    n = 1 << 16
+    d = datagen.Workload("unique", n, n).rank_inputs()
+    d["s_pays"] = d["s_pays"].copy()
+    d["s_pays"][12345] += np.uint32(1)
+    cfg = mgj.make_config(r_capacity=n, s_capacity=n, compress=True)
+    j = mgj.Join(cfg)
+    j.partition(*[dev(d[k]) for k in ("r_keys", "r_pays", "s_keys", "s_pays")])
+    j.shuffle()
+    j.join()
+    assert j.result(check=False)["status"] == -1
+    j.close()
+
+
+@pytest.mark.slow
+def test_compress_full_size_m2(mgj):
+    """M2 at one GPU (2^29 x 2^29) through the compressed shuffle: closed-form
+    count and checksum, pair digest by device inverse permutation."""
+    n = 1 << 29
+    cols = [torch.empty(n, dtype=torch.int32, device="cuda") for _ in range(4)]
+    mgj.gen_relation("unique", 0, n, n, 0.0, 0, n, cols[0], cols[1])
+    mgj.gen_relation("unique", 1, n, n, 0.0, 0, n, cols[2], cols[3])
+    j = mgj.Join(mgj.make_config(r_capacity=n, s_capacity=n, compress=True))
+    res = j.run(*cols)
+    assert res["match_count"] == n
+    assert res["checksum"] == 0xf1fffffff0000000
+    assert res["pair_digest"] == _device_pair_digest_unique(cols[0], cols[2], cols[3], n)
+    assert (res["recv_r"] + res["recv_s"]) * 32 < 6.5 * 2 * n  # bytes in the receive buffers
+    j.close()

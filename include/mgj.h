@@ -97,7 +97,13 @@ typedef struct {
                                           its row's offset in its source tile, five per 32-byte unit
                                           (+ source rank, tile, count): 6.4 instead of 8 bytes.  Forces a
                                           single local pass */
-    int32_t  reserved[2];              /* must be zero */
+    int32_t  assign;                   /* a2 partition assignment: 0 = contiguous ranges balanced on counts
+                                          (the optimum for random placement on a uniform one-hop fabric);
+                                          1 = placement-aware (NEXT-2, the migration step of Track-Join
+                                          the paper adopts): each partition goes to the rank
+                                          holding most of its tuples unless that rank's load would pass
+                                          9/8 of the mean.  MGJ_SHUFFLE_P2P only */
+    int32_t  reserved[1];              /* must be zero */
 } mgj_config;
 
 /*
@@ -225,7 +231,8 @@ const char *mgj_strerror(mgj_status s);
 mgj_status mgj_plan_host(int32_t world_size, int32_t rank, int32_t bits,
                          const uint32_t *hist, int32_t *owner,
                          uint64_t *send_off, uint64_t *recv_size,
-                         int32_t skew_bcast, uint8_t *bcast, uint8_t *skip);
+                         int32_t skew_bcast, uint8_t *bcast, uint8_t *skip,
+                         int32_t assign);
 
 #ifdef __cplusplus
 }

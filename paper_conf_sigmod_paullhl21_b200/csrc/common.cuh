@@ -103,6 +103,7 @@ struct Ctx {
     int32_t materialize;
     int32_t ext;                  // shuffle mode EXTERNAL: scatter into send_buf, caller exchanges
     int32_t comp;                 // NEXT-1 compressed shuffle (units of CU_N entries, see scatter.cuh)
+    int32_t assign;               // NEXT-2 placement-aware partition assignment (k_plan)
     int32_t chunk_units;          // compress: local-pass chunk in units
     uint32_t *rowbase;            // compress: [2][MAX_RANKS][G] global row id of each (rank, tile)'s first row
     uint32_t *rank_units;         // compress: [2][P] this rank's 32-byte units per partition

@@ -278,6 +278,28 @@ __host__ __device__ inline bool bcast_of(uint64_t r, uint64_t s, uint64_t s_tota
 // shuffled, partitioned or probed.  P2P shuffle only.
 __host__ __device__ inline bool skip_of(uint64_t r, uint64_t s) { return (r == 0) != (s == 0); }
 
+// Placement-aware assignment (NEXT-2, Track-Join migration): partitions in
+// order go to their preferred rank (the one holding most of their tuples)
+// unless its assigned weight would pass cap = 9/8 of the mean, then to the
+// least-loaded rank.  Shared by k_plan (thread 0) and mgj_plan_host.
+template <typename WF, typename BF>
+__host__ __device__ inline void assign_greedy(int N, int P, WF weight, BF pref, int32_t *owner) {
+    uint64_t load[MAX_RANKS] = {}, total = 0;
+    for (int p = 0; p < P; ++p) total += weight(p);
+    const uint64_t cap = total / (uint64_t)N + total / (8ull * (uint64_t)N) + 1;
+    for (int p = 0; p < P; ++p) {
+        const uint64_t w = weight(p);
+        int d = pref(p);
+        if (w && load[d] + w > cap) {
+            d = 0;
+            for (int g = 1; g < N; ++g)
+                if (load[g] < load[d]) d = g;
+        }
+        owner[p] = d;
+        load[d] += w;
+    }
+}
+
 // Weight of p in the owner ranges: a broadcast partition's S stays spread
 // over the ranks, its owner (the root, which receives R_p) gets R_p + S_p/N.
 __host__ __device__ inline uint64_t owner_weight(uint64_t r, uint64_t s, bool bc, int N) {
@@ -458,19 +480,95 @@ __global__ void __launch_bounds__(1024) k_plan(Ctx c) {
         // in a region of recv_cap tuples
         if (c.ext && d == 0 && c.n_in[rel] > c.recv_cap[rel]) atomicOr(&cap_bad, 1);
     }
-    const int plo = first[c.rank] < P ? first[c.rank] : 0;
-    const int phi = first[c.rank] < P ? endp[c.rank] : 0;
+    int plo = first[c.rank] < P ? first[c.rank] : 0;
+    int phi = first[c.rank] < P ? endp[c.rank] : 0;
     __syncthreads();
     // owned list: the range, then the broadcast partitions outside it (ascending)
     for (int p = tid; p < P; p += blockDim.x) chn[p] = (bcf[p] && (p < plo || p >= phi)) ? 1u : 0u;
     __syncthreads();
     const int nout = (int)block_excl_scan_u32(chn, P, tmp32);
-    const int nr = phi - plo, np = nr + nout;
+    int nr = phi - plo, np = nr + nout;
     for (int p = tid; p < P; p += blockDim.x) {
         if (p >= plo && p < phi) c.plist[p - plo] = p;
         else if (bcf[p]) c.plist[nr + chn[p]] = p;
     }
     __syncthreads();
+    if (c.assign) {
+        // Placement-aware assignment (NEXT-2; the paper's migration step after
+        // Track-Join [34]): with uniform one-hop costs a partition's
+        // cheapest single destination is the rank that already holds most of
+        // its tuples (of R for a broadcast partition, whose S stays spread), so
+        // it moves there unless that rank's assigned weight would pass 9/8 of
+        // the mean, then to the least-loaded rank (thread 0, partitions in
+        // order: deterministic, the same on every rank; host mirror
+        // mgj_plan_host).  Owners are no longer contiguous ranges: the layout
+        // of rank d is its partitions ascending (one block scan per rank and
+        // relation), then, for S, its own tuples of broadcast partitions.
+        uint8_t *best = reinterpret_cast<uint8_t *>(ut1 + P);  // [P] (after the unit totals)
+        for (int p = tid; p < P; p += blockDim.x) {
+            int b = 0;
+            uint64_t hb = 0;
+            for (int g = 0; g < N; ++g) {
+                const uint64_t h = (uint64_t)H(g, 0, p) + (bcf[p] ? 0u : H(g, 1, p));
+                if (h > hb) hb = h, b = g;
+            }
+            best[p] = (uint8_t)b;
+        }
+        __syncthreads();
+        if (tid == 0) assign_greedy(N, P, [&](int p) { return owner_weight(tot0[p], tot1[p], bcf[p], N); },
+                                    [&](int p) { return (int)best[p]; }, own);
+        __syncthreads();
+        for (int p = tid; p < P; p += blockDim.x) c.owner[p] = own[p];
+        __shared__ unsigned long long rsum[2][MAX_RANKS];
+        for (int rel = 0; rel < 2; ++rel)
+            for (int d = 0; d < N; ++d) {
+                for (int p = tid; p < P; p += blockDim.x)
+                    cum[p] = (own[p] == d && !(rel && bcf[p])) ? LT(rel, p) : 0;
+                __syncthreads();
+                const uint64_t tot_d = block_excl_scan_u64(cum, P, tmp);
+                for (int p = tid; p < P; p += blockDim.x) {
+                    if (own[p] != d || (rel && bcf[p])) continue;
+                    uint64_t m = 0;  // this rank's tuples of p go after those of lower ranks
+                    for (int g = 0; g < c.rank; ++g) m += HL(g, rel, p);
+                    c.send_off[rel * P + p] = cum[p] + m;
+                    if (rel == 0 || d == c.rank) c.seg_start[rel * P + p] = cum[p];
+                }
+                if (tid == 0) rsum[rel][d] = tot_d;
+                __syncthreads();
+            }
+        // S of broadcast partitions: this rank's own tuples, after its assigned part
+        for (int p = tid; p < P; p += blockDim.x) cum[p] = bcf[p] ? HL(c.rank, 1, p) : 0u;
+        __syncthreads();
+        block_excl_scan_u64(cum, P, tmp);
+        for (int p = tid; p < P; p += blockDim.x)
+            if (bcf[p]) c.send_off[P + p] = c.seg_start[P + p] = rsum[1][c.rank] + cum[p];
+        __syncthreads();
+        if (tid == 0) {
+            cap_bad &= ~1;
+            for (int d = 0; d < N; ++d)
+                for (int rel = 0; rel < 2; ++rel) {
+                    const uint64_t size = rsum[rel][d] + (rel ? bcs[d] : 0);
+                    c.recv_size[rel * MAX_RANKS + d] = size;
+                    if (size > (c.comp ? c.recv_cap_u[rel] : c.recv_cap[rel])) cap_bad |= 1;
+                }
+        }
+        // owned list: the partitions assigned here, then the broadcast ones rooted elsewhere
+        __syncthreads();
+        for (int p = tid; p < P; p += blockDim.x) chn[p] = own[p] == c.rank ? 1u : 0u;
+        __syncthreads();
+        const int nmine = (int)block_excl_scan_u32(chn, P, tmp32);
+        for (int p = tid; p < P; p += blockDim.x)
+            if (own[p] == c.rank) c.plist[chn[p]] = p;
+        __syncthreads();
+        for (int p = tid; p < P; p += blockDim.x) chn[p] = (bcf[p] && own[p] != c.rank) ? 1u : 0u;
+        __syncthreads();
+        const int nb = (int)block_excl_scan_u32(chn, P, tmp32);
+        for (int p = tid; p < P; p += blockDim.x)
+            if (bcf[p] && own[p] != c.rank) c.plist[nmine + chn[p]] = p;
+        plo = phi = nr = 0;
+        np = nmine + nb;
+        __syncthreads();
+    }
     // per owned partition: R and S sizes of its received pieces
     auto own_p = [&](int i) -> int { return i < nr ? plo + i : c.plist[i]; };
     auto own_len = [&](int rel, int p) -> uint64_t { return rel ? (bcf[p] ? (uint64_t)H(c.rank, 1, p) : tot1[p]) : tot0[p]; };  // 0 if skipped

@@ -43,8 +43,10 @@ int ceil_log2(uint64_t x) {
 mgj_status normalize(const mgj_config *in, Norm *o) {
     if (!in) return MGJ_EINVAL;
     mgj_config c = *in;
-    for (int i = 0; i < 2; ++i)
+    for (int i = 0; i < 1; ++i)
         if (c.reserved[i]) return MGJ_EINVAL;
+    if (c.assign != 0 && c.assign != 1) return MGJ_EINVAL;
+    if (c.assign && c.shuffle_mode != MGJ_SHUFFLE_P2P) return MGJ_EINVAL;  // EXTERNAL needs contiguous owners
     if (c.peer_timeout_ms < 0) return MGJ_EINVAL;
     if (c.shuffle_overlap < -1 || c.shuffle_overlap > 1 || c.overlap_local_sms < 0) return MGJ_EINVAL;
     if (c.trace != 0 && c.trace != 1) return MGJ_EINVAL;
@@ -211,7 +213,8 @@ size_t hist_smem(const Norm &n) {
     return (size_t)hist_nb(T, n.c.key_bytes) * T * n.c.key_bytes + (size_t)n.P * 8;
 }
 size_t plan_smem(const Norm &n) {
-    return (size_t)n.P * 5 * 8 + (size_t)n.P * 4 + (size_t)(n.P + 1) * 4 + (size_t)n.P + 8 + (size_t)n.P * 2 * 8;
+    return (size_t)n.P * 5 * 8 + (size_t)n.P * 4 + (size_t)(n.P + 1) * 4 + (size_t)n.P + 8 + (size_t)n.P * 2 * 8 +
+           (size_t)n.P;  // ... unit totals, preferred ranks
 }
 size_t scatter_smem(const Norm &n) { return scatter_smem_bytes(n.P, n.c.key_bytes); }
 size_t planA_smem(const Norm &n) { return ((size_t)local2_vcap(n.P) + 1) * 12; }
@@ -431,6 +434,7 @@ mgj_status mgj_plan(const mgj_config *cfg, const mgj_peers *peers, mgj_handle *o
     c.timeout_ns = (n.c.peer_timeout_ms ? (uint64_t)n.c.peer_timeout_ms : 20000ull) * 1000000ull;
     c.ext = n.c.shuffle_mode == MGJ_SHUFFLE_EXTERNAL;
     c.comp = n.c.compress;
+    c.assign = n.c.assign;
     c.chunk_units = CHUNK_UNITS;
     c.max_items = (uint32_t)n.max_items;
     c.recv_cap[0] = n.recv_cap[0];
@@ -693,9 +697,9 @@ void mgj_destroy(mgj_handle h) {
 
 mgj_status mgj_plan_host(int32_t world_size, int32_t rank, int32_t bits, const uint32_t *hist, int32_t *owner,
                          uint64_t *send_off, uint64_t *recv_size, int32_t skew_bcast, uint8_t *bcast,
-                         uint8_t *skip) {
+                         uint8_t *skip, int32_t assign) {
     if (world_size < 1 || world_size > MAX_RANKS || rank < 0 || rank >= world_size || bits < 1 || bits > MAX_B1 ||
-        !hist || !owner || !send_off || !recv_size || skew_bcast < -1 || skew_bcast > 1)
+        !hist || !owner || !send_off || !recv_size || skew_bcast < -1 || skew_bcast > 1 || assign < 0 || assign > 1)
         return MGJ_EINVAL;
     const int P = 1 << bits, N = world_size;
     auto H = [&](int g, int rel, int p) -> uint64_t { return hist[((size_t)g * 2 + rel) * P + p]; };
@@ -729,6 +733,46 @@ mgj_status mgj_plan_host(int32_t world_size, int32_t rank, int32_t bits, const u
         run[0] += tot[p];
         pre[P + p] = run[1];
         run[1] += bc[p] ? 0 : tot[P + p];
+    }
+    if (assign) {  // placement-aware (k_plan's assign branch, same formulas)
+        assign_greedy(
+            N, P, [&](int p) { return owner_weight(tot[p], tot[P + p], bc[p], N); },
+            [&](int p) {
+                int b = 0;
+                uint64_t hb = 0;
+                for (int g = 0; g < N; ++g) {
+                    const uint64_t h = H(g, 0, p) + (bc[p] ? 0 : H(g, 1, p));
+                    if (h > hb) hb = h, b = g;
+                }
+                return b;
+            },
+            owner);
+        uint64_t run[2][MAX_RANKS] = {};
+        for (int p = 0; p < P; ++p)
+            for (int rel = 0; rel < 2; ++rel) {
+                if (rel && bc[p]) continue;
+                uint64_t m = 0;
+                for (int g = 0; g < rank; ++g) m += H(g, rel, p);
+                send_off[rel * P + p] = run[rel][owner[p]] + m;
+                run[rel][owner[p]] += tot[rel * P + p];
+            }
+        uint64_t own_bc = 0;
+        for (int p = 0; p < P; ++p)
+            if (bc[p]) {
+                send_off[P + p] = run[1][rank] + own_bc;
+                own_bc += H(rank, 1, p);
+            }
+        for (int rel = 0; rel < 2; ++rel)
+            for (int d = 0; d < N; ++d) {
+                uint64_t sz = run[rel][d];
+                if (rel)
+                    for (int p = 0; p < P; ++p) sz += bc[p] ? H(d, 1, p) : 0;
+                recv_size[rel * N + d] = sz;
+            }
+        delete[] tot;
+        delete[] pre;
+        delete[] bc;
+        return MGJ_OK;
     }
     uint64_t cum = 0;
     int first[MAX_RANKS], endp[MAX_RANKS];

@@ -54,7 +54,7 @@ class Config(ctypes.Structure):
                 ("local_split_bits", ctypes.c_int32), ("skew_bcast", ctypes.c_int32),
                 ("peer_timeout_ms", ctypes.c_int32), ("shuffle_overlap", ctypes.c_int32),
                 ("overlap_local_sms", ctypes.c_int32), ("trace", ctypes.c_int32),
-                ("compress", ctypes.c_int32), ("reserved", ctypes.c_int32 * 2)]
+                ("compress", ctypes.c_int32), ("assign", ctypes.c_int32), ("reserved", ctypes.c_int32 * 1)]
 
 
 class Exchange(ctypes.Structure):
@@ -100,7 +100,8 @@ _lib.mgj_result.argtypes = [_H, ctypes.POINTER(Result)]
 _lib.mgj_destroy.restype = None
 _lib.mgj_destroy.argtypes = [_H]
 _lib.mgj_plan_host.restype = ctypes.c_int
-_lib.mgj_plan_host.argtypes = [ctypes.c_int32, ctypes.c_int32, ctypes.c_int32, _P, _P, _P, _P, ctypes.c_int32, _P, _P]
+_lib.mgj_plan_host.argtypes = [ctypes.c_int32, ctypes.c_int32, ctypes.c_int32, _P, _P, _P, _P, ctypes.c_int32, _P, _P,
+                               ctypes.c_int32]
 _lib.mgj_gen_relation.restype = ctypes.c_int
 _lib.mgj_gen_relation.argtypes = [ctypes.c_int32, ctypes.c_int32, _U64, _U64, ctypes.c_double,
                                   _U64, _U64, _P, _P, _P]
@@ -139,7 +140,8 @@ def _stream(stream):
 def make_config(rank=0, world_size=1, key_bytes=4, r_capacity=0, s_capacity=0, recv_capacity_r=0,
                 recv_capacity_s=0, radix_bits_global=0, radix_bits_local=0, materialize=False,
                 num_sms=0, out_capacity=0, shuffle_mode=0, local_split_bits=0, skew_bcast=0,
-                peer_timeout_ms=0, shuffle_overlap=0, overlap_local_sms=0, trace=False, compress=False) -> Config:
+                peer_timeout_ms=0, shuffle_overlap=0, overlap_local_sms=0, trace=False, compress=False,
+                assign=0) -> Config:
     c = Config()
     c.rank, c.world_size = rank, world_size
     c.key_bytes = c.payload_bytes = key_bytes
@@ -157,6 +159,7 @@ def make_config(rank=0, world_size=1, key_bytes=4, r_capacity=0, s_capacity=0, r
     c.overlap_local_sms = overlap_local_sms
     c.trace = int(bool(trace))
     c.compress = int(bool(compress))
+    c.assign = assign
     return c
 
 
@@ -317,7 +320,8 @@ def device_bytes(ptr: int, nbytes: int):
     return torch.as_tensor(_DevBuf(ptr, nbytes), device="cuda")
 
 
-def plan_host(world: int, rank: int, bits: int, hist: np.ndarray, skew_bcast: int = 0, with_bcast: bool = False):
+def plan_host(world: int, rank: int, bits: int, hist: np.ndarray, skew_bcast: int = 0, with_bcast: bool = False,
+              assign: int = 0):
     """Host reference of the a2 assignment (mgj_plan_host): owner, send offsets, receive sizes
     (and, with with_bcast=True, the selective-broadcast flags and the empty-side skip flags)."""
     P = 1 << bits
@@ -328,7 +332,8 @@ def plan_host(world: int, rank: int, bits: int, hist: np.ndarray, skew_bcast: in
     bcast = np.empty(P, np.uint8)
     skip = np.empty(P, np.uint8)
     _check(_lib.mgj_plan_host(world, rank, bits, hist.ctypes.data, owner.ctypes.data, send_off.ctypes.data,
-                              recv_size.ctypes.data, skew_bcast, bcast.ctypes.data, skip.ctypes.data), "mgj_plan_host")
+                              recv_size.ctypes.data, skew_bcast, bcast.ctypes.data, skip.ctypes.data, assign),
+           "mgj_plan_host")
     return (owner, send_off, recv_size, bcast, skip) if with_bcast else (owner, send_off, recv_size)
 
 

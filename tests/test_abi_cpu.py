@@ -50,7 +50,7 @@ def test_strerror(mgj):
                                  dict(skew_bcast=-2), dict(peer_timeout_ms=-1), dict(shuffle_overlap=2),
                                  dict(shuffle_overlap=-2), dict(overlap_local_sms=-1),
                                  dict(compress=1, key_bytes=8), dict(compress=1, shuffle_mode=1),
-                                 dict(compress=1, radix_bits_global=11)])
+                                 dict(compress=1, radix_bits_global=11), dict(assign=2), dict(assign=1, shuffle_mode=1)])
 def test_invalid_config_rejected_without_gpu(mgj, bad):
     kw = dict(r_capacity=1024, s_capacity=1024)
     kw.update(bad)
@@ -79,14 +79,14 @@ def test_arena_layout_size(mgj):
     assert 2 * 8 * (1 << 20) <= nb <= 2 * 8 * (1 << 20) + (1 << 20)
 
 
-def check_plan_invariants(mgj, hist, bits, skew_bcast=0):
+def check_plan_invariants(mgj, hist, bits, skew_bcast=0, assign=0):
     """Every rank computes the same plan; for each destination d and relation, the
     (source rank, partition) ranges the plan sends to d tile [0, recv_size[d]) exactly.
     A selectively broadcast partition (NEXT-2) sends R to its owner (the root) and
     keeps each rank's S at that rank."""
     N = hist.shape[0]
     P = 1 << bits
-    plans = [mgj.plan_host(N, g, bits, hist, skew_bcast=skew_bcast, with_bcast=True) for g in range(N)]
+    plans = [mgj.plan_host(N, g, bits, hist, skew_bcast=skew_bcast, with_bcast=True, assign=assign) for g in range(N)]
     owner, recv, bc, skip = plans[0][0], plans[0][2], plans[0][3], plans[0][4]
     for o, _, rs, b, sk in plans:  # every rank computes the same assignment
         assert np.array_equal(o, owner) and np.array_equal(rs, recv) and np.array_equal(b, bc)
@@ -95,7 +95,9 @@ def check_plan_invariants(mgj, hist, bits, skew_bcast=0):
     # the histogram as a Bloom filter: exactly the partitions with one empty side
     np.testing.assert_array_equal(skip != 0, (tot[0] == 0) != (tot[1] == 0))
     assert not (bc.astype(bool) & skip.astype(bool)).any()
-    assert np.all(np.diff(owner) >= 0) and owner.min() >= 0 and owner.max() < N
+    assert owner.min() >= 0 and owner.max() < N
+    if not assign:  # contiguous ranges
+        assert np.all(np.diff(owner) >= 0)
     if N == 1 or skew_bcast < 0:
         assert not bc.any()
     for rel in range(2):
@@ -179,3 +181,20 @@ def test_plan_host_all_empty(mgj):
     hist = np.zeros((4, 2, 1 << 5), np.uint32)
     owner, recv, _, _ = check_plan_invariants(mgj, hist, 5)
     assert np.array_equal(owner, np.arange(32) * 4 // 32)
+
+
+@pytest.mark.parametrize("N", [2, 3, 5, 8])
+def test_plan_host_placement_aware(mgj, N):
+    """assign = 1: the same tiling invariants with non-contiguous owners; a partition
+    whose tuples mostly sit on one rank is assigned there while loads allow."""
+    rng = np.random.default_rng(10 + N)
+    bits = 6
+    P = 1 << bits
+    hist = rng.integers(0, 20, size=(N, 2, P)).astype(np.uint32)
+    for p in range(P):  # partition p lives mostly on rank p % N
+        hist[p % N, :, p] += 200
+    owner, recv, bc, skip = check_plan_invariants(mgj, hist, bits, assign=1)
+    assert np.mean(owner == np.arange(P) % N) > 0.9
+    check_plan_invariants(mgj, hist, bits, assign=1, skew_bcast=1)
+    load = recv.sum(axis=0)
+    assert load.max() <= load.mean() * 9 / 8 + hist.sum(axis=(0, 1)).max()

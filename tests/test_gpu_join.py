@@ -1071,3 +1071,74 @@ def test_compress_full_size_m2(mgj):
     assert res["pair_digest"] == _device_pair_digest_unique(cols[0], cols[2], cols[3], n)
     assert (res["recv_r"] + res["recv_s"]) * 32 < 6.5 * 2 * n  # bytes in the receive buffers
     j.close()
+
+
+# ------------------------------------------------------------ NEXT-2: placement-aware assignment
+class PlacedWorkload:
+    """Global R and S (unique keys, ids) whose tuples sit on rank key % N with
+    probability `alpha`, on a random rank otherwise (placement skew)."""
+
+    def __init__(self, n, N, alpha, seed=5):
+        w = datagen.Workload("unique", n, n)
+        self.a = w.rank_inputs()
+        self.n_r = self.n_s = n
+        self.key_bytes = 4
+        rng = np.random.default_rng(seed)
+        self.where = {}
+        for rel in ("r", "s"):
+            k = self.a[rel + "_keys"]
+            pref = (k % N).astype(np.int64)
+            rnd = rng.integers(0, N, k.size)
+            self.where[rel] = np.where(rng.random(k.size) < alpha, pref, rnd)
+
+    def rank_inputs(self, rank=0, world=1):
+        if world == 1:
+            return dict(self.a)
+        out = {}
+        for rel in ("r", "s"):
+            m = self.where[rel] == rank
+            out[rel + "_keys"] = self.a[rel + "_keys"][m].copy()
+            out[rel + "_pays"] = self.a[rel + "_pays"][m].copy()
+        return out
+
+
+def _moved_tuples(owner, mail):
+    """Tuples that leave their rank under owner[] (mail: [N][2][P] histograms)."""
+    N = mail.shape[0]
+    return int(sum(mail[g, :, owner != g].sum() for g in range(N)))
+
+
+@pytest.mark.parametrize("N", [2, 4])
+def test_placement_aware_assignment(mgj, N):
+    """assign = 1 (Track-Join migration): partitions go where most
+    of their tuples already are.  Exact vs the oracle either way; the device
+    plan equals the host plan; with placement skew (80% of each partition's
+    tuples on one rank) far fewer tuples cross ranks than with ranges."""
+    w = PlacedWorkload(1 << 18, N, 0.8)
+    d = w.rank_inputs()
+    ref = oracle.join(d["r_keys"], d["r_pays"], d["s_keys"], d["s_pays"], materialize=True)
+    moved = {}
+    for assign in (0, 1):
+        joins, res, _ = run_virtual(mgj, w, N, materialize=True, assign=assign, radix_bits_global=8)
+        for r in res:
+            assert r["status"] == 0
+            assert (r["match_count"], r["checksum"], r["pair_digest"]) == (ref["count"], ref["checksum"], ref["pair_digest"])
+        trip = [j.materialized(r) for j, r in zip(joins, res)]
+        k, a, b = sort_trip(*(np.concatenate([t[i] for t in trip]) for i in range(3)))
+        np.testing.assert_array_equal(k, ref["key"])
+        np.testing.assert_array_equal(b, ref["pay_s"])
+        P = 1 << 8
+        mail = joins[0].debug("MAIL_HIST", np.uint32).reshape(N, 2, P)
+        owner = joins[0].debug("OWNER", np.int32)
+        for g, j in enumerate(joins):
+            o, send_off, recv_size = mgj.plan_host(N, g, 8, mail, assign=assign)
+            np.testing.assert_array_equal(j.debug("OWNER", np.int32), o)
+            np.testing.assert_array_equal(j.debug("SEND_OFF", np.uint64).reshape(2, P), send_off)
+            assert res[g]["recv_r"] == recv_size[0, g] and res[g]["recv_s"] == recv_size[1, g]
+        moved[assign] = _moved_tuples(owner, mail.astype(np.int64))
+        if assign:  # the receive load stays within 9/8 of the mean (+ one partition)
+            load = np.array([r["recv_r"] + r["recv_s"] for r in res])
+            assert load.max() <= load.mean() * 9 / 8 + 2 * (w.n_r + w.n_s) / P
+        for j in joins:
+            j.close()
+    assert moved[1] < 0.5 * moved[0], moved

@@ -26,7 +26,7 @@ def _free_port():
     return p
 
 
-def _worker(rank, world, port, bits, kind, skew, q):
+def _worker(rank, world, port, bits, kind, skew, q, assign=0):
     import sys
     sys.path.insert(0, ROOT)
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
@@ -42,7 +42,8 @@ def _worker(rank, world, port, bits, kind, skew, q):
         allh = [torch.zeros(2, P, dtype=torch.int64) for _ in range(world)]
         dist.all_gather(allh, torch.from_numpy(hist))
         H = np.stack([h.numpy() for h in allh]).astype(np.uint32)
-        owner, send_off, recv_size, bc, skip = mgj.plan_host(world, rank, bits, H, skew_bcast=skew, with_bcast=True)
+        owner, send_off, recv_size, bc, skip = mgj.plan_host(world, rank, bits, H, skew_bcast=skew, with_bcast=True,
+                                                             assign=assign)
         if skew < 0:
             assert not bc.any()
         out = {}
@@ -94,16 +95,17 @@ def _worker(rank, world, port, bits, kind, skew, q):
         dist.destroy_process_group()
 
 
-@pytest.mark.parametrize("world,bits,kind,skew", [(2, 8, "unique", 0), (4, 6, "unique", 0), (2, 7, "zipf", -1),
-                                                  (2, 7, "zipf", 0), (4, 7, "zipf", 1)])
-def test_gloo_partitioned_join(world, bits, kind, skew):
+@pytest.mark.parametrize("world,bits,kind,skew,assign", [(2, 8, "unique", 0, 0), (4, 6, "unique", 0, 0),
+                                                         (2, 7, "zipf", -1, 0), (2, 7, "zipf", 0, 0), (4, 7, "zipf", 1, 0),
+                                                         (3, 6, "unique", 0, 1), (4, 7, "zipf", 1, 1)])
+def test_gloo_partitioned_join(world, bits, kind, skew, assign):
     """skew: mgj_config.skew_bcast (selective broadcast of heavy S partitions, NEXT-2)."""
     import __graft_entry__
     __graft_entry__.build()
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    procs = [ctx.Process(target=_worker, args=(r, world, port, bits, kind, skew, q)) for r in range(world)]
+    procs = [ctx.Process(target=_worker, args=(r, world, port, bits, kind, skew, q, assign)) for r in range(world)]
     for p in procs:
         p.start()
     for p in procs:

@@ -57,6 +57,10 @@ def parse():
                     help="§8(e): R's local pass beside S's scatter (auto: on for N > 1 with the P2P shuffle)")
     ap.add_argument("--overlap-local-sms", type=int, default=0)
     ap.add_argument("--trace", action="store_true", help="kernel timeline of the last step in the JSON line")
+    ap.add_argument("--placement-z", type=float, default=0.0,
+                    help="N>1: rank g holds a 1/(g+1)^z share of the rows (Fig. 9's placement-skew reading)")
+    ap.add_argument("--assign", type=int, default=0, choices=[0, 1],
+                    help="a2 assignment: 0 contiguous ranges, 1 placement-aware (Track-Join migration)")
     ap.add_argument("--compress", action="store_true",
                     help="NEXT-1 compressed shuffle (4-byte keys, id payloads): 32-byte units of five entries")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -285,8 +289,9 @@ def main():
         n_r, n_s = world * per // 4, world * per  # |R|:|S| = 1:4
     else:
         n_r = n_s = world * per
-    r_lo, r_hi = n_r * rank // world, n_r * (rank + 1) // world
-    s_lo, s_hi = n_s * rank // world, n_s * (rank + 1) // world
+    from paper_conf_sigmod_paullhl21_b200 import datagen as _dg
+    r_lo, r_hi = _dg.shard_bounds(n_r, rank, world, a.placement_z)
+    s_lo, s_hi = _dg.shard_bounds(n_s, rank, world, a.placement_z)
     nr, ns = r_hi - r_lo, s_hi - s_lo
     cols = [torch.empty(x, dtype=dt, device=dev) for x in (nr, nr, ns, ns)]
     with torch.cuda.stream(stream):
@@ -297,12 +302,16 @@ def main():
     cfg = mgj.make_config(rank=rank, world_size=world, key_bytes=kb, r_capacity=nr, s_capacity=ns,
                           materialize=a.materialize, radix_bits_global=a.radix_bits_global,
                           radix_bits_local=a.radix_bits_local, local_split_bits=a.local_split_bits,
-                          recv_capacity_r=(n_r if world > 1 and a.workload == "zipf" else 0),
-                          recv_capacity_s=(n_s // 2 if world > 1 and a.workload == "zipf" else 0),
+                          # job-wide receive capacities (identical on every rank): skewed keys or
+                          # placement can concentrate a relation on one rank
+                          recv_capacity_r=(n_r if world > 1 and (a.workload == "zipf" or a.placement_z) else 0),
+                          recv_capacity_s=(n_s // 2 if world > 1 and a.workload == "zipf" and not a.placement_z
+                                           else (n_s if world > 1 and a.placement_z else 0)),
                           shuffle_mode=(mgj.SHUFFLE_EXTERNAL if a.shuffle == "nccl" else mgj.SHUFFLE_P2P),
                           skew_bcast=a.skew_bcast, num_sms=a.num_sms,
                           shuffle_overlap={"auto": 0, "on": 1, "off": -1}[a.overlap],
-                          overlap_local_sms=a.overlap_local_sms, trace=a.trace, compress=a.compress)
+                          overlap_local_sms=a.overlap_local_sms, trace=a.trace, compress=a.compress,
+                          assign=a.assign)
     # N>1 (or MGJ_SYMM_ARENA=1): the library's symmetric-memory setup (mgj.symmetric_join)
     join = mgj.symmetric_join(cfg) if distributed else mgj.Join(cfg)
 

@@ -135,6 +135,20 @@ def zipf_ranks(rows: np.ndarray, n: int, z: float, seed: int = SEED_Z) -> np.nda
     return r.astype(np.uint64)
 
 
+def shard_bounds(n: int, rank: int, world: int, placement_z: float = 0.0) -> tuple[int, int]:
+    """Rows [lo, hi) of `rank` among `world` contiguous slices of n rows; with
+    placement_z > 0 slice g holds a share 1/(g+1)^z / sum_h 1/(h+1)^z (exact
+    integer boundaries from the cumulative weights)."""
+    if placement_z == 0.0:
+        return (n * rank) // world, (n * (rank + 1)) // world
+    w = [1.0 / (g + 1) ** placement_z for g in range(world)]
+    tot = sum(w)
+    cum = [0]
+    for g in range(world):
+        cum.append(n if g == world - 1 else int(n * (sum(w[:g + 1]) / tot)))
+    return cum[rank], cum[rank + 1]
+
+
 @dataclasses.dataclass(frozen=True)
 class Workload:
     """A synthetic join input.
@@ -151,6 +165,7 @@ class Workload:
     n_r: int
     n_s: int
     z: float = 0.0
+    placement_z: float = 0.0  # rank shares of the rows ~ 1/(g+1)^placement_z (0: equal shares)
 
     @property
     def key_bytes(self) -> int:
@@ -161,8 +176,10 @@ class Workload:
         return self.key_bytes
 
     def shard(self, n: int, rank: int, world: int) -> tuple[int, int]:
-        """Rows [lo, hi) held by `rank` (contiguous slices)."""
-        return (n * rank) // world, (n * (rank + 1)) // world
+        """Rows [lo, hi) held by `rank` (contiguous slices).  With
+        placement_z > 0 the slices follow a Zipf law over the ranks (rank g's share
+        proportional to 1/(g+1)^z: the placement-skew reading of Fig. 9)."""
+        return shard_bounds(n, rank, world, self.placement_z)
 
     def relation(self, rel: str, lo: int, hi: int) -> tuple[np.ndarray, np.ndarray]:
         rows = np.arange(lo, hi, dtype=_U64)

@@ -86,3 +86,17 @@ def test_torch_inverses_match_numpy(k):
     z = datagen.mix64(x)
     got = datagen.unmix64_t(torch.from_numpy(z.view(np.int64))).numpy().view(np.uint64)
     np.testing.assert_array_equal(got, x)
+
+
+@pytest.mark.parametrize("world,z", [(1, 1.0), (4, 0.0), (4, 1.0), (8, 0.5)])
+def test_placement_shards_tile_rows(world, z):
+    """Placement-skewed shards (Fig. 9 reading) still tile [0, n) in rank order, rank 0 largest."""
+    n = 1000003
+    b = [datagen.shard_bounds(n, g, world, z) for g in range(world)]
+    assert b[0][0] == 0 and b[-1][1] == n
+    assert all(b[g][1] == b[g + 1][0] for g in range(world - 1))
+    sizes = [hi - lo for lo, hi in b]
+    assert sizes == sorted(sizes, reverse=True) or z == 0.0
+    w = datagen.Workload("unique", n, n, placement_z=z)
+    d = w.rank_inputs(world - 1, world)
+    assert d["r_keys"].size == sizes[-1] and int(d["r_pays"][0]) == b[-1][0]

@@ -8,7 +8,9 @@ pieces), counts digit1 with torch.bincount, and runs the library's host plan
 roots), and the cross-rank tuples the shuffle moves.  These are exact counts of
 the plan, not timings (one GPU here: N > 1 cannot be timed).
 
-usage: python tools/skew_plan.py [--z 1.0] [--gpus 8] [--bits 10] > out.json
+usage: python tools/skew_plan.py [--workload zipf|unique] [--z 1.0] [--placement-z 0] [--gpus 8] [--bits 10] > out.json
+(--placement-z: rank g holds a 1/(g+1)^z share of the rows, Fig. 9's placement reading;
+modes: ranges with/without selective broadcast, and the placement-aware assignment)
 """
 import argparse
 import json
@@ -41,20 +43,28 @@ def main():
     ap.add_argument("--bits", type=int, default=10)
     ap.add_argument("--log2-r-per-gpu", type=int, default=27)
     ap.add_argument("--log2-s-per-gpu", type=int, default=29)
+    ap.add_argument("--workload", default="zipf", choices=["zipf", "unique"])
+    ap.add_argument("--placement-z", type=float, default=0.0)
     a = ap.parse_args()
+    from paper_conf_sigmod_paullhl21_b200 import datagen
     N, P = a.gpus, 1 << a.bits
     n_r, n_s = N << a.log2_r_per_gpu, N << a.log2_s_per_gpu
     H = np.zeros((N, 2, P), np.uint64)
     for g in range(N):
-        H[g, 0] = hist_of("zipf", 0, n_r, n_s, a.z, n_r * g // N, n_r * (g + 1) // N, P)
-        H[g, 1] = hist_of("zipf", 1, n_r, n_s, a.z, n_s * g // N, n_s * (g + 1) // N, P)
-    out = {"workload": f"M4 zipf z={a.z}: {n_r} R + {n_s} S tuples over {N} GPUs (8-byte tuples)", "B1": a.bits,
-           "modes": {}}
+        rlo, rhi = datagen.shard_bounds(n_r, g, N, a.placement_z)
+        slo, shi = datagen.shard_bounds(n_s, g, N, a.placement_z)
+        H[g, 0] = hist_of(a.workload, 0, n_r, n_s, a.z, rlo, rhi, P)
+        H[g, 1] = hist_of(a.workload, 1, n_r, n_s, a.z, slo, shi, P)
+    out = {"workload": f"{a.workload} z={a.z}, placement z={a.placement_z}: {n_r} R + {n_s} S tuples over {N} GPUs "
+                       f"(8-byte tuples)", "B1": a.bits, "modes": {}}
     tot = H.sum(axis=0)
-    for mode, name in ((-1, "hash (single owner per partition)"), (0, "selective broadcast (auto)")):
-        plans = [mgj.plan_host(N, g, a.bits, H.astype(np.uint32), skew_bcast=mode, with_bcast=True)
+    for mode, assign, name in ((-1, 0, "hash (single owner per partition, contiguous ranges)"),
+                               (0, 0, "selective broadcast (auto)"),
+                               (-1, 1, "placement-aware assignment (Track-Join migration)"),
+                               (0, 1, "placement-aware + selective broadcast")):
+        plans = [mgj.plan_host(N, g, a.bits, H.astype(np.uint32), skew_bcast=mode, with_bcast=True, assign=assign)
                  for g in range(N)]
-        owner, _, recv, bc = plans[0]
+        owner, _, recv, bc, _skip = plans[0]
         moved = 0  # tuples that leave their rank in the shuffle
         for g in range(N):
             for rel in range(2):
@@ -66,7 +76,7 @@ def main():
                  for d in range(N)]
         work = [built[d] + int(recv[1, d]) for d in range(N)]
         out["modes"][name] = {
-            "skew_bcast": mode, "broadcast_partitions": int(bc.sum()),
+            "skew_bcast": mode, "assign": assign, "broadcast_partitions": int(bc.sum()),
             "recv_r": [int(x) for x in recv[0]], "recv_s": [int(x) for x in recv[1]],
             "tuples_joined_per_rank": work,
             "max_over_mean_work": max(work) / (sum(work) / N),

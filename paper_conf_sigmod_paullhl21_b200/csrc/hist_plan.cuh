@@ -353,7 +353,9 @@ __global__ void __launch_bounds__(1024) k_plan(Ctx c) {
     uint32_t *chn = reinterpret_cast<uint32_t *>(own + P);  // [P+1] scratch scans (u32)
     uint8_t *bcf = reinterpret_cast<uint8_t *>(chn + P + 1);  // [P] broadcast flags
     // compressed shuffle: the receive layout counts 32-byte units, ownership still tuples
-    uint64_t *ut0 = reinterpret_cast<uint64_t *>((reinterpret_cast<uintptr_t>(bcf + P) + 7) & ~(uintptr_t)7), *ut1 = ut0 + P;
+    // (present only with compression, P <= 1024: P = 4096 would not fit shared memory otherwise)
+    const int PU = c.comp ? P : 0;
+    uint64_t *ut0 = reinterpret_cast<uint64_t *>((reinterpret_cast<uintptr_t>(bcf + P) + 7) & ~(uintptr_t)7), *ut1 = ut0 + PU;
     __shared__ uint64_t tmp[33];
     __shared__ uint32_t tmp32[33];
     __shared__ int first[MAX_RANKS], endp[MAX_RANKS];
@@ -410,8 +412,7 @@ __global__ void __launch_bounds__(1024) k_plan(Ctx c) {
             tot0[p] = t0;
             pre0[p] = c.comp ? u0 : t0;
             tot1[p] = t1;
-            ut0[p] = u0;
-            ut1[p] = u1;
+            if (c.comp) ut0[p] = u0, ut1[p] = u1;
             st += t1;
         }
         st = warp_sum(st);
@@ -504,7 +505,7 @@ __global__ void __launch_bounds__(1024) k_plan(Ctx c) {
         // mgj_plan_host).  Owners are no longer contiguous ranges: the layout
         // of rank d is its partitions ascending (one block scan per rank and
         // relation), then, for S, its own tuples of broadcast partitions.
-        uint8_t *best = reinterpret_cast<uint8_t *>(ut1 + P);  // [P] (after the unit totals)
+        uint8_t *best = reinterpret_cast<uint8_t *>(ut1 + PU);  // [P] (after the unit totals, if any)
         for (int p = tid; p < P; p += blockDim.x) {
             int b = 0;
             uint64_t hb = 0;

@@ -213,8 +213,10 @@ size_t hist_smem(const Norm &n) {
     return (size_t)hist_nb(T, n.c.key_bytes) * T * n.c.key_bytes + (size_t)n.P * 8;
 }
 size_t plan_smem(const Norm &n) {
-    return (size_t)n.P * 5 * 8 + (size_t)n.P * 4 + (size_t)(n.P + 1) * 4 + (size_t)n.P + 8 + (size_t)n.P * 2 * 8 +
-           (size_t)n.P;  // ... unit totals, preferred ranks
+    // totals, prefixes, owners, scan scratch, broadcast flags, then the unit
+    // totals (compression only) and the preferred ranks (assignment only)
+    return (size_t)n.P * 5 * 8 + (size_t)n.P * 4 + (size_t)(n.P + 1) * 4 + (size_t)n.P + 8 +
+           (n.c.compress ? (size_t)n.P * 2 * 8 : 0) + (n.c.assign ? (size_t)n.P : 0);
 }
 size_t scatter_smem(const Norm &n) { return scatter_smem_bytes(n.P, n.c.key_bytes); }
 size_t planA_smem(const Norm &n) { return ((size_t)local2_vcap(n.P) + 1) * 12; }

@@ -53,8 +53,8 @@ def parse():
     ap.add_argument("--skew-bcast", type=int, default=0, choices=[-1, 0, 1],
                     help="a2 selective broadcast of heavy S partitions (N>1): 0 auto, -1 never, 1 forced")
     ap.add_argument("--num-sms", type=int, default=0, help="SMs the library's persistent kernels use (0 = all)")
-    ap.add_argument("--overlap", default="auto", choices=["auto", "on", "off"],
-                    help="§8(e): R's local pass beside S's scatter (auto: on for N > 1 with the P2P shuffle)")
+    ap.add_argument("--overlap", default="auto", choices=["auto", "on", "off", "stream"],
+                    help="§8(e): R's local pass beside S's scatter (auto: on for N > 1 with the P2P shuffle); stream: S's local pass too, chunk by chunk as scatter rounds complete (NEXT-3)")
     ap.add_argument("--overlap-local-sms", type=int, default=0)
     ap.add_argument("--trace", action="store_true", help="kernel timeline of the last step in the JSON line")
     ap.add_argument("--placement-z", type=float, default=0.0,
@@ -309,7 +309,7 @@ def main():
                                            else (n_s if world > 1 and a.placement_z else 0)),
                           shuffle_mode=(mgj.SHUFFLE_EXTERNAL if a.shuffle == "nccl" else mgj.SHUFFLE_P2P),
                           skew_bcast=a.skew_bcast, num_sms=a.num_sms,
-                          shuffle_overlap={"auto": 0, "on": 1, "off": -1}[a.overlap],
+                          shuffle_overlap={"auto": 0, "on": 1, "off": -1, "stream": 2}[a.overlap],
                           overlap_local_sms=a.overlap_local_sms, trace=a.trace, compress=a.compress,
                           assign=a.assign)
     # N>1 (or MGJ_SYMM_ARENA=1): the library's symmetric-memory setup (mgj.symmetric_join)

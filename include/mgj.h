@@ -85,7 +85,15 @@ typedef struct {
     int32_t  shuffle_overlap;          /* SURVEY.md §8(e) / P:455-468: local-partition R (on a second
                                           stream, overlap_local_sms SMs) while S is still being shuffled
                                           (the rest of the SMs).  0 = auto (on for world_size > 1 with
-                                          MGJ_SHUFFLE_P2P), 1 = on, -1 = off.  Never with EXTERNAL */
+                                          MGJ_SHUFFLE_P2P), 1 = on, -1 = off.  Never with EXTERNAL.
+                                          2 = on, plus chunk streaming (NEXT-3): S's local
+                                          pass also runs on the second stream, beside S's scatter, and
+                                          starts each received chunk as soon as the scatter rounds that
+                                          fill it are complete at every source rank (S tiles complete in
+                                          rounds; each completed tile is counted at every owner, which
+                                          waits in the kernel, bounded by peer_timeout_ms).  P2P only.
+                                          Ranks sharing one GPU (virtual ranks) then hold at most half the
+                                          SMs with their local passes together */
     int32_t  overlap_local_sms;        /* SMs of R's local pass during the overlap (0 = half the SMs) */
     int32_t  trace;                    /* 1: record the first start and last end (globaltimer, ns) of
                                           every kernel of the run (mgj_debug_copy MGJ_DBG_TRACE) */

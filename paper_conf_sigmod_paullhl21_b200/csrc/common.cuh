@@ -42,6 +42,11 @@ constexpr int RES_W = 8;  // u64 words per rank in the result mailbox (a6)
 constexpr int CU_N = 5;
 constexpr int CU_ENTRY_BITS = 44;
 constexpr int CHUNK_UNITS = 2048;  // local-pass chunk with the compressed shuffle: 2 units per thread
+// NEXT-3 chunk streaming: the S scatter's tiles complete in rounds (round r =
+// the r-th tile of every scatter CTA); at most STREAM_RMAX rounds, tiles per
+// scatter CTA STREAM_TPC (fewer if the rounds would exceed STREAM_RMAX)
+constexpr int STREAM_RMAX = 16;
+constexpr int STREAM_TPC = 4;
 // peer flags: histograms published (a1), R / S tuples all stored (a3), partial sums published (a6)
 enum Sig { SIG_HIST = 0, SIG_DATA_R = 1, SIG_RES = 2, SIG_DATA_S = 3, SIG_COUNT = 4 };
 enum Ticket { TK_HIST = 0, TK_SCAT_R = 1, TK_SCAT_S = 2, TK_SCAT_DONE = 3, TK_ITEMS = 4,
@@ -71,6 +76,8 @@ struct Arena {
     uint64_t resmail;  // u64 res[MAX_RANKS][RES_W] (count, checksum, n_out, status, pair digest)
     uint64_t cfgmail;  // u64 cfg[MAX_RANKS][4] (recv_cap R, recv_cap S, arena bytes, B1) published with a1
     uint64_t umail;    // u32 units[MAX_RANKS][2][P] (compress: 32-byte units per partition) published with a1
+    uint64_t rbmail;   // u32 ntile[STREAM_RMAX], then rb[STREAM_RMAX][P]: this rank's S rounds (streaming)
+    uint64_t rdone;    // u64 done[STREAM_RMAX]: epoch << 32 | this rank's S tiles of round r stored (streaming)
     uint64_t recv[2];  // received tuples of R, S
     uint64_t total;
 };
@@ -105,6 +112,12 @@ struct Ctx {
     int32_t comp;                 // NEXT-1 compressed shuffle (units of CU_N entries, see scatter.cuh)
     int32_t assign;               // NEXT-2 placement-aware partition assignment (k_plan)
     int32_t chunk_units;          // compress: local-pass chunk in units
+    int32_t stream;               // NEXT-3: S's local pass streams chunks as their scatter rounds complete
+    int32_t sgrid;                //   S scatter CTAs (tiles per round)
+    int32_t nrounds;              //   rounds of the S scatter: ceil(G / sgrid) <= STREAM_RMAX
+    uint32_t *cwait;              //   [max_chunks] S chunk li: first source << 8 | last source << 4 | its last round
+    uint32_t *corder;             //   [max_chunks] S chunks in round order
+    uint32_t *rcount;             //   [2][STREAM_RMAX] S chunks per round, placement cursors (zeroed per run)
     uint32_t *rowbase;            // compress: [2][MAX_RANKS][G] global row id of each (rank, tile)'s first row
     uint32_t *rank_units;         // compress: [2][P] this rank's 32-byte units per partition
     uint32_t max_items;
@@ -219,6 +232,20 @@ __device__ inline bool wait_all_flags(const Ctx &c, int kind) {
         }
     }
     return true;
+}
+
+// NEXT-3 streaming, in the arena of source rank g: the completed S tiles of
+// its round r (epoch << 32 | count: k_tilescan sets the epoch, each tile adds
+// one; a later run's value compares above any earlier one), and the rounds'
+// non-empty tiles and per-partition first offsets.
+__device__ __forceinline__ unsigned long long *rdone_ptr(char *arena, const Arena &lay, int r) {
+    return reinterpret_cast<unsigned long long *>(arena + lay.rdone) + r;
+}
+__device__ __forceinline__ uint32_t *rb_ntile(char *arena, const Arena &lay) {
+    return reinterpret_cast<uint32_t *>(arena + lay.rbmail);
+}
+__device__ __forceinline__ uint32_t *rb_first(char *arena, const Arena &lay, int P, int r, int p) {
+    return reinterpret_cast<uint32_t *>(arena + lay.rbmail) + STREAM_RMAX + (size_t)r * P + p;
 }
 
 // Raise flag `kind` of this rank at every peer (call after a system fence).

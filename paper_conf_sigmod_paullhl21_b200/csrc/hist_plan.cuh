@@ -35,6 +35,14 @@ __host__ __device__ inline int hist_nb(int T, int key_bytes) {
 // The fused exchange of a1 (one CTA): the rank histogram (and, compressed,
 // the unit counts) and the job-wide configuration words into every peer's
 // mailbox, then SIG_HIST everywhere.
+// Job-wide configuration word checked equal on every rank by k_plan: B1, the
+// compressed shuffle and, with chunk streaming, the tile geometry the round
+// counts assume (tiles per relation, S scatter CTAs).
+__device__ __forceinline__ uint64_t cfg_word(const Ctx &c) {
+    return (uint64_t)(c.B1 | c.comp << 8 | c.stream << 9) |
+           (c.stream ? ((uint64_t)c.G << 16 | (uint64_t)c.sgrid << 40) : 0ull);
+}
+
 __device__ inline void publish_hist(const Ctx &c) {
     const int P = c.P;
     for (int d = 0; d < c.world; ++d) {
@@ -46,7 +54,7 @@ __device__ inline void publish_hist(const Ctx &c) {
         }
         // this rank's job-wide configuration words, checked equal on every rank by k_plan
         if (threadIdx.x < 4) {
-            const uint64_t w[4] = {c.recv_cap[0], c.recv_cap[1], c.lay.total, (uint64_t)(c.B1 | c.comp << 8)};
+            const uint64_t w[4] = {c.recv_cap[0], c.recv_cap[1], c.lay.total, cfg_word(c)};
             reinterpret_cast<uint64_t *>(c.arena[d] + c.lay.cfgmail)[c.rank * 4 + threadIdx.x] = w[threadIdx.x];
         }
     }
@@ -194,7 +202,8 @@ __global__ void __launch_bounds__(HIST_THREADS, 2) k_hist(Ctx c) {
     __shared__ int last;
     if (threadIdx.x == 0) last = (atomicAdd(&c.ticket[TK_HIST], 1u) == gridDim.x * gridDim.y - 1);
     __syncthreads();
-    if (!last || c.comp) return;  // compressed shuffle: k_tilescan publishes, with the unit counts
+    // compressed shuffle / chunk streaming: k_tilescan publishes (unit counts, round boundaries)
+    if (!last || c.comp || c.stream) return;
     __threadfence();
     publish_hist(c);
 }
@@ -215,6 +224,28 @@ __global__ void k_tilescan(Ctx c) {
         auto val = [&](uint32_t v) { return c.comp ? (v + CU_N - 1) / CU_N : v; };
         uint32_t run = 0;
         int t = 0;
+        if (c.stream && rel == 1) {
+            // NEXT-3: S round boundaries — offset of round r's first tile in this
+            // rank's piece of p (round r = tiles [r * sgrid, (r + 1) * sgrid)),
+            // read by p's owner to tell which rounds a received chunk needs
+            for (; t < c.G; ++t) {
+                if (t % c.sgrid == 0) *rb_first(c.arena[c.rank], c.lay, c.P, t / c.sgrid, p) = run;
+                dst[t * stride] = run;
+                run += val(src[t * stride]);
+            }
+            if (p == 0) {  // the rounds' non-empty tiles, and their counters opened for this run
+                for (int r = 0; r < c.nrounds; ++r) {
+                    uint32_t nt = 0;
+                    for (int u = r * c.sgrid; u < c.G && u < (r + 1) * c.sgrid; ++u) {
+                        uint64_t lo, hi;
+                        tile_range(c.n_in[1], c.G, u, lo, hi);
+                        nt += hi > lo;
+                    }
+                    rb_ntile(c.arena[c.rank], c.lay)[r] = nt;
+                    *rdone_ptr(c.arena[c.rank], c.lay, r) = c.epoch << 32;
+                }
+            }
+        }
         for (; t + 4 <= c.G; t += 4) {
             const uint32_t v0 = src[(t + 0) * stride], v1 = src[(t + 1) * stride];
             const uint32_t v2 = src[(t + 2) * stride], v3 = src[(t + 3) * stride];
@@ -234,7 +265,7 @@ __global__ void k_tilescan(Ctx c) {
         }
         if (c.comp) c.rank_units[idx] = run;
     }
-    if (!c.comp) return;
+    if (!c.comp && !c.stream) return;
     __shared__ int last;
     __threadfence();
     __syncthreads();
@@ -377,7 +408,7 @@ __global__ void __launch_bounds__(1024) k_plan(Ctx c) {
         // must have planned with the same ones, else peers store at offsets
         // that differ from the receiver's layout
         const uint64_t *cf = reinterpret_cast<const uint64_t *>(c.arena[c.rank] + c.lay.cfgmail);
-        const uint64_t w[4] = {c.recv_cap[0], c.recv_cap[1], c.lay.total, (uint64_t)(c.B1 | c.comp << 8)};
+        const uint64_t w[4] = {c.recv_cap[0], c.recv_cap[1], c.lay.total, cfg_word(c)};
         for (int g = 0; g < N && ok; ++g)
             for (int i = 0; i < 4; ++i)
                 if (__ldcg(cf + g * 4 + i) != w[i]) {

@@ -78,7 +78,81 @@ __global__ void k_chunkmap(Ctx c, ChunkDesc *desc) {
         d.len = (uint32_t)min(C, (uint64_t)c.piece_len[pidx] - k * C);
         d.pi = (uint32_t)lo;
         desc[ci] = d;
+        if (c.stream && rel == 1) {
+            // NEXT-3: the S rounds this chunk needs.  A P2P segment holds the
+            // sources' pieces back to back (sources ascending; a broadcast
+            // partition's S only this rank's own): sources g_lo..g_hi overlap
+            // the chunk; those before g_hi end inside it (all their rounds),
+            // g_hi needs the rounds whose first offset lies below the chunk's end
+            const int pg = c.plist[lo];
+            const uint64_t o0 = k * C, o1 = o0 + d.len;
+            int glo = c.rank, ghi = c.rank;
+            uint64_t base_hi = 0;
+            if (!c.bcast[pg]) {
+                const uint32_t *cnt = reinterpret_cast<const uint32_t *>(c.arena[c.rank] + (c.comp ? c.lay.umail : c.lay.mail));
+                uint64_t b = 0;
+                glo = -1;
+                for (int s = 0; s < c.world; ++s) {
+                    const uint64_t e = b + __ldcg(cnt + (size_t)(s * 2 + 1) * P + pg);
+                    if (e > o0 && b < o1) {
+                        if (glo < 0) glo = s;
+                        ghi = s;
+                        base_hi = b;
+                    }
+                    b = e;
+                }
+                if (glo < 0) glo = ghi = c.rank;  // (an empty chunk: none)
+            }
+            int rh = 0;
+            while (rh + 1 < c.nrounds && base_hi + __ldcg(rb_first(c.arena[ghi], c.lay, P, rh + 1, pg)) < o1) ++rh;
+#ifdef MGJ_DBG_WAITALL
+            rh = c.nrounds - 1;
+#endif
+            c.cwait[li] = (uint32_t)(glo << 8 | ghi << 4 | rh);
+            atomicAdd(&c.rcount[glo < ghi ? c.nrounds - 1 : rh], 1u);
+        }    }
+}
+
+// NEXT-3: the S chunks in round order (a counting sort by the last round each
+// needs; the order inside a round is free: outputs are placed by chunk index).
+__global__ void k_chunkorder(Ctx c) {
+    if (!c.meta[MT_OK] || !c.stream) return;
+    __shared__ uint32_t base[STREAM_RMAX];
+    if (threadIdx.x == 0) {
+        uint32_t a = 0;
+        for (int r = 0; r < STREAM_RMAX; ++r) base[r] = a, a += __ldcg(&c.rcount[r]);
     }
+    __syncthreads();
+    const uint32_t nch_s = (uint32_t)c.meta[MT_NCH_S];
+    for (uint32_t li = blockIdx.x * blockDim.x + threadIdx.x; li < nch_s; li += gridDim.x * blockDim.x) {
+        const uint32_t w = c.cwait[li];
+        const int r = ((w >> 8) & 15u) < ((w >> 4) & 15u) ? c.nrounds - 1 : (int)(w & 15u);
+        c.corder[base[r] + atomicAdd(&c.rcount[STREAM_RMAX + r], 1u)] = li;
+    }
+}
+
+// NEXT-3: thread-level wait until every source rank g_lo..g_hi of a chunk
+// has stored every non-empty S tile of the rounds the chunk needs for this
+// run (w = g_lo << 8 | g_hi << 4 | rh: all rounds of g < g_hi, rounds 0..rh
+// of g_hi; the sources' counters, polled over NVLink), then order the async
+// proxy's (TMA) reads of the received tuples after it.
+__device__ inline void stream_wait(const Ctx &c, uint32_t w) {
+    const int glo = (int)((w >> 8) & 15u), ghi = (int)((w >> 4) & 15u), rh = (int)(w & 15u);
+    const uint64_t t0 = globaltimer();
+    for (int g = glo; g <= ghi; ++g) {
+        for (int r = 0; r <= (g < ghi ? c.nrounds - 1 : rh); ++r) {
+            const uint64_t want = c.epoch << 32 | __ldcg(rb_ntile(c.arena[g], c.lay) + r);
+            const uint64_t *f = reinterpret_cast<const uint64_t *>(rdone_ptr(c.arena[g], c.lay, r));
+            while (ld_acquire_sys(f) < want) {
+                if (globaltimer() - t0 > c.timeout_ns) {
+                    set_err(c, MGJ_EPEER);
+                    return;
+                }
+                __nanosleep(64);
+            }
+        }
+    }
+    fence_proxy_async_global();
 }
 
 // ---------------------------------------------------------------------------
@@ -252,7 +326,7 @@ __global__ void __launch_bounds__(512) k_countA(Ctx c, const ChunkDesc *cdesc) {
 // ---------------------------------------------------------------------------
 enum LocalMode { LM_SINGLE = 0, LM_SPLIT = 1, LM_SECOND = 2 };
 
-template <typename K, int MODE, int RSEL = 2, bool COMP = false>
+template <typename K, int MODE, int RSEL = 2, bool COMP = false, bool STRM = false>
 __device__ __forceinline__ void local_body(const Ctx &c, const ChunkDesc *cdesc) {
     static_assert(!COMP || (MODE == LM_SINGLE && sizeof(K) == 4), "compressed input: single pass, 4-byte keys");
     constexpr bool SPLIT = MODE == LM_SPLIT;
@@ -283,6 +357,14 @@ __device__ __forceinline__ void local_body(const Ctx &c, const ChunkDesc *cdesc)
     const uint32_t c0 = RSEL == 1 ? nch_r : 0u, c1 = RSEL == 0 ? nch_r : total;
     const uint32_t span = c1 - c0;
     const uint32_t mine = span > blockIdx.x ? (span - blockIdx.x + gridDim.x - 1) / gridDim.x : 0;
+    // NEXT-3 streaming (S pass beside S's scatter): the chunks in round order,
+    // each loaded once the scatter rounds it needs are complete
+    static_assert(!STRM || (RSEL == 1 && MODE == LM_SINGLE), "streaming: S's single pass");
+    constexpr bool strm = STRM;
+    auto cidx = [&](uint32_t j) -> uint32_t {
+        const uint32_t k = blockIdx.x + j * gridDim.x;
+        return c0 + (strm ? __ldcg(c.corder + k) : k);
+    };
     constexpr bool from_mid = MODE == LM_SECOND;
     // source of a chunk: the first pass's output, or a receive buffer (this
     // rank's, or a broadcast partition root's for its R side: piece_src)
@@ -300,8 +382,12 @@ __device__ __forceinline__ void local_body(const Ctx &c, const ChunkDesc *cdesc)
     const uint64_t pol = policy_evict_first();
     // thread 0: TMA chunk j (16-byte-aligned superset) into buffer j & 1
     auto issue = [&](uint32_t j, const ChunkDesc &d) {
-        const uint32_t ci = c0 + blockIdx.x + j * gridDim.x;
+        const uint32_t ci = cidx(j);
         const int rel = ci < nch_r ? 0 : 1;
+        if (strm) stream_wait(c, __ldcg(c.cwait + (ci - c0)));
+#ifdef MGJ_DBG_WAITSIG
+        if (strm) wait_all_flags(c, SIG_DATA_S);
+#endif
         sdesc[j & 1] = d;
         uint64_t *b = &bar[j & 1];
         if constexpr (COMP) {  // whole 32-byte units
@@ -322,11 +408,11 @@ __device__ __forceinline__ void local_body(const Ctx &c, const ChunkDesc *cdesc)
     ChunkDesc nxt{};
     constexpr int LI = 32;  // the thread that issues the chunk loads (and the chunked pass's stores)
     if (tid == LI) {
-        if (mine > 0) issue(0, cdesc[c0 + blockIdx.x]);
-        if (mine > 1) nxt = cdesc[c0 + blockIdx.x + gridDim.x];
+        if (mine > 0) issue(0, cdesc[cidx(0)]);
+        if (mine > 1) nxt = cdesc[cidx(1)];
     }
     for (uint32_t j = 0; j < mine; ++j) {
-        const uint32_t ci = c0 + blockIdx.x + j * gridDim.x;
+        const uint32_t ci = cidx(j);
         const int rel = ci < nch_r ? 0 : 1;
         const uint32_t li = rel ? ci - nch_r : ci;
         const int X = j & 1;
@@ -389,7 +475,7 @@ __device__ __forceinline__ void local_body(const Ctx &c, const ChunkDesc *cdesc)
         if (tid == LI && j + 1 < mine) {
             if (!SPLIT) bulk_wait_read0();
             issue(j + 1, nxt);
-            if (j + 2 < mine) nxt = cdesc[c0 + blockIdx.x + (j + 2) * gridDim.x];
+            if (j + 2 < mine) nxt = cdesc[cidx(j + 2)];
         }
         if (tid >= 32) {  // the other bin array (last read by chunk j-1 before its S3) for chunk j+1
             uint32_t *const bn = bins2 + (X ^ 1) * QL;
@@ -517,14 +603,14 @@ __global__ void __launch_bounds__(LOCAL_THREADS, 1) k_local_second(Ctx c, const 
 // the chunks of R (rsel 0), of S (1) or of both (2).  With the shuffle
 // overlapped (§8(e)), R's launch first waits for every rank's R tuples
 // (SIG_DATA_R) and runs beside the scatter of S on the SMs it leaves free.
-template <typename K, int RSEL, bool COMP = false>
+template <typename K, int RSEL, bool COMP = false, bool STRM = false>
 __global__ void __launch_bounds__(LOCAL_THREADS, 1) k_local(Ctx c, const ChunkDesc *cdesc) {
     if (!c.meta[MT_OK] || c.meta[MT_BA]) return;
     // timeline stamps for the overlapped launches only: in the single launch
     // over both relations (the one-GPU path) they cost a 4-byte spill
     constexpr int id = RSEL == 0 ? MGJ_TR_LOCAL_R : MGJ_TR_LOCAL_S;
     if constexpr (RSEL != 2) trace_begin(c, id);
-    local_body<K, LM_SINGLE, RSEL, COMP>(c, cdesc);
+    local_body<K, LM_SINGLE, RSEL, COMP, STRM>(c, cdesc);
     if constexpr (RSEL != 2) trace_end(c, id);
 }
 

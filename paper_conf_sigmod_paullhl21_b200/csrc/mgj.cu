@@ -48,7 +48,9 @@ mgj_status normalize(const mgj_config *in, Norm *o) {
     if (c.assign != 0 && c.assign != 1) return MGJ_EINVAL;
     if (c.assign && c.shuffle_mode != MGJ_SHUFFLE_P2P) return MGJ_EINVAL;  // EXTERNAL needs contiguous owners
     if (c.peer_timeout_ms < 0) return MGJ_EINVAL;
-    if (c.shuffle_overlap < -1 || c.shuffle_overlap > 1 || c.overlap_local_sms < 0) return MGJ_EINVAL;
+    if (c.shuffle_overlap < -1 || c.shuffle_overlap > 2 || c.overlap_local_sms < 0) return MGJ_EINVAL;
+    // chunk streaming (NEXT-3) needs the in-kernel shuffle's completion counts
+    if (c.shuffle_overlap == 2 && c.shuffle_mode != MGJ_SHUFFLE_P2P) return MGJ_EINVAL;
     if (c.trace != 0 && c.trace != 1) return MGJ_EINVAL;
     if (c.compress != 0 && c.compress != 1) return MGJ_EINVAL;
     // the compressed shuffle (NEXT-1): 4-byte keys and payloads, in-kernel peer stores
@@ -133,6 +135,10 @@ mgj_status normalize(const mgj_config *in, Norm *o) {
     off = align_up(off + (uint64_t)MAX_RANKS * 2 * o->P * 4, 4096);
     L.cfgmail = off;
     off = align_up(off + MAX_RANKS * 4 * 8, 4096);
+    L.rbmail = off;
+    off = align_up(off + (uint64_t)STREAM_RMAX * (o->P + 1) * 4, 4096);
+    L.rdone = off;
+    off = align_up(off + STREAM_RMAX * 8, 4096);
     // compressed: a (source rank, tile, partition) run ends in a partial unit, so
     // short runs take more room than their tuples (at most one unit per tuple);
     // the bound counts <= 8 ranks x 256 tiles x P partial units
@@ -237,15 +243,44 @@ cudaError_t set_attrs(const Norm &n) {
         if ((e = cudaFuncSetAttribute(k_local<uint32_t, 0, true>, A, (int)local_smem(n)))) return e;
         if ((e = cudaFuncSetAttribute(k_local<uint32_t, 1, true>, A, (int)local_smem(n)))) return e;
         if ((e = cudaFuncSetAttribute(k_local<uint32_t, 2, true>, A, (int)local_smem(n)))) return e;
+        if ((e = cudaFuncSetAttribute(k_local<uint32_t, 1, true, true>, A, (int)local_smem(n)))) return e;
     }
     if ((e = cudaFuncSetAttribute(k_local<K, 0>, A, (int)local_smem(n)))) return e;
     if ((e = cudaFuncSetAttribute(k_local<K, 1>, A, (int)local_smem(n)))) return e;
     if ((e = cudaFuncSetAttribute(k_local<K, 2>, A, (int)local_smem(n)))) return e;
+    if ((e = cudaFuncSetAttribute(k_local<K, 1, false, true>, A, (int)local_smem(n)))) return e;
     if ((e = cudaFuncSetAttribute(k_local_second<K>, A, (int)local_smem2(n)))) return e;
     if ((e = cudaFuncSetAttribute(k_local_split<K>, A, (int)local_smem1s(n)))) return e;
     if ((e = cudaFuncSetAttribute(k_planA, A, (int)planA_smem(n)))) return e;
     if ((e = cudaFuncSetAttribute(k_probe<K, false>, A, (int)probe_smem(n)))) return e;
     return cudaFuncSetAttribute(k_probe<K, true>, A, (int)probe_smem(n));
+}
+
+// Load every kernel of the plan now.  With lazy module loading (the CUDA
+// default) a kernel's first launch loads its module, and the loader waits for
+// the device: a launch issued while another rank's kernel on this GPU spins on
+// a peer signal (virtual ranks; k_plan waiting for a histogram that the
+// blocked host thread has yet to launch) would stall until that wait times out.
+template <typename K>
+cudaError_t preload_kernels(const Norm &n) {
+    cudaFuncAttributes a;
+    const void *f[] = {(const void *)k_hist<K>, (const void *)k_tilescan, (const void *)k_plan,
+                       (const void *)k_chunkmap, (const void *)k_chunkorder, (const void *)scatter_kernel<K>(n.P),
+                       (const void *)k_wait, (const void *)k_local<K, 0>, (const void *)k_local<K, 1>,
+                       (const void *)k_local<K, 2>, (const void *)k_local<K, 1, false, true>,
+                       (const void *)k_countA<K>, (const void *)k_planA, (const void *)k_local_split<K>,
+                       (const void *)k_local_second<K>, (const void *)k_itemize<K>, (const void *)k_probe<K, false>,
+                       (const void *)k_probe<K, true>, (const void *)k_reduce};
+    for (const void *fn : f)
+        if (cudaError_t e = cudaFuncGetAttributes(&a, fn)) return e;
+    if (n.c.compress && n.P <= 1024) {
+        const void *fc[] = {(const void *)scatter_kernel_comp(), (const void *)k_local<uint32_t, 0, true>,
+                            (const void *)k_local<uint32_t, 1, true>, (const void *)k_local<uint32_t, 2, true>,
+                            (const void *)k_local<uint32_t, 1, true, true>};
+        for (const void *fn : fc)
+            if (cudaError_t e = cudaFuncGetAttributes(&a, fn)) return e;
+    }
+    return cudaSuccess;
 }
 
 bool is_device_ptr(const void *p) {
@@ -270,6 +305,7 @@ void launch_shuffle(mgj_plan_s *h, cudaStream_t s) {
     k_tilescan<<<(2 * n.P + 127) / 128, 128, 0, s>>>(h->ctx);
     k_plan<<<1, 1024, plan_smem(n), s>>>(h->ctx);
     k_chunkmap<<<h->nsm * 2, 256, 0, s>>>(h->ctx, h->cdesc);
+    if (h->ctx.stream) k_chunkorder<<<h->nsm, 256, 0, s>>>(h->ctx);
     cudaEventRecord(h->ev[2], s);
     Ctx cs = h->ctx;
     if (cs.ext)
@@ -278,8 +314,9 @@ void launch_shuffle(mgj_plan_s *h, cudaStream_t s) {
     const auto scat = comp ? scatter_kernel_comp() : scatter_kernel<K>(n.P);
     const size_t ssm = comp ? scat_smem_bytes_comp(n.P) : scatter_smem(n);
     const int nt = scatter_threads(n.P, n.c.key_bytes);
+    const int sg = std::min(h->ctx.G, h->nsm);  // persistent scatter CTAs (tiles blockIdx + k * grid)
     if (h->overlap) {
-        scat<<<h->ctx.G, nt, ssm, s>>>(cs, 0, 0);  // a3, R
+        scat<<<sg, nt, ssm, s>>>(cs, 0, 0);  // a3, R
         // §8(e) ("data distribution and local partitioning start
         // together"; Rationale 2): once every rank's R tuples have
         // landed, R is partitioned locally on local_sms SMs of a second stream
@@ -291,11 +328,20 @@ void launch_shuffle(mgj_plan_s *h, cudaStream_t s) {
             k_local<uint32_t, 0, true><<<h->local_sms, LOCAL_THREADS, local_smem(n), h->aux>>>(h->ctx, h->cdesc);
         else
             k_local<K, 0><<<h->local_sms, LOCAL_THREADS, local_smem(n), h->aux>>>(h->ctx, h->cdesc);
+        if (h->ctx.stream) {
+            // NEXT-3 ("packets" as they arrive): S's local pass right
+            // after R's, each chunk once the S scatter rounds it needs are done
+            if (comp)
+                k_local<uint32_t, 1, true, true><<<h->local_sms, LOCAL_THREADS, local_smem(n), h->aux>>>(h->ctx, h->cdesc);
+            else
+                k_local<K, 1, false, true><<<h->local_sms, LOCAL_THREADS, local_smem(n), h->aux>>>(h->ctx, h->cdesc);
+            h->launches += 2;  // chunk order, S's local pass
+        }
         cudaEventRecord(h->ev_join, h->aux);
         scat<<<h->scatter_sms, nt, ssm, s>>>(cs, 1, 1);  // a3, S
         h->launches += 7;
     } else {
-        scat<<<h->ctx.G, nt, ssm, s>>>(cs, 0, 1);  // a3, R then S in one launch
+        scat<<<sg, nt, ssm, s>>>(cs, 0, 1);  // a3, R then S in one launch
         h->launches += 4;
     }
 }
@@ -323,7 +369,9 @@ void launch_join(mgj_plan_s *h, cudaStream_t s) {
         k_local_second<K><<<h->nsm, LOCAL_THREADS, local_smem2(n), s>>>(h->ctx, h->cdescB);
         h->launches += 4;
     }
-    if (h->overlap)
+    if (h->ctx.stream)
+        h->launches -= 1;  // S's local pass already ran, streamed beside the scatter
+    else if (h->overlap)
         if (h->ctx.comp)
             k_local<uint32_t, 1, true><<<h->nsm, LOCAL_THREADS, local_smem(n), s>>>(h->ctx, h->cdesc);
         else
@@ -401,6 +449,32 @@ mgj_status mgj_plan(const mgj_config *cfg, const mgj_peers *peers, mgj_handle *o
     }
     const int P = n.P;
     const uint64_t Qm = 1ull << n.b2_max;
+    // §8(e) overlap: R's local pass on a second stream beside S's scatter;
+    // NEXT-3 streaming adds S's local pass there, chunk by chunk
+    const bool ext = n.c.shuffle_mode == MGJ_SHUFFLE_EXTERNAL;
+    h->overlap = !ext && (n.c.shuffle_overlap > 0 || (n.c.shuffle_overlap == 0 && W > 1));
+    const bool stream = !ext && n.c.shuffle_overlap == 2;
+    if (h->overlap) {
+        h->local_sms = n.c.overlap_local_sms ? std::min(n.c.overlap_local_sms, h->nsm - 1) : h->nsm / 2;
+        if (stream && W > 1) {
+            // ranks sharing this GPU (virtual ranks): their streaming local
+            // passes wait inside the kernel for the others' scatter, so they
+            // may hold at most half the SMs together
+            bool colocated = false;
+            for (int g = 0; g < W; ++g) {
+                cudaPointerAttributes a;
+                if (g != n.c.rank && cudaPointerGetAttributes(&a, h->arena[g]) == cudaSuccess && a.device == h->dev)
+                    colocated = true;
+            }
+            (void)cudaGetLastError();
+            if (colocated) h->local_sms = std::min(h->local_sms, h->nsm / (2 * W));
+        }
+        h->local_sms = std::max(h->local_sms, 1);
+        h->scatter_sms = std::max(h->nsm - h->local_sms, 1);
+    }
+    // scatter tiles per relation: one per SM, or (streaming) STREAM_TPC per
+    // S scatter CTA, in at most STREAM_RMAX rounds
+    const int G = stream ? std::min(h->nsm * STREAM_TPC, STREAM_RMAX * h->scatter_sms) : h->nsm;
     // per-run zero block: rank_hist, ticket, meta, acc, err, cop_slots
     size_t zo = 0;
     const size_t z_hist = zo; zo += align_up(2ull * P * 4, 256);
@@ -409,8 +483,8 @@ mgj_status mgj_plan(const mgj_config *cfg, const mgj_peers *peers, mgj_handle *o
     const size_t z_acc = zo; zo += 256;
     const size_t z_err = zo; zo += 256;
     const size_t z_cop = zo; zo += align_up(2ull * P * Qm * 4, 256);
-    const int G = h->nsm;  // scatter tiles: one per scatter CTA, one CTA per SM
     const size_t z_th = zo; zo += align_up(2ull * G * P * 4, 256);
+    const size_t z_rc = zo; zo += 256;  // streaming: chunks per round + cursors
     const size_t z_ha = zo; zo += align_up(2ull * local2_vcap(P) * 4, 256);
     h->zero_bytes = zo;
     char *zb = static_cast<char *>(dalloc(h, zo, &st));
@@ -423,7 +497,10 @@ mgj_status mgj_plan(const mgj_config *cfg, const mgj_peers *peers, mgj_handle *o
     c.b2_cfg = n.c.radix_bits_local;
     c.b2_max = n.b2_max;
     c.G = G;
-    c.hist_split = 2;  // k_hist: two CTAs per SM
+    c.hist_split = G > h->nsm ? 1 : 2;  // k_hist: two CTAs per SM
+    c.stream = stream;
+    c.sgrid = stream ? h->scatter_sms : 0;
+    c.nrounds = stream ? (G + c.sgrid - 1) / c.sgrid : 0;
     c.chunk_tuples = n.chunk_tuples;
     c.chunk_region = n.chunk_region;
     c.chunk_tuples2 = n.chunk_tuples2;
@@ -456,6 +533,7 @@ mgj_status mgj_plan(const mgj_config *cfg, const mgj_peers *peers, mgj_handle *o
         c.cop_slots = reinterpret_cast<uint32_t *>(zb + z_cop);
         c.tile_hist = reinterpret_cast<uint32_t *>(zb + z_th);
         c.hA = reinterpret_cast<uint32_t *>(zb + z_ha);
+        c.rcount = reinterpret_cast<uint32_t *>(zb + z_rc);
     }
     c.tile_base = static_cast<uint32_t *>(dalloc(h, 2ull * c.G * P * 4, &st));
     if (c.comp) {
@@ -466,6 +544,10 @@ mgj_status mgj_plan(const mgj_config *cfg, const mgj_peers *peers, mgj_handle *o
     c.sub_ns = (int32_t)((std::max(n.c.r_capacity, n.c.s_capacity) / c.G + 8) / c.scat_T + 2);
     c.sub_hist = static_cast<uint16_t *>(dalloc(h, 2ull * c.G * c.sub_ns * P * 2, &st));
     h->cdesc = static_cast<ChunkDesc *>(dalloc(h, 2 * n.max_chunks * sizeof(ChunkDesc), &st));
+    if (stream) {
+        c.cwait = static_cast<uint32_t *>(dalloc(h, n.max_chunks * 4, &st));
+        c.corder = static_cast<uint32_t *>(dalloc(h, n.max_chunks * 4, &st));
+    }
     if (n.split) h->cdescB = static_cast<ChunkDesc *>(dalloc(h, 2 * n.max_chunks * sizeof(ChunkDesc), &st));
     c.owner = static_cast<int32_t *>(dalloc(h, P * 4, &st));
     c.bcast = static_cast<uint8_t *>(dalloc(h, P, &st));
@@ -504,11 +586,7 @@ mgj_status mgj_plan(const mgj_config *cfg, const mgj_peers *peers, mgj_handle *o
         c.out_b = dalloc(h, n.out_cap * n.c.key_bytes, &st);
     }
     if (n.c.trace) c.trace = static_cast<unsigned long long *>(dalloc(h, MGJ_TRACE_COUNT * 2 * 8, &st));
-    h->overlap = !c.ext && (n.c.shuffle_overlap > 0 || (n.c.shuffle_overlap == 0 && W > 1));
     if (h->overlap) {
-        h->local_sms = n.c.overlap_local_sms ? std::min(n.c.overlap_local_sms, h->nsm - 1) : h->nsm / 2;
-        h->local_sms = std::max(h->local_sms, 1);
-        h->scatter_sms = std::max(h->nsm - h->local_sms, 1);
         if (st == MGJ_OK) st = cuda_ok(cudaStreamCreateWithFlags(&h->aux, cudaStreamNonBlocking));
         if (st == MGJ_OK) st = cuda_ok(cudaEventCreateWithFlags(&h->ev_fork, cudaEventDisableTiming));
         if (st == MGJ_OK) st = cuda_ok(cudaEventCreateWithFlags(&h->ev_join, cudaEventDisableTiming));
@@ -517,6 +595,7 @@ mgj_status mgj_plan(const mgj_config *cfg, const mgj_peers *peers, mgj_handle *o
     if (st == MGJ_OK) h->h_meta = reinterpret_cast<int32_t *>(h->h_res + 8);
     for (int i = 0; i < 7 && st == MGJ_OK; ++i) st = cuda_ok(cudaEventCreate(&h->ev[i]));
     if (st == MGJ_OK) st = cuda_ok(n.c.key_bytes == 4 ? set_attrs<uint32_t>(n) : set_attrs<uint64_t>(n));
+    if (st == MGJ_OK) st = cuda_ok(n.c.key_bytes == 4 ? preload_kernels<uint32_t>(n) : preload_kernels<uint64_t>(n));
     if (st != MGJ_OK) {
         mgj_destroy(h);
         return st;

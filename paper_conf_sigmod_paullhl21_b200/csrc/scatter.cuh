@@ -407,6 +407,19 @@ __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c, int rel0, int rel1) {
     // b mod N's share of them (owner ranges are contiguous in p, so in group order)
     const uint32_t rot_num = c.world > 1 ? (uint32_t)(blockIdx.x % c.world) : 0u;
 
+    // NEXT-3 chunk streaming (S launch): every completed S tile counts once in
+    // its round's counter in this rank's arena (after a system fence by every
+    // thread that stored its tuples; one atomic by thread 0), which owners
+    // poll before they start the local pass of a chunk the round fills.
+    // (The condition is re-read from the parameters and the tile to count
+    // kept in shared memory: more registers in the sub-tile loop spill.)
+#define MGJ_SCAT_STRM (c.stream && rel0 == 1)
+    auto sig_round = [&](int tile) {  // thread 0, after a system fence
+        atomicAdd_system(rdone_ptr(c.arena[c.rank], c.lay, tile / c.sgrid), 1ull);
+    };
+    __shared__ int done_tile;  // an S tile whose stores are fenced, counted after the next barrier
+    if (tid == 0) done_tile = -1;
+
     Cur u = at_tile(rel0, (int)blockIdx.x);
     uint32_t ncnt[PPT];
     load_counts(u, ncnt);
@@ -423,7 +436,13 @@ __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c, int rel0, int rel1) {
         const Cur nx = next_cur(u);
         const uint32_t row0 = cbase_rel(u.rel);  // COMP: global row id of this rank's first row
         if (u.rel * c.G + u.tile != cur_tile) {  // thread-private partition state: no barrier needed
-            if (cur_tile >= 0) flush(cur_tile / c.G, cur_tile % c.G);
+            if (cur_tile >= 0) {
+                flush(cur_tile / c.G, cur_tile % c.G);
+                if (MGJ_SCAT_STRM && cur_tile >= c.G) {
+                    __threadfence_system();
+                    if (tid == 0) done_tile = cur_tile - c.G;
+                }
+            }
             set_base(u.rel, u.tile);
             cur_tile = u.rel * c.G + u.tile;
         }
@@ -439,6 +458,11 @@ __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c, int rel0, int rel1) {
         load_counts(nx, ncnt);  // prefetch (consumed next iteration)
         uint32_t total;
         uint32_t o = block_scan_reg(tsum, tmp, total);  // its barriers: the last write-out is done
+        if (MGJ_SCAT_STRM && tid == 0 && done_tile >= 0) {  // every thread has fenced the tile's stores
+            __threadfence_system();
+            sig_round(done_tile);
+            done_tile = -1;
+        }
 #pragma unroll
         for (int k = 0; k < PPT; ++k) {
             const int p = tid * PPT + k;
@@ -554,6 +578,7 @@ __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c, int rel0, int rel1) {
     __syncthreads();
     for (int rel = rel0; rel <= rel1; ++rel) trace_end(c, rel ? MGJ_TR_SCATTER_S : MGJ_TR_SCATTER_R);
     if (tid == 0) {
+        if (MGJ_SCAT_STRM && cur_tile >= c.G) sig_round(cur_tile - c.G);  // the last S tile (fenced above)
         const uint32_t t = atomicAdd(&c.ticket[rel0 ? TK_SCAT_S : TK_SCAT_R], 1u);
         if (t == gridDim.x - 1) {
             __threadfence_system();
@@ -561,6 +586,8 @@ __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c, int rel0, int rel1) {
         }
     }
 }
+
+#undef MGJ_SCAT_STRM
 
 // The compressed-shuffle instance (NEXT-1): 4-byte keys, P <= 1024.
 constexpr ScatGeom scat_geom_comp() { return ScatGeom{8192, CU_N, 1, 1024}; }

@@ -47,7 +47,8 @@ def test_strerror(mgj):
 @pytest.mark.parametrize("bad", [dict(key_bytes=3), dict(world_size=0), dict(world_size=9), dict(rank=2, world_size=2),
                                  dict(radix_bits_global=13), dict(radix_bits_local=12), dict(r_capacity=1 << 32),
                                  dict(local_split_bits=7), dict(local_split_bits=-2), dict(skew_bcast=2),
-                                 dict(skew_bcast=-2), dict(peer_timeout_ms=-1), dict(shuffle_overlap=2),
+                                 dict(skew_bcast=-2), dict(peer_timeout_ms=-1), dict(shuffle_overlap=3),
+                                 dict(shuffle_overlap=2, shuffle_mode=1),
                                  dict(shuffle_overlap=-2), dict(overlap_local_sms=-1),
                                  dict(compress=1, key_bytes=8), dict(compress=1, shuffle_mode=1),
                                  dict(compress=1, radix_bits_global=11), dict(assign=2), dict(assign=1, shuffle_mode=1)])

@@ -1008,6 +1008,90 @@ def test_overlap_timeline(mgj):
         j.close()
 
 
+# ------------------------------------------------------------ NEXT-3: chunk streaming
+@pytest.mark.parametrize("N,kind,kw", [(1, "unique", {}), (2, "unique", {"materialize": True}), (4, "unique", {}),
+                                       (8, "unique", {"materialize": True}), (3, "zipf", {"skew_bcast": 1}),
+                                       (2, "m1", {"compress": True, "materialize": True}), (4, "m1", {"compress": True}),
+                                       (2, "wide", {"materialize": True}), (1, "unique", {"radix_bits_global": 4}),
+                                       (2, "unique", {"local_split_bits": 2})])
+def test_stream_parity(mgj, N, kind, kw):
+    """shuffle_overlap = 2: S's local pass
+    runs beside S's scatter and starts every chunk once the scatter rounds that
+    fill it are complete at its source rank.  Bit-exact vs the oracle (count,
+    checksum, pair digest; sorted triples when materialised) on N virtual
+    ranks, with broadcast, compression, 8-byte keys, small P and the
+    two-level local pass (which then runs after the shuffle, unstreamed)."""
+    w = {"unique": datagen.Workload("unique", 300007, 400009), "m1": datagen.M1(),
+         "zipf": datagen.Workload("zipf", 1 << 16, 1 << 18, 1.0),
+         "wide": datagen.Workload("wide", 200003, 300007)}[kind]
+    kw = dict(kw)
+    mat = kw.pop("materialize", False)
+    joins, res, _ = run_virtual(mgj, w, N, materialize=mat, shuffle_overlap=2, **kw)
+    d = w.rank_inputs()
+    ref = oracle.join(d["r_keys"], d["r_pays"], d["s_keys"], d["s_pays"], materialize=mat)
+    for r in res:
+        assert r["status"] == 0
+        assert (r["match_count"], r["checksum"], r["pair_digest"]) == (ref["count"], ref["checksum"], ref["pair_digest"])
+    if mat:
+        trip = [j.materialized(r) for j, r in zip(joins, res)]
+        k, a, b = sort_trip(*(np.concatenate([t[i] for t in trip]) for i in range(3)))
+        np.testing.assert_array_equal(k, ref["key"])
+        np.testing.assert_array_equal(a, ref["pay_r"])
+        np.testing.assert_array_equal(b, ref["pay_s"])
+    for j in joins:
+        j.close()
+
+
+def test_stream_repeated_runs(mgj):
+    """The round counters carry the run's epoch: three runs of one plan with
+    different S sizes (so different non-empty tiles per round), 2 virtual ranks."""
+    N = 2
+    cap = 1 << 18
+    cfgs = [mgj.make_config(rank=g, world_size=N, r_capacity=cap, s_capacity=cap, recv_capacity_r=2 * cap,
+                            recv_capacity_s=2 * cap, shuffle_overlap=2) for g in range(N)]
+    nb = mgj.arena_bytes(cfgs[0])
+    arenas = [torch.zeros(nb, dtype=torch.uint8, device="cuda") for _ in range(N)]
+    joins = [mgj.Join(cfgs[g], [a.data_ptr() for a in arenas], nb) for g in range(N)]
+    streams = [torch.cuda.Stream() for _ in range(N)]
+    for n_s in (cap, 1000, 77777):
+        w = datagen.Workload("unique", cap, n_s)
+        parts = [w.rank_inputs(g, N) for g in range(N)]
+        tens = [[dev(p[k]) for k in ("r_keys", "r_pays", "s_keys", "s_pays")] for p in parts]
+        torch.cuda.synchronize()
+        for g in range(N):
+            joins[g].partition(*tens[g], stream=streams[g])
+        for g in range(N):
+            joins[g].shuffle(streams[g])
+        for g in range(N):
+            joins[g].join(streams[g])
+        res = [joins[g].result() for g in range(N)]
+        d = w.rank_inputs()
+        ref = oracle.join(d["r_keys"], d["r_pays"], d["s_keys"], d["s_pays"])
+        for r in res:
+            assert r["status"] == 0
+            assert (r["match_count"], r["checksum"], r["pair_digest"]) == (ref["count"], ref["checksum"], ref["pair_digest"])
+    for j in joins:
+        j.close()
+
+
+def test_stream_timeline(mgj):
+    """With chunk streaming (one rank, trace=1) S's local pass starts while S
+    is still being scattered — unlike shuffle_overlap = 1, where it starts
+    after S's scatter (test_overlap_timeline) — and the result is exact."""
+    n = 1 << 24
+    cols = [torch.empty(n, dtype=torch.int32, device="cuda") for _ in range(4)]
+    mgj.gen_relation("unique", 0, n, n, 0.0, 0, n, cols[0], cols[1])
+    mgj.gen_relation("unique", 1, n, n, 0.0, 0, n, cols[2], cols[3])
+    j = mgj.Join(mgj.make_config(r_capacity=n, s_capacity=n, shuffle_overlap=2, trace=True))
+    for _ in range(2):
+        res = j.run(*cols)
+        assert res["match_count"] == n and res["status"] == 0
+    t = j.trace()
+    assert t["local_R"][0] < t["scatter_S"][1], t
+    assert t["local_S"][0] < t["scatter_S"][1], t
+    j.close()
+
+
 # ------------------------------------------------------------ NEXT-1: the compressed shuffle
 @pytest.mark.parametrize("N,kind,kw", [(1, "m1", {}), (2, "m1", {}), (4, "m1", {}), (1, "m1", {"radix_bits_global": 4}),
                                        (3, "zipf", {}), (4, "zipf", {"skew_bcast": 1, "radix_bits_global": 8}),

@@ -105,9 +105,6 @@ __global__ void k_chunkmap(Ctx c, ChunkDesc *desc) {
             }
             int rh = 0;
             while (rh + 1 < c.nrounds && base_hi + __ldcg(rb_first(c.arena[ghi], c.lay, P, rh + 1, pg)) < o1) ++rh;
-#ifdef MGJ_DBG_WAITALL
-            rh = c.nrounds - 1;
-#endif
             c.cwait[li] = (uint32_t)(glo << 8 | ghi << 4 | rh);
             atomicAdd(&c.rcount[glo < ghi ? c.nrounds - 1 : rh], 1u);
         }    }
@@ -385,9 +382,6 @@ __device__ __forceinline__ void local_body(const Ctx &c, const ChunkDesc *cdesc)
         const uint32_t ci = cidx(j);
         const int rel = ci < nch_r ? 0 : 1;
         if (strm) stream_wait(c, __ldcg(c.cwait + (ci - c0)));
-#ifdef MGJ_DBG_WAITSIG
-        if (strm) wait_all_flags(c, SIG_DATA_S);
-#endif
         sdesc[j & 1] = d;
         uint64_t *b = &bar[j & 1];
         if constexpr (COMP) {  // whole 32-byte units

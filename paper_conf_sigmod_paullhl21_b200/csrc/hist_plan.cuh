@@ -228,22 +228,39 @@ __global__ void k_tilescan(Ctx c) {
             // NEXT-3: S round boundaries — offset of round r's first tile in this
             // rank's piece of p (round r = tiles [r * sgrid, (r + 1) * sgrid)),
             // read by p's owner to tell which rounds a received chunk needs
-            for (; t < c.G; ++t) {
-                if (t % c.sgrid == 0) *rb_first(c.arena[c.rank], c.lay, c.P, t / c.sgrid, p) = run;
-                dst[t * stride] = run;
-                run += val(src[t * stride]);
+            for (int r = 0; r < c.nrounds; ++r) {
+                *rb_first(c.arena[c.rank], c.lay, c.P, r, p) = run;
+                const int t1 = min(c.G, (r + 1) * c.sgrid);
+                for (; t + 4 <= t1; t += 4) {
+                    const uint32_t v0 = src[(t + 0) * stride], v1 = src[(t + 1) * stride];
+                    const uint32_t v2 = src[(t + 2) * stride], v3 = src[(t + 3) * stride];
+                    dst[(t + 0) * stride] = run;
+                    run += val(v0);
+                    dst[(t + 1) * stride] = run;
+                    run += val(v1);
+                    dst[(t + 2) * stride] = run;
+                    run += val(v2);
+                    dst[(t + 3) * stride] = run;
+                    run += val(v3);
+                }
+                for (; t < t1; ++t) {
+                    dst[t * stride] = run;
+                    run += val(src[t * stride]);
+                }
             }
-            if (p == 0) {  // the rounds' non-empty tiles, and their counters opened for this run
-                for (int r = 0; r < c.nrounds; ++r) {
-                    uint32_t nt = 0;
-                    for (int u = r * c.sgrid; u < c.G && u < (r + 1) * c.sgrid; ++u) {
+            if (p < c.nrounds) {  // round p's non-empty tiles, and its counter opened for this run
+                const int r = p, u0 = r * c.sgrid, u1 = min(c.G, (r + 1) * c.sgrid);
+                uint32_t nt = (uint32_t)(u1 - u0);
+                if (c.n_in[1] < 8ull * (uint64_t)c.G) {  // small input: some tiles are empty
+                    nt = 0;
+                    for (int u = u0; u < u1; ++u) {
                         uint64_t lo, hi;
                         tile_range(c.n_in[1], c.G, u, lo, hi);
                         nt += hi > lo;
                     }
-                    rb_ntile(c.arena[c.rank], c.lay)[r] = nt;
-                    *rdone_ptr(c.arena[c.rank], c.lay, r) = c.epoch << 32;
                 }
+                rb_ntile(c.arena[c.rank], c.lay)[r] = nt;
+                *rdone_ptr(c.arena[c.rank], c.lay, r) = c.epoch << 32;
             }
         }
         for (; t + 4 <= c.G; t += 4) {

@@ -8,6 +8,7 @@ python -c "import __graft_entry__ as g; g.smoke()" > $O/smoke.txt 2>&1; echo "sm
 timeout 900 python bench.py > $O/bench.json 2> $O/bench.err; echo "bench rc=$?"
 timeout 600 python bench.py --impl reference > $O/bench_reference.json 2> $O/bench_reference.err; echo "reference rc=$?"
 timeout 600 python bench.py --steps 10 --warmup 3 --no-cpu-baseline --no-e2e --overlap on --trace > $O/bench_overlap_trace.json 2>/dev/null; echo "overlap rc=$?"
+timeout 600 python bench.py --steps 10 --warmup 3 --no-cpu-baseline --no-e2e --overlap stream --trace > $O/bench_stream_trace.json 2>/dev/null; echo "stream rc=$?"
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $O/launches.csv \
     python bench.py --steps 2 --warmup 1 --profile > $O/launch_bench.log 2>&1; echo "launch list rc=$?"
 timeout 1800 ncu --set full --clock-control none --import-source on --kernel-name-base function \

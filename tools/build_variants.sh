@@ -1,5 +1,5 @@
 # Build library variants for an A/B run: tools/build_variants.sh name:"-DFLAG=1 ..." ...
-# -> paper_conf_sigmod_paullhl21_b200/libmgj_<name>.so (run them with tools/gpu_ab.sh)
+# -> paper_conf_sigmod_paullhl21_b200/libmgj_<name>.so (run them with tools/gpu_ab2.sh)
 R=$(cd "$(dirname "$0")/.." && pwd)
 for v in "$@"; do
   n=${v%%:*}; f=${v#*:}

@@ -35,6 +35,10 @@ one({"r_keys": rng.integers(0, 1 << 14, 50000, dtype=np.uint64).astype(np.uint32
     materialize=False, radix_bits_global=10, radix_bits_local=6)
 # the overlapped shuffle (R's local pass on a second stream beside S's scatter) at one rank
 one(datagen.Workload("unique", 1 << 17, 1 << 17).rank_inputs(), materialize=True, shuffle_overlap=1, trace=True)
+# chunk streaming (NEXT-3) at one rank, and the compressed shuffle (NEXT-1)
+one(datagen.Workload("unique", 1 << 17, 1 << 17).rank_inputs(), materialize=True, shuffle_overlap=2,
+    peer_timeout_ms=600000)
+one(datagen.Workload("unique", 1 << 17, 1 << 17).rank_inputs(), materialize=True, compress=True)
 
 
 def virtual(w, N, **kw):
@@ -66,4 +70,8 @@ if os.environ.get("MGJ_SAN_VIRTUAL", "1") == "1":
     virtual(datagen.Workload("unique", 1 << 15, 1 << 15), 2)
     virtual(datagen.Workload("zipf", 1 << 13, 1 << 15, 1.0), 4, skew_bcast=1, radix_bits_global=6)
     virtual(datagen.Workload("zipf", 1 << 13, 1 << 15, 1.0), 4, skew_bcast=1, radix_bits_global=6, local_split_bits=2)
+    # round 2: chunk streaming, compressed + streaming, placement-aware assignment
+    virtual(datagen.Workload("unique", 1 << 15, 1 << 15), 2, shuffle_overlap=2, peer_timeout_ms=600000)
+    virtual(datagen.Workload("unique", 1 << 15, 1 << 15), 2, compress=True, shuffle_overlap=2, peer_timeout_ms=600000)
+    virtual(datagen.Workload("unique", 1 << 15, 1 << 15), 3, assign=1, peer_timeout_ms=600000)
 print("sanitize workload ok")

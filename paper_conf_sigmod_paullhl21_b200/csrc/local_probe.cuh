@@ -12,7 +12,11 @@ namespace mgj {
 // bulk copies 4.64, lane copies of short runs (Zipf z = 1: 3.13-3.55 vs
 // 2.80), an even R + S split between the producers 2.35, a software-
 // pipelined packed probe 2.02, two S slots per step 2.00, the packed table
-// for 8-byte keys 3.04 vs 2.82 at M5.)
+// for 8-byte keys 3.04 vs 2.82 at M5.  Round 2, against 1.885 ms: fewer
+// instructions per match 1.902, S slots in batches of 2 / 4 per thread
+// 2.015 / 2.116, head exchanges 2 / 4 at a time 1.899 / 1.889, the build of
+// item j+1 beside the probe of item j in a second table 2.86 — the consumers
+// are busy 94% of the time and the copies keep up.)
 
 template <typename K> struct Layout {
     using Tup = typename TupT<K>::T;

@@ -52,14 +52,17 @@ typedef enum {
     MGJ_DBG_OUT_KEY = 15,    /* materialised triples (n_materialized entries, key_bytes wide) */
     MGJ_DBG_OUT_PAY_R = 16,
     MGJ_DBG_OUT_PAY_S = 17,
-    MGJ_DBG_MID_R = 18,      /* tuples after the first local pass (sub-partitions, two-level a4 only) */
+    MGJ_DBG_MID_R = 18,      /* tuples after the first local pass (two-level a4 only): first-pass chunk k
+                                at slots [k * region, k * region + E[k][2^BA]), region = chunk_tuples1s + 64 */
     MGJ_DBG_MID_S = 19,
-    MGJ_DBG_VSTART = 20,     /* u64[2][L+1] sub-partition starts (slots) in MID_R / MID_S */
+    MGJ_DBG_MID_OFF_R = 20,  /* u16[chunks][65] first-pass run offsets E[k][a] (start | odd count for 8-byte
+                                tuples; E[k][2^BA] = the chunk's slots) of MID_R */
     MGJ_DBG_BCAST = 21,      /* u8[P]                selective-broadcast flag of each global partition (a2) */
     MGJ_DBG_PLIST = 22,      /* i32[np]              owned partitions: the range, then broadcast ones outside it */
     MGJ_DBG_SKIP = 23,       /* u8[P]                partition has no R or no S tuple anywhere: not shuffled (a2) */
-    MGJ_DBG_TRACE = 24       /* u64[MGJ_TRACE_COUNT][2] (first start, last end) in ns of each kernel of
+    MGJ_DBG_TRACE = 24,      /* u64[MGJ_TRACE_COUNT][2] (first start, last end) in ns of each kernel of
                                 the last run (globaltimer; 0 = not run); needs mgj_config.trace = 1 */
+    MGJ_DBG_MID_OFF_S = 25   /* as MID_OFF_R, of MID_S */
 } mgj_debug_what;
 
 /* Trace slots (MGJ_DBG_TRACE), in pipeline order. */

@@ -31,6 +31,7 @@ constexpr int PROBE_HEAD8 = 128;        // headroom: co-partition target = capac
 constexpr int PROBE_MAXP = 1024;        // chunk pieces per relation per item
 constexpr int MAX_BA = 6;               // two-level local partitioning: at most 2^6 sub-partitions per pass A
 constexpr int LOCAL2_NCH = 256;         // a partition of more chunks than this gets the first local pass
+constexpr int EA_STRIDE = (1 << MAX_BA) + 1;  // first-pass run offsets per chunk (2^BA runs + the end)
 // sub-partitions of a first local pass: at most local2_vcap(P) in total
 __host__ __device__ constexpr int local2_vcap(int P) { return 4 * P > 4096 ? 4 * P : 4096; }
 constexpr uint64_t WAIT_TIMEOUT_NS = 20ull * 1000 * 1000 * 1000;  // default peer-signal wait bound
@@ -127,9 +128,9 @@ struct Ctx {
     uint64_t recv_cap_u[2];       // compressed shuffle: receive capacity in 32-byte units
     uint64_t max_chunks;
     uint64_t out_cap;
-    uint64_t mid_cap;             // slots of each first-pass output buffer
+    uint64_t mid_cap;             // slots of each first-pass output buffer (max_chunks * chunk_region1)
     int32_t vcap;                 // local2_vcap(P)
-    int32_t cb_stride;            // entries per relation of chunk_base, vstart (vcap + 1)
+    int32_t cb_stride;            // entries per relation of chunk_base, chunk_base1 (vcap + 1)
     int32_t split_cfg;            // mgj_config.local_split_bits
     Arena lay;
     char *arena[MAX_RANKS];       // arena bases as mapped in this process
@@ -160,9 +161,10 @@ struct Ctx {
     uint64_t *ext_counts;         // [2 (send, recv)][2 rel][MAX_RANKS] (EXTERNAL shuffle)
     uint32_t *chunk_base;         // [2][cb_stride] first chunk of each (sub-)partition of the chunked pass
     uint32_t *hA;                 // [2][vcap] first local pass: padded slots per sub-partition
-    uint64_t *vstart;             // [2][vcap+1] sub-partition start (slots) in mid
-    unsigned long long *vcur;     // [2][vcap+1] write cursor of each sub-partition
-    void *mid[2];                 // first local pass output (sub-partitions, contiguous)
+    uint32_t *chunk_base1;        // [2][cb_stride] first chunk of each owned partition in the first pass
+    uint16_t *eoffA[2];           // [chunks][EA_STRIDE] first pass: run offsets in each chunk's output
+    void *mid[2];                 // first local pass output: chunk li at slot li * chunk_region1
+    int32_t chunk_region1;        // slots per first-pass chunk region (chunk_tuples1s + 2^MAX_BA, even)
     uint16_t *eoff[2];            // run offsets, [(Q+1)*chunk_base[p] + q*nch_p + k]
     uint32_t *cop_slots;          // [2][P][2^b2_max] padded slots per co-partition
     Item *items;                  // [max_items]

@@ -744,16 +744,19 @@ __global__ void __launch_bounds__(1024) k_plan(Ctx c) {
     if (tid == 0) {
         // two-level local partitioning: when the owned
         // partitions span more than LOCAL2_NCH chunks on average, a first
-        // histogram-based pass splits every owned partition into 2^BA
-        // contiguous sub-partitions of ~64 chunks, and the chunked pass then
-        // uses the remaining B2 - BA bits.  The mean, not the maximum: a few
+        // pass splits every owned partition into 2^BA sub-partitions (runs
+        // stored in place per chunk), and the chunked pass then gathers each
+        // sub-partition's runs and uses the remaining B2 - BA bits.  The mean, not the maximum: a few
         // heavy-hitter partitions (Zipf) are not helped by splitting the rest
         const uint32_t meannch = np ? (max(nch[0], nch[1]) + np - 1) / np : 0;
         int BA = 0;
         if (c.split_cfg > 0) {
             BA = c.split_cfg;
         } else if (c.split_cfg == 0 && meannch > (uint32_t)LOCAL2_NCH) {
-            BA = ceil_log2_u64((meannch + 63) / 64);  // measured at N=8-sized partitions: BA 3 > 4 > 2
+            // sub-partitions of ~32 chunks; measured at N=8-sized partitions (B1 = 7, mean
+            // 341 chunks): BA 4 12.13 ms > 3 12.30 > 5 12.42 > 2 13.34 (round 1, with a
+            // counting pass and contiguous sub-partitions: 3 > 4 > 2)
+            BA = ceil_log2_u64((meannch + 31) / 32);
             while (BA > 0 && (np << BA) > c.vcap) --BA;
         }
         if (BA > B2) BA = B2;

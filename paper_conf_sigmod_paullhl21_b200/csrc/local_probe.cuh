@@ -162,70 +162,37 @@ __device__ inline void stream_wait(const Ctx &c, uint32_t w) {
 // partition of nch chunks leaves each co-partition in nch runs of ~C/Q
 // tuples.  At N = 8 (M2) an owner's partitions are 8x larger than at N = 1
 // and the runs shrink to a dozen tuples, which the probe cannot fetch
-// efficiently.  Then (k_plan sets BA > 0) a first pass splits every owned
-// partition by the BA key bits above B1 into 2^BA contiguous sub-partitions
-// (k_countA: padded sizes; k_planA: extents; k_local<K, true>: the chunked
-// sort with one bulk store per run at a reserved offset), and the chunked
-// pass runs on the sub-partitions with the remaining B2 - BA bits.
+// efficiently.  Then (k_plan sets BA > 0) a first pass (k_local_split, the
+// chunked sort by the BA key bits above B1, each chunk stored in place with
+// its run offsets, like the paper's histogram-free local pass) leaves every
+// (owned partition, BA-bit digit) sub-partition v as one run per chunk of
+// ~C/2^BA tuples; k_planA numbers the chunks of the second pass (ceil of each
+// sub-partition's padded size, counted by the first pass, over C2), k_emit2
+// cuts each sub-partition's runs into those chunks, and the chunked pass
+// (k_local_second) gathers a chunk's runs by bulk copies and partitions it by
+// the remaining B2 - BA bits.  No pass only counts.
 // ---------------------------------------------------------------------------
 __device__ __forceinline__ uint32_t nch_local(const Ctx &c, int rel) {
     return (uint32_t)c.meta[c.meta[MT_BA] ? MT_NCHB_R + rel : MT_NCH_R + rel];
 }
 
-// Padded size (slots) of every (owned partition, first-pass digit) run, summed
-// over the chunks of the partition: exactly the slots k_local<K, LM_SPLIT>
-// reserves.  QA <= 32: each thread counts its <= 24 tuples
-// of a chunk in eight 8-bit fields of one register, reduced per warp once per
-// chunk; larger QA: warp-aggregated shared atomics (one per distinct digit).
-// Per-thread digit counts of one chunk in NA packed registers (eight 8-bit
-// fields each: digit q -> register q / 8, field q % 8; a thread sees at most
-// C / 512 <= 24 tuples), reduced per warp into the shared counters.
-template <int NA, typename Tup>
-__device__ __forceinline__ void count_packed(const Tup *src, uint32_t len, int tid, uint32_t nt, int lane, int B1,
-                                             int QA, uint32_t *cnt) {
-    unsigned long long acc[NA];
-#pragma unroll
-    for (int a = 0; a < NA; ++a) acc[a] = 0;
-#define MGJ_COUNT_ADD(qq)                                                  \
-    do {                                                                   \
-        const uint32_t q_ = (qq);                                          \
-        const unsigned long long one_ = 1ull << (8 * (q_ & 7u));           \
-        _Pragma("unroll") for (int a_ = 0; a_ < NA; ++a_) acc[a_] += (q_ >> 3) == (uint32_t)a_ ? one_ : 0ull; \
-    } while (0)
-    uint32_t i = tid;
-    for (; i + 3 * nt < len; i += 4 * nt) {
-        const auto k0 = __ldcs(&src[i].x), k1 = __ldcs(&src[i + nt].x);
-        const auto k2 = __ldcs(&src[i + 2 * nt].x), k3 = __ldcs(&src[i + 3 * nt].x);
-        MGJ_COUNT_ADD(digit2(k0, B1, QA));
-        MGJ_COUNT_ADD(digit2(k1, B1, QA));
-        MGJ_COUNT_ADD(digit2(k2, B1, QA));
-        MGJ_COUNT_ADD(digit2(k3, B1, QA));
-    }
-    for (; i < len; i += nt) MGJ_COUNT_ADD(digit2(__ldcs(&src[i].x), B1, QA));
-#undef MGJ_COUNT_ADD
-#pragma unroll
-    for (int a = 0; a < NA; ++a)
-#pragma unroll
-        for (int f = 0; f < 8; ++f) {
-            const int q = a * 8 + f;
-            if (q < QA) {
-                const uint32_t v = __reduce_add_sync(0xffffffffu, (uint32_t)(acc[a] >> (8 * f)) & 0xffu);
-                if (lane == 0 && v) atomicAdd(&cnt[q], v);
-            }
-        }
-}
+// A chunk of the second pass: the slots [(k0, a0), (k1, a1)) of sub-partition
+// v's runs, run k being sub-partition v's run in first-pass chunk k (chunk
+// indices of the relation, ascending), a a slot offset inside it.
+struct ChunkDescB {
+    uint32_t v, k0, a0, k1, a1, len;
+};
 
-// Extents of the sub-partitions in mid (exclusive scan of the padded sizes)
-// and the chunk table of the chunked pass over them.  One CTA.  (Run by the
-// last CTA of k_countA instead, measured 0.28-0.47 ms slower at B1 = 7: the
-// planner's registers and shared memory cut k_countA's occupancy.)
+// Chunk table of the second pass: first chunk of every sub-partition v (the
+// exclusive scan of ceil(padded size / C2)); the first pass's table of the
+// owned partitions is kept in chunk_base1 for k_emit2.  One CTA.
 __global__ void __launch_bounds__(1024) k_planA(Ctx c) {
     extern __shared__ uint64_t sv[];  // [L+1] then u32 [L+1]
     __shared__ uint64_t tmp[33];
     __shared__ uint32_t tmp32[33];
     if (!c.meta[MT_OK] || !c.meta[MT_BA]) return;
     const int BA = c.meta[MT_BA];
-    const int L = c.meta[MT_NP] << BA;
+    const int np = c.meta[MT_NP], L = np << BA;
     const int tid = threadIdx.x;
     uint32_t *nch = reinterpret_cast<uint32_t *>(sv + L + 1);
     const uint64_t C = (uint64_t)c.chunk_tuples2;  // the chunked pass after the first pass
@@ -233,21 +200,16 @@ __global__ void __launch_bounds__(1024) k_planA(Ctx c) {
     bool bad = false;
     for (int rel = 0; rel < 2; ++rel) {
         const uint32_t *h = c.hA + (size_t)rel * c.vcap;
+        uint32_t *cb = c.chunk_base + (size_t)rel * c.cb_stride;
+        for (int i = tid; i <= np; i += blockDim.x) c.chunk_base1[(size_t)rel * c.cb_stride + i] = cb[i];
         for (int v = tid; v <= L; v += blockDim.x) {
             const uint32_t n = v < L ? __ldcg(h + v) : 0;
-            sv[v] = n;
             nch[v] = (uint32_t)((n + C - 1) / C);
         }
-        __syncthreads();
-        const uint64_t slots = block_excl_scan_u64(sv, L + 1, tmp);
+        __syncthreads();  // (the first pass's table is copied before it is overwritten)
         tot_ch[rel] = block_excl_scan_u32(nch, L + 1, tmp32);
-        bad |= slots > c.mid_cap || tot_ch[rel] > c.max_chunks;
-        uint64_t *vs = c.vstart + (size_t)rel * c.cb_stride;
-        for (int v = tid; v <= L; v += blockDim.x) {
-            vs[v] = sv[v];
-            if (v < L) c.vcur[(size_t)rel * c.cb_stride + v] = sv[v];
-            c.chunk_base[(size_t)rel * c.cb_stride + v] = nch[v];
-        }
+        bad |= tot_ch[rel] > c.max_chunks;
+        for (int v = tid; v <= L; v += blockDim.x) cb[v] = nch[v];
         __syncthreads();
     }
     if (tid == 0) {
@@ -259,46 +221,65 @@ __global__ void __launch_bounds__(1024) k_planA(Ctx c) {
             c.meta[MT_OK] = 0;
         }
     }
+    (void)tmp;
 }
 
-// First local pass, step 1 (only when k_plan chose BA > 0; a no-op
-// otherwise): padded size of every (owned partition, BA-bit digit) run over
-// the chunks of the partition, exactly the slots k_local<K, LM_SPLIT>
-// reserves.
+// The second pass's chunk descriptors: one warp per (relation, sub-partition
+// v) walks v's runs in first-pass chunk order (32 at a time, a warp scan of
+// their padded sizes) and cuts them at every multiple of C2: chunk s of v is
+// the slots [s * C2, min((s + 1) * C2, total)) of the concatenated runs.
 template <typename K>
-__global__ void __launch_bounds__(512) k_countA(Ctx c, const ChunkDesc *cdesc) {
-    using Tup = typename Layout<K>::Tup;
+__global__ void k_emit2(Ctx c, ChunkDescB *descB) {
     constexpr int ALIGN = Layout<K>::ALIGN;
-    __shared__ uint32_t cnt[1 << MAX_BA];
     if (!c.meta[MT_OK] || !c.meta[MT_BA]) return;
     const int BA = c.meta[MT_BA], QA = 1 << BA;
-    const uint32_t nch_r = (uint32_t)c.meta[MT_NCH_R], total = nch_r + (uint32_t)c.meta[MT_NCH_S];
-    const int tid = threadIdx.x, lane = tid & 31;
-    const uint32_t nt = blockDim.x;
-    for (uint32_t ci = blockIdx.x; ci < total; ci += gridDim.x) {
-        const int rel = ci < nch_r ? 0 : 1;
-        const ChunkDesc d = cdesc[ci];
-        const Tup *src = reinterpret_cast<const Tup *>(c.arena[piece_src(d.start)] + c.lay.recv[rel]) + piece_off(d.start);
-        if (tid < QA) cnt[tid] = 0;
-        __syncthreads();
-        if (QA <= 8) {
-            count_packed<1>(src, d.len, tid, nt, lane, c.B1, QA, cnt);
-        } else if (QA <= 16) {
-            count_packed<2>(src, d.len, tid, nt, lane, c.B1, QA, cnt);
-        } else if (QA <= 32) {
-            count_packed<4>(src, d.len, tid, nt, lane, c.B1, QA, cnt);
-        } else {
-            for (uint32_t i = tid; i < d.len; i += nt) {
-                const uint32_t q = digit2(__ldcs(&src[i].x), c.B1, QA);
-                const uint32_t peers = __match_any_sync(__activemask(), q);
-                if (lane == __ffs(peers) - 1) atomicAdd(&cnt[q], __popc(peers));
+    const int L = c.meta[MT_NLP];
+    const uint32_t C2 = (uint32_t)c.chunk_tuples2;
+    const uint32_t nchb_r = (uint32_t)c.meta[MT_NCHB_R];
+    const int lane = threadIdx.x & 31;
+    const uint32_t warps = (gridDim.x * blockDim.x) >> 5;
+    for (uint32_t w = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; w < 2u * (uint32_t)L; w += warps) {
+        const int rel = w >= (uint32_t)L, v = (int)(w - (rel ? L : 0));
+        const int pi = v >> BA, a = v & (QA - 1);
+        const uint32_t *cb1 = c.chunk_base1 + (size_t)rel * c.cb_stride;
+        const uint32_t kb = __ldcg(cb1 + pi), ke = __ldcg(cb1 + pi + 1);
+        const uint32_t out0 = (rel ? nchb_r : 0u) + __ldcg(c.chunk_base + (size_t)rel * c.cb_stride + v);
+        const uint16_t *E = c.eoffA[rel];
+        uint32_t pre = 0;  // slots of v's runs before this batch
+        for (uint32_t k0 = kb; k0 < ke; k0 += 32) {
+            const uint32_t k = k0 + lane;
+            uint32_t slots = 0, st = 0, valid = 0;
+            if (k < ke) decode_run<ALIGN>(E[(size_t)k * EA_STRIDE + a], E[(size_t)k * EA_STRIDE + a + 1], st, slots, valid);
+            uint32_t incl = slots;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const uint32_t y = __shfl_up_sync(0xffffffffu, incl, o);
+                if (lane >= o) incl += y;
             }
+            const uint32_t lo = pre + incl - slots, hi = pre + incl;  // this run: [lo, hi) of v's slots
+            // every chunk boundary s * C2 inside [lo, hi): chunk s starts here, chunk s - 1 ends here
+            for (uint32_t s = (lo + C2 - 1) / C2; s * C2 < hi; ++s) {
+                ChunkDescB *d = descB + out0 + s;
+                d->v = (uint32_t)v;
+                d->k0 = k;
+                d->a0 = s * C2 - lo;
+                if (s > 0) {
+                    ChunkDescB *e = d - 1;
+                    e->k1 = k;
+                    e->a1 = s * C2 - lo;
+                    e->len = C2;
+                }
+            }
+            pre += __shfl_sync(0xffffffffu, incl, 31);
+            (void)valid;
         }
-        __syncthreads();
-        if (tid < QA && cnt[tid])
-            atomicAdd(&c.hA[(size_t)rel * c.vcap + ((size_t)d.pi << BA) + tid],
-                      (cnt[tid] + ALIGN - 1) & ~(uint32_t)(ALIGN - 1));
-        __syncthreads();
+        if (lane == 0 && pre > 0) {  // the last chunk ends after v's last run
+            const uint32_t s = (pre - 1) / C2;
+            ChunkDescB *d = descB + out0 + s;
+            d->k1 = ke;
+            d->a1 = 0;
+            d->len = pre - s * C2;
+        }
     }
 }
 
@@ -316,27 +297,34 @@ __global__ void __launch_bounds__(512) k_countA(Ctx c, const ChunkDesc *cdesc) {
 //  MODE = LM_SINGLE (the only pass, BA = 0) / LM_SECOND (after a first
 //    pass): the chunked pass.  digit = the B2 - BA key bits above B1 + BA,
 //    one bulk store per chunk, run offsets to E[(Q+1)*chunk_base[v] +
-//    q*nch_v + k] (contiguous per (v, q)).  LM_SECOND reads the
-//    sub-partitions and drops the first pass's padding tuples (digit1 != p).
+//    q*nch_v + k] (contiguous per (v, q)).  LM_SECOND gathers its chunk from
+//    the first pass's runs of sub-partition v (k_emit2's descriptors, one
+//    bulk copy per run piece) and drops the first pass's padding tuples
+//    (digit1 != p).
 //  MODE = LM_SPLIT (first pass of two-level partitioning): digit = the BA
-//    bits above B1; every run is stored by its own bulk copy at an offset
-//    reserved in its sub-partition's extent (k_planA).
+//    bits above B1; the sorted chunk is stored in place (chunk li at
+//    mid + li * chunk_region1) with its run offsets in eoffA, and each run's
+//    padded size is added to its sub-partition's total (hA).
 // Each instance returns at once when the run's BA does not select it.
 // R co-partitions larger than the table are built in pieces by a5
 // (P:450-452's skew case).
 // ---------------------------------------------------------------------------
 enum LocalMode { LM_SINGLE = 0, LM_SPLIT = 1, LM_SECOND = 2 };
 
+template <int MODE> struct LocalDesc { using T = ChunkDesc; };
+template <> struct LocalDesc<2> { using T = ChunkDescB; };
+
 template <typename K, int MODE, int RSEL = 2, bool COMP = false, bool STRM = false>
-__device__ __forceinline__ void local_body(const Ctx &c, const ChunkDesc *cdesc) {
+__device__ __forceinline__ void local_body(const Ctx &c, const typename LocalDesc<MODE>::T *cdesc) {
     static_assert(!COMP || (MODE == LM_SINGLE && sizeof(K) == 4), "compressed input: single pass, 4-byte keys");
+    using Desc = typename LocalDesc<MODE>::T;
     constexpr bool SPLIT = MODE == LM_SPLIT;
     using Tup = typename Layout<K>::Tup;
     constexpr int TB = Layout<K>::TB, ALIGN = Layout<K>::ALIGN;
     constexpr int VMAX = local_vmax(TB);
     extern __shared__ __align__(128) unsigned char smem[];
     __shared__ __align__(8) uint64_t bar[2];
-    __shared__ ChunkDesc sdesc[2];
+    __shared__ Desc sdesc[2];
     __shared__ uint32_t tmp[33];
     const int BA = MODE == LM_SINGLE ? 0 : c.meta[MT_BA];
     const int tid = threadIdx.x;
@@ -367,10 +355,9 @@ __device__ __forceinline__ void local_body(const Ctx &c, const ChunkDesc *cdesc)
         return c0 + (strm ? __ldcg(c.corder + k) : k);
     };
     constexpr bool from_mid = MODE == LM_SECOND;
-    // source of a chunk: the first pass's output, or a receive buffer (this
-    // rank's, or a broadcast partition root's for its R side: piece_src)
+    // source of a chunk: a receive buffer (this rank's, or a broadcast
+    // partition root's for its R side: piece_src)
     auto chunk_src = [&](int rel, uint64_t start) -> const Tup * {
-        if (from_mid) return static_cast<const Tup *>(c.mid[rel]) + start;
         return reinterpret_cast<const Tup *>(c.arena[piece_src(start)] + c.lay.recv[rel]) + piece_off(start);
     };
     if (tid == 0) {
@@ -382,13 +369,48 @@ __device__ __forceinline__ void local_body(const Ctx &c, const ChunkDesc *cdesc)
     __syncthreads();
     const uint64_t pol = policy_evict_first();
     // thread 0: TMA chunk j (16-byte-aligned superset) into buffer j & 1
-    auto issue = [&](uint32_t j, const ChunkDesc &d) {
+    auto issue = [&](uint32_t j, const Desc &d) {
         const uint32_t ci = cidx(j);
         const int rel = ci < nch_r ? 0 : 1;
         if (strm) stream_wait(c, __ldcg(c.cwait + (ci - c0)));
         sdesc[j & 1] = d;
         uint64_t *b = &bar[j & 1];
-        if constexpr (COMP) {  // whole 32-byte units
+        if constexpr (from_mid) {
+            // the pieces of sub-partition d.v's runs, back to back: the issuing
+            // warp's lanes take 32 runs at a time (their offsets loaded in
+            // parallel, destinations by a warp scan), each lane its own copy
+            const int lane = tid & 31;
+            if (lane == 0) mbar_arrive_expect_tx(b, d.len * TB);
+            __syncwarp();
+            const int a = (int)(d.v & ((1u << BA) - 1));
+            const uint16_t *E = c.eoffA[rel];
+            const Tup *mid = static_cast<const Tup *>(c.mid[rel]);
+            uint32_t at = 0;
+            for (uint32_t kb = d.k0; kb <= d.k1; kb += 32) {
+                const uint32_t k = kb + lane;
+                uint32_t pc = 0;
+                size_t src = 0;
+                if (k <= d.k1 && !(k == d.k1 && d.a1 == 0)) {
+                    uint32_t st, slots, valid;
+                    decode_run<ALIGN>(__ldcg(E + (size_t)k * EA_STRIDE + a), __ldcg(E + (size_t)k * EA_STRIDE + a + 1), st,
+                                      slots, valid);
+                    const uint32_t alo = k == d.k0 ? d.a0 : 0u, ahi = k == d.k1 ? d.a1 : slots;
+                    if (ahi > alo) {
+                        pc = ahi - alo;
+                        src = (size_t)k * c.chunk_region1 + st + alo;
+                    }
+                }
+                uint32_t incl = pc;
+#pragma unroll
+                for (int o = 1; o < 32; o <<= 1) {
+                    const uint32_t y = __shfl_up_sync(0xffffffffu, incl, o);
+                    if (lane >= o) incl += y;
+                }
+                if (pc) tma_load_1d(buf(j & 1) + at + incl - pc, mid + src, pc * TB, b, pol);
+                at += __shfl_sync(0xffffffffu, incl, 31);
+            }
+            return;
+        } else if constexpr (COMP) {  // whole 32-byte units
             const uint32_t bytes = d.len * 32u;
             mbar_arrive_expect_tx(b, bytes);
             if (bytes)
@@ -396,16 +418,20 @@ __device__ __forceinline__ void local_body(const Ctx &c, const ChunkDesc *cdesc)
                             pol);
             return;
         }
-        const uint64_t st = from_mid ? d.start : piece_off(d.start);
-        const uint64_t g0 = st & ~(uint64_t)(ALIGN - 1);
-        const uint64_t g1 = (st + d.len + ALIGN - 1) & ~(uint64_t)(ALIGN - 1);
-        const uint32_t bytes = (uint32_t)((g1 - g0) * TB);
-        mbar_arrive_expect_tx(b, bytes);
-        if (bytes) tma_load_1d(buf(j & 1), chunk_src(rel, d.start) - (st - g0), bytes, b, pol);
+        else {
+            const uint64_t st = piece_off(d.start);
+            const uint64_t g0 = st & ~(uint64_t)(ALIGN - 1);
+            const uint64_t g1 = (st + d.len + ALIGN - 1) & ~(uint64_t)(ALIGN - 1);
+            const uint32_t bytes = (uint32_t)((g1 - g0) * TB);
+            mbar_arrive_expect_tx(b, bytes);
+            if (bytes) tma_load_1d(buf(j & 1), chunk_src(rel, d.start) - (st - g0), bytes, b, pol);
+        }
     };
-    ChunkDesc nxt{};
+    Desc nxt{};
     constexpr int LI = 32;  // the thread that issues the chunk loads (and the chunked pass's stores)
-    if (tid == LI) {
+    // (the second pass issues its run pieces with the whole of LI's warp)
+    auto issuer = [&]() { return from_mid ? (tid >> 5) == (LI >> 5) : tid == LI; };
+    if (issuer()) {
         if (mine > 0) issue(0, cdesc[cidx(0)]);
         if (mine > 1) nxt = cdesc[cidx(1)];
     }
@@ -416,10 +442,17 @@ __device__ __forceinline__ void local_body(const Ctx &c, const ChunkDesc *cdesc)
         const int X = j & 1;
         uint32_t *const bins = bins2 + X * QL;  // zero (cleared during chunk j - 1)
         mbar_wait(&bar[X], (j >> 1) & 1);
-        const ChunkDesc d = sdesc[X];
-        const uint32_t len = d.len, skip = (uint32_t)(d.start & (ALIGN - 1));
+        const Desc d = sdesc[X];
+        uint32_t skip = 0, dpi = 0;  // slots before the chunk's first tuple; its (sub-)partition
+        if constexpr (from_mid) {
+            dpi = d.v;
+        } else {
+            skip = (uint32_t)(d.start & (ALIGN - 1));
+            dpi = d.pi;
+        }
+        const uint32_t len = d.len;
         // partition of this chunk's tuples (a first pass's padding tuples lie in another one)
-        const uint32_t p = (uint32_t)c.plist[from_mid ? d.pi >> BA : d.pi];
+        const uint32_t p = (uint32_t)c.plist[from_mid ? dpi >> BA : dpi];
         Tup t[VMAX];
         uint32_t cvalid = 0;  // COMP: bit v set if t[v] holds a decoded tuple
         if constexpr (COMP) {
@@ -466,12 +499,12 @@ __device__ __forceinline__ void local_body(const Ctx &c, const ChunkDesc *cdesc)
                 rq[v] = (atomicAdd(&bins[q], 1u) << 16) | q;
             }
         }
-        if (SPLIT && tid < Q) bulk_wait_read0();  // run stores of chunk j-1 have read buffer X^1
         __syncthreads();  // S1: buffer X consumed (it becomes this chunk's sorted output), bins final
         // chunk j+1 -> buffer X^1 once chunk j-1's stores have read it; the issuing
         // thread (warp 1, LI) also issues the chunk's bulk store, warp 0 scans meanwhile
-        if (tid == LI && j + 1 < mine) {
-            if (!SPLIT) bulk_wait_read0();
+        if (issuer() && j + 1 < mine) {
+            if (tid == LI) bulk_wait_read0();
+            if (from_mid) __syncwarp();
             issue(j + 1, nxt);
             if (j + 2 < mine) nxt = cdesc[cidx(j + 2)];
         }
@@ -498,11 +531,24 @@ __device__ __forceinline__ void local_body(const Ctx &c, const ChunkDesc *cdesc)
         }
         __syncthreads();  // S2b
         const uint32_t tot = tmp[0];
-        if (!SPLIT) {
+        if (SPLIT) {  // run offsets of the chunk stored in place; padded run sizes per sub-partition
+            uint16_t *E = c.eoffA[rel] + (size_t)li * EA_STRIDE;
+            for (int q = tid; q <= Q; q += LOCAL_THREADS) {
+                if (q < Q) {
+                    const uint32_t n = bins[q];
+                    E[q] = (uint16_t)(abin[q] | (ALIGN == 2 ? (n & 1u) : 0u));
+                    if (n)
+                        atomicAdd(&c.hA[(size_t)rel * c.vcap + ((size_t)dpi << BA) + q],
+                                  (n + ALIGN - 1) & ~(uint32_t)(ALIGN - 1));
+                } else {
+                    E[q] = (uint16_t)tot;
+                }
+            }
+        } else {
             const uint32_t *cb = c.chunk_base + (size_t)rel * c.cb_stride;
-            const uint32_t cbp = cb[d.pi], nchp = cb[d.pi + 1] - cbp;
+            const uint32_t cbp = cb[dpi], nchp = cb[dpi + 1] - cbp;
             uint16_t *E = c.eoff[rel] + (size_t)(Q + 1) * cbp + (li - cbp);
-            uint32_t *cop = c.cop_slots + (size_t)rel * P * Qmax + (size_t)d.pi * Q;
+            uint32_t *cop = c.cop_slots + (size_t)rel * P * Qmax + (size_t)dpi * Q;
             for (int q = tid; q <= Q; q += LOCAL_THREADS) {
                 if (q < Q) {
                     const uint32_t n = bins[q];
@@ -533,16 +579,9 @@ __device__ __forceinline__ void local_body(const Ctx &c, const ChunkDesc *cdesc)
         }
         fence_proxy_async_smem();
         __syncthreads();  // S3
-        if (SPLIT) {
-            if (tid < Q && bins[tid]) {  // one bulk store per run, at a reserved offset of its sub-partition
-                const uint32_t slots = (bins[tid] + ALIGN - 1) & ~(uint32_t)(ALIGN - 1);
-                const unsigned long long at =
-                    atomicAdd(&c.vcur[(size_t)rel * c.cb_stride + ((size_t)d.pi << BA) + tid], slots);
-                tma_store_1d(static_cast<Tup *>(c.mid[rel]) + at, sorted + abin[tid], slots * TB);
-                bulk_commit();
-            }
-        } else if (tid == LI && tot) {
-            Tup *dst = static_cast<Tup *>(c.local[rel]) + (size_t)li * CR;
+        if (tid == LI && tot) {  // the sorted chunk in place: first pass -> mid, else -> local
+            Tup *dst = SPLIT ? static_cast<Tup *>(c.mid[rel]) + (size_t)li * c.chunk_region1
+                             : static_cast<Tup *>(c.local[rel]) + (size_t)li * CR;
             tma_store_1d(dst, sorted, tot * TB);
             bulk_commit();
         }
@@ -550,47 +589,19 @@ __device__ __forceinline__ void local_body(const Ctx &c, const ChunkDesc *cdesc)
     bulk_wait0();
 }
 
-// Chunk descriptors of the chunked pass over the sub-partitions (one piece
-// each): chunk li of relation rel lies in the sub-partition v whose chunk
-// range [chunk_base[v], chunk_base[v + 1]) holds it.
-__device__ inline void chunkmap_second(const Ctx &c, ChunkDesc *desc) {
-    const int L = c.meta[MT_NLP];
-    const uint32_t nch_r = (uint32_t)c.meta[MT_NCHB_R], total = nch_r + (uint32_t)c.meta[MT_NCHB_S];
-    const uint64_t C = (uint64_t)c.chunk_tuples2;  // the chunked pass after the first pass
-    for (uint32_t ci = blockIdx.x * blockDim.x + threadIdx.x; ci < total; ci += gridDim.x * blockDim.x) {
-        const int rel = ci < nch_r ? 0 : 1;
-        const uint32_t li = rel ? ci - nch_r : ci;
-        const uint32_t *cb = c.chunk_base + (size_t)rel * c.cb_stride;
-        int lo = 0, hi = L - 1;
-        while (lo < hi) {
-            const int mid = (lo + hi + 1) >> 1;
-            if (__ldcg(cb + mid) <= li) lo = mid; else hi = mid - 1;
-        }
-        const uint64_t k = li - __ldcg(cb + lo);
-        const uint64_t *vs = c.vstart + (size_t)rel * c.cb_stride;
-        ChunkDesc d;
-        d.start = __ldcg(vs + lo) + k * C;
-        d.len = (uint32_t)min(C, __ldcg(vs + lo + 1) - d.start);
-        d.pi = (uint32_t)lo;
-        desc[ci] = d;
-    }
-}
-
 // The first pass of two-level local partitioning (a no-op unless k_plan chose
-// BA > 0).  Its CTAs also write the chunked pass's chunk descriptors (they
-// depend only on k_countA's layout, not on this pass's output).
+// BA > 0).
 template <typename K>
-__global__ void __launch_bounds__(LOCAL_THREADS, 1) k_local_split(Ctx c, const ChunkDesc *cdesc, ChunkDesc *descB) {
+__global__ void __launch_bounds__(LOCAL_THREADS, 1) k_local_split(Ctx c, const ChunkDesc *cdesc) {
     if (!c.meta[MT_OK] || !c.meta[MT_BA]) return;
     trace_begin(c, MGJ_TR_LOCAL_SPLIT);
-    chunkmap_second(c, descB);
     local_body<K, LM_SPLIT>(c, cdesc);
     trace_end(c, MGJ_TR_LOCAL_SPLIT);
 }
 
 // The chunked pass over the first pass's sub-partitions (a no-op when BA = 0).
 template <typename K>
-__global__ void __launch_bounds__(LOCAL_THREADS, 1) k_local_second(Ctx c, const ChunkDesc *descB) {
+__global__ void __launch_bounds__(LOCAL_THREADS, 1) k_local_second(Ctx c, const ChunkDescB *descB) {
     if (!c.meta[MT_OK] || !c.meta[MT_BA]) return;
     trace_begin(c, MGJ_TR_LOCAL_SECOND);
     local_body<K, LM_SECOND>(c, descB);

@@ -118,7 +118,8 @@ mgj_status normalize(const mgj_config *in, Norm *o) {
     // the first local pass exists if forced, or (auto) if one owned partition could
     // span more than LOCAL2_NCH chunks; its output pads each (chunk, run) once
     o->split = c.local_split_bits > 0 || (c.local_split_bits == 0 && rmax > (uint64_t)LOCAL2_NCH * C);
-    o->mid_cap = o->split ? rmax + (rmax / C + o->P + 2) * (1ull << MAX_BA) : 0;
+    // the first pass stores every chunk in place: a region of C1s + 2^MAX_BA slots per chunk
+    o->mid_cap = o->split ? o->max_chunks * (uint64_t)(o->chunk_tuples1s + (1 << MAX_BA)) : 0;
     o->max_items = (uint64_t)o->P * Qm + o->recv_cap[1] / (o->probe_slots / 2) * 2 +
                    o->recv_cap[0] / (o->probe_slots / 2) * 2 + 4096;
     if (o->max_items > 0x7fffffffull) o->max_items = 0x7fffffffull;
@@ -171,7 +172,7 @@ struct mgj_plan_s {
     int nalloc = 0;
     Ctx ctx{};
     ChunkDesc *cdesc = nullptr;   // chunks of the (first) local pass, written by k_chunkmap
-    ChunkDesc *cdescB = nullptr;  // chunks of the chunked pass after a first pass (k_countA)
+    ChunkDescB *cdescB = nullptr;  // chunks of the chunked pass after a first pass (k_emit2)
     char *send_arena = nullptr;  // EXTERNAL shuffle
     uint64_t epoch = 0;
     int state = 0;
@@ -268,7 +269,7 @@ cudaError_t preload_kernels(const Norm &n) {
                        (const void *)k_chunkmap, (const void *)k_chunkorder, (const void *)scatter_kernel<K>(n.P),
                        (const void *)k_wait, (const void *)k_local<K, 0>, (const void *)k_local<K, 1>,
                        (const void *)k_local<K, 2>, (const void *)k_local<K, 1, false, true>,
-                       (const void *)k_countA<K>, (const void *)k_planA, (const void *)k_local_split<K>,
+                       (const void *)k_emit2<K>, (const void *)k_planA, (const void *)k_local_split<K>,
                        (const void *)k_local_second<K>, (const void *)k_itemize<K>, (const void *)k_probe<K, false>,
                        (const void *)k_probe<K, true>, (const void *)k_reduce};
     for (const void *fn : f)
@@ -361,11 +362,13 @@ void launch_join(mgj_plan_s *h, cudaStream_t s) {
     // it chooses one pass these four kernels return at once.  (Measured, not
     // kept: a guard kernel that tail-launches the chosen kernels from the
     // device costs 18 us; one kernel for both chunked passes spills, +0.1 ms at
-    // M2; k_planA run by k_countA's last CTA, +0.28 ms at B1 = 7.)
+    // M2; k_planA run by k_countA's last CTA, +0.28 ms at B1 = 7.)  Round 2: the
+    // first pass stores its chunks in place and counts the sub-partitions
+    // itself, so no counting pass reads the received data first.
     if (n.split) {
-        k_countA<K><<<h->nsm * 4, 512, 0, s>>>(h->ctx, h->cdesc);
+        k_local_split<K><<<h->nsm, LOCAL_THREADS, local_smem1s(n), s>>>(h->ctx, h->cdesc);
         k_planA<<<1, 1024, planA_smem(n), s>>>(h->ctx);
-        k_local_split<K><<<h->nsm, LOCAL_THREADS, local_smem1s(n), s>>>(h->ctx, h->cdesc, h->cdescB);
+        k_emit2<K><<<h->nsm * 4, 256, 0, s>>>(h->ctx, h->cdescB);
         k_local_second<K><<<h->nsm, LOCAL_THREADS, local_smem2(n), s>>>(h->ctx, h->cdescB);
         h->launches += 4;
     }
@@ -548,7 +551,7 @@ mgj_status mgj_plan(const mgj_config *cfg, const mgj_peers *peers, mgj_handle *o
         c.cwait = static_cast<uint32_t *>(dalloc(h, n.max_chunks * 4, &st));
         c.corder = static_cast<uint32_t *>(dalloc(h, n.max_chunks * 4, &st));
     }
-    if (n.split) h->cdescB = static_cast<ChunkDesc *>(dalloc(h, 2 * n.max_chunks * sizeof(ChunkDesc), &st));
+    if (n.split) h->cdescB = static_cast<ChunkDescB *>(dalloc(h, 2 * n.max_chunks * sizeof(ChunkDescB), &st));
     c.owner = static_cast<int32_t *>(dalloc(h, P * 4, &st));
     c.bcast = static_cast<uint8_t *>(dalloc(h, P, &st));
     c.pskip = static_cast<uint8_t *>(dalloc(h, P, &st));
@@ -571,9 +574,12 @@ mgj_status mgj_plan(const mgj_config *cfg, const mgj_peers *peers, mgj_handle *o
     c.split_cfg = n.c.local_split_bits;
     c.mid_cap = n.mid_cap;
     c.chunk_base = static_cast<uint32_t *>(dalloc(h, 2ull * c.cb_stride * 4, &st));
-    c.vstart = static_cast<uint64_t *>(dalloc(h, 2ull * c.cb_stride * 8, &st));
-    c.vcur = static_cast<unsigned long long *>(dalloc(h, 2ull * c.cb_stride * 8, &st));
-    for (int r = 0; r < 2 && n.split; ++r) c.mid[r] = dalloc(h, n.mid_cap * n.tuple_bytes, &st);
+    c.chunk_base1 = static_cast<uint32_t *>(dalloc(h, 2ull * c.cb_stride * 4, &st));
+    c.chunk_region1 = n.chunk_tuples1s + (1 << MAX_BA);
+    for (int r = 0; r < 2 && n.split; ++r) {
+        c.mid[r] = dalloc(h, n.mid_cap * n.tuple_bytes, &st);
+        c.eoffA[r] = static_cast<uint16_t *>(dalloc(h, n.max_chunks * EA_STRIDE * 2, &st));
+    }
     for (int r = 0; r < 2; ++r)
         c.eoff[r] = static_cast<uint16_t *>(dalloc(h, n.max_chunks * (Qm + 1) * 2, &st));
     c.items = static_cast<Item *>(dalloc(h, n.max_items * sizeof(ItemX), &st));
@@ -966,15 +972,18 @@ mgj_status mgj_debug_copy(mgj_handle h, int32_t what, void *dst, uint64_t bytes,
         case MGJ_DBG_MID_S: {
             if (!meta[MT_BA]) return MGJ_EINVAL;
             const int r = what == MGJ_DBG_MID_S;
-            const int L = meta[MT_NLP];
-            uint64_t end = 0;
-            if (cudaMemcpy(&end, c.vstart + (size_t)r * c.cb_stride + L, 8, cudaMemcpyDeviceToHost) != cudaSuccess)
-                return MGJ_ECUDA;
-            src = c.mid[r];
-            size = end * n.tuple_bytes;
+            src = c.mid[r];  // the first pass's chunks in place, chunk_region1 slots each
+            size = (uint64_t)meta[MT_NCH_R + r] * c.chunk_region1 * n.tuple_bytes;
             break;
         }
-        case MGJ_DBG_VSTART: src = c.vstart; size = 2ull * c.cb_stride * 8; break;
+        case MGJ_DBG_MID_OFF_R:
+        case MGJ_DBG_MID_OFF_S: {
+            if (!meta[MT_BA]) return MGJ_EINVAL;
+            const int r = what == MGJ_DBG_MID_OFF_S;
+            src = c.eoffA[r];
+            size = (uint64_t)meta[MT_NCH_R + r] * EA_STRIDE * 2;
+            break;
+        }
         case MGJ_DBG_TRACE: {
             if (!c.trace) return MGJ_EINVAL;
             unsigned long long t[MGJ_TRACE_COUNT * 2];

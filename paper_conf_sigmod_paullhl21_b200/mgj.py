@@ -27,8 +27,8 @@ MAX_RANKS = 8
 # mgj_debug_what
 DBG = dict(RANK_HIST=1, MAIL_HIST=2, OWNER=3, SEND_OFF=4, RECV_SIZE=5, RECV_R=6, RECV_S=7,
            LOCAL_R=8, LOCAL_S=9, META=10, CHUNK_OFF_R=11, CHUNK_OFF_S=12, CHUNK_BASE=13, SEGMENTS=14,
-           OUT_KEY=15, OUT_PAY_R=16, OUT_PAY_S=17, MID_R=18, MID_S=19, VSTART=20, BCAST=21, PLIST=22, SKIP=23,
-           TRACE=24)
+           OUT_KEY=15, OUT_PAY_R=16, OUT_PAY_S=17, MID_R=18, MID_S=19, MID_OFF_R=20, BCAST=21, PLIST=22, SKIP=23,
+           TRACE=24, MID_OFF_S=25)
 # trace slots (include/mgj_aux.h MGJ_TR_*), in pipeline order
 TRACE_NAMES = ["hist", "plan", "scatter_R", "scatter_S", "local_R", "local_S", "local_RS", "local_split",
                "local_second", "itemize", "probe", "reduce"]

@@ -162,9 +162,11 @@ def test_m1_parity_materialized(mgj):
 @pytest.mark.parametrize("ba", [1, 3, 6])
 def test_two_level_local_phases(mgj, ba):
     """Forced first local pass (BA bits) on M1 with B1 = 4 (16 partitions of
-    2^16): every sub-partition v = (p, qa) of MID holds exactly the received
-    tuples of p whose next BA key bits are qa, plus padding tuples of another
-    global partition (at most one per chunk run); the join stays exact."""
+    2^16): every first-pass chunk is stored in place as 2^BA runs; run a holds
+    only tuples whose next BA key bits are a (plus, for an odd run, one padding
+    tuple: its first tuple with a low key bit flipped, i.e. of another global
+    partition), and the runs of all chunks hold exactly the received tuples;
+    the join stays exact."""
     d = datagen.M1().rank_inputs()
     ref = oracle.join(d["r_keys"], d["r_pays"], d["s_keys"], d["s_pays"], materialize=False)
     j, res = run_one(mgj, d, radix_bits_global=4, local_split_bits=ba)
@@ -173,21 +175,27 @@ def test_two_level_local_phases(mgj, ba):
     B1, P = 4, 16
     BA, QB, L = int(meta[8]), int(meta[9]), int(meta[10])
     assert BA == min(ba, res["radix_bits_local"]) and QB == res["radix_bits_local"] - BA and L == P << BA
-    vstart = j.debug("VSTART", np.uint64).reshape(2, -1)
+    QA = 1 << BA
     for rel, name in ((0, "R"), (1, "S")):
         recv = j.debug("RECV_" + name, np.uint32).reshape(-1, 2)
         mid = j.debug("MID_" + name, np.uint32).reshape(-1, 2)
-        assert mid.shape[0] == int(vstart[rel, L])
-        for v in range(L):
-            p, qa = v >> BA, v & ((1 << BA) - 1)
-            seg = mid[int(vstart[rel, v]):int(vstart[rel, v + 1])]
-            real = seg[(seg[:, 0] & (P - 1)) == p]
-            pads = seg[(seg[:, 0] & (P - 1)) != p]
-            assert np.all(((real[:, 0] >> B1) & ((1 << BA) - 1)) == qa)
-            assert np.all((pads[:, 0] & (P - 1)) == (p ^ (2 if (rel == 1 and P >= 4) else 1)))
-            exp = recv[((recv[:, 0] & (P - 1)) == p) & (((recv[:, 0] >> B1) & ((1 << BA) - 1)) == qa)]
-            pack = lambda x: np.sort(x[:, 0].astype(np.uint64) | (x[:, 1].astype(np.uint64) << np.uint64(32)))
-            np.testing.assert_array_equal(pack(real), pack(exp))
+        E = j.debug("MID_OFF_" + name, np.uint16).reshape(-1, 65).astype(np.int64)
+        nch = E.shape[0]
+        assert nch == int(meta[4 + rel]) and mid.shape[0] % nch == 0
+        region = mid.shape[0] // nch
+        real = []
+        for k in range(nch):
+            for a in range(QA):
+                st, en = E[k, a] & ~1, E[k, a + 1] & ~1
+                valid = en - st - (E[k, a] & 1)
+                run = mid[k * region + st:k * region + en]
+                assert np.all(((run[:valid, 0] >> B1) & (QA - 1)) == a)
+                if valid < en - st:  # padding: the run's first tuple, a low key bit flipped
+                    assert run[valid, 0] == run[0, 0] ^ (2 if (rel == 1 and P >= 4) else 1)
+                real.append(run[:valid])
+        real = np.concatenate(real)
+        pack = lambda x: np.sort(x[:, 0].astype(np.uint64) | (x[:, 1].astype(np.uint64) << np.uint64(32)))
+        np.testing.assert_array_equal(pack(real), pack(recv))
     j.close()
 
 

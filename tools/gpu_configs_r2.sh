@@ -25,6 +25,8 @@ run m3_n2size "--log2-per-gpu 30"
 run m2_b1_7 "--radix-bits-global 7"
 run m2_compress "--compress"
 run m2_overlap "--overlap on"
+run m2_stream "--overlap stream"
+run m2_b1_7_mat "--radix-bits-global 7 --materialize"
 for k in 24 26 28; do run size_2p$k "--log2-per-gpu $k"; done
 run m2_b1_9 "--radix-bits-global 9"
 run m2_b2_6 "--radix-bits-local 6"

@@ -23,6 +23,7 @@ namespace {
 enum State { ST_PLANNED = 1, ST_PARTITIONED = 2, ST_SHUFFLED = 3, ST_JOINED = 4, ST_DONE = 5 };
 
 uint64_t align_up(uint64_t x, uint64_t a) { return (x + a - 1) / a * a; }
+constexpr int COMP_MAX_TILES = 1024;  // compressed shuffle: scatter tiles per relation and rank at most
 
 struct Norm {  // validated config with the automatic fields filled in
     mgj_config c;
@@ -142,10 +143,11 @@ mgj_status normalize(const mgj_config *in, Norm *o) {
     off = align_up(off + STREAM_RMAX * 8, 4096);
     // compressed: a (source rank, tile, partition) run ends in a partial unit, so
     // short runs take more room than their tuples (at most one unit per tuple);
-    // the bound counts <= 8 ranks x 256 tiles x P partial units
+    // the bound counts <= 8 ranks x COMP_MAX_TILES tiles x P partial units (mgj_plan
+    // rejects a plan with more tiles per relation: chunk streaming uses 4 per SM)
     for (int r = 0; r < 2; ++r)
         o->recv_cap_u[r] = c.compress ? std::min<uint64_t>(o->recv_cap[r], o->recv_cap[r] / CU_N + 1 +
-                                                                               (uint64_t)MAX_RANKS * 256 * o->P)
+                                                                               (uint64_t)MAX_RANKS * COMP_MAX_TILES * o->P)
                                       : 0;
     auto recv_bytes = [&](int r) {
         return std::max<uint64_t>(o->recv_cap[r] * o->tuple_bytes, o->recv_cap_u[r] * 32);
@@ -478,6 +480,10 @@ mgj_status mgj_plan(const mgj_config *cfg, const mgj_peers *peers, mgj_handle *o
     // scatter tiles per relation: one per SM, or (streaming) STREAM_TPC per
     // S scatter CTA, in at most STREAM_RMAX rounds
     const int G = stream ? std::min(h->nsm * STREAM_TPC, STREAM_RMAX * h->scatter_sms) : h->nsm;
+    if (n.c.compress && G > COMP_MAX_TILES) {  // the receive capacity in units assumes at most this many
+        mgj_destroy(h);
+        return MGJ_EINVAL;
+    }
     // per-run zero block: rank_hist, ticket, meta, acc, err, cop_slots
     size_t zo = 0;
     const size_t z_hist = zo; zo += align_up(2ull * P * 4, 256);

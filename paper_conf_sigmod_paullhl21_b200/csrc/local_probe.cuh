@@ -368,7 +368,11 @@ __device__ __forceinline__ void local_body(const Ctx &c, const typename LocalDes
     for (int q = tid; q < 2 * QL; q += LOCAL_THREADS) bins2[q] = 0;
     __syncthreads();
     const uint64_t pol = policy_evict_first();
-    // thread 0: TMA chunk j (16-byte-aligned superset) into buffer j & 1
+    constexpr int LI = 32;  // the thread that issues the chunk loads (and the chunked pass's stores)
+    // LM_SECOND: warps issuing a chunk's run copies (measured at B1 = 7 / 8-byte keys at
+    // B1 = 6, local pass: 1 warp 6.28 / 6.79 ms, 2 6.20 / 6.32, 4 6.25 / 6.11, 8 6.27 / 6.15)
+    constexpr int GW = 4;
+    // thread LI: TMA chunk j (16-byte-aligned superset) into buffer j & 1
     auto issue = [&](uint32_t j, const Desc &d) {
         const uint32_t ci = cidx(j);
         const int rel = ci < nch_r ? 0 : 1;
@@ -377,11 +381,12 @@ __device__ __forceinline__ void local_body(const Ctx &c, const typename LocalDes
         uint64_t *b = &bar[j & 1];
         if constexpr (from_mid) {
             // the pieces of sub-partition d.v's runs, back to back: the issuing
-            // warp's lanes take 32 runs at a time (their offsets loaded in
-            // parallel, destinations by a warp scan), each lane its own copy
-            const int lane = tid & 31;
-            if (lane == 0) mbar_arrive_expect_tx(b, d.len * TB);
-            __syncwarp();
+            // warps' lanes take 32 runs at a time (their offsets loaded in
+            // parallel, destinations by a warp scan); piece i is copied by lane i
+            // of issuing warp i mod GW, so the copies issue from GW warps at once
+            const int lane = tid & 31, gw = (tid >> 5) - (LI >> 5);
+            if (tid == LI) mbar_arrive_expect_tx(b, d.len * TB);
+            named_bar_sync(2, 32 * GW);  // the expected bytes are set before any copy lands
             const int a = (int)(d.v & ((1u << BA) - 1));
             const uint16_t *E = c.eoffA[rel];
             const Tup *mid = static_cast<const Tup *>(c.mid[rel]);
@@ -406,7 +411,7 @@ __device__ __forceinline__ void local_body(const Ctx &c, const typename LocalDes
                     const uint32_t y = __shfl_up_sync(0xffffffffu, incl, o);
                     if (lane >= o) incl += y;
                 }
-                if (pc) tma_load_1d(buf(j & 1) + at + incl - pc, mid + src, pc * TB, b, pol);
+                if (pc && (lane % GW) == gw) tma_load_1d(buf(j & 1) + at + incl - pc, mid + src, pc * TB, b, pol);
                 at += __shfl_sync(0xffffffffu, incl, 31);
             }
             return;
@@ -428,9 +433,8 @@ __device__ __forceinline__ void local_body(const Ctx &c, const typename LocalDes
         }
     };
     Desc nxt{};
-    constexpr int LI = 32;  // the thread that issues the chunk loads (and the chunked pass's stores)
-    // (the second pass issues its run pieces with the whole of LI's warp)
-    auto issuer = [&]() { return from_mid ? (tid >> 5) == (LI >> 5) : tid == LI; };
+    // (the second pass issues its run pieces with GW whole warps from LI's on)
+    auto issuer = [&]() { return from_mid ? (unsigned)((tid >> 5) - (LI >> 5)) < (unsigned)GW : tid == LI; };
     if (issuer()) {
         if (mine > 0) issue(0, cdesc[cidx(0)]);
         if (mine > 1) nxt = cdesc[cidx(1)];
@@ -503,8 +507,7 @@ __device__ __forceinline__ void local_body(const Ctx &c, const typename LocalDes
         // chunk j+1 -> buffer X^1 once chunk j-1's stores have read it; the issuing
         // thread (warp 1, LI) also issues the chunk's bulk store, warp 0 scans meanwhile
         if (issuer() && j + 1 < mine) {
-            if (tid == LI) bulk_wait_read0();
-            if (from_mid) __syncwarp();
+            if (tid == LI) bulk_wait_read0();  // (issue's barrier orders the other issuers after it)
             issue(j + 1, nxt);
             if (j + 2 < mine) nxt = cdesc[cidx(j + 2)];
         }

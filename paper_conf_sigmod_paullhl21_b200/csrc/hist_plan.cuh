@@ -248,8 +248,8 @@ __global__ void k_tilescan(Ctx c) {
                     run += val(src[t * stride]);
                 }
             }
-            if (p < c.nrounds) {  // round p's non-empty tiles, and its counter opened for this run
-                const int r = p, u0 = r * c.sgrid, u1 = min(c.G, (r + 1) * c.sgrid);
+            for (int r = p; r < c.nrounds; r += c.P) {  // round r's non-empty tiles, its counter opened
+                const int u0 = r * c.sgrid, u1 = min(c.G, (r + 1) * c.sgrid);
                 uint32_t nt = (uint32_t)(u1 - u0);
                 if (c.n_in[1] < 8ull * (uint64_t)c.G) {  // small input: some tiles are empty
                     nt = 0;

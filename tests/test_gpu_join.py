@@ -1021,6 +1021,7 @@ def test_overlap_timeline(mgj):
                                        (8, "unique", {"materialize": True}), (3, "zipf", {"skew_bcast": 1}),
                                        (2, "m1", {"compress": True, "materialize": True}), (4, "m1", {"compress": True}),
                                        (2, "wide", {"materialize": True}), (1, "unique", {"radix_bits_global": 4}),
+                                       (1, "unique", {"radix_bits_global": 1}), (2, "unique", {"radix_bits_global": 2}),
                                        (2, "unique", {"local_split_bits": 2})])
 def test_stream_parity(mgj, N, kind, kw):
     """shuffle_overlap = 2: S's local pass

@@ -39,8 +39,9 @@ def keys(rng, n, kb, dom, zipf):
 def case(rng):
     kb = 8 if rng.random() < 0.25 else 4
     N = int(rng.choice([1, 1, 2, 3, 4, 8]))
-    nr = int(rng.integers(0, 1 << int(rng.integers(4, 18))))
-    ns = int(rng.integers(0, 1 << int(rng.integers(4, 19))))
+    big = rng.random() < 0.15  # sometimes several chunks and tiles per partition and rank
+    nr = int(rng.integers(0, 1 << int(rng.integers(4, 22 if big else 18))))
+    ns = int(rng.integers(0, 1 << int(rng.integers(4, 23 if big else 19))))
     dom = int(rng.choice([2, 37, 1000, 1 << 14, 1 << 20, (1 << 32) - 1 if kb == 4 else 1 << 40]))
     zipf = float(rng.choice([0, 0, 0.5, 1.0]))
     kw = dict(radix_bits_global=int(rng.choice([0, 1, 4, 7, 10, 12])),

@@ -50,11 +50,32 @@ def case(rng):
               local_split_bits=int(rng.choice([0, 0, 0, 2, 4])),
               shuffle_overlap=int(rng.choice([0, 1, 2, -1])) if N > 1 else int(rng.choice([0, 1, 2])),
               skew_bcast=int(rng.choice([0, 0, 1, -1])))
-    if kb == 4 and kw["radix_bits_global"] <= 10 and rng.random() < 0.25:
+    if rng.random() < 0.15:  # EXTERNAL: the caller's all-to-all (emulated with device copies)
+        kw["shuffle_mode"] = mgj.SHUFFLE_EXTERNAL
+        kw["shuffle_overlap"] = 0
+        kw["skew_bcast"] = 0
+    elif kb == 4 and kw["radix_bits_global"] <= 10 and rng.random() < 0.25:
         kw["compress"] = True
-    if N > 1 and rng.random() < 0.25:
+    if N > 1 and rng.random() < 0.25 and "shuffle_mode" not in kw:
         kw["assign"] = 1
     return dict(kb=kb, N=N, nr=nr, ns=ns, dom=dom, zipf=zipf, kw=kw)
+
+
+def exchange(joins, N):
+    """EXTERNAL mode: the all-to-all NCCL all_to_all_single would do, as device copies."""
+    lays = [j.exchange_layout() for j in joins]
+    tb = lays[0]["tuple_bytes"]
+    for rel in range(2):
+        for g in range(N):
+            so = 0
+            for d in range(N):
+                cnt = lays[g]["send_count"][rel][d]
+                ro = sum(lays[d]["recv_count"][rel][:g])
+                if cnt:
+                    mgj.device_bytes(lays[d]["recv"][rel] + ro * tb, cnt * tb).copy_(
+                        mgj.device_bytes(lays[g]["send"][rel] + so * tb, cnt * tb))
+                so += cnt
+    torch.cuda.synchronize()
 
 
 def dataset(c, rng, nr, ns):
@@ -112,6 +133,9 @@ def run(c, rng):
             joins[g].partition(*tens[g], stream=streams[g])
         for g in range(N):
             joins[g].shuffle(streams[g])
+        if kw.get("shuffle_mode") == mgj.SHUFFLE_EXTERNAL:
+            torch.cuda.synchronize()
+            exchange(joins, N)
         for g in range(N):
             joins[g].join(streams[g])
         res = [j.result() for j in joins]

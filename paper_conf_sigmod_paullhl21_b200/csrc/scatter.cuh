@@ -129,8 +129,10 @@ template <> struct Vec<32> { struct __align__(32) T { uint4 a, b; }; };
 template <int BYTES>
 __device__ __forceinline__ void st_group(void *dst, const typename Vec<BYTES>::T &v) {
     if constexpr (BYTES == 32) {
-        asm volatile("st.global.v8.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};" ::"l"(dst), "r"(v.a.x), "r"(v.a.y),
-                     "r"(v.a.z), "r"(v.a.w), "r"(v.b.x), "r"(v.b.y), "r"(v.b.z), "r"(v.b.w)
+        // L1::no_allocate: the scattered sectors are never read back here
+        // (measured at M2: scatter 3.85 -> 3.80 ms; .cs streaming stores: no change)
+        asm volatile("st.global.L1::no_allocate.v8.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};" ::"l"(dst), "r"(v.a.x),
+                     "r"(v.a.y), "r"(v.a.z), "r"(v.a.w), "r"(v.b.x), "r"(v.b.y), "r"(v.b.z), "r"(v.b.w)
                      : "memory");
     } else {
         *static_cast<typename Vec<BYTES>::T *>(dst) = v;
@@ -323,7 +325,7 @@ __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c, int rel0, int rel1) {
                     e[i] = i < (int)cc[0] ? unit_enc((uint32_t)carry[0][i < CW ? i : 0].x, (uint32_t)carry[0][i < CW ? i : 0].y, tb0) : 0ull;
                 unit_pack(e, cc[0] | (uint32_t)c.rank << 3 | (uint32_t)tile << 6, a);
                 char *d = c.arena[dstr[0]] + c.lay.recv[rel] + (size_t)bidx[0] * 32;
-                asm volatile("st.global.v4.u64 [%0], {%1,%2,%3,%4};" ::"l"(d), "l"(a[0]), "l"(a[1]), "l"(a[2]), "l"(a[3]) : "memory");
+                asm volatile("st.global.L1::no_allocate.v4.u64 [%0], {%1,%2,%3,%4};" ::"l"(d), "l"(a[0]), "l"(a[1]), "l"(a[2]), "l"(a[3]) : "memory");
             }
         } else {
 #pragma unroll
@@ -541,7 +543,7 @@ __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c, int rel0, int rel1) {
                     for (int x = 0; x < CU_N; ++x) e[x] = unit_enc((uint32_t)tt[x].x, (uint32_t)tt[x].y, tbase);
                     unit_pack(e, (uint32_t)CU_N | (uint32_t)c.rank << 3 | (uint32_t)u.tile << 6, a);
                     char *dst = reinterpret_cast<char *>(ob + (ull)(uint32_t)(pv.x + slot / SG) * 32);
-                    asm volatile("st.global.v4.u64 [%0], {%1,%2,%3,%4};" ::"l"(dst), "l"(a[0]), "l"(a[1]), "l"(a[2]),
+                    asm volatile("st.global.L1::no_allocate.v4.u64 [%0], {%1,%2,%3,%4};" ::"l"(dst), "l"(a[0]), "l"(a[1]), "l"(a[2]),
                                  "l"(a[3])
                                  : "memory");
                 }

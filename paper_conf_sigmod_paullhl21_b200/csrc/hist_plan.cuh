@@ -330,6 +330,7 @@ __host__ __device__ inline bool skip_of(uint64_t r, uint64_t s) { return (r == 0
 // order go to their preferred rank (the one holding most of their tuples)
 // unless its assigned weight would pass cap = 9/8 of the mean, then to the
 // least-loaded rank.  Shared by k_plan (thread 0) and mgj_plan_host.
+#pragma nv_exec_check_disable  // host lambdas from mgj_plan_host, device lambdas from k_plan
 template <typename WF, typename BF>
 __host__ __device__ inline void assign_greedy(int N, int P, WF weight, BF pref, int32_t *owner) {
     uint64_t load[MAX_RANKS] = {}, total = 0;

@@ -188,7 +188,6 @@ struct ChunkDescB {
 // owned partitions is kept in chunk_base1 for k_emit2.  One CTA.
 __global__ void __launch_bounds__(1024) k_planA(Ctx c) {
     extern __shared__ uint64_t sv[];  // [L+1] then u32 [L+1]
-    __shared__ uint64_t tmp[33];
     __shared__ uint32_t tmp32[33];
     if (!c.meta[MT_OK] || !c.meta[MT_BA]) return;
     const int BA = c.meta[MT_BA];
@@ -221,7 +220,6 @@ __global__ void __launch_bounds__(1024) k_planA(Ctx c) {
             c.meta[MT_OK] = 0;
         }
     }
-    (void)tmp;
 }
 
 // The second pass's chunk descriptors: one warp per (relation, sub-partition

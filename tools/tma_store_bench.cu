@@ -23,13 +23,39 @@ __global__ void __launch_bounds__(1024, 1) k_bulk(char *dst, size_t region, int 
         for (int r = 0; r < rounds; ++r) {
             for (int p = w * 32 + lane; p < P; p += 32 * nw) {
                 char *g = dst + ((size_t)blockIdx.x * P + p) * region + (size_t)r * B;
-                const char *s = sm + ((p * B) & (64 * 1024 - 1));
+                const char *s = sm + ((p * 64) & (32 * 1024 - 1));
                 asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(g), "r"(smem_u32(s)),
                              "r"(B)
                              : "memory");
             }
             asm volatile("cp.async.bulk.commit_group;" ::: "memory");
             // keep at most a few groups in flight per thread (the shared source is reused)
+            asm volatile("cp.async.bulk.wait_group.read 4;" ::: "memory");
+        }
+        asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+    }
+}
+
+// one lane per issuing warp issues copies back to back (operands of one thread:
+// no per-lane serialisation loop), unrolled by 4
+__global__ void __launch_bounds__(1024, 1) k_bulk1(char *dst, size_t region, int B, int rounds, int nw) {
+    extern __shared__ __align__(128) char sm[];
+    const int P = 1024;
+    for (int i = threadIdx.x; i < 64 * 1024 / 4; i += blockDim.x) reinterpret_cast<uint32_t *>(sm)[i] = i;
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    __syncthreads();
+    const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    if (w < nw && lane == 0) {
+        for (int r = 0; r < rounds; ++r) {
+#pragma unroll 4
+            for (int p = w; p < P; p += nw) {
+                char *g = dst + ((size_t)blockIdx.x * P + p) * region + (size_t)r * B;
+                const char *s = sm + ((p * 64) & (32 * 1024 - 1));
+                asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(g), "r"(smem_u32(s)),
+                             "r"(B)
+                             : "memory");
+            }
+            asm volatile("cp.async.bulk.commit_group;" ::: "memory");
             asm volatile("cp.async.bulk.wait_group.read 4;" ::: "memory");
         }
         asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
@@ -65,13 +91,14 @@ int main() {
     const size_t region = total / ((size_t)nsm * 1024) / 256 * 256;  // ~110 KB per partition
     cudaFuncSetAttribute(k_bulk, cudaFuncAttributeMaxDynamicSharedMemorySize, 64 * 1024);
     cudaFuncSetAttribute(k_stg, cudaFuncAttributeMaxDynamicSharedMemorySize, 64 * 1024);
+    cudaFuncSetAttribute(k_bulk1, cudaFuncAttributeMaxDynamicSharedMemorySize, 64 * 1024);
     cudaEvent_t a, b;
     cudaEventCreate(&a);
     cudaEventCreate(&b);
-    for (int B : {32, 64, 128, 256}) {
+    for (int B : {48, 64, 96, 128}) {
         const int rounds = (int)(region / B) < 512 ? (int)(region / B) : 512;
         const double bytes = (double)nsm * 1024 * B * rounds;
-        for (int nw : {1, 4, 8, 16, 32}) {
+        for (int nw : {1, 2, 4, 8, 32}) {
             k_bulk<<<nsm, 1024, 64 * 1024>>>(dst, region, B, rounds, nw);
             cudaEventRecord(a);
             k_bulk<<<nsm, 1024, 64 * 1024>>>(dst, region, B, rounds, nw);
@@ -82,6 +109,18 @@ int main() {
             printf("bulk  B=%4d nw=%2d: %8.1f GB/s  %6.2f cyc/copy/SM (at 1.965 GHz)  %s\n", B, nw, bytes / ms / 1e6,
                    ms * 1e-3 * 1.965e9 / (1024.0 * rounds), cudaGetErrorString(cudaGetLastError()));
         }
+        for (int nw : {1, 2, 4, 8, 16}) {
+            k_bulk1<<<nsm, 1024, 64 * 1024>>>(dst, region, B, rounds, nw);
+            cudaEventRecord(a);
+            k_bulk1<<<nsm, 1024, 64 * 1024>>>(dst, region, B, rounds, nw);
+            cudaEventRecord(b);
+            cudaEventSynchronize(b);
+            float ms;
+            cudaEventElapsedTime(&ms, a, b);
+            printf("bulk1 B=%4d nw=%2d: %8.1f GB/s  %6.2f cyc/copy/SM (one lane per warp)  %s\n", B, nw, bytes / ms / 1e6,
+                   ms * 1e-3 * 1.965e9 / (1024.0 * rounds), cudaGetErrorString(cudaGetLastError()));
+        }
+        if (B % 32) continue;
         k_stg<<<nsm, 1024, 64 * 1024>>>(dst, region, B, rounds);
         cudaEventRecord(a);
         k_stg<<<nsm, 1024, 64 * 1024>>>(dst, region, B, rounds);

@@ -8,9 +8,6 @@
 
 namespace mgj {
 
-#ifndef HIST_FOLD16
-#define HIST_FOLD16 1  // 4-byte keys: fold four bins per thread with 16-byte accesses (P >= 4)
-#endif
 constexpr int HIST_NB = 3;  // k_hist: TMA ring depth at most (sub-tiles in flight per CTA; 2 CTAs per SM)
 // ring depth for sub-tiles of T keys: about 96 KB in flight per CTA, 2..HIST_NB deep
 __host__ __device__ inline int hist_nb(int T, int key_bytes) {
@@ -146,9 +143,9 @@ __global__ void __launch_bounds__(HIST_THREADS, 2) k_hist(Ctx c) {
         if (tid == 0 && g + NB < ntot) issue(g + NB);
         // sub-tile histogram (u16 pairs) for the scatter's layout, then fold into acc
         uint32_t *o32 = reinterpret_cast<uint32_t *>(c.sub_hist + (((size_t)rel * c.G + tile) * c.sub_ns + j) * P);
-        if constexpr (sizeof(K) == 4) {  // 8-byte shared accesses, pairs of bins (measured: M2 0.83 -> 0.78 ms;
-                                         // slower for 8-byte keys, 0.71 -> 0.75, which keep the scalar fold)
-#if HIST_FOLD16
+        if constexpr (sizeof(K) == 4) {  // wide shared accesses, four bins per thread (measured at M2: pairs of
+                                         // bins 0.83 -> 0.78 ms, then four bins; slower for 8-byte keys,
+                                         // 0.71 -> 0.75, which keep the scalar fold)
             for (int q = tid; q < P / 4; q += blockDim.x) {  // 16-byte accesses, four bins (P >= 4 below)
                 const uint4 x = reinterpret_cast<const uint4 *>(sub)[q];
                 reinterpret_cast<uint2 *>(o32)[q] = make_uint2(x.x | x.y << 16, x.z | x.w << 16);
@@ -167,17 +164,6 @@ __global__ void __launch_bounds__(HIST_THREADS, 2) k_hist(Ctx c) {
                 acc[1] += x1;
                 sub[0] = sub[1] = 0;
             }
-#else
-            for (int q = tid; q < P / 2; q += blockDim.x) {
-                const uint2 x = reinterpret_cast<const uint2 *>(sub)[q];
-                o32[q] = x.x | x.y << 16;
-                uint2 a = reinterpret_cast<const uint2 *>(acc)[q];
-                a.x += x.x;
-                a.y += x.y;
-                reinterpret_cast<uint2 *>(acc)[q] = a;
-                reinterpret_cast<uint2 *>(sub)[q] = make_uint2(0u, 0u);
-            }
-#endif
         } else {
             for (int q = tid; q < P / 2; q += blockDim.x) {
                 const uint32_t x0 = sub[2 * q], x1 = sub[2 * q + 1];

@@ -202,12 +202,36 @@ __global__ void __launch_bounds__(HIST_THREADS, 2) k_hist(Ctx c) {
 // then publishes the histograms with the rank's unit totals (publish_hist).
 __global__ void k_tilescan(Ctx c) {
     const int idx = blockIdx.x * blockDim.x + threadIdx.x;
-    if (idx < 2 * c.P) {
+    auto val = [&](uint32_t v) { return c.comp ? (v + CU_N - 1) / CU_N : v; };
+    if (!c.stream) {
+        // one warp per (rel, p): the tiles' counts loaded 32 at a time and
+        // scanned across the lanes (measured at M2: 27 us with a thread per
+        // (rel, p) walking the tiles one after another, 8 us like this)
+        const int w = idx >> 5, lane = threadIdx.x & 31;
+        if (w < 2 * c.P) {
+            const int rel = w / c.P, p = w % c.P;
+            const uint32_t *src = c.tile_hist + (size_t)rel * c.G * c.P + p;
+            uint32_t *dst = c.tile_base + (size_t)rel * c.G * c.P + p;
+            uint32_t run = 0;
+            for (int t0 = 0; t0 < c.G; t0 += 32) {
+                const int t = t0 + lane;
+                const uint32_t v = t < c.G ? val(__ldcg(src + (size_t)t * c.P)) : 0u;
+                uint32_t incl = v;
+#pragma unroll
+                for (int o = 1; o < 32; o <<= 1) {
+                    const uint32_t y = __shfl_up_sync(0xffffffffu, incl, o);
+                    if (lane >= o) incl += y;
+                }
+                if (t < c.G) dst[(size_t)t * c.P] = run + incl - v;
+                run += __shfl_sync(0xffffffffu, incl, 31);
+            }
+            if (c.comp && lane == 0) c.rank_units[w] = run;
+        }
+    } else if (idx < 2 * c.P) {
         const int rel = idx / c.P, p = idx % c.P;
         const size_t stride = c.P;
         const uint32_t *src = c.tile_hist + (size_t)rel * c.G * c.P + p;
         uint32_t *dst = c.tile_base + (size_t)rel * c.G * c.P + p;
-        auto val = [&](uint32_t v) { return c.comp ? (v + CU_N - 1) / CU_N : v; };
         uint32_t run = 0;
         int t = 0;
         if (c.stream && rel == 1) {

@@ -305,7 +305,10 @@ void launch_partition(mgj_plan_s *h, cudaStream_t s) {
 template <typename K>
 void launch_shuffle(mgj_plan_s *h, cudaStream_t s) {
     const Norm &n = h->n;
-    k_tilescan<<<(2 * n.P + 127) / 128, 128, 0, s>>>(h->ctx);
+    if (h->ctx.stream)
+        k_tilescan<<<(2 * n.P + 127) / 128, 128, 0, s>>>(h->ctx);  // a thread per (rel, p): round boundaries
+    else
+        k_tilescan<<<(2 * n.P * 32 + 255) / 256, 256, 0, s>>>(h->ctx);  // a warp per (rel, p)
     k_plan<<<1, 1024, plan_smem(n), s>>>(h->ctx);
     k_chunkmap<<<h->nsm * 2, 256, 0, s>>>(h->ctx, h->cdesc);
     if (h->ctx.stream) k_chunkorder<<<h->nsm, 256, 0, s>>>(h->ctx);

@@ -664,11 +664,10 @@ __global__ void __launch_bounds__(1024) k_plan(Ctx c) {
             for (int i = tid; i < np; i += blockDim.x) {
                 const int p = own_p(i);
                 const uint64_t src = rel ? (uint64_t)c.rank : (uint64_t)own[p];
-                for (int g = 0; g < MAX_RANKS; ++g) {
-                    ps[(size_t)i * MAX_RANKS + g] = g == 0 ? (c.seg_start[rel * P + p] | src << PIECE_SRC_SHIFT) : 0;
-                    pl[(size_t)i * MAX_RANKS + g] =
-                        g == 0 ? (uint32_t)(rel ? (bcf[p] ? (uint64_t)HL(c.rank, 1, p) : LT(1, p)) : LT(0, p)) : 0;
-                }
+                // piece 0 only: with the P2P shuffle nothing reads pieces 1.. (chunk_table,
+                // k_chunkmap); storing them was most of this kernel's time (LSU-bound)
+                ps[(size_t)i * MAX_RANKS] = c.seg_start[rel * P + p] | src << PIECE_SRC_SHIFT;
+                pl[(size_t)i * MAX_RANKS] = (uint32_t)(rel ? (bcf[p] ? (uint64_t)HL(c.rank, 1, p) : LT(1, p)) : LT(0, p));
             }
             continue;
         }
@@ -712,12 +711,16 @@ __global__ void __launch_bounds__(1024) k_plan(Ctx c) {
             uint32_t *pc = c.piece_chunk + (size_t)rel * P * (MAX_RANKS + 1);
             for (int i = tid; i <= np; i += blockDim.x) {
                 uint32_t t = 0;
-                if (i < np)
+                if (i < np && !c.ext) {  // one piece (P2P)
+                    pc[(size_t)i * (MAX_RANKS + 1)] = 0;
+                    t = (uint32_t)((pl[(size_t)i * MAX_RANKS] + C - 1) / C);
+                } else if (i < np) {
                     for (int g = 0; g < MAX_RANKS; ++g) {
                         pc[(size_t)i * (MAX_RANKS + 1) + g] = t;
                         t += (uint32_t)((pl[(size_t)i * MAX_RANKS + g] + C - 1) / C);
                     }
-                if (i < np) pc[(size_t)i * (MAX_RANKS + 1) + MAX_RANKS] = t;
+                    pc[(size_t)i * (MAX_RANKS + 1) + MAX_RANKS] = t;
+                }
                 chn[i] = t;
             }
             __syncthreads();

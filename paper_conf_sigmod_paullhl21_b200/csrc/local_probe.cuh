@@ -74,7 +74,7 @@ __global__ void k_chunkmap(Ctx c, ChunkDesc *desc) {
         const uint32_t j = li - cb[lo];
         const uint32_t *pc = c.piece_chunk + ((size_t)rel * P + lo) * (MAX_RANKS + 1);
         int g = 0;
-        while (g + 1 < MAX_RANKS && pc[g + 1] <= j) ++g;  // piece holding chunk j of partition lo
+        while (c.ext && g + 1 < MAX_RANKS && pc[g + 1] <= j) ++g;  // piece holding chunk j of partition lo (P2P: one)
         const uint64_t k = j - pc[g];
         const size_t pidx = ((size_t)rel * P + lo) * MAX_RANKS + g;
         ChunkDesc d;

@@ -359,9 +359,9 @@ void launch_join(mgj_plan_s *h, cudaStream_t s) {
         cudaStreamWaitEvent(s, h->ev_join, 0);  // R's local pass (second stream) is done
         k_wait<<<1, 32, 0, s>>>(h->ctx, SIG_DATA_S, -1);
         h->launches += 1;
-    } else if (!h->ctx.ext) {  // EXTERNAL: the caller's exchange is stream-ordered
-        k_wait<<<1, 32, 0, s>>>(h->ctx, SIG_DATA_R, SIG_DATA_S);
-        h->launches += 1;
+    } else if (!h->ctx.ext && h->ctx.world > 1) {  // EXTERNAL: the caller's exchange is stream-ordered;
+        k_wait<<<1, 32, 0, s>>>(h->ctx, SIG_DATA_R, SIG_DATA_S);  // one rank: its own scatter precedes
+        h->launches += 1;                                           // in stream order
     }
     // two-level local partitioning: k_plan decides on the device (MT_BA); when
     // it chooses one pass these four kernels return at once.  (Measured, not

@@ -552,6 +552,29 @@ def test_virtual_ranks_wide(mgj):
 
 
 # ------------------------------------------------------------ error paths
+@pytest.mark.parametrize("sms,kind,mat", [(1, "unique", True), (7, "wide", False), (31, "zipf", False),
+                                           (33, "unique", True), (100, "wide", True)])
+def test_grid_sizes(mgj, sms, kind, mat):
+    """num_sms bounds every persistent grid and the tile count G (= SMs): one CTA,
+    fewer tiles than a warp (the tile scan's partial warp), just over a warp, and
+    an uneven grid all join bit-exact with the oracle."""
+    w = {"unique": datagen.Workload("unique", 200003, 300007), "wide": datagen.Workload("wide", 200003, 300007),
+         "zipf": datagen.Workload("zipf", 1 << 16, 1 << 18, 1.0)}[kind]
+    d = w.rank_inputs()
+    cfg = mgj.make_config(r_capacity=w.n_r, s_capacity=w.n_s, num_sms=sms, materialize=mat,
+                          key_bytes=w.key_bytes)
+    j = mgj.Join(cfg)
+    res = j.run(*[dev(d[x]) for x in ("r_keys", "r_pays", "s_keys", "s_pays")])
+    ref = oracle.join(d["r_keys"], d["r_pays"], d["s_keys"], d["s_pays"], materialize=mat)
+    assert (res["match_count"], res["checksum"], res["pair_digest"]) == (ref["count"], ref["checksum"], ref["pair_digest"])
+    if mat:
+        k, a, b = sort_trip(*j.materialized(res))
+        np.testing.assert_array_equal(k, ref["key"])
+        np.testing.assert_array_equal(a, ref["pay_r"])
+        np.testing.assert_array_equal(b, ref["pay_s"])
+    j.close()
+
+
 def test_error_paths(mgj):
     n = 4096
     cfg = mgj.make_config(r_capacity=n, s_capacity=n)

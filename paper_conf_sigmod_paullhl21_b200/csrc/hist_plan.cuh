@@ -10,6 +10,9 @@ namespace mgj {
 
 constexpr int HIST_NB = 3;  // k_hist: TMA ring depth at most (sub-tiles in flight per CTA; 2 CTAs per SM)
 // ring depth for sub-tiles of T keys: about 96 KB in flight per CTA, 2..HIST_NB deep
+// k_hist reads a scatter sub-tile of T keys in HN blocks of T / HN keys (two for
+// 16384 4-byte keys: a 64 KB ring entry would leave room for one CTA per SM)
+__host__ __device__ inline int hist_halves(int T, int key_bytes) { return T * key_bytes > 49152 ? 2 : 1; }
 __host__ __device__ inline int hist_nb(int T, int key_bytes) {
     const int nb = 98304 / (T * key_bytes);
     return nb < 2 ? 2 : (nb > HIST_NB ? HIST_NB : nb);
@@ -62,11 +65,11 @@ __device__ inline void publish_hist(const Ctx &c) {
 
 template <typename K>
 __global__ void __launch_bounds__(HIST_THREADS, 2) k_hist(Ctx c) {
-    extern __shared__ __align__(128) unsigned char hsm[];  // ring[HIST_NB][T] keys | sub[P] | acc[P]
+    extern __shared__ __align__(128) unsigned char hsm[];  // ring[NB][TB] keys | sub[P] | acc[P]
     __shared__ __align__(8) uint64_t bar[HIST_NB];
-    const int P = c.P, T = c.scat_T, NB = hist_nb(T, sizeof(K));
-    K *const ring = reinterpret_cast<K *>(hsm);
-    uint32_t *const sub = reinterpret_cast<uint32_t *>(ring + (size_t)NB * T);
+    const int P = c.P, T = c.scat_T, HN = hist_halves(T, sizeof(K)), TB = T / HN, NB = hist_nb(TB, sizeof(K));
+    K *const ring = reinterpret_cast<K *>(hsm);  // NB entries of TB keys (block b: half b % HN of sub-tile b / HN)
+    uint32_t *const sub = reinterpret_cast<uint32_t *>(ring + (size_t)NB * TB);
     uint32_t *const acc = sub + P;
     const int tid = threadIdx.x, HS = c.hist_split, tile = blockIdx.x / HS, part = blockIdx.x % HS;
     constexpr int LU = 16 / (int)sizeof(K);
@@ -86,23 +89,31 @@ __global__ void __launch_bounds__(HIST_THREADS, 2) k_hist(Ctx c) {
         len = (uint32_t)min((uint64_t)T, (rel ? hi1 : hi0) - first);
     };
     const uint64_t pol = policy_evict_first();
-    auto issue = [&](uint32_t g) {  // thread 0: TMA the 16-byte-aligned body of sub-tile g's keys
+    auto block = [&](uint32_t b, int &rel, uint32_t &j, uint64_t &first, uint32_t &len) {  // keys of block b
+        uint32_t slen;
+        subtile(b / HN, rel, j, first, slen);
+        const uint32_t o = (b % HN) * (uint32_t)TB;
+        first += o;
+        len = slen > o ? min(slen - o, (uint32_t)TB) : 0u;
+    };
+    auto issue = [&](uint32_t b) {  // thread 0: TMA the 16-byte-aligned body of block b's keys
         int rel;
         uint32_t j, len;
         uint64_t first;
-        subtile(g, rel, j, first, len);
-        uint64_t *b = &bar[g % NB];
+        block(b, rel, j, first, len);
+        uint64_t *br = &bar[b % NB];
         const uint32_t bytes = (len & ~(uint32_t)(LU - 1)) * (uint32_t)sizeof(K);
-        mbar_arrive_expect_tx(b, bytes);
+        mbar_arrive_expect_tx(br, bytes);
         if (bytes)
-            tma_load_1d(ring + (size_t)(g % NB) * T, static_cast<const K *>(c.in_key[rel]) + first, bytes, b, pol);
+            tma_load_1d(ring + (size_t)(b % NB) * TB, static_cast<const K *>(c.in_key[rel]) + first, bytes, br, pol);
     };
+    const uint32_t nblk = ntot * (uint32_t)HN;
     trace_begin(c, MGJ_TR_HIST);
     for (int i = tid; i < 2 * P; i += blockDim.x) sub[i] = 0;
     if (tid == 0) {
         for (int i = 0; i < NB; ++i) mbar_init(&bar[i], 1);
         fence_mbar_init();
-        for (uint32_t g = 0; g < ntot && g < (uint32_t)NB; ++g) issue(g);
+        for (uint32_t b = 0; b < nblk && b < (uint32_t)NB; ++b) issue(b);
     }
     __syncthreads();
     const uint32_t m = (uint32_t)(P - 1);
@@ -117,13 +128,14 @@ __global__ void __launch_bounds__(HIST_THREADS, 2) k_hist(Ctx c) {
             acc[p] = 0;
         }
     };
-    for (uint32_t g = 0; g < ntot; ++g) {
+    for (uint32_t b = 0; b < nblk; ++b) {
         int rel;
         uint32_t j, len;
         uint64_t first;
-        subtile(g, rel, j, first, len);
-        const K *buf = ring + (size_t)(g % NB) * T;
-        mbar_wait(&bar[g % NB], (g / NB) & 1);
+        block(b, rel, j, first, len);
+        const uint32_t g = b / HN;  // the sub-tile
+        const K *buf = ring + (size_t)(b % NB) * TB;
+        mbar_wait(&bar[b % NB], (b / NB) & 1);
         const uint32_t body = len & ~(uint32_t)(LU - 1);
         for (uint32_t i0 = (uint32_t)tid * LU; i0 < body; i0 += (uint32_t)blockDim.x * LU) {
             const uint4 v = *reinterpret_cast<const uint4 *>(buf + i0);
@@ -139,8 +151,11 @@ __global__ void __launch_bounds__(HIST_THREADS, 2) k_hist(Ctx c) {
         }
         if (tid < (int)(len - body))  // < LU trailing tuples of the relation: from global
             atomicAdd(&sub[digit1(static_cast<const K *>(c.in_key[rel])[first + body + tid], P)], 1u);
-        __syncthreads();  // counts final; ring slot g % NB free
-        if (tid == 0 && g + NB < ntot) issue(g + NB);
+        // (measured, not kept: the last warp done reading a slot refilling it instead of
+        // this barrier, M2 727 -> 755 us with 12288-key sub-tiles)
+        __syncthreads();  // counts final; ring slot b % NB free
+        if (tid == 0 && b + NB < nblk) issue(b + NB);
+        if (b % HN != (uint32_t)(HN - 1)) continue;  // the sub-tile's other block comes next
         // sub-tile histogram (u16 pairs) for the scatter's layout, then fold into acc
         uint32_t *o32 = reinterpret_cast<uint32_t *>(c.sub_hist + (((size_t)rel * c.G + tile) * c.sub_ns + j) * P);
         if constexpr (sizeof(K) == 4) {  // wide shared accesses, four bins per thread (measured at M2: pairs of

@@ -219,7 +219,8 @@ int scat_T_of(const Norm &n) { return n.c.compress ? scat_geom_comp().T : scat_g
 
 size_t hist_smem(const Norm &n) {
     const int T = scat_T_of(n);
-    return (size_t)hist_nb(T, n.c.key_bytes) * T * n.c.key_bytes + (size_t)n.P * 8;
+    const int TB = T / hist_halves(T, n.c.key_bytes);  // k_hist's ring blocks
+    return (size_t)hist_nb(TB, n.c.key_bytes) * TB * n.c.key_bytes + (size_t)n.P * 8;
 }
 size_t plan_smem(const Norm &n) {
     // totals, prefixes, owners, scan scratch, broadcast flags, then the unit

@@ -23,13 +23,17 @@ namespace mgj {
 // 4.16 ms for this design at M2.)
 struct ScatGeom {
     int T, SG, PPT, NT;
+    int NH;  // key-stage pieces: the sub-tile's keys arrive in NH pieces through one stage of T / NH keys
+             // (P <= 1024, 4-byte keys: 16384-tuple sub-tiles whose keys come in two halves; measured at
+             // M2 against 12288 tuples with one key stage: scatter 3.79 -> 3.73 ms, k_hist, which counts
+             // them in two 8192-key blocks, 0.727 -> 0.774 ms, step 9.34 -> 9.32 ms)
 };
 __host__ __device__ constexpr ScatGeom scat_geom(int P, int key_bytes) {
     return key_bytes == 4
-               ? (P <= 1024 ? ScatGeom{12288, 4, 1, 1024}
-                  : P == 2048 ? ScatGeom{4096, 4, 2, 1024} : ScatGeom{8192, 1, 4, 1024})
-               : (P <= 1024 ? ScatGeom{6144, 2, 1, 1024} : P == 2048 ? ScatGeom{2048, 2, 2, 1024}
-                                                                      : ScatGeom{4096, 1, 4, 1024});
+               ? (P <= 1024 ? ScatGeom{16384, 4, 1, 1024, 2}
+                  : P == 2048 ? ScatGeom{4096, 4, 2, 1024, 1} : ScatGeom{8192, 1, 4, 1024, 1})
+               : (P <= 1024 ? ScatGeom{6144, 2, 1, 1024, 1} : P == 2048 ? ScatGeom{2048, 2, 2, 1024, 1}
+                                                                         : ScatGeom{4096, 1, 4, 1024, 1});
 }
 
 // Per-partition write-out descriptor of the current sub-tile (8 bytes, one
@@ -49,7 +53,7 @@ constexpr uint16_t PI_NONE = 0xffff;
 __host__ __device__ inline size_t scat_smem_bytes(int P, int key_bytes) {
     const ScatGeom g = scat_geom(P, key_bytes);
     const size_t TB = 2 * (size_t)key_bytes;
-    return (size_t)g.T * key_bytes                             // input stage: keys (payloads: L2 prefetch + loads)
+    return (size_t)g.T / g.NH * key_bytes                      // input stage: keys (payloads: L2 prefetch + loads)
            + ((size_t)g.T + 2 * (size_t)(g.SG - 1) * P) * TB  // partition-sorted sub-tile (+ carries, group padding)
            + (size_t)P * sizeof(PInfo)                         // write-out descriptors
            + (size_t)P * 4                                     // next free slot per partition
@@ -158,8 +162,9 @@ __device__ __forceinline__ void st_group(void *dst, const typename Vec<BYTES>::T
 // (one tile per CTA at full grid; fewer CTAs when the launch shares the GPU
 // with the local pass of the other relation, §8(e) overlap) and stream each
 // tile in sub-tiles of T tuples whose keys a TMA bulk copy brings into shared
-// memory one sub-tile ahead (payloads: L2 prefetch, then registers).  Per
-// sub-tile:
+// memory ahead of their use (NH = 2: in two halves through one stage, half 1
+// arriving while half 0 is ranked; payloads: L2 prefetch, then registers).
+// Per sub-tile:
 //  1. thread t owns partitions t*PPT.. (PPT per thread) and keeps, in
 //     registers, each one's destination cursor and its < 32-byte tail
 //     (carry) from the previous sub-tile; a block scan of the per-partition
@@ -184,7 +189,7 @@ __device__ __forceinline__ void st_group(void *dst, const typename Vec<BYTES>::T
 // spread over all peers' links instead of visiting the ranks in step.  The
 // last CTA raises SIG_DATA_R / SIG_DATA_S at every peer after a system fence.
 // ---------------------------------------------------------------------------
-template <typename K, int T, int SG, int PPT, int NT, bool COMP = false>
+template <typename K, int T, int SG, int PPT, int NT, bool COMP = false, int NH = 1>
 __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c, int rel0, int rel1) {
     using Tup = typename TupT<K>::T;
     constexpr int TB = (int)sizeof(Tup);
@@ -192,6 +197,11 @@ __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c, int rel0, int rel1) {
     constexpr int LU = 16 / (int)sizeof(K);    // tuples per 16-byte stage vector
     constexpr int NU = V / LU;                 // vectors per thread
     static_assert(NU * LU == V && NU >= 1, "sub-tile");
+    // NH = 2: the keys arrive in two halves of TH through a stage of TH keys (the
+    // shared memory of a full key stage goes to the larger sorted sub-tile);
+    // half h of the sub-tile is ranked while half h + 1 is loaded
+    constexpr int TH = T / NH, VH = V / NH, NUH = NU / NH;
+    static_assert(NH == 1 || (NH == 2 && !COMP && NUH * NH == NU && NUH >= 1), "key-stage halves");
     // COMP (NEXT-1): a group is one 32-byte unit of SG = CU_N encoded tuples
     static_assert(!COMP || (SG == CU_N && sizeof(K) == 4 && PPT == 1), "compressed scatter");
     constexpr int GB = COMP ? 32 : SG * TB;    // group bytes at the destination
@@ -208,7 +218,7 @@ __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c, int rel0, int rel1) {
     extern __shared__ __align__(128) unsigned char smem[];
     const int P = c.P;
     K *const skey = reinterpret_cast<K *>(smem);  // stage: the sub-tile's keys
-    Tup *const sorted = reinterpret_cast<Tup *>(smem + T * sizeof(K));
+    Tup *const sorted = reinterpret_cast<Tup *>(smem + TH * sizeof(K));
     PInfo *const pinfo = reinterpret_cast<PInfo *>(sorted + T + 2 * (SG - 1) * P);  // 8-byte aligned
     uint32_t *const off = reinterpret_cast<uint32_t *>(pinfo + P);  // next free slot per partition
     unsigned long long *const obase = reinterpret_cast<unsigned long long *>(off + P);  // [2][MAX_RANKS]
@@ -298,16 +308,21 @@ __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c, int rel0, int rel1) {
         own8[P + p] = (uint8_t)(c.bcast[p] ? c.rank : c.owner[p]);  // S of a broadcast partition stays here
     }
 
-    auto issue = [&](const Cur &u) {  // thread 0: TMA the 16-byte-aligned body of sub-tile u's keys
+    // keys of half h of sub-tile u: [h * TH, h * TH + hlen)
+    auto half_len = [&](uint32_t len, int h) -> uint32_t {
+        return len > (uint32_t)(h * TH) ? min(len - (uint32_t)(h * TH), (uint32_t)TH) : 0u;
+    };
+    auto issue = [&](const Cur &u, int h) {  // thread 0: TMA the 16-byte-aligned body of half h of sub-tile u's keys
         uint64_t first;
         uint32_t len;
         span(u, first, len);
         const K *in_key = static_cast<const K *>(c.in_key[u.rel]);
         const K *in_pay = static_cast<const K *>(c.in_pay[u.rel]);
+        const uint32_t kbytes = (half_len(len, h) & ~(uint32_t)(LU - 1)) * (uint32_t)sizeof(K);
         const uint32_t bytes = (len & ~(uint32_t)(LU - 1)) * (uint32_t)sizeof(K);
-        mbar_arrive_expect_tx(&bar, bytes);
-        if (bytes) {
-            tma_load_1d(skey, in_key + first, bytes, &bar, pol);
+        mbar_arrive_expect_tx(&bar, kbytes);
+        if (kbytes) tma_load_1d(skey, in_key + first + h * TH, kbytes, &bar, pol);
+        if (h == 0 && bytes) {
             // payloads: brought into L2 now and loaded into registers while the
             // previous sub-tile is written out (the shared memory of a payload
             // stage goes to a 1.5x larger sub-tile instead; measured at M2:
@@ -406,8 +421,9 @@ __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c, int rel0, int rel1) {
     };
     // payloads of sub-tile u (L2-resident since issue(u)), loaded into
     // registers while the previous sub-tile is written out
+    // (half h = the vectors [h * NUH, (h + 1) * NUH) of every thread)
     K pp[V];
-    auto load_pay = [&](const Cur &u) {
+    auto load_pay = [&](const Cur &u, int h) {
         uint64_t first;
         uint32_t len;
         span(u, first, len);
@@ -415,17 +431,20 @@ __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c, int rel0, int rel1) {
         if (len == T) {
 #pragma unroll
             for (int x = 0; x < NU; ++x) {
+                if (x / NUH != h) continue;
                 const uint4 b = __ldcs(reinterpret_cast<const uint4 *>(gp + (uint32_t)(x * NT + tid) * LU));
                 memcpy(&pp[x * LU], &b, 16);
             }
         } else {
 #pragma unroll
-            for (int x = 0; x < NU; ++x)
+            for (int x = 0; x < NU; ++x) {
+                if (x / NUH != h) continue;
 #pragma unroll
                 for (int e = 0; e < LU; ++e) {
                     const uint32_t i = (uint32_t)(x * NT + tid) * LU + e;
                     pp[x * LU + e] = i < len ? __ldcs(gp + i) : (K)0;
                 }
+            }
         }
     };
     // write-out rotation (N > 1): CTA b starts its sweep of the groups at rank
@@ -449,8 +468,8 @@ __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c, int rel0, int rel1) {
     uint32_t ncnt[PPT];
     load_counts(u, ncnt);
     if (u.rel <= rel1) {
-        if (tid == 0) issue(u);
-        load_pay(u);
+        if (tid == 0) issue(u, 0);
+        load_pay(u, 0);
     }
     int cur_tile = -1;       // (relation, tile) the partition state belongs to: rel * G + tile
     uint32_t nsub_done = 0;  // sub-tiles processed (the stage barrier's phase parity)
@@ -511,40 +530,50 @@ __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c, int rel0, int rel1) {
         }
         pending = SG > 1;
         K kk[V];
-        mbar_wait(&bar, nsub_done & 1);
-        const uint32_t body = len & ~(uint32_t)(LU - 1);
         const K *gk = static_cast<const K *>(c.in_key[u.rel]) + first;
-        if (len == T) {  // full sub-tile: branch-free vector loads
 #pragma unroll
-            for (int x = 0; x < NU; ++x) {
-                const uint4 a = *reinterpret_cast<const uint4 *>(skey + (uint32_t)(x * NT + tid) * LU);
-                memcpy(&kk[x * LU], &a, 16);
+        for (int h = 0; h < NH; ++h) {  // (NH = 2: half 0 ranked while half 1 arrives)
+            mbar_wait(&bar, NH == 1 ? (nsub_done & 1) : (uint32_t)h);
+            const uint32_t hl = half_len(len, h), body = hl & ~(uint32_t)(LU - 1);
+            if (hl == (uint32_t)TH) {  // full half: branch-free vector loads
+#pragma unroll
+                for (int x = 0; x < NU; ++x) {
+                    if (x / NUH != h) continue;
+                    const uint4 a = *reinterpret_cast<const uint4 *>(skey + (uint32_t)((x - h * NUH) * NT + tid) * LU);
+                    memcpy(&kk[x * LU], &a, 16);
+                }
+            } else {
+#pragma unroll
+                for (int x = 0; x < NU; ++x) {
+                    if (x / NUH != h) continue;
+#pragma unroll
+                    for (int e = 0; e < LU; ++e) {  // < LU trailing tuples of the relation come from global
+                        const uint32_t i = (uint32_t)((x - h * NUH) * NT + tid) * LU + e;  // index in the half
+                        kk[x * LU + e] = i < body ? skey[i] : (i < hl ? gk[h * TH + i] : (K)0);
+                    }
+                }
             }
-        } else {
+            __syncthreads();  // S1 (half 0: offsets and carries in place too): stage consumed
+            if (tid == 0) {
+                if (h + 1 < NH) issue(u, h + 1);
+                else if (nx.rel <= rel1) issue(nx, 0);
+            }
+            if (h + 1 < NH) load_pay(u, h + 1);  // (in L2 since the sub-tile's first issue)
 #pragma unroll
-            for (int x = 0; x < NU; ++x) {
-#pragma unroll
-                for (int e = 0; e < LU; ++e) {  // < LU trailing tuples of the relation come from global
-                    const uint32_t i = (uint32_t)(x * NT + tid) * LU + e;
-                    kk[x * LU + e] = i < body ? skey[i] : (i < len ? gk[i] : (K)0);
+            for (int v = 0; v < V; ++v) {
+                if (v / VH != h) continue;
+                const uint32_t i = (uint32_t)((v / LU) * NT + tid) * LU + (v % LU);
+                if (i < len) {
+                    Tup t;
+                    t.x = kk[v];
+                    t.y = pp[v];
+                    if constexpr (COMP) bad_pay |= (uint32_t)pp[v] != row0 + (uint32_t)(first + i);
+                    sput(atomicAdd(&off[digit1(kk[v], P)], 1u), t);
                 }
             }
         }
-        __syncthreads();  // S1: offsets and carries in place, stage consumed
-        if (tid == 0 && nx.rel <= rel1) issue(nx);
-#pragma unroll
-        for (int v = 0; v < V; ++v) {
-            const uint32_t i = (uint32_t)((v / LU) * NT + tid) * LU + (v % LU);
-            if (i < len) {
-                Tup t;
-                t.x = kk[v];
-                t.y = pp[v];
-                if constexpr (COMP) bad_pay |= (uint32_t)pp[v] != row0 + (uint32_t)(first + i);
-                sput(atomicAdd(&off[digit1(kk[v], P)], 1u), t);
-            }
-        }
         __syncthreads();  // S2
-        if (nx.rel <= rel1) load_pay(nx);  // the ranking of this sub-tile has consumed pp
+        if (nx.rel <= rel1) load_pay(nx, 0);  // the ranking of this sub-tile has consumed pp
         // write-out: one group per thread per step, rotated by rank share for N > 1
         const uint32_t ngroups = total / SG;
         const ull ob_rel = (ull)(c.arena[0] + c.lay.recv[u.rel]);  // N = 1: the one receive buffer
@@ -617,7 +646,7 @@ __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c, int rel0, int rel1) {
 // The compressed-shuffle instance (NEXT-1): 4-byte keys, P <= 1024.
 // (12288-tuple sub-tiles like the uncompressed instance, measured at M2:
 // scatter 4.94 vs 5.36 ms with 8192, in spite of a 92-byte spill)
-constexpr ScatGeom scat_geom_comp() { return ScatGeom{12288, CU_N, 1, 1024}; }
+constexpr ScatGeom scat_geom_comp() { return ScatGeom{12288, CU_N, 1, 1024, 1}; }
 inline size_t scat_smem_bytes_comp(int P) {
     const ScatGeom g = scat_geom_comp();
     return (size_t)g.T * 4 + ((size_t)g.T + 2 * (size_t)(g.SG - 1) * P) * 8 + (size_t)P * sizeof(PInfo) +
@@ -631,7 +660,7 @@ inline void (*scatter_kernel_comp())(Ctx, int, int) {
 template <typename K>
 inline void (*scatter_kernel(int P))(Ctx, int, int) {
     constexpr ScatGeom g1 = scat_geom(1024, sizeof(K)), g2 = scat_geom(2048, sizeof(K)), g4 = scat_geom(4096, sizeof(K));
-    if (P <= 1024) return k_scatter<K, g1.T, g1.SG, g1.PPT, g1.NT>;
+    if (P <= 1024) return k_scatter<K, g1.T, g1.SG, g1.PPT, g1.NT, false, g1.NH>;
     if (P == 2048) return k_scatter<K, g2.T, g2.SG, g2.PPT, g2.NT>;
     return k_scatter<K, g4.T, g4.SG, g4.PPT, g4.NT>;
 }

@@ -578,7 +578,7 @@ __global__ void __launch_bounds__(NT, 1) k_scatter(Ctx c, int rel0, int rel1) {
         const uint32_t ngroups = total / SG;
         const ull ob_rel = (ull)(c.arena[0] + c.lay.recv[u.rel]);  // N = 1: the one receive buffer
         const uint32_t tbase = row0 + (uint32_t)u.lo;  // COMP: global row id of this tile's first row
-        const uint32_t rot = (uint32_t)(((uint64_t)ngroups * rot_num) / (uint32_t)c.world);
+        const uint32_t rot = c.world > 1 ? (uint32_t)(((uint64_t)ngroups * rot_num) / (uint32_t)c.world) : 0u;
         for (uint32_t w = tid; w < ngroups; w += NT) {
             const uint32_t gi = w + rot < ngroups ? w + rot : w + rot - ngroups;
             const uint32_t slot = gi * SG;

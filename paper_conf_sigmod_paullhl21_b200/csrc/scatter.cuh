@@ -26,7 +26,7 @@ struct ScatGeom {
     int NH;  // key-stage pieces: the sub-tile's keys arrive in NH pieces through one stage of T / NH keys
              // (P <= 1024, 4-byte keys: 16384-tuple sub-tiles whose keys come in two halves; measured at
              // M2 against 12288 tuples with one key stage: scatter 3.79 -> 3.73 ms, k_hist, which counts
-             // them in two 8192-key blocks, 0.727 -> 0.774 ms, step 9.34 -> 9.32 ms)
+             // them in two 8192-key blocks, 0.73 -> 0.74 ms, step 9.34 -> 9.29 ms)
 };
 __host__ __device__ constexpr ScatGeom scat_geom(int P, int key_bytes) {
     return key_bytes == 4

@@ -116,14 +116,6 @@ __device__ __forceinline__ void sts_at(uint32_t a, const uint2 &v) {
 __device__ __forceinline__ void sts_at(uint32_t a, const ulonglong2 &v) {
     asm volatile("st.shared.v2.u64 [%0], {%1,%2};" ::"r"(a), "l"(v.x), "l"(v.y) : "memory");
 }
-// A shared-window address the compiler cannot rematerialise (an asm volatile
-// result): without it ptxas re-derived the window base (S2R SR_CgaCtaId) in
-// every write-out iteration to save a register.
-__device__ __forceinline__ uint32_t smem_pin(const void *p) {
-    uint32_t r;
-    asm volatile("{\n\t.reg .u64 t;\n\tcvta.to.shared.u64 t, %1;\n\tcvt.u32.u64 %0, t;\n\t}" : "=r"(r) : "l"(p));
-    return r;
-}
 template <typename Tup> __device__ __forceinline__ Tup lds_tup(uint32_t a);
 template <> __device__ __forceinline__ uint2 lds_tup<uint2>(uint32_t a) { return lds64_at(a); }
 template <> __device__ __forceinline__ ulonglong2 lds_tup<ulonglong2>(uint32_t a) {

@@ -10,6 +10,20 @@ __device__ __forceinline__ uint32_t smem_u32(const void *p) {
     return static_cast<uint32_t>(__cvta_generic_to_shared(p));
 }
 
+// A shared-window address the compiler cannot rematerialise (an asm volatile
+// result): without it ptxas re-derives the window base (S2R SR_CgaCtaId) in
+// loops to save a register (the scatter's write-out, the probe's item loop).
+__device__ __forceinline__ uint32_t smem_pin(const void *p) {
+    uint32_t r;
+    asm volatile("{\n\t.reg .u64 t;\n\tcvta.to.shared.u64 t, %1;\n\tcvt.u32.u64 %0, t;\n\t}" : "=r"(r) : "l"(p));
+    return r;
+}
+__device__ __forceinline__ uint32_t lds_u32_at(uint32_t a) {
+    uint32_t v;
+    asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(a));
+    return v;
+}
+
 __device__ __forceinline__ void mbar_init(uint64_t *bar, uint32_t count) {
     asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
 }
